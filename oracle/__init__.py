@@ -1,0 +1,116 @@
+"""THE ORACLE -- test infrastructure only.
+
+Only tests/, __graft_entry__.smoke() and bench.py's cpu_baseline / `--impl
+reference` legs may import this package.  The product path
+(paper_conf_ipps_dellinggnw11_b200/) never imports it, and the two share no code.
+
+Plain binary-heap Dijkstra on the ORIGINAL graph (§II-A), exact by
+Theorem 3.1 (§III) for what PHAST computes; diameter (PAPER.md:20
+§VII-B); O(n+m) optimality certificate.  See oracle.c for the
+passage each function follows.  Pins: tests/test_oracle.py.  Parity status of
+every function: pinned.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+import numpy as np
+
+INF = 0xFFFFFFFF
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_LIB_PATH = os.path.join(_HERE, "liboracle.so")
+_lib = None
+
+
+def _load():
+    global _lib
+    if _lib is None:
+        if not os.path.exists(_LIB_PATH):
+            raise RuntimeError(f"{_LIB_PATH} missing: run __graft_entry__.build()")
+        lib = ctypes.CDLL(_LIB_PATH)
+        u32, u64, vp = ctypes.c_uint32, ctypes.c_uint64, ctypes.c_void_p
+        lib.oracle_sssp.argtypes = [u32, vp, vp, vp, u32, vp]
+        lib.oracle_sssp_many.argtypes = [u32, vp, vp, vp, vp, u64, vp, vp, u32]
+        lib.oracle_diameter.argtypes = [u32, vp, vp, vp, vp, u64, u32, vp]
+        lib.oracle_certify.argtypes = [u32, vp, vp, vp, u32, vp]
+        for f in (lib.oracle_sssp, lib.oracle_sssp_many, lib.oracle_diameter, lib.oracle_certify):
+            f.restype = ctypes.c_int
+        _lib = lib
+    return _lib
+
+
+def _csr(g):
+    first = np.ascontiguousarray(g.first, dtype=np.uint64)
+    head = np.ascontiguousarray(g.head, dtype=np.uint32)
+    ln = np.ascontiguousarray(g.len, dtype=np.uint32)
+    if head.size == 0:
+        head = np.zeros(1, np.uint32)
+        ln = np.zeros(1, np.uint32)
+    return first, head, ln
+
+
+def _threads(threads):
+    return int(threads) if threads else (os.cpu_count() or 1)
+
+
+def sssp(g, s: int) -> np.ndarray:
+    """uint32[n]: min(dist(s, v), INF) on the original graph."""
+    first, head, ln = _csr(g)
+    out = np.empty(g.n, dtype=np.uint32)
+    rc = _load().oracle_sssp(g.n, first.ctypes.data, head.ctypes.data, ln.ctypes.data, int(s),
+                             out.ctypes.data)
+    if rc:
+        raise ValueError(f"oracle_sssp: {rc}")
+    return out
+
+
+def sssp_many(g, sources, threads: int | None = None) -> np.ndarray:
+    """uint32[count, n]: one tree per source, one source per worker thread."""
+    first, head, ln = _csr(g)
+    src = np.ascontiguousarray(sources, dtype=np.uint32)
+    out = np.empty((src.size, g.n), dtype=np.uint32)
+    rc = _load().oracle_sssp_many(g.n, first.ctypes.data, head.ctypes.data, ln.ctypes.data,
+                                  src.ctypes.data, src.size, out.ctypes.data, None,
+                                  _threads(threads))
+    if rc:
+        raise ValueError(f"oracle_sssp_many: {rc}")
+    return out
+
+
+def tree_maxima(g, sources, threads: int | None = None) -> np.ndarray:
+    """uint32[count]: max finite label of each tree (no trees stored)."""
+    first, head, ln = _csr(g)
+    src = np.ascontiguousarray(sources, dtype=np.uint32)
+    maxs = np.empty(max(src.size, 1), dtype=np.uint32)
+    rc = _load().oracle_sssp_many(g.n, first.ctypes.data, head.ctypes.data, ln.ctypes.data,
+                                  src.ctypes.data, src.size, None, maxs.ctypes.data,
+                                  _threads(threads))
+    if rc:
+        raise ValueError(f"oracle_sssp_many: {rc}")
+    return maxs[: src.size]
+
+
+def diameter(g, sources, threads: int | None = None) -> int:
+    """max over sources s and vertices v with dist(s,v) != INF of dist(s,v)."""
+    first, head, ln = _csr(g)
+    src = np.ascontiguousarray(sources, dtype=np.uint32)
+    out = np.zeros(1, dtype=np.uint32)
+    rc = _load().oracle_diameter(g.n, first.ctypes.data, head.ctypes.data, ln.ctypes.data,
+                                 src.ctypes.data, src.size, _threads(threads), out.ctypes.data)
+    if rc:
+        raise ValueError(f"oracle_diameter: {rc}")
+    return int(out[0])
+
+
+def certify(g, s: int, d) -> int:
+    """0 iff d == min(dist(s, .), INF); else 1/2/3 = which optimality condition fails."""
+    first, head, ln = _csr(g)
+    d = np.ascontiguousarray(d, dtype=np.uint32)
+    if d.size != g.n:
+        raise ValueError("label vector has wrong length")
+    rc = _load().oracle_certify(g.n, first.ctypes.data, head.ctypes.data, ln.ctypes.data, int(s),
+                                d.ctypes.data)
+    if rc < 0:
+        raise ValueError(f"oracle_certify: {rc}")
+    return rc
