@@ -1,0 +1,268 @@
+"""Thin Python binding of libphast.so (include/phast.h) -- argument marshalling only.
+
+Every step of a PHAST query (upward CH search, seeding, the level-ordered downward
+sweep, the diameter max) runs in the library's sm_100a kernels; this module only
+converts arrays and torch tensors to pointers.  There is no CPU path: if the
+library is missing, importing this package raises.  PyTorch provides device
+memory and streams (plumbing only).
+
+Names follow include/phast.h; see DESIGN.md for the paper passages.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+from dataclasses import dataclass
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libphast.so")
+
+INF = 0xFFFFFFFF
+KMAX = 64
+K_ALLOWED = (1, 2, 4, 8, 16, 32, 64)
+FLAG_HOST_ONLY = 1
+
+STATUS = {0: "OK", -1: "EINVAL", -2: "ENOMEM", -3: "ECUDA", -4: "ERANGE", -5: "ESTATE", -6: "EIO",
+          -7: "EINTERNAL"}
+
+
+class PhastError(RuntimeError):
+    def __init__(self, fn, status):
+        self.status = status
+        super().__init__(f"{fn}: {STATUS.get(status, status)} ({_lib.phast_strerror(status).decode()})")
+
+
+class _Opts(ctypes.Structure):
+    _fields_ = [("hop_limit_lo", ctypes.c_uint32), ("hop_limit_hi", ctypes.c_uint32),
+                ("settled_cap", ctypes.c_uint32), ("threads", ctypes.c_uint32),
+                ("flags", ctypes.c_uint32), ("reserved", ctypes.c_uint32), ("seed", ctypes.c_uint64)]
+
+
+class _Info(ctypes.Structure):
+    _fields_ = [("n", ctypes.c_uint32), ("levels", ctypes.c_uint32), ("m", ctypes.c_uint64),
+                ("m_up", ctypes.c_uint64), ("m_down", ctypes.c_uint64), ("n_tail", ctypes.c_uint64),
+                ("shortcuts", ctypes.c_uint64), ("rounds", ctypes.c_uint32), ("device", ctypes.c_uint32),
+                ("build_seconds", ctypes.c_double)]
+
+
+def _load_lib():
+    if not os.path.exists(LIB_PATH):
+        raise RuntimeError(f"{LIB_PATH} is missing: build it with `python __graft_entry__.py` "
+                           "(there is no CPU fallback)")
+    lib = ctypes.CDLL(LIB_PATH)
+    u32, u64, vp = ctypes.c_uint32, ctypes.c_uint64, ctypes.c_void_p
+    pp = ctypes.POINTER(vp)
+    sig = {
+        "phast_build": ([u32, vp, vp, vp, ctypes.POINTER(_Opts), pp], ctypes.c_int),
+        "phast_trees": ([vp, vp, u32, vp, vp], ctypes.c_int),
+        "phast_trees_host": ([vp, vp, u32, vp, vp], ctypes.c_int),
+        "phast_sync": ([vp, vp], ctypes.c_int),
+        "phast_diameter": ([vp, vp, u64, u32, vp, vp, vp], ctypes.c_int),
+        "phast_info": ([vp, ctypes.POINTER(_Info)], ctypes.c_int),
+        "phast_level_sizes": ([vp, vp], ctypes.c_int),
+        "phast_order": ([vp, vp], ctypes.c_int),
+        "phast_export": ([vp, vp, vp, vp, vp, vp, vp, vp], ctypes.c_int),
+        "phast_save": ([vp, ctypes.c_char_p], ctypes.c_int),
+        "phast_load": ([ctypes.c_char_p, u32, pp], ctypes.c_int),
+        "phast_free": ([vp], None),
+        "phast_strerror": ([ctypes.c_int], ctypes.c_char_p),
+        "phast_launch_count": ([], u64),
+        "phast_timing": ([vp, ctypes.c_int], ctypes.c_int),
+        "phast_timing_read": ([vp, ctypes.POINTER(ctypes.c_double), ctypes.POINTER(ctypes.c_double),
+                               ctypes.POINTER(ctypes.c_uint64)], ctypes.c_int),
+    }
+    for name, (args, res) in sig.items():
+        f = getattr(lib, name)
+        f.argtypes = args
+        f.restype = res
+    return lib
+
+
+_lib = _load_lib()
+EXPORTED = ("phast_build", "phast_trees", "phast_trees_host", "phast_sync", "phast_diameter", "phast_info",
+            "phast_level_sizes", "phast_order", "phast_export", "phast_save", "phast_load", "phast_free",
+            "phast_strerror", "phast_launch_count", "phast_timing", "phast_timing_read")
+
+
+def _check(fn, rc):
+    if rc != 0:
+        raise PhastError(fn, rc)
+
+
+def launch_count() -> int:
+    """Kernels launched by libphast in this process."""
+    return int(_lib.phast_launch_count())
+
+
+def _stream_ptr(stream):
+    if stream is None:
+        import torch
+        return torch.cuda.current_stream().cuda_stream
+    return getattr(stream, "cuda_stream", stream)
+
+
+@dataclass
+class Info:
+    n: int
+    levels: int
+    m: int
+    m_up: int
+    m_down: int
+    n_tail: int
+    shortcuts: int
+    rounds: int
+    device: int
+    build_seconds: float
+
+
+class Phast:
+    """A built hierarchy bound to one CUDA device (phast_ctx)."""
+
+    def __init__(self, n=None, first=None, head=None, length=None, *, host_only=False, threads=0,
+                 hop_limit_lo=0, hop_limit_hi=0, settled_cap=0, _handle=None):
+        self._h = None
+        if _handle is not None:
+            self._h = _handle
+        else:
+            first = np.ascontiguousarray(first, dtype=np.uint64)
+            head = np.ascontiguousarray(head, dtype=np.uint32)
+            length = np.ascontiguousarray(length, dtype=np.uint32)
+            if head.size == 0:
+                head = np.zeros(1, np.uint32)
+                length = np.zeros(1, np.uint32)
+            o = _Opts(hop_limit_lo, hop_limit_hi, settled_cap, threads, FLAG_HOST_ONLY if host_only else 0, 0, 0)
+            h = ctypes.c_void_p()
+            _check("phast_build", _lib.phast_build(int(n), first.ctypes.data, head.ctypes.data,
+                                                   length.ctypes.data, ctypes.byref(o), ctypes.byref(h)))
+            self._h = h
+        inf = self.info()
+        self.n = inf.n
+        self.levels = inf.levels
+        self._perm = None
+
+    @classmethod
+    def from_graph(cls, g, **kw):
+        return cls(g.n, g.first, g.head, g.len, **kw)
+
+    @classmethod
+    def load(cls, path, host_only=False):
+        h = ctypes.c_void_p()
+        _check("phast_load", _lib.phast_load(path.encode(), FLAG_HOST_ONLY if host_only else 0, ctypes.byref(h)))
+        return cls(_handle=h)
+
+    def save(self, path):
+        _check("phast_save", _lib.phast_save(self._h, path.encode()))
+
+    def close(self):
+        if self._h is not None:
+            _lib.phast_free(self._h)
+            self._h = None
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.close()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    # ------------------------------------------------------------- queries
+    def trees(self, sources, out=None, stream=None):
+        """k = len(sources) trees; returns the device tensor [n, k] (uint32 bits in int32),
+        rows in internal order (see to_original)."""
+        import torch
+        src = np.ascontiguousarray(sources, dtype=np.uint32)
+        k = int(src.size)
+        if k not in K_ALLOWED:
+            raise ValueError(f"k must be one of {K_ALLOWED}, got {k}")
+        if out is None:
+            out = torch.empty((self.n, k), dtype=torch.int32, device="cuda")
+        _check("phast_trees", _lib.phast_trees(self._h, src.ctypes.data, k, out.data_ptr(), _stream_ptr(stream)))
+        return out
+
+    def trees_into(self, sources: np.ndarray, out_ptr: int, stream_ptr: int):
+        """Lowest-overhead form for the bench: raw pointers, no checks beyond the library's."""
+        _check("phast_trees", _lib.phast_trees(self._h, sources.ctypes.data, sources.size, out_ptr, stream_ptr))
+
+    def trees_host(self, sources, out: np.ndarray, stream=None):
+        """End-to-end entry with host buffers: result copied into `out` (uint32[n, k])."""
+        src = np.ascontiguousarray(sources, dtype=np.uint32)
+        assert out.dtype == np.uint32 and out.size == self.n * src.size and out.flags.c_contiguous
+        _check("phast_trees_host", _lib.phast_trees_host(self._h, src.ctypes.data, src.size, out.ctypes.data,
+                                                         _stream_ptr(stream)))
+        return out
+
+    def sync(self, stream=None):
+        _check("phast_sync", _lib.phast_sync(self._h, _stream_ptr(stream)))
+
+    def diameter(self, sources, k_batch=64, stream=None, batch_max=None):
+        """Max finite distance over the given sources (device-side; returns int after sync)."""
+        import torch
+        src = np.ascontiguousarray(sources, dtype=np.uint32)
+        out = torch.zeros(1, dtype=torch.int32, device="cuda")
+        bm_ptr = None if batch_max is None else batch_max.data_ptr()
+        _check("phast_diameter", _lib.phast_diameter(self._h, src.ctypes.data, src.size, k_batch, out.data_ptr(),
+                                                     bm_ptr, _stream_ptr(stream)))
+        self.sync(stream)
+        return int(out.cpu().numpy().view(np.uint32)[0])
+
+    def diameter_async(self, sources, k_batch, max_out, stream=None, batch_max=None):
+        src = np.ascontiguousarray(sources, dtype=np.uint32)
+        bm_ptr = None if batch_max is None else batch_max.data_ptr()
+        _check("phast_diameter", _lib.phast_diameter(self._h, src.ctypes.data, src.size, k_batch,
+                                                     max_out.data_ptr(), bm_ptr, _stream_ptr(stream)))
+
+    def timing(self, enable: bool):
+        _check("phast_timing", _lib.phast_timing(self._h, 1 if enable else 0))
+
+    def timing_read(self):
+        """(ms of upward+seed, ms of sweep+clear, batches) summed over recorded batches."""
+        a, b, c = ctypes.c_double(), ctypes.c_double(), ctypes.c_uint64()
+        _check("phast_timing_read", _lib.phast_timing_read(self._h, ctypes.byref(a), ctypes.byref(b), ctypes.byref(c)))
+        return a.value, b.value, c.value
+
+    # ------------------------------------------------------------- layout / stats
+    def info(self) -> Info:
+        i = _Info()
+        _check("phast_info", _lib.phast_info(self._h, ctypes.byref(i)))
+        return Info(i.n, i.levels, i.m, i.m_up, i.m_down, i.n_tail, i.shortcuts, i.rounds,
+                    -1 if i.device == 0xFFFFFFFF else i.device, i.build_seconds)
+
+    def level_sizes(self) -> np.ndarray:
+        out = np.empty(self.levels, np.uint32)
+        _check("phast_level_sizes", _lib.phast_level_sizes(self._h, out.ctypes.data))
+        return out
+
+    def order(self) -> np.ndarray:
+        """internal_of_original[v]."""
+        if self._perm is None:
+            out = np.empty(self.n, np.uint32)
+            _check("phast_order", _lib.phast_order(self._h, out.ctypes.data))
+            self._perm = out
+        return self._perm
+
+    def export(self) -> dict:
+        inf = self.info()
+        a = dict(lvl_off=np.empty(inf.levels + 1, np.uint32), dn_first=np.empty(inf.n + 1, np.uint32),
+                 dn_tail=np.empty(max(inf.m_down, 1), np.uint32), dn_len=np.empty(max(inf.m_down, 1), np.uint32),
+                 up_first=np.empty(inf.n + 1, np.uint32), up_head=np.empty(max(inf.m_up, 1), np.uint32),
+                 up_len=np.empty(max(inf.m_up, 1), np.uint32))
+        _check("phast_export", _lib.phast_export(self._h, *[a[k].ctypes.data for k in
+                                                           ("lvl_off", "dn_first", "dn_tail", "dn_len", "up_first",
+                                                            "up_head", "up_len")]))
+        a["dn_tail"] = a["dn_tail"][:inf.m_down]
+        a["dn_len"] = a["dn_len"][:inf.m_down]
+        a["up_head"] = a["up_head"][:inf.m_up]
+        a["up_len"] = a["up_len"][:inf.m_up]
+        return a
+
+    def to_original(self, rows: np.ndarray) -> np.ndarray:
+        """[n, k] internal-order labels (any 32-bit dtype) -> [k, n] uint32 in original ids."""
+        rows = np.asarray(rows).view(np.uint32).reshape(self.n, -1)
+        return np.ascontiguousarray(rows[self.order()].T)

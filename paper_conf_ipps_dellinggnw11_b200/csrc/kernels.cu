@@ -1,0 +1,375 @@
+// kernels.cu -- PHAST's hot path on sm_100a.
+//
+// a1 upward CH search  : one CTA per source, exact labels in G-up by label-correcting
+//                        relaxation over a shared-memory hash table (global fallback).
+//                        PAPER.md:14 §III "it runs Dijkstra's algorithm from s in G-up,
+//                        stopping when the priority queue becomes empty"; any method
+//                        giving exact G-up distances is valid (reading R9).
+// a2 seed + implicit init: visited bits (§IV-C "we mark vertices visited
+//                        during the CH search with a single bit"), rows of the search
+//                        space reset to INF, then labels scattered (two launches so
+//                        every reset precedes every scatter).
+// a3 downward sweep    : per level, d(v) = min(flag(v) ? d(v) : INF,
+//                        min_{(u,v) in A-down} sat(d(u) + l(u,v))) for k trees at once
+//                        (§III, §IV-B).  k/4 lanes per vertex,
+//                        16-byte label loads per lane (the B200 analogue of "four trees
+//                        per SSE register", §IV-B).
+// a5 diameter          : max over finite labels fused into the sweep (PAPER.md:20
+//                        §VII-B "making each core keep track of the maximum label it
+//                        encounters").
+// No tensor cores: the loop is an integer (min,+) gather with no reuse.
+#include <atomic>
+#include <cstdio>
+
+#include "kernels.h"
+
+namespace phast {
+
+static std::atomic<uint64_t> g_launches{0};
+uint64_t launches() { return g_launches.load(); }
+
+int num_sms() {
+    static int sms = 0;
+    if (!sms) {
+        int dev = 0;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+        if (sms <= 0) sms = 148;
+    }
+    return sms;
+}
+
+namespace {
+
+constexpr uint32_t EMPTY = 0xFFFFFFFFu;
+constexpr int UP_THREADS = 512;
+constexpr uint32_t UP_SMEM_CAP = 4096;   // shared-memory table entries per source
+
+__device__ __forceinline__ uint32_t sat_add(uint32_t a, uint32_t l) {
+    // min(a + l, INF) without wrap: min(a, INF - l) + l   (reading R1)
+    return min(a, INF - l) + l;
+}
+__device__ __forceinline__ uint32_t hash32(uint32_t x) {
+    x ^= x >> 16; x *= 0x7feb352dU; x ^= x >> 15; x *= 0x846ca68bU; x ^= x >> 16;
+    return x;
+}
+
+// ------------------------------------------------------------------ a1 upward
+struct UpTable {
+    uint32_t* keys;
+    uint32_t* vals;
+    uint32_t* inq;
+    uint32_t* qa;
+    uint32_t* qb;
+    uint32_t cap;  // power of two
+};
+
+struct UpShared {
+    uint32_t qn, nn, used, over, cnt;
+};
+
+// Returns the slot of w (inserting it), or EMPTY when the table is 3/4 full.
+__device__ __forceinline__ uint32_t up_insert(const UpTable& t, uint32_t w, UpShared& c) {
+    uint32_t mask = t.cap - 1;
+    uint32_t h = hash32(w) & mask;
+    for (uint32_t probe = 0; probe < t.cap; probe++) {
+        uint32_t k = *((volatile uint32_t*)&t.keys[h]);
+        if (k == w) return h;
+        if (k == EMPTY) {
+            if (atomicAdd(&c.used, 0u) * 4 >= t.cap * 3) return EMPTY;
+            uint32_t old = atomicCAS(&t.keys[h], EMPTY, w);
+            if (old == EMPTY) { atomicAdd(&c.used, 1u); return h; }
+            if (old == w) return h;
+        }
+        h = (h + 1) & mask;
+    }
+    return EMPTY;
+}
+
+// Label-correcting relaxation of G-up from s, wave-synchronous; on return the
+// table holds exact G-up distances of every vertex reachable from s (Bellman-Ford
+// fixed point with saturating sums).  Returns false on table overflow.
+__device__ bool up_search(const uint32_t* __restrict__ up_first, const uint2* __restrict__ up_arc,
+                          uint32_t s, UpTable t, UpShared& c) {
+    const uint32_t tid = threadIdx.x;
+    for (uint32_t i = tid; i < t.cap; i += blockDim.x) { t.keys[i] = EMPTY; t.vals[i] = INF; t.inq[i] = 0; }
+    __syncthreads();
+    if (tid == 0) {
+        uint32_t h = hash32(s) & (t.cap - 1);
+        t.keys[h] = s; t.vals[h] = 0; t.inq[h] = 1; t.qa[0] = h;
+        c.qn = 1; c.nn = 0; c.used = 1; c.over = 0; c.cnt = 0;
+    }
+    __syncthreads();
+    uint32_t* qa = t.qa;
+    uint32_t* qb = t.qb;
+    for (;;) {
+        uint32_t qn = c.qn;
+        if (qn == 0 || c.over) break;
+        for (uint32_t idx = tid; idx < qn; idx += blockDim.x) {
+            uint32_t slot = qa[idx];
+            atomicExch(&t.inq[slot], 0u);
+            __threadfence_block();
+            uint32_t v = t.keys[slot];
+            uint32_t dv = *((volatile uint32_t*)&t.vals[slot]);
+            uint32_t e1 = __ldg(&up_first[v + 1]);
+            for (uint32_t e = __ldg(&up_first[v]); e < e1; e++) {
+                uint2 a = __ldg(&up_arc[e]);
+                uint32_t nd = sat_add(dv, a.y);
+                if (nd == INF) continue;
+                uint32_t ws = up_insert(t, a.x, c);
+                if (ws == EMPTY) { c.over = 1; break; }
+                uint32_t old = atomicMin(&t.vals[ws], nd);
+                if (nd < old) {
+                    __threadfence_block();
+                    if (atomicExch(&t.inq[ws], 1u) == 0u) qb[atomicAdd(&c.nn, 1u)] = ws;
+                }
+            }
+        }
+        __syncthreads();
+        if (tid == 0) { c.qn = c.nn; c.nn = 0; }
+        uint32_t* tmp = qa; qa = qb; qb = tmp;
+        __syncthreads();
+    }
+    bool ok = !c.over;
+    __syncthreads();
+    return ok;
+}
+
+template <int K>
+__global__ void __launch_bounds__(UP_THREADS) upward_kernel(DevImage g, Sources src, uint32_t* __restrict__ dist) {
+    extern __shared__ uint32_t smem[];
+    __shared__ UpShared c;
+    const uint32_t i = blockIdx.x;
+    const uint32_t s = src.s[i];
+    const uint32_t sc = g.smem_cap;
+    UpTable t{smem, smem + sc, smem + 2 * sc, smem + 3 * sc, smem + 4 * sc, sc};
+    bool ok = up_search(g.up_first, g.up_arc, s, t, c);
+    if (!ok) {   // global-memory fallback with the per-source capacity
+        uint32_t* base = g.gscratch + (size_t)i * g.seed_cap * 5;
+        UpTable gt{base, base + g.seed_cap, base + 2 * (size_t)g.seed_cap, base + 3 * (size_t)g.seed_cap,
+                   base + 4 * (size_t)g.seed_cap, g.seed_cap};
+        t = gt;
+        ok = up_search(g.up_first, g.up_arc, s, t, c);
+        if (!ok) {
+            if (threadIdx.x == 0) { atomicOr(g.err, 1u); g.seed_cnt[i] = 0; }
+            return;
+        }
+    }
+    // emit the search space, set visited bits
+    uint32_t* sv = g.seed_v + (size_t)i * g.seed_cap;
+    uint32_t* sd = g.seed_d + (size_t)i * g.seed_cap;
+    for (uint32_t slot = threadIdx.x; slot < t.cap; slot += blockDim.x) {
+        uint32_t v = t.keys[slot];
+        if (v == EMPTY) continue;
+        uint32_t pos = atomicAdd(&c.cnt, 1u);
+        sv[pos] = v;
+        sd[pos] = t.vals[slot];
+        atomicOr(&g.flags[v >> 5], 1u << (v & 31));
+    }
+    __syncthreads();
+    const uint32_t cnt = c.cnt;
+    if (threadIdx.x == 0) g.seed_cnt[i] = cnt;
+    // reset the rows of the search space to INF (phase 1 of a2)
+    if constexpr (K % 4 == 0) {
+        constexpr uint32_t W = K / 4;
+        const uint4 inf4 = make_uint4(INF, INF, INF, INF);
+        for (uint32_t j = threadIdx.x; j < cnt * W; j += blockDim.x)
+            reinterpret_cast<uint4*>(dist + (size_t)sv[j / W] * K)[j % W] = inf4;
+    } else {
+        for (uint32_t j = threadIdx.x; j < cnt * K; j += blockDim.x) dist[(size_t)sv[j / K] * K + j % K] = INF;
+    }
+}
+
+__global__ void scatter_kernel(DevImage g, uint32_t k, uint32_t* __restrict__ dist) {
+    const uint32_t i = blockIdx.x;
+    const uint32_t cnt = g.seed_cnt[i];
+    const uint32_t* sv = g.seed_v + (size_t)i * g.seed_cap;
+    const uint32_t* sd = g.seed_d + (size_t)i * g.seed_cap;
+    for (uint32_t j = threadIdx.x; j < cnt; j += blockDim.x) dist[(size_t)sv[j] * k + i] = sd[j];
+}
+
+__global__ void clear_flags_kernel(DevImage g) {
+    const uint32_t i = blockIdx.x;
+    const uint32_t cnt = g.seed_cnt[i];
+    const uint32_t* sv = g.seed_v + (size_t)i * g.seed_cap;
+    for (uint32_t j = threadIdx.x; j < cnt; j += blockDim.x) g.flags[sv[j] >> 5] = 0u;
+}
+
+// ------------------------------------------------------------------ a3 sweep
+template <int K> struct RowT;
+template <> struct RowT<1> { using T = uint32_t; static constexpr int W = 1; };
+template <> struct RowT<2> { using T = uint2; static constexpr int W = 2; };
+template <int K> struct RowT { using T = uint4; static constexpr int W = 4; };
+
+__device__ __forceinline__ uint32_t vinf(uint32_t) { return INF; }
+__device__ __forceinline__ uint32_t relax(uint32_t acc, uint32_t x, uint32_t l) { return min(acc, sat_add(x, l)); }
+__device__ __forceinline__ uint2 relax(uint2 acc, uint2 x, uint32_t l) {
+    uint32_t c = INF - l;
+    return make_uint2(min(acc.x, min(x.x, c) + l), min(acc.y, min(x.y, c) + l));
+}
+__device__ __forceinline__ uint4 relax(uint4 acc, uint4 x, uint32_t l) {
+    uint32_t c = INF - l;
+    return make_uint4(min(acc.x, min(x.x, c) + l), min(acc.y, min(x.y, c) + l),
+                      min(acc.z, min(x.z, c) + l), min(acc.w, min(x.w, c) + l));
+}
+__device__ __forceinline__ uint32_t fmax_of(uint32_t a) { return a == INF ? 0u : a; }
+__device__ __forceinline__ uint32_t fmax_of(uint2 a) { return max(fmax_of(a.x), fmax_of(a.y)); }
+__device__ __forceinline__ uint32_t fmax_of(uint4 a) {
+    return max(max(fmax_of(a.x), fmax_of(a.y)), max(fmax_of(a.z), fmax_of(a.w)));
+}
+template <class T> __device__ __forceinline__ T inf_row();
+template <> __device__ __forceinline__ uint32_t inf_row<uint32_t>() { return INF; }
+template <> __device__ __forceinline__ uint2 inf_row<uint2>() { return make_uint2(INF, INF); }
+template <> __device__ __forceinline__ uint4 inf_row<uint4>() { return make_uint4(INF, INF, INF, INF); }
+
+template <class T> __device__ __forceinline__ void st_stream(T* p, T v) { __stcs(p, v); }
+
+constexpr int SWEEP_THREADS = 256;
+
+template <int K, bool DIAM, bool STORE, bool STREAM>
+__global__ void __launch_bounds__(SWEEP_THREADS) sweep_kernel(const uint32_t* __restrict__ first,
+                                                               const uint2* __restrict__ arcs,
+                                                               uint32_t* __restrict__ d,
+                                                               const uint32_t* __restrict__ flags,
+                                                               uint32_t vbeg, uint32_t vend,
+                                                               uint32_t* __restrict__ diam) {
+    using T = typename RowT<K>::T;
+    constexpr uint32_t W = RowT<K>::W;
+    constexpr uint32_t G = K / W;   // lanes per vertex
+    const uint64_t total = (uint64_t)(vend - vbeg) * G;
+    uint32_t mx = 0;
+    for (uint64_t t = (uint64_t)blockIdx.x * SWEEP_THREADS + threadIdx.x; t < total;
+         t += (uint64_t)gridDim.x * SWEEP_THREADS) {
+        const uint32_t v = vbeg + (uint32_t)(t / G);
+        const uint32_t lane = (uint32_t)(t % G);
+        T acc = inf_row<T>();
+        if ((__ldg(&flags[v >> 5]) >> (v & 31)) & 1u)   // visited by an upward search
+            acc = __ldg(reinterpret_cast<const T*>(d + (size_t)v * K) + lane);
+        const uint32_t e0 = __ldg(&first[v]), e1 = __ldg(&first[v + 1]);
+#pragma unroll 4
+        for (uint32_t e = e0; e < e1; e++) {
+            const uint2 a = __ldg(&arcs[e]);
+            const T x = __ldg(reinterpret_cast<const T*>(d + (size_t)a.x * K) + lane);
+            acc = relax(acc, x, a.y);
+        }
+        if constexpr (STORE) {
+            T* p = reinterpret_cast<T*>(d + (size_t)v * K) + lane;
+            if constexpr (STREAM) st_stream(p, acc); else *p = acc;
+        }
+        if constexpr (DIAM) mx = max(mx, fmax_of(acc));
+    }
+    if constexpr (DIAM) {
+        __shared__ uint32_t wmax[SWEEP_THREADS / 32];
+        mx = __reduce_max_sync(0xFFFFFFFFu, mx);
+        if ((threadIdx.x & 31) == 0) wmax[threadIdx.x >> 5] = mx;
+        __syncthreads();
+        if (threadIdx.x < 32) {
+            uint32_t w = threadIdx.x < SWEEP_THREADS / 32 ? wmax[threadIdx.x] : 0u;
+            w = __reduce_max_sync(0xFFFFFFFFu, w);
+            if (threadIdx.x == 0 && w) atomicMax(diam, w);
+        }
+    }
+}
+
+template <int K, bool DIAM, bool STORE, bool STREAM>
+cudaError_t sweep_launch(const DevImage& g, uint32_t vbeg, uint32_t vend, uint32_t* dist, uint32_t* diam,
+                         cudaStream_t st) {
+    constexpr uint32_t G = K / RowT<K>::W;
+    uint64_t total = (uint64_t)(vend - vbeg) * G;
+    uint64_t blocks = (total + SWEEP_THREADS - 1) / SWEEP_THREADS;
+    uint64_t cap = (uint64_t)num_sms() * 8;
+    if (blocks > cap) blocks = cap;
+    if (blocks == 0) return cudaSuccess;
+    sweep_kernel<K, DIAM, STORE, STREAM><<<(unsigned)blocks, SWEEP_THREADS, 0, st>>>(g.dn_first, g.dn_arc, dist,
+                                                                                 g.flags, vbeg, vend, diam);
+    g_launches++;
+    return cudaGetLastError();
+}
+
+template <int K>
+cudaError_t sweep_k(const DevImage& g, uint32_t vbeg, uint32_t vend, uint32_t* dist, uint32_t* diam, bool store,
+                    bool last, cudaStream_t st) {
+    if (diam) {
+        if (!store) return sweep_launch<K, true, false, false>(g, vbeg, vend, dist, diam, st);
+        return last ? sweep_launch<K, true, true, true>(g, vbeg, vend, dist, diam, st)
+                    : sweep_launch<K, true, true, false>(g, vbeg, vend, dist, diam, st);
+    }
+    return last ? sweep_launch<K, false, true, true>(g, vbeg, vend, dist, diam, st)
+                : sweep_launch<K, false, true, false>(g, vbeg, vend, dist, diam, st);
+}
+
+template <int K>
+cudaError_t upward_k(const DevImage& g, const Sources& src, uint32_t k, uint32_t* dist, cudaStream_t st) {
+    static bool attr = false;
+    size_t smem = 5 * (size_t)g.smem_cap * sizeof(uint32_t);
+    if (!attr) {
+        cudaError_t e = cudaFuncSetAttribute(upward_kernel<K>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                             (int)(5 * UP_SMEM_CAP * sizeof(uint32_t)));
+        if (e != cudaSuccess) return e;
+        attr = true;
+    }
+    upward_kernel<K><<<k, UP_THREADS, smem, st>>>(g, src, dist);
+    g_launches++;
+    return cudaGetLastError();
+}
+
+__global__ void max_reduce_kernel(const uint32_t* __restrict__ in, uint32_t count, uint32_t* out) {
+    uint32_t mx = 0;
+    for (uint32_t i = threadIdx.x; i < count; i += blockDim.x) mx = max(mx, in[i]);
+    __shared__ uint32_t w[32];
+    mx = __reduce_max_sync(0xFFFFFFFFu, mx);
+    if ((threadIdx.x & 31) == 0) w[threadIdx.x >> 5] = mx;
+    __syncthreads();
+    if (threadIdx.x < 32) {
+        uint32_t x = threadIdx.x < blockDim.x / 32 ? w[threadIdx.x] : 0u;
+        x = __reduce_max_sync(0xFFFFFFFFu, x);
+        if (threadIdx.x == 0) *out = x;
+    }
+}
+
+}  // namespace
+
+#define PHAST_K_SWITCH(k, CALL)      \
+    switch (k) {                     \
+        case 1: return CALL(1);      \
+        case 2: return CALL(2);      \
+        case 4: return CALL(4);      \
+        case 8: return CALL(8);      \
+        case 16: return CALL(16);    \
+        case 32: return CALL(32);    \
+        case 64: return CALL(64);    \
+        default: return cudaErrorInvalidValue; \
+    }
+
+cudaError_t launch_upward(const DevImage& g, const Sources& src, uint32_t k, uint32_t* dist, cudaStream_t st) {
+#define CALL_UP(K) upward_k<K>(g, src, k, dist, st)
+    PHAST_K_SWITCH(k, CALL_UP)
+#undef CALL_UP
+}
+
+cudaError_t launch_scatter(const DevImage& g, uint32_t k, uint32_t* dist, cudaStream_t st) {
+    scatter_kernel<<<k, 256, 0, st>>>(g, k, dist);
+    g_launches++;
+    return cudaGetLastError();
+}
+
+cudaError_t launch_sweep_level(const DevImage& g, uint32_t k, uint32_t vbeg, uint32_t vend, uint32_t* dist,
+                               uint32_t* diam, bool store, bool last_level, cudaStream_t st) {
+#define CALL_SW(K) sweep_k<K>(g, vbeg, vend, dist, diam, store, last_level, st)
+    PHAST_K_SWITCH(k, CALL_SW)
+#undef CALL_SW
+}
+
+cudaError_t launch_clear_flags(const DevImage& g, uint32_t k, cudaStream_t st) {
+    clear_flags_kernel<<<k, 256, 0, st>>>(g);
+    g_launches++;
+    return cudaGetLastError();
+}
+
+cudaError_t launch_max_reduce(const uint32_t* in, uint32_t count, uint32_t* out, cudaStream_t st) {
+    max_reduce_kernel<<<1, 1024, 0, st>>>(in, count, out);
+    g_launches++;
+    return cudaGetLastError();
+}
+
+}  // namespace phast

@@ -1,0 +1,52 @@
+// kernels.h -- internal launch API of libphast's sm_100a kernels (not the C ABI).
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+
+namespace phast {
+
+constexpr uint32_t INF = 0xFFFFFFFFu;
+constexpr uint32_t KMAX = 64;
+
+// Device image of the hierarchy + per-handle scratch (all device pointers).
+struct DevImage {
+    uint32_t n = 0;
+    const uint32_t* dn_first = nullptr;  // [n+1]   G-down in-arcs by head (internal ids)
+    const uint2* dn_arc = nullptr;       // [m_down] {tail, len}
+    const uint32_t* up_first = nullptr;  // [n+1]   G-up out-arcs by tail
+    const uint2* up_arc = nullptr;       // [m_up]   {head, len}
+    uint32_t* flags = nullptr;           // [ceil(n/32)] visited bits (§IV-C), zero between calls
+    uint32_t* seed_v = nullptr;          // [KMAX * seed_cap] upward search spaces: vertex
+    uint32_t* seed_d = nullptr;          // [KMAX * seed_cap] upward search spaces: label
+    uint32_t* seed_cnt = nullptr;        // [KMAX]
+    uint32_t* gscratch = nullptr;        // [KMAX * seed_cap * 5] global-memory fallback tables
+    uint32_t* err = nullptr;             // [1] sticky device error word
+    uint32_t seed_cap = 0;               // entries per source (power of two)
+    uint32_t smem_cap = 4096;            // shared-memory table entries (power of two, <= 4096)
+};
+
+struct Sources {
+    uint32_t s[KMAX];  // internal ids, passed by value in the kernel parameter space
+};
+
+// a1 + a2 (phase 1): one CTA per source; exact G-up labels; writes the search space
+// to seed_*, sets the visited bits, and resets the rows of the search space to INF.
+cudaError_t launch_upward(const DevImage& g, const Sources& src, uint32_t k, uint32_t* dist,
+                          cudaStream_t st);
+// a2 (phase 2): dist[v*k + i] = label_i(v) for every search-space entry of source i.
+cudaError_t launch_scatter(const DevImage& g, uint32_t k, uint32_t* dist, cudaStream_t st);
+// a3: one level [vbeg, vend) of the downward sweep; diam != nullptr fuses the max (a5);
+// store == false skips the row stores (diameter mode, level 0 rows are never read).
+cudaError_t launch_sweep_level(const DevImage& g, uint32_t k, uint32_t vbeg, uint32_t vend,
+                               uint32_t* dist, uint32_t* diam, bool store, bool last_level,
+                               cudaStream_t st);
+// after the sweep: clear the visited bits of every search-space vertex ("After
+// scanning v we unmark the vertex", §IV-C).
+cudaError_t launch_clear_flags(const DevImage& g, uint32_t k, cudaStream_t st);
+// max of per-batch maxima (diameter)
+cudaError_t launch_max_reduce(const uint32_t* in, uint32_t count, uint32_t* out, cudaStream_t st);
+
+uint64_t launches();
+int num_sms();
+
+}  // namespace phast

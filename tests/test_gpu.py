@@ -1,0 +1,205 @@
+"""GPU parity tests (-m gpu): the CUDA path, called through the C ABI, against the
+oracle, element by element, bit-exact (all lengths and labels are uint32; Theorem
+3.1, §III makes PHAST exact, so the bar is equality)."""
+import numpy as np
+import pytest
+
+import oracle
+import phastgen
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+if not torch.cuda.is_available():
+    pytest.skip("no CUDA device", allow_module_level=True)
+
+import paper_conf_ipps_dellinggnw11_b200 as P  # noqa: E402
+
+INF = 0xFFFFFFFF
+
+
+def gpu_trees(h, src, stream=None):
+    d = h.trees(np.asarray(src, np.uint32), stream=stream)
+    h.sync(stream)
+    return h.to_original(d.cpu().numpy())
+
+
+@pytest.fixture(scope="module")
+def c1():
+    g = phastgen.CONFIGS["C1"]["graph"]()
+    return g, P.Phast.from_graph(g)
+
+
+@pytest.fixture(scope="module")
+def road():
+    g = phastgen.road(150_000, seed=31)
+    return g, P.Phast.from_graph(g)
+
+
+def test_library_is_the_cuda_path():
+    # the package imports libphast.so (no CPU fallback exists); kernels count up
+    before = P.launch_count()
+    g = phastgen.grid(8, 8)
+    with P.Phast.from_graph(g) as h:
+        gpu_trees(h, [0])
+    assert P.launch_count() > before
+
+
+def test_c1_all_sources(c1):
+    """C1: 100x100 grid, every one of the 10 000 sources, k=64 batches (+ k=1 on a
+    sample), bit-exact."""
+    g, h = c1
+    want = oracle.sssp_many(g, np.arange(g.n))
+    for b in range(0, g.n, 64):
+        src = np.arange(b, b + 64) % g.n
+        got = gpu_trees(h, src)
+        assert np.array_equal(got, want[src]), b
+    for s in (0, 5050, 9999, 123):
+        assert np.array_equal(gpu_trees(h, [s])[0], want[s])
+
+
+@pytest.mark.parametrize("k", P.K_ALLOWED)
+def test_every_k_with_duplicates(road, k):
+    g, h = road
+    src = phastgen.sources(g.n, k, seed=100 + k, distinct=False)
+    if k >= 4:
+        src[1] = src[0]                      # duplicate sources are allowed
+    got = gpu_trees(h, src)
+    assert np.array_equal(got, oracle.sssp_many(g, src))
+
+
+def test_repeated_calls_no_stale_state(road):
+    """Visited bits and seeded rows must not leak between calls (§IV-C
+    "After scanning v we unmark the vertex")."""
+    g, h = road
+    out = torch.empty((g.n, 16), dtype=torch.int32, device="cuda")
+    for rep in range(4):
+        src = phastgen.sources(g.n, 16, seed=200 + rep)
+        h.trees(src, out=out)
+        h.sync()
+        assert np.array_equal(h.to_original(out.cpu().numpy()), oracle.sssp_many(g, src)), rep
+    # same buffer, alternating k
+    for k in (64, 1, 32, 4):
+        src = phastgen.sources(g.n, k, seed=300 + k)
+        assert np.array_equal(gpu_trees(h, src), oracle.sssp_many(g, src))
+
+
+EDGE_GRAPHS = {
+    "zero_lengths": lambda: phastgen.random_digraph(500, 1800, 0, 3, seed=41),
+    "grid_zero": lambda: phastgen.grid(80, 40, 0, 4, seed=46),
+    "saturating": lambda: phastgen.random_digraph(1500, 6000, 1 << 30, 0xFFFFFFFF, seed=42),
+    "unreachable": lambda: phastgen.random_digraph(4000, 3000, 1, 1000, seed=43),
+    "unit_grid": lambda: phastgen.grid(70, 30, 1, 2, seed=44),
+}
+
+
+@pytest.mark.parametrize("name", sorted(EDGE_GRAPHS))
+def test_edge_case_graphs(name):
+    g = EDGE_GRAPHS[name]()
+    with P.Phast.from_graph(g) as h:
+        for k in (1, 16, 64):
+            src = phastgen.sources(g.n, k, seed=7 + k)
+            assert np.array_equal(gpu_trees(h, src), oracle.sssp_many(g, src)), k
+
+
+def test_upward_global_fallback_and_overflow(monkeypatch):
+    """A shared-memory table too small for the search space falls back to the global
+    table (same labels); a per-source capacity too small is reported as ERANGE by
+    phast_sync (never silently wrong labels)."""
+    g = phastgen.grid(100, 100, 1, 1 << 20, seed=1)   # upward spaces ~200-300 vertices
+    src = phastgen.sources(g.n, 16, seed=3)
+    want = oracle.sssp_many(g, src)
+    monkeypatch.setenv("PHAST_UP_SMEM_CAP", "32")
+    with P.Phast.from_graph(g) as h:
+        assert np.array_equal(gpu_trees(h, src), want)
+    monkeypatch.setenv("PHAST_SEED_CAP", "32")
+    with P.Phast.from_graph(g) as h:
+        h.trees(src)
+        with pytest.raises(P.PhastError) as e:
+            h.sync()
+        assert e.value.status == -4
+        h.sync()                                       # error word is cleared
+
+
+def test_tiny_and_degenerate():
+    for g in (phastgen.Graph(1, np.array([0, 0], np.uint64), np.zeros(0, np.uint32), np.zeros(0, np.uint32)),
+              phastgen.grid(1, 2), phastgen.grid(3, 1, 0, 1)):
+        with P.Phast.from_graph(g) as h:
+            src = np.zeros(4, np.uint32)
+            src[1::2] = g.n - 1
+            assert np.array_equal(gpu_trees(h, src), oracle.sssp_many(g, src))
+
+
+def test_source_out_of_range(road):
+    g, h = road
+    with pytest.raises(P.PhastError) as e:
+        h.trees(np.array([g.n], np.uint32))
+    assert e.value.status == -4
+    with pytest.raises(ValueError):
+        h.trees(np.zeros(3, np.uint32))
+
+
+def test_host_entry_point(road):
+    g, h = road
+    src = phastgen.sources(g.n, 8, seed=77)
+    out = np.empty((g.n, 8), np.uint32)
+    h.trees_host(src, out)
+    assert np.array_equal(h.to_original(out), oracle.sssp_many(g, src))
+
+
+def test_diameter_c1_all_sources(c1):
+    """Exact diameter (§VII-B) of C1 over all 10 000 sources; per-batch
+    maxima against the oracle's per-tree maxima; count not divisible by k_batch."""
+    g, h = c1
+    allsrc = np.arange(g.n, dtype=np.uint32)
+    tm = oracle.tree_maxima(g, allsrc)
+    assert h.diameter(allsrc, k_batch=64) == int(tm.max())
+    sub = allsrc[:1000]                      # 1000 = 15*64 + 40: ragged last batch
+    bm = torch.zeros(16, dtype=torch.int32, device="cuda")
+    d = h.diameter(sub, k_batch=64, batch_max=bm)
+    assert d == int(tm[:1000].max())
+    bmv = bm.cpu().numpy().view(np.uint32)
+    for b in range(16):
+        assert bmv[b] == tm[b * 64:(b + 1) * 64].max(), b
+    for kb in (1, 16):
+        assert h.diameter(sub[:37], k_batch=kb) == int(tm[:37].max())
+
+
+def test_diameter_road_and_unreachable(road):
+    g, h = road
+    src = phastgen.sources(g.n, 100, seed=5)
+    assert h.diameter(src, k_batch=32) == oracle.diameter(g, src)
+    g2 = EDGE_GRAPHS["unreachable"]()
+    with P.Phast.from_graph(g2) as h2:
+        src = np.arange(0, g2.n, 7, dtype=np.uint32)
+        assert h2.diameter(src, k_batch=64) == oracle.diameter(g2, src)
+
+
+def test_c2_1m_k16():
+    """C2: ~1M-vertex road-like graph, k=16 (BASELINE.json configs[1]), all 16
+    trees bit-exact, then a 64-tree batch certified by the O(n+m) certificate."""
+    cfg = phastgen.CONFIGS["C2"]
+    g = cfg["graph"]()
+    with P.Phast.from_graph(g) as h:
+        src = phastgen.sources(g.n, 16, seed=cfg["src_seed"])
+        assert np.array_equal(gpu_trees(h, src), oracle.sssp_many(g, src))
+        src64 = phastgen.sources(g.n, 64, seed=cfg["src_seed"] + 1)
+        got = gpu_trees(h, src64)
+        for i in range(64):
+            assert oracle.certify(g, int(src64[i]), got[i]) == 0, i
+
+
+@pytest.mark.slow
+def test_c3_europe_scale_bench_config():
+    """C3 at full size (~18M vertices, ~42M arcs) in the bench's launch configuration
+    (k=64): 4 sampled trees bit-exact against the oracle, 16 more certified."""
+    cfg = phastgen.CONFIGS["C3"]
+    g = cfg["graph"]()
+    with P.Phast.from_graph(g) as h:
+        src = phastgen.sources(g.n, 64, seed=cfg["src_seed"])
+        got = gpu_trees(h, src)
+        pick = [0, 17, 40, 63]
+        want = oracle.sssp_many(g, src[pick])
+        assert np.array_equal(got[pick], want)
+        for i in range(1, 64, 4):
+            assert oracle.certify(g, int(src[i]), got[i]) == 0, i

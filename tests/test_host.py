@@ -1,0 +1,166 @@
+"""Host-side tests (-m "not gpu"): the C ABI library loads and exports every symbol
+include/phast.h declares; the host CH build and layout are correct (checked through
+a numpy re-execution of PHAST's two subphases against the oracle); Lemma 4.1 and
+the level layout hold; save/load round-trips; invalid input is rejected.  No
+compute call here touches a GPU (handles are built with PHAST_FLAG_HOST_ONLY)."""
+import os
+import re
+
+import numpy as np
+import pytest
+
+import oracle
+import phastgen
+import chref
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+P = pytest.importorskip("paper_conf_ipps_dellinggnw11_b200")
+
+
+def declared_symbols():
+    src = open(os.path.join(ROOT, "include", "phast.h")).read()
+    src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
+    return sorted(set(re.findall(r"\b(phast_[a-z_]+)\s*\(", src)))
+
+
+def test_library_exports_every_declared_symbol():
+    import ctypes
+    lib = ctypes.CDLL(P.LIB_PATH)
+    syms = declared_symbols()
+    assert len(syms) == len(P.EXPORTED)
+    for s in syms:
+        assert hasattr(lib, s), s
+    assert set(P.EXPORTED) <= set(syms)
+
+
+def test_strerror_and_launch_count():
+    assert P._lib.phast_strerror(0) == b"ok"
+    assert P._lib.phast_strerror(-4) == b"value out of range"
+    assert P.launch_count() >= 0
+
+
+GRAPHS = {
+    "grid": lambda: phastgen.grid(60, 40, 1, 1 << 20, seed=1),
+    "unit_grid": lambda: phastgen.grid(50, 50, 1, 2, seed=2),
+    "road": lambda: phastgen.road(60_000, seed=9),
+    "rand_zero": lambda: phastgen.random_digraph(400, 1400, 0, 4, seed=3),
+    "grid_zero": lambda: phastgen.grid(40, 30, 0, 4, seed=6),
+    "rand_sat": lambda: phastgen.random_digraph(800, 4000, 1 << 30, 0xFFFFFFFF, seed=4),
+    "rand_sparse": lambda: phastgen.random_digraph(3000, 2500, 1, 100, seed=5),
+}
+
+
+@pytest.mark.parametrize("name", sorted(GRAPHS))
+def test_host_hierarchy_sweep_equals_oracle(name):
+    """Theorem 3.1 (§III) on the built hierarchy: upward search + level
+    sweep over the exported G-up/G-down equals Dijkstra on the original graph."""
+    g = GRAPHS[name]()
+    h = P.Phast.from_graph(g, host_only=True)
+    ex = h.export()
+    src = np.concatenate([phastgen.sources(g.n, 6, seed=7), [0, g.n - 1]]).astype(np.uint32)
+    got = chref.phast_cpu(h, ex, src)
+    want = oracle.sssp_many(g, src)
+    assert np.array_equal(got, want)
+
+
+@pytest.mark.parametrize("name", sorted(GRAPHS))
+def test_layout_invariants(name):
+    g = GRAPHS[name]()
+    h = P.Phast.from_graph(g, host_only=True)
+    ex = h.export()
+    n, L = h.n, h.levels
+    lo = ex["lvl_off"]
+    assert lo[0] == 0 and lo[-1] == n and np.all(np.diff(lo.astype(np.int64)) > 0)
+    # level index of every internal id (0 = top level, processed first)
+    lev = np.repeat(np.arange(L), np.diff(lo.astype(np.int64)))
+    heads = np.repeat(np.arange(n), np.diff(ex["dn_first"].astype(np.int64)))
+    # Lemma 4.1 (§IV-A): every tail of a G-down arc is on a strictly higher
+    # level, i.e. processed in an earlier level group
+    assert np.all(lev[ex["dn_tail"]] < lev[heads])
+    tails = np.repeat(np.arange(n), np.diff(ex["up_first"].astype(np.int64)))
+    assert np.all(lev[ex["up_head"]] < lev[tails])
+    # level sizes agree with lvl_off; level 0 (lowest) is the last group
+    ls = h.level_sizes()
+    assert ls.sum() == n and ls[0] == lo[-1] - lo[-2]
+    # permutation is a bijection; within a level, original ids ascend (DFS order kept)
+    perm = h.order()
+    assert np.array_equal(np.sort(perm), np.arange(n, dtype=np.uint32))
+    inv = np.empty_like(perm)
+    inv[perm] = np.arange(n, dtype=np.uint32)
+    for j in range(L):
+        seg = inv[lo[j]:lo[j + 1]]
+        assert np.all(np.diff(seg.astype(np.int64)) > 0)
+    # level-0 vertices are never tails (their rows need not be stored in diameter mode)
+    assert np.all(lev[ex["dn_tail"]] < L - 1) if ex["dn_tail"].size else True
+
+
+def test_shortcut_lengths_dominate_distances():
+    """Every A-down / A-up arc length >= the true distance between its endpoints
+    (shortcuts represent real paths, §II-B)."""
+    g = GRAPHS["road"]()
+    h = P.Phast.from_graph(g, host_only=True)
+    ex = h.export()
+    perm = h.order()
+    inv = np.empty_like(perm)
+    inv[perm] = np.arange(h.n, dtype=np.uint32)
+    heads = np.repeat(np.arange(h.n), np.diff(ex["dn_first"].astype(np.int64)))
+    rng = np.random.default_rng(0)
+    pick = rng.choice(ex["dn_tail"].size, 40, replace=False)
+    for e in pick:
+        t, v = int(inv[ex["dn_tail"][e]]), int(inv[heads[e]])
+        assert int(ex["dn_len"][e]) >= int(oracle.sssp(g, t)[v])
+
+
+def test_deterministic_across_thread_counts():
+    g = phastgen.road(30_000, seed=21)
+    a = P.Phast.from_graph(g, host_only=True, threads=1).export()
+    b = P.Phast.from_graph(g, host_only=True, threads=7).export()
+    for k in a:
+        assert np.array_equal(a[k], b[k]), k
+
+
+def test_save_load_roundtrip(tmp_path):
+    g = phastgen.road(20_000, seed=22)
+    h = P.Phast.from_graph(g, host_only=True)
+    p = str(tmp_path / "h.phast")
+    h.save(p)
+    h2 = P.Phast.load(p, host_only=True)
+    a, b = h.export(), h2.export()
+    for k in a:
+        assert np.array_equal(a[k], b[k]), k
+    assert np.array_equal(h.order(), h2.order())
+    with pytest.raises(P.PhastError):
+        P.Phast.load(str(tmp_path / "missing"), host_only=True)
+
+
+def test_invalid_inputs_rejected():
+    g = phastgen.grid(4, 4)
+    with pytest.raises(P.PhastError) as e:
+        P.Phast(0, np.zeros(1, np.uint64), g.head, g.len, host_only=True)
+    assert e.value.status == -1
+    bad_head = g.head.copy()
+    bad_head[3] = 99
+    with pytest.raises(P.PhastError):
+        P.Phast(g.n, g.first, bad_head, g.len, host_only=True)
+    bad_first = g.first.copy()
+    bad_first[2], bad_first[3] = bad_first[3], bad_first[2]
+    with pytest.raises(P.PhastError):
+        P.Phast(g.n, bad_first, g.head, g.len, host_only=True)
+    h = P.Phast.from_graph(g, host_only=True)
+    # no device image: queries fail loudly (no CPU fallback)
+    with pytest.raises(P.PhastError) as e:
+        P._check("phast_trees", P._lib.phast_trees(h._h, np.zeros(1, np.uint32).ctypes.data, 1, 16, None))
+    assert e.value.status == -5
+
+
+def test_degenerate_graphs():
+    # single vertex, no arcs; graph with only self-loops and INF arcs
+    g1 = phastgen.Graph(1, np.array([0, 0], np.uint64), np.zeros(0, np.uint32), np.zeros(0, np.uint32))
+    h = P.Phast.from_graph(g1, host_only=True)
+    assert h.levels == 1 and h.info().m_down == 0
+    g2 = phastgen.Graph(3, np.array([0, 2, 3, 3], np.uint64), np.array([0, 1, 2], np.uint32),
+                        np.array([5, 0xFFFFFFFF, 7], np.uint32))
+    h2 = P.Phast.from_graph(g2, host_only=True)
+    ex = h2.export()
+    got = chref.phast_cpu(h2, ex, [0, 1, 2])
+    assert np.array_equal(got, oracle.sssp_many(g2, [0, 1, 2]))
