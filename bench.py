@@ -188,17 +188,10 @@ def main():
     # hierarchy: rank 0 builds (host CH, not the timed target) and shares it via a file
     path = args.cache or f"/tmp/phast_{args.config}_{os.getpid() if world == 1 else 'dist'}.phast"
     if world > 1:
-        if rank == 0:
-            t = time.time()
-            h = P.Phast.from_graph(g)
-            h.save(path)
-            log(f"[bench] CH build {time.time() - t:.1f}s")
-        barrier()
-        if rank != 0:
-            h = P.Phast.load(path)
-        barrier()
-        if rank == 0:
-            os.unlink(path)
+        from paper_conf_ipps_dellinggnw11_b200.parallel import share_hierarchy
+        t = time.time()
+        h = share_hierarchy(lambda: P.Phast.from_graph(g), P.Phast.load, path, rank, barrier)
+        log(f"[bench] rank {rank}: hierarchy ready in {time.time() - t:.1f}s")
     elif args.cache and os.path.exists(args.cache):
         h = P.Phast.load(args.cache)
     else:

@@ -13,6 +13,7 @@
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
+#include <map>
 #include <memory>
 #include <new>
 #include <vector>
@@ -40,6 +41,15 @@ struct phast_ctx {
     size_t dist_scratch_elems = 0;
     uint32_t* batch_max_scratch = nullptr;
     size_t batch_max_elems = 0;
+    // persistent-sweep plans, one per k (built on first use)
+    struct Plan {
+        SweepPlan p;
+        uint32_t epoch = 0;
+        bool ok = false;
+    };
+    std::map<uint32_t, Plan> plans;
+    std::vector<uint32_t> level_of;   // processing index of every internal id (lazy)
+    int sweep_mode = 0;               // 0 = persistent, 1 = one launch per level
     // stage timing (phast_timing)
     bool timing = false;
     std::vector<cudaEvent_t> ev;     // 3 per recorded batch
@@ -78,6 +88,12 @@ void free_device(phast_ctx* h) {
     if (h->device < 0) return;
     DeviceGuard dg(h->device);
     cudaDeviceSynchronize();
+    for (auto& kv : h->plans) {
+        cudaFree((void*)kv.second.p.chunk_v); cudaFree((void*)kv.second.p.chunk_meta);
+        cudaFree((void*)kv.second.p.chunk_start); cudaFree((void*)kv.second.p.lvl_off);
+        cudaFree(kv.second.p.level_done);
+    }
+    h->plans.clear();
     for (cudaEvent_t e : h->ev) cudaEventDestroy(e);
     h->ev.clear();
     h->ev_used = 0;
@@ -204,6 +220,56 @@ int map_sources(const phast_ctx* h, const uint32_t* src, uint32_t k, Sources& S)
     return PHAST_OK;
 }
 
+// build (once per k) the chunk table of the persistent sweep
+phast_ctx::Plan* get_plan(phast_ctx* h, uint32_t k) {
+    auto it = h->plans.find(k);
+    if (it != h->plans.end()) return it->second.ok ? &it->second : nullptr;
+    phast_ctx::Plan& P = h->plans[k];
+    if (h->levels == 0 || h->levels > 65534) return nullptr;
+    if (h->level_of.empty()) {
+        h->level_of.resize(h->n);
+        for (uint32_t j = 0; j < h->levels; j++)
+            for (uint32_t v = h->lvl_off[j]; v < h->lvl_off[j + 1]; v++) h->level_of[v] = j;
+    }
+    const uint32_t CV = sweep_chunk_vertices(k);
+    std::vector<uint32_t> cstart(h->levels + 1, 0), cv, cmeta;
+    for (uint32_t j = 0; j < h->levels; j++) {
+        cstart[j] = (uint32_t)cv.size();
+        for (uint32_t vb = h->lvl_off[j]; vb < h->lvl_off[j + 1]; vb += CV) {
+            uint32_t ve = std::min(vb + CV, h->lvl_off[j + 1]);
+            int D = -1;
+            for (uint32_t e = h->dn_first[vb]; e < h->dn_first[ve]; e++)
+                D = std::max(D, (int)h->level_of[h->dn_arc[e].x]);
+            if (D >= (int)j) return nullptr;                      // would violate Lemma 4.1
+            cv.push_back(vb);
+            cmeta.push_back((j << 16) | (uint32_t)(D + 1));
+        }
+    }
+    cstart[h->levels] = (uint32_t)cv.size();
+    int occ = std::min(sweep_blocks_per_sm(k, false), sweep_blocks_per_sm(k, true));
+    SweepPlan& p = P.p;
+    p.k = k;
+    p.nchunks = (uint32_t)cv.size();
+    p.levels = h->levels;
+    p.grid = (uint32_t)std::max(1, occ * num_sms());
+    p.chunk_vertices = CV;
+    uint32_t *a, *b, *c, *d, *e;
+    if (dmalloc(&a, cv.size()) || dmalloc(&b, cmeta.size()) || dmalloc(&c, cstart.size()) ||
+        dmalloc(&d, h->lvl_off.size()) || dmalloc(&e, h->levels))
+        return nullptr;
+    p.chunk_v = a; p.chunk_meta = b; p.chunk_start = c; p.lvl_off = d; p.level_done = e;
+    if (cudaMemcpy(a, cv.data(), cv.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess ||
+        cudaMemcpy(b, cmeta.data(), cmeta.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess ||
+        cudaMemcpy(c, cstart.data(), cstart.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess ||
+        cudaMemcpy(d, h->lvl_off.data(), h->lvl_off.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess ||
+        cudaMemset(e, 0, h->levels * 4) != cudaSuccess) {
+        cudaGetLastError();
+        return nullptr;
+    }
+    P.ok = true;
+    return &P;
+}
+
 // one full query (a1-a3) for k mapped sources; diam != nullptr -> fused max, no level-0 stores
 constexpr size_t MAX_TIMED_BATCHES = 16384;
 
@@ -228,11 +294,21 @@ int run_query(phast_ctx* h, const Sources& S, uint32_t k, uint32_t* dist, uint32
     if ((e = launch_upward(h->g, S, k, dist, st)) != cudaSuccess) return PHAST_ECUDA;
     if ((e = launch_scatter(h->g, k, dist, st)) != cudaSuccess) return PHAST_ECUDA;
     if (e1) cudaEventRecord(e1, st);
-    for (uint32_t j = 0; j < h->levels; j++) {
-        bool last = (j + 1 == h->levels);
-        bool store = !(diam && last);   // level-0 rows are never read again (diameter mode)
-        e = launch_sweep_level(h->g, k, h->lvl_off[j], h->lvl_off[j + 1], dist, diam, store, last, st);
-        if (e != cudaSuccess) return PHAST_ECUDA;
+    phast_ctx::Plan* plan = h->sweep_mode == 0 ? get_plan(h, k) : nullptr;
+    if (plan) {                          // a3+a4: one persistent launch, dataflow over levels
+        if ((uint64_t)(plan->epoch + 1) * plan->p.grid >= 0x7FFFFFFFull) {
+            if (cudaMemsetAsync(plan->p.level_done, 0, plan->p.levels * 4, st) != cudaSuccess) return PHAST_ECUDA;
+            plan->epoch = 0;
+        }
+        plan->epoch++;
+        if (launch_sweep_persistent(h->g, plan->p, plan->epoch, dist, diam, st) != cudaSuccess) return PHAST_ECUDA;
+    } else {                             // one launch per level (§VI)
+        for (uint32_t j = 0; j < h->levels; j++) {
+            bool last = (j + 1 == h->levels);
+            bool store = !(diam && last);   // level-0 rows are never read again (diameter mode)
+            e = launch_sweep_level(h->g, k, h->lvl_off[j], h->lvl_off[j + 1], dist, diam, store, last, st);
+            if (e != cudaSuccess) return PHAST_ECUDA;
+        }
     }
     if ((e = launch_clear_flags(h->g, k, st)) != cudaSuccess) return PHAST_ECUDA;
     if (e2) cudaEventRecord(e2, st);

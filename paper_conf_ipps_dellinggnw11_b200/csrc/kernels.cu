@@ -298,6 +298,132 @@ cudaError_t sweep_k(const DevImage& g, uint32_t vbeg, uint32_t vend, uint32_t* d
                 : sweep_launch<K, false, true, false>(g, vbeg, vend, dist, diam, st);
 }
 
+// ------------------------------------------------------------------ a3+a4 persistent
+constexpr uint32_t CHUNK_PASSES = 8;   // passes of the CTA over G-lane vertex groups per chunk
+
+__device__ __forceinline__ uint32_t ld_acquire_gpu(const uint32_t* p) {
+    uint32_t v;
+    asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+// label loads bypass L1: a row read earlier on this SM (e.g. a seeded row) may since
+// have been rewritten by another SM within the same launch
+__device__ __forceinline__ uint32_t ldl(const uint32_t* p) { return __ldcg(p); }
+__device__ __forceinline__ uint2 ldl(const uint2* p) { return __ldcg(p); }
+__device__ __forceinline__ uint4 ldl(const uint4* p) { return __ldcg(p); }
+
+template <int K, bool DIAM>
+__global__ void __launch_bounds__(SWEEP_THREADS) sweep_persistent_kernel(const uint32_t* __restrict__ first,
+                                                                          const uint2* __restrict__ arcs,
+                                                                          uint32_t* __restrict__ d,
+                                                                          const uint32_t* __restrict__ flags,
+                                                                          SweepPlan p, uint32_t epoch,
+                                                                          uint32_t* __restrict__ diam) {
+    using T = typename RowT<K>::T;
+    constexpr uint32_t W = RowT<K>::W;
+    constexpr uint32_t G = K / W;                   // lanes per vertex
+    constexpr uint32_t VPP = SWEEP_THREADS / G;     // vertices per pass
+    __shared__ uint32_t s_known;                    // leading levels known complete
+    if (threadIdx.x == 0) s_known = 0;
+    const uint32_t grid = gridDim.x;
+    const uint32_t last = p.levels - 1;
+    const uint32_t lane = threadIdx.x % G;
+    uint32_t mx = 0;
+    for (uint32_t c = blockIdx.x; c < p.nchunks; c += grid) {
+        const uint32_t meta = __ldg(&p.chunk_meta[c]);
+        const uint32_t J = meta >> 16;
+        const int D = (int)(meta & 0xFFFFu) - 1;
+        if (threadIdx.x == 0) {
+            uint32_t known = s_known;
+            while ((int)known <= D) {
+                const uint32_t need = epoch * min(__ldg(&p.chunk_start[known + 1]) - __ldg(&p.chunk_start[known]), grid);
+                uint32_t ns = 32;
+                while (ld_acquire_gpu(&p.level_done[known]) < need) {
+                    __nanosleep(ns);
+                    ns = min(ns * 2, 256u);
+                }
+                known++;
+            }
+            s_known = known;
+            __threadfence();
+        }
+        __syncthreads();
+        const uint32_t vbeg = __ldg(&p.chunk_v[c]);
+        const uint32_t vend = min(vbeg + p.chunk_vertices, __ldg(&p.lvl_off[J + 1]));
+        const bool store = !DIAM || J != last;     // diameter mode: level-0 rows are never read again
+        const bool stream_store = (J == last);     // level-0 rows are never re-read in this sweep
+        for (uint32_t base = vbeg; base < vend; base += VPP) {
+            const uint32_t v = base + threadIdx.x / G;
+            if (v >= vend) break;
+            T acc = inf_row<T>();
+            if ((__ldg(&flags[v >> 5]) >> (v & 31)) & 1u)
+                acc = ldl(reinterpret_cast<const T*>(d + (size_t)v * K) + lane);
+            uint32_t e = __ldg(&first[v]);
+            const uint32_t e1 = __ldg(&first[v + 1]);
+            while (e < e1) {                         // up to 4 gathers in flight per lane
+                const uint32_t cnt = min(e1 - e, 4u);
+                uint2 a[4];
+                T x[4];
+#pragma unroll
+                for (uint32_t j = 0; j < 4; j++)
+                    if (j < cnt) a[j] = __ldg(&arcs[e + j]);
+#pragma unroll
+                for (uint32_t j = 0; j < 4; j++)
+                    if (j < cnt) x[j] = ldl(reinterpret_cast<const T*>(d + (size_t)a[j].x * K) + lane);
+#pragma unroll
+                for (uint32_t j = 0; j < 4; j++)
+                    if (j < cnt) acc = relax(acc, x[j], a[j].y);
+                e += cnt;
+            }
+            if (store) {
+                T* q = reinterpret_cast<T*>(d + (size_t)v * K) + lane;
+                if (stream_store) st_stream(q, acc); else *q = acc;
+            }
+            if constexpr (DIAM) mx = max(mx, fmax_of(acc));
+        }
+        __syncthreads();                             // every row of this chunk is written
+        if (threadIdx.x == 0 && c + grid >= __ldg(&p.chunk_start[J + 1])) {
+            __threadfence();                         // release: rows before the counter
+            atomicAdd(&p.level_done[J], 1u);         // this CTA's last chunk of level J
+        }
+    }
+    if constexpr (DIAM) {
+        __shared__ uint32_t wmax[SWEEP_THREADS / 32];
+        mx = __reduce_max_sync(0xFFFFFFFFu, mx);
+        if ((threadIdx.x & 31) == 0) wmax[threadIdx.x >> 5] = mx;
+        __syncthreads();
+        if (threadIdx.x < 32) {
+            uint32_t w = threadIdx.x < SWEEP_THREADS / 32 ? wmax[threadIdx.x] : 0u;
+            w = __reduce_max_sync(0xFFFFFFFFu, w);
+            if (threadIdx.x == 0 && w) atomicMax(diam, w);
+        }
+    }
+}
+
+template <int K, bool DIAM>
+int persistent_occupancy() {
+    int b = 0;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, sweep_persistent_kernel<K, DIAM>, SWEEP_THREADS, 0) !=
+        cudaSuccess) {
+        cudaGetLastError();
+        return 1;
+    }
+    return b > 0 ? b : 1;
+}
+
+template <int K>
+cudaError_t persistent_k(const DevImage& g, const SweepPlan& p, uint32_t epoch, uint32_t* dist, uint32_t* diam,
+                         cudaStream_t st) {
+    if (diam)
+        sweep_persistent_kernel<K, true><<<p.grid, SWEEP_THREADS, 0, st>>>(g.dn_first, g.dn_arc, dist, g.flags, p,
+                                                                           epoch, diam);
+    else
+        sweep_persistent_kernel<K, false><<<p.grid, SWEEP_THREADS, 0, st>>>(g.dn_first, g.dn_arc, dist, g.flags, p,
+                                                                            epoch, nullptr);
+    g_launches++;
+    return cudaGetLastError();
+}
+
 template <int K>
 cudaError_t upward_k(const DevImage& g, const Sources& src, uint32_t k, uint32_t* dist, cudaStream_t st) {
     static bool attr = false;
@@ -358,6 +484,33 @@ cudaError_t launch_sweep_level(const DevImage& g, uint32_t k, uint32_t vbeg, uin
 #define CALL_SW(K) sweep_k<K>(g, vbeg, vend, dist, diam, store, last_level, st)
     PHAST_K_SWITCH(k, CALL_SW)
 #undef CALL_SW
+}
+
+uint32_t sweep_chunk_vertices(uint32_t k) {
+    uint32_t G = k >= 4 ? k / 4 : 1;
+    return (SWEEP_THREADS / G) * CHUNK_PASSES;
+}
+
+int sweep_blocks_per_sm(uint32_t k, bool diam) {
+#define OCC(K) (diam ? persistent_occupancy<K, true>() : persistent_occupancy<K, false>())
+    switch (k) {
+        case 1: return OCC(1);
+        case 2: return OCC(2);
+        case 4: return OCC(4);
+        case 8: return OCC(8);
+        case 16: return OCC(16);
+        case 32: return OCC(32);
+        case 64: return OCC(64);
+        default: return 1;
+    }
+#undef OCC
+}
+
+cudaError_t launch_sweep_persistent(const DevImage& g, const SweepPlan& p, uint32_t epoch, uint32_t* dist,
+                                    uint32_t* diam, cudaStream_t st) {
+#define CALL_PS(K) persistent_k<K>(g, p, epoch, dist, diam, st)
+    PHAST_K_SWITCH(p.k, CALL_PS)
+#undef CALL_PS
 }
 
 cudaError_t launch_clear_flags(const DevImage& g, uint32_t k, cudaStream_t st) {

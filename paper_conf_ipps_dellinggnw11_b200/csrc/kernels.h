@@ -40,6 +40,27 @@ cudaError_t launch_scatter(const DevImage& g, uint32_t k, uint32_t* dist, cudaSt
 cudaError_t launch_sweep_level(const DevImage& g, uint32_t k, uint32_t vbeg, uint32_t vend,
                                uint32_t* dist, uint32_t* diam, bool store, bool last_level,
                                cudaStream_t st);
+// Plan of the persistent (single-launch) sweep for one k: the vertex range of every
+// level is cut into chunks that never straddle a level; each chunk records its
+// level (processing index J, 0 = top) and D = the latest processing index among the
+// levels of its in-arc tails (-1 if none).  A CTA may start chunk c once levels
+// 0..D are complete (Lemma 4.1 guarantees D < J).
+struct SweepPlan {
+    uint32_t k = 0, nchunks = 0, levels = 0, grid = 0, chunk_vertices = 0;
+    const uint32_t* chunk_v = nullptr;      // [nchunks] first vertex of each chunk
+    const uint32_t* chunk_meta = nullptr;   // [nchunks] J << 16 | (D + 1)
+    const uint32_t* chunk_start = nullptr;  // [levels+1] first chunk of each level
+    const uint32_t* lvl_off = nullptr;      // [levels+1]
+    uint32_t* level_done = nullptr;         // [levels] monotone completion counters
+};
+// vertices per chunk and CTAs per SM the persistent sweep uses for this k
+uint32_t sweep_chunk_vertices(uint32_t k);
+int sweep_blocks_per_sm(uint32_t k, bool diam);
+// a3 + a4 in ONE launch: dataflow over levels through the completion counters
+// (epoch = number of launches of this plan so far, 1-based).
+cudaError_t launch_sweep_persistent(const DevImage& g, const SweepPlan& p, uint32_t epoch, uint32_t* dist,
+                                    uint32_t* diam, cudaStream_t st);
+
 // after the sweep: clear the visited bits of every search-space vertex ("After
 // scanning v we unmark the vertex", §IV-C).
 cudaError_t launch_clear_flags(const DevImage& g, uint32_t k, cudaStream_t st);

@@ -121,6 +121,20 @@ def test_upward_global_fallback_and_overflow(monkeypatch):
         h.sync()                                       # error word is cleared
 
 
+@pytest.mark.parametrize("mode", ["levels", "persistent"])
+def test_sweep_modes(monkeypatch, mode):
+    """Both level schedules (one launch per level, §VI; and the single
+    persistent launch with per-level completion counters) are bit-exact."""
+    monkeypatch.setenv("PHAST_SWEEP", mode)
+    g = phastgen.road(120_000, seed=33)
+    with P.Phast.from_graph(g) as h:
+        for k in (1, 2, 16, 64):
+            src = phastgen.sources(g.n, k, seed=900 + k)
+            assert np.array_equal(gpu_trees(h, src), oracle.sssp_many(g, src)), k
+        src = phastgen.sources(g.n, 200, seed=901)
+        assert h.diameter(src, k_batch=64) == oracle.diameter(g, src)
+
+
 def test_tiny_and_degenerate():
     for g in (phastgen.Graph(1, np.array([0, 0], np.uint64), np.zeros(0, np.uint32), np.zeros(0, np.uint32)),
               phastgen.grid(1, 2), phastgen.grid(3, 1, 0, 1)):
