@@ -23,6 +23,7 @@ INF = 0xFFFFFFFF
 KMAX = 64
 K_ALLOWED = (1, 2, 4, 8, 16, 32, 64)
 FLAG_HOST_ONLY = 1
+FLAG_LEVEL_LAYOUT = 2
 
 STATUS = {0: "OK", -1: "EINVAL", -2: "ENOMEM", -3: "ECUDA", -4: "ERANGE", -5: "ESTATE", -6: "EIO",
           -7: "EINTERNAL"}
@@ -37,14 +38,14 @@ class PhastError(RuntimeError):
 class _Opts(ctypes.Structure):
     _fields_ = [("hop_limit_lo", ctypes.c_uint32), ("hop_limit_hi", ctypes.c_uint32),
                 ("settled_cap", ctypes.c_uint32), ("threads", ctypes.c_uint32),
-                ("flags", ctypes.c_uint32), ("reserved", ctypes.c_uint32), ("seed", ctypes.c_uint64)]
+                ("flags", ctypes.c_uint32), ("delta", ctypes.c_uint32), ("seed", ctypes.c_uint64)]
 
 
 class _Info(ctypes.Structure):
     _fields_ = [("n", ctypes.c_uint32), ("levels", ctypes.c_uint32), ("m", ctypes.c_uint64),
                 ("m_up", ctypes.c_uint64), ("m_down", ctypes.c_uint64), ("n_tail", ctypes.c_uint64),
                 ("shortcuts", ctypes.c_uint64), ("rounds", ctypes.c_uint32), ("device", ctypes.c_uint32),
-                ("build_seconds", ctypes.c_double)]
+                ("layout", ctypes.c_uint32), ("delta", ctypes.c_uint32), ("build_seconds", ctypes.c_double)]
 
 
 def _load_lib():
@@ -114,6 +115,8 @@ class Info:
     shortcuts: int
     rounds: int
     device: int
+    layout: int
+    delta: int
     build_seconds: float
 
 
@@ -121,7 +124,7 @@ class Phast:
     """A built hierarchy bound to one CUDA device (phast_ctx)."""
 
     def __init__(self, n=None, first=None, head=None, length=None, *, host_only=False, threads=0,
-                 hop_limit_lo=0, hop_limit_hi=0, settled_cap=0, _handle=None):
+                 hop_limit_lo=0, hop_limit_hi=0, settled_cap=0, level_layout=False, delta=0, _handle=None):
         self._h = None
         if _handle is not None:
             self._h = _handle
@@ -132,7 +135,8 @@ class Phast:
             if head.size == 0:
                 head = np.zeros(1, np.uint32)
                 length = np.zeros(1, np.uint32)
-            o = _Opts(hop_limit_lo, hop_limit_hi, settled_cap, threads, FLAG_HOST_ONLY if host_only else 0, 0, 0)
+            flags = (FLAG_HOST_ONLY if host_only else 0) | (FLAG_LEVEL_LAYOUT if level_layout else 0)
+            o = _Opts(hop_limit_lo, hop_limit_hi, settled_cap, threads, flags, delta, 0)
             h = ctypes.c_void_p()
             _check("phast_build", _lib.phast_build(int(n), first.ctypes.data, head.ctypes.data,
                                                    length.ctypes.data, ctypes.byref(o), ctypes.byref(h)))
@@ -232,7 +236,7 @@ class Phast:
         i = _Info()
         _check("phast_info", _lib.phast_info(self._h, ctypes.byref(i)))
         return Info(i.n, i.levels, i.m, i.m_up, i.m_down, i.n_tail, i.shortcuts, i.rounds,
-                    -1 if i.device == 0xFFFFFFFF else i.device, i.build_seconds)
+                    -1 if i.device == 0xFFFFFFFF else i.device, i.layout, i.delta, i.build_seconds)
 
     def level_sizes(self) -> np.ndarray:
         out = np.empty(self.levels, np.uint32)
@@ -249,12 +253,12 @@ class Phast:
 
     def export(self) -> dict:
         inf = self.info()
-        a = dict(lvl_off=np.empty(inf.levels + 1, np.uint32), dn_first=np.empty(inf.n + 1, np.uint32),
+        a = dict(level=np.empty(inf.n, np.uint32), dn_first=np.empty(inf.n + 1, np.uint32),
                  dn_tail=np.empty(max(inf.m_down, 1), np.uint32), dn_len=np.empty(max(inf.m_down, 1), np.uint32),
                  up_first=np.empty(inf.n + 1, np.uint32), up_head=np.empty(max(inf.m_up, 1), np.uint32),
                  up_len=np.empty(max(inf.m_up, 1), np.uint32))
         _check("phast_export", _lib.phast_export(self._h, *[a[k].ctypes.data for k in
-                                                           ("lvl_off", "dn_first", "dn_tail", "dn_len", "up_first",
+                                                           ("level", "dn_first", "dn_tail", "dn_len", "up_first",
                                                             "up_head", "up_len")]))
         a["dn_tail"] = a["dn_tail"][:inf.m_down]
         a["dn_len"] = a["dn_len"][:inf.m_down]

@@ -1,14 +1,10 @@
-// capi.cu -- the C ABI of include/phast.h: handle lifetime, validation, layout
-// (renumbering by level), device image upload, and query orchestration.
+// capi.cu -- the C ABI of include/phast.h: handle lifetime, validation, device
+// image upload, sweep plans and query orchestration.
 //
-// Layout:
-//   internal ids sorted by (level descending, original id ascending): "We assign
-//   lower IDs to vertices at higher levels; within each level, we keep the DFS
-//   order" (§IV-A; the generator's ids are the DFS order).  Then the
-//   sweep is "a simple linear sweep in increasing order of IDs", and every level is
-//   one contiguous id range [lvl_off[j], lvl_off[j+1]).
-//   G-down: in-arcs by head, {tail, len} (§IV-A), sentinel dn_first[n].
-//   G-up:   out-arcs by tail, {head, len}.
+// Layout (layout.cpp): internal ids follow a reverse topological order
+// of G-down, so that the sweep is "a simple linear sweep in increasing order of IDs"
+// (§IV-A).  G-down: in-arcs by head, {tail, len} (§IV-A),
+// sentinel dn_first[n].  G-up: out-arcs by tail, {head, len}.
 #include <algorithm>
 #include <cstdio>
 #include <cstdlib>
@@ -21,23 +17,21 @@
 #include "../../include/phast.h"
 #include "ch.h"
 #include "kernels.h"
+#include "layout.h"
 
 using namespace phast;
 
 struct phast_ctx {
-    uint32_t n = 0, levels = 0;
+    uint32_t n = 0;
     uint64_t m = 0, shortcuts = 0;
     uint32_t rounds = 0;
     double build_seconds = 0;
-    std::vector<uint32_t> perm;      // internal_of_original
-    std::vector<uint32_t> iperm;     // original_of_internal
-    std::vector<uint32_t> lvl_off;   // [levels+1], j = 0 is the top level
-    std::vector<uint32_t> dn_first, up_first;
-    std::vector<uint2> dn_arc, up_arc;
+    Layout L;
+    std::vector<uint32_t> tail_bits;   // bit v: internal id v is the tail of some G-down arc
     // device
     int device = -1;
     DevImage g;
-    uint32_t* dist_scratch = nullptr;   // diameter mode label buffer
+    uint32_t* dist_scratch = nullptr;   // phast_trees_host / phast_diameter label buffer
     size_t dist_scratch_elems = 0;
     uint32_t* batch_max_scratch = nullptr;
     size_t batch_max_elems = 0;
@@ -48,17 +42,17 @@ struct phast_ctx {
         bool ok = false;
     };
     std::map<uint32_t, Plan> plans;
-    std::vector<uint32_t> level_of;   // processing index of every internal id (lazy)
-    int sweep_mode = 0;               // 0 = persistent, 1 = one launch per level
+    int sweep_mode = 0;   // 0 = persistent + bulk-staged arcs, 1 = one launch per level, 2 = persistent, no staging
     // stage timing (phast_timing)
     bool timing = false;
-    std::vector<cudaEvent_t> ev;     // 3 per recorded batch
+    std::vector<cudaEvent_t> ev;   // 3 per recorded batch
     size_t ev_used = 0;
 };
 
 namespace {
 
 constexpr uint32_t SEED_CAP = 1u << 16;   // per-source search-space capacity (global fallback)
+constexpr uint32_t DEFAULT_DELTA = 65536;
 
 bool k_ok(uint32_t k) { return k == 1 || k == 2 || k == 4 || k == 8 || k == 16 || k == 32 || k == 64; }
 
@@ -80,31 +74,46 @@ int dmalloc(T** p, size_t elems) {
     *p = nullptr;
     if (elems == 0) elems = 1;
     cudaError_t e = cudaMalloc((void**)p, elems * sizeof(T));
-    if (e != cudaSuccess) { cudaGetLastError(); *p = nullptr; return e == cudaErrorMemoryAllocation ? PHAST_ENOMEM : PHAST_ECUDA; }
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        *p = nullptr;
+        return e == cudaErrorMemoryAllocation ? PHAST_ENOMEM : PHAST_ECUDA;
+    }
     return PHAST_OK;
+}
+
+void free_plans(phast_ctx* h) {
+    for (auto& kv : h->plans) {
+        cudaFree((void*)kv.second.p.chunk_v);
+        cudaFree((void*)kv.second.p.chunk_dep);
+        cudaFree(kv.second.p.wave_done);
+    }
+    h->plans.clear();
 }
 
 void free_device(phast_ctx* h) {
     if (h->device < 0) return;
     DeviceGuard dg(h->device);
     cudaDeviceSynchronize();
-    for (auto& kv : h->plans) {
-        cudaFree((void*)kv.second.p.chunk_v); cudaFree((void*)kv.second.p.chunk_meta);
-        cudaFree((void*)kv.second.p.chunk_start); cudaFree((void*)kv.second.p.lvl_off);
-        cudaFree(kv.second.p.level_done);
-    }
-    h->plans.clear();
+    free_plans(h);
     for (cudaEvent_t e : h->ev) cudaEventDestroy(e);
     h->ev.clear();
     h->ev_used = 0;
     cudaFree((void*)h->g.dn_first); cudaFree((void*)h->g.dn_arc);
     cudaFree((void*)h->g.up_first); cudaFree((void*)h->g.up_arc);
-    cudaFree(h->g.flags); cudaFree(h->g.seed_v); cudaFree(h->g.seed_d); cudaFree(h->g.seed_cnt);
+    cudaFree(h->g.flags); cudaFree((void*)h->g.tail_bits);
+    cudaFree(h->g.seed_v); cudaFree(h->g.seed_d); cudaFree(h->g.seed_cnt);
     cudaFree(h->g.gscratch); cudaFree(h->g.err);
     cudaFree(h->dist_scratch); cudaFree(h->batch_max_scratch);
     h->g = DevImage();
     h->dist_scratch = nullptr; h->batch_max_scratch = nullptr;
+    h->dist_scratch_elems = 0; h->batch_max_elems = 0;
     h->device = -1;
+}
+
+void compute_tail_bits(phast_ctx* h) {
+    h->tail_bits.assign(((size_t)h->n + 31) / 32, 0u);
+    for (const Arc& a : h->L.dn_arc) h->tail_bits[a.x >> 5] |= 1u << (a.x & 31);
 }
 
 int upload(phast_ctx* h) {
@@ -113,90 +122,47 @@ int upload(phast_ctx* h) {
     h->device = dev;
     DevImage& g = h->g;
     g.n = h->n;
-    // test knobs (power of two): shrink the shared-memory table / per-source capacity to
-    // exercise the global-memory fallback and the overflow error path
+    if (const char* e = std::getenv("PHAST_SWEEP"))
+        h->sweep_mode = std::strcmp(e, "levels") == 0 ? 1 : std::strcmp(e, "persistent") == 0 ? 2 : 0;
+    if (h->sweep_mode == 1 && h->L.mode != LAYOUT_LEVELS) h->sweep_mode = 0;   // needs contiguous levels
+    // test knobs (rounded down to powers of two): shrink the shared-memory table / the
+    // per-source capacity to exercise the global fallback and the overflow error path
     uint32_t seed_cap = SEED_CAP, smem_cap = 4096;
-    if (const char* e = std::getenv("PHAST_SEED_CAP")) seed_cap = std::max(16u, std::min<uint32_t>(SEED_CAP, (uint32_t)std::atoi(e)));
-    if (const char* e = std::getenv("PHAST_UP_SMEM_CAP")) smem_cap = std::max(16u, std::min<uint32_t>(4096u, (uint32_t)std::atoi(e)));
+    if (const char* e = std::getenv("PHAST_SEED_CAP"))
+        seed_cap = std::max(16u, std::min<uint32_t>(SEED_CAP, (uint32_t)std::atoi(e)));
+    if (const char* e = std::getenv("PHAST_UP_SMEM_CAP"))
+        smem_cap = std::max(16u, std::min<uint32_t>(4096u, (uint32_t)std::atoi(e)));
     auto pow2 = [](uint32_t x) { uint32_t p = 1; while (p * 2 <= x) p *= 2; return p; };
     g.seed_cap = pow2(seed_cap);
     g.smem_cap = pow2(smem_cap);
-    uint32_t *dnf, *upf;
-    uint2 *dna, *upa;
+    const Layout& L = h->L;
+    uint32_t *dnf = nullptr, *upf = nullptr, *tb = nullptr;
+    uint2 *dna = nullptr, *upa = nullptr;
     int rc;
     size_t nw = ((size_t)h->n + 31) / 32;
-    if ((rc = dmalloc(&dnf, h->dn_first.size())) || (rc = dmalloc(&dna, h->dn_arc.size())) ||
-        (rc = dmalloc(&upf, h->up_first.size())) || (rc = dmalloc(&upa, h->up_arc.size())) ||
-        (rc = dmalloc(&g.flags, nw)) || (rc = dmalloc(&g.seed_v, (size_t)KMAX * g.seed_cap)) ||
-        (rc = dmalloc(&g.seed_d, (size_t)KMAX * g.seed_cap)) || (rc = dmalloc(&g.seed_cnt, KMAX)) ||
-        (rc = dmalloc(&g.gscratch, (size_t)KMAX * g.seed_cap * 5)) || (rc = dmalloc(&g.err, 1))) {
-        g.dn_first = dnf; g.dn_arc = dna; g.up_first = upf; g.up_arc = upa;
+    // +4 / +2 elements: 16-byte aligned bulk copies may read up to 12 bytes past the end
+    if ((rc = dmalloc(&dnf, L.dn_first.size() + 4)) || (rc = dmalloc(&dna, L.dn_arc.size() + 2)) ||
+        (rc = dmalloc(&upf, L.up_first.size())) || (rc = dmalloc(&upa, L.up_arc.size())) ||
+        (rc = dmalloc(&g.flags, nw)) || (rc = dmalloc(&tb, nw)) ||
+        (rc = dmalloc(&g.seed_v, (size_t)KMAX * g.seed_cap)) || (rc = dmalloc(&g.seed_d, (size_t)KMAX * g.seed_cap)) ||
+        (rc = dmalloc(&g.seed_cnt, KMAX)) || (rc = dmalloc(&g.gscratch, (size_t)KMAX * g.seed_cap * 5)) ||
+        (rc = dmalloc(&g.err, 1))) {
+        g.dn_first = dnf; g.dn_arc = dna; g.up_first = upf; g.up_arc = upa; g.tail_bits = tb;
         free_device(h);
         return rc;
     }
-    g.dn_first = dnf; g.dn_arc = dna; g.up_first = upf; g.up_arc = upa;
-    bool ok = cudaMemcpy(dnf, h->dn_first.data(), h->dn_first.size() * 4, cudaMemcpyHostToDevice) == cudaSuccess &&
-              cudaMemcpy(dna, h->dn_arc.data(), h->dn_arc.size() * 8, cudaMemcpyHostToDevice) == cudaSuccess &&
-              cudaMemcpy(upf, h->up_first.data(), h->up_first.size() * 4, cudaMemcpyHostToDevice) == cudaSuccess &&
-              cudaMemcpy(upa, h->up_arc.data(), h->up_arc.size() * 8, cudaMemcpyHostToDevice) == cudaSuccess &&
+    g.dn_first = dnf; g.dn_arc = dna; g.up_first = upf; g.up_arc = upa; g.tail_bits = tb;
+    bool ok = cudaMemset(dnf, 0, (L.dn_first.size() + 4) * 4) == cudaSuccess &&
+              cudaMemset(dna, 0, (L.dn_arc.size() + 2) * 8) == cudaSuccess &&
+              cudaMemcpy(dnf, L.dn_first.data(), L.dn_first.size() * 4, cudaMemcpyHostToDevice) == cudaSuccess &&
+              cudaMemcpy(dna, L.dn_arc.data(), L.dn_arc.size() * 8, cudaMemcpyHostToDevice) == cudaSuccess &&
+              cudaMemcpy(upf, L.up_first.data(), L.up_first.size() * 4, cudaMemcpyHostToDevice) == cudaSuccess &&
+              cudaMemcpy(upa, L.up_arc.data(), L.up_arc.size() * 8, cudaMemcpyHostToDevice) == cudaSuccess &&
+              cudaMemcpy(tb, h->tail_bits.data(), nw * 4, cudaMemcpyHostToDevice) == cudaSuccess &&
               cudaMemset(g.flags, 0, nw * 4) == cudaSuccess && cudaMemset(g.err, 0, 4) == cudaSuccess &&
               cudaMemset(g.seed_cnt, 0, KMAX * 4) == cudaSuccess && cudaDeviceSynchronize() == cudaSuccess;
     if (!ok) { cudaGetLastError(); free_device(h); return PHAST_ECUDA; }
     return PHAST_OK;
-}
-
-// renumber by (level desc, id asc) and build the two CSRs in internal ids
-int layout(phast_ctx* h, const ChResult& R) {
-    const uint32_t n = R.n;
-    uint32_t L = 0;
-    for (uint32_t v = 0; v < n; v++) L = std::max(L, R.level[v] + 1);
-    h->levels = L;
-    std::vector<uint32_t> cnt(L, 0);
-    for (uint32_t v = 0; v < n; v++) cnt[R.level[v]]++;
-    h->lvl_off.assign(L + 1, 0);
-    for (uint32_t j = 0; j < L; j++) h->lvl_off[j + 1] = h->lvl_off[j] + cnt[L - 1 - j];
-    std::vector<uint32_t> pos(L);
-    for (uint32_t j = 0; j < L; j++) pos[L - 1 - j] = h->lvl_off[j];
-    h->perm.resize(n);
-    h->iperm.resize(n);
-    for (uint32_t v = 0; v < n; v++) {   // ascending original id within each level
-        uint32_t r = pos[R.level[v]]++;
-        h->perm[v] = r;
-        h->iperm[r] = v;
-    }
-    uint64_t mdn = R.dn_first[n], mup = R.up_first[n];
-    if (mdn >= 0xFFFFFFFFull || mup >= 0xFFFFFFFFull) return PHAST_ERANGE;
-    h->dn_first.assign((size_t)n + 1, 0);
-    h->up_first.assign((size_t)n + 1, 0);
-    h->dn_arc.resize(mdn);
-    h->up_arc.resize(mup);
-    for (uint32_t r = 0; r < n; r++) {
-        uint32_t v = h->iperm[r];
-        h->dn_first[r + 1] = h->dn_first[r] + (uint32_t)(R.dn_first[v + 1] - R.dn_first[v]);
-        h->up_first[r + 1] = h->up_first[r] + (uint32_t)(R.up_first[v + 1] - R.up_first[v]);
-    }
-    bool lemma_ok = true;
-    for (uint32_t r = 0; r < n; r++) {
-        uint32_t v = h->iperm[r];
-        uint32_t p = h->dn_first[r];
-        for (uint64_t e = R.dn_first[v]; e < R.dn_first[v + 1]; e++) {
-            uint32_t t = R.dn_tail[e];
-            // Lemma 4.1: (t, v) in A-down => L(t) > L(v)  (§IV-A)
-            if (!(R.level[t] > R.level[v])) lemma_ok = false;
-            h->dn_arc[p++] = make_uint2(h->perm[t], R.dn_len[e]);
-        }
-        std::sort(h->dn_arc.begin() + h->dn_first[r], h->dn_arc.begin() + h->dn_first[r + 1],
-                  [](const uint2& a, const uint2& b) { return a.x < b.x || (a.x == b.x && a.y < b.y); });
-        p = h->up_first[r];
-        for (uint64_t e = R.up_first[v]; e < R.up_first[v + 1]; e++) {
-            uint32_t w = R.up_head[e];
-            if (!(R.level[w] > R.level[v])) lemma_ok = false;    // same rule for A-up
-            h->up_arc[p++] = make_uint2(h->perm[w], R.up_len[e]);
-        }
-        std::sort(h->up_arc.begin() + h->up_first[r], h->up_arc.begin() + h->up_first[r + 1],
-                  [](const uint2& a, const uint2& b) { return a.x < b.x || (a.x == b.x && a.y < b.y); });
-    }
-    return lemma_ok ? PHAST_OK : PHAST_EINTERNAL;
 }
 
 int validate_csr(uint32_t n, const uint64_t* first, const uint32_t* head, const uint32_t* len) {
@@ -214,55 +180,59 @@ int validate_csr(uint32_t n, const uint64_t* first, const uint32_t* head, const 
 int map_sources(const phast_ctx* h, const uint32_t* src, uint32_t k, Sources& S) {
     for (uint32_t i = 0; i < k; i++) {
         if (src[i] >= h->n) return PHAST_ERANGE;
-        S.s[i] = h->perm[src[i]];
+        S.s[i] = h->L.perm[src[i]];
     }
     for (uint32_t i = k; i < KMAX; i++) S.s[i] = 0;
     return PHAST_OK;
 }
 
-// build (once per k) the chunk table of the persistent sweep
+// Plan of the persistent sweep for one k.  Chunks are contiguous internal-id ranges
+// of at most CV vertices, cut wherever a vertex has a G-down tail inside the open
+// chunk (so a chunk never waits on itself).  Chunk c is processed by CTA c % grid in
+// iteration c / grid; it depends on the iteration of the latest chunk holding one
+// of its tails, and may start once every CTA has finished that iteration.
 phast_ctx::Plan* get_plan(phast_ctx* h, uint32_t k) {
     auto it = h->plans.find(k);
     if (it != h->plans.end()) return it->second.ok ? &it->second : nullptr;
     phast_ctx::Plan& P = h->plans[k];
-    if (h->levels == 0 || h->levels > 65534) return nullptr;
-    if (h->level_of.empty()) {
-        h->level_of.resize(h->n);
-        for (uint32_t j = 0; j < h->levels; j++)
-            for (uint32_t v = h->lvl_off[j]; v < h->lvl_off[j + 1]; v++) h->level_of[v] = j;
-    }
+    const Layout& L = h->L;
+    const uint32_t n = h->n;
     const uint32_t CV = sweep_chunk_vertices(k);
-    std::vector<uint32_t> cstart(h->levels + 1, 0), cv, cmeta;
-    for (uint32_t j = 0; j < h->levels; j++) {
-        cstart[j] = (uint32_t)cv.size();
-        for (uint32_t vb = h->lvl_off[j]; vb < h->lvl_off[j + 1]; vb += CV) {
-            uint32_t ve = std::min(vb + CV, h->lvl_off[j + 1]);
-            int D = -1;
-            for (uint32_t e = h->dn_first[vb]; e < h->dn_first[ve]; e++)
-                D = std::max(D, (int)h->level_of[h->dn_arc[e].x]);
-            if (D >= (int)j) return nullptr;                      // would violate Lemma 4.1
-            cv.push_back(vb);
-            cmeta.push_back((j << 16) | (uint32_t)(D + 1));
-        }
-    }
-    cstart[h->levels] = (uint32_t)cv.size();
-    int occ = std::min(sweep_blocks_per_sm(k, false), sweep_blocks_per_sm(k, true));
     SweepPlan& p = P.p;
     p.k = k;
-    p.nchunks = (uint32_t)cv.size();
-    p.levels = h->levels;
+    p.variant = h->sweep_mode == 2 ? 0u : 1u;
+    p.chunk_cap = CV;
+    int occ = std::min(sweep_blocks_per_sm(k, false, p.variant), sweep_blocks_per_sm(k, true, p.variant));
     p.grid = (uint32_t)std::max(1, occ * num_sms());
-    p.chunk_vertices = CV;
-    uint32_t *a, *b, *c, *d, *e;
-    if (dmalloc(&a, cv.size()) || dmalloc(&b, cmeta.size()) || dmalloc(&c, cstart.size()) ||
-        dmalloc(&d, h->lvl_off.size()) || dmalloc(&e, h->levels))
-        return nullptr;
-    p.chunk_v = a; p.chunk_meta = b; p.chunk_start = c; p.lvl_off = d; p.level_done = e;
+    std::vector<uint32_t> cv, chunk_of(n);
+    uint32_t s = 0;
+    cv.push_back(0);
+    for (uint32_t v = 0; v < n; v++) {
+        bool cut = (v - s == CV);
+        if (!cut && v > s)
+            for (uint32_t e = L.dn_first[v]; e < L.dn_first[v + 1]; e++)
+                if (L.dn_arc[e].x >= s) { cut = true; break; }
+        if (cut) { cv.push_back(v); s = v; }
+        chunk_of[v] = (uint32_t)cv.size() - 1;
+    }
+    cv.push_back(n);
+    const uint32_t nchunks = (uint32_t)cv.size() - 1;
+    std::vector<uint32_t> dep(nchunks, 0);
+    for (uint32_t c = 0; c < nchunks; c++) {
+        int64_t d = -1;
+        for (uint32_t e = L.dn_first[cv[c]]; e < L.dn_first[cv[c + 1]]; e++)
+            d = std::max<int64_t>(d, chunk_of[L.dn_arc[e].x]);
+        if (d >= (int64_t)c) return nullptr;                    // would break the topological order
+        dep[c] = d < 0 ? 0u : (uint32_t)(d / p.grid) + 1u;      // 1 + iteration to wait for; 0 = none
+    }
+    p.nchunks = nchunks;
+    p.iters = (nchunks + p.grid - 1) / p.grid;
+    uint32_t *a, *b, *w;
+    if (dmalloc(&a, cv.size()) || dmalloc(&b, dep.size()) || dmalloc(&w, p.iters)) return nullptr;
+    p.chunk_v = a; p.chunk_dep = b; p.wave_done = w;
     if (cudaMemcpy(a, cv.data(), cv.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess ||
-        cudaMemcpy(b, cmeta.data(), cmeta.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess ||
-        cudaMemcpy(c, cstart.data(), cstart.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess ||
-        cudaMemcpy(d, h->lvl_off.data(), h->lvl_off.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess ||
-        cudaMemset(e, 0, h->levels * 4) != cudaSuccess) {
+        cudaMemcpy(b, dep.data(), dep.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess ||
+        cudaMemset(w, 0, (size_t)p.iters * 4) != cudaSuccess) {
         cudaGetLastError();
         return nullptr;
     }
@@ -270,7 +240,6 @@ phast_ctx::Plan* get_plan(phast_ctx* h, uint32_t k) {
     return &P;
 }
 
-// one full query (a1-a3) for k mapped sources; diam != nullptr -> fused max, no level-0 stores
 constexpr size_t MAX_TIMED_BATCHES = 16384;
 
 cudaEvent_t timing_event(phast_ctx* h) {
@@ -283,34 +252,39 @@ cudaEvent_t timing_event(phast_ctx* h) {
     return h->ev[h->ev_used++];
 }
 
+// one full query (a1-a3) for k mapped sources; diam != nullptr: fused max, rows of
+// vertices that are nobody's tail are not stored
 int run_query(phast_ctx* h, const Sources& S, uint32_t k, uint32_t* dist, uint32_t* diam, cudaStream_t st) {
-    cudaError_t e;
     cudaEvent_t e0 = nullptr, e1 = nullptr, e2 = nullptr;
     if (h->timing && h->ev_used + 3 <= 3 * MAX_TIMED_BATCHES) {
         e0 = timing_event(h); e1 = timing_event(h); e2 = timing_event(h);
         if (!e0 || !e1 || !e2) return PHAST_ECUDA;
         cudaEventRecord(e0, st);
     }
-    if ((e = launch_upward(h->g, S, k, dist, st)) != cudaSuccess) return PHAST_ECUDA;
-    if ((e = launch_scatter(h->g, k, dist, st)) != cudaSuccess) return PHAST_ECUDA;
+    if (launch_upward(h->g, S, k, dist, st) != cudaSuccess) return PHAST_ECUDA;
+    if (launch_scatter(h->g, k, dist, st) != cudaSuccess) return PHAST_ECUDA;
     if (e1) cudaEventRecord(e1, st);
-    phast_ctx::Plan* plan = h->sweep_mode == 0 ? get_plan(h, k) : nullptr;
-    if (plan) {                          // a3+a4: one persistent launch, dataflow over levels
+    phast_ctx::Plan* plan = h->sweep_mode != 1 ? get_plan(h, k) : nullptr;
+    if (plan) {   // a3 + a4: one persistent launch, dataflow over chunk waves
         if ((uint64_t)(plan->epoch + 1) * plan->p.grid >= 0x7FFFFFFFull) {
-            if (cudaMemsetAsync(plan->p.level_done, 0, plan->p.levels * 4, st) != cudaSuccess) return PHAST_ECUDA;
+            if (cudaMemsetAsync(plan->p.wave_done, 0, (size_t)plan->p.iters * 4, st) != cudaSuccess) return PHAST_ECUDA;
             plan->epoch = 0;
         }
         plan->epoch++;
         if (launch_sweep_persistent(h->g, plan->p, plan->epoch, dist, diam, st) != cudaSuccess) return PHAST_ECUDA;
-    } else {                             // one launch per level (§VI)
-        for (uint32_t j = 0; j < h->levels; j++) {
-            bool last = (j + 1 == h->levels);
+    } else if (!h->L.lvl_off.empty()) {   // one launch per level (§VI), level layout only
+        const uint32_t levels = h->L.levels;
+        for (uint32_t j = 0; j < levels; j++) {
+            bool last = (j + 1 == levels);
             bool store = !(diam && last);   // level-0 rows are never read again (diameter mode)
-            e = launch_sweep_level(h->g, k, h->lvl_off[j], h->lvl_off[j + 1], dist, diam, store, last, st);
-            if (e != cudaSuccess) return PHAST_ECUDA;
+            if (launch_sweep_level(h->g, k, h->L.lvl_off[j], h->L.lvl_off[j + 1], dist, diam, store, last, st) !=
+                cudaSuccess)
+                return PHAST_ECUDA;
         }
+    } else {
+        return PHAST_EINTERNAL;
     }
-    if ((e = launch_clear_flags(h->g, k, st)) != cudaSuccess) return PHAST_ECUDA;
+    if (launch_clear_flags(h->g, k, st) != cudaSuccess) return PHAST_ECUDA;
     if (e2) cudaEventRecord(e2, st);
     return PHAST_OK;
 }
@@ -326,18 +300,31 @@ ChOptions to_ch_options(const phast_opts* o) {
     return c;
 }
 
+int ensure_scratch(phast_ctx* h, size_t elems) {
+    if (h->dist_scratch_elems >= elems) return PHAST_OK;
+    cudaFree(h->dist_scratch);
+    h->dist_scratch = nullptr;
+    h->dist_scratch_elems = 0;
+    int rc = dmalloc(&h->dist_scratch, elems);
+    if (rc) return rc;
+    h->dist_scratch_elems = elems;
+    return PHAST_OK;
+}
+
 }  // namespace
 
 extern "C" {
 
-int phast_build(uint32_t n, const uint64_t* first, const uint32_t* head, const uint32_t* len,
-                const phast_opts* opts, phast_ctx** out) {
+int phast_build(uint32_t n, const uint64_t* first, const uint32_t* head, const uint32_t* len, const phast_opts* opts,
+                phast_ctx** out) {
     if (!out) return PHAST_EINVAL;
     *out = nullptr;
     int rc = validate_csr(n, first, head, len);
     if (rc) return rc;
     std::unique_ptr<phast_ctx> h(new (std::nothrow) phast_ctx());
     if (!h) return PHAST_ENOMEM;
+    uint32_t flags = opts ? opts->flags : 0u;
+    uint32_t delta = (opts && opts->delta) ? opts->delta : DEFAULT_DELTA;
     try {
         ChResult R;
         rc = ch_build(n, first, head, len, to_ch_options(opts), R);
@@ -346,13 +333,15 @@ int phast_build(uint32_t n, const uint64_t* first, const uint32_t* head, const u
         h->m = first[n];
         h->shortcuts = R.shortcuts;
         h->rounds = R.rounds;
+        rc = layout_build(R, first, head, (flags & PHAST_FLAG_LEVEL_LAYOUT) ? LAYOUT_LEVELS : LAYOUT_WAVEFRONT, delta,
+                          h->L);
         h->build_seconds = R.seconds;
-        rc = layout(h.get(), R);
         if (rc) return rc;
+        compute_tail_bits(h.get());
     } catch (const std::bad_alloc&) {
         return PHAST_ENOMEM;
     }
-    if (!(opts && (opts->flags & PHAST_FLAG_HOST_ONLY))) {
+    if (!(flags & PHAST_FLAG_HOST_ONLY)) {
         rc = upload(h.get());
         if (rc) return rc;
     }
@@ -391,15 +380,9 @@ int phast_trees_host(phast_ctx* h, const uint32_t* sources, uint32_t k, uint32_t
     if (h->device < 0) return PHAST_ESTATE;
     DeviceGuard dg(h->device);
     size_t elems = (size_t)h->n * k;
-    if (h->dist_scratch_elems < elems) {
-        cudaFree(h->dist_scratch);
-        h->dist_scratch = nullptr;
-        h->dist_scratch_elems = 0;
-        int rc = dmalloc(&h->dist_scratch, elems);
-        if (rc) return rc;
-        h->dist_scratch_elems = elems;
-    }
-    int rc = phast_trees(h, sources, k, h->dist_scratch, stream);
+    int rc = ensure_scratch(h, elems);
+    if (rc) return rc;
+    rc = phast_trees(h, sources, k, h->dist_scratch, stream);
     if (rc) return rc;
     cudaStream_t st = (cudaStream_t)stream;
     if (cudaMemcpyAsync(host_dist, h->dist_scratch, elems * 4, cudaMemcpyDeviceToHost, st) != cudaSuccess)
@@ -416,15 +399,8 @@ int phast_diameter(phast_ctx* h, const uint32_t* sources, uint64_t count, uint32
     DeviceGuard dg(h->device);
     if (!dg.ok) return PHAST_ECUDA;
     cudaStream_t st = (cudaStream_t)stream;
-    size_t elems = (size_t)h->n * k_batch;
-    if (h->dist_scratch_elems < elems) {
-        cudaFree(h->dist_scratch);
-        h->dist_scratch = nullptr;
-        h->dist_scratch_elems = 0;
-        int rc = dmalloc(&h->dist_scratch, elems);
-        if (rc) return rc;
-        h->dist_scratch_elems = elems;
-    }
+    int rc = ensure_scratch(h, (size_t)h->n * k_batch);
+    if (rc) return rc;
     uint64_t nb = (count + k_batch - 1) / k_batch;
     if (nb > 0xFFFFFFFFull) return PHAST_ERANGE;
     uint32_t* bm = batch_max_dev;
@@ -433,7 +409,7 @@ int phast_diameter(phast_ctx* h, const uint32_t* sources, uint64_t count, uint32
             cudaFree(h->batch_max_scratch);
             h->batch_max_scratch = nullptr;
             h->batch_max_elems = 0;
-            int rc = dmalloc(&h->batch_max_scratch, nb);
+            rc = dmalloc(&h->batch_max_scratch, nb);
             if (rc) return rc;
             h->batch_max_elems = nb;
         }
@@ -445,9 +421,9 @@ int phast_diameter(phast_ctx* h, const uint32_t* sources, uint64_t count, uint32
         uint64_t base = b * k_batch;
         for (uint32_t i = 0; i < k_batch; i++) {
             uint64_t idx = base + i < count ? base + i : base;   // pad with a duplicate (max unchanged)
-            S.s[i] = h->perm[sources[idx]];
+            S.s[i] = h->L.perm[sources[idx]];
         }
-        int rc = run_query(h, S, k_batch, h->dist_scratch, bm + b, st);
+        rc = run_query(h, S, k_batch, h->dist_scratch, bm + b, st);
         if (rc) return rc;
     }
     if (launch_max_reduce(bm, (uint32_t)nb, max_dev, st) != cudaSuccess) return PHAST_ECUDA;
@@ -458,67 +434,68 @@ int phast_info(const phast_ctx* h, phast_info_t* o) {
     if (!h || !o) return PHAST_EINVAL;
     std::memset(o, 0, sizeof(*o));
     o->n = h->n;
-    o->levels = h->levels;
+    o->levels = h->L.levels;
     o->m = h->m;
-    o->m_up = h->up_arc.size();
-    o->m_down = h->dn_arc.size();
-    std::vector<uint8_t> is_tail(h->n, 0);
-    for (const uint2& a : h->dn_arc) is_tail[a.x] = 1;
+    o->m_up = h->L.up_arc.size();
+    o->m_down = h->L.dn_arc.size();
     uint64_t nt = 0;
-    for (uint8_t t : is_tail) nt += t;
+    for (uint32_t w : h->tail_bits) nt += (uint64_t)__builtin_popcount(w);
     o->n_tail = nt;
     o->shortcuts = h->shortcuts;
     o->rounds = h->rounds;
     o->device = h->device < 0 ? 0xFFFFFFFFu : (uint32_t)h->device;
+    o->layout = h->L.mode;
+    o->delta = h->L.delta;
     o->build_seconds = h->build_seconds;
     return PHAST_OK;
 }
 
 int phast_level_sizes(const phast_ctx* h, uint32_t* out) {
     if (!h || !out) return PHAST_EINVAL;
-    for (uint32_t j = 0; j < h->levels; j++) out[h->levels - 1 - j] = h->lvl_off[j + 1] - h->lvl_off[j];
+    std::memset(out, 0, (size_t)h->L.levels * 4);
+    for (uint32_t l : h->L.level) out[l]++;
     return PHAST_OK;
 }
 
 int phast_order(const phast_ctx* h, uint32_t* o) {
     if (!h || !o) return PHAST_EINVAL;
-    std::memcpy(o, h->perm.data(), (size_t)h->n * 4);
+    std::memcpy(o, h->L.perm.data(), (size_t)h->n * 4);
     return PHAST_OK;
 }
 
-int phast_export(const phast_ctx* h, uint32_t* lvl_off, uint32_t* dn_first, uint32_t* dn_tail, uint32_t* dn_len,
+int phast_export(const phast_ctx* h, uint32_t* level, uint32_t* dn_first, uint32_t* dn_tail, uint32_t* dn_len,
                  uint32_t* up_first, uint32_t* up_head, uint32_t* up_len) {
     if (!h) return PHAST_EINVAL;
-    if (lvl_off) std::memcpy(lvl_off, h->lvl_off.data(), h->lvl_off.size() * 4);
-    if (dn_first) std::memcpy(dn_first, h->dn_first.data(), h->dn_first.size() * 4);
-    if (up_first) std::memcpy(up_first, h->up_first.data(), h->up_first.size() * 4);
-    for (size_t i = 0; i < h->dn_arc.size(); i++) {
-        if (dn_tail) dn_tail[i] = h->dn_arc[i].x;
-        if (dn_len) dn_len[i] = h->dn_arc[i].y;
+    const Layout& L = h->L;
+    if (level) std::memcpy(level, L.level.data(), L.level.size() * 4);
+    if (dn_first) std::memcpy(dn_first, L.dn_first.data(), L.dn_first.size() * 4);
+    if (up_first) std::memcpy(up_first, L.up_first.data(), L.up_first.size() * 4);
+    for (size_t i = 0; i < L.dn_arc.size(); i++) {
+        if (dn_tail) dn_tail[i] = L.dn_arc[i].x;
+        if (dn_len) dn_len[i] = L.dn_arc[i].y;
     }
-    for (size_t i = 0; i < h->up_arc.size(); i++) {
-        if (up_head) up_head[i] = h->up_arc[i].x;
-        if (up_len) up_len[i] = h->up_arc[i].y;
+    for (size_t i = 0; i < L.up_arc.size(); i++) {
+        if (up_head) up_head[i] = L.up_arc[i].x;
+        if (up_len) up_len[i] = L.up_arc[i].y;
     }
     return PHAST_OK;
 }
 
 // ---------------------------------------------------------------- save / load
-static const char MAGIC[8] = {'P', 'H', 'A', 'S', 'T', 'B', '2', '1'};
+static const char MAGIC[8] = {'P', 'H', 'A', 'S', 'T', 'B', '2', '2'};
 
 int phast_save(const phast_ctx* h, const char* path) {
     if (!h || !path) return PHAST_EINVAL;
     FILE* f = std::fopen(path, "wb");
     if (!f) return PHAST_EIO;
-    uint64_t hdr[8] = {h->n, h->levels, h->m, h->shortcuts, h->rounds, h->dn_arc.size(), h->up_arc.size(), 0};
-    bool ok = std::fwrite(MAGIC, 1, 8, f) == 8 && std::fwrite(hdr, 8, 8, f) == 8 &&
-              std::fwrite(&h->build_seconds, 8, 1, f) == 1 &&
-              std::fwrite(h->perm.data(), 4, h->n, f) == h->n &&
-              std::fwrite(h->lvl_off.data(), 4, h->lvl_off.size(), f) == h->lvl_off.size() &&
-              std::fwrite(h->dn_first.data(), 4, h->dn_first.size(), f) == h->dn_first.size() &&
-              std::fwrite(h->up_first.data(), 4, h->up_first.size(), f) == h->up_first.size() &&
-              std::fwrite(h->dn_arc.data(), 8, h->dn_arc.size(), f) == h->dn_arc.size() &&
-              std::fwrite(h->up_arc.data(), 8, h->up_arc.size(), f) == h->up_arc.size();
+    const Layout& L = h->L;
+    uint64_t hdr[10] = {h->n, L.levels, h->m, h->shortcuts, h->rounds, L.dn_arc.size(), L.up_arc.size(),
+                        L.mode, L.delta, L.lvl_off.size()};
+    auto wr = [&](const void* p, size_t sz, size_t cnt) { return std::fwrite(p, sz, cnt, f) == cnt; };
+    bool ok = wr(MAGIC, 1, 8) && wr(hdr, 8, 10) && wr(&h->build_seconds, 8, 1) && wr(L.perm.data(), 4, h->n) &&
+              wr(L.level.data(), 4, h->n) && wr(L.lvl_off.data(), 4, L.lvl_off.size()) &&
+              wr(L.dn_first.data(), 4, L.dn_first.size()) && wr(L.up_first.data(), 4, L.up_first.size()) &&
+              wr(L.dn_arc.data(), 8, L.dn_arc.size()) && wr(L.up_arc.data(), 8, L.up_arc.size());
     ok = (std::fclose(f) == 0) && ok;
     return ok ? PHAST_OK : PHAST_EIO;
 }
@@ -530,34 +507,35 @@ int phast_load(const char* path, uint32_t flags, phast_ctx** out) {
     if (!f) return PHAST_EIO;
     std::unique_ptr<phast_ctx> h(new (std::nothrow) phast_ctx());
     char magic[8];
-    uint64_t hdr[8];
-    bool ok = h && std::fread(magic, 1, 8, f) == 8 && std::memcmp(magic, MAGIC, 8) == 0 &&
-              std::fread(hdr, 8, 8, f) == 8 && std::fread(&h->build_seconds, 8, 1, f) == 1;
+    uint64_t hdr[10];
+    auto rd = [&](void* p, size_t sz, size_t cnt) { return std::fread(p, sz, cnt, f) == cnt; };
+    bool ok = h && rd(magic, 1, 8) && std::memcmp(magic, MAGIC, 8) == 0 && rd(hdr, 8, 10) &&
+              rd(&h->build_seconds, 8, 1) && hdr[0] > 0 && hdr[0] < 0xFFFFFFFFull;
     if (ok) {
+        Layout& L = h->L;
         try {
-            h->n = (uint32_t)hdr[0]; h->levels = (uint32_t)hdr[1]; h->m = hdr[2];
+            h->n = (uint32_t)hdr[0]; L.levels = (uint32_t)hdr[1]; h->m = hdr[2];
             h->shortcuts = hdr[3]; h->rounds = (uint32_t)hdr[4];
-            h->perm.resize(h->n); h->iperm.resize(h->n);
-            h->lvl_off.resize((size_t)h->levels + 1);
-            h->dn_first.resize((size_t)h->n + 1); h->up_first.resize((size_t)h->n + 1);
-            h->dn_arc.resize(hdr[5]); h->up_arc.resize(hdr[6]);
+            L.mode = (uint32_t)hdr[7]; L.delta = (uint32_t)hdr[8];
+            L.perm.resize(h->n); L.iperm.resize(h->n); L.level.resize(h->n);
+            L.lvl_off.resize(hdr[9]);
+            L.dn_first.resize((size_t)h->n + 1); L.up_first.resize((size_t)h->n + 1);
+            L.dn_arc.resize(hdr[5]); L.up_arc.resize(hdr[6]);
         } catch (const std::bad_alloc&) {
             std::fclose(f);
             return PHAST_ENOMEM;
         }
-        ok = std::fread(h->perm.data(), 4, h->n, f) == h->n &&
-             std::fread(h->lvl_off.data(), 4, h->lvl_off.size(), f) == h->lvl_off.size() &&
-             std::fread(h->dn_first.data(), 4, h->dn_first.size(), f) == h->dn_first.size() &&
-             std::fread(h->up_first.data(), 4, h->up_first.size(), f) == h->up_first.size() &&
-             std::fread(h->dn_arc.data(), 8, h->dn_arc.size(), f) == h->dn_arc.size() &&
-             std::fread(h->up_arc.data(), 8, h->up_arc.size(), f) == h->up_arc.size();
+        ok = rd(L.perm.data(), 4, h->n) && rd(L.level.data(), 4, h->n) && rd(L.lvl_off.data(), 4, L.lvl_off.size()) &&
+             rd(L.dn_first.data(), 4, L.dn_first.size()) && rd(L.up_first.data(), 4, L.up_first.size()) &&
+             rd(L.dn_arc.data(), 8, L.dn_arc.size()) && rd(L.up_arc.data(), 8, L.up_arc.size());
     }
     std::fclose(f);
     if (!ok) return PHAST_EIO;
     for (uint32_t v = 0; v < h->n; v++) {
-        if (h->perm[v] >= h->n) return PHAST_EIO;
-        h->iperm[h->perm[v]] = v;
+        if (h->L.perm[v] >= h->n) return PHAST_EIO;
+        h->L.iperm[h->L.perm[v]] = v;
     }
+    compute_tail_bits(h.get());
     if (!(flags & PHAST_FLAG_HOST_ONLY)) {
         int rc = upload(h.get());
         if (rc) return rc;
@@ -603,10 +581,16 @@ int phast_timing_read(phast_ctx* h, double* ms_up, double* ms_sweep, uint64_t* b
         float x = 0, y = 0;
         if (cudaEventSynchronize(h->ev[i + 2]) != cudaSuccess) { cudaGetLastError(); return PHAST_ECUDA; }
         if (cudaEventElapsedTime(&x, h->ev[i], h->ev[i + 1]) != cudaSuccess ||
-            cudaEventElapsedTime(&y, h->ev[i + 1], h->ev[i + 2]) != cudaSuccess) { cudaGetLastError(); return PHAST_ECUDA; }
-        a += x; b += y;
+            cudaEventElapsedTime(&y, h->ev[i + 1], h->ev[i + 2]) != cudaSuccess) {
+            cudaGetLastError();
+            return PHAST_ECUDA;
+        }
+        a += x;
+        b += y;
     }
-    *ms_up = a; *ms_sweep = b; *batches = h->ev_used / 3;
+    *ms_up = a;
+    *ms_sweep = b;
+    *batches = h->ev_used / 3;
     return PHAST_OK;
 }
 

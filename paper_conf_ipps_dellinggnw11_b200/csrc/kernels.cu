@@ -298,93 +298,183 @@ cudaError_t sweep_k(const DevImage& g, uint32_t vbeg, uint32_t vend, uint32_t* d
                 : sweep_launch<K, false, true, false>(g, vbeg, vend, dist, diam, st);
 }
 
-// ------------------------------------------------------------------ a3+a4 persistent
-constexpr uint32_t CHUNK_PASSES = 8;   // passes of the CTA over G-lane vertex groups per chunk
+// ------------------------------------------------------------------ a3+a4 persistent sweep
+// ONE launch for the whole sweep.  The internal order is topological (layout.cpp),
+// so the sweep is "a simple linear sweep in increasing order of IDs" (PAPER.md:16
+// §IV-A), cut into chunks of consecutive ids.  CTA b takes chunks b, b+grid, ...; a
+// chunk waits until every CTA has finished the iteration that produced its latest
+// tail (per-iteration completion counters, release/acquire at gpu scope), replacing
+// the paper's kernel launch per level (§VI).  STAGE: each chunk's
+// offsets first[vbeg..vend] and its contiguous G-down arc block are moved into shared
+// memory by the bulk-copy engine (cp.async.bulk + mbarrier), double-buffered: the
+// copy for the CTA's next chunk is in flight while the current chunk gathers, so a
+// gather waits on one HBM/L2 round trip (the tail row), not two.
+constexpr uint32_t CHUNK_PASSES = 4;     // passes of the CTA over G-lane vertex groups per chunk
+constexpr uint32_t STAGE_ARCS = 1024;    // arcs per shared-memory buffer (8 KB)
 
 __device__ __forceinline__ uint32_t ld_acquire_gpu(const uint32_t* p) {
     uint32_t v;
     asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
     return v;
 }
-// label loads bypass L1: a row read earlier on this SM (e.g. a seeded row) may since
-// have been rewritten by another SM within the same launch
-__device__ __forceinline__ uint32_t ldl(const uint32_t* p) { return __ldcg(p); }
-__device__ __forceinline__ uint2 ldl(const uint2* p) { return __ldcg(p); }
-__device__ __forceinline__ uint4 ldl(const uint4* p) { return __ldcg(p); }
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+    return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive_tx(uint64_t* bar, uint32_t bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t phase) {
+    asm volatile(
+        "{\n"
+        ".reg .pred P1;\n"
+        "WAIT_%=:\n"
+        "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1;\n"
+        "@!P1 bra WAIT_%=;\n"
+        "}\n" ::"r"(smem_u32(bar)),
+        "r"(phase)
+        : "memory");
+}
+__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                     smem_u32(dst)),
+                 "l"(src), "r"(bytes), "r"(smem_u32(bar))
+                 : "memory");
+}
 
-template <int K, bool DIAM>
-__global__ void __launch_bounds__(SWEEP_THREADS) sweep_persistent_kernel(const uint32_t* __restrict__ first,
-                                                                          const uint2* __restrict__ arcs,
-                                                                          uint32_t* __restrict__ d,
-                                                                          const uint32_t* __restrict__ flags,
-                                                                          SweepPlan p, uint32_t epoch,
-                                                                          uint32_t* __restrict__ diam) {
+struct StageInfo {
+    uint32_t vbeg, vend, dep;   // chunk [vbeg, vend); dep = 1 + iteration to wait for (0 = none)
+    uint32_t f0;                // vertex id of sfirst[0] (multiple of 4)
+    uint32_t a0;                // arc index of sarc[0] (even)
+    uint32_t staged;            // 1 if first/arcs are in shared memory
+};
+
+template <int K, bool DIAM, bool STAGE>
+__global__ void __launch_bounds__(SWEEP_THREADS, 4) sweep_persistent_kernel(const uint32_t* __restrict__ first,
+                                                                            const uint2* __restrict__ arcs,
+                                                                            uint32_t* __restrict__ d,
+                                                                            const uint32_t* __restrict__ flags,
+                                                                            const uint32_t* __restrict__ tail_bits,
+                                                                            SweepPlan p, uint32_t epoch,
+                                                                            uint32_t* __restrict__ diam) {
     using T = typename RowT<K>::T;
     constexpr uint32_t W = RowT<K>::W;
-    constexpr uint32_t G = K / W;                   // lanes per vertex
-    constexpr uint32_t VPP = SWEEP_THREADS / G;     // vertices per pass
-    __shared__ uint32_t s_known;                    // leading levels known complete
-    if (threadIdx.x == 0) s_known = 0;
+    constexpr uint32_t G = K / W;                               // lanes per vertex
+    constexpr uint32_t VPP = SWEEP_THREADS / G;                 // vertices per pass
+    constexpr uint32_t STAGE_FIRST = VPP * CHUNK_PASSES + 8;    // first[vbeg..vend], 16-byte aligned
+    __shared__ __align__(16) uint2 sarc[STAGE ? 2 : 1][STAGE ? STAGE_ARCS : 2];
+    __shared__ __align__(16) uint32_t sfirst[STAGE ? 2 : 1][STAGE ? STAGE_FIRST : 4];
+    __shared__ __align__(8) uint64_t bar[2];
+    __shared__ StageInfo info[2];
+    __shared__ uint32_t s_known;                                // leading iterations known complete
     const uint32_t grid = gridDim.x;
-    const uint32_t last = p.levels - 1;
     const uint32_t lane = threadIdx.x % G;
+    if (threadIdx.x == 0) {
+        s_known = 0;
+        if constexpr (STAGE) {
+            mbar_init(&bar[0], 1);
+            mbar_init(&bar[1], 1);
+            asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+        }
+    }
+    __syncthreads();
+
+    // thread 0: describe chunk c in info[b] and start its bulk copies
+    auto stage = [&](uint32_t b, uint32_t c) {
+        StageInfo in;
+        in.vbeg = __ldg(&p.chunk_v[c]);
+        in.vend = __ldg(&p.chunk_v[c + 1]);
+        in.dep = __ldg(&p.chunk_dep[c]);
+        in.f0 = in.vbeg & ~3u;
+        in.a0 = 0;
+        in.staged = 0;
+        if constexpr (STAGE) {
+            const uint32_t f1 = (in.vend + 1 + 3) & ~3u;      // [f0, f1) covers first[vbeg..vend]
+            const uint32_t e0 = __ldg(&first[in.vbeg]), e1 = __ldg(&first[in.vend]);
+            in.a0 = e0 & ~1u;
+            const uint32_t a1 = (e1 + 1) & ~1u;
+            if (f1 - in.f0 <= STAGE_FIRST && a1 - in.a0 <= STAGE_ARCS) {
+                in.staged = 1;
+                asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+                const uint32_t fb = (f1 - in.f0) * 4, ab = (a1 - in.a0) * 8;
+                mbar_arrive_tx(&bar[b], fb + ab);
+                bulk_g2s(&sfirst[b][0], first + in.f0, fb, &bar[b]);
+                if (ab) bulk_g2s(&sarc[b][0], arcs + in.a0, ab, &bar[b]);
+            }
+        }
+        info[b] = in;
+    };
+
+    uint32_t phase = 0;   // bit b = parity of the next completion of bar[b]
     uint32_t mx = 0;
-    for (uint32_t c = blockIdx.x; c < p.nchunks; c += grid) {
-        const uint32_t meta = __ldg(&p.chunk_meta[c]);
-        const uint32_t J = meta >> 16;
-        const int D = (int)(meta & 0xFFFFu) - 1;
+    if (threadIdx.x == 0 && blockIdx.x < p.nchunks) stage(0, blockIdx.x);
+    uint32_t it = 0;
+    for (uint32_t c = blockIdx.x; c < p.nchunks; c += grid, it++) {
+        const uint32_t b = it & 1u;
         if (threadIdx.x == 0) {
-            uint32_t known = s_known;
-            while ((int)known <= D) {
-                const uint32_t need = epoch * min(__ldg(&p.chunk_start[known + 1]) - __ldg(&p.chunk_start[known]), grid);
+            const uint32_t dep = info[b].dep;
+            if (dep > s_known) {                               // wait for iteration dep-1 everywhere
+                const uint32_t w = dep - 1;
+                const uint32_t need = epoch * min(grid, p.nchunks - w * grid);
                 uint32_t ns = 32;
-                while (ld_acquire_gpu(&p.level_done[known]) < need) {
+                while (ld_acquire_gpu(&p.wave_done[w]) < need) {
                     __nanosleep(ns);
                     ns = min(ns * 2, 256u);
                 }
-                known++;
+                s_known = dep;                                 // counters are monotone in w
+                __threadfence();                               // drop older L1 lines of this SM
             }
-            s_known = known;
-            __threadfence();
         }
         __syncthreads();
-        const uint32_t vbeg = __ldg(&p.chunk_v[c]);
-        const uint32_t vend = min(vbeg + p.chunk_vertices, __ldg(&p.lvl_off[J + 1]));
-        const bool store = !DIAM || J != last;     // diameter mode: level-0 rows are never read again
-        const bool stream_store = (J == last);     // level-0 rows are never re-read in this sweep
-        for (uint32_t base = vbeg; base < vend; base += VPP) {
+        const StageInfo in = info[b];
+        if (threadIdx.x == 0 && c + grid < p.nchunks) stage(b ^ 1u, c + grid);   // prefetch the next chunk
+        if (STAGE && in.staged) {
+            mbar_wait(&bar[b], (phase >> b) & 1u);
+            phase ^= 1u << b;
+        }
+        for (uint32_t base = in.vbeg; base < in.vend; base += VPP) {
             const uint32_t v = base + threadIdx.x / G;
-            if (v >= vend) break;
+            if (v >= in.vend) break;
             T acc = inf_row<T>();
-            if ((__ldg(&flags[v >> 5]) >> (v & 31)) & 1u)
-                acc = ldl(reinterpret_cast<const T*>(d + (size_t)v * K) + lane);
-            uint32_t e = __ldg(&first[v]);
-            const uint32_t e1 = __ldg(&first[v + 1]);
-            while (e < e1) {                         // up to 4 gathers in flight per lane
+            if ((__ldg(&flags[v >> 5]) >> (v & 31)) & 1u)   // visited by an upward search (§IV-C)
+                acc = reinterpret_cast<const T*>(d + (size_t)v * K)[lane];
+            uint32_t e, e1;
+            if (STAGE && in.staged) {
+                e = sfirst[b][v - in.f0];
+                e1 = sfirst[b][v + 1 - in.f0];
+            } else {
+                e = __ldg(&first[v]);
+                e1 = __ldg(&first[v + 1]);
+            }
+            while (e < e1) {                                   // up to 4 gathers in flight per lane
                 const uint32_t cnt = min(e1 - e, 4u);
                 uint2 a[4];
                 T x[4];
 #pragma unroll
                 for (uint32_t j = 0; j < 4; j++)
-                    if (j < cnt) a[j] = __ldg(&arcs[e + j]);
+                    if (j < cnt) a[j] = (STAGE && in.staged) ? sarc[b][e + j - in.a0] : __ldg(&arcs[e + j]);
 #pragma unroll
                 for (uint32_t j = 0; j < 4; j++)
-                    if (j < cnt) x[j] = ldl(reinterpret_cast<const T*>(d + (size_t)a[j].x * K) + lane);
+                    if (j < cnt) x[j] = reinterpret_cast<const T*>(d + (size_t)a[j].x * K)[lane];
 #pragma unroll
                 for (uint32_t j = 0; j < 4; j++)
                     if (j < cnt) acc = relax(acc, x[j], a[j].y);
                 e += cnt;
             }
-            if (store) {
+            const bool is_tail = (__ldg(&tail_bits[v >> 5]) >> (v & 31)) & 1u;
+            if (!DIAM || is_tail) {                            // diameter: rows nobody reads are not stored
                 T* q = reinterpret_cast<T*>(d + (size_t)v * K) + lane;
-                if (stream_store) st_stream(q, acc); else *q = acc;
+                if (is_tail) *q = acc;                         // re-read soon from L2
+                else st_stream(q, acc);                        // never re-read: evict first
             }
             if constexpr (DIAM) mx = max(mx, fmax_of(acc));
         }
-        __syncthreads();                             // every row of this chunk is written
-        if (threadIdx.x == 0 && c + grid >= __ldg(&p.chunk_start[J + 1])) {
-            __threadfence();                         // release: rows before the counter
-            atomicAdd(&p.level_done[J], 1u);         // this CTA's last chunk of level J
+        __syncthreads();                                       // every row of this chunk is written
+        if (threadIdx.x == 0) {
+            __threadfence();                                   // release: rows before the counter
+            atomicAdd(&p.wave_done[it], 1u);
         }
     }
     if constexpr (DIAM) {
@@ -400,28 +490,35 @@ __global__ void __launch_bounds__(SWEEP_THREADS) sweep_persistent_kernel(const u
     }
 }
 
-template <int K, bool DIAM>
+template <int K, bool DIAM, bool STAGE>
 int persistent_occupancy() {
     int b = 0;
-    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, sweep_persistent_kernel<K, DIAM>, SWEEP_THREADS, 0) !=
-        cudaSuccess) {
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, sweep_persistent_kernel<K, DIAM, STAGE>, SWEEP_THREADS,
+                                                      0) != cudaSuccess) {
         cudaGetLastError();
         return 1;
     }
     return b > 0 ? b : 1;
 }
 
+template <int K, bool STAGE>
+cudaError_t persistent_k2(const DevImage& g, const SweepPlan& p, uint32_t epoch, uint32_t* dist, uint32_t* diam,
+                          cudaStream_t st) {
+    if (diam)
+        sweep_persistent_kernel<K, true, STAGE><<<p.grid, SWEEP_THREADS, 0, st>>>(
+            g.dn_first, g.dn_arc, dist, g.flags, g.tail_bits, p, epoch, diam);
+    else
+        sweep_persistent_kernel<K, false, STAGE><<<p.grid, SWEEP_THREADS, 0, st>>>(
+            g.dn_first, g.dn_arc, dist, g.flags, g.tail_bits, p, epoch, nullptr);
+    g_launches++;
+    return cudaGetLastError();
+}
+
 template <int K>
 cudaError_t persistent_k(const DevImage& g, const SweepPlan& p, uint32_t epoch, uint32_t* dist, uint32_t* diam,
                          cudaStream_t st) {
-    if (diam)
-        sweep_persistent_kernel<K, true><<<p.grid, SWEEP_THREADS, 0, st>>>(g.dn_first, g.dn_arc, dist, g.flags, p,
-                                                                           epoch, diam);
-    else
-        sweep_persistent_kernel<K, false><<<p.grid, SWEEP_THREADS, 0, st>>>(g.dn_first, g.dn_arc, dist, g.flags, p,
-                                                                            epoch, nullptr);
-    g_launches++;
-    return cudaGetLastError();
+    return p.variant == 1 ? persistent_k2<K, true>(g, p, epoch, dist, diam, st)
+                          : persistent_k2<K, false>(g, p, epoch, dist, diam, st);
 }
 
 template <int K>
@@ -491,8 +588,10 @@ uint32_t sweep_chunk_vertices(uint32_t k) {
     return (SWEEP_THREADS / G) * CHUNK_PASSES;
 }
 
-int sweep_blocks_per_sm(uint32_t k, bool diam) {
-#define OCC(K) (diam ? persistent_occupancy<K, true>() : persistent_occupancy<K, false>())
+int sweep_blocks_per_sm(uint32_t k, bool diam, uint32_t variant) {
+#define OCC(K)                                                                                               \
+    (variant == 1 ? (diam ? persistent_occupancy<K, true, true>() : persistent_occupancy<K, false, true>())   \
+                  : (diam ? persistent_occupancy<K, true, false>() : persistent_occupancy<K, false, false>()))
     switch (k) {
         case 1: return OCC(1);
         case 2: return OCC(2);

@@ -16,6 +16,7 @@ struct DevImage {
     const uint32_t* up_first = nullptr;  // [n+1]   G-up out-arcs by tail
     const uint2* up_arc = nullptr;       // [m_up]   {head, len}
     uint32_t* flags = nullptr;           // [ceil(n/32)] visited bits (§IV-C), zero between calls
+    const uint32_t* tail_bits = nullptr; // [ceil(n/32)] bit v: v is the tail of some G-down arc
     uint32_t* seed_v = nullptr;          // [KMAX * seed_cap] upward search spaces: vertex
     uint32_t* seed_d = nullptr;          // [KMAX * seed_cap] upward search spaces: label
     uint32_t* seed_cnt = nullptr;        // [KMAX]
@@ -40,22 +41,20 @@ cudaError_t launch_scatter(const DevImage& g, uint32_t k, uint32_t* dist, cudaSt
 cudaError_t launch_sweep_level(const DevImage& g, uint32_t k, uint32_t vbeg, uint32_t vend,
                                uint32_t* dist, uint32_t* diam, bool store, bool last_level,
                                cudaStream_t st);
-// Plan of the persistent (single-launch) sweep for one k: the vertex range of every
-// level is cut into chunks that never straddle a level; each chunk records its
-// level (processing index J, 0 = top) and D = the latest processing index among the
-// levels of its in-arc tails (-1 if none).  A CTA may start chunk c once levels
-// 0..D are complete (Lemma 4.1 guarantees D < J).
+// Plan of the persistent (single-launch) sweep for one k: the internal order is cut
+// into chunks of consecutive ids (no chunk contains both ends of a G-down arc);
+// chunk c runs on CTA c % grid in iteration c / grid and depends on iteration
+// chunk_dep[c] - 1 (0 = no dependency).
 struct SweepPlan {
-    uint32_t k = 0, nchunks = 0, levels = 0, grid = 0, chunk_vertices = 0;
-    const uint32_t* chunk_v = nullptr;      // [nchunks] first vertex of each chunk
-    const uint32_t* chunk_meta = nullptr;   // [nchunks] J << 16 | (D + 1)
-    const uint32_t* chunk_start = nullptr;  // [levels+1] first chunk of each level
-    const uint32_t* lvl_off = nullptr;      // [levels+1]
-    uint32_t* level_done = nullptr;         // [levels] monotone completion counters
+    uint32_t k = 0, nchunks = 0, grid = 0, iters = 0, chunk_cap = 0;
+    uint32_t variant = 1;                   // 1: bulk-staged arcs, 0: arcs read from global
+    const uint32_t* chunk_v = nullptr;      // [nchunks+1] chunk boundaries
+    const uint32_t* chunk_dep = nullptr;    // [nchunks]
+    uint32_t* wave_done = nullptr;          // [iters] monotone completion counters (epochs)
 };
 // vertices per chunk and CTAs per SM the persistent sweep uses for this k
 uint32_t sweep_chunk_vertices(uint32_t k);
-int sweep_blocks_per_sm(uint32_t k, bool diam);
+int sweep_blocks_per_sm(uint32_t k, bool diam, uint32_t variant);
 // a3 + a4 in ONE launch: dataflow over levels through the completion counters
 // (epoch = number of launches of this plan so far, 1-based).
 cudaError_t launch_sweep_persistent(const DevImage& g, const SweepPlan& p, uint32_t epoch, uint32_t* dist,

@@ -1,0 +1,39 @@
+// layout.h -- vertex renumbering and the G-up / G-down CSRs in internal ids.
+// Internal to libphast.so.
+#pragma once
+#include <cstdint>
+#include <vector>
+
+#include "ch.h"
+
+namespace phast {
+
+enum LayoutMode : uint32_t {
+    LAYOUT_WAVEFRONT = 0,   // skewed spatial wavefront (default)
+    LAYOUT_LEVELS = 1,      // the paper's: level descending, input (DFS) order within a level
+};
+
+struct Arc {
+    uint32_t x, y;          // {tail, len} in G-down; {head, len} in G-up (same bytes as CUDA uint2)
+};
+
+struct Layout {
+    uint32_t mode = LAYOUT_WAVEFRONT;
+    uint32_t delta = 0;
+    uint32_t levels = 0;
+    std::vector<uint32_t> perm;      // internal_of_original
+    std::vector<uint32_t> iperm;     // original_of_internal
+    std::vector<uint32_t> level;     // CH level L of every internal id (0 = lowest)
+    std::vector<uint32_t> lvl_off;   // LAYOUT_LEVELS only: [levels+1], j = 0 is the top level
+    std::vector<uint32_t> dn_first, up_first;   // [n+1]
+    std::vector<Arc> dn_arc, up_arc;
+};
+
+// Builds the renumbering from the CH result.  first/head: the input graph (used
+// for the BFS that gives the spatial rank in LAYOUT_WAVEFRONT).  Returns 0,
+// PHAST_ERANGE (more than 2^32-2 arcs) or PHAST_EINTERNAL (an ordering invariant
+// failed: Lemma 4.1, or a G-down tail not before its head).
+int layout_build(const ChResult& R, const uint64_t* first, const uint32_t* head, uint32_t mode, uint32_t delta,
+                 Layout& out);
+
+}  // namespace phast

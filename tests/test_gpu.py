@@ -121,13 +121,16 @@ def test_upward_global_fallback_and_overflow(monkeypatch):
         h.sync()                                       # error word is cleared
 
 
-@pytest.mark.parametrize("mode", ["levels", "persistent"])
-def test_sweep_modes(monkeypatch, mode):
-    """Both level schedules (one launch per level, §VI; and the single
-    persistent launch with per-level completion counters) are bit-exact."""
+@pytest.mark.parametrize("mode,level_layout,delta", [("levels", True, 0), ("staged", True, 0),
+                                                     ("persistent", False, 0), ("staged", False, 0),
+                                                     ("staged", False, 300)])
+def test_sweep_modes(monkeypatch, mode, level_layout, delta):
+    """Every schedule is bit-exact: one launch per level on the paper's level layout
+    (§VI), and the single persistent launch (with and without bulk-staged
+    arcs) on both layouts, including a small wavefront skew (many short dependencies)."""
     monkeypatch.setenv("PHAST_SWEEP", mode)
     g = phastgen.road(120_000, seed=33)
-    with P.Phast.from_graph(g) as h:
+    with P.Phast.from_graph(g, level_layout=level_layout, delta=delta) as h:
         for k in (1, 2, 16, 64):
             src = phastgen.sources(g.n, k, seed=900 + k)
             assert np.array_equal(gpu_trees(h, src), oracle.sssp_many(g, src)), k

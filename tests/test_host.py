@@ -63,35 +63,47 @@ def test_host_hierarchy_sweep_equals_oracle(name):
     assert np.array_equal(got, want)
 
 
+@pytest.mark.parametrize("level_layout", [False, True])
 @pytest.mark.parametrize("name", sorted(GRAPHS))
-def test_layout_invariants(name):
+def test_layout_invariants(name, level_layout):
     g = GRAPHS[name]()
-    h = P.Phast.from_graph(g, host_only=True)
+    h = P.Phast.from_graph(g, host_only=True, level_layout=level_layout)
     ex = h.export()
     n, L = h.n, h.levels
-    lo = ex["lvl_off"]
-    assert lo[0] == 0 and lo[-1] == n and np.all(np.diff(lo.astype(np.int64)) > 0)
-    # level index of every internal id (0 = top level, processed first)
-    lev = np.repeat(np.arange(L), np.diff(lo.astype(np.int64)))
+    lev = ex["level"].astype(np.int64)
     heads = np.repeat(np.arange(n), np.diff(ex["dn_first"].astype(np.int64)))
-    # Lemma 4.1 (§IV-A): every tail of a G-down arc is on a strictly higher
-    # level, i.e. processed in an earlier level group
-    assert np.all(lev[ex["dn_tail"]] < lev[heads])
-    tails = np.repeat(np.arange(n), np.diff(ex["up_first"].astype(np.int64)))
-    assert np.all(lev[ex["up_head"]] < lev[tails])
-    # level sizes agree with lvl_off; level 0 (lowest) is the last group
+    tails = ex["dn_tail"].astype(np.int64)
+    # Lemma 4.1 (§IV-A): every tail of a G-down arc is on a strictly higher level
+    assert np.all(lev[tails] > lev[heads])
+    # the internal order is a reverse topological order of G-down: a linear sweep in
+    # increasing id order sees every tail before its head (§III)
+    assert np.all(tails < heads)
+    uh = ex["up_head"].astype(np.int64)
+    utails = np.repeat(np.arange(n), np.diff(ex["up_first"].astype(np.int64)))
+    assert np.all(lev[uh] > lev[utails])
     ls = h.level_sizes()
-    assert ls.sum() == n and ls[0] == lo[-1] - lo[-2]
-    # permutation is a bijection; within a level, original ids ascend (DFS order kept)
+    assert ls.sum() == n and len(ls) == L and np.array_equal(ls, np.bincount(lev, minlength=L))
     perm = h.order()
     assert np.array_equal(np.sort(perm), np.arange(n, dtype=np.uint32))
-    inv = np.empty_like(perm)
-    inv[perm] = np.arange(n, dtype=np.uint32)
-    for j in range(L):
-        seg = inv[lo[j]:lo[j + 1]]
-        assert np.all(np.diff(seg.astype(np.int64)) > 0)
     # level-0 vertices are never tails (their rows need not be stored in diameter mode)
-    assert np.all(lev[ex["dn_tail"]] < L - 1) if ex["dn_tail"].size else True
+    assert np.all(lev[tails] > 0)
+    assert h.info().layout == (1 if level_layout else 0)
+    if level_layout:
+        inv = np.empty_like(perm)
+        inv[perm] = np.arange(n, dtype=np.uint32)
+        # levels are contiguous, highest first; DFS (input) order kept within a level
+        assert np.all(np.diff(lev) <= 0)
+        for l in range(L):
+            seg = inv[lev == l]
+            assert np.all(np.diff(seg.astype(np.int64)) > 0)
+
+
+@pytest.mark.parametrize("level_layout", [False, True])
+def test_both_layouts_sweep_equals_oracle(level_layout):
+    g = phastgen.road(40_000, seed=12)
+    h = P.Phast.from_graph(g, host_only=True, level_layout=level_layout, delta=5000)
+    src = phastgen.sources(g.n, 5, seed=3)
+    assert np.array_equal(chref.phast_cpu(h, h.export(), src), oracle.sssp_many(g, src))
 
 
 def test_shortcut_lengths_dominate_distances():
