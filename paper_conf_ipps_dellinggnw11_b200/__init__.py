@@ -71,6 +71,7 @@ def _load_lib():
         "phast_strerror": ([ctypes.c_int], ctypes.c_char_p),
         "phast_launch_count": ([], u64),
         "phast_timing": ([vp, ctypes.c_int], ctypes.c_int),
+        "phast_plan_stats": ([vp, u32, u32, vp], ctypes.c_int),
         "phast_timing_read": ([vp, ctypes.POINTER(ctypes.c_double), ctypes.POINTER(ctypes.c_double),
                                ctypes.POINTER(ctypes.c_uint64)], ctypes.c_int),
     }
@@ -84,7 +85,8 @@ def _load_lib():
 _lib = _load_lib()
 EXPORTED = ("phast_build", "phast_trees", "phast_trees_host", "phast_sync", "phast_diameter", "phast_info",
             "phast_level_sizes", "phast_order", "phast_export", "phast_save", "phast_load", "phast_free",
-            "phast_strerror", "phast_launch_count", "phast_timing", "phast_timing_read")
+            "phast_strerror", "phast_launch_count", "phast_timing", "phast_timing_read",
+            "phast_plan_stats")
 
 
 def _check(fn, rc):
@@ -221,6 +223,11 @@ class Phast:
         bm_ptr = None if batch_max is None else batch_max.data_ptr()
         _check("phast_diameter", _lib.phast_diameter(self._h, src.ctypes.data, src.size, k_batch,
                                                      max_out.data_ptr(), bm_ptr, _stream_ptr(stream)))
+
+    def plan_stats(self, k: int, grid: int) -> dict:
+        out = np.zeros(5, np.uint64)
+        _check("phast_plan_stats", _lib.phast_plan_stats(self._h, k, grid, out.ctypes.data))
+        return dict(chunks=int(out[0]), slots=int(out[1]), pads=int(out[2]), iterations=int(out[3]), chunk_cap=int(out[4]))
 
     def timing(self, enable: bool):
         _check("phast_timing", _lib.phast_timing(self._h, 1 if enable else 0))

@@ -186,6 +186,17 @@ int map_sources(const phast_ctx* h, const uint32_t* src, uint32_t k, Sources& S)
     return PHAST_OK;
 }
 
+// Chunk size: at most sweep_chunk_vertices(k); in the wavefront layout small enough
+// that one iteration of all CTAs (grid * cap vertices) stays under delta / 2, so that
+// almost every dependency points at least one iteration back (few pad slots).
+uint32_t chunk_cap_for(const Layout& L, uint32_t k, uint32_t grid) {
+    const uint32_t vmax = sweep_chunk_vertices(k), vpp = sweep_pass_vertices(k);
+    if (L.mode != LAYOUT_WAVEFRONT) return vmax;
+    uint32_t cap = L.delta / (2 * std::max(1u, grid));
+    cap = cap / vpp * vpp;
+    return std::max(vpp, std::min(vmax, cap));
+}
+
 // Plan of the persistent sweep for one k.  Chunks are contiguous internal-id ranges
 // of at most CV vertices, cut wherever a vertex has a G-down tail inside the open
 // chunk (so a chunk never waits on itself).  Chunk c is processed by CTA c % grid in
@@ -196,40 +207,23 @@ phast_ctx::Plan* get_plan(phast_ctx* h, uint32_t k) {
     if (it != h->plans.end()) return it->second.ok ? &it->second : nullptr;
     phast_ctx::Plan& P = h->plans[k];
     const Layout& L = h->L;
-    const uint32_t n = h->n;
-    const uint32_t CV = sweep_chunk_vertices(k);
     SweepPlan& p = P.p;
     p.k = k;
     p.variant = h->sweep_mode == 2 ? 0u : 1u;
-    p.chunk_cap = CV;
     int occ = std::min(sweep_blocks_per_sm(k, false, p.variant), sweep_blocks_per_sm(k, true, p.variant));
     p.grid = (uint32_t)std::max(1, occ * num_sms());
-    std::vector<uint32_t> cv, chunk_of(n);
-    uint32_t s = 0;
-    cv.push_back(0);
-    for (uint32_t v = 0; v < n; v++) {
-        bool cut = (v - s == CV);
-        if (!cut && v > s)
-            for (uint32_t e = L.dn_first[v]; e < L.dn_first[v + 1]; e++)
-                if (L.dn_arc[e].x >= s) { cut = true; break; }
-        if (cut) { cv.push_back(v); s = v; }
-        chunk_of[v] = (uint32_t)cv.size() - 1;
-    }
-    cv.push_back(n);
-    const uint32_t nchunks = (uint32_t)cv.size() - 1;
-    std::vector<uint32_t> dep(nchunks, 0);
-    for (uint32_t c = 0; c < nchunks; c++) {
-        int64_t d = -1;
-        for (uint32_t e = L.dn_first[cv[c]]; e < L.dn_first[cv[c + 1]]; e++)
-            d = std::max<int64_t>(d, chunk_of[L.dn_arc[e].x]);
-        if (d >= (int64_t)c) return nullptr;                    // would break the topological order
-        dep[c] = d < 0 ? 0u : (uint32_t)(d / p.grid) + 1u;      // 1 + iteration to wait for; 0 = none
-    }
-    p.nchunks = nchunks;
-    p.iters = (nchunks + p.grid - 1) / p.grid;
+    const uint32_t CV = chunk_cap_for(h->L, k, p.grid);
+    p.chunk_cap = CV;
+    ChunkPlan cp;
+    if (plan_chunks(L, CV, p.grid, cp)) return nullptr;
+    p.nchunks = cp.slots;
+    p.iters = (cp.slots + p.grid - 1) / p.grid;
+    const std::vector<uint32_t>& cv = cp.slot_v;
+    const std::vector<uint32_t>& dep = cp.dep;
     uint32_t *a, *b, *w;
     if (dmalloc(&a, cv.size()) || dmalloc(&b, dep.size()) || dmalloc(&w, p.iters)) return nullptr;
     p.chunk_v = a; p.chunk_dep = b; p.wave_done = w;
+    p.err = h->g.err;
     if (cudaMemcpy(a, cv.data(), cv.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess ||
         cudaMemcpy(b, dep.data(), dep.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess ||
         cudaMemset(w, 0, (size_t)p.iters * 4) != cudaSuccess) {
@@ -370,7 +364,7 @@ int phast_sync(phast_ctx* h, void* stream) {
     if (cudaMemcpy(&err, h->g.err, 4, cudaMemcpyDeviceToHost) != cudaSuccess) return PHAST_ECUDA;
     if (err) {
         cudaMemset(h->g.err, 0, 4);
-        return PHAST_ERANGE;
+        return (err & 1u) ? PHAST_ERANGE : PHAST_ECUDA;   // bit 0: search-space overflow; bit 1: watchdog
     }
     return PHAST_OK;
 }
@@ -591,6 +585,19 @@ int phast_timing_read(phast_ctx* h, double* ms_up, double* ms_sweep, uint64_t* b
     *ms_up = a;
     *ms_sweep = b;
     *batches = h->ev_used / 3;
+    return PHAST_OK;
+}
+
+int phast_plan_stats(const phast_ctx* h, uint32_t k, uint32_t grid, uint64_t* out) {
+    if (!h || !out || !k_ok(k) || grid == 0) return PHAST_EINVAL;
+    ChunkPlan cp;
+    int rc = plan_chunks(h->L, chunk_cap_for(h->L, k, grid), grid, cp);
+    if (rc) return rc;
+    out[0] = cp.chunks;
+    out[1] = cp.slots;
+    out[2] = cp.pads;
+    out[3] = (cp.slots + grid - 1) / grid;
+    out[4] = chunk_cap_for(h->L, k, grid);
     return PHAST_OK;
 }
 

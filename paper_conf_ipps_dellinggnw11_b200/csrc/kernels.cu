@@ -317,6 +317,11 @@ __device__ __forceinline__ uint32_t ld_acquire_gpu(const uint32_t* p) {
     asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
     return v;
 }
+__device__ __forceinline__ uint64_t globaltimer_ns() {
+    uint64_t t;
+    asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+    return t;
+}
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
     return static_cast<uint32_t>(__cvta_generic_to_shared(p));
 }
@@ -419,9 +424,14 @@ __global__ void __launch_bounds__(SWEEP_THREADS, 4) sweep_persistent_kernel(cons
                 const uint32_t w = dep - 1;
                 const uint32_t need = epoch * min(grid, p.nchunks - w * grid);
                 uint32_t ns = 32;
+                const uint64_t t0 = globaltimer_ns();
                 while (ld_acquire_gpu(&p.wave_done[w]) < need) {
                     __nanosleep(ns);
                     ns = min(ns * 2, 256u);
+                    if (globaltimer_ns() - t0 > 4000000000ull) {   // watchdog: never hang the GPU;
+                        atomicOr(p.err, 2u);                        // phast_sync reports ECUDA
+                        break;
+                    }
                 }
                 s_known = dep;                                 // counters are monotone in w
                 __threadfence();                               // drop older L1 lines of this SM
@@ -582,6 +592,8 @@ cudaError_t launch_sweep_level(const DevImage& g, uint32_t k, uint32_t vbeg, uin
     PHAST_K_SWITCH(k, CALL_SW)
 #undef CALL_SW
 }
+
+uint32_t sweep_pass_vertices(uint32_t k) { return SWEEP_THREADS / (k >= 4 ? k / 4 : 1); }
 
 uint32_t sweep_chunk_vertices(uint32_t k) {
     uint32_t G = k >= 4 ? k / 4 : 1;

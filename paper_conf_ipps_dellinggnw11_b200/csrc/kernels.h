@@ -51,9 +51,11 @@ struct SweepPlan {
     const uint32_t* chunk_v = nullptr;      // [nchunks+1] chunk boundaries
     const uint32_t* chunk_dep = nullptr;    // [nchunks]
     uint32_t* wave_done = nullptr;          // [iters] monotone completion counters (epochs)
+    uint32_t* err = nullptr;                // sticky device error word (bit 1: dependency watchdog)
 };
 // vertices per chunk and CTAs per SM the persistent sweep uses for this k
-uint32_t sweep_chunk_vertices(uint32_t k);
+uint32_t sweep_chunk_vertices(uint32_t k);   // max vertices per chunk
+uint32_t sweep_pass_vertices(uint32_t k);    // vertices per pass of a CTA
 int sweep_blocks_per_sm(uint32_t k, bool diam, uint32_t variant);
 // a3 + a4 in ONE launch: dataflow over levels through the completion counters
 // (epoch = number of launches of this plan so far, 1-based).

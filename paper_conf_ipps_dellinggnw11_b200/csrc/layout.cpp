@@ -168,4 +168,50 @@ int layout_build(const ChResult& R, const uint64_t* first, const uint32_t* head,
     return ok ? 0 : kEinternal;
 }
 
+int plan_chunks(const Layout& L, uint32_t cap, uint32_t grid, ChunkPlan& P) {
+    const uint32_t n = (uint32_t)L.perm.size();
+    if (cap == 0 || grid == 0) return kEinternal;
+    // 1. chunk boundaries and each chunk's latest tail chunk (unpadded numbering)
+    std::vector<uint32_t> cb{0}, chunk_of(n);
+    uint32_t s = 0;
+    for (uint32_t v = 0; v < n; v++) {
+        bool cut = (v - s == cap);
+        if (!cut && v > s)
+            for (uint32_t e = L.dn_first[v]; e < L.dn_first[v + 1]; e++)
+                if (L.dn_arc[e].x >= s) { cut = true; break; }
+        if (cut) { cb.push_back(v); s = v; }
+        chunk_of[v] = (uint32_t)cb.size() - 1;
+    }
+    cb.push_back(n);
+    const uint32_t nch = (uint32_t)cb.size() - 1;
+    // 2. slots with padding so that a dependency is always in an earlier iteration
+    std::vector<uint32_t> slot(nch);
+    P.slot_v.clear();
+    P.dep.clear();
+    uint64_t next = 0;
+    P.pads = 0;
+    for (uint32_t c = 0; c < nch; c++) {
+        int64_t d = -1;
+        for (uint32_t e = L.dn_first[cb[c]]; e < L.dn_first[cb[c + 1]]; e++)
+            d = std::max<int64_t>(d, chunk_of[L.dn_arc[e].x]);
+        if (d >= (int64_t)c) return kEinternal;
+        uint64_t j = next;
+        if (d >= 0 && slot[d] / grid == j / grid) j = (j / grid + 1) * grid;
+        if (j > 0xFFFFFFF0ull) return kErange;
+        for (uint64_t q = next; q < j; q++) {              // pads: empty ranges
+            P.slot_v.push_back(cb[c]);
+            P.dep.push_back(0);
+            P.pads++;
+        }
+        slot[c] = (uint32_t)j;
+        P.slot_v.push_back(cb[c]);
+        P.dep.push_back(d < 0 ? 0u : slot[d] / grid + 1u);
+        next = j + 1;
+    }
+    P.slot_v.push_back(n);
+    P.chunks = nch;
+    P.slots = (uint32_t)P.dep.size();
+    return 0;
+}
+
 }  // namespace phast

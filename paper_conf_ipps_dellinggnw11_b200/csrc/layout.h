@@ -36,4 +36,18 @@ struct Layout {
 int layout_build(const ChResult& R, const uint64_t* first, const uint32_t* head, uint32_t mode, uint32_t delta,
                  Layout& out);
 
+// Static schedule of the persistent sweep: the internal order is cut into chunks of
+// consecutive ids (at most cap vertices; cut wherever a vertex has a G-down tail in
+// the open chunk).  Chunk slot j runs on CTA j % grid in iteration j / grid.  A chunk
+// whose latest tail chunk would fall in its own iteration is moved to the next
+// iteration (empty pad slots in between), so every dependency points to an earlier
+// iteration.  slot_v[j]..slot_v[j+1] is slot j's vertex range (empty for pads);
+// dep[j] = 1 + iteration it waits for (0 = none).
+struct ChunkPlan {
+    std::vector<uint32_t> slot_v;   // [slots+1]
+    std::vector<uint32_t> dep;      // [slots]
+    uint32_t chunks = 0, slots = 0, pads = 0;
+};
+int plan_chunks(const Layout& L, uint32_t cap, uint32_t grid, ChunkPlan& out);
+
 }  // namespace phast

@@ -176,3 +176,20 @@ def test_degenerate_graphs():
     ex = h2.export()
     got = chref.phast_cpu(h2, ex, [0, 1, 2])
     assert np.array_equal(got, oracle.sssp_many(g2, [0, 1, 2]))
+
+
+@pytest.mark.parametrize("level_layout", [False, True])
+def test_sweep_schedule_is_well_formed(level_layout):
+    """The persistent sweep's static schedule (layout.cpp plan_chunks): every chunk is
+    placed in an iteration after the one producing its latest tail; pad slots fill the
+    gaps.  plan_chunks itself fails (EINTERNAL) if a dependency is not strictly earlier."""
+    g = phastgen.road(60_000, seed=9)
+    h = P.Phast.from_graph(g, host_only=True, level_layout=level_layout)
+    for k in (1, 16, 64):
+        for grid in (1, 7, 148, 592):
+            st = h.plan_stats(k, grid)
+            assert st["slots"] == st["chunks"] + st["pads"]
+            assert st["iterations"] == -(-st["slots"] // grid)
+            assert st["chunks"] >= -(-g.n // (4 * 256 // max(1, k // 4)))
+    with pytest.raises(P.PhastError):
+        h.plan_stats(3, 148)
