@@ -42,7 +42,8 @@ struct phast_ctx {
         bool ok = false;
     };
     std::map<uint32_t, Plan> plans;
-    int sweep_mode = 0;   // 0 = persistent + bulk-staged arcs, 1 = one launch per level, 2 = persistent, no staging
+    // 0 = warp dataflow (default), 1 = one launch per level, 2 = CTA waves, 3 = CTA waves + bulk-staged arcs
+    int sweep_mode = 0;
     // stage timing (phast_timing)
     bool timing = false;
     std::vector<cudaEvent_t> ev;   // 3 per recorded batch
@@ -87,6 +88,9 @@ void free_plans(phast_ctx* h) {
         cudaFree((void*)kv.second.p.chunk_v);
         cudaFree((void*)kv.second.p.chunk_dep);
         cudaFree(kv.second.p.wave_done);
+        cudaFree((void*)kv.second.p.wmeta);
+        cudaFree((void*)kv.second.p.wdeps);
+        cudaFree(kv.second.p.done);
     }
     h->plans.clear();
 }
@@ -123,7 +127,10 @@ int upload(phast_ctx* h) {
     DevImage& g = h->g;
     g.n = h->n;
     if (const char* e = std::getenv("PHAST_SWEEP"))
-        h->sweep_mode = std::strcmp(e, "levels") == 0 ? 1 : std::strcmp(e, "persistent") == 0 ? 2 : 0;
+        h->sweep_mode = std::strcmp(e, "levels") == 0       ? 1
+                        : std::strcmp(e, "persistent") == 0 ? 2
+                        : std::strcmp(e, "staged") == 0     ? 3
+                                                            : 0;
     if (h->sweep_mode == 1 && h->L.mode != LAYOUT_LEVELS) h->sweep_mode = 0;   // needs contiguous levels
     // test knobs (rounded down to powers of two): shrink the shared-memory table / the
     // per-source capacity to exercise the global fallback and the overflow error path
@@ -209,9 +216,29 @@ phast_ctx::Plan* get_plan(phast_ctx* h, uint32_t k) {
     const Layout& L = h->L;
     SweepPlan& p = P.p;
     p.k = k;
-    p.variant = h->sweep_mode == 2 ? 0u : 1u;
+    p.variant = h->sweep_mode == 2 ? 0u : h->sweep_mode == 3 ? 1u : 2u;
     int occ = std::min(sweep_blocks_per_sm(k, false, p.variant), sweep_blocks_per_sm(k, true, p.variant));
     p.grid = (uint32_t)std::max(1, occ * num_sms());
+    p.err = h->g.err;
+    if (p.variant == 2) {
+        p.workers = p.grid * (SWEEP_WARPS);
+        WarpPlan wp;
+        if (plan_warp_chunks(L, sweep_warp_chunk_vertices(k), p.workers, wp)) return nullptr;
+        p.nchunks = wp.chunks;
+        p.chunk_cap = sweep_warp_chunk_vertices(k);
+        uint32_t *a, *b, *w;
+        if (dmalloc(&a, wp.meta.size()) || dmalloc(&b, wp.deps.size()) || dmalloc(&w, wp.chunks)) return nullptr;
+        p.wmeta = reinterpret_cast<const uint4*>(a); p.wdeps = b; p.done = w;
+        if (cudaMemcpy(a, wp.meta.data(), wp.meta.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess ||
+            (!wp.deps.empty() &&
+             cudaMemcpy(b, wp.deps.data(), wp.deps.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess) ||
+            cudaMemset(w, 0, (size_t)wp.chunks * 4) != cudaSuccess) {
+            cudaGetLastError();
+            return nullptr;
+        }
+        P.ok = true;
+        return &P;
+    }
     const uint32_t CV = chunk_cap_for(h->L, k, p.grid);
     p.chunk_cap = CV;
     ChunkPlan cp;
@@ -223,7 +250,6 @@ phast_ctx::Plan* get_plan(phast_ctx* h, uint32_t k) {
     uint32_t *a, *b, *w;
     if (dmalloc(&a, cv.size()) || dmalloc(&b, dep.size()) || dmalloc(&w, p.iters)) return nullptr;
     p.chunk_v = a; p.chunk_dep = b; p.wave_done = w;
-    p.err = h->g.err;
     if (cudaMemcpy(a, cv.data(), cv.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess ||
         cudaMemcpy(b, dep.data(), dep.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess ||
         cudaMemset(w, 0, (size_t)p.iters * 4) != cudaSuccess) {
@@ -260,7 +286,7 @@ int run_query(phast_ctx* h, const Sources& S, uint32_t k, uint32_t* dist, uint32
     if (e1) cudaEventRecord(e1, st);
     phast_ctx::Plan* plan = h->sweep_mode != 1 ? get_plan(h, k) : nullptr;
     if (plan) {   // a3 + a4: one persistent launch, dataflow over chunk waves
-        if ((uint64_t)(plan->epoch + 1) * plan->p.grid >= 0x7FFFFFFFull) {
+        if (plan->p.variant != 2 && (uint64_t)(plan->epoch + 1) * plan->p.grid >= 0x7FFFFFFFull) {
             if (cudaMemsetAsync(plan->p.wave_done, 0, (size_t)plan->p.iters * 4, st) != cudaSuccess) return PHAST_ECUDA;
             plan->epoch = 0;
         }

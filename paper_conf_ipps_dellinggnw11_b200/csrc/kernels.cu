@@ -500,6 +500,117 @@ __global__ void __launch_bounds__(SWEEP_THREADS, 4) sweep_persistent_kernel(cons
     }
 }
 
+// ------------------------------------------------------------------ a3+a4 warp dataflow (variant 2)
+// ONE launch; the unit of work is a chunk of consecutive ids handled by ONE warp.
+// Chunk c runs on warp c % workers; before gathering, the warp's lanes acquire the
+// completion flags of the chunks holding its tails (precomputed list, only chunks of
+// other warps).  No CTA barriers, no level or wave coupling: a chunk starts as soon
+// as its own tails are final.  Label rows are read with ld.global.cg (L2), never
+// from a possibly stale L1 line.
+constexpr uint32_t WARP_PASSES = 4;
+constexpr uint32_t WARP_STAGE_ARCS = 64;
+constexpr uint32_t WARPS_PER_CTA = SWEEP_THREADS / 32;
+
+template <int K, bool DIAM>
+__global__ void __launch_bounds__(SWEEP_THREADS, 5) sweep_warp_kernel(const uint32_t* __restrict__ first,
+                                                                      const uint2* __restrict__ arcs,
+                                                                      uint32_t* __restrict__ d,
+                                                                      const uint32_t* __restrict__ flags,
+                                                                      const uint32_t* __restrict__ tail_bits,
+                                                                      SweepPlan p, uint32_t epoch,
+                                                                      uint32_t* __restrict__ diam) {
+    using T = typename RowT<K>::T;
+    constexpr uint32_t W = RowT<K>::W;
+    constexpr uint32_t G = K / W;              // lanes per vertex
+    constexpr uint32_t VPW = 32 / G;           // vertices per warp pass
+    constexpr uint32_t CAP = VPW * WARP_PASSES;
+    __shared__ uint2 sarc[WARPS_PER_CTA][WARP_STAGE_ARCS];
+    __shared__ uint32_t sfirst[WARPS_PER_CTA][CAP + 1];
+    const uint32_t wid = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const uint32_t gl = lane % G, grp = lane / G;
+    uint32_t mx = 0;
+    for (uint32_t c = blockIdx.x * WARPS_PER_CTA + wid; c < p.nchunks; c += p.workers) {
+        const uint4 m = __ldg(&p.wmeta[c]);    // {vbeg, vend, dbeg, dend}
+        for (uint32_t i = m.z + lane; i < m.w; i += 32) {
+            const uint32_t x = __ldg(&p.wdeps[i]);
+            if (ld_acquire_gpu(&p.done[x]) < epoch) {
+                uint32_t ns = 32;
+                const uint64_t t0 = globaltimer_ns();
+                while (ld_acquire_gpu(&p.done[x]) < epoch) {
+                    __nanosleep(ns);
+                    ns = min(ns * 2, 512u);
+                    if (globaltimer_ns() - t0 > 4000000000ull) {   // watchdog: never hang the GPU
+                        atomicOr(p.err, 2u);
+                        break;
+                    }
+                }
+            }
+        }
+        __syncwarp();
+        const uint32_t nv = m.y - m.x;
+        for (uint32_t i = lane; i <= nv; i += 32) sfirst[wid][i] = __ldg(&first[m.x + i]);
+        __syncwarp();
+        const uint32_t e0 = sfirst[wid][0];
+        const uint32_t na = sfirst[wid][nv] - e0;
+        const bool staged = na <= WARP_STAGE_ARCS;
+        if (staged)
+            for (uint32_t i = lane; i < na; i += 32) sarc[wid][i] = __ldg(&arcs[e0 + i]);
+        __syncwarp();
+        for (uint32_t base = 0; base < nv; base += VPW) {
+            const uint32_t li = base + grp;
+            if (li >= nv) break;
+            const uint32_t v = m.x + li;
+            T acc = inf_row<T>();
+            if ((__ldg(&flags[v >> 5]) >> (v & 31)) & 1u)   // visited by an upward search (§IV-C)
+                acc = __ldcg(reinterpret_cast<const T*>(d + (size_t)v * K) + gl);
+            uint32_t e = sfirst[wid][li];
+            const uint32_t e1 = sfirst[wid][li + 1];
+            while (e < e1) {                                   // up to 4 gathers in flight per lane
+                const uint32_t cnt = min(e1 - e, 4u);
+                uint2 a[4];
+                T x[4];
+#pragma unroll
+                for (uint32_t j = 0; j < 4; j++)
+                    if (j < cnt) a[j] = staged ? sarc[wid][e + j - e0] : __ldg(&arcs[e + j]);
+#pragma unroll
+                for (uint32_t j = 0; j < 4; j++)
+                    if (j < cnt) x[j] = __ldcg(reinterpret_cast<const T*>(d + (size_t)a[j].x * K) + gl);
+#pragma unroll
+                for (uint32_t j = 0; j < 4; j++)
+                    if (j < cnt) acc = relax(acc, x[j], a[j].y);
+                e += cnt;
+            }
+            const bool is_tail = (__ldg(&tail_bits[v >> 5]) >> (v & 31)) & 1u;
+            if (!DIAM || is_tail) {                            // diameter: rows nobody reads are not stored
+                T* q = reinterpret_cast<T*>(d + (size_t)v * K) + gl;
+                if (is_tail) *q = acc;                         // re-read soon, from L2
+                else st_stream(q, acc);                        // never re-read: evict first
+            }
+            if constexpr (DIAM) mx = max(mx, fmax_of(acc));
+        }
+        __syncwarp();                                          // all rows of the chunk are issued
+        if (lane == 0) {
+            __threadfence();                                   // release the rows before the flag
+            atomicExch(&p.done[c], epoch);
+        }
+    }
+    if constexpr (DIAM) {
+        mx = __reduce_max_sync(0xFFFFFFFFu, mx);
+        if (lane == 0 && mx) atomicMax(diam, mx);
+    }
+}
+
+template <int K, bool DIAM>
+int warp_occupancy() {
+    int b = 0;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, sweep_warp_kernel<K, DIAM>, SWEEP_THREADS, 0) !=
+        cudaSuccess) {
+        cudaGetLastError();
+        return 1;
+    }
+    return b > 0 ? b : 1;
+}
+
 template <int K, bool DIAM, bool STAGE>
 int persistent_occupancy() {
     int b = 0;
@@ -527,6 +638,16 @@ cudaError_t persistent_k2(const DevImage& g, const SweepPlan& p, uint32_t epoch,
 template <int K>
 cudaError_t persistent_k(const DevImage& g, const SweepPlan& p, uint32_t epoch, uint32_t* dist, uint32_t* diam,
                          cudaStream_t st) {
+    if (p.variant == 2) {
+        if (diam)
+            sweep_warp_kernel<K, true><<<p.grid, SWEEP_THREADS, 0, st>>>(g.dn_first, g.dn_arc, dist, g.flags,
+                                                                         g.tail_bits, p, epoch, diam);
+        else
+            sweep_warp_kernel<K, false><<<p.grid, SWEEP_THREADS, 0, st>>>(g.dn_first, g.dn_arc, dist, g.flags,
+                                                                          g.tail_bits, p, epoch, nullptr);
+        g_launches++;
+        return cudaGetLastError();
+    }
     return p.variant == 1 ? persistent_k2<K, true>(g, p, epoch, dist, diam, st)
                           : persistent_k2<K, false>(g, p, epoch, dist, diam, st);
 }
@@ -593,6 +714,8 @@ cudaError_t launch_sweep_level(const DevImage& g, uint32_t k, uint32_t vbeg, uin
 #undef CALL_SW
 }
 
+uint32_t sweep_warp_chunk_vertices(uint32_t k) { return (32 / (k >= 4 ? k / 4 : 1)) * WARP_PASSES; }
+
 uint32_t sweep_pass_vertices(uint32_t k) { return SWEEP_THREADS / (k >= 4 ? k / 4 : 1); }
 
 uint32_t sweep_chunk_vertices(uint32_t k) {
@@ -602,7 +725,8 @@ uint32_t sweep_chunk_vertices(uint32_t k) {
 
 int sweep_blocks_per_sm(uint32_t k, bool diam, uint32_t variant) {
 #define OCC(K)                                                                                               \
-    (variant == 1 ? (diam ? persistent_occupancy<K, true, true>() : persistent_occupancy<K, false, true>())   \
+    (variant == 2 ? (diam ? warp_occupancy<K, true>() : warp_occupancy<K, false>()) :                         \
+     variant == 1 ? (diam ? persistent_occupancy<K, true, true>() : persistent_occupancy<K, false, true>())   \
                   : (diam ? persistent_occupancy<K, true, false>() : persistent_occupancy<K, false, false>()))
     switch (k) {
         case 1: return OCC(1);

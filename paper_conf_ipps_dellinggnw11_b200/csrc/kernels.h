@@ -47,7 +47,12 @@ cudaError_t launch_sweep_level(const DevImage& g, uint32_t k, uint32_t vbeg, uin
 // chunk_dep[c] - 1 (0 = no dependency).
 struct SweepPlan {
     uint32_t k = 0, nchunks = 0, grid = 0, iters = 0, chunk_cap = 0;
-    uint32_t variant = 1;                   // 1: bulk-staged arcs, 0: arcs read from global
+    uint32_t variant = 2;                   // 2: warp dataflow; 1: CTA waves + bulk-staged arcs; 0: CTA waves
+    // variant 2 (warp dataflow)
+    uint32_t workers = 0;                   // warps in the grid
+    const uint4* wmeta = nullptr;           // [nchunks] {vbeg, vend, dbeg, dend}
+    const uint32_t* wdeps = nullptr;        // dependency chunk ids
+    uint32_t* done = nullptr;               // [nchunks] epoch of the last completion
     const uint32_t* chunk_v = nullptr;      // [nchunks+1] chunk boundaries
     const uint32_t* chunk_dep = nullptr;    // [nchunks]
     uint32_t* wave_done = nullptr;          // [iters] monotone completion counters (epochs)
@@ -56,6 +61,8 @@ struct SweepPlan {
 // vertices per chunk and CTAs per SM the persistent sweep uses for this k
 uint32_t sweep_chunk_vertices(uint32_t k);   // max vertices per chunk
 uint32_t sweep_pass_vertices(uint32_t k);    // vertices per pass of a CTA
+uint32_t sweep_warp_chunk_vertices(uint32_t k);
+constexpr uint32_t SWEEP_WARPS = 8;               // warps per CTA of the persistent sweeps   // vertices per chunk of one warp (variant 2)
 int sweep_blocks_per_sm(uint32_t k, bool diam, uint32_t variant);
 // a3 + a4 in ONE launch: dataflow over levels through the completion counters
 // (epoch = number of launches of this plan so far, 1-based).

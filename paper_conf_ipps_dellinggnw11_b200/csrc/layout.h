@@ -50,4 +50,16 @@ struct ChunkPlan {
 };
 int plan_chunks(const Layout& L, uint32_t cap, uint32_t grid, ChunkPlan& out);
 
+// Warp-granular dataflow schedule (default sweep): chunks of consecutive ids (at most
+// cap vertices, cut at intra-chunk dependencies), chunk c handled by worker (warp)
+// c % workers in program order.  meta[4c..4c+3] = {vbeg, vend, dbeg, dend}:
+// deps[dbeg..dend) are the distinct chunks holding a tail of chunk c that another
+// worker handles (same-worker chunks are earlier in that worker's program order).
+struct WarpPlan {
+    std::vector<uint32_t> meta;
+    std::vector<uint32_t> deps;
+    uint32_t chunks = 0;
+};
+int plan_warp_chunks(const Layout& L, uint32_t cap, uint32_t workers, WarpPlan& out);
+
 }  // namespace phast

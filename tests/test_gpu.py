@@ -121,13 +121,15 @@ def test_upward_global_fallback_and_overflow(monkeypatch):
         h.sync()                                       # error word is cleared
 
 
-@pytest.mark.parametrize("mode,level_layout,delta", [("levels", True, 0), ("staged", True, 0),
-                                                     ("persistent", False, 0), ("staged", False, 0),
+@pytest.mark.parametrize("mode,level_layout,delta", [("levels", True, 0), ("warp", True, 0), ("staged", True, 0),
+                                                     ("warp", False, 0), ("persistent", False, 0),
+                                                     ("staged", False, 0), ("warp", False, 300),
                                                      ("staged", False, 300)])
 def test_sweep_modes(monkeypatch, mode, level_layout, delta):
     """Every schedule is bit-exact: one launch per level on the paper's level layout
-    (§VI), and the single persistent launch (with and without bulk-staged
-    arcs) on both layouts, including a small wavefront skew (many short dependencies)."""
+    (§VI); the single persistent launch as warp dataflow (default) or CTA
+    waves (with and without bulk-staged arcs), on both layouts, including a small
+    wavefront skew (many short dependencies)."""
     monkeypatch.setenv("PHAST_SWEEP", mode)
     g = phastgen.road(120_000, seed=33)
     with P.Phast.from_graph(g, level_layout=level_layout, delta=delta) as h:
