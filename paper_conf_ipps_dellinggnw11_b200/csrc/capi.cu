@@ -131,7 +131,9 @@ int upload(phast_ctx* h) {
                         : std::strcmp(e, "persistent") == 0 ? 2
                         : std::strcmp(e, "staged") == 0     ? 3
                                                             : 0;
-    if (h->sweep_mode == 1 && h->L.mode != LAYOUT_LEVELS) h->sweep_mode = 0;   // needs contiguous levels
+    // level layouts default to one launch per level (the fastest schedule measured on them)
+    if (!std::getenv("PHAST_SWEEP") && !h->L.lvl_off.empty()) h->sweep_mode = 1;
+    if (h->sweep_mode == 1 && h->L.lvl_off.empty()) h->sweep_mode = 0;   // needs contiguous levels
     // test knobs (rounded down to powers of two): shrink the shared-memory table / the
     // per-source capacity to exercise the global fallback and the overflow error path
     uint32_t seed_cap = SEED_CAP, smem_cap = 4096;
@@ -353,8 +355,10 @@ int phast_build(uint32_t n, const uint64_t* first, const uint32_t* head, const u
         h->m = first[n];
         h->shortcuts = R.shortcuts;
         h->rounds = R.rounds;
-        rc = layout_build(R, first, head, (flags & PHAST_FLAG_LEVEL_LAYOUT) ? LAYOUT_LEVELS : LAYOUT_WAVEFRONT, delta,
-                          h->L);
+        const uint32_t mode = (flags & PHAST_FLAG_LEVEL_LAYOUT)
+                                  ? ((flags & PHAST_FLAG_BFS_IN_LEVEL) ? LAYOUT_LEVELS_BFS : LAYOUT_LEVELS)
+                                  : LAYOUT_WAVEFRONT;
+        rc = layout_build(R, first, head, mode, delta, h->L);
         h->build_seconds = R.seconds;
         if (rc) return rc;
         compute_tail_bits(h.get());

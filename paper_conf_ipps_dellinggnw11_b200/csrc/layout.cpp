@@ -89,14 +89,20 @@ int layout_build(const ChResult& R, const uint64_t* first, const uint32_t* head,
     if (mdn >= 0xFFFFFFFEull || mup >= 0xFFFFFFFEull) return kErange;
 
     std::vector<uint32_t> order(n);   // order[i] = original id with internal id i
-    if (mode == LAYOUT_LEVELS) {
+    if (mode == LAYOUT_LEVELS || mode == LAYOUT_LEVELS_BFS) {
         std::vector<uint32_t> cnt(levels, 0);
         for (uint32_t v = 0; v < n; v++) cnt[R.level[v]]++;
         L.lvl_off.assign(levels + 1, 0);
         for (uint32_t j = 0; j < levels; j++) L.lvl_off[j + 1] = L.lvl_off[j] + cnt[levels - 1 - j];
         std::vector<uint32_t> pos(levels);
         for (uint32_t j = 0; j < levels; j++) pos[levels - 1 - j] = L.lvl_off[j];
-        for (uint32_t v = 0; v < n; v++) order[pos[R.level[v]]++] = v;   // ascending input id within a level
+        std::vector<uint32_t> by(n);                 // within-level order: input id, or BFS rank
+        std::iota(by.begin(), by.end(), 0u);
+        if (mode == LAYOUT_LEVELS_BFS) {
+            std::vector<uint32_t> rank = bfs_rank(n, first, head);
+            std::sort(by.begin(), by.end(), [&](uint32_t a, uint32_t b) { return rank[a] < rank[b]; });
+        }
+        for (uint32_t v : by) order[pos[R.level[v]]++] = v;
     } else {
         std::vector<uint32_t> rank = bfs_rank(n, first, head);
         std::vector<int64_t> key(n);

@@ -11,6 +11,7 @@ namespace phast {
 enum LayoutMode : uint32_t {
     LAYOUT_WAVEFRONT = 0,   // skewed spatial wavefront (default)
     LAYOUT_LEVELS = 1,      // the paper's: level descending, input (DFS) order within a level
+    LAYOUT_LEVELS_BFS = 2,  // level descending, BFS (spatial sweep) order within a level
 };
 
 struct Arc {

@@ -121,7 +121,8 @@ def test_upward_global_fallback_and_overflow(monkeypatch):
         h.sync()                                       # error word is cleared
 
 
-@pytest.mark.parametrize("mode,level_layout,delta", [("levels", True, 0), ("warp", True, 0), ("staged", True, 0),
+@pytest.mark.parametrize("mode,level_layout,delta", [("levels", True, 0), ("levels", "bfs", 0),
+                                                     ("warp", True, 0), ("staged", True, 0),
                                                      ("warp", False, 0), ("persistent", False, 0),
                                                      ("staged", False, 0), ("warp", False, 300),
                                                      ("staged", False, 300)])
@@ -132,7 +133,8 @@ def test_sweep_modes(monkeypatch, mode, level_layout, delta):
     wavefront skew (many short dependencies)."""
     monkeypatch.setenv("PHAST_SWEEP", mode)
     g = phastgen.road(120_000, seed=33)
-    with P.Phast.from_graph(g, level_layout=level_layout, delta=delta) as h:
+    with P.Phast.from_graph(g, level_layout=bool(level_layout), bfs_in_level=level_layout == "bfs",
+                            delta=delta) as h:
         for k in (1, 2, 16, 64):
             src = phastgen.sources(g.n, k, seed=900 + k)
             assert np.array_equal(gpu_trees(h, src), oracle.sssp_many(g, src)), k

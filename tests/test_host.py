@@ -63,11 +63,16 @@ def test_host_hierarchy_sweep_equals_oracle(name):
     assert np.array_equal(got, want)
 
 
-@pytest.mark.parametrize("level_layout", [False, True])
+LAYOUTS = {"wavefront": {}, "levels": dict(level_layout=True),
+           "levels-bfs": dict(level_layout=True, bfs_in_level=True)}
+
+
+@pytest.mark.parametrize("layout", sorted(LAYOUTS))
 @pytest.mark.parametrize("name", sorted(GRAPHS))
-def test_layout_invariants(name, level_layout):
+def test_layout_invariants(name, layout):
     g = GRAPHS[name]()
-    h = P.Phast.from_graph(g, host_only=True, level_layout=level_layout)
+    h = P.Phast.from_graph(g, host_only=True, **LAYOUTS[layout])
+    level_layout = layout != "wavefront"
     ex = h.export()
     n, L = h.n, h.levels
     lev = ex["level"].astype(np.int64)
@@ -87,8 +92,10 @@ def test_layout_invariants(name, level_layout):
     assert np.array_equal(np.sort(perm), np.arange(n, dtype=np.uint32))
     # level-0 vertices are never tails (their rows need not be stored in diameter mode)
     assert np.all(lev[tails] > 0)
-    assert h.info().layout == (1 if level_layout else 0)
+    assert h.info().layout == {"wavefront": 0, "levels": 1, "levels-bfs": 2}[layout]
     if level_layout:
+        assert np.all(np.diff(lev) <= 0)                 # levels contiguous, highest first
+    if layout == "levels":
         inv = np.empty_like(perm)
         inv[perm] = np.arange(n, dtype=np.uint32)
         # levels are contiguous, highest first; DFS (input) order kept within a level
@@ -98,10 +105,10 @@ def test_layout_invariants(name, level_layout):
             assert np.all(np.diff(seg.astype(np.int64)) > 0)
 
 
-@pytest.mark.parametrize("level_layout", [False, True])
-def test_both_layouts_sweep_equals_oracle(level_layout):
+@pytest.mark.parametrize("layout", sorted(LAYOUTS))
+def test_every_layout_sweep_equals_oracle(layout):
     g = phastgen.road(40_000, seed=12)
-    h = P.Phast.from_graph(g, host_only=True, level_layout=level_layout, delta=5000)
+    h = P.Phast.from_graph(g, host_only=True, delta=5000, **LAYOUTS[layout])
     src = phastgen.sources(g.n, 5, seed=3)
     assert np.array_equal(chref.phast_cpu(h, h.export(), src), oracle.sssp_many(g, src))
 
@@ -178,13 +185,13 @@ def test_degenerate_graphs():
     assert np.array_equal(got, oracle.sssp_many(g2, [0, 1, 2]))
 
 
-@pytest.mark.parametrize("level_layout", [False, True])
-def test_sweep_schedule_is_well_formed(level_layout):
+@pytest.mark.parametrize("layout", sorted(LAYOUTS))
+def test_sweep_schedule_is_well_formed(layout):
     """The persistent sweep's static schedule (layout.cpp plan_chunks): every chunk is
     placed in an iteration after the one producing its latest tail; pad slots fill the
     gaps.  plan_chunks itself fails (EINTERNAL) if a dependency is not strictly earlier."""
     g = phastgen.road(60_000, seed=9)
-    h = P.Phast.from_graph(g, host_only=True, level_layout=level_layout)
+    h = P.Phast.from_graph(g, host_only=True, **LAYOUTS[layout])
     for k in (1, 16, 64):
         for grid in (1, 7, 148, 592):
             st = h.plan_stats(k, grid)
