@@ -42,7 +42,8 @@ struct phast_ctx {
         bool ok = false;
     };
     std::map<uint32_t, Plan> plans;
-    // 0 = warp dataflow (default), 1 = one launch per level, 2 = CTA waves, 3 = CTA waves + bulk-staged arcs
+    // 0 = warp dataflow (default), 1 = one launch per level, 2 = CTA waves, 3 = CTA waves + bulk-staged
+    // arcs, 4 = pipelined gather (k >= 4; else warp dataflow)
     int sweep_mode = 0;
     // stage timing (phast_timing)
     bool timing = false;
@@ -89,6 +90,7 @@ void free_plans(phast_ctx* h) {
         cudaFree((void*)kv.second.p.chunk_dep);
         cudaFree(kv.second.p.wave_done);
         cudaFree((void*)kv.second.p.wmeta);
+        cudaFree((void*)kv.second.p.pinfo);
         cudaFree((void*)kv.second.p.wdeps);
         cudaFree(kv.second.p.done);
     }
@@ -130,6 +132,7 @@ int upload(phast_ctx* h) {
         h->sweep_mode = std::strcmp(e, "levels") == 0       ? 1
                         : std::strcmp(e, "persistent") == 0 ? 2
                         : std::strcmp(e, "staged") == 0     ? 3
+                        : std::strcmp(e, "pipe") == 0       ? 4
                                                             : 0;
     // level layouts default to one launch per level (the fastest schedule measured on them)
     if (!std::getenv("PHAST_SWEEP") && !h->L.lvl_off.empty()) h->sweep_mode = 1;
@@ -218,7 +221,7 @@ phast_ctx::Plan* get_plan(phast_ctx* h, uint32_t k) {
     const Layout& L = h->L;
     SweepPlan& p = P.p;
     p.k = k;
-    p.variant = h->sweep_mode == 2 ? 0u : h->sweep_mode == 3 ? 1u : 2u;
+    p.variant = h->sweep_mode == 2 ? 0u : h->sweep_mode == 3 ? 1u : h->sweep_mode == 4 && k >= 4 ? 3u : 2u;
     int occ = std::min(sweep_blocks_per_sm(k, false, p.variant), sweep_blocks_per_sm(k, true, p.variant));
     p.grid = (uint32_t)std::max(1, occ * num_sms());
     p.err = h->g.err;
@@ -241,10 +244,17 @@ phast_ctx::Plan* get_plan(phast_ctx* h, uint32_t k) {
         P.ok = true;
         return &P;
     }
-    const uint32_t CV = chunk_cap_for(h->L, k, p.grid);
+    uint32_t CV = chunk_cap_for(h->L, k, p.grid), cap_arcs = 0, lag = 1;
+    if (p.variant == 3) {   // pipelined: chunks bounded by the stage buffer, dependencies two iterations back
+        uint32_t gv = 0;
+        sweep_pipe_geometry(k, &gv, &cap_arcs);
+        const uint32_t vpp = sweep_pass_vertices(k);
+        CV = L.mode == LAYOUT_WAVEFRONT ? std::max(vpp, std::min(gv, L.delta / (3 * p.grid) / vpp * vpp)) : gv;
+        lag = 2;
+    }
     p.chunk_cap = CV;
     ChunkPlan cp;
-    if (plan_chunks(L, CV, p.grid, cp)) return nullptr;
+    if (plan_chunks(L, CV, p.grid, cp, cap_arcs, lag)) return nullptr;
     p.nchunks = cp.slots;
     p.iters = (cp.slots + p.grid - 1) / p.grid;
     const std::vector<uint32_t>& cv = cp.slot_v;
@@ -252,6 +262,22 @@ phast_ctx::Plan* get_plan(phast_ctx* h, uint32_t k) {
     uint32_t *a, *b, *w;
     if (dmalloc(&a, cv.size()) || dmalloc(&b, dep.size()) || dmalloc(&w, p.iters)) return nullptr;
     p.chunk_v = a; p.chunk_dep = b; p.wave_done = w;
+    if (p.variant == 3) {
+        std::vector<uint32_t> info((size_t)cp.slots * 4);
+        for (uint32_t j = 0; j < cp.slots; j++) {
+            info[4 * (size_t)j + 0] = cv[j];
+            info[4 * (size_t)j + 1] = cv[j + 1];
+            info[4 * (size_t)j + 2] = L.dn_first[cv[j]];
+            info[4 * (size_t)j + 3] = L.dn_first[cv[j + 1]];
+        }
+        uint32_t* pi;
+        if (dmalloc(&pi, info.size())) return nullptr;
+        p.pinfo = reinterpret_cast<const uint4*>(pi);
+        if (cudaMemcpy(pi, info.data(), info.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess) {
+            cudaGetLastError();
+            return nullptr;
+        }
+    }
     if (cudaMemcpy(a, cv.data(), cv.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess ||
         cudaMemcpy(b, dep.data(), dep.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess ||
         cudaMemset(w, 0, (size_t)p.iters * 4) != cudaSuccess) {

@@ -611,6 +611,195 @@ int warp_occupancy() {
     return b > 0 ? b : 1;
 }
 
+// ------------------------------------------------------------------ a3+a4 pipelined gather (variant 3)
+// CTA chunks on the wavefront layout with a one-chunk lookahead: while chunk c is
+// reduced from shared memory, the tail rows of the CTA's next chunk are already in
+// flight into the other shared-memory stage (cp.async.cg, 16 B per lane, no register
+// staging).  A chunk's dependencies are at least two iterations back (plan lag 2),
+// so its gathers can be issued one iteration early.  Two CTA barriers per chunk.
+constexpr uint32_t PIPE_STAGE_BYTES = 32768;   // tail rows of one chunk
+
+__device__ __forceinline__ void cp_async16(void* smem, const void* gmem) {
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(smem_u32(smem)), "l"(gmem) : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+__device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_group 0;" ::: "memory"); }
+
+template <int K>
+struct PipeGeom {
+    static constexpr uint32_t G = K / 4;                          // lanes (16 B each) per row
+    static constexpr uint32_t AMAX = PIPE_STAGE_BYTES / (K * 4);  // staged arcs per chunk
+    static constexpr uint32_t VPP = SWEEP_THREADS / G;
+    static constexpr uint32_t CV = (VPP * 4 < AMAX / 2 ? VPP * 4 : AMAX / 2) < VPP ? VPP
+                                   : (VPP * 4 < AMAX / 2 ? VPP * 4 : AMAX / 2);
+};
+
+template <int K, bool DIAM>
+__global__ void __launch_bounds__(SWEEP_THREADS, 3) sweep_pipe_kernel(const uint32_t* __restrict__ first,
+                                                                      const uint2* __restrict__ arcs,
+                                                                      uint32_t* __restrict__ d,
+                                                                      const uint32_t* __restrict__ flags,
+                                                                      const uint32_t* __restrict__ tail_bits,
+                                                                      SweepPlan p, uint32_t epoch,
+                                                                      uint32_t* __restrict__ diam) {
+    static_assert(K >= 4 && K % 4 == 0, "pipelined sweep needs 16-byte rows");
+    using Geo = PipeGeom<K>;
+    constexpr uint32_t G = Geo::G, AMAX = Geo::AMAX, VPP = Geo::VPP, CV = Geo::CV;
+    extern __shared__ __align__(16) uint8_t pipe_smem[];
+    uint4* rows = reinterpret_cast<uint4*>(pipe_smem);                                  // [2][AMAX*G]
+    uint2* sarc = reinterpret_cast<uint2*>(pipe_smem + 2 * PIPE_STAGE_BYTES);           // [2][AMAX]
+    uint32_t* sfirst = reinterpret_cast<uint32_t*>(sarc + 2 * AMAX);                   // [2][CV+1]
+    __shared__ uint4 sinfo[2];
+    __shared__ uint32_t s_known;
+    const uint32_t grid = gridDim.x;
+    const uint32_t gl = threadIdx.x % G, grp = threadIdx.x / G;
+    uint32_t mx = 0;
+
+    // thread 0: wait until iteration dep-1 is complete on every CTA
+    auto wait_dep = [&](uint32_t c) {
+        const uint32_t dep = __ldg(&p.chunk_dep[c]);
+        if (dep > s_known) {
+            const uint32_t w = dep - 1;
+            const uint32_t need = epoch * min(grid, p.nchunks - w * grid);
+            uint32_t ns = 32;
+            const uint64_t t0 = globaltimer_ns();
+            while (ld_acquire_gpu(&p.wave_done[w]) < need) {
+                __nanosleep(ns);
+                ns = min(ns * 2, 256u);
+                if (globaltimer_ns() - t0 > 4000000000ull) { atomicOr(p.err, 2u); break; }
+            }
+            s_known = dep;
+        }
+    };
+    // all threads: offsets and arcs of the chunk described by sinfo[b] into stage b
+    auto stage = [&](uint32_t b) {
+        const uint4 in = sinfo[b];
+        for (uint32_t i = threadIdx.x; i <= in.y - in.x; i += SWEEP_THREADS) sfirst[b * (CV + 1) + i] = __ldg(&first[in.x + i]);
+        if (in.w - in.z <= AMAX)
+            for (uint32_t i = threadIdx.x; i < in.w - in.z; i += SWEEP_THREADS) sarc[b * AMAX + i] = __ldg(&arcs[in.z + i]);
+    };
+    // all threads: 16-byte cp.async of every tail row slice of stage b's chunk
+    auto gather = [&](uint32_t b) {
+        const uint4 in = sinfo[b];
+        const uint32_t na = in.w - in.z;
+        if (na <= AMAX) {
+            for (uint32_t i = threadIdx.x; i < na * G; i += SWEEP_THREADS) {
+                const uint32_t a = i / G, part = i % G;
+                const uint32_t t = sarc[b * AMAX + a].x;
+                cp_async16(&rows[(size_t)b * AMAX * G + i], reinterpret_cast<const uint4*>(d + (size_t)t * K) + part);
+            }
+        }
+        cp_async_commit();
+    };
+
+    if (threadIdx.x == 0) s_known = 0;
+    uint32_t c = blockIdx.x;
+    if (c < p.nchunks) {
+        if (threadIdx.x == 0) sinfo[0] = __ldg(&p.pinfo[c]);
+        __syncthreads();
+        stage(0);
+        if (threadIdx.x == 0) { wait_dep(c); __threadfence(); }
+        __syncthreads();
+        gather(0);
+    }
+    uint4 nxt = make_uint4(0, 0, 0, 0);
+    if (threadIdx.x == 0 && c + grid < p.nchunks) nxt = __ldg(&p.pinfo[c + grid]);
+    uint32_t it = 0;
+    for (; c < p.nchunks; c += grid, it++) {
+        const uint32_t b = it & 1u;
+        const uint32_t cn = c + grid;
+        if (threadIdx.x == 0 && cn < p.nchunks) {
+            sinfo[b ^ 1u] = nxt;
+            if (cn + grid < p.nchunks) nxt = __ldg(&p.pinfo[cn + grid]);   // one more iteration ahead
+        }
+        __syncthreads();                                                       // [A]
+        if (threadIdx.x == 0 && it > 0) {                                      // chunk c-grid fully written
+            __threadfence();
+            atomicAdd(&p.wave_done[it - 1], 1u);
+        }
+        if (cn < p.nchunks) stage(b ^ 1u);
+        if (threadIdx.x == 0 && cn < p.nchunks) { wait_dep(cn); __threadfence(); }
+        cp_async_wait_all();                                                   // my slices of chunk c
+        __syncthreads();                                                       // [B]
+        if (cn < p.nchunks) gather(b ^ 1u);                                    // lookahead: chunk cn in flight
+        const uint4 in = sinfo[b];
+        const bool staged = in.w - in.z <= AMAX;
+        const uint32_t* fb = sfirst + b * (CV + 1);
+        for (uint32_t base = in.x; base < in.y; base += VPP) {
+            const uint32_t v = base + grp;
+            if (v >= in.y) break;
+            uint4 acc = make_uint4(INF, INF, INF, INF);
+            if ((__ldg(&flags[v >> 5]) >> (v & 31)) & 1u)
+                acc = __ldcg(reinterpret_cast<const uint4*>(d + (size_t)v * K) + gl);
+            const uint32_t e0 = fb[v - in.x], e1 = fb[v - in.x + 1];
+            if (staged) {
+                for (uint32_t e = e0; e < e1; e++) {
+                    const uint32_t a = e - in.z;
+                    acc = relax(acc, rows[(size_t)b * AMAX * G + a * G + gl], sarc[b * AMAX + a].y);
+                }
+            } else {
+                for (uint32_t e = e0; e < e1; e++) {
+                    const uint2 a = __ldg(&arcs[e]);
+                    acc = relax(acc, __ldcg(reinterpret_cast<const uint4*>(d + (size_t)a.x * K) + gl), a.y);
+                }
+            }
+            const bool is_tail = (__ldg(&tail_bits[v >> 5]) >> (v & 31)) & 1u;
+            if (!DIAM || is_tail) {
+                uint4* q = reinterpret_cast<uint4*>(d + (size_t)v * K) + gl;
+                if (is_tail) *q = acc; else st_stream(q, acc);
+            }
+            if constexpr (DIAM) mx = max(mx, fmax_of(acc));
+        }
+    }
+    __syncthreads();
+    if (threadIdx.x == 0 && it > 0) {
+        __threadfence();
+        atomicAdd(&p.wave_done[it - 1], 1u);
+    }
+    cp_async_wait_all();
+    if constexpr (DIAM) {
+        __shared__ uint32_t wmax[SWEEP_THREADS / 32];
+        mx = __reduce_max_sync(0xFFFFFFFFu, mx);
+        if ((threadIdx.x & 31) == 0) wmax[threadIdx.x >> 5] = mx;
+        __syncthreads();
+        if (threadIdx.x < 32) {
+            uint32_t w = threadIdx.x < SWEEP_THREADS / 32 ? wmax[threadIdx.x] : 0u;
+            w = __reduce_max_sync(0xFFFFFFFFu, w);
+            if (threadIdx.x == 0 && w) atomicMax(diam, w);
+        }
+    }
+}
+
+template <int K>
+size_t pipe_smem_bytes() {
+    using Geo = PipeGeom<K>;
+    return 2 * PIPE_STAGE_BYTES + 2 * Geo::AMAX * sizeof(uint2) + 2 * (Geo::CV + 1) * sizeof(uint32_t);
+}
+
+template <int K, bool DIAM>
+int pipe_occupancy() {
+    if constexpr (K < 4) {
+        return 0;
+    } else {
+        static bool attr = false;
+        if (!attr) {
+            if (cudaFuncSetAttribute(sweep_pipe_kernel<K, DIAM>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                     (int)pipe_smem_bytes<K>()) != cudaSuccess) {
+                cudaGetLastError();
+                return 0;
+            }
+            attr = true;
+        }
+        int b = 0;
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, sweep_pipe_kernel<K, DIAM>, SWEEP_THREADS,
+                                                          pipe_smem_bytes<K>()) != cudaSuccess) {
+            cudaGetLastError();
+            return 0;
+        }
+        return b;
+    }
+}
+
 template <int K, bool DIAM, bool STAGE>
 int persistent_occupancy() {
     int b = 0;
@@ -638,6 +827,19 @@ cudaError_t persistent_k2(const DevImage& g, const SweepPlan& p, uint32_t epoch,
 template <int K>
 cudaError_t persistent_k(const DevImage& g, const SweepPlan& p, uint32_t epoch, uint32_t* dist, uint32_t* diam,
                          cudaStream_t st) {
+    if constexpr (K >= 4) {
+        if (p.variant == 3) {
+            const size_t smem = pipe_smem_bytes<K>();
+            if (diam)
+                sweep_pipe_kernel<K, true><<<p.grid, SWEEP_THREADS, smem, st>>>(g.dn_first, g.dn_arc, dist, g.flags,
+                                                                                 g.tail_bits, p, epoch, diam);
+            else
+                sweep_pipe_kernel<K, false><<<p.grid, SWEEP_THREADS, smem, st>>>(g.dn_first, g.dn_arc, dist, g.flags,
+                                                                                  g.tail_bits, p, epoch, nullptr);
+            g_launches++;
+            return cudaGetLastError();
+        }
+    }
     if (p.variant == 2) {
         if (diam)
             sweep_warp_kernel<K, true><<<p.grid, SWEEP_THREADS, 0, st>>>(g.dn_first, g.dn_arc, dist, g.flags,
@@ -714,6 +916,17 @@ cudaError_t launch_sweep_level(const DevImage& g, uint32_t k, uint32_t vbeg, uin
 #undef CALL_SW
 }
 
+void sweep_pipe_geometry(uint32_t k, uint32_t* cap_vertices, uint32_t* cap_arcs) {
+    switch (k) {
+        case 4: *cap_vertices = PipeGeom<4>::CV; *cap_arcs = PipeGeom<4>::AMAX; return;
+        case 8: *cap_vertices = PipeGeom<8>::CV; *cap_arcs = PipeGeom<8>::AMAX; return;
+        case 16: *cap_vertices = PipeGeom<16>::CV; *cap_arcs = PipeGeom<16>::AMAX; return;
+        case 32: *cap_vertices = PipeGeom<32>::CV; *cap_arcs = PipeGeom<32>::AMAX; return;
+        case 64: *cap_vertices = PipeGeom<64>::CV; *cap_arcs = PipeGeom<64>::AMAX; return;
+        default: *cap_vertices = 0; *cap_arcs = 0; return;
+    }
+}
+
 uint32_t sweep_warp_chunk_vertices(uint32_t k) { return (32 / (k >= 4 ? k / 4 : 1)) * WARP_PASSES; }
 
 uint32_t sweep_pass_vertices(uint32_t k) { return SWEEP_THREADS / (k >= 4 ? k / 4 : 1); }
@@ -725,7 +938,8 @@ uint32_t sweep_chunk_vertices(uint32_t k) {
 
 int sweep_blocks_per_sm(uint32_t k, bool diam, uint32_t variant) {
 #define OCC(K)                                                                                               \
-    (variant == 2 ? (diam ? warp_occupancy<K, true>() : warp_occupancy<K, false>()) :                         \
+    (variant == 3 ? (diam ? pipe_occupancy<K, true>() : pipe_occupancy<K, false>()) :                         \
+     variant == 2 ? (diam ? warp_occupancy<K, true>() : warp_occupancy<K, false>()) :                         \
      variant == 1 ? (diam ? persistent_occupancy<K, true, true>() : persistent_occupancy<K, false, true>())   \
                   : (diam ? persistent_occupancy<K, true, false>() : persistent_occupancy<K, false, false>()))
     switch (k) {

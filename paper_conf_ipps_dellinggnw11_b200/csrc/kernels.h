@@ -47,7 +47,9 @@ cudaError_t launch_sweep_level(const DevImage& g, uint32_t k, uint32_t vbeg, uin
 // chunk_dep[c] - 1 (0 = no dependency).
 struct SweepPlan {
     uint32_t k = 0, nchunks = 0, grid = 0, iters = 0, chunk_cap = 0;
-    uint32_t variant = 2;                   // 2: warp dataflow; 1: CTA waves + bulk-staged arcs; 0: CTA waves
+    uint32_t variant = 2;   // 3: pipelined gather; 2: warp dataflow; 1: CTA waves + bulk-staged arcs; 0: CTA waves
+    // variant 3 (pipelined gather): per slot {vbeg, vend, e0 = first[vbeg], e1 = first[vend]}
+    const uint4* pinfo = nullptr;
     // variant 2 (warp dataflow)
     uint32_t workers = 0;                   // warps in the grid
     const uint4* wmeta = nullptr;           // [nchunks] {vbeg, vend, dbeg, dend}
@@ -62,7 +64,9 @@ struct SweepPlan {
 uint32_t sweep_chunk_vertices(uint32_t k);   // max vertices per chunk
 uint32_t sweep_pass_vertices(uint32_t k);    // vertices per pass of a CTA
 uint32_t sweep_warp_chunk_vertices(uint32_t k);
-constexpr uint32_t SWEEP_WARPS = 8;               // warps per CTA of the persistent sweeps   // vertices per chunk of one warp (variant 2)
+constexpr uint32_t SWEEP_WARPS = 8;               // warps per CTA of the persistent sweeps
+// variant 3: max vertices and arcs per chunk for k (k >= 4; 0 otherwise)
+void sweep_pipe_geometry(uint32_t k, uint32_t* cap_vertices, uint32_t* cap_arcs);   // vertices per chunk of one warp (variant 2)
 int sweep_blocks_per_sm(uint32_t k, bool diam, uint32_t variant);
 // a3 + a4 in ONE launch: dataflow over levels through the completion counters
 // (epoch = number of launches of this plan so far, 1-based).

@@ -212,14 +212,15 @@ int plan_warp_chunks(const Layout& L, uint32_t cap, uint32_t workers, WarpPlan& 
     return 0;
 }
 
-int plan_chunks(const Layout& L, uint32_t cap, uint32_t grid, ChunkPlan& P) {
+int plan_chunks(const Layout& L, uint32_t cap, uint32_t grid, ChunkPlan& P, uint32_t cap_arcs, uint32_t lag) {
     const uint32_t n = (uint32_t)L.perm.size();
-    if (cap == 0 || grid == 0) return kEinternal;
+    if (cap == 0 || grid == 0 || lag == 0) return kEinternal;
     // 1. chunk boundaries and each chunk's latest tail chunk (unpadded numbering)
     std::vector<uint32_t> cb{0}, chunk_of(n);
     uint32_t s = 0;
     for (uint32_t v = 0; v < n; v++) {
         bool cut = (v - s == cap);
+        if (!cut && v > s && cap_arcs && L.dn_first[v + 1] - L.dn_first[s] > cap_arcs) cut = true;
         if (!cut && v > s)
             for (uint32_t e = L.dn_first[v]; e < L.dn_first[v + 1]; e++)
                 if (L.dn_arc[e].x >= s) { cut = true; break; }
@@ -228,7 +229,7 @@ int plan_chunks(const Layout& L, uint32_t cap, uint32_t grid, ChunkPlan& P) {
     }
     cb.push_back(n);
     const uint32_t nch = (uint32_t)cb.size() - 1;
-    // 2. slots with padding so that a dependency is always in an earlier iteration
+    // 2. slots with padding so that a dependency is always >= lag iterations earlier
     std::vector<uint32_t> slot(nch);
     P.slot_v.clear();
     P.dep.clear();
@@ -240,7 +241,7 @@ int plan_chunks(const Layout& L, uint32_t cap, uint32_t grid, ChunkPlan& P) {
             d = std::max<int64_t>(d, chunk_of[L.dn_arc[e].x]);
         if (d >= (int64_t)c) return kEinternal;
         uint64_t j = next;
-        if (d >= 0 && slot[d] / grid == j / grid) j = (j / grid + 1) * grid;
+        if (d >= 0 && slot[d] / grid + lag > j / grid) j = (uint64_t)(slot[d] / grid + lag) * grid;
         if (j > 0xFFFFFFF0ull) return kErange;
         for (uint64_t q = next; q < j; q++) {              // pads: empty ranges
             P.slot_v.push_back(cb[c]);

@@ -49,7 +49,10 @@ struct ChunkPlan {
     std::vector<uint32_t> dep;      // [slots]
     uint32_t chunks = 0, slots = 0, pads = 0;
 };
-int plan_chunks(const Layout& L, uint32_t cap, uint32_t grid, ChunkPlan& out);
+// cap_arcs (0 = none): also cut before a chunk's G-down arcs exceed cap_arcs;
+// lag: every dependency is at least `lag` iterations earlier.
+int plan_chunks(const Layout& L, uint32_t cap, uint32_t grid, ChunkPlan& out, uint32_t cap_arcs = 0,
+                uint32_t lag = 1);
 
 // Warp-granular dataflow schedule (default sweep): chunks of consecutive ids (at most
 // cap vertices, cut at intra-chunk dependencies), chunk c handled by worker (warp)
