@@ -45,6 +45,11 @@ struct phast_ctx {
     // 0 = warp dataflow (default), 1 = one launch per level, 2 = CTA waves, 3 = CTA waves + bulk-staged
     // arcs, 4 = pipelined gather (k >= 4; else warp dataflow)
     int sweep_mode = 0;
+    // upward searches run on a side stream, one seed slot ahead of the sweep
+    cudaStream_t side = nullptr;
+    cudaEvent_t up_done[SEED_SLOTS] = {};
+    cudaEvent_t slot_free[SEED_SLOTS] = {};
+    uint32_t slot_next = 0;
     // stage timing (phast_timing)
     bool timing = false;
     std::vector<cudaEvent_t> ev;   // 3 per recorded batch
@@ -105,6 +110,13 @@ void free_device(phast_ctx* h) {
     for (cudaEvent_t e : h->ev) cudaEventDestroy(e);
     h->ev.clear();
     h->ev_used = 0;
+    for (uint32_t s = 0; s < SEED_SLOTS; s++) {
+        if (h->up_done[s]) cudaEventDestroy(h->up_done[s]);
+        if (h->slot_free[s]) cudaEventDestroy(h->slot_free[s]);
+        h->up_done[s] = h->slot_free[s] = nullptr;
+    }
+    if (h->side) cudaStreamDestroy(h->side);
+    h->side = nullptr;
     cudaFree((void*)h->g.dn_first); cudaFree((void*)h->g.dn_arc);
     cudaFree((void*)h->g.up_first); cudaFree((void*)h->g.up_arc);
     cudaFree(h->g.flags); cudaFree((void*)h->g.tail_bits);
@@ -156,8 +168,9 @@ int upload(phast_ctx* h) {
     if ((rc = dmalloc(&dnf, L.dn_first.size() + 4)) || (rc = dmalloc(&dna, L.dn_arc.size() + 2)) ||
         (rc = dmalloc(&upf, L.up_first.size())) || (rc = dmalloc(&upa, L.up_arc.size())) ||
         (rc = dmalloc(&g.flags, nw)) || (rc = dmalloc(&tb, nw)) ||
-        (rc = dmalloc(&g.seed_v, (size_t)KMAX * g.seed_cap)) || (rc = dmalloc(&g.seed_d, (size_t)KMAX * g.seed_cap)) ||
-        (rc = dmalloc(&g.seed_cnt, KMAX)) || (rc = dmalloc(&g.gscratch, (size_t)KMAX * g.seed_cap * 5)) ||
+        (rc = dmalloc(&g.seed_v, (size_t)SEED_SLOTS * KMAX * g.seed_cap)) ||
+        (rc = dmalloc(&g.seed_d, (size_t)SEED_SLOTS * KMAX * g.seed_cap)) ||
+        (rc = dmalloc(&g.seed_cnt, SEED_SLOTS * KMAX)) || (rc = dmalloc(&g.gscratch, (size_t)KMAX * g.seed_cap * 5)) ||
         (rc = dmalloc(&g.err, 1))) {
         g.dn_first = dnf; g.dn_arc = dna; g.up_first = upf; g.up_arc = upa; g.tail_bits = tb;
         free_device(h);
@@ -172,7 +185,12 @@ int upload(phast_ctx* h) {
               cudaMemcpy(upa, L.up_arc.data(), L.up_arc.size() * 8, cudaMemcpyHostToDevice) == cudaSuccess &&
               cudaMemcpy(tb, h->tail_bits.data(), nw * 4, cudaMemcpyHostToDevice) == cudaSuccess &&
               cudaMemset(g.flags, 0, nw * 4) == cudaSuccess && cudaMemset(g.err, 0, 4) == cudaSuccess &&
-              cudaMemset(g.seed_cnt, 0, KMAX * 4) == cudaSuccess && cudaDeviceSynchronize() == cudaSuccess;
+              cudaMemset(g.seed_cnt, 0, SEED_SLOTS * KMAX * 4) == cudaSuccess &&
+              cudaStreamCreateWithFlags(&h->side, cudaStreamNonBlocking) == cudaSuccess &&
+              cudaDeviceSynchronize() == cudaSuccess;
+    for (uint32_t s = 0; ok && s < SEED_SLOTS; s++)
+        ok = cudaEventCreateWithFlags(&h->up_done[s], cudaEventDisableTiming) == cudaSuccess &&
+             cudaEventCreateWithFlags(&h->slot_free[s], cudaEventDisableTiming) == cudaSuccess;
     if (!ok) { cudaGetLastError(); free_device(h); return PHAST_ECUDA; }
     return PHAST_OK;
 }
@@ -309,8 +327,14 @@ int run_query(phast_ctx* h, const Sources& S, uint32_t k, uint32_t* dist, uint32
         if (!e0 || !e1 || !e2) return PHAST_ECUDA;
         cudaEventRecord(e0, st);
     }
-    if (launch_upward(h->g, S, k, dist, st) != cudaSuccess) return PHAST_ECUDA;
-    if (launch_scatter(h->g, k, dist, st) != cudaSuccess) return PHAST_ECUDA;
+    // a1 on the side stream (overlaps the previous batch's sweep), a2 on the caller's stream
+    const uint32_t slot = h->slot_next;
+    h->slot_next = (h->slot_next + 1) % SEED_SLOTS;
+    if (cudaStreamWaitEvent(h->side, h->slot_free[slot], 0) != cudaSuccess) return PHAST_ECUDA;
+    if (launch_upward(h->g, S, k, slot, h->side) != cudaSuccess) return PHAST_ECUDA;
+    if (cudaEventRecord(h->up_done[slot], h->side) != cudaSuccess) return PHAST_ECUDA;
+    if (cudaStreamWaitEvent(st, h->up_done[slot], 0) != cudaSuccess) return PHAST_ECUDA;
+    if (launch_seed(h->g, k, slot, dist, st) != cudaSuccess) return PHAST_ECUDA;
     if (e1) cudaEventRecord(e1, st);
     phast_ctx::Plan* plan = h->sweep_mode != 1 ? get_plan(h, k) : nullptr;
     if (plan) {   // a3 + a4: one persistent launch, dataflow over chunk waves
@@ -332,7 +356,8 @@ int run_query(phast_ctx* h, const Sources& S, uint32_t k, uint32_t* dist, uint32
     } else {
         return PHAST_EINTERNAL;
     }
-    if (launch_clear_flags(h->g, k, st) != cudaSuccess) return PHAST_ECUDA;
+    if (launch_clear_flags(h->g, k, slot, st) != cudaSuccess) return PHAST_ECUDA;
+    if (cudaEventRecord(h->slot_free[slot], st) != cudaSuccess) return PHAST_ECUDA;   // seeds of `slot` consumed
     if (e2) cudaEventRecord(e2, st);
     return PHAST_OK;
 }
@@ -415,10 +440,16 @@ int phast_sync(phast_ctx* h, void* stream) {
     if (!h) return PHAST_EINVAL;
     if (h->device < 0) return PHAST_ESTATE;
     DeviceGuard dg(h->device);
-    if (cudaStreamSynchronize((cudaStream_t)stream) != cudaSuccess) { cudaGetLastError(); return PHAST_ECUDA; }
+    cudaError_t ce = cudaStreamSynchronize((cudaStream_t)stream);
+    if (ce != cudaSuccess) {
+        cudaGetLastError();
+        if (std::getenv("PHAST_VERBOSE")) std::fprintf(stderr, "phast_sync: %s\n", cudaGetErrorString(ce));
+        return PHAST_ECUDA;
+    }
     uint32_t err = 0;
     if (cudaMemcpy(&err, h->g.err, 4, cudaMemcpyDeviceToHost) != cudaSuccess) return PHAST_ECUDA;
     if (err) {
+        if (std::getenv("PHAST_VERBOSE")) std::fprintf(stderr, "phast_sync: device error word 0x%x\n", err);
         cudaMemset(h->g.err, 0, 4);
         return (err & 1u) ? PHAST_ERANGE : PHAST_ECUDA;   // bit 0: search-space overflow; bit 1: watchdog
     }

@@ -135,13 +135,16 @@ __device__ bool up_search(const uint32_t* __restrict__ up_first, const uint2* __
     return ok;
 }
 
-template <int K>
-__global__ void __launch_bounds__(UP_THREADS) upward_kernel(DevImage g, Sources src, uint32_t* __restrict__ dist) {
+// a1: search only; the search space goes to seed slot `slot` (the sweep of the
+// previous batch may still be running on the main stream: nothing here touches the
+// visited bits or the label rows).
+__global__ void __launch_bounds__(UP_THREADS) upward_kernel(DevImage g, Sources src, uint32_t slot) {
     extern __shared__ uint32_t smem[];
     __shared__ UpShared c;
     const uint32_t i = blockIdx.x;
     const uint32_t s = src.s[i];
     const uint32_t sc = g.smem_cap;
+    const size_t so = ((size_t)slot * KMAX + i) * g.seed_cap;
     UpTable t{smem, smem + sc, smem + 2 * sc, smem + 3 * sc, smem + 4 * sc, sc};
     bool ok = up_search(g.up_first, g.up_arc, s, t, c);
     if (!ok) {   // global-memory fallback with the per-source capacity
@@ -151,25 +154,33 @@ __global__ void __launch_bounds__(UP_THREADS) upward_kernel(DevImage g, Sources 
         t = gt;
         ok = up_search(g.up_first, g.up_arc, s, t, c);
         if (!ok) {
-            if (threadIdx.x == 0) { atomicOr(g.err, 1u); g.seed_cnt[i] = 0; }
+            if (threadIdx.x == 0) { atomicOr(g.err, 1u); g.seed_cnt[slot * KMAX + i] = 0; }
             return;
         }
     }
-    // emit the search space, set visited bits
-    uint32_t* sv = g.seed_v + (size_t)i * g.seed_cap;
-    uint32_t* sd = g.seed_d + (size_t)i * g.seed_cap;
-    for (uint32_t slot = threadIdx.x; slot < t.cap; slot += blockDim.x) {
-        uint32_t v = t.keys[slot];
+    uint32_t* sv = g.seed_v + so;
+    uint32_t* sd = g.seed_d + so;
+    for (uint32_t e = threadIdx.x; e < t.cap; e += blockDim.x) {
+        uint32_t v = t.keys[e];
         if (v == EMPTY) continue;
         uint32_t pos = atomicAdd(&c.cnt, 1u);
         sv[pos] = v;
-        sd[pos] = t.vals[slot];
-        atomicOr(&g.flags[v >> 5], 1u << (v & 31));
+        sd[pos] = t.vals[e];
     }
     __syncthreads();
-    const uint32_t cnt = c.cnt;
-    if (threadIdx.x == 0) g.seed_cnt[i] = cnt;
-    // reset the rows of the search space to INF (phase 1 of a2)
+    if (threadIdx.x == 0) g.seed_cnt[slot * KMAX + i] = c.cnt;
+}
+
+// a2 phase 1: visited bits of the search space, and its rows reset to INF
+template <int K>
+__global__ void seed_rows_kernel(DevImage g, uint32_t slot, uint32_t* __restrict__ dist) {
+    const uint32_t i = blockIdx.x;
+    const uint32_t cnt = g.seed_cnt[slot * KMAX + i];
+    const uint32_t* sv = g.seed_v + ((size_t)slot * KMAX + i) * g.seed_cap;
+    for (uint32_t j = threadIdx.x; j < cnt; j += blockDim.x) {
+        const uint32_t v = sv[j];
+        atomicOr(&g.flags[v >> 5], 1u << (v & 31));
+    }
     if constexpr (K % 4 == 0) {
         constexpr uint32_t W = K / 4;
         const uint4 inf4 = make_uint4(INF, INF, INF, INF);
@@ -180,18 +191,19 @@ __global__ void __launch_bounds__(UP_THREADS) upward_kernel(DevImage g, Sources 
     }
 }
 
-__global__ void scatter_kernel(DevImage g, uint32_t k, uint32_t* __restrict__ dist) {
+// a2 phase 2 (after every reset of phase 1): the labels
+__global__ void scatter_kernel(DevImage g, uint32_t slot, uint32_t k, uint32_t* __restrict__ dist) {
     const uint32_t i = blockIdx.x;
-    const uint32_t cnt = g.seed_cnt[i];
-    const uint32_t* sv = g.seed_v + (size_t)i * g.seed_cap;
-    const uint32_t* sd = g.seed_d + (size_t)i * g.seed_cap;
+    const uint32_t cnt = g.seed_cnt[slot * KMAX + i];
+    const uint32_t* sv = g.seed_v + ((size_t)slot * KMAX + i) * g.seed_cap;
+    const uint32_t* sd = g.seed_d + ((size_t)slot * KMAX + i) * g.seed_cap;
     for (uint32_t j = threadIdx.x; j < cnt; j += blockDim.x) dist[(size_t)sv[j] * k + i] = sd[j];
 }
 
-__global__ void clear_flags_kernel(DevImage g) {
+__global__ void clear_flags_kernel(DevImage g, uint32_t slot) {
     const uint32_t i = blockIdx.x;
-    const uint32_t cnt = g.seed_cnt[i];
-    const uint32_t* sv = g.seed_v + (size_t)i * g.seed_cap;
+    const uint32_t cnt = g.seed_cnt[slot * KMAX + i];
+    const uint32_t* sv = g.seed_v + ((size_t)slot * KMAX + i) * g.seed_cap;
     for (uint32_t j = threadIdx.x; j < cnt; j += blockDim.x) g.flags[sv[j] >> 5] = 0u;
 }
 
@@ -649,7 +661,7 @@ __global__ void __launch_bounds__(SWEEP_THREADS, 3) sweep_pipe_kernel(const uint
     uint4* rows = reinterpret_cast<uint4*>(pipe_smem);                                  // [2][AMAX*G]
     uint2* sarc = reinterpret_cast<uint2*>(pipe_smem + 2 * PIPE_STAGE_BYTES);           // [2][AMAX]
     uint32_t* sfirst = reinterpret_cast<uint32_t*>(sarc + 2 * AMAX);                   // [2][CV+1]
-    __shared__ uint4 sinfo[2];
+    __shared__ uint4 sinfo[3];   // chunk descriptors, indexed by iteration % 3 (thread 0 runs <1 iteration ahead)
     __shared__ uint32_t s_known;
     const uint32_t grid = gridDim.x;
     const uint32_t gl = threadIdx.x % G, grp = threadIdx.x / G;
@@ -672,15 +684,15 @@ __global__ void __launch_bounds__(SWEEP_THREADS, 3) sweep_pipe_kernel(const uint
         }
     };
     // all threads: offsets and arcs of the chunk described by sinfo[b] into stage b
-    auto stage = [&](uint32_t b) {
-        const uint4 in = sinfo[b];
+    auto stage = [&](uint32_t b, uint32_t si) {
+        const uint4 in = sinfo[si];
         for (uint32_t i = threadIdx.x; i <= in.y - in.x; i += SWEEP_THREADS) sfirst[b * (CV + 1) + i] = __ldg(&first[in.x + i]);
         if (in.w - in.z <= AMAX)
             for (uint32_t i = threadIdx.x; i < in.w - in.z; i += SWEEP_THREADS) sarc[b * AMAX + i] = __ldg(&arcs[in.z + i]);
     };
     // all threads: 16-byte cp.async of every tail row slice of stage b's chunk
-    auto gather = [&](uint32_t b) {
-        const uint4 in = sinfo[b];
+    auto gather = [&](uint32_t b, uint32_t si) {
+        const uint4 in = sinfo[si];
         const uint32_t na = in.w - in.z;
         if (na <= AMAX) {
             for (uint32_t i = threadIdx.x; i < na * G; i += SWEEP_THREADS) {
@@ -697,19 +709,20 @@ __global__ void __launch_bounds__(SWEEP_THREADS, 3) sweep_pipe_kernel(const uint
     if (c < p.nchunks) {
         if (threadIdx.x == 0) sinfo[0] = __ldg(&p.pinfo[c]);
         __syncthreads();
-        stage(0);
+        stage(0, 0);
         if (threadIdx.x == 0) { wait_dep(c); __threadfence(); }
         __syncthreads();
-        gather(0);
+        gather(0, 0);
     }
     uint4 nxt = make_uint4(0, 0, 0, 0);
     if (threadIdx.x == 0 && c + grid < p.nchunks) nxt = __ldg(&p.pinfo[c + grid]);
     uint32_t it = 0;
     for (; c < p.nchunks; c += grid, it++) {
         const uint32_t b = it & 1u;
+        const uint32_t si = it % 3u, sn = (it + 1) % 3u;
         const uint32_t cn = c + grid;
         if (threadIdx.x == 0 && cn < p.nchunks) {
-            sinfo[b ^ 1u] = nxt;
+            sinfo[sn] = nxt;
             if (cn + grid < p.nchunks) nxt = __ldg(&p.pinfo[cn + grid]);   // one more iteration ahead
         }
         __syncthreads();                                                       // [A]
@@ -717,12 +730,12 @@ __global__ void __launch_bounds__(SWEEP_THREADS, 3) sweep_pipe_kernel(const uint
             __threadfence();
             atomicAdd(&p.wave_done[it - 1], 1u);
         }
-        if (cn < p.nchunks) stage(b ^ 1u);
+        if (cn < p.nchunks) stage(b ^ 1u, sn);
         if (threadIdx.x == 0 && cn < p.nchunks) { wait_dep(cn); __threadfence(); }
         cp_async_wait_all();                                                   // my slices of chunk c
         __syncthreads();                                                       // [B]
-        if (cn < p.nchunks) gather(b ^ 1u);                                    // lookahead: chunk cn in flight
-        const uint4 in = sinfo[b];
+        if (cn < p.nchunks) gather(b ^ 1u, sn);                                // lookahead: chunk cn in flight
+        const uint4 in = sinfo[si];
         const bool staged = in.w - in.z <= AMAX;
         const uint32_t* fb = sfirst + b * (CV + 1);
         for (uint32_t base = in.x; base < in.y; base += VPP) {
@@ -854,17 +867,23 @@ cudaError_t persistent_k(const DevImage& g, const SweepPlan& p, uint32_t epoch, 
                           : persistent_k2<K, false>(g, p, epoch, dist, diam, st);
 }
 
-template <int K>
-cudaError_t upward_k(const DevImage& g, const Sources& src, uint32_t k, uint32_t* dist, cudaStream_t st) {
+cudaError_t upward_launch(const DevImage& g, const Sources& src, uint32_t k, uint32_t slot, cudaStream_t st) {
     static bool attr = false;
     size_t smem = 5 * (size_t)g.smem_cap * sizeof(uint32_t);
     if (!attr) {
-        cudaError_t e = cudaFuncSetAttribute(upward_kernel<K>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+        cudaError_t e = cudaFuncSetAttribute(upward_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                              (int)(5 * UP_SMEM_CAP * sizeof(uint32_t)));
         if (e != cudaSuccess) return e;
         attr = true;
     }
-    upward_kernel<K><<<k, UP_THREADS, smem, st>>>(g, src, dist);
+    upward_kernel<<<k, UP_THREADS, smem, st>>>(g, src, slot);
+    g_launches++;
+    return cudaGetLastError();
+}
+
+template <int K>
+cudaError_t seed_rows_k(const DevImage& g, uint32_t k, uint32_t slot, uint32_t* dist, cudaStream_t st) {
+    seed_rows_kernel<K><<<k, 256, 0, st>>>(g, slot, dist);
     g_launches++;
     return cudaGetLastError();
 }
@@ -897,14 +916,16 @@ __global__ void max_reduce_kernel(const uint32_t* __restrict__ in, uint32_t coun
         default: return cudaErrorInvalidValue; \
     }
 
-cudaError_t launch_upward(const DevImage& g, const Sources& src, uint32_t k, uint32_t* dist, cudaStream_t st) {
-#define CALL_UP(K) upward_k<K>(g, src, k, dist, st)
-    PHAST_K_SWITCH(k, CALL_UP)
-#undef CALL_UP
+cudaError_t launch_upward(const DevImage& g, const Sources& src, uint32_t k, uint32_t slot, cudaStream_t st) {
+    return upward_launch(g, src, k, slot, st);
 }
 
-cudaError_t launch_scatter(const DevImage& g, uint32_t k, uint32_t* dist, cudaStream_t st) {
-    scatter_kernel<<<k, 256, 0, st>>>(g, k, dist);
+cudaError_t launch_seed(const DevImage& g, uint32_t k, uint32_t slot, uint32_t* dist, cudaStream_t st) {
+#define CALL_SR(K) seed_rows_k<K>(g, k, slot, dist, st)
+    cudaError_t e = [&]() -> cudaError_t { PHAST_K_SWITCH(k, CALL_SR) }();
+#undef CALL_SR
+    if (e != cudaSuccess) return e;
+    scatter_kernel<<<k, 256, 0, st>>>(g, slot, k, dist);
     g_launches++;
     return cudaGetLastError();
 }
@@ -962,8 +983,8 @@ cudaError_t launch_sweep_persistent(const DevImage& g, const SweepPlan& p, uint3
 #undef CALL_PS
 }
 
-cudaError_t launch_clear_flags(const DevImage& g, uint32_t k, cudaStream_t st) {
-    clear_flags_kernel<<<k, 256, 0, st>>>(g);
+cudaError_t launch_clear_flags(const DevImage& g, uint32_t k, uint32_t slot, cudaStream_t st) {
+    clear_flags_kernel<<<k, 256, 0, st>>>(g, slot);
     g_launches++;
     return cudaGetLastError();
 }

@@ -7,6 +7,7 @@ namespace phast {
 
 constexpr uint32_t INF = 0xFFFFFFFFu;
 constexpr uint32_t KMAX = 64;
+constexpr uint32_t SEED_SLOTS = 2;
 
 // Device image of the hierarchy + per-handle scratch (all device pointers).
 struct DevImage {
@@ -17,9 +18,9 @@ struct DevImage {
     const uint2* up_arc = nullptr;       // [m_up]   {head, len}
     uint32_t* flags = nullptr;           // [ceil(n/32)] visited bits (§IV-C), zero between calls
     const uint32_t* tail_bits = nullptr; // [ceil(n/32)] bit v: v is the tail of some G-down arc
-    uint32_t* seed_v = nullptr;          // [KMAX * seed_cap] upward search spaces: vertex
-    uint32_t* seed_d = nullptr;          // [KMAX * seed_cap] upward search spaces: label
-    uint32_t* seed_cnt = nullptr;        // [KMAX]
+    uint32_t* seed_v = nullptr;          // [SEED_SLOTS][KMAX][seed_cap] upward search spaces: vertex
+    uint32_t* seed_d = nullptr;          // [SEED_SLOTS][KMAX][seed_cap] upward search spaces: label
+    uint32_t* seed_cnt = nullptr;        // [SEED_SLOTS][KMAX]
     uint32_t* gscratch = nullptr;        // [KMAX * seed_cap * 5] global-memory fallback tables
     uint32_t* err = nullptr;             // [1] sticky device error word
     uint32_t seed_cap = 0;               // entries per source (power of two)
@@ -30,12 +31,12 @@ struct Sources {
     uint32_t s[KMAX];  // internal ids, passed by value in the kernel parameter space
 };
 
-// a1 + a2 (phase 1): one CTA per source; exact G-up labels; writes the search space
-// to seed_*, sets the visited bits, and resets the rows of the search space to INF.
-cudaError_t launch_upward(const DevImage& g, const Sources& src, uint32_t k, uint32_t* dist,
-                          cudaStream_t st);
-// a2 (phase 2): dist[v*k + i] = label_i(v) for every search-space entry of source i.
-cudaError_t launch_scatter(const DevImage& g, uint32_t k, uint32_t* dist, cudaStream_t st);
+// a1: one CTA per source; exact G-up labels; the search space goes to seed slot `slot`
+// (SEED_SLOTS slots, so the next batch's searches can run beside this batch's sweep).
+cudaError_t launch_upward(const DevImage& g, const Sources& src, uint32_t k, uint32_t slot, cudaStream_t st);
+// a2: visited bits + rows of the search spaces reset to INF, then (second launch, so
+// that every reset precedes every label) dist[v*k + i] = label_i(v).
+cudaError_t launch_seed(const DevImage& g, uint32_t k, uint32_t slot, uint32_t* dist, cudaStream_t st);
 // a3: one level [vbeg, vend) of the downward sweep; diam != nullptr fuses the max (a5);
 // store == false skips the row stores (diameter mode, level 0 rows are never read).
 cudaError_t launch_sweep_level(const DevImage& g, uint32_t k, uint32_t vbeg, uint32_t vend,
@@ -75,7 +76,7 @@ cudaError_t launch_sweep_persistent(const DevImage& g, const SweepPlan& p, uint3
 
 // after the sweep: clear the visited bits of every search-space vertex ("After
 // scanning v we unmark the vertex", §IV-C).
-cudaError_t launch_clear_flags(const DevImage& g, uint32_t k, cudaStream_t st);
+cudaError_t launch_clear_flags(const DevImage& g, uint32_t k, uint32_t slot, cudaStream_t st);
 // max of per-batch maxima (diameter)
 cudaError_t launch_max_reduce(const uint32_t* in, uint32_t count, uint32_t* out, cudaStream_t st);
 
