@@ -262,17 +262,43 @@ phast_ctx::Plan* get_plan(phast_ctx* h, uint32_t k) {
         P.ok = true;
         return &P;
     }
-    uint32_t CV = chunk_cap_for(h->L, k, p.grid), cap_arcs = 0, lag = 1;
-    if (p.variant == 3) {   // pipelined: chunks bounded by the stage buffer, dependencies two iterations back
-        uint32_t gv = 0;
+    if (p.variant == 3) {   // pipelined gather: CTA chunks, per-chunk completion flags, one-chunk lookahead
+        uint32_t gv = 0, cap_arcs = 0;
         sweep_pipe_geometry(k, &gv, &cap_arcs);
-        const uint32_t vpp = sweep_pass_vertices(k);
-        CV = L.mode == LAYOUT_WAVEFRONT ? std::max(vpp, std::min(gv, L.delta / (3 * p.grid) / vpp * vpp)) : gv;
-        lag = 2;
+        p.workers = p.grid;
+        p.chunk_cap = gv;
+        WarpPlan wp;
+        if (plan_warp_chunks(L, gv, p.workers, wp, cap_arcs)) return nullptr;
+        p.nchunks = wp.chunks;
+        std::vector<uint32_t> info((size_t)wp.chunks * 4);
+        for (uint32_t j = 0; j < wp.chunks; j++) {
+            const uint32_t vb = wp.meta[4 * (size_t)j], ve = wp.meta[4 * (size_t)j + 1];
+            info[4 * (size_t)j + 0] = vb;
+            info[4 * (size_t)j + 1] = ve;
+            info[4 * (size_t)j + 2] = L.dn_first[vb];
+            info[4 * (size_t)j + 3] = L.dn_first[ve];
+        }
+        uint32_t *a, *b, *w, *pi;
+        if (dmalloc(&a, wp.meta.size()) || dmalloc(&b, wp.deps.size()) || dmalloc(&w, wp.chunks) ||
+            dmalloc(&pi, info.size()))
+            return nullptr;
+        p.wmeta = reinterpret_cast<const uint4*>(a); p.wdeps = b; p.done = w;
+        p.pinfo = reinterpret_cast<const uint4*>(pi);
+        if (cudaMemcpy(a, wp.meta.data(), wp.meta.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess ||
+            (!wp.deps.empty() &&
+             cudaMemcpy(b, wp.deps.data(), wp.deps.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess) ||
+            cudaMemcpy(pi, info.data(), info.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess ||
+            cudaMemset(w, 0, (size_t)wp.chunks * 4) != cudaSuccess) {
+            cudaGetLastError();
+            return nullptr;
+        }
+        P.ok = true;
+        return &P;
     }
+    const uint32_t CV = chunk_cap_for(h->L, k, p.grid);
     p.chunk_cap = CV;
     ChunkPlan cp;
-    if (plan_chunks(L, CV, p.grid, cp, cap_arcs, lag)) return nullptr;
+    if (plan_chunks(L, CV, p.grid, cp)) return nullptr;
     p.nchunks = cp.slots;
     p.iters = (cp.slots + p.grid - 1) / p.grid;
     const std::vector<uint32_t>& cv = cp.slot_v;
@@ -280,22 +306,6 @@ phast_ctx::Plan* get_plan(phast_ctx* h, uint32_t k) {
     uint32_t *a, *b, *w;
     if (dmalloc(&a, cv.size()) || dmalloc(&b, dep.size()) || dmalloc(&w, p.iters)) return nullptr;
     p.chunk_v = a; p.chunk_dep = b; p.wave_done = w;
-    if (p.variant == 3) {
-        std::vector<uint32_t> info((size_t)cp.slots * 4);
-        for (uint32_t j = 0; j < cp.slots; j++) {
-            info[4 * (size_t)j + 0] = cv[j];
-            info[4 * (size_t)j + 1] = cv[j + 1];
-            info[4 * (size_t)j + 2] = L.dn_first[cv[j]];
-            info[4 * (size_t)j + 3] = L.dn_first[cv[j + 1]];
-        }
-        uint32_t* pi;
-        if (dmalloc(&pi, info.size())) return nullptr;
-        p.pinfo = reinterpret_cast<const uint4*>(pi);
-        if (cudaMemcpy(pi, info.data(), info.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess) {
-            cudaGetLastError();
-            return nullptr;
-        }
-    }
     if (cudaMemcpy(a, cv.data(), cv.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess ||
         cudaMemcpy(b, dep.data(), dep.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess ||
         cudaMemset(w, 0, (size_t)p.iters * 4) != cudaSuccess) {
@@ -338,7 +348,7 @@ int run_query(phast_ctx* h, const Sources& S, uint32_t k, uint32_t* dist, uint32
     if (e1) cudaEventRecord(e1, st);
     phast_ctx::Plan* plan = h->sweep_mode != 1 ? get_plan(h, k) : nullptr;
     if (plan) {   // a3 + a4: one persistent launch, dataflow over chunk waves
-        if (plan->p.variant != 2 && (uint64_t)(plan->epoch + 1) * plan->p.grid >= 0x7FFFFFFFull) {
+        if (plan->p.variant < 2 && (uint64_t)(plan->epoch + 1) * plan->p.grid >= 0x7FFFFFFFull) {
             if (cudaMemsetAsync(plan->p.wave_done, 0, (size_t)plan->p.iters * 4, st) != cudaSuccess) return PHAST_ECUDA;
             plan->epoch = 0;
         }

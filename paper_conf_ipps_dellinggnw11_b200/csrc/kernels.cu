@@ -542,7 +542,8 @@ __global__ void __launch_bounds__(SWEEP_THREADS, 5) sweep_warp_kernel(const uint
     const uint32_t gl = lane % G, grp = lane / G;
     uint32_t mx = 0;
     for (uint32_t c = blockIdx.x * WARPS_PER_CTA + wid; c < p.nchunks; c += p.workers) {
-        const uint4 m = __ldg(&p.wmeta[c]);    // {vbeg, vend, dbeg, dend}
+        uint4 m = __ldg(&p.wmeta[c]);          // {vbeg, vend, dbeg, dend | bit 31}
+        m.w &= 0x7FFFFFFFu;
         for (uint32_t i = m.z + lane; i < m.w; i += 32) {
             const uint32_t x = __ldg(&p.wdeps[i]);
             if (ld_acquire_gpu(&p.done[x]) < epoch) {
@@ -662,27 +663,31 @@ __global__ void __launch_bounds__(SWEEP_THREADS, 3) sweep_pipe_kernel(const uint
     uint2* sarc = reinterpret_cast<uint2*>(pipe_smem + 2 * PIPE_STAGE_BYTES);           // [2][AMAX]
     uint32_t* sfirst = reinterpret_cast<uint32_t*>(sarc + 2 * AMAX);                   // [2][CV+1]
     __shared__ uint4 sinfo[3];   // chunk descriptors, indexed by iteration % 3 (thread 0 runs <1 iteration ahead)
-    __shared__ uint32_t s_known;
     const uint32_t grid = gridDim.x;
     const uint32_t gl = threadIdx.x % G, grp = threadIdx.x / G;
     uint32_t mx = 0;
 
-    // thread 0: wait until iteration dep-1 is complete on every CTA
+    // warp 0: acquire the completion flags of the chunks (of other CTAs) holding the
+    // tails of chunk c
     auto wait_dep = [&](uint32_t c) {
-        const uint32_t dep = __ldg(&p.chunk_dep[c]);
-        if (dep > s_known) {
-            const uint32_t w = dep - 1;
-            const uint32_t need = epoch * min(grid, p.nchunks - w * grid);
-            uint32_t ns = 32;
-            const uint64_t t0 = globaltimer_ns();
-            while (ld_acquire_gpu(&p.wave_done[w]) < need) {
-                __nanosleep(ns);
-                ns = min(ns * 2, 256u);
-                if (globaltimer_ns() - t0 > 4000000000ull) { atomicOr(p.err, 2u); break; }
+        const uint4 m = __ldg(&p.wmeta[c]);
+        const uint32_t lane = threadIdx.x & 31, dend = m.w & 0x7FFFFFFFu;
+        for (uint32_t i = m.z + lane; i < dend; i += 32) {
+            const uint32_t x = __ldg(&p.wdeps[i]);
+            if (ld_acquire_gpu(&p.done[x]) < epoch) {
+                uint32_t ns = 32;
+                const uint64_t t0 = globaltimer_ns();
+                while (ld_acquire_gpu(&p.done[x]) < epoch) {
+                    __nanosleep(ns);
+                    ns = min(ns * 2, 256u);
+                    if (globaltimer_ns() - t0 > 4000000000ull) { atomicOr(p.err, 2u); break; }
+                }
             }
-            s_known = dep;
         }
+        __syncwarp();
+        if (lane == 0) __threadfence();
     };
+    auto defers = [&](uint32_t c) { return (__ldg(&p.wmeta[c].w) >> 31) != 0u; };
     // all threads: offsets and arcs of the chunk described by sinfo[b] into stage b
     auto stage = [&](uint32_t b, uint32_t si) {
         const uint4 in = sinfo[si];
@@ -704,13 +709,12 @@ __global__ void __launch_bounds__(SWEEP_THREADS, 3) sweep_pipe_kernel(const uint
         cp_async_commit();
     };
 
-    if (threadIdx.x == 0) s_known = 0;
     uint32_t c = blockIdx.x;
     if (c < p.nchunks) {
         if (threadIdx.x == 0) sinfo[0] = __ldg(&p.pinfo[c]);
         __syncthreads();
         stage(0, 0);
-        if (threadIdx.x == 0) { wait_dep(c); __threadfence(); }
+        if (threadIdx.x < 32) wait_dep(c);
         __syncthreads();
         gather(0, 0);
     }
@@ -728,13 +732,14 @@ __global__ void __launch_bounds__(SWEEP_THREADS, 3) sweep_pipe_kernel(const uint
         __syncthreads();                                                       // [A]
         if (threadIdx.x == 0 && it > 0) {                                      // chunk c-grid fully written
             __threadfence();
-            atomicAdd(&p.wave_done[it - 1], 1u);
+            atomicExch(&p.done[c - grid], epoch);
         }
+        if (it > 0 && defers(c)) gather(b, si);          // c reads rows of c-grid: gathered only now
         if (cn < p.nchunks) stage(b ^ 1u, sn);
-        if (threadIdx.x == 0 && cn < p.nchunks) { wait_dep(cn); __threadfence(); }
+        if (threadIdx.x < 32 && cn < p.nchunks) wait_dep(cn);
         cp_async_wait_all();                                                   // my slices of chunk c
         __syncthreads();                                                       // [B]
-        if (cn < p.nchunks) gather(b ^ 1u, sn);                                // lookahead: chunk cn in flight
+        if (cn < p.nchunks && !defers(cn)) gather(b ^ 1u, sn);               // lookahead: chunk cn in flight
         const uint4 in = sinfo[si];
         const bool staged = in.w - in.z <= AMAX;
         const uint32_t* fb = sfirst + b * (CV + 1);
@@ -767,7 +772,7 @@ __global__ void __launch_bounds__(SWEEP_THREADS, 3) sweep_pipe_kernel(const uint
     __syncthreads();
     if (threadIdx.x == 0 && it > 0) {
         __threadfence();
-        atomicAdd(&p.wave_done[it - 1], 1u);
+        atomicExch(&p.done[c - grid], epoch);
     }
     cp_async_wait_all();
     if constexpr (DIAM) {

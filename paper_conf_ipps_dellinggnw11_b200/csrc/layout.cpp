@@ -174,13 +174,14 @@ int layout_build(const ChResult& R, const uint64_t* first, const uint32_t* head,
     return ok ? 0 : kEinternal;
 }
 
-int plan_warp_chunks(const Layout& L, uint32_t cap, uint32_t workers, WarpPlan& P) {
+int plan_warp_chunks(const Layout& L, uint32_t cap, uint32_t workers, WarpPlan& P, uint32_t cap_arcs) {
     const uint32_t n = (uint32_t)L.perm.size();
     if (cap == 0 || workers == 0) return kEinternal;
     std::vector<uint32_t> cb{0}, chunk_of(n);
     uint32_t s = 0;
     for (uint32_t v = 0; v < n; v++) {
         bool cut = (v - s == cap);
+        if (!cut && v > s && cap_arcs && L.dn_first[v + 1] - L.dn_first[s] > cap_arcs) cut = true;
         if (!cut && v > s)
             for (uint32_t e = L.dn_first[v]; e < L.dn_first[v + 1]; e++)
                 if (L.dn_arc[e].x >= s) { cut = true; break; }
@@ -194,19 +195,21 @@ int plan_warp_chunks(const Layout& L, uint32_t cap, uint32_t workers, WarpPlan& 
     std::vector<uint32_t> tmp;
     for (uint32_t c = 0; c < nch; c++) {
         tmp.clear();
+        bool prev = false;
         for (uint32_t e = L.dn_first[cb[c]]; e < L.dn_first[cb[c + 1]]; e++) {
             uint32_t x = chunk_of[L.dn_arc[e].x];
             if (x >= c) return kEinternal;                       // not topological
             if (x % workers != c % workers) tmp.push_back(x);     // same worker: already done
+            else if (x + workers == c) prev = true;               // the worker's previous chunk
         }
         std::sort(tmp.begin(), tmp.end());
         tmp.erase(std::unique(tmp.begin(), tmp.end()), tmp.end());
-        if (P.deps.size() + tmp.size() >= 0xFFFFFFF0ull) return kErange;
+        if (P.deps.size() + tmp.size() >= 0x7FFFFFF0ull) return kErange;
         P.meta[4 * (size_t)c + 0] = cb[c];
         P.meta[4 * (size_t)c + 1] = cb[c + 1];
         P.meta[4 * (size_t)c + 2] = (uint32_t)P.deps.size();
         P.deps.insert(P.deps.end(), tmp.begin(), tmp.end());
-        P.meta[4 * (size_t)c + 3] = (uint32_t)P.deps.size();
+        P.meta[4 * (size_t)c + 3] = (uint32_t)P.deps.size() | (prev ? 0x80000000u : 0u);
     }
     P.chunks = nch;
     return 0;

@@ -59,11 +59,14 @@ int plan_chunks(const Layout& L, uint32_t cap, uint32_t grid, ChunkPlan& out, ui
 // c % workers in program order.  meta[4c..4c+3] = {vbeg, vend, dbeg, dend}:
 // deps[dbeg..dend) are the distinct chunks holding a tail of chunk c that another
 // worker handles (same-worker chunks are earlier in that worker's program order).
+// Bit 31 of dend is set when chunk c depends on its worker's immediately preceding
+// chunk (c - workers): a lookahead pipeline must not start chunk c before that one is
+// written.  cap_arcs (0 = none) also cuts chunks before their arcs exceed it.
 struct WarpPlan {
     std::vector<uint32_t> meta;
     std::vector<uint32_t> deps;
     uint32_t chunks = 0;
 };
-int plan_warp_chunks(const Layout& L, uint32_t cap, uint32_t workers, WarpPlan& out);
+int plan_warp_chunks(const Layout& L, uint32_t cap, uint32_t workers, WarpPlan& out, uint32_t cap_arcs = 0);
 
 }  // namespace phast
