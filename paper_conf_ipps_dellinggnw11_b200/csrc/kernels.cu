@@ -440,9 +440,9 @@ __global__ void __launch_bounds__(SWEEP_THREADS, 4) sweep_persistent_kernel(cons
                 while (ld_acquire_gpu(&p.wave_done[w]) < need) {
                     __nanosleep(ns);
                     ns = min(ns * 2, 256u);
-                    if (globaltimer_ns() - t0 > 4000000000ull) {   // watchdog: never hang the GPU;
-                        atomicOr(p.err, 2u);                        // phast_sync reports ECUDA
-                        break;
+                    if ((*(volatile uint32_t*)p.err & 2u) || globaltimer_ns() - t0 > 4000000000ull) {
+                        atomicOr(p.err, 2u);                        // watchdog: never hang the GPU;
+                        break;                                      // phast_sync reports ECUDA
                     }
                 }
                 s_known = dep;                                 // counters are monotone in w
@@ -552,8 +552,8 @@ __global__ void __launch_bounds__(SWEEP_THREADS, 5) sweep_warp_kernel(const uint
                 while (ld_acquire_gpu(&p.done[x]) < epoch) {
                     __nanosleep(ns);
                     ns = min(ns * 2, 512u);
-                    if (globaltimer_ns() - t0 > 4000000000ull) {   // watchdog: never hang the GPU
-                        atomicOr(p.err, 2u);
+                    if ((*(volatile uint32_t*)p.err & 2u) || globaltimer_ns() - t0 > 4000000000ull) {
+                        atomicOr(p.err, 2u);                       // watchdog: never hang the GPU
                         break;
                     }
                 }
@@ -667,8 +667,19 @@ __global__ void __launch_bounds__(SWEEP_THREADS, 3) sweep_pipe_kernel(const uint
     const uint32_t gl = threadIdx.x % G, grp = threadIdx.x / G;
     uint32_t mx = 0;
 
-    // warp 0: acquire the completion flags of the chunks (of other CTAs) holding the
-    // tails of chunk c
+    // warp 0, non-blocking: are the chunks (of other CTAs) holding the tails of chunk c
+    // complete?  A lookahead must never block: the CTA still owes its current chunk.
+    auto deps_done = [&](uint32_t c) {
+        const uint4 m = __ldg(&p.wmeta[c]);
+        const uint32_t lane = threadIdx.x & 31, dend = m.w & 0x7FFFFFFFu;
+        bool ok = (m.w >> 31) == 0u;                  // depends on this CTA's current chunk: not yet
+        for (uint32_t i = m.z + lane; ok && i < dend; i += 32)
+            ok = ld_acquire_gpu(&p.done[__ldg(&p.wdeps[i])]) >= epoch;
+        ok = __all_sync(0xFFFFFFFFu, ok);
+        if (ok && lane == 0) __threadfence();
+        return ok;
+    };
+    // warp 0, blocking: acquire the completion flags of the tails' chunks of chunk c
     auto wait_dep = [&](uint32_t c) {
         const uint4 m = __ldg(&p.wmeta[c]);
         const uint32_t lane = threadIdx.x & 31, dend = m.w & 0x7FFFFFFFu;
@@ -680,14 +691,17 @@ __global__ void __launch_bounds__(SWEEP_THREADS, 3) sweep_pipe_kernel(const uint
                 while (ld_acquire_gpu(&p.done[x]) < epoch) {
                     __nanosleep(ns);
                     ns = min(ns * 2, 256u);
-                    if (globaltimer_ns() - t0 > 4000000000ull) { atomicOr(p.err, 2u); break; }
+                    if ((*(volatile uint32_t*)p.err & 2u) || globaltimer_ns() - t0 > 4000000000ull) {
+                        atomicOr(p.err, 2u);   // watchdog: report, never hang
+                        break;
+                    }
                 }
             }
         }
         __syncwarp();
         if (lane == 0) __threadfence();
     };
-    auto defers = [&](uint32_t c) { return (__ldg(&p.wmeta[c].w) >> 31) != 0u; };
+    __shared__ uint32_t s_ready[2];   // stage b's gathers were issued as a lookahead
     // all threads: offsets and arcs of the chunk described by sinfo[b] into stage b
     auto stage = [&](uint32_t b, uint32_t si) {
         const uint4 in = sinfo[si];
@@ -715,6 +729,7 @@ __global__ void __launch_bounds__(SWEEP_THREADS, 3) sweep_pipe_kernel(const uint
         __syncthreads();
         stage(0, 0);
         if (threadIdx.x < 32) wait_dep(c);
+        if (threadIdx.x == 0) s_ready[0] = 1;
         __syncthreads();
         gather(0, 0);
     }
@@ -734,12 +749,19 @@ __global__ void __launch_bounds__(SWEEP_THREADS, 3) sweep_pipe_kernel(const uint
             __threadfence();
             atomicExch(&p.done[c - grid], epoch);
         }
-        if (it > 0 && defers(c)) gather(b, si);          // c reads rows of c-grid: gathered only now
+        if (!s_ready[b]) {                               // no lookahead for c: wait (blocking) and gather now
+            if (threadIdx.x < 32) wait_dep(c);
+            __syncthreads();
+            gather(b, si);
+        }
         if (cn < p.nchunks) stage(b ^ 1u, sn);
-        if (threadIdx.x < 32 && cn < p.nchunks) wait_dep(cn);
+        if (threadIdx.x < 32) {
+            const bool ok = cn < p.nchunks && deps_done(cn);
+            if (threadIdx.x == 0) s_ready[b ^ 1u] = ok ? 1u : 0u;
+        }
         cp_async_wait_all();                                                   // my slices of chunk c
         __syncthreads();                                                       // [B]
-        if (cn < p.nchunks && !defers(cn)) gather(b ^ 1u, sn);               // lookahead: chunk cn in flight
+        if (cn < p.nchunks && s_ready[b ^ 1u]) gather(b ^ 1u, sn);             // lookahead: chunk cn in flight
         const uint4 in = sinfo[si];
         const bool staged = in.w - in.z <= AMAX;
         const uint32_t* fb = sfirst + b * (CV + 1);
