@@ -329,6 +329,9 @@ __device__ __forceinline__ uint32_t ld_acquire_gpu(const uint32_t* p) {
     asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
     return v;
 }
+__device__ __forceinline__ void st_release_gpu(uint32_t* p, uint32_t v) {
+    asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
 __device__ __forceinline__ uint64_t globaltimer_ns() {
     uint64_t t;
     asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
@@ -602,10 +605,7 @@ __global__ void __launch_bounds__(SWEEP_THREADS, 5) sweep_warp_kernel(const uint
             if constexpr (DIAM) mx = max(mx, fmax_of(acc));
         }
         __syncwarp();                                          // all rows of the chunk are issued
-        if (lane == 0) {
-            __threadfence();                                   // release the rows before the flag
-            atomicExch(&p.done[c], epoch);
-        }
+        if (lane == 0) st_release_gpu(&p.done[c], epoch);     // release: cumulative over the warp
     }
     if constexpr (DIAM) {
         mx = __reduce_max_sync(0xFFFFFFFFu, mx);
@@ -630,7 +630,7 @@ int warp_occupancy() {
 // flight into the other shared-memory stage (cp.async.cg, 16 B per lane, no register
 // staging).  A chunk's dependencies are at least two iterations back (plan lag 2),
 // so its gathers can be issued one iteration early.  Two CTA barriers per chunk.
-constexpr uint32_t PIPE_STAGE_BYTES = 32768;   // tail rows of one chunk
+constexpr uint32_t PIPE_STAGE_BYTES = 16384;   // tail rows of one chunk
 
 __device__ __forceinline__ void cp_async16(void* smem, const void* gmem) {
     asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(smem_u32(smem)), "l"(gmem) : "memory");
@@ -648,7 +648,7 @@ struct PipeGeom {
 };
 
 template <int K, bool DIAM>
-__global__ void __launch_bounds__(SWEEP_THREADS, 3) sweep_pipe_kernel(const uint32_t* __restrict__ first,
+__global__ void __launch_bounds__(SWEEP_THREADS, 4) sweep_pipe_kernel(const uint32_t* __restrict__ first,
                                                                       const uint2* __restrict__ arcs,
                                                                       uint32_t* __restrict__ d,
                                                                       const uint32_t* __restrict__ flags,
@@ -669,15 +669,15 @@ __global__ void __launch_bounds__(SWEEP_THREADS, 3) sweep_pipe_kernel(const uint
 
     // warp 0, non-blocking: are the chunks (of other CTAs) holding the tails of chunk c
     // complete?  A lookahead must never block: the CTA still owes its current chunk.
-    auto deps_done = [&](uint32_t c) {
-        const uint4 m = __ldg(&p.wmeta[c]);
+    // m, dl: the chunk's meta and this lane's first dependency id, loaded one iteration
+    // ahead (so only the completion flags are read here)
+    auto deps_done = [&](const uint4& m, uint32_t dl) {
         const uint32_t lane = threadIdx.x & 31, dend = m.w & 0x7FFFFFFFu;
         bool ok = (m.w >> 31) == 0u;                  // depends on this CTA's current chunk: not yet
-        for (uint32_t i = m.z + lane; ok && i < dend; i += 32)
+        if (ok && m.z + lane < dend) ok = ld_acquire_gpu(&p.done[dl]) >= epoch;
+        for (uint32_t i = m.z + lane + 32; ok && i < dend; i += 32)
             ok = ld_acquire_gpu(&p.done[__ldg(&p.wdeps[i])]) >= epoch;
-        ok = __all_sync(0xFFFFFFFFu, ok);
-        if (ok && lane == 0) __threadfence();
-        return ok;
+        return __all_sync(0xFFFFFFFFu, ok);
     };
     // warp 0, blocking: acquire the completion flags of the tails' chunks of chunk c
     auto wait_dep = [&](uint32_t c) {
@@ -699,7 +699,6 @@ __global__ void __launch_bounds__(SWEEP_THREADS, 3) sweep_pipe_kernel(const uint
             }
         }
         __syncwarp();
-        if (lane == 0) __threadfence();
     };
     __shared__ uint32_t s_ready[2];   // stage b's gathers were issued as a lookahead
     // all threads: offsets and arcs of the chunk described by sinfo[b] into stage b
@@ -735,6 +734,12 @@ __global__ void __launch_bounds__(SWEEP_THREADS, 3) sweep_pipe_kernel(const uint
     }
     uint4 nxt = make_uint4(0, 0, 0, 0);
     if (threadIdx.x == 0 && c + grid < p.nchunks) nxt = __ldg(&p.pinfo[c + grid]);
+    uint4 wm = make_uint4(0, 0, 0, 0);   // warp 0: meta + first dependency of the next chunk
+    uint32_t wd = 0;
+    if (threadIdx.x < 32 && c + grid < p.nchunks) {
+        wm = __ldg(&p.wmeta[c + grid]);
+        if (wm.z + threadIdx.x < (wm.w & 0x7FFFFFFFu)) wd = __ldg(&p.wdeps[wm.z + threadIdx.x]);
+    }
     uint32_t it = 0;
     for (; c < p.nchunks; c += grid, it++) {
         const uint32_t b = it & 1u;
@@ -745,10 +750,8 @@ __global__ void __launch_bounds__(SWEEP_THREADS, 3) sweep_pipe_kernel(const uint
             if (cn + grid < p.nchunks) nxt = __ldg(&p.pinfo[cn + grid]);   // one more iteration ahead
         }
         __syncthreads();                                                       // [A]
-        if (threadIdx.x == 0 && it > 0) {                                      // chunk c-grid fully written
-            __threadfence();
-            atomicExch(&p.done[c - grid], epoch);
-        }
+        if (threadIdx.x == 0 && it > 0)                                        // chunk c-grid fully written
+            st_release_gpu(&p.done[c - grid], epoch);                          // (release, cumulative over the CTA)
         if (!s_ready[b]) {                               // no lookahead for c: wait (blocking) and gather now
             if (threadIdx.x < 32) wait_dep(c);
             __syncthreads();
@@ -756,8 +759,12 @@ __global__ void __launch_bounds__(SWEEP_THREADS, 3) sweep_pipe_kernel(const uint
         }
         if (cn < p.nchunks) stage(b ^ 1u, sn);
         if (threadIdx.x < 32) {
-            const bool ok = cn < p.nchunks && deps_done(cn);
+            const bool ok = cn < p.nchunks && deps_done(wm, wd);
             if (threadIdx.x == 0) s_ready[b ^ 1u] = ok ? 1u : 0u;
+            if (cn + grid < p.nchunks) {                                       // prefetch for the next lookahead
+                wm = __ldg(&p.wmeta[cn + grid]);
+                if (wm.z + threadIdx.x < (wm.w & 0x7FFFFFFFu)) wd = __ldg(&p.wdeps[wm.z + threadIdx.x]);
+            }
         }
         cp_async_wait_all();                                                   // my slices of chunk c
         __syncthreads();                                                       // [B]
@@ -792,10 +799,7 @@ __global__ void __launch_bounds__(SWEEP_THREADS, 3) sweep_pipe_kernel(const uint
         }
     }
     __syncthreads();
-    if (threadIdx.x == 0 && it > 0) {
-        __threadfence();
-        atomicExch(&p.done[c - grid], epoch);
-    }
+    if (threadIdx.x == 0 && it > 0) st_release_gpu(&p.done[c - grid], epoch);
     cp_async_wait_all();
     if constexpr (DIAM) {
         __shared__ uint32_t wmax[SWEEP_THREADS / 32];
