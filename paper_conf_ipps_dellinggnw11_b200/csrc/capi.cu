@@ -42,8 +42,8 @@ struct phast_ctx {
         bool ok = false;
     };
     std::map<uint32_t, Plan> plans;
-    // 0 = warp dataflow (default), 1 = one launch per level, 2 = CTA waves, 3 = CTA waves + bulk-staged
-    // arcs, 4 = pipelined gather (k >= 4; else warp dataflow)
+    // 0 = warp pipeline (default), 1 = one launch per level, 2 = CTA waves, 3 = CTA waves + bulk-staged
+    // arcs, 4 = pipelined CTA gather (k >= 4; else warp pipeline), 5 = warp dataflow without pipeline
     int sweep_mode = 0;
     // upward searches run on a side stream, one seed slot ahead of the sweep
     cudaStream_t side = nullptr;
@@ -145,6 +145,7 @@ int upload(phast_ctx* h) {
                         : std::strcmp(e, "persistent") == 0 ? 2
                         : std::strcmp(e, "staged") == 0     ? 3
                         : std::strcmp(e, "pipe") == 0       ? 4
+                        : std::strcmp(e, "warp") == 0       ? 5
                                                             : 0;
     // level layouts default to one launch per level (the fastest schedule measured on them)
     if (!std::getenv("PHAST_SWEEP") && !h->L.lvl_off.empty()) h->sweep_mode = 1;
@@ -239,16 +240,35 @@ phast_ctx::Plan* get_plan(phast_ctx* h, uint32_t k) {
     const Layout& L = h->L;
     SweepPlan& p = P.p;
     p.k = k;
-    p.variant = h->sweep_mode == 2 ? 0u : h->sweep_mode == 3 ? 1u : h->sweep_mode == 4 && k >= 4 ? 3u : 2u;
+    p.variant = h->sweep_mode == 2 ? 0u : h->sweep_mode == 3 ? 1u : h->sweep_mode == 4 && k >= 4 ? 3u
+              : h->sweep_mode == 5 ? 2u : 4u;
     int occ = std::min(sweep_blocks_per_sm(k, false, p.variant), sweep_blocks_per_sm(k, true, p.variant));
     p.grid = (uint32_t)std::max(1, occ * num_sms());
     p.err = h->g.err;
-    if (p.variant == 2) {
+    if (p.variant == 2 || p.variant == 4) {
         p.workers = p.grid * (SWEEP_WARPS);
         WarpPlan wp;
-        if (plan_warp_chunks(L, sweep_warp_chunk_vertices(k), p.workers, wp)) return nullptr;
+        const uint32_t cap = p.variant == 4 ? sweep_wpipe_chunk_vertices(k) : sweep_warp_chunk_vertices(k);
+        if (plan_warp_chunks(L, cap, p.workers, wp, p.variant == 4 ? 126u : 0u)) return nullptr;
         p.nchunks = wp.chunks;
-        p.chunk_cap = sweep_warp_chunk_vertices(k);
+        p.chunk_cap = cap;
+        if (p.variant == 4) {   // per-chunk {vbeg, vend, e0, e1} for the cp.async staging
+            std::vector<uint32_t> info((size_t)wp.chunks * 4);
+            for (uint32_t j = 0; j < wp.chunks; j++) {
+                const uint32_t vb = wp.meta[4 * (size_t)j], ve = wp.meta[4 * (size_t)j + 1];
+                info[4 * (size_t)j + 0] = vb;
+                info[4 * (size_t)j + 1] = ve;
+                info[4 * (size_t)j + 2] = L.dn_first[vb];
+                info[4 * (size_t)j + 3] = L.dn_first[ve];
+            }
+            uint32_t* pi;
+            if (dmalloc(&pi, info.size())) return nullptr;
+            p.pinfo = reinterpret_cast<const uint4*>(pi);
+            if (cudaMemcpy(pi, info.data(), info.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess) {
+                cudaGetLastError();
+                return nullptr;
+            }
+        }
         uint32_t *a, *b, *w;
         if (dmalloc(&a, wp.meta.size()) || dmalloc(&b, wp.deps.size()) || dmalloc(&w, wp.chunks)) return nullptr;
         p.wmeta = reinterpret_cast<const uint4*>(a); p.wdeps = b; p.done = w;

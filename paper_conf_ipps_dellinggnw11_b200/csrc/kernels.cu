@@ -340,6 +340,11 @@ __device__ __forceinline__ uint64_t globaltimer_ns() {
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
     return static_cast<uint32_t>(__cvta_generic_to_shared(p));
 }
+__device__ __forceinline__ void cp_async16(void* smem, const void* gmem) {
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(smem_u32(smem)), "l"(gmem) : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+__device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_group 0;" ::: "memory"); }
 __device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
     asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
 }
@@ -613,6 +618,165 @@ __global__ void __launch_bounds__(SWEEP_THREADS, 5) sweep_warp_kernel(const uint
     }
 }
 
+// ------------------------------------------------------------------ a3+a4 warp pipeline (variant 4)
+// Warp dataflow (as variant 2) with a software pipeline inside each warp: the chunk
+// descriptors and dependency ids are loaded two chunks ahead, the chunk's offsets
+// and arc block are copied into shared memory by cp.async one chunk ahead (three
+// rotating buffers), so the per-chunk critical path is one acquire of the producers'
+// completion flags (usually already set) plus one round trip of tail-row gathers.
+constexpr uint32_t WP_ARCS = 128;
+
+template <int K>
+struct WpGeom {
+    static constexpr uint32_t W = RowT<K>::W;
+    static constexpr uint32_t G = K / W;
+    static constexpr uint32_t VPW = 32 / G;
+    static constexpr uint32_t CAP = VPW * 4 < 32 ? VPW * 4 : 32;
+    static constexpr uint32_t FCAP = CAP + 8;
+};
+
+template <int K, bool DIAM>
+__global__ void __launch_bounds__(SWEEP_THREADS, 4) sweep_wpipe_kernel(const uint32_t* __restrict__ first,
+                                                                       const uint2* __restrict__ arcs,
+                                                                       uint32_t* __restrict__ d,
+                                                                       const uint32_t* __restrict__ flags,
+                                                                       const uint32_t* __restrict__ tail_bits,
+                                                                       SweepPlan p, uint32_t epoch,
+                                                                       uint32_t* __restrict__ diam) {
+    using T = typename RowT<K>::T;
+    using Geo = WpGeom<K>;
+    constexpr uint32_t G = Geo::G, VPW = Geo::VPW, FCAP = Geo::FCAP;
+    __shared__ __align__(16) uint2 sarc[WARPS_PER_CTA][3][WP_ARCS];
+    __shared__ __align__(16) uint32_t sfirst[WARPS_PER_CTA][3][FCAP];
+    const uint32_t wid = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const uint32_t gl = lane % G, grp = lane / G;
+    const uint32_t NW = p.workers;
+    uint32_t mx = 0;
+
+    auto stage = [&](uint32_t buf, const uint4& in) {   // cp.async offsets + arc block of a chunk
+        const uint32_t f0 = in.x & ~3u, f1 = (in.y + 1 + 3) & ~3u;
+        for (uint32_t i = lane; i < (f1 - f0) / 4; i += 32) cp_async16(&sfirst[wid][buf][i * 4], first + f0 + i * 4);
+        const uint32_t a0 = in.z & ~1u, a1 = (in.w + 1) & ~1u;
+        if (a1 - a0 <= WP_ARCS)
+            for (uint32_t i = lane; i < (a1 - a0) / 2; i += 32) cp_async16(&sarc[wid][buf][i * 2], arcs + a0 + i * 2);
+        cp_async_commit();
+    };
+    auto load_dep = [&](uint32_t c) -> uint2 {          // {dbeg, dend & flag}
+        return __ldg(reinterpret_cast<const uint2*>(&p.wmeta[c]) + 1);
+    };
+
+    uint32_t c = blockIdx.x * WARPS_PER_CTA + wid;
+    uint4 in_c = make_uint4(0, 0, 0, 0), in_n = in_c, in_nn = in_c;
+    uint2 dr_c = make_uint2(0, 0), dr_n = dr_c, dr_nn = dr_c;
+    uint32_t did_c = 0, did_n = 0;                       // this lane's first dependency id
+    if (c < p.nchunks) {
+        in_c = __ldg(&p.pinfo[c]);
+        dr_c = load_dep(c);
+        if (dr_c.x + lane < (dr_c.y & 0x7FFFFFFFu)) did_c = __ldg(&p.wdeps[dr_c.x + lane]);
+        stage(0, in_c);
+        if (c + NW < p.nchunks) {
+            in_n = __ldg(&p.pinfo[c + NW]);
+            dr_n = load_dep(c + NW);
+            if (dr_n.x + lane < (dr_n.y & 0x7FFFFFFFu)) did_n = __ldg(&p.wdeps[dr_n.x + lane]);
+            stage(1, in_n);
+        } else {
+            cp_async_commit();
+        }
+    }
+    uint32_t bc = 0;
+    for (; c < p.nchunks; c += NW) {
+        const uint32_t cn = c + NW, cnn = cn + NW;
+        if (cnn < p.nchunks) { in_nn = __ldg(&p.pinfo[cnn]); dr_nn = load_dep(cnn); }
+        // 1. producers of c: acquire their completion flags
+        {
+            const uint32_t dend = dr_c.y & 0x7FFFFFFFu;
+            for (uint32_t i = dr_c.x + lane; i < dend; i += 32) {
+                const uint32_t x = (i == dr_c.x + lane) ? did_c : __ldg(&p.wdeps[i]);
+                if (ld_acquire_gpu(&p.done[x]) < epoch) {
+                    uint32_t ns = 32;
+                    const uint64_t t0 = globaltimer_ns();
+                    while (ld_acquire_gpu(&p.done[x]) < epoch) {
+                        __nanosleep(ns);
+                        ns = min(ns * 2, 256u);
+                        if ((*(volatile uint32_t*)p.err & 2u) || globaltimer_ns() - t0 > 4000000000ull) {
+                            atomicOr(p.err, 2u);   // watchdog: report, never hang
+                            break;
+                        }
+                    }
+                }
+            }
+        }
+        // 2. offsets and arcs of c are in shared memory (stage of cn may still fly)
+        asm volatile("cp.async.wait_group 1;" ::: "memory");
+        __syncwarp();
+        const uint32_t* sf = sfirst[wid][bc];
+        const uint2* sa = sarc[wid][bc];
+        const uint32_t f0 = in_c.x & ~3u, a0 = in_c.z & ~1u;
+        const bool staged = ((in_c.w + 1) & ~1u) - a0 <= WP_ARCS;
+        const uint32_t nv = in_c.y - in_c.x;
+        for (uint32_t base = 0; base < nv; base += VPW) {
+            const uint32_t li = base + grp;
+            if (li >= nv) break;
+            const uint32_t v = in_c.x + li;
+            T acc = inf_row<T>();
+            if ((__ldg(&flags[v >> 5]) >> (v & 31)) & 1u)   // visited by an upward search (§IV-C)
+                acc = __ldcg(reinterpret_cast<const T*>(d + (size_t)v * K) + gl);
+            uint32_t e = sf[v - f0];
+            const uint32_t e1 = sf[v + 1 - f0];
+            while (e < e1) {                                   // up to 4 gathers in flight per lane
+                const uint32_t cnt = min(e1 - e, 4u);
+                uint2 a[4];
+                T x[4];
+#pragma unroll
+                for (uint32_t j = 0; j < 4; j++)
+                    if (j < cnt) a[j] = staged ? sa[e + j - a0] : __ldg(&arcs[e + j]);
+#pragma unroll
+                for (uint32_t j = 0; j < 4; j++)
+                    if (j < cnt) x[j] = __ldcg(reinterpret_cast<const T*>(d + (size_t)a[j].x * K) + gl);
+#pragma unroll
+                for (uint32_t j = 0; j < 4; j++)
+                    if (j < cnt) acc = relax(acc, x[j], a[j].y);
+                e += cnt;
+            }
+            const bool is_tail = (__ldg(&tail_bits[v >> 5]) >> (v & 31)) & 1u;
+            if (!DIAM || is_tail) {
+                T* q = reinterpret_cast<T*>(d + (size_t)v * K) + gl;
+                if (is_tail) *q = acc; else st_stream(q, acc);
+            }
+            if constexpr (DIAM) mx = max(mx, fmax_of(acc));
+        }
+        __syncwarp();
+        if (lane == 0) st_release_gpu(&p.done[c], epoch);     // release: cumulative over the warp
+        // 3. lookahead: dependency ids of cn's successor, staging of cnn
+        uint32_t did_nn = 0;
+        if (cnn < p.nchunks) {
+            if (dr_nn.x + lane < (dr_nn.y & 0x7FFFFFFFu)) did_nn = __ldg(&p.wdeps[dr_nn.x + lane]);
+            stage((bc + 2) % 3, in_nn);
+        } else {
+            cp_async_commit();
+        }
+        in_c = in_n; dr_c = dr_n; did_c = did_n;
+        in_n = in_nn; dr_n = dr_nn; did_n = did_nn;
+        bc = (bc + 1) % 3;
+    }
+    asm volatile("cp.async.wait_group 0;" ::: "memory");
+    if constexpr (DIAM) {
+        mx = __reduce_max_sync(0xFFFFFFFFu, mx);
+        if (lane == 0 && mx) atomicMax(diam, mx);
+    }
+}
+
+template <int K, bool DIAM>
+int wpipe_occupancy() {
+    int b = 0;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, sweep_wpipe_kernel<K, DIAM>, SWEEP_THREADS, 0) !=
+        cudaSuccess) {
+        cudaGetLastError();
+        return 1;
+    }
+    return b > 0 ? b : 1;
+}
+
 template <int K, bool DIAM>
 int warp_occupancy() {
     int b = 0;
@@ -632,11 +796,6 @@ int warp_occupancy() {
 // so its gathers can be issued one iteration early.  Two CTA barriers per chunk.
 constexpr uint32_t PIPE_STAGE_BYTES = 16384;   // tail rows of one chunk
 
-__device__ __forceinline__ void cp_async16(void* smem, const void* gmem) {
-    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(smem_u32(smem)), "l"(gmem) : "memory");
-}
-__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
-__device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_group 0;" ::: "memory"); }
 
 template <int K>
 struct PipeGeom {
@@ -884,6 +1043,16 @@ cudaError_t persistent_k(const DevImage& g, const SweepPlan& p, uint32_t epoch, 
             return cudaGetLastError();
         }
     }
+    if (p.variant == 4) {
+        if (diam)
+            sweep_wpipe_kernel<K, true><<<p.grid, SWEEP_THREADS, 0, st>>>(g.dn_first, g.dn_arc, dist, g.flags,
+                                                                          g.tail_bits, p, epoch, diam);
+        else
+            sweep_wpipe_kernel<K, false><<<p.grid, SWEEP_THREADS, 0, st>>>(g.dn_first, g.dn_arc, dist, g.flags,
+                                                                           g.tail_bits, p, epoch, nullptr);
+        g_launches++;
+        return cudaGetLastError();
+    }
     if (p.variant == 2) {
         if (diam)
             sweep_warp_kernel<K, true><<<p.grid, SWEEP_THREADS, 0, st>>>(g.dn_first, g.dn_arc, dist, g.flags,
@@ -979,6 +1148,18 @@ void sweep_pipe_geometry(uint32_t k, uint32_t* cap_vertices, uint32_t* cap_arcs)
     }
 }
 
+uint32_t sweep_wpipe_chunk_vertices(uint32_t k) {
+    switch (k) {
+        case 1: return WpGeom<1>::CAP;
+        case 2: return WpGeom<2>::CAP;
+        case 4: return WpGeom<4>::CAP;
+        case 8: return WpGeom<8>::CAP;
+        case 16: return WpGeom<16>::CAP;
+        case 32: return WpGeom<32>::CAP;
+        default: return WpGeom<64>::CAP;
+    }
+}
+
 uint32_t sweep_warp_chunk_vertices(uint32_t k) { return (32 / (k >= 4 ? k / 4 : 1)) * WARP_PASSES; }
 
 uint32_t sweep_pass_vertices(uint32_t k) { return SWEEP_THREADS / (k >= 4 ? k / 4 : 1); }
@@ -990,7 +1171,8 @@ uint32_t sweep_chunk_vertices(uint32_t k) {
 
 int sweep_blocks_per_sm(uint32_t k, bool diam, uint32_t variant) {
 #define OCC(K)                                                                                               \
-    (variant == 3 ? (diam ? pipe_occupancy<K, true>() : pipe_occupancy<K, false>()) :                         \
+    (variant == 4 ? (diam ? wpipe_occupancy<K, true>() : wpipe_occupancy<K, false>()) :                       \
+     variant == 3 ? (diam ? pipe_occupancy<K, true>() : pipe_occupancy<K, false>()) :                         \
      variant == 2 ? (diam ? warp_occupancy<K, true>() : warp_occupancy<K, false>()) :                         \
      variant == 1 ? (diam ? persistent_occupancy<K, true, true>() : persistent_occupancy<K, false, true>())   \
                   : (diam ? persistent_occupancy<K, true, false>() : persistent_occupancy<K, false, false>()))

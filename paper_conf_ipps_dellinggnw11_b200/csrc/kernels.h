@@ -48,7 +48,7 @@ cudaError_t launch_sweep_level(const DevImage& g, uint32_t k, uint32_t vbeg, uin
 // chunk_dep[c] - 1 (0 = no dependency).
 struct SweepPlan {
     uint32_t k = 0, nchunks = 0, grid = 0, iters = 0, chunk_cap = 0;
-    uint32_t variant = 2;   // 3: pipelined gather; 2: warp dataflow; 1: CTA waves + bulk-staged arcs; 0: CTA waves
+    uint32_t variant = 2;   // 4: warp pipeline; 3: pipelined gather; 2: warp dataflow; 1: CTA waves + bulk-staged arcs; 0: CTA waves
     // variant 3 (pipelined gather): per slot {vbeg, vend, e0 = first[vbeg], e1 = first[vend]}
     const uint4* pinfo = nullptr;
     // variant 2 (warp dataflow)
@@ -65,6 +65,7 @@ struct SweepPlan {
 uint32_t sweep_chunk_vertices(uint32_t k);   // max vertices per chunk
 uint32_t sweep_pass_vertices(uint32_t k);    // vertices per pass of a CTA
 uint32_t sweep_warp_chunk_vertices(uint32_t k);
+uint32_t sweep_wpipe_chunk_vertices(uint32_t k);  // variant 4
 constexpr uint32_t SWEEP_WARPS = 8;               // warps per CTA of the persistent sweeps
 // variant 3: max vertices and arcs per chunk for k (k >= 4; 0 otherwise)
 void sweep_pipe_geometry(uint32_t k, uint32_t* cap_vertices, uint32_t* cap_arcs);   // vertices per chunk of one warp (variant 2)

@@ -124,6 +124,7 @@ def test_upward_global_fallback_and_overflow(monkeypatch):
 @pytest.mark.parametrize("mode,level_layout,delta", [("levels", True, 0), ("levels", "bfs", 0),
                                                      ("warp", True, 0), ("staged", True, 0),
                                                      ("warp", False, 0), ("persistent", False, 0),
+                                                     ("wpipe", False, 0), ("wpipe", False, 300), ("wpipe", True, 0),
                                                      ("pipe", False, 0), ("pipe", False, 300), ("pipe", True, 0),
                                                      ("staged", False, 0), ("warp", False, 300),
                                                      ("staged", False, 300)])
