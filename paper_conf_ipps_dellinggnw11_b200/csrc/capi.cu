@@ -39,6 +39,7 @@ struct phast_ctx {
     struct Plan {
         SweepPlan p;
         uint32_t epoch = 0;
+        uint32_t top_levels = 0;   // hybrid (per-level mode): levels [0, top_levels) run as one persistent launch
         bool ok = false;
     };
     std::map<uint32_t, Plan> plans;
@@ -242,6 +243,17 @@ phast_ctx::Plan* get_plan(phast_ctx* h, uint32_t k) {
     p.k = k;
     p.variant = h->sweep_mode == 2 ? 0u : h->sweep_mode == 3 ? 1u : h->sweep_mode == 4 && k >= 4 ? 3u
               : h->sweep_mode == 5 ? 2u : 4u;
+    uint32_t limit = 0;
+    if (h->sweep_mode == 1) {   // hybrid: the small top levels as one CTA-wave launch, big levels one launch each
+        uint32_t thresh = 65536;
+        if (const char* e = std::getenv("PHAST_TOP_THRESH")) thresh = (uint32_t)std::atoi(e);
+        uint32_t J = 0;
+        while (J < L.levels && L.lvl_off[J + 1] - L.lvl_off[J] < thresh) J++;
+        if (J < 2) return nullptr;           // nothing worth fusing
+        P.top_levels = J;
+        limit = L.lvl_off[J];
+        p.variant = 0;
+    }
     int occ = std::min(sweep_blocks_per_sm(k, false, p.variant), sweep_blocks_per_sm(k, true, p.variant));
     p.grid = (uint32_t)std::max(1, occ * num_sms());
     p.err = h->g.err;
@@ -318,7 +330,7 @@ phast_ctx::Plan* get_plan(phast_ctx* h, uint32_t k) {
     const uint32_t CV = chunk_cap_for(h->L, k, p.grid);
     p.chunk_cap = CV;
     ChunkPlan cp;
-    if (plan_chunks(L, CV, p.grid, cp)) return nullptr;
+    if (plan_chunks(L, CV, p.grid, cp, 0, 1, limit)) return nullptr;
     p.nchunks = cp.slots;
     p.iters = (cp.slots + p.grid - 1) / p.grid;
     const std::vector<uint32_t>& cv = cp.slot_v;
@@ -366,8 +378,8 @@ int run_query(phast_ctx* h, const Sources& S, uint32_t k, uint32_t* dist, uint32
     if (cudaStreamWaitEvent(st, h->up_done[slot], 0) != cudaSuccess) return PHAST_ECUDA;
     if (launch_seed(h->g, k, slot, dist, st) != cudaSuccess) return PHAST_ECUDA;
     if (e1) cudaEventRecord(e1, st);
-    phast_ctx::Plan* plan = h->sweep_mode != 1 ? get_plan(h, k) : nullptr;
-    if (plan) {   // a3 + a4: one persistent launch, dataflow over chunk waves
+    phast_ctx::Plan* plan = get_plan(h, k);
+    if (plan && plan->top_levels == 0) {   // a3 + a4: one persistent launch, dataflow over chunks
         if (plan->p.variant < 2 && (uint64_t)(plan->epoch + 1) * plan->p.grid >= 0x7FFFFFFFull) {
             if (cudaMemsetAsync(plan->p.wave_done, 0, (size_t)plan->p.iters * 4, st) != cudaSuccess) return PHAST_ECUDA;
             plan->epoch = 0;
@@ -376,7 +388,19 @@ int run_query(phast_ctx* h, const Sources& S, uint32_t k, uint32_t* dist, uint32
         if (launch_sweep_persistent(h->g, plan->p, plan->epoch, dist, diam, st) != cudaSuccess) return PHAST_ECUDA;
     } else if (!h->L.lvl_off.empty()) {   // one launch per level (§VI), level layout only
         const uint32_t levels = h->L.levels;
-        for (uint32_t j = 0; j < levels; j++) {
+        uint32_t j0 = 0;
+        if (plan) {                           // hybrid: small top levels in one persistent launch
+            if ((uint64_t)(plan->epoch + 1) * plan->p.grid >= 0x7FFFFFFFull) {
+                if (cudaMemsetAsync(plan->p.wave_done, 0, (size_t)plan->p.iters * 4, st) != cudaSuccess)
+                    return PHAST_ECUDA;
+                plan->epoch = 0;
+            }
+            plan->epoch++;
+            if (launch_sweep_persistent(h->g, plan->p, plan->epoch, dist, diam, st) != cudaSuccess)
+                return PHAST_ECUDA;
+            j0 = plan->top_levels;
+        }
+        for (uint32_t j = j0; j < levels; j++) {
             bool last = (j + 1 == levels);
             bool store = !(diam && last);   // level-0 rows are never read again (diameter mode)
             if (launch_sweep_level(h->g, k, h->L.lvl_off[j], h->L.lvl_off[j + 1], dist, diam, store, last, st) !=

@@ -215,8 +215,9 @@ int plan_warp_chunks(const Layout& L, uint32_t cap, uint32_t workers, WarpPlan& 
     return 0;
 }
 
-int plan_chunks(const Layout& L, uint32_t cap, uint32_t grid, ChunkPlan& P, uint32_t cap_arcs, uint32_t lag) {
-    const uint32_t n = (uint32_t)L.perm.size();
+int plan_chunks(const Layout& L, uint32_t cap, uint32_t grid, ChunkPlan& P, uint32_t cap_arcs, uint32_t lag,
+                uint32_t limit) {
+    const uint32_t n = limit ? limit : (uint32_t)L.perm.size();
     if (cap == 0 || grid == 0 || lag == 0) return kEinternal;
     // 1. chunk boundaries and each chunk's latest tail chunk (unpadded numbering)
     std::vector<uint32_t> cb{0}, chunk_of(n);

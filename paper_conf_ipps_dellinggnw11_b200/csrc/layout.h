@@ -51,8 +51,9 @@ struct ChunkPlan {
 };
 // cap_arcs (0 = none): also cut before a chunk's G-down arcs exceed cap_arcs;
 // lag: every dependency is at least `lag` iterations earlier.
+// limit (0 = n): plan only ids [0, limit) (a prefix of the order is closed under tails).
 int plan_chunks(const Layout& L, uint32_t cap, uint32_t grid, ChunkPlan& out, uint32_t cap_arcs = 0,
-                uint32_t lag = 1);
+                uint32_t lag = 1, uint32_t limit = 0);
 
 // Warp-granular dataflow schedule (default sweep): chunks of consecutive ids (at most
 // cap vertices, cut at intra-chunk dependencies), chunk c handled by worker (warp)

@@ -122,6 +122,7 @@ def test_upward_global_fallback_and_overflow(monkeypatch):
 
 
 @pytest.mark.parametrize("mode,level_layout,delta", [("levels", True, 0), ("levels", "bfs", 0),
+                                                     ("levels-hybrid", True, 0), ("levels-flat", "bfs", 0),
                                                      ("warp", True, 0), ("staged", True, 0),
                                                      ("warp", False, 0), ("persistent", False, 0),
                                                      ("wpipe", False, 0), ("wpipe", False, 300), ("wpipe", True, 0),
@@ -133,6 +134,12 @@ def test_sweep_modes(monkeypatch, mode, level_layout, delta):
     (§VI); the single persistent launch as warp dataflow (default) or CTA
     waves (with and without bulk-staged arcs), on both layouts, including a small
     wavefront skew (many short dependencies)."""
+    if mode == "levels-hybrid":                  # a few small top levels fused, the rest one launch each
+        monkeypatch.setenv("PHAST_TOP_THRESH", "3000")
+        mode = "levels"
+    elif mode == "levels-flat":                  # one launch per level, no fusion
+        monkeypatch.setenv("PHAST_TOP_THRESH", "0")
+        mode = "levels"
     monkeypatch.setenv("PHAST_SWEEP", mode)
     g = phastgen.road(120_000, seed=33)
     with P.Phast.from_graph(g, level_layout=bool(level_layout), bfs_in_level=level_layout == "bfs",
