@@ -245,7 +245,7 @@ phast_ctx::Plan* get_plan(phast_ctx* h, uint32_t k) {
               : h->sweep_mode == 5 ? 2u : 4u;
     uint32_t limit = 0;
     if (h->sweep_mode == 1) {   // hybrid: the small top levels as one CTA-wave launch, big levels one launch each
-        uint32_t thresh = 65536;
+        uint32_t thresh = 0;   // measured: one launch per level is faster on C3; opt-in
         if (const char* e = std::getenv("PHAST_TOP_THRESH")) thresh = (uint32_t)std::atoi(e);
         uint32_t J = 0;
         while (J < L.levels && L.lvl_off[J + 1] - L.lvl_off[J] < thresh) J++;

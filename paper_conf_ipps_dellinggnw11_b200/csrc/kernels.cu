@@ -238,6 +238,11 @@ template <class T> __device__ __forceinline__ void st_stream(T* p, T v) { __stcs
 
 constexpr int SWEEP_THREADS = 256;
 
+// One level [vbeg, vend) (§VI "The CPU starts, for each level i, a kernel on
+// the GPU").  Each thread owns two (vertex, 16-byte lane) items per grid-stride step
+// and issues the gathers of both before reducing (more bytes in flight per thread).
+// Launched with programmatic dependent launch: the next level's grid is launched while
+// this one drains and blocks in griddepcontrol.wait until this grid's rows are visible.
 template <int K, bool DIAM, bool STORE, bool STREAM>
 __global__ void __launch_bounds__(SWEEP_THREADS) sweep_kernel(const uint32_t* __restrict__ first,
                                                                const uint2* __restrict__ arcs,
@@ -248,27 +253,57 @@ __global__ void __launch_bounds__(SWEEP_THREADS) sweep_kernel(const uint32_t* __
     using T = typename RowT<K>::T;
     constexpr uint32_t W = RowT<K>::W;
     constexpr uint32_t G = K / W;   // lanes per vertex
+    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+    asm volatile("griddepcontrol.wait;" ::: "memory");          // previous level complete and visible
     const uint64_t total = (uint64_t)(vend - vbeg) * G;
+    const uint64_t stride = (uint64_t)gridDim.x * SWEEP_THREADS;
     uint32_t mx = 0;
-    for (uint64_t t = (uint64_t)blockIdx.x * SWEEP_THREADS + threadIdx.x; t < total;
-         t += (uint64_t)gridDim.x * SWEEP_THREADS) {
-        const uint32_t v = vbeg + (uint32_t)(t / G);
-        const uint32_t lane = (uint32_t)(t % G);
-        T acc = inf_row<T>();
-        if ((__ldg(&flags[v >> 5]) >> (v & 31)) & 1u)   // visited by an upward search
-            acc = __ldg(reinterpret_cast<const T*>(d + (size_t)v * K) + lane);
-        const uint32_t e0 = __ldg(&first[v]), e1 = __ldg(&first[v + 1]);
-#pragma unroll 4
-        for (uint32_t e = e0; e < e1; e++) {
-            const uint2 a = __ldg(&arcs[e]);
-            const T x = __ldg(reinterpret_cast<const T*>(d + (size_t)a.x * K) + lane);
-            acc = relax(acc, x, a.y);
+    for (uint64_t t0 = (uint64_t)blockIdx.x * SWEEP_THREADS + threadIdx.x; t0 < total; t0 += 2 * stride) {
+        uint32_t v[2], lane[2], e[2], e1[2];
+        bool live[2];
+        T acc[2];
+#pragma unroll
+        for (int q = 0; q < 2; q++) {
+            const uint64_t t = t0 + q * stride;
+            live[q] = t < total;
+            v[q] = vbeg + (uint32_t)((live[q] ? t : t0) / G);
+            lane[q] = (uint32_t)((live[q] ? t : t0) % G);
+            acc[q] = inf_row<T>();
+            if (live[q] && ((__ldg(&flags[v[q] >> 5]) >> (v[q] & 31)) & 1u))   // visited by an upward search
+                acc[q] = __ldg(reinterpret_cast<const T*>(d + (size_t)v[q] * K) + lane[q]);
+            e[q] = live[q] ? __ldg(&first[v[q]]) : 0u;
+            e1[q] = live[q] ? __ldg(&first[v[q] + 1]) : 0u;
         }
-        if constexpr (STORE) {
-            T* p = reinterpret_cast<T*>(d + (size_t)v * K) + lane;
-            if constexpr (STREAM) st_stream(p, acc); else *p = acc;
+        while (e[0] < e1[0] || e[1] < e1[1]) {       // up to 2 x 3 gathers in flight
+            uint2 a[2][3];
+            T x[2][3];
+#pragma unroll
+            for (int q = 0; q < 2; q++)
+#pragma unroll
+                for (uint32_t j = 0; j < 3; j++)
+                    if (e[q] + j < e1[q]) a[q][j] = __ldg(&arcs[e[q] + j]);
+#pragma unroll
+            for (int q = 0; q < 2; q++)
+#pragma unroll
+                for (uint32_t j = 0; j < 3; j++)
+                    if (e[q] + j < e1[q]) x[q][j] = __ldg(reinterpret_cast<const T*>(d + (size_t)a[q][j].x * K) + lane[q]);
+#pragma unroll
+            for (int q = 0; q < 2; q++)
+#pragma unroll
+                for (uint32_t j = 0; j < 3; j++)
+                    if (e[q] + j < e1[q]) acc[q] = relax(acc[q], x[q][j], a[q][j].y);
+            e[0] = min(e[0] + 3, max(e[0], e1[0]));
+            e[1] = min(e[1] + 3, max(e[1], e1[1]));
         }
-        if constexpr (DIAM) mx = max(mx, fmax_of(acc));
+#pragma unroll
+        for (int q = 0; q < 2; q++) {
+            if (!live[q]) continue;
+            if constexpr (STORE) {
+                T* p = reinterpret_cast<T*>(d + (size_t)v[q] * K) + lane[q];
+                if constexpr (STREAM) st_stream(p, acc[q]); else *p = acc[q];
+            }
+            if constexpr (DIAM) mx = max(mx, fmax_of(acc[q]));
+        }
     }
     if constexpr (DIAM) {
         __shared__ uint32_t wmax[SWEEP_THREADS / 32];
@@ -288,14 +323,32 @@ cudaError_t sweep_launch(const DevImage& g, uint32_t vbeg, uint32_t vend, uint32
                          cudaStream_t st) {
     constexpr uint32_t G = K / RowT<K>::W;
     uint64_t total = (uint64_t)(vend - vbeg) * G;
-    uint64_t blocks = (total + SWEEP_THREADS - 1) / SWEEP_THREADS;
-    uint64_t cap = (uint64_t)num_sms() * 8;
+    uint64_t blocks = (total + 2 * SWEEP_THREADS - 1) / (2 * SWEEP_THREADS);
+    static int occ = 0;   // one resident wave: blocks beyond it would only add a tail
+    if (!occ) {
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, sweep_kernel<K, DIAM, STORE, STREAM>, SWEEP_THREADS,
+                                                          0) != cudaSuccess || occ <= 0) {
+            cudaGetLastError();
+            occ = 4;
+        }
+    }
+    uint64_t cap = (uint64_t)num_sms() * occ;
     if (blocks > cap) blocks = cap;
     if (blocks == 0) return cudaSuccess;
-    sweep_kernel<K, DIAM, STORE, STREAM><<<(unsigned)blocks, SWEEP_THREADS, 0, st>>>(g.dn_first, g.dn_arc, dist,
-                                                                                 g.flags, vbeg, vend, diam);
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3((unsigned)blocks);
+    cfg.blockDim = dim3(SWEEP_THREADS);
+    cfg.dynamicSmemBytes = 0;
+    cfg.stream = st;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    cudaError_t e = cudaLaunchKernelEx(&cfg, sweep_kernel<K, DIAM, STORE, STREAM>, g.dn_first, g.dn_arc, dist,
+                                       (const uint32_t*)g.flags, vbeg, vend, diam);
     g_launches++;
-    return cudaGetLastError();
+    return e;
 }
 
 template <int K>
