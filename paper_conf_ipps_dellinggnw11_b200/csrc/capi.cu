@@ -147,6 +147,7 @@ int upload(phast_ctx* h) {
                         : std::strcmp(e, "staged") == 0     ? 3
                         : std::strcmp(e, "pipe") == 0       ? 4
                         : std::strcmp(e, "warp") == 0       ? 5
+                        : std::strcmp(e, "wave") == 0       ? 6
                                                             : 0;
     // level layouts default to one launch per level (the fastest schedule measured on them)
     if (!std::getenv("PHAST_SWEEP") && !h->L.lvl_off.empty()) h->sweep_mode = 1;
@@ -242,7 +243,7 @@ phast_ctx::Plan* get_plan(phast_ctx* h, uint32_t k) {
     SweepPlan& p = P.p;
     p.k = k;
     p.variant = h->sweep_mode == 2 ? 0u : h->sweep_mode == 3 ? 1u : h->sweep_mode == 4 && k >= 4 ? 3u
-              : h->sweep_mode == 5 ? 2u : 4u;
+              : h->sweep_mode == 5 ? 2u : h->sweep_mode == 6 ? 5u : 4u;
     uint32_t limit = 0;
     if (h->sweep_mode == 1) {   // hybrid: the small top levels as one CTA-wave launch, big levels one launch each
         uint32_t thresh = 0;   // measured: one launch per level is faster on C3; opt-in
@@ -257,6 +258,34 @@ phast_ctx::Plan* get_plan(phast_ctx* h, uint32_t k) {
     int occ = std::min(sweep_blocks_per_sm(k, false, p.variant), sweep_blocks_per_sm(k, true, p.variant));
     p.grid = (uint32_t)std::max(1, occ * num_sms());
     p.err = h->g.err;
+    if (p.variant == 5) {   // warp waves: one wave = one chunk of every warp (layout.cpp: plan_waves)
+        p.workers = p.grid * SWEEP_WARPS;
+        uint32_t window = 4;
+        if (const char* e = std::getenv("PHAST_WAVE_WINDOW")) window = (uint32_t)std::atoi(e);
+        WavePlan wp;
+        if (plan_waves(L, sweep_wave_chunk_vertices(k), sweep_wave_chunk_arcs(), p.workers, window, wp))
+            return nullptr;
+        p.nchunks = wp.chunks;
+        p.iters = wp.waves;
+        p.chunk_cap = (wp.waves + 63) / 64 * 64;   // sub-counter stride: each sub-counter array on its own lines
+        if (std::getenv("PHAST_VERBOSE"))
+            std::fprintf(stderr, "wave plan k=%u: T=%u chunks=%u waves=%u pads=%u lag1=%llu lag2=%llu lag3=%llu lag4+=%llu\n",
+                         k, p.workers, wp.chunks, wp.waves, wp.pads, (unsigned long long)wp.lag_hist[0],
+                         (unsigned long long)wp.lag_hist[1], (unsigned long long)wp.lag_hist[2],
+                         (unsigned long long)wp.lag_hist[3]);
+        uint32_t *a, *w;
+        const size_t nc = (size_t)sweep_wave_subcounters() * p.chunk_cap;
+        if (dmalloc(&a, wp.desc.size() + 4) || dmalloc(&w, nc)) return nullptr;
+        p.wdesc = reinterpret_cast<const uint4*>(a);
+        p.wave_done = w;
+        if ((!wp.desc.empty() && cudaMemcpy(a, wp.desc.data(), wp.desc.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess) ||
+            cudaMemset(w, 0, nc * 4) != cudaSuccess) {
+            cudaGetLastError();
+            return nullptr;
+        }
+        P.ok = true;
+        return &P;
+    }
     if (p.variant == 2 || p.variant == 4) {
         p.workers = p.grid * (SWEEP_WARPS);
         WarpPlan wp;
@@ -382,6 +411,13 @@ int run_query(phast_ctx* h, const Sources& S, uint32_t k, uint32_t* dist, uint32
     if (plan && plan->top_levels == 0) {   // a3 + a4: one persistent launch, dataflow over chunks
         if (plan->p.variant < 2 && (uint64_t)(plan->epoch + 1) * plan->p.grid >= 0x7FFFFFFFull) {
             if (cudaMemsetAsync(plan->p.wave_done, 0, (size_t)plan->p.iters * 4, st) != cudaSuccess) return PHAST_ECUDA;
+            plan->epoch = 0;
+        }
+        if (plan->p.variant == 5 &&
+            (uint64_t)(plan->epoch + 1) * (plan->p.workers / sweep_wave_subcounters()) >= 0x7FFFFFFFull) {
+            if (cudaMemsetAsync(plan->p.wave_done, 0,
+                                (size_t)sweep_wave_subcounters() * plan->p.chunk_cap * 4, st) != cudaSuccess)
+                return PHAST_ECUDA;
             plan->epoch = 0;
         }
         plan->epoch++;

@@ -239,10 +239,12 @@ template <class T> __device__ __forceinline__ void st_stream(T* p, T v) { __stcs
 constexpr int SWEEP_THREADS = 256;
 
 // One level [vbeg, vend) (§VI "The CPU starts, for each level i, a kernel on
-// the GPU").  Each thread owns two (vertex, 16-byte lane) items per grid-stride step
-// and issues the gathers of both before reducing (more bytes in flight per thread).
-// Launched with programmatic dependent launch: the next level's grid is launched while
-// this one drains and blocks in griddepcontrol.wait until this grid's rows are visible.
+// the GPU").  One (vertex, 16-byte lane) item per thread per grid-stride step; the
+// grid fills every SM (8 CTAs of 256 threads), which keeps the most gathers in flight
+// (measured: a two-items-per-thread variant with fewer resident CTAs was 30 % slower
+// on level 0, profiles/r1_launches_*).  Launched with programmatic dependent launch:
+// the next level's grid is launched while this one drains and blocks in
+// griddepcontrol.wait until this grid's rows are visible.
 template <int K, bool DIAM, bool STORE, bool STREAM>
 __global__ void __launch_bounds__(SWEEP_THREADS) sweep_kernel(const uint32_t* __restrict__ first,
                                                                const uint2* __restrict__ arcs,
@@ -256,54 +258,26 @@ __global__ void __launch_bounds__(SWEEP_THREADS) sweep_kernel(const uint32_t* __
     asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
     asm volatile("griddepcontrol.wait;" ::: "memory");          // previous level complete and visible
     const uint64_t total = (uint64_t)(vend - vbeg) * G;
-    const uint64_t stride = (uint64_t)gridDim.x * SWEEP_THREADS;
     uint32_t mx = 0;
-    for (uint64_t t0 = (uint64_t)blockIdx.x * SWEEP_THREADS + threadIdx.x; t0 < total; t0 += 2 * stride) {
-        uint32_t v[2], lane[2], e[2], e1[2];
-        bool live[2];
-        T acc[2];
-#pragma unroll
-        for (int q = 0; q < 2; q++) {
-            const uint64_t t = t0 + q * stride;
-            live[q] = t < total;
-            v[q] = vbeg + (uint32_t)((live[q] ? t : t0) / G);
-            lane[q] = (uint32_t)((live[q] ? t : t0) % G);
-            acc[q] = inf_row<T>();
-            if (live[q] && ((__ldg(&flags[v[q] >> 5]) >> (v[q] & 31)) & 1u))   // visited by an upward search
-                acc[q] = __ldg(reinterpret_cast<const T*>(d + (size_t)v[q] * K) + lane[q]);
-            e[q] = live[q] ? __ldg(&first[v[q]]) : 0u;
-            e1[q] = live[q] ? __ldg(&first[v[q] + 1]) : 0u;
+    for (uint64_t t = (uint64_t)blockIdx.x * SWEEP_THREADS + threadIdx.x; t < total;
+         t += (uint64_t)gridDim.x * SWEEP_THREADS) {
+        const uint32_t v = vbeg + (uint32_t)(t / G);
+        const uint32_t lane = (uint32_t)(t % G);
+        T acc = inf_row<T>();
+        if ((__ldg(&flags[v >> 5]) >> (v & 31)) & 1u)   // visited by an upward search
+            acc = __ldg(reinterpret_cast<const T*>(d + (size_t)v * K) + lane);
+        const uint32_t e0 = __ldg(&first[v]), e1 = __ldg(&first[v + 1]);
+#pragma unroll 4
+        for (uint32_t e = e0; e < e1; e++) {
+            const uint2 a = __ldg(&arcs[e]);
+            const T x = __ldg(reinterpret_cast<const T*>(d + (size_t)a.x * K) + lane);
+            acc = relax(acc, x, a.y);
         }
-        while (e[0] < e1[0] || e[1] < e1[1]) {       // up to 2 x 3 gathers in flight
-            uint2 a[2][3];
-            T x[2][3];
-#pragma unroll
-            for (int q = 0; q < 2; q++)
-#pragma unroll
-                for (uint32_t j = 0; j < 3; j++)
-                    if (e[q] + j < e1[q]) a[q][j] = __ldg(&arcs[e[q] + j]);
-#pragma unroll
-            for (int q = 0; q < 2; q++)
-#pragma unroll
-                for (uint32_t j = 0; j < 3; j++)
-                    if (e[q] + j < e1[q]) x[q][j] = __ldg(reinterpret_cast<const T*>(d + (size_t)a[q][j].x * K) + lane[q]);
-#pragma unroll
-            for (int q = 0; q < 2; q++)
-#pragma unroll
-                for (uint32_t j = 0; j < 3; j++)
-                    if (e[q] + j < e1[q]) acc[q] = relax(acc[q], x[q][j], a[q][j].y);
-            e[0] = min(e[0] + 3, max(e[0], e1[0]));
-            e[1] = min(e[1] + 3, max(e[1], e1[1]));
+        if constexpr (STORE) {
+            T* p = reinterpret_cast<T*>(d + (size_t)v * K) + lane;
+            if constexpr (STREAM) st_stream(p, acc); else *p = acc;
         }
-#pragma unroll
-        for (int q = 0; q < 2; q++) {
-            if (!live[q]) continue;
-            if constexpr (STORE) {
-                T* p = reinterpret_cast<T*>(d + (size_t)v[q] * K) + lane[q];
-                if constexpr (STREAM) st_stream(p, acc[q]); else *p = acc[q];
-            }
-            if constexpr (DIAM) mx = max(mx, fmax_of(acc[q]));
-        }
+        if constexpr (DIAM) mx = max(mx, fmax_of(acc));
     }
     if constexpr (DIAM) {
         __shared__ uint32_t wmax[SWEEP_THREADS / 32];
@@ -323,16 +297,8 @@ cudaError_t sweep_launch(const DevImage& g, uint32_t vbeg, uint32_t vend, uint32
                          cudaStream_t st) {
     constexpr uint32_t G = K / RowT<K>::W;
     uint64_t total = (uint64_t)(vend - vbeg) * G;
-    uint64_t blocks = (total + 2 * SWEEP_THREADS - 1) / (2 * SWEEP_THREADS);
-    static int occ = 0;   // one resident wave: blocks beyond it would only add a tail
-    if (!occ) {
-        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, sweep_kernel<K, DIAM, STORE, STREAM>, SWEEP_THREADS,
-                                                          0) != cudaSuccess || occ <= 0) {
-            cudaGetLastError();
-            occ = 4;
-        }
-    }
-    uint64_t cap = (uint64_t)num_sms() * occ;
+    uint64_t blocks = (total + SWEEP_THREADS - 1) / SWEEP_THREADS;
+    uint64_t cap = (uint64_t)num_sms() * 8;
     if (blocks > cap) blocks = cap;
     if (blocks == 0) return cudaSuccess;
     cudaLaunchConfig_t cfg = {};
@@ -852,6 +818,201 @@ int warp_occupancy() {
     return b > 0 ? b : 1;
 }
 
+// ------------------------------------------------------------------ a3+a4 warp waves (variant 5)
+// ONE launch; T = gridDim.x * 8 warps, every one resident.  Warp w runs slots w, w+T,
+// w+2T, ... of the wave plan (layout.cpp: plan_waves), so slot j*T + w is its j-th
+// chunk and "wave j" is the j-th chunk of every warp.  A warp finishes its chunks in
+// order, hence "wave j complete" (all T warps signalled j) implies every wave < j is
+// complete: a chunk waits on ONE condition, the wave of its latest tail chunk, which
+// the plan puts strictly before the chunk's own wave (§III "(For
+// correctness, any reverse topological order will do.)").  A warp caches how many
+// leading waves it knows to be complete, so in the bulk of the wavefront (tails about
+// delta ids, i.e. several waves, back) a check costs nothing.
+// Completion: 8 sub-counters per wave (warp w adds to w % 8), monotone over launches
+// (each reaches T/8 * epoch), spread over separate 256-byte lines.
+// Per warp, the chunk's offsets and arc block are staged into shared memory by
+// cp.async one chunk ahead, the descriptors two ahead; inside a chunk every lane owns
+// STEPS (vertex, 16-byte lane) items and issues the first WAVE_R gathers of all of
+// them before reducing any (up to STEPS*WAVE_R 16-byte loads in flight per lane).
+constexpr uint32_t WAVE_STEPS = 4;
+constexpr uint32_t WAVE_R = 2;          // gathers per item issued together
+constexpr uint32_t WAVE_ACAP = 64;      // staged arcs per chunk
+constexpr uint32_t WAVE_SUB = 8;        // sub-counters per wave
+
+template <int K>
+struct WaveGeom {
+    static constexpr uint32_t G = K / RowT<K>::W;        // lanes per row
+    static constexpr uint32_t VPS = 32 / G;              // vertices per warp step
+    static constexpr uint32_t U = VPS * WAVE_STEPS;      // vertices per chunk (<= 128)
+    static constexpr uint32_t FCAP = U + 8;              // staged offsets (16-byte aligned window)
+};
+
+template <int K, bool DIAM>
+__global__ void __launch_bounds__(SWEEP_THREADS, 2) sweep_wave_kernel(const uint32_t* __restrict__ first,
+                                                                      const uint2* __restrict__ arcs,
+                                                                      uint32_t* __restrict__ d,
+                                                                      const uint32_t* __restrict__ flags,
+                                                                      const uint32_t* __restrict__ tail_bits,
+                                                                      SweepPlan p, uint32_t epoch,
+                                                                      uint32_t* __restrict__ diam) {
+    using T = typename RowT<K>::T;
+    using Geo = WaveGeom<K>;
+    constexpr uint32_t G = Geo::G, VPS = Geo::VPS, FCAP = Geo::FCAP;
+    __shared__ __align__(16) uint2 sarc[WARPS_PER_CTA][2][WAVE_ACAP];
+    __shared__ __align__(16) uint32_t sfirst[WARPS_PER_CTA][2][FCAP];
+    const uint32_t wid = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const uint32_t gl = lane % G, grp = lane / G;
+    const uint32_t NT = p.workers;                       // T
+    const uint32_t w = blockIdx.x * WARPS_PER_CTA + wid;
+    const uint32_t nw = p.iters;                         // waves
+    const uint32_t stride = p.chunk_cap;                 // sub-counter stride (words)
+    const uint32_t target = (NT / WAVE_SUB) * epoch;
+    const uint4* __restrict__ desc = p.wdesc;
+    uint32_t* cnt = p.wave_done;
+    uint32_t mx = 0;
+
+    auto stage = [&](uint32_t buf, const uint4& in) {   // cp.async offsets + arc block of a chunk
+        const uint32_t vn = in.y & 0xFFu;
+        if (vn) {
+            const uint32_t f0 = in.x & ~3u, f1 = (in.x + vn + 1 + 3) & ~3u;
+            for (uint32_t i = lane; i < (f1 - f0) / 4; i += 32) cp_async16(&sfirst[wid][buf][i * 4], first + f0 + i * 4);
+            const uint32_t a0 = in.z & ~1u, a1 = (in.w + 1) & ~1u;
+            if (a1 - a0 <= WAVE_ACAP)
+                for (uint32_t i = lane; i < (a1 - a0) / 2; i += 32) cp_async16(&sarc[wid][buf][i * 2], arcs + a0 + i * 2);
+        }
+        cp_async_commit();
+    };
+
+    const uint4 zero = make_uint4(0, 0, 0, 0);
+    uint4 in_c = nw > 0 ? __ldg(&desc[w]) : zero;
+    uint4 in_n = nw > 1 ? __ldg(&desc[(size_t)NT + w]) : zero;
+    stage(0, in_c);
+    uint32_t known = 0;                                  // waves [0, known) are complete
+    for (uint32_t j = 0; j < nw; j++) {
+        const uint4 in_nn = j + 2 < nw ? __ldg(&desc[(size_t)(j + 2) * NT + w]) : zero;
+        stage((j + 1) & 1, in_n);
+        // 1. the wave holding this chunk's latest tail must be complete
+        const uint32_t dep1 = in_c.y >> 8;
+        if (dep1 > known) {
+            const uint32_t x = dep1 - 1;
+            bool ok = lane >= WAVE_SUB || ld_flag(&cnt[(size_t)lane * stride + x]) >= target;
+            if (!__all_sync(0xFFFFFFFFu, ok)) {
+                uint32_t ns = 32;
+                const uint64_t t0 = globaltimer_ns();
+                for (;;) {
+                    __nanosleep(ns);
+                    ns = min(ns * 2, 256u);
+                    ok = lane >= WAVE_SUB || ld_flag(&cnt[(size_t)lane * stride + x]) >= target;
+                    if (__all_sync(0xFFFFFFFFu, ok)) break;
+                    bool dead = lane == 0 && ((*(volatile uint32_t*)p.err & 2u) ||
+                                              globaltimer_ns() - t0 > 4000000000ull);
+                    if (__any_sync(0xFFFFFFFFu, dead)) {
+                        if (lane == 0) atomicOr(p.err, 2u);   // watchdog: report, never hang
+                        break;
+                    }
+                }
+            }
+            known = dep1;
+        }
+        // 2. this chunk's offsets and arcs are in shared memory (the next chunk's may fly)
+        asm volatile("cp.async.wait_group 1;" ::: "memory");
+        __syncwarp();
+        const uint32_t vn = in_c.y & 0xFFu;
+        if (vn) {
+            const uint32_t* sf = sfirst[wid][j & 1];
+            const uint2* sa = sarc[wid][j & 1];
+            const uint32_t f0 = in_c.x & ~3u, a0 = in_c.z & ~1u;
+            const bool staged = ((in_c.w + 1) & ~1u) - a0 <= WAVE_ACAP;
+            uint32_t v[WAVE_STEPS], e[WAVE_STEPS], e1[WAVE_STEPS];
+            T acc[WAVE_STEPS];
+#pragma unroll
+            for (uint32_t s = 0; s < WAVE_STEPS; s++) {
+                const uint32_t li = s * VPS + grp;
+                v[s] = in_c.x + li;
+                acc[s] = inf_row<T>();
+                e[s] = e1[s] = 0;
+                if (li < vn) {
+                    if ((__ldg(&flags[v[s] >> 5]) >> (v[s] & 31)) & 1u)   // visited (§IV-C)
+                        acc[s] = __ldcg(reinterpret_cast<const T*>(d + (size_t)v[s] * K) + gl);
+                    e[s] = sf[v[s] - f0];
+                    e1[s] = sf[v[s] + 1 - f0];
+                }
+            }
+            {   // first round: WAVE_R gathers of every item in flight together
+                uint2 a[WAVE_STEPS][WAVE_R];
+                T x[WAVE_STEPS][WAVE_R];
+#pragma unroll
+                for (uint32_t s = 0; s < WAVE_STEPS; s++)
+#pragma unroll
+                    for (uint32_t r = 0; r < WAVE_R; r++)
+                        if (e[s] + r < e1[s]) a[s][r] = staged ? sa[e[s] + r - a0] : __ldg(&arcs[e[s] + r]);
+#pragma unroll
+                for (uint32_t s = 0; s < WAVE_STEPS; s++)
+#pragma unroll
+                    for (uint32_t r = 0; r < WAVE_R; r++)
+                        if (e[s] + r < e1[s]) x[s][r] = __ldcg(reinterpret_cast<const T*>(d + (size_t)a[s][r].x * K) + gl);
+#pragma unroll
+                for (uint32_t s = 0; s < WAVE_STEPS; s++)
+#pragma unroll
+                    for (uint32_t r = 0; r < WAVE_R; r++)
+                        if (e[s] + r < e1[s]) acc[s] = relax(acc[s], x[s][r], a[s][r].y);
+            }
+#pragma unroll
+            for (uint32_t s = 0; s < WAVE_STEPS; s++) {   // the rest (high in-degree vertices)
+                for (uint32_t q = e[s] + WAVE_R; q < e1[s]; q += 4) {
+                    const uint32_t c = min(e1[s] - q, 4u);
+                    uint2 a[4];
+                    T x[4];
+#pragma unroll
+                    for (uint32_t r = 0; r < 4; r++)
+                        if (r < c) a[r] = staged ? sa[q + r - a0] : __ldg(&arcs[q + r]);
+#pragma unroll
+                    for (uint32_t r = 0; r < 4; r++)
+                        if (r < c) x[r] = __ldcg(reinterpret_cast<const T*>(d + (size_t)a[r].x * K) + gl);
+#pragma unroll
+                    for (uint32_t r = 0; r < 4; r++)
+                        if (r < c) acc[s] = relax(acc[s], x[r], a[r].y);
+                }
+            }
+#pragma unroll
+            for (uint32_t s = 0; s < WAVE_STEPS; s++) {
+                if (s * VPS + grp >= vn) continue;
+                const bool is_tail = (__ldg(&tail_bits[v[s] >> 5]) >> (v[s] & 31)) & 1u;
+                if (!DIAM || is_tail) {                          // diameter: rows nobody reads are not stored
+                    T* q = reinterpret_cast<T*>(d + (size_t)v[s] * K) + gl;
+                    if (is_tail) *q = acc[s];                    // re-read soon, from L2
+                    else st_stream(q, acc[s]);                   // never re-read: evict first
+                }
+                if constexpr (DIAM) mx = max(mx, fmax_of(acc[s]));
+            }
+        }
+        // 3. signal wave j: every lane's rows are performed at gpu scope, then one add
+        __threadfence();
+        __syncwarp();
+        if (lane == 0)
+            asm volatile("red.relaxed.gpu.global.add.u32 [%0], 1;" ::"l"(&cnt[(size_t)(w % WAVE_SUB) * stride + j])
+                         : "memory");
+        in_c = in_n;
+        in_n = in_nn;
+    }
+    asm volatile("cp.async.wait_group 0;" ::: "memory");
+    if constexpr (DIAM) {
+        mx = __reduce_max_sync(0xFFFFFFFFu, mx);
+        if (lane == 0 && mx) atomicMax(diam, mx);
+    }
+}
+
+template <int K, bool DIAM>
+int wave_occupancy() {
+    int b = 0;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, sweep_wave_kernel<K, DIAM>, SWEEP_THREADS, 0) !=
+        cudaSuccess) {
+        cudaGetLastError();
+        return 1;
+    }
+    return b > 0 ? b : 1;
+}
+
 // ------------------------------------------------------------------ a3+a4 pipelined gather (variant 3)
 // CTA chunks on the wavefront layout with a one-chunk lookahead: while chunk c is
 // reduced from shared memory, the tail rows of the CTA's next chunk are already in
@@ -1107,6 +1268,16 @@ cudaError_t persistent_k(const DevImage& g, const SweepPlan& p, uint32_t epoch, 
             return cudaGetLastError();
         }
     }
+    if (p.variant == 5) {
+        if (diam)
+            sweep_wave_kernel<K, true><<<p.grid, SWEEP_THREADS, 0, st>>>(g.dn_first, g.dn_arc, dist, g.flags,
+                                                                         g.tail_bits, p, epoch, diam);
+        else
+            sweep_wave_kernel<K, false><<<p.grid, SWEEP_THREADS, 0, st>>>(g.dn_first, g.dn_arc, dist, g.flags,
+                                                                          g.tail_bits, p, epoch, nullptr);
+        g_launches++;
+        return cudaGetLastError();
+    }
     if (p.variant == 4) {
         if (diam)
             sweep_wpipe_kernel<K, true><<<p.grid, SWEEP_THREADS, 0, st>>>(g.dn_first, g.dn_arc, dist, g.flags,
@@ -1224,6 +1395,20 @@ uint32_t sweep_wpipe_chunk_vertices(uint32_t k) {
     }
 }
 
+uint32_t sweep_wave_chunk_vertices(uint32_t k) {
+    switch (k) {
+        case 1: return WaveGeom<1>::U;
+        case 2: return WaveGeom<2>::U;
+        case 4: return WaveGeom<4>::U;
+        case 8: return WaveGeom<8>::U;
+        case 16: return WaveGeom<16>::U;
+        case 32: return WaveGeom<32>::U;
+        default: return WaveGeom<64>::U;
+    }
+}
+uint32_t sweep_wave_chunk_arcs() { return WAVE_ACAP - 2; }
+uint32_t sweep_wave_subcounters() { return WAVE_SUB; }
+
 uint32_t sweep_warp_chunk_vertices(uint32_t k) { return (32 / (k >= 4 ? k / 4 : 1)) * WARP_PASSES; }
 
 uint32_t sweep_pass_vertices(uint32_t k) { return SWEEP_THREADS / (k >= 4 ? k / 4 : 1); }
@@ -1235,7 +1420,8 @@ uint32_t sweep_chunk_vertices(uint32_t k) {
 
 int sweep_blocks_per_sm(uint32_t k, bool diam, uint32_t variant) {
 #define OCC(K)                                                                                               \
-    (variant == 4 ? (diam ? wpipe_occupancy<K, true>() : wpipe_occupancy<K, false>()) :                       \
+    (variant == 5 ? (diam ? wave_occupancy<K, true>() : wave_occupancy<K, false>()) :                         \
+     variant == 4 ? (diam ? wpipe_occupancy<K, true>() : wpipe_occupancy<K, false>()) :                       \
      variant == 3 ? (diam ? pipe_occupancy<K, true>() : pipe_occupancy<K, false>()) :                         \
      variant == 2 ? (diam ? warp_occupancy<K, true>() : warp_occupancy<K, false>()) :                         \
      variant == 1 ? (diam ? persistent_occupancy<K, true, true>() : persistent_occupancy<K, false, true>())   \

@@ -48,7 +48,7 @@ cudaError_t launch_sweep_level(const DevImage& g, uint32_t k, uint32_t vbeg, uin
 // chunk_dep[c] - 1 (0 = no dependency).
 struct SweepPlan {
     uint32_t k = 0, nchunks = 0, grid = 0, iters = 0, chunk_cap = 0;
-    uint32_t variant = 2;   // 4: warp pipeline; 3: pipelined gather; 2: warp dataflow; 1: CTA waves + bulk-staged arcs; 0: CTA waves
+    uint32_t variant = 2;   // 5: warp waves (wave plan, per-wave sub-counters); 4: warp pipeline; 3: pipelined gather; 2: warp dataflow; 1: CTA waves + bulk-staged arcs; 0: CTA waves
     // variant 3 (pipelined gather): per slot {vbeg, vend, e0 = first[vbeg], e1 = first[vend]}
     const uint4* pinfo = nullptr;
     // variant 2 (warp dataflow)
@@ -58,7 +58,9 @@ struct SweepPlan {
     uint32_t* done = nullptr;               // [nchunks] epoch of the last completion
     const uint32_t* chunk_v = nullptr;      // [nchunks+1] chunk boundaries
     const uint32_t* chunk_dep = nullptr;    // [nchunks]
-    uint32_t* wave_done = nullptr;          // [iters] monotone completion counters (epochs)
+    uint32_t* wave_done = nullptr;          // [iters] monotone completion counters (epochs);
+                                            // variant 5: [8][chunk_cap] sub-counters, chunk_cap = stride
+    const uint4* wdesc = nullptr;           // variant 5: [iters * workers] chunk descriptors (plan_waves)
     uint32_t* err = nullptr;                // sticky device error word (bit 1: dependency watchdog)
 };
 // vertices per chunk and CTAs per SM the persistent sweep uses for this k
@@ -66,6 +68,9 @@ uint32_t sweep_chunk_vertices(uint32_t k);   // max vertices per chunk
 uint32_t sweep_pass_vertices(uint32_t k);    // vertices per pass of a CTA
 uint32_t sweep_warp_chunk_vertices(uint32_t k);
 uint32_t sweep_wpipe_chunk_vertices(uint32_t k);  // variant 4
+uint32_t sweep_wave_chunk_vertices(uint32_t k);   // variant 5: vertices per chunk
+uint32_t sweep_wave_chunk_arcs();                 // variant 5: max G-down arcs per chunk (staged)
+uint32_t sweep_wave_subcounters();                // variant 5: completion sub-counters per wave
 constexpr uint32_t SWEEP_WARPS = 8;               // warps per CTA of the persistent sweeps
 // variant 3: max vertices and arcs per chunk for k (k >= 4; 0 otherwise)
 void sweep_pipe_geometry(uint32_t k, uint32_t* cap_vertices, uint32_t* cap_arcs);   // vertices per chunk of one warp (variant 2)

@@ -263,4 +263,70 @@ int plan_chunks(const Layout& L, uint32_t cap, uint32_t grid, ChunkPlan& P, uint
     return 0;
 }
 
+int plan_waves(const Layout& L, uint32_t cap, uint32_t cap_arcs, uint32_t T, uint32_t window, WavePlan& P) {
+    const uint32_t n = (uint32_t)L.perm.size();
+    if (cap == 0 || cap > 255 || T == 0) return kEinternal;
+    // 1. chunk boundaries (no chunk holds both ends of a G-down arc)
+    std::vector<uint32_t> cb{0}, chunk_of(n);
+    uint32_t s = 0;
+    for (uint32_t v = 0; v < n; v++) {
+        bool cut = (v - s == cap);
+        if (!cut && v > s && cap_arcs && L.dn_first[v + 1] - L.dn_first[s] > cap_arcs) cut = true;
+        if (!cut && v > s)
+            for (uint32_t e = L.dn_first[v]; e < L.dn_first[v + 1]; e++)
+                if (L.dn_arc[e].x >= s) { cut = true; break; }
+        if (cut) { cb.push_back(v); s = v; }
+        chunk_of[v] = (uint32_t)cb.size() - 1;
+    }
+    cb.push_back(n);
+    const uint32_t nch = (uint32_t)cb.size() - 1;
+    // 2. first-fit placement in id order
+    std::vector<uint32_t> wave(nch), dep(nch), fill, nxt;   // nxt[w]: a later wave to try when w is full
+    auto grow = [&](uint32_t w) {
+        while (fill.size() <= w) { nxt.push_back((uint32_t)fill.size()); fill.push_back(0); }
+    };
+    auto find = [&](uint32_t w) {   // first wave >= w with a free slot (path-compressed skips)
+        grow(w);
+        uint32_t r = w;
+        while (fill[r] == T) { r = nxt[r]; grow(r); }
+        while (w != r) { const uint32_t nx = nxt[w]; nxt[w] = r; w = nx; }
+        return r;
+    };
+    uint32_t hi = 0;
+    for (uint32_t c = 0; c < nch; c++) {
+        int64_t dw = -1;
+        for (uint32_t e = L.dn_first[cb[c]]; e < L.dn_first[cb[c + 1]]; e++) {
+            const uint32_t x = chunk_of[L.dn_arc[e].x];
+            if (x >= c) return kEinternal;                     // not topological
+            dw = std::max<int64_t>(dw, wave[x]);
+        }
+        uint32_t lo = (uint32_t)(dw + 1);
+        if (hi > window) lo = std::max(lo, hi - window);
+        const uint32_t w = find(lo);
+        if (w > 0xFFFFF0u) return kErange;
+        wave[c] = w;
+        dep[c] = (uint32_t)(dw + 1);
+        if (++fill[w] == T) nxt[w] = w + 1;
+        hi = std::max(hi, w);
+        const uint64_t lag = dw < 0 ? 4 : w - (uint64_t)dw;
+        P.lag_hist[std::min<uint64_t>(lag, 4) - 1]++;
+    }
+    // 3. slot table
+    const uint32_t waves = nch ? hi + 1 : 0;
+    P.desc.assign((size_t)4 * waves * T, 0);
+    std::fill(fill.begin(), fill.end(), 0);
+    for (uint32_t c = 0; c < nch; c++) {
+        const size_t sl = (size_t)wave[c] * T + fill[wave[c]]++;
+        uint32_t* q = &P.desc[4 * sl];
+        q[0] = cb[c];
+        q[1] = (cb[c + 1] - cb[c]) | (dep[c] << 8);
+        q[2] = L.dn_first[cb[c]];
+        q[3] = L.dn_first[cb[c + 1]];
+    }
+    P.chunks = nch;
+    P.waves = waves;
+    P.pads = (uint32_t)((uint64_t)waves * T - nch);
+    return 0;
+}
+
 }  // namespace phast

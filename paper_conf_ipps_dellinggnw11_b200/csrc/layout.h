@@ -70,4 +70,20 @@ struct WarpPlan {
 };
 int plan_warp_chunks(const Layout& L, uint32_t cap, uint32_t workers, WarpPlan& out, uint32_t cap_arcs = 0);
 
+// Wave schedule of the warp-wave sweep (sweep_wave_kernel).  T warps run in lock-free
+// "waves": wave j is slot j*T + w of every warp w, and a wave is complete when all T
+// warps have signalled it.  Chunks (consecutive ids, at most cap vertices and cap_arcs
+// arcs, cut at intra-chunk arcs) are placed in increasing id order, each in the first
+// wave with a free slot that is (i) after the waves of all chunks holding its tails
+// and (ii) at least `window` waves below the highest wave used so far -- so the
+// schedule stays close to the id order (the wavefront's L2 reuse) while a chunk never
+// waits on its own wave.  Unfilled slots are empty pads.
+// desc[s] = {vbeg, vcount | (dep + 1) << 8 (0: no dependency), e0 = first[vbeg], e1 = first[vbeg+vcount]}.
+struct WavePlan {
+    std::vector<uint32_t> desc;     // [4 * waves * T]
+    uint32_t chunks = 0, waves = 0, pads = 0;
+    uint64_t lag_hist[4] = {0, 0, 0, 0};   // chunks by (wave - dependency wave): 1, 2, 3, >= 4 (or none)
+};
+int plan_waves(const Layout& L, uint32_t cap, uint32_t cap_arcs, uint32_t T, uint32_t window, WavePlan& out);
+
 }  // namespace phast

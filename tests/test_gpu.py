@@ -128,7 +128,8 @@ def test_upward_global_fallback_and_overflow(monkeypatch):
                                                      ("wpipe", False, 0), ("wpipe", False, 300), ("wpipe", True, 0),
                                                      ("pipe", False, 0), ("pipe", False, 300), ("pipe", True, 0),
                                                      ("staged", False, 0), ("warp", False, 300),
-                                                     ("staged", False, 300)])
+                                                     ("staged", False, 300), ("wave", False, 0),
+                                                     ("wave", False, 300), ("wave", True, 0), ("wave", "bfs", 0)])
 def test_sweep_modes(monkeypatch, mode, level_layout, delta):
     """Every schedule is bit-exact: one launch per level on the paper's level layout
     (§VI); the single persistent launch as warp dataflow (default) or CTA
@@ -149,6 +150,21 @@ def test_sweep_modes(monkeypatch, mode, level_layout, delta):
             assert np.array_equal(gpu_trees(h, src), oracle.sssp_many(g, src)), k
         src = phastgen.sources(g.n, 200, seed=901)
         assert h.diameter(src, k_batch=64) == oracle.diameter(g, src)
+
+
+@pytest.mark.parametrize("window", ["0", "1", "64"])
+def test_wave_sweep_every_k(monkeypatch, window):
+    """The warp-wave sweep (plan_waves + sweep_wave_kernel) at every k (each k has its
+    own chunk geometry) and several placement windows, bit-exact, repeated calls
+    (epoch-monotone completion counters)."""
+    monkeypatch.setenv("PHAST_SWEEP", "wave")
+    monkeypatch.setenv("PHAST_WAVE_WINDOW", window)
+    g = phastgen.road(60_000, seed=35)
+    with P.Phast.from_graph(g, delta=2000) as h:
+        for k in (1, 2, 4, 8, 16, 32, 64):
+            for rep in range(2):
+                src = phastgen.sources(g.n, k, seed=950 + k + rep)
+                assert np.array_equal(gpu_trees(h, src), oracle.sssp_many(g, src)), (k, rep)
 
 
 def test_tiny_and_degenerate():
