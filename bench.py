@@ -162,7 +162,7 @@ def main():
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cache", default="", help="hierarchy file to reuse/create (optional)")
-    ap.add_argument("--layout", default="levels-bfs", choices=["wavefront", "levels", "levels-bfs"],
+    ap.add_argument("--layout", default="levels-bfs", choices=["wavefront", "levels", "levels-bfs", "diagonal"],
                     help="vertex order: wavefront, the paper's level layout (DFS within a level), or level "
                          "layout with BFS order within a level (default)")
     ap.add_argument("--delta", type=int, default=0, help="wavefront skew (0 = library default)")
@@ -189,8 +189,8 @@ def main():
 
     g, cfg = build_graph(args.config)
     k = args.k
-    bopts = dict(level_layout=args.layout != "wavefront", bfs_in_level=args.layout == "levels-bfs",
-                 delta=args.delta)
+    bopts = dict(level_layout=args.layout in ("levels", "levels-bfs"), bfs_in_level=args.layout == "levels-bfs",
+                 diagonal=args.layout == "diagonal", delta=args.delta)
     # hierarchy: rank 0 builds (host CH, not the timed target) and shares it via a file
     path = args.cache or f"/tmp/phast_{args.config}_{os.getpid() if world == 1 else 'dist'}.phast"
     if world > 1:
@@ -294,7 +294,7 @@ def main():
             "vs_baseline": None, "dtype": "u32", "data": "synthetic",
             "config": {"workload": f"{args.config}: {cfg['desc']}", "k": k, "trees_per_step_per_gpu": k,
                        "n": info.n, "m": info.m, "m_down": info.m_down, "m_up": info.m_up, "n_tail": info.n_tail,
-                       "levels": info.levels, "layout": ["wavefront", "levels", "levels-bfs"][info.layout],
+                       "levels": info.levels, "layout": ["wavefront", "levels", "levels-bfs", "diagonal"][info.layout],
                        "delta": info.delta, "sweep": os.environ.get("PHAST_SWEEP", "levels" if info.layout else "warp"), "parallelism": f"sources sharded over {world} GPU(s), graph replicated",
                        "l2": f"label array {4 * k * info.n / 1e9:.2f} GB >> 126 MB L2 (no flush needed)",
                        "ch_build_s": round(info.build_seconds, 1)},

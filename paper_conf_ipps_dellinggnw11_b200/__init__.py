@@ -25,6 +25,7 @@ K_ALLOWED = (1, 2, 4, 8, 16, 32, 64)
 FLAG_HOST_ONLY = 1
 FLAG_LEVEL_LAYOUT = 2
 FLAG_BFS_IN_LEVEL = 4
+FLAG_DIAGONAL = 8
 
 STATUS = {0: "OK", -1: "EINVAL", -2: "ENOMEM", -3: "ECUDA", -4: "ERANGE", -5: "ESTATE", -6: "EIO",
           -7: "EINTERNAL"}
@@ -127,7 +128,8 @@ class Phast:
     """A built hierarchy bound to one CUDA device (phast_ctx)."""
 
     def __init__(self, n=None, first=None, head=None, length=None, *, host_only=False, threads=0,
-                 hop_limit_lo=0, hop_limit_hi=0, settled_cap=0, level_layout=False, bfs_in_level=False, delta=0, _handle=None):
+                 hop_limit_lo=0, hop_limit_hi=0, settled_cap=0, level_layout=False, bfs_in_level=False, diagonal=False, delta=0,
+                 _handle=None):
         self._h = None
         if _handle is not None:
             self._h = _handle
@@ -139,7 +141,7 @@ class Phast:
                 head = np.zeros(1, np.uint32)
                 length = np.zeros(1, np.uint32)
             flags = ((FLAG_HOST_ONLY if host_only else 0) | (FLAG_LEVEL_LAYOUT if level_layout else 0)
-                     | (FLAG_BFS_IN_LEVEL if bfs_in_level else 0))
+                     | (FLAG_BFS_IN_LEVEL if bfs_in_level else 0) | (FLAG_DIAGONAL if diagonal else 0))
             o = _Opts(hop_limit_lo, hop_limit_hi, settled_cap, threads, flags, delta, 0)
             h = ctypes.c_void_p()
             _check("phast_build", _lib.phast_build(int(n), first.ctypes.data, head.ctypes.data,

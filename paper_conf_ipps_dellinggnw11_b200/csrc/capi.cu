@@ -148,10 +148,11 @@ int upload(phast_ctx* h) {
                         : std::strcmp(e, "pipe") == 0       ? 4
                         : std::strcmp(e, "warp") == 0       ? 5
                         : std::strcmp(e, "wave") == 0       ? 6
+                        : std::strcmp(e, "segments") == 0   ? 7
                                                             : 0;
     // level layouts default to one launch per level (the fastest schedule measured on them)
     if (!std::getenv("PHAST_SWEEP") && !h->L.lvl_off.empty()) h->sweep_mode = 1;
-    if (h->sweep_mode == 1 && h->L.lvl_off.empty()) h->sweep_mode = 0;   // needs contiguous levels
+    if ((h->sweep_mode == 1 || h->sweep_mode == 7) && h->L.lvl_off.empty()) h->sweep_mode = 0;   // needs segments
     // test knobs (rounded down to powers of two): shrink the shared-memory table / the
     // per-source capacity to exercise the global fallback and the overflow error path
     uint32_t seed_cap = SEED_CAP, smem_cap = 4096;
@@ -243,21 +244,45 @@ phast_ctx::Plan* get_plan(phast_ctx* h, uint32_t k) {
     SweepPlan& p = P.p;
     p.k = k;
     p.variant = h->sweep_mode == 2 ? 0u : h->sweep_mode == 3 ? 1u : h->sweep_mode == 4 && k >= 4 ? 3u
-              : h->sweep_mode == 5 ? 2u : h->sweep_mode == 6 ? 5u : 4u;
-    uint32_t limit = 0;
-    if (h->sweep_mode == 1) {   // hybrid: the small top levels as one CTA-wave launch, big levels one launch each
-        uint32_t thresh = 0;   // measured: one launch per level is faster on C3; opt-in
+              : h->sweep_mode == 5 ? 2u : h->sweep_mode == 6 ? 5u : h->sweep_mode == 7 ? 6u : 4u;
+    uint32_t nseg_top = 0;
+    if (h->sweep_mode == 1) {   // hybrid: the small top segments as one segment-barrier launch, big ones one launch each
+        uint32_t thresh = 0;
         if (const char* e = std::getenv("PHAST_TOP_THRESH")) thresh = (uint32_t)std::atoi(e);
         uint32_t J = 0;
-        while (J < L.levels && L.lvl_off[J + 1] - L.lvl_off[J] < thresh) J++;
+        while (J + 1 < L.lvl_off.size() && L.lvl_off[J + 1] - L.lvl_off[J] < thresh) J++;
         if (J < 2) return nullptr;           // nothing worth fusing
         P.top_levels = J;
-        limit = L.lvl_off[J];
-        p.variant = 0;
+        nseg_top = J;
+        p.variant = 6;
     }
     int occ = std::min(sweep_blocks_per_sm(k, false, p.variant), sweep_blocks_per_sm(k, true, p.variant));
     p.grid = (uint32_t)std::max(1, occ * num_sms());
     p.err = h->g.err;
+    if (p.variant == 6) {   // segment barriers: the segments of the layout, one grid barrier between two
+        if ((uint64_t)h->n * 16 >= 0x7FFFFFFFull) return nullptr;   // 32-bit item indices
+        // CTAs per SM: all (8) for a whole sweep; for the hybrid's top levels fewer, so
+        // that the next batch's upward searches (side stream) stay co-resident and never
+        // hold back a CTA of this grid (every CTA must be resident for the barriers)
+        int per_sm = nseg_top ? 4 : 8;
+        if (const char* e = std::getenv(nseg_top ? "PHAST_TOP_CTAS" : "PHAST_SEG_CTAS")) per_sm = std::max(1, std::atoi(e));
+        p.grid = (uint32_t)std::max(1, std::min(occ, per_sm) * num_sms());
+        const uint32_t nseg = nseg_top ? nseg_top : (uint32_t)L.lvl_off.size() - 1;
+        p.nchunks = p.iters = nseg;
+        p.chunk_cap = L.mode == LAYOUT_DIAGONAL ? L.levels - L.cut : nseg;   // diagonals: store by tail bit
+        p.stream_last = nseg_top ? 0u : 1u;   // the layout's last segment is nobody's tail
+        uint32_t *a, *w;
+        if (dmalloc(&a, nseg + 1) || dmalloc(&w, nseg)) return nullptr;
+        p.chunk_v = a;
+        p.wave_done = w;
+        if (cudaMemcpy(a, L.lvl_off.data(), (size_t)(nseg + 1) * 4, cudaMemcpyHostToDevice) != cudaSuccess ||
+            cudaMemset(w, 0, (size_t)nseg * 4) != cudaSuccess) {
+            cudaGetLastError();
+            return nullptr;
+        }
+        P.ok = true;
+        return &P;
+    }
     if (p.variant == 5) {   // warp waves: one wave = one chunk of every warp (layout.cpp: plan_waves)
         p.workers = p.grid * SWEEP_WARPS;
         uint32_t window = 4;
@@ -359,7 +384,7 @@ phast_ctx::Plan* get_plan(phast_ctx* h, uint32_t k) {
     const uint32_t CV = chunk_cap_for(h->L, k, p.grid);
     p.chunk_cap = CV;
     ChunkPlan cp;
-    if (plan_chunks(L, CV, p.grid, cp, 0, 1, limit)) return nullptr;
+    if (plan_chunks(L, CV, p.grid, cp, 0, 1, 0)) return nullptr;
     p.nchunks = cp.slots;
     p.iters = (cp.slots + p.grid - 1) / p.grid;
     const std::vector<uint32_t>& cv = cp.slot_v;
@@ -409,7 +434,7 @@ int run_query(phast_ctx* h, const Sources& S, uint32_t k, uint32_t* dist, uint32
     if (e1) cudaEventRecord(e1, st);
     phast_ctx::Plan* plan = get_plan(h, k);
     if (plan && plan->top_levels == 0) {   // a3 + a4: one persistent launch, dataflow over chunks
-        if (plan->p.variant < 2 && (uint64_t)(plan->epoch + 1) * plan->p.grid >= 0x7FFFFFFFull) {
+        if ((plan->p.variant < 2 || plan->p.variant == 6) && (uint64_t)(plan->epoch + 1) * plan->p.grid >= 0x7FFFFFFFull) {
             if (cudaMemsetAsync(plan->p.wave_done, 0, (size_t)plan->p.iters * 4, st) != cudaSuccess) return PHAST_ECUDA;
             plan->epoch = 0;
         }
@@ -423,7 +448,8 @@ int run_query(phast_ctx* h, const Sources& S, uint32_t k, uint32_t* dist, uint32
         plan->epoch++;
         if (launch_sweep_persistent(h->g, plan->p, plan->epoch, dist, diam, st) != cudaSuccess) return PHAST_ECUDA;
     } else if (!h->L.lvl_off.empty()) {   // one launch per level (§VI), level layout only
-        const uint32_t levels = h->L.levels;
+        const uint32_t levels = (uint32_t)h->L.lvl_off.size() - 1;   // segments
+        const bool diagonal = h->L.mode == LAYOUT_DIAGONAL;
         uint32_t j0 = 0;
         if (plan) {                           // hybrid: small top levels in one persistent launch
             if ((uint64_t)(plan->epoch + 1) * plan->p.grid >= 0x7FFFFFFFull) {
@@ -439,7 +465,9 @@ int run_query(phast_ctx* h, const Sources& S, uint32_t k, uint32_t* dist, uint32
         for (uint32_t j = j0; j < levels; j++) {
             bool last = (j + 1 == levels);
             bool store = !(diam && last);   // level-0 rows are never read again (diameter mode)
-            if (launch_sweep_level(h->g, k, h->L.lvl_off[j], h->L.lvl_off[j + 1], dist, diam, store, last, st) !=
+            const bool by_tail = diagonal && j >= h->L.levels - h->L.cut;   // diagonals mix levels
+            if (launch_sweep_level(h->g, k, h->L.lvl_off[j], h->L.lvl_off[j + 1], dist, diam, store, last, by_tail,
+                                   st) !=
                 cudaSuccess)
                 return PHAST_ECUDA;
         }
@@ -496,7 +524,8 @@ int phast_build(uint32_t n, const uint64_t* first, const uint32_t* head, const u
         h->m = first[n];
         h->shortcuts = R.shortcuts;
         h->rounds = R.rounds;
-        const uint32_t mode = (flags & PHAST_FLAG_LEVEL_LAYOUT)
+        const uint32_t mode = (flags & PHAST_FLAG_DIAGONAL) ? LAYOUT_DIAGONAL
+                              : (flags & PHAST_FLAG_LEVEL_LAYOUT)
                                   ? ((flags & PHAST_FLAG_BFS_IN_LEVEL) ? LAYOUT_LEVELS_BFS : LAYOUT_LEVELS)
                                   : LAYOUT_WAVEFRONT;
         rc = layout_build(R, first, head, mode, delta, h->L);
@@ -661,7 +690,7 @@ int phast_save(const phast_ctx* h, const char* path) {
     if (!f) return PHAST_EIO;
     const Layout& L = h->L;
     uint64_t hdr[10] = {h->n, L.levels, h->m, h->shortcuts, h->rounds, L.dn_arc.size(), L.up_arc.size(),
-                        L.mode, L.delta, L.lvl_off.size()};
+                        L.mode | ((uint64_t)L.cut << 32), L.delta, L.lvl_off.size()};
     auto wr = [&](const void* p, size_t sz, size_t cnt) { return std::fwrite(p, sz, cnt, f) == cnt; };
     bool ok = wr(MAGIC, 1, 8) && wr(hdr, 8, 10) && wr(&h->build_seconds, 8, 1) && wr(L.perm.data(), 4, h->n) &&
               wr(L.level.data(), 4, h->n) && wr(L.lvl_off.data(), 4, L.lvl_off.size()) &&
@@ -687,7 +716,7 @@ int phast_load(const char* path, uint32_t flags, phast_ctx** out) {
         try {
             h->n = (uint32_t)hdr[0]; L.levels = (uint32_t)hdr[1]; h->m = hdr[2];
             h->shortcuts = hdr[3]; h->rounds = (uint32_t)hdr[4];
-            L.mode = (uint32_t)hdr[7]; L.delta = (uint32_t)hdr[8];
+            L.mode = (uint32_t)hdr[7]; L.cut = (uint32_t)(hdr[7] >> 32); L.delta = (uint32_t)hdr[8];
             L.perm.resize(h->n); L.iperm.resize(h->n); L.level.resize(h->n);
             L.lvl_off.resize(hdr[9]);
             L.dn_first.resize((size_t)h->n + 1); L.up_first.resize((size_t)h->n + 1);

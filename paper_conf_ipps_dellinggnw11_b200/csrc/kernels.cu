@@ -245,11 +245,14 @@ constexpr int SWEEP_THREADS = 256;
 // on level 0, profiles/r1_launches_*).  Launched with programmatic dependent launch:
 // the next level's grid is launched while this one drains and blocks in
 // griddepcontrol.wait until this grid's rows are visible.
-template <int K, bool DIAM, bool STORE, bool STREAM>
+// TB (segments that mix levels): per vertex, tails are stored normally (re-read soon,
+// from L2) and the other rows with evict-first stores (diameter: not stored at all).
+template <int K, bool DIAM, bool STORE, bool STREAM, bool TB>
 __global__ void __launch_bounds__(SWEEP_THREADS) sweep_kernel(const uint32_t* __restrict__ first,
                                                                const uint2* __restrict__ arcs,
                                                                uint32_t* __restrict__ d,
                                                                const uint32_t* __restrict__ flags,
+                                                               const uint32_t* __restrict__ tail_bits,
                                                                uint32_t vbeg, uint32_t vend,
                                                                uint32_t* __restrict__ diam) {
     using T = typename RowT<K>::T;
@@ -273,7 +276,11 @@ __global__ void __launch_bounds__(SWEEP_THREADS) sweep_kernel(const uint32_t* __
             const T x = __ldg(reinterpret_cast<const T*>(d + (size_t)a.x * K) + lane);
             acc = relax(acc, x, a.y);
         }
-        if constexpr (STORE) {
+        if constexpr (TB) {
+            T* p = reinterpret_cast<T*>(d + (size_t)v * K) + lane;
+            if ((__ldg(&tail_bits[v >> 5]) >> (v & 31)) & 1u) *p = acc;
+            else if constexpr (!DIAM) st_stream(p, acc);
+        } else if constexpr (STORE) {
             T* p = reinterpret_cast<T*>(d + (size_t)v * K) + lane;
             if constexpr (STREAM) st_stream(p, acc); else *p = acc;
         }
@@ -292,7 +299,7 @@ __global__ void __launch_bounds__(SWEEP_THREADS) sweep_kernel(const uint32_t* __
     }
 }
 
-template <int K, bool DIAM, bool STORE, bool STREAM>
+template <int K, bool DIAM, bool STORE, bool STREAM, bool TB>
 cudaError_t sweep_launch(const DevImage& g, uint32_t vbeg, uint32_t vend, uint32_t* dist, uint32_t* diam,
                          cudaStream_t st) {
     constexpr uint32_t G = K / RowT<K>::W;
@@ -311,22 +318,25 @@ cudaError_t sweep_launch(const DevImage& g, uint32_t vbeg, uint32_t vend, uint32
     attr[0].val.programmaticStreamSerializationAllowed = 1;
     cfg.attrs = attr;
     cfg.numAttrs = 1;
-    cudaError_t e = cudaLaunchKernelEx(&cfg, sweep_kernel<K, DIAM, STORE, STREAM>, g.dn_first, g.dn_arc, dist,
-                                       (const uint32_t*)g.flags, vbeg, vend, diam);
+    cudaError_t e = cudaLaunchKernelEx(&cfg, sweep_kernel<K, DIAM, STORE, STREAM, TB>, g.dn_first, g.dn_arc, dist,
+                                       (const uint32_t*)g.flags, g.tail_bits, vbeg, vend, diam);
     g_launches++;
     return e;
 }
 
 template <int K>
 cudaError_t sweep_k(const DevImage& g, uint32_t vbeg, uint32_t vend, uint32_t* dist, uint32_t* diam, bool store,
-                    bool last, cudaStream_t st) {
+                    bool last, bool by_tail, cudaStream_t st) {
+    if (by_tail)
+        return diam ? sweep_launch<K, true, true, false, true>(g, vbeg, vend, dist, diam, st)
+                    : sweep_launch<K, false, true, false, true>(g, vbeg, vend, dist, diam, st);
     if (diam) {
-        if (!store) return sweep_launch<K, true, false, false>(g, vbeg, vend, dist, diam, st);
-        return last ? sweep_launch<K, true, true, true>(g, vbeg, vend, dist, diam, st)
-                    : sweep_launch<K, true, true, false>(g, vbeg, vend, dist, diam, st);
+        if (!store) return sweep_launch<K, true, false, false, false>(g, vbeg, vend, dist, diam, st);
+        return last ? sweep_launch<K, true, true, true, false>(g, vbeg, vend, dist, diam, st)
+                    : sweep_launch<K, true, true, false, false>(g, vbeg, vend, dist, diam, st);
     }
-    return last ? sweep_launch<K, false, true, true>(g, vbeg, vend, dist, diam, st)
-                : sweep_launch<K, false, true, false>(g, vbeg, vend, dist, diam, st);
+    return last ? sweep_launch<K, false, true, true, false>(g, vbeg, vend, dist, diam, st)
+                : sweep_launch<K, false, true, false, false>(g, vbeg, vend, dist, diam, st);
 }
 
 // ------------------------------------------------------------------ a3+a4 persistent sweep
@@ -1013,6 +1023,153 @@ int wave_occupancy() {
     return b > 0 ? b : 1;
 }
 
+// ------------------------------------------------------------------ a3+a4 segment barriers (variant 6)
+// ONE launch for a segmented layout (levels, or the diagonal layout's levels +
+// diagonals; layout.h: lvl_off): the grid walks the segments in order, each one
+// exactly like one per-level launch (grid-stride (vertex, 16-byte lane) items,
+// PAPER.md:18 §VI), and meets at a grid-wide barrier between segments -- the
+// paper's kernel boundary between levels (§VI "The CPU starts, for each
+// level i, a kernel on the GPU") without its launch and drain cost.  The barrier is
+// one arrival per CTA on a per-segment counter (monotone over launches: it reaches
+// grid * epoch) and an acquire spin by thread 0, which also drops the SM's L1 lines
+// (tail rows are read with plain L1-cached loads; the lines of rows finalised in
+// the segment just completed may be stale there).  All CTAs are resident (grid
+// sized by the occupancy calculator); a 4 s watchdog turns a stuck barrier into
+// PHAST_ECUDA instead of a hang.
+// BATCH: the next item's offsets are prefetched while the current one gathers, and
+// up to 4 arcs (then their 4 tail rows) are loaded together: two dependent round
+// trips per item instead of 1 + 2 * degree.
+template <int K, bool DIAM, bool BATCH>
+__global__ void __launch_bounds__(SWEEP_THREADS, BATCH ? 6 : 8) sweep_seg_kernel(const uint32_t* __restrict__ first,
+                                                                  const uint2* __restrict__ arcs,
+                                                                  uint32_t* __restrict__ d,
+                                                                  const uint32_t* __restrict__ flags,
+                                                                  const uint32_t* __restrict__ tail_bits,
+                                                                  SweepPlan p, uint32_t epoch,
+                                                                  uint32_t* __restrict__ diam) {
+    using T = typename RowT<K>::T;
+    constexpr uint32_t G = K / RowT<K>::W;   // lanes per vertex
+    const uint32_t nseg = p.nchunks, tb_from = p.chunk_cap;
+    const uint32_t target = gridDim.x * epoch;
+    const uint32_t stride = gridDim.x * SWEEP_THREADS;   // host: n * G < 2^31
+    uint32_t mx = 0;
+    uint32_t vb = __ldg(&p.chunk_v[0]);
+    for (uint32_t j = 0; j < nseg; j++) {
+        const uint32_t ve = __ldg(&p.chunk_v[j + 1]);
+        const bool tb = j >= tb_from, last = p.stream_last && j + 1 == nseg;
+        const uint32_t total = (ve - vb) * G;
+        uint32_t t = blockIdx.x * SWEEP_THREADS + threadIdx.x;
+        uint32_t nf0 = 0, nf1 = 0;
+        if (BATCH && t < total) {
+            const uint32_t v = vb + (t / G);
+            nf0 = __ldg(&first[v]);
+            nf1 = __ldg(&first[v + 1]);
+        }
+        for (; t < total; t += stride) {
+            const uint32_t v = vb + (t / G);
+            const uint32_t lane = (t % G);
+            T acc = inf_row<T>();
+            if ((__ldg(&flags[v >> 5]) >> (v & 31)) & 1u)   // visited by an upward search (§IV-C)
+                acc = __ldcg(reinterpret_cast<const T*>(d + (size_t)v * K) + lane);
+            if constexpr (BATCH) {
+                const uint32_t e0 = nf0, e1 = nf1;
+                if (t + stride < total) {                    // prefetch the next item's offsets
+                    const uint32_t vn = vb + ((t + stride) / G);
+                    nf0 = __ldg(&first[vn]);
+                    nf1 = __ldg(&first[vn + 1]);
+                }
+                for (uint32_t e = e0; e < e1; e += 4) {
+                    uint2 a[4];
+                    T x[4];
+#pragma unroll
+                    for (uint32_t r = 0; r < 4; r++)
+                        if (e + r < e1) a[r] = __ldg(&arcs[e + r]);
+#pragma unroll
+                    for (uint32_t r = 0; r < 4; r++)
+                        if (e + r < e1) x[r] = __ldca(reinterpret_cast<const T*>(d + (size_t)a[r].x * K) + lane);
+#pragma unroll
+                    for (uint32_t r = 0; r < 4; r++)
+                        if (e + r < e1) acc = relax(acc, x[r], a[r].y);
+                }
+            } else {
+                const uint32_t e0 = __ldg(&first[v]), e1 = __ldg(&first[v + 1]);
+#pragma unroll 4
+                for (uint32_t e = e0; e < e1; e++) {
+                    const uint2 a = __ldg(&arcs[e]);
+                    const T x = __ldca(reinterpret_cast<const T*>(d + (size_t)a.x * K) + lane);
+                    acc = relax(acc, x, a.y);
+                }
+            }
+            T* q = reinterpret_cast<T*>(d + (size_t)v * K) + lane;
+            if (tb) {
+                if ((__ldg(&tail_bits[v >> 5]) >> (v & 31)) & 1u) *q = acc;   // re-read soon, from L2
+                else if (!DIAM) st_stream(q, acc);                             // never re-read
+            } else if (last) {
+                if (!DIAM) st_stream(q, acc);                                  // level 0: nobody's tail
+            } else {
+                *q = acc;
+            }
+            if constexpr (DIAM) mx = max(mx, fmax_of(acc));
+        }
+        if (j + 1 < nseg) {   // grid barrier: segment j complete and visible
+            __syncthreads();
+            if (threadIdx.x == 0) {
+                asm volatile("red.release.gpu.global.add.u32 [%0], 1;" ::"l"(&p.wave_done[j]) : "memory");
+                // relaxed spin (an acquire load per poll would drop the L1 lines of the
+                // CTAs still working on this SM), then one acquire fence
+                if (ld_flag(&p.wave_done[j]) < target) {
+                    uint32_t ns = 32;
+                    const uint64_t t0 = globaltimer_ns();
+                    while (ld_flag(&p.wave_done[j]) < target) {
+                        __nanosleep(ns);
+                        ns = min(ns * 2, 256u);
+                        if ((*(volatile uint32_t*)p.err & 2u) || globaltimer_ns() - t0 > 4000000000ull) {
+                            atomicOr(p.err, 2u);   // watchdog: report, never hang
+                            break;
+                        }
+                    }
+                }
+                asm volatile("fence.acq_rel.gpu;" ::: "memory");
+            }
+            __syncthreads();
+        }
+        vb = ve;
+    }
+    if constexpr (DIAM) {
+        __shared__ uint32_t wmax[SWEEP_THREADS / 32];
+        mx = __reduce_max_sync(0xFFFFFFFFu, mx);
+        if ((threadIdx.x & 31) == 0) wmax[threadIdx.x >> 5] = mx;
+        __syncthreads();
+        if (threadIdx.x < 32) {
+            uint32_t w = threadIdx.x < SWEEP_THREADS / 32 ? wmax[threadIdx.x] : 0u;
+            w = __reduce_max_sync(0xFFFFFFFFu, w);
+            if (threadIdx.x == 0 && w) atomicMax(diam, w);
+        }
+    }
+}
+
+bool seg_batch() {
+    static int b = -1;
+    if (b < 0) {
+        const char* e = std::getenv("PHAST_SEG_BATCH");
+        b = e ? std::atoi(e) != 0 : 1;
+    }
+    return b != 0;
+}
+
+template <int K, bool DIAM>
+int seg_occupancy() {
+    int b = 0;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, seg_batch() ? (const void*)sweep_seg_kernel<K, DIAM, true>
+                                                                      : (const void*)sweep_seg_kernel<K, DIAM, false>,
+                                                      SWEEP_THREADS, 0) !=
+        cudaSuccess) {
+        cudaGetLastError();
+        return 1;
+    }
+    return b > 0 ? b : 1;
+}
+
 // ------------------------------------------------------------------ a3+a4 pipelined gather (variant 3)
 // CTA chunks on the wavefront layout with a one-chunk lookahead: while chunk c is
 // reduced from shared memory, the tail rows of the CTA's next chunk are already in
@@ -1268,6 +1425,17 @@ cudaError_t persistent_k(const DevImage& g, const SweepPlan& p, uint32_t epoch, 
             return cudaGetLastError();
         }
     }
+    if (p.variant == 6) {
+        const bool b = seg_batch();
+        if (diam)
+            (b ? sweep_seg_kernel<K, true, true> : sweep_seg_kernel<K, true, false>)<<<p.grid, SWEEP_THREADS, 0, st>>>(
+                g.dn_first, g.dn_arc, dist, g.flags, g.tail_bits, p, epoch, diam);
+        else
+            (b ? sweep_seg_kernel<K, false, true> : sweep_seg_kernel<K, false, false>)<<<p.grid, SWEEP_THREADS, 0, st>>>(
+                g.dn_first, g.dn_arc, dist, g.flags, g.tail_bits, p, epoch, nullptr);
+        g_launches++;
+        return cudaGetLastError();
+    }
     if (p.variant == 5) {
         if (diam)
             sweep_wave_kernel<K, true><<<p.grid, SWEEP_THREADS, 0, st>>>(g.dn_first, g.dn_arc, dist, g.flags,
@@ -1366,8 +1534,8 @@ cudaError_t launch_seed(const DevImage& g, uint32_t k, uint32_t slot, uint32_t* 
 }
 
 cudaError_t launch_sweep_level(const DevImage& g, uint32_t k, uint32_t vbeg, uint32_t vend, uint32_t* dist,
-                               uint32_t* diam, bool store, bool last_level, cudaStream_t st) {
-#define CALL_SW(K) sweep_k<K>(g, vbeg, vend, dist, diam, store, last_level, st)
+                               uint32_t* diam, bool store, bool last_level, bool by_tail, cudaStream_t st) {
+#define CALL_SW(K) sweep_k<K>(g, vbeg, vend, dist, diam, store, last_level, by_tail, st)
     PHAST_K_SWITCH(k, CALL_SW)
 #undef CALL_SW
 }
@@ -1420,7 +1588,8 @@ uint32_t sweep_chunk_vertices(uint32_t k) {
 
 int sweep_blocks_per_sm(uint32_t k, bool diam, uint32_t variant) {
 #define OCC(K)                                                                                               \
-    (variant == 5 ? (diam ? wave_occupancy<K, true>() : wave_occupancy<K, false>()) :                         \
+    (variant == 6 ? (diam ? seg_occupancy<K, true>() : seg_occupancy<K, false>()) :                           \
+     variant == 5 ? (diam ? wave_occupancy<K, true>() : wave_occupancy<K, false>()) :                         \
      variant == 4 ? (diam ? wpipe_occupancy<K, true>() : wpipe_occupancy<K, false>()) :                       \
      variant == 3 ? (diam ? pipe_occupancy<K, true>() : pipe_occupancy<K, false>()) :                         \
      variant == 2 ? (diam ? warp_occupancy<K, true>() : warp_occupancy<K, false>()) :                         \

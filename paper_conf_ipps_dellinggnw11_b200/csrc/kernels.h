@@ -39,16 +39,20 @@ cudaError_t launch_upward(const DevImage& g, const Sources& src, uint32_t k, uin
 cudaError_t launch_seed(const DevImage& g, uint32_t k, uint32_t slot, uint32_t* dist, cudaStream_t st);
 // a3: one level [vbeg, vend) of the downward sweep; diam != nullptr fuses the max (a5);
 // store == false skips the row stores (diameter mode, level 0 rows are never read).
+// by_tail: the segment mixes levels; store each row by its tail bit (tails normally,
+// others evict-first; diameter: others not stored).
 cudaError_t launch_sweep_level(const DevImage& g, uint32_t k, uint32_t vbeg, uint32_t vend,
                                uint32_t* dist, uint32_t* diam, bool store, bool last_level,
-                               cudaStream_t st);
+                               bool by_tail, cudaStream_t st);
 // Plan of the persistent (single-launch) sweep for one k: the internal order is cut
 // into chunks of consecutive ids (no chunk contains both ends of a G-down arc);
 // chunk c runs on CTA c % grid in iteration c / grid and depends on iteration
 // chunk_dep[c] - 1 (0 = no dependency).
 struct SweepPlan {
     uint32_t k = 0, nchunks = 0, grid = 0, iters = 0, chunk_cap = 0;
-    uint32_t variant = 2;   // 5: warp waves (wave plan, per-wave sub-counters); 4: warp pipeline; 3: pipelined gather; 2: warp dataflow; 1: CTA waves + bulk-staged arcs; 0: CTA waves
+    uint32_t variant = 2;   // 6: segment barriers (chunk_v = segment offsets, nchunks = segments,
+                            //    chunk_cap = first segment stored by tail bit, wave_done = per-segment counters);
+                            // 5: warp waves (wave plan, per-wave sub-counters); 4: warp pipeline; 3: pipelined gather; 2: warp dataflow; 1: CTA waves + bulk-staged arcs; 0: CTA waves
     // variant 3 (pipelined gather): per slot {vbeg, vend, e0 = first[vbeg], e1 = first[vend]}
     const uint4* pinfo = nullptr;
     // variant 2 (warp dataflow)
@@ -62,6 +66,7 @@ struct SweepPlan {
                                             // variant 5: [8][chunk_cap] sub-counters, chunk_cap = stride
     const uint4* wdesc = nullptr;           // variant 5: [iters * workers] chunk descriptors (plan_waves)
     uint32_t* err = nullptr;                // sticky device error word (bit 1: dependency watchdog)
+    uint32_t stream_last = 1;               // variant 6: the last segment's rows are nobody's tail
 };
 // vertices per chunk and CTAs per SM the persistent sweep uses for this k
 uint32_t sweep_chunk_vertices(uint32_t k);   // max vertices per chunk

@@ -7,7 +7,19 @@
 // (§IV-A), so that the sweep is "a simple linear sweep in increasing
 // order of IDs".  LAYOUT_LEVELS reproduces that.
 //
-// LAYOUT_WAVEFRONT (default) keeps the linear sweep but chooses a
+// LAYOUT_DIAGONAL keeps the paper's level order for the few vertices of the top
+// levels (>= cut) and interleaves the bottom levels -- which hold almost all
+// vertices and whose G-down arcs are short (level-0 in-arcs are original arcs) -- in
+// "diagonals": with band(v) = rank(v) / delta (BFS rank, below) and per-level offsets
+// o(l), key(v) = band(v) + o(L(v)); o is the smallest non-negative offset with
+// key(tail) < key(head) on every bottom arc, computed top-down by level.  Diagonal j
+// holds the bottom vertices with key j, so a diagonal never holds both ends of an arc,
+// and each diagonal touches only a few consecutive bands of every bottom level: a
+// tail row is written shortly before its bottom-level heads read it and stays in L2,
+// where a level-by-level pass re-reads it from HBM once per level of its heads
+// (profiles/r1_l2sim.md).
+//
+// LAYOUT_WAVEFRONT keeps the linear sweep but chooses a
 // different topological order, one that keeps label rows in the B200's L2 cache.
 //   rank(v) = BFS discovery order of the input graph (undirected) from a
 //             pseudo-peripheral vertex: a spatial sweep line across the network.
@@ -103,6 +115,42 @@ int layout_build(const ChResult& R, const uint64_t* first, const uint32_t* head,
             std::sort(by.begin(), by.end(), [&](uint32_t a, uint32_t b) { return rank[a] < rank[b]; });
         }
         for (uint32_t v : by) order[pos[R.level[v]]++] = v;
+    } else if (mode == LAYOUT_DIAGONAL) {
+        std::vector<uint32_t> rank = bfs_rank(n, first, head);
+        std::vector<uint32_t> cnt(levels, 0);
+        for (uint32_t v = 0; v < n; v++) cnt[R.level[v]]++;
+        // cut: the lowest level whose part above holds at most n / 256 vertices
+        uint32_t cut = levels;
+        {
+            uint64_t above = 0;
+            while (cut > 1 && above + cnt[cut - 1] <= n / 256) above += cnt[--cut];
+        }
+        L.cut = cut;
+        const uint32_t band_w = std::max(1u, delta);
+        auto band = [&](uint32_t v) { return (int64_t)(rank[v] / band_w); };
+        std::vector<int64_t> o(levels, 0);
+        {   // offsets top-down: o(l) = max over bottom arcs (t -> v), L(v) = l, of o(L(t)) + band(t) - band(v) + 1
+            std::vector<std::vector<uint32_t>> by_level(cut);
+            for (uint32_t v = 0; v < n; v++)
+                if (R.level[v] < cut) by_level[R.level[v]].push_back(v);
+            for (int64_t l = (int64_t)cut - 1; l >= 0; l--)
+                for (uint32_t v : by_level[l])
+                    for (uint64_t e = R.dn_first[v]; e < R.dn_first[v + 1]; e++) {
+                        const uint32_t t = R.dn_tail[e];
+                        if (R.level[t] < cut) o[l] = std::max(o[l], o[R.level[t]] + band(t) - band(v) + 1);
+                    }
+        }
+        std::iota(order.begin(), order.end(), 0u);
+        auto key = [&](uint32_t v) { return R.level[v] >= cut ? -1 - (int64_t)R.level[v] : band(v) + o[R.level[v]]; };
+        std::sort(order.begin(), order.end(), [&](uint32_t a, uint32_t b) {
+            const int64_t ka = key(a), kb = key(b);
+            if (ka != kb) return ka < kb;
+            if (R.level[a] != R.level[b]) return R.level[a] > R.level[b];
+            return rank[a] < rank[b];
+        });
+        L.lvl_off.assign(1, 0);
+        for (uint32_t r = 1; r <= n; r++)
+            if (r == n || key(order[r]) != key(order[r - 1])) L.lvl_off.push_back(r);
     } else {
         std::vector<uint32_t> rank = bfs_rank(n, first, head);
         std::vector<int64_t> key(n);
@@ -170,6 +218,14 @@ int layout_build(const ChResult& R, const uint64_t* first, const uint32_t* head,
             L.up_arc[p++] = Arc{L.perm[w], R.up_len[e]};
         }
         std::sort(L.up_arc.begin() + L.up_first[r], L.up_arc.begin() + L.up_first[r + 1], by_x);
+    }
+    if (ok && !L.lvl_off.empty()) {   // segments: no G-down arc inside one segment
+        std::vector<uint32_t> seg(n);
+        for (uint32_t j = 0; j + 1 < L.lvl_off.size(); j++)
+            for (uint32_t r = L.lvl_off[j]; r < L.lvl_off[j + 1]; r++) seg[r] = j;
+        for (uint32_t r = 0; r < n && ok; r++)
+            for (uint32_t e = L.dn_first[r]; e < L.dn_first[r + 1]; e++)
+                if (!(seg[L.dn_arc[e].x] < seg[r])) { ok = false; break; }
     }
     return ok ? 0 : kEinternal;
 }

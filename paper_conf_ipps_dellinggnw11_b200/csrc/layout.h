@@ -12,6 +12,7 @@ enum LayoutMode : uint32_t {
     LAYOUT_WAVEFRONT = 0,   // skewed spatial wavefront (default)
     LAYOUT_LEVELS = 1,      // the paper's: level descending, input (DFS) order within a level
     LAYOUT_LEVELS_BFS = 2,  // level descending, BFS (spatial sweep) order within a level
+    LAYOUT_DIAGONAL = 3,    // top levels as LEVELS_BFS, then the bottom levels in banded diagonals
 };
 
 struct Arc {
@@ -25,7 +26,12 @@ struct Layout {
     std::vector<uint32_t> perm;      // internal_of_original
     std::vector<uint32_t> iperm;     // original_of_internal
     std::vector<uint32_t> level;     // CH level L of every internal id (0 = lowest)
-    std::vector<uint32_t> lvl_off;   // LAYOUT_LEVELS only: [levels+1], j = 0 is the top level
+    // Segments of the per-segment sweep, in processing order: [segments+1] internal-id
+    // offsets; no G-down arc has both ends in one segment.  LAYOUT_LEVELS(_BFS): one
+    // segment per level, j = 0 the top level.  LAYOUT_DIAGONAL: the top levels (>= cut)
+    // one each, then one per diagonal.  Empty for LAYOUT_WAVEFRONT.
+    std::vector<uint32_t> lvl_off;
+    uint32_t cut = 0;                // LAYOUT_DIAGONAL: levels >= cut form the top part
     std::vector<uint32_t> dn_first, up_first;   // [n+1]
     std::vector<Arc> dn_arc, up_arc;
 };

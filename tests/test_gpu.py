@@ -123,13 +123,17 @@ def test_upward_global_fallback_and_overflow(monkeypatch):
 
 @pytest.mark.parametrize("mode,level_layout,delta", [("levels", True, 0), ("levels", "bfs", 0),
                                                      ("levels-hybrid", True, 0), ("levels-flat", "bfs", 0),
+                                                     ("levels-hybrid", "bfs", 0), ("levels-hybrid", "diagonal", 0),
                                                      ("warp", True, 0), ("staged", True, 0),
                                                      ("warp", False, 0), ("persistent", False, 0),
                                                      ("wpipe", False, 0), ("wpipe", False, 300), ("wpipe", True, 0),
                                                      ("pipe", False, 0), ("pipe", False, 300), ("pipe", True, 0),
                                                      ("staged", False, 0), ("warp", False, 300),
                                                      ("staged", False, 300), ("wave", False, 0),
-                                                     ("wave", False, 300), ("wave", True, 0), ("wave", "bfs", 0)])
+                                                     ("wave", False, 300), ("wave", True, 0), ("wave", "bfs", 0),
+                                                     ("levels", "diagonal", 0), ("levels", "diagonal", 500),
+                                                     ("segments", True, 0), ("segments", "bfs", 0),
+                                                     ("segments", "diagonal", 0), ("segments", "diagonal", 500)])
 def test_sweep_modes(monkeypatch, mode, level_layout, delta):
     """Every schedule is bit-exact: one launch per level on the paper's level layout
     (§VI); the single persistent launch as warp dataflow (default) or CTA
@@ -143,8 +147,8 @@ def test_sweep_modes(monkeypatch, mode, level_layout, delta):
         mode = "levels"
     monkeypatch.setenv("PHAST_SWEEP", mode)
     g = phastgen.road(120_000, seed=33)
-    with P.Phast.from_graph(g, level_layout=bool(level_layout), bfs_in_level=level_layout == "bfs",
-                            delta=delta) as h:
+    with P.Phast.from_graph(g, level_layout=level_layout in (True, "bfs"), bfs_in_level=level_layout == "bfs",
+                            diagonal=level_layout == "diagonal", delta=delta) as h:
         for k in (1, 2, 16, 64):
             src = phastgen.sources(g.n, k, seed=900 + k)
             assert np.array_equal(gpu_trees(h, src), oracle.sssp_many(g, src)), k

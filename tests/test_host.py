@@ -64,7 +64,7 @@ def test_host_hierarchy_sweep_equals_oracle(name):
 
 
 LAYOUTS = {"wavefront": {}, "levels": dict(level_layout=True),
-           "levels-bfs": dict(level_layout=True, bfs_in_level=True)}
+           "levels-bfs": dict(level_layout=True, bfs_in_level=True), "diagonal": dict(diagonal=True)}
 
 
 @pytest.mark.parametrize("layout", sorted(LAYOUTS))
@@ -92,8 +92,8 @@ def test_layout_invariants(name, layout):
     assert np.array_equal(np.sort(perm), np.arange(n, dtype=np.uint32))
     # level-0 vertices are never tails (their rows need not be stored in diameter mode)
     assert np.all(lev[tails] > 0)
-    assert h.info().layout == {"wavefront": 0, "levels": 1, "levels-bfs": 2}[layout]
-    if level_layout:
+    assert h.info().layout == {"wavefront": 0, "levels": 1, "levels-bfs": 2, "diagonal": 3}[layout]
+    if layout in ("levels", "levels-bfs"):
         assert np.all(np.diff(lev) <= 0)                 # levels contiguous, highest first
     if layout == "levels":
         inv = np.empty_like(perm)
