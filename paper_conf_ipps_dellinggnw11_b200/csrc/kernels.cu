@@ -20,6 +20,7 @@
 // No tensor cores: the loop is an integer (min,+) gather with no reuse.
 #include <atomic>
 #include <cstdio>
+#include <cstdlib>
 
 #include "kernels.h"
 
@@ -247,8 +248,10 @@ constexpr int SWEEP_THREADS = 256;
 // griddepcontrol.wait until this grid's rows are visible.
 // TB (segments that mix levels): per vertex, tails are stored normally (re-read soon,
 // from L2) and the other rows with evict-first stores (diameter: not stored at all).
-template <int K, bool DIAM, bool STORE, bool STREAM, bool TB>
-__global__ void __launch_bounds__(SWEEP_THREADS) sweep_kernel(const uint32_t* __restrict__ first,
+// AB > 1: up to AB arcs of the item (then their AB tail rows) are loaded together,
+// so an item costs two dependent round trips after its offsets, not 2 * degree.
+template <int K, bool DIAM, bool STORE, bool STREAM, bool TB, int AB>
+__global__ void __launch_bounds__(SWEEP_THREADS, AB >= 3 ? 6 : 8) sweep_kernel(const uint32_t* __restrict__ first,
                                                                const uint2* __restrict__ arcs,
                                                                uint32_t* __restrict__ d,
                                                                const uint32_t* __restrict__ flags,
@@ -260,21 +263,36 @@ __global__ void __launch_bounds__(SWEEP_THREADS) sweep_kernel(const uint32_t* __
     constexpr uint32_t G = K / W;   // lanes per vertex
     asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
     asm volatile("griddepcontrol.wait;" ::: "memory");          // previous level complete and visible
-    const uint64_t total = (uint64_t)(vend - vbeg) * G;
+    const uint32_t total = (vend - vbeg) * G;   // host: < 2^31 (sweep_launch splits longer segments)
     uint32_t mx = 0;
-    for (uint64_t t = (uint64_t)blockIdx.x * SWEEP_THREADS + threadIdx.x; t < total;
-         t += (uint64_t)gridDim.x * SWEEP_THREADS) {
-        const uint32_t v = vbeg + (uint32_t)(t / G);
-        const uint32_t lane = (uint32_t)(t % G);
+    for (uint32_t t = blockIdx.x * SWEEP_THREADS + threadIdx.x; t < total; t += gridDim.x * SWEEP_THREADS) {
+        const uint32_t v = vbeg + t / G;
+        const uint32_t lane = t % G;
         T acc = inf_row<T>();
         if ((__ldg(&flags[v >> 5]) >> (v & 31)) & 1u)   // visited by an upward search
             acc = __ldg(reinterpret_cast<const T*>(d + (size_t)v * K) + lane);
         const uint32_t e0 = __ldg(&first[v]), e1 = __ldg(&first[v + 1]);
+        if constexpr (AB == 1) {
 #pragma unroll 4
-        for (uint32_t e = e0; e < e1; e++) {
-            const uint2 a = __ldg(&arcs[e]);
-            const T x = __ldg(reinterpret_cast<const T*>(d + (size_t)a.x * K) + lane);
-            acc = relax(acc, x, a.y);
+            for (uint32_t e = e0; e < e1; e++) {
+                const uint2 a = __ldg(&arcs[e]);
+                const T x = __ldg(reinterpret_cast<const T*>(d + (size_t)a.x * K) + lane);
+                acc = relax(acc, x, a.y);
+            }
+        } else {
+            for (uint32_t e = e0; e < e1; e += AB) {
+                uint2 a[AB];
+                T x[AB];
+#pragma unroll
+                for (int r = 0; r < AB; r++)
+                    if (e + r < e1) a[r] = __ldg(&arcs[e + r]);
+#pragma unroll
+                for (int r = 0; r < AB; r++)
+                    if (e + r < e1) x[r] = __ldg(reinterpret_cast<const T*>(d + (size_t)a[r].x * K) + lane);
+#pragma unroll
+                for (int r = 0; r < AB; r++)
+                    if (e + r < e1) acc = relax(acc, x[r], a[r].y);
+            }
         }
         if constexpr (TB) {
             T* p = reinterpret_cast<T*>(d + (size_t)v * K) + lane;
@@ -299,10 +317,25 @@ __global__ void __launch_bounds__(SWEEP_THREADS) sweep_kernel(const uint32_t* __
     }
 }
 
+int arc_batch() {   // PHAST_ARC_BATCH: 1, 2 (default), 3 or 4 (sweep_kernel AB)
+    static int b = 0;
+    if (!b) {
+        const char* e = std::getenv("PHAST_ARC_BATCH");
+        b = e ? std::atoi(e) : 2;
+        if (b < 1 || b > 4) b = 2;
+    }
+    return b;
+}
+
 template <int K, bool DIAM, bool STORE, bool STREAM, bool TB>
 cudaError_t sweep_launch(const DevImage& g, uint32_t vbeg, uint32_t vend, uint32_t* dist, uint32_t* diam,
                          cudaStream_t st) {
     constexpr uint32_t G = K / RowT<K>::W;
+    constexpr uint32_t VMAX = (1u << 31) / G;   // 32-bit item indices in the kernel
+    if (vend - vbeg > VMAX) {                    // a level has no internal arcs: split it freely
+        cudaError_t e = sweep_launch<K, DIAM, STORE, STREAM, TB>(g, vbeg, vbeg + VMAX, dist, diam, st);
+        return e != cudaSuccess ? e : sweep_launch<K, DIAM, STORE, STREAM, TB>(g, vbeg + VMAX, vend, dist, diam, st);
+    }
     uint64_t total = (uint64_t)(vend - vbeg) * G;
     uint64_t blocks = (total + SWEEP_THREADS - 1) / SWEEP_THREADS;
     uint64_t cap = (uint64_t)num_sms() * 8;
@@ -318,8 +351,13 @@ cudaError_t sweep_launch(const DevImage& g, uint32_t vbeg, uint32_t vend, uint32
     attr[0].val.programmaticStreamSerializationAllowed = 1;
     cfg.attrs = attr;
     cfg.numAttrs = 1;
-    cudaError_t e = cudaLaunchKernelEx(&cfg, sweep_kernel<K, DIAM, STORE, STREAM, TB>, g.dn_first, g.dn_arc, dist,
-                                       (const uint32_t*)g.flags, g.tail_bits, vbeg, vend, diam);
+    const int ab = arc_batch();
+    cudaError_t e = cudaLaunchKernelEx(&cfg, ab == 4 ? sweep_kernel<K, DIAM, STORE, STREAM, TB, 4>
+                                             : ab == 3 ? sweep_kernel<K, DIAM, STORE, STREAM, TB, 3>
+                                             : ab == 2 ? sweep_kernel<K, DIAM, STORE, STREAM, TB, 2>
+                                                       : sweep_kernel<K, DIAM, STORE, STREAM, TB, 1>,
+                                       g.dn_first, g.dn_arc, dist, (const uint32_t*)g.flags, g.tail_bits, vbeg, vend,
+                                       diam);
     g_launches++;
     return e;
 }
