@@ -189,8 +189,7 @@ def main():
 
     g, cfg = build_graph(args.config)
     k = args.k
-    bopts = dict(level_layout=args.layout in ("levels", "levels-bfs"), bfs_in_level=args.layout == "levels-bfs",
-                 diagonal=args.layout == "diagonal", delta=args.delta)
+    bopts = dict(layout=args.layout, delta=args.delta)
     # hierarchy: rank 0 builds (host CH, not the timed target) and shares it via a file
     path = args.cache or f"/tmp/phast_{args.config}_{os.getpid() if world == 1 else 'dist'}.phast"
     if world > 1:
@@ -294,7 +293,7 @@ def main():
             "vs_baseline": None, "dtype": "u32", "data": "synthetic",
             "config": {"workload": f"{args.config}: {cfg['desc']}", "k": k, "trees_per_step_per_gpu": k,
                        "n": info.n, "m": info.m, "m_down": info.m_down, "m_up": info.m_up, "n_tail": info.n_tail,
-                       "levels": info.levels, "layout": ["wavefront", "levels", "levels-bfs", "diagonal"][info.layout],
+                       "levels": info.levels, "layout": P.LAYOUT_NAMES[info.layout],
                        "delta": info.delta, "sweep": os.environ.get("PHAST_SWEEP", "levels" if info.layout else "warp"), "parallelism": f"sources sharded over {world} GPU(s), graph replicated",
                        "l2": f"label array {4 * k * info.n / 1e9:.2f} GB >> 126 MB L2 (no flush needed)",
                        "ch_build_s": round(info.build_seconds, 1)},

@@ -26,6 +26,9 @@ FLAG_HOST_ONLY = 1
 FLAG_LEVEL_LAYOUT = 2
 FLAG_BFS_IN_LEVEL = 4
 FLAG_DIAGONAL = 8
+FLAG_WAVEFRONT = 16
+LAYOUT_FLAGS = {"levels-bfs": 0, "levels": FLAG_LEVEL_LAYOUT, "diagonal": FLAG_DIAGONAL, "wavefront": FLAG_WAVEFRONT}
+LAYOUT_NAMES = {0: "wavefront", 1: "levels", 2: "levels-bfs", 3: "diagonal"}   # phast_info_t.layout
 
 STATUS = {0: "OK", -1: "EINVAL", -2: "ENOMEM", -3: "ECUDA", -4: "ERANGE", -5: "ESTATE", -6: "EIO",
           -7: "EINTERNAL"}
@@ -128,8 +131,7 @@ class Phast:
     """A built hierarchy bound to one CUDA device (phast_ctx)."""
 
     def __init__(self, n=None, first=None, head=None, length=None, *, host_only=False, threads=0,
-                 hop_limit_lo=0, hop_limit_hi=0, settled_cap=0, level_layout=False, bfs_in_level=False, diagonal=False, delta=0,
-                 _handle=None):
+                 hop_limit_lo=0, hop_limit_hi=0, settled_cap=0, layout="levels-bfs", delta=0, _handle=None):
         self._h = None
         if _handle is not None:
             self._h = _handle
@@ -140,8 +142,9 @@ class Phast:
             if head.size == 0:
                 head = np.zeros(1, np.uint32)
                 length = np.zeros(1, np.uint32)
-            flags = ((FLAG_HOST_ONLY if host_only else 0) | (FLAG_LEVEL_LAYOUT if level_layout else 0)
-                     | (FLAG_BFS_IN_LEVEL if bfs_in_level else 0) | (FLAG_DIAGONAL if diagonal else 0))
+            if layout not in LAYOUT_FLAGS:
+                raise ValueError(f"layout must be one of {sorted(LAYOUT_FLAGS)}")
+            flags = (FLAG_HOST_ONLY if host_only else 0) | LAYOUT_FLAGS[layout]
             o = _Opts(hop_limit_lo, hop_limit_hi, settled_cap, threads, flags, delta, 0)
             h = ctypes.c_void_p()
             _check("phast_build", _lib.phast_build(int(n), first.ctypes.data, head.ctypes.data,

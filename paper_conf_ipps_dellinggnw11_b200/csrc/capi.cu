@@ -524,10 +524,11 @@ int phast_build(uint32_t n, const uint64_t* first, const uint32_t* head, const u
         h->m = first[n];
         h->shortcuts = R.shortcuts;
         h->rounds = R.rounds;
-        const uint32_t mode = (flags & PHAST_FLAG_DIAGONAL) ? LAYOUT_DIAGONAL
-                              : (flags & PHAST_FLAG_LEVEL_LAYOUT)
-                                  ? ((flags & PHAST_FLAG_BFS_IN_LEVEL) ? LAYOUT_LEVELS_BFS : LAYOUT_LEVELS)
-                                  : LAYOUT_WAVEFRONT;
+        const uint32_t mode = (flags & PHAST_FLAG_DIAGONAL)    ? LAYOUT_DIAGONAL
+                              : (flags & PHAST_FLAG_WAVEFRONT) ? LAYOUT_WAVEFRONT
+                              : ((flags & PHAST_FLAG_LEVEL_LAYOUT) && !(flags & PHAST_FLAG_BFS_IN_LEVEL))
+                                  ? LAYOUT_LEVELS
+                                  : LAYOUT_LEVELS_BFS;
         rc = layout_build(R, first, head, mode, delta, h->L);
         h->build_seconds = R.seconds;
         if (rc) return rc;

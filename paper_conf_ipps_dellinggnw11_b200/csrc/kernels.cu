@@ -251,7 +251,7 @@ constexpr int SWEEP_THREADS = 256;
 // AB > 1: up to AB arcs of the item (then their AB tail rows) are loaded together,
 // so an item costs two dependent round trips after its offsets, not 2 * degree.
 template <int K, bool DIAM, bool STORE, bool STREAM, bool TB, int AB>
-__global__ void __launch_bounds__(SWEEP_THREADS, AB >= 3 ? 6 : 8) sweep_kernel(const uint32_t* __restrict__ first,
+__global__ void __launch_bounds__(SWEEP_THREADS, AB >= 3 && AB < 8 ? 6 : 8) sweep_kernel(const uint32_t* __restrict__ first,
                                                                const uint2* __restrict__ arcs,
                                                                uint32_t* __restrict__ d,
                                                                const uint32_t* __restrict__ flags,
@@ -279,18 +279,40 @@ __global__ void __launch_bounds__(SWEEP_THREADS, AB >= 3 ? 6 : 8) sweep_kernel(c
                 const T x = __ldg(reinterpret_cast<const T*>(d + (size_t)a.x * K) + lane);
                 acc = relax(acc, x, a.y);
             }
-        } else {
-            for (uint32_t e = e0; e < e1; e += AB) {
-                uint2 a[AB];
-                T x[AB];
+        } else if constexpr (AB >= 8 && RowT<K>::W == 4) {
+            // AB = 8: four arcs per batch, their tail rows copied into shared memory by
+            // cp.async (no registers held by loads in flight), then reduced from there
+            __shared__ __align__(16) uint4 srow[4][SWEEP_THREADS];
+            for (uint32_t e = e0; e < e1; e += 4) {
+                uint2 a[4];
 #pragma unroll
-                for (int r = 0; r < AB; r++)
+                for (int r = 0; r < 4; r++)
                     if (e + r < e1) a[r] = __ldg(&arcs[e + r]);
 #pragma unroll
-                for (int r = 0; r < AB; r++)
+                for (int r = 0; r < 4; r++)
+                    if (e + r < e1)
+                        asm volatile("cp.async.ca.shared.global [%0], [%1], 16;" ::"r"(
+                                         static_cast<uint32_t>(__cvta_generic_to_shared(&srow[r][threadIdx.x]))),
+                                     "l"(reinterpret_cast<const uint4*>(d + (size_t)a[r].x * K) + lane)
+                                     : "memory");
+                asm volatile("cp.async.commit_group;\ncp.async.wait_group 0;" ::: "memory");
+#pragma unroll
+                for (int r = 0; r < 4; r++)
+                    if (e + r < e1) acc = relax(acc, srow[r][threadIdx.x], a[r].y);
+            }
+        } else {
+            for (uint32_t e = e0; e < e1; e += (AB >= 8 ? 4 : AB)) {
+                constexpr int B = AB >= 8 ? 4 : AB;
+                uint2 a[B];
+                T x[B];
+#pragma unroll
+                for (int r = 0; r < B; r++)
+                    if (e + r < e1) a[r] = __ldg(&arcs[e + r]);
+#pragma unroll
+                for (int r = 0; r < B; r++)
                     if (e + r < e1) x[r] = __ldg(reinterpret_cast<const T*>(d + (size_t)a[r].x * K) + lane);
 #pragma unroll
-                for (int r = 0; r < AB; r++)
+                for (int r = 0; r < B; r++)
                     if (e + r < e1) acc = relax(acc, x[r], a[r].y);
             }
         }
@@ -317,13 +339,10 @@ __global__ void __launch_bounds__(SWEEP_THREADS, AB >= 3 ? 6 : 8) sweep_kernel(c
     }
 }
 
-int arc_batch() {   // PHAST_ARC_BATCH: 1, 2 (default), 3 or 4 (sweep_kernel AB)
-    static int b = 0;
-    if (!b) {
-        const char* e = std::getenv("PHAST_ARC_BATCH");
-        b = e ? std::atoi(e) : 2;
-        if (b < 1 || b > 4) b = 2;
-    }
+int arc_batch() {   // PHAST_ARC_BATCH: 1, 2 (default), 3, 4 or 8 (staged; sweep_kernel AB), read per launch
+    const char* e = std::getenv("PHAST_ARC_BATCH");
+    int b = e ? std::atoi(e) : 2;
+    if (b != 8 && (b < 1 || b > 4)) b = 2;
     return b;
 }
 
@@ -352,7 +371,8 @@ cudaError_t sweep_launch(const DevImage& g, uint32_t vbeg, uint32_t vend, uint32
     cfg.attrs = attr;
     cfg.numAttrs = 1;
     const int ab = arc_batch();
-    cudaError_t e = cudaLaunchKernelEx(&cfg, ab == 4 ? sweep_kernel<K, DIAM, STORE, STREAM, TB, 4>
+    cudaError_t e = cudaLaunchKernelEx(&cfg, ab == 8 ? sweep_kernel<K, DIAM, STORE, STREAM, TB, 8>
+                                             : ab == 4 ? sweep_kernel<K, DIAM, STORE, STREAM, TB, 4>
                                              : ab == 3 ? sweep_kernel<K, DIAM, STORE, STREAM, TB, 3>
                                              : ab == 2 ? sweep_kernel<K, DIAM, STORE, STREAM, TB, 2>
                                                        : sweep_kernel<K, DIAM, STORE, STREAM, TB, 1>,
@@ -1186,13 +1206,9 @@ __global__ void __launch_bounds__(SWEEP_THREADS, BATCH ? 6 : 8) sweep_seg_kernel
     }
 }
 
-bool seg_batch() {
-    static int b = -1;
-    if (b < 0) {
-        const char* e = std::getenv("PHAST_SEG_BATCH");
-        b = e ? std::atoi(e) != 0 : 1;
-    }
-    return b != 0;
+bool seg_batch() {   // PHAST_SEG_BATCH (default 0: measured slower, fewer CTAs per SM)
+    const char* e = std::getenv("PHAST_SEG_BATCH");
+    return e && std::atoi(e) != 0;
 }
 
 template <int K, bool DIAM>

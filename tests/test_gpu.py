@@ -124,6 +124,9 @@ def test_upward_global_fallback_and_overflow(monkeypatch):
 @pytest.mark.parametrize("mode,level_layout,delta", [("levels", True, 0), ("levels", "bfs", 0),
                                                      ("levels-hybrid", True, 0), ("levels-flat", "bfs", 0),
                                                      ("levels-hybrid", "bfs", 0), ("levels-hybrid", "diagonal", 0),
+                                                     ("levels-ab1", "bfs", 0), ("levels-ab3", "bfs", 0),
+                                                     ("levels-ab4", "bfs", 0), ("levels-ab8", "bfs", 0),
+                                                     ("levels-ab8", "diagonal", 0),
                                                      ("warp", True, 0), ("staged", True, 0),
                                                      ("warp", False, 0), ("persistent", False, 0),
                                                      ("wpipe", False, 0), ("wpipe", False, 300), ("wpipe", True, 0),
@@ -139,7 +142,10 @@ def test_sweep_modes(monkeypatch, mode, level_layout, delta):
     (§VI); the single persistent launch as warp dataflow (default) or CTA
     waves (with and without bulk-staged arcs), on both layouts, including a small
     wavefront skew (many short dependencies)."""
-    if mode == "levels-hybrid":                  # a few small top levels fused, the rest one launch each
+    if mode.startswith("levels-ab"):            # per-level launches, other arc batch (1, 3, 4, 8 = cp.async staged)
+        monkeypatch.setenv("PHAST_ARC_BATCH", mode[len("levels-ab"):])
+        mode = "levels"
+    elif mode == "levels-hybrid":                # a few small top levels fused, the rest one launch each
         monkeypatch.setenv("PHAST_TOP_THRESH", "3000")
         mode = "levels"
     elif mode == "levels-flat":                  # one launch per level, no fusion
@@ -147,8 +153,8 @@ def test_sweep_modes(monkeypatch, mode, level_layout, delta):
         mode = "levels"
     monkeypatch.setenv("PHAST_SWEEP", mode)
     g = phastgen.road(120_000, seed=33)
-    with P.Phast.from_graph(g, level_layout=level_layout in (True, "bfs"), bfs_in_level=level_layout == "bfs",
-                            diagonal=level_layout == "diagonal", delta=delta) as h:
+    layout = {True: "levels", "bfs": "levels-bfs", False: "wavefront"}.get(level_layout, level_layout)
+    with P.Phast.from_graph(g, layout=layout, delta=delta) as h:
         for k in (1, 2, 16, 64):
             src = phastgen.sources(g.n, k, seed=900 + k)
             assert np.array_equal(gpu_trees(h, src), oracle.sssp_many(g, src)), k
@@ -164,7 +170,7 @@ def test_wave_sweep_every_k(monkeypatch, window):
     monkeypatch.setenv("PHAST_SWEEP", "wave")
     monkeypatch.setenv("PHAST_WAVE_WINDOW", window)
     g = phastgen.road(60_000, seed=35)
-    with P.Phast.from_graph(g, delta=2000) as h:
+    with P.Phast.from_graph(g, layout="wavefront", delta=2000) as h:
         for k in (1, 2, 4, 8, 16, 32, 64):
             for rep in range(2):
                 src = phastgen.sources(g.n, k, seed=950 + k + rep)

@@ -63,8 +63,7 @@ def test_host_hierarchy_sweep_equals_oracle(name):
     assert np.array_equal(got, want)
 
 
-LAYOUTS = {"wavefront": {}, "levels": dict(level_layout=True),
-           "levels-bfs": dict(level_layout=True, bfs_in_level=True), "diagonal": dict(diagonal=True)}
+LAYOUTS = {name: dict(layout=name) for name in ("wavefront", "levels", "levels-bfs", "diagonal")}
 
 
 @pytest.mark.parametrize("layout", sorted(LAYOUTS))
