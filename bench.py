@@ -166,6 +166,8 @@ def main():
                     help="vertex order: wavefront, the paper's level layout (DFS within a level), or level "
                          "layout with BFS order within a level (default)")
     ap.add_argument("--delta", type=int, default=0, help="wavefront skew (0 = library default)")
+    ap.add_argument("--parents", action="store_true",
+                    help="also time the parent-pointer pass (phast_parents, NEXT-1) on the last batch")
     args = ap.parse_args()
     args.warmup = max(3, args.warmup)
     if args.impl == "reference":
@@ -259,6 +261,29 @@ def main():
     except Exception:
         pass
 
+    # NEXT-1: parent pointers of the last timed batch (a separate pass, not in `value`)
+    parents = None
+    if args.parents:
+        par_buf = torch.empty((g.n, k), dtype=torch.int32, device="cuda")
+        last = srcs[args.warmup + args.steps - 1]
+        h.parents(last, dist_buf, out=par_buf, stream=stream)
+        h.sync(stream)
+        p0, p1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        reps = max(1, min(args.steps, 10))
+        p0.record(stream)
+        for _ in range(reps):
+            h.parents(last, dist_buf, out=par_buf, stream=stream)
+        p1.record(stream)
+        h.sync(stream)
+        pms = p0.elapsed_time(p1) / reps
+        m_in = g.m   # original arcs (self-loops, if any, are dropped by the library)
+        B_par = 8 * m_in + 4 * (g.n + 1) + 12 * k * g.n
+        parents = {"ms_per_pass": pms, "alg_bytes": B_par, "achieved_GBps": B_par / (pms / 1e3) / 1e9,
+                   "frac": B_par / (pms / 1e3) / 1e9 / peaks()[0],
+                   "note": "B = 8m + 4(n+1) + 12kn: in-arcs, offsets, own row read, in-neighbour rows read "
+                           "at least once, parent row written"}
+        del par_buf
+
     # end to end through the public host entry point (sources in, all labels out)
     e2e = None
     if args.e2e_steps > 0:
@@ -302,6 +327,7 @@ def main():
                          "alg_bytes_per_sweep": B_alg, "sweep_ms": sweep_ms, "upward_ms": ms_up / max(nb, 1),
                          "peak_source": peak_src},
             "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": launches, "clocks": clk.summary(),
+            **({"parents": parents} if parents else {}),
         }
         print(json.dumps(line), flush=True)
     if world > 1:

@@ -6,7 +6,8 @@ reference` legs may import this package.  The product path
 
 Plain binary-heap Dijkstra on the ORIGINAL graph (§II-A), exact by
 Theorem 3.1 (§III) for what PHAST computes; diameter (PAPER.md:20
-§VII-B); O(n+m) optimality certificate.  See oracle.c for the
+§VII-B); O(n+m) optimality certificate; canonical parent
+pointers by the tight-arc identity (§VII-A, reading R14).  See oracle.c for the
 passage each function follows.  Pins: tests/test_oracle.py.  Parity status of
 every function: pinned.
 """
@@ -34,7 +35,9 @@ def _load():
         lib.oracle_sssp_many.argtypes = [u32, vp, vp, vp, vp, u64, vp, vp, u32]
         lib.oracle_diameter.argtypes = [u32, vp, vp, vp, vp, u64, u32, vp]
         lib.oracle_certify.argtypes = [u32, vp, vp, vp, u32, vp]
-        for f in (lib.oracle_sssp, lib.oracle_sssp_many, lib.oracle_diameter, lib.oracle_certify):
+        lib.oracle_parents.argtypes = [u32, vp, vp, vp, u32, vp, vp]
+        for f in (lib.oracle_sssp, lib.oracle_sssp_many, lib.oracle_diameter, lib.oracle_certify,
+                  lib.oracle_parents):
             f.restype = ctypes.c_int
         _lib = lib
     return _lib
@@ -114,3 +117,16 @@ def certify(g, s: int, d) -> int:
     if rc < 0:
         raise ValueError(f"oracle_certify: {rc}")
     return rc
+
+
+def parents(g, s: int, d=None) -> np.ndarray:
+    """uint32[n]: canonical parent of every vertex in the tree of s (oracle.c:
+    oracle_parents; d defaults to the oracle's own labels sssp(g, s))."""
+    first, head, ln = _csr(g)
+    d = sssp(g, s) if d is None else np.ascontiguousarray(d, dtype=np.uint32)
+    out = np.empty(g.n, dtype=np.uint32)
+    rc = _load().oracle_parents(g.n, first.ctypes.data, head.ctypes.data, ln.ctypes.data, int(s),
+                                d.ctypes.data, out.ctypes.data)
+    if rc:
+        raise ValueError(f"oracle_parents: {rc}")
+    return out

@@ -64,6 +64,7 @@ def _load_lib():
         "phast_build": ([u32, vp, vp, vp, ctypes.POINTER(_Opts), pp], ctypes.c_int),
         "phast_trees": ([vp, vp, u32, vp, vp], ctypes.c_int),
         "phast_trees_host": ([vp, vp, u32, vp, vp], ctypes.c_int),
+        "phast_parents": ([vp, vp, u32, vp, vp, vp], ctypes.c_int),
         "phast_sync": ([vp, vp], ctypes.c_int),
         "phast_diameter": ([vp, vp, u64, u32, vp, vp, vp], ctypes.c_int),
         "phast_info": ([vp, ctypes.POINTER(_Info)], ctypes.c_int),
@@ -88,7 +89,7 @@ def _load_lib():
 
 
 _lib = _load_lib()
-EXPORTED = ("phast_build", "phast_trees", "phast_trees_host", "phast_sync", "phast_diameter", "phast_info",
+EXPORTED = ("phast_build", "phast_trees", "phast_trees_host", "phast_parents", "phast_sync", "phast_diameter", "phast_info",
             "phast_level_sizes", "phast_order", "phast_export", "phast_save", "phast_load", "phast_free",
             "phast_strerror", "phast_launch_count", "phast_timing", "phast_timing_read",
             "phast_plan_stats")
@@ -210,6 +211,28 @@ class Phast:
         _check("phast_trees_host", _lib.phast_trees_host(self._h, src.ctypes.data, src.size, out.ctypes.data,
                                                          _stream_ptr(stream)))
         return out
+
+    def parents(self, sources, dist, out=None, stream=None):
+        """Parent pointers (phast_parents) of the k trees in `dist` (the device tensor
+        phast_trees wrote for the same sources); device tensor [n, k] of internal ids
+        (see parents_to_original)."""
+        import torch
+        src = np.ascontiguousarray(sources, dtype=np.uint32)
+        k = int(src.size)
+        if out is None:
+            out = torch.empty((self.n, k), dtype=torch.int32, device="cuda")
+        _check("phast_parents", _lib.phast_parents(self._h, src.ctypes.data, k, dist.data_ptr(), out.data_ptr(),
+                                                   _stream_ptr(stream)))
+        return out
+
+    def parents_to_original(self, rows: np.ndarray) -> np.ndarray:
+        """[n, k] internal-order parent rows of internal ids -> [k, n] original ids (INF kept)."""
+        t = self.to_original(rows)
+        iperm = np.empty(self.n, np.uint32)
+        iperm[self.order()] = np.arange(self.n, dtype=np.uint32)   # original id of each internal id
+        fin = t != INF
+        t[fin] = iperm[t[fin]]
+        return t
 
     def sync(self, stream=None):
         _check("phast_sync", _lib.phast_sync(self._h, _stream_ptr(stream)))

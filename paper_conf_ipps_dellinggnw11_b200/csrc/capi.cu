@@ -35,6 +35,8 @@ struct phast_ctx {
     size_t dist_scratch_elems = 0;
     uint32_t* batch_max_scratch = nullptr;
     size_t batch_max_elems = 0;
+    uint32_t* d_in_first = nullptr;     // original in-CSR on the device (parents; uploaded on first use)
+    uint2* d_in_arc = nullptr;
     // persistent-sweep plans, one per k (built on first use)
     struct Plan {
         SweepPlan p;
@@ -124,6 +126,8 @@ void free_device(phast_ctx* h) {
     cudaFree(h->g.seed_v); cudaFree(h->g.seed_d); cudaFree(h->g.seed_cnt);
     cudaFree(h->g.gscratch); cudaFree(h->g.err);
     cudaFree(h->dist_scratch); cudaFree(h->batch_max_scratch);
+    cudaFree(h->d_in_first); cudaFree(h->d_in_arc);
+    h->d_in_first = nullptr; h->d_in_arc = nullptr;
     h->g = DevImage();
     h->dist_scratch = nullptr; h->batch_max_scratch = nullptr;
     h->dist_scratch_elems = 0; h->batch_max_elems = 0;
@@ -532,6 +536,8 @@ int phast_build(uint32_t n, const uint64_t* first, const uint32_t* head, const u
         rc = layout_build(R, first, head, mode, delta, h->L);
         h->build_seconds = R.seconds;
         if (rc) return rc;
+        rc = build_in_csr(h->L, n, first, head, len);
+        if (rc) return rc;
         compute_tail_bits(h.get());
     } catch (const std::bad_alloc&) {
         return PHAST_ENOMEM;
@@ -589,6 +595,39 @@ int phast_trees_host(phast_ctx* h, const uint32_t* sources, uint32_t k, uint32_t
     if (cudaMemcpyAsync(host_dist, h->dist_scratch, elems * 4, cudaMemcpyDeviceToHost, st) != cudaSuccess)
         return PHAST_ECUDA;
     return phast_sync(h, stream);
+}
+
+int phast_parents(phast_ctx* h, const uint32_t* sources, uint32_t k, const uint32_t* dist, uint32_t* parent,
+                  void* stream) {
+    if (!h || !sources || !dist || !parent || !k_ok(k)) return PHAST_EINVAL;
+    if (h->device < 0) return PHAST_ESTATE;
+    if (k % 4 == 0 && (((uintptr_t)dist & 15) || ((uintptr_t)parent & 15))) return PHAST_EINVAL;
+    if (h->L.in_first.size() != (size_t)h->n + 1) return PHAST_ESTATE;
+    Sources S;
+    int rc = map_sources(h, sources, k, S);
+    if (rc) return rc;
+    DeviceGuard dg(h->device);
+    if (!h->d_in_first) {   // upload the original in-CSR on first use
+        uint32_t* f = nullptr;
+        uint2* a = nullptr;
+        if ((rc = dmalloc(&f, h->L.in_first.size())) || (rc = dmalloc(&a, h->L.in_arc.size() + 1))) {
+            cudaFree(f);
+            return rc;
+        }
+        if (cudaMemcpy(f, h->L.in_first.data(), h->L.in_first.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess ||
+            (!h->L.in_arc.empty() &&
+             cudaMemcpy(a, h->L.in_arc.data(), h->L.in_arc.size() * 8, cudaMemcpyHostToDevice) != cudaSuccess)) {
+            cudaGetLastError();
+            cudaFree(f);
+            cudaFree(a);
+            return PHAST_ECUDA;
+        }
+        h->d_in_first = f;
+        h->d_in_arc = a;
+    }
+    if (launch_parents(h->d_in_first, h->d_in_arc, h->n, S, k, dist, parent, (cudaStream_t)stream) != cudaSuccess)
+        return PHAST_ECUDA;
+    return PHAST_OK;
 }
 
 int phast_diameter(phast_ctx* h, const uint32_t* sources, uint64_t count, uint32_t k_batch, uint32_t* max_dev,
@@ -683,7 +722,7 @@ int phast_export(const phast_ctx* h, uint32_t* level, uint32_t* dn_first, uint32
 }
 
 // ---------------------------------------------------------------- save / load
-static const char MAGIC[8] = {'P', 'H', 'A', 'S', 'T', 'B', '2', '2'};
+static const char MAGIC[8] = {'P', 'H', 'A', 'S', 'T', 'B', '2', '3'};
 
 int phast_save(const phast_ctx* h, const char* path) {
     if (!h || !path) return PHAST_EINVAL;
@@ -697,6 +736,8 @@ int phast_save(const phast_ctx* h, const char* path) {
               wr(L.level.data(), 4, h->n) && wr(L.lvl_off.data(), 4, L.lvl_off.size()) &&
               wr(L.dn_first.data(), 4, L.dn_first.size()) && wr(L.up_first.data(), 4, L.up_first.size()) &&
               wr(L.dn_arc.data(), 8, L.dn_arc.size()) && wr(L.up_arc.data(), 8, L.up_arc.size());
+    const uint64_t n_in = L.in_arc.size();
+    ok = ok && wr(&n_in, 8, 1) && wr(L.in_first.data(), 4, L.in_first.size()) && wr(L.in_arc.data(), 8, n_in);
     ok = (std::fclose(f) == 0) && ok;
     return ok ? PHAST_OK : PHAST_EIO;
 }
@@ -729,6 +770,19 @@ int phast_load(const char* path, uint32_t flags, phast_ctx** out) {
         ok = rd(L.perm.data(), 4, h->n) && rd(L.level.data(), 4, h->n) && rd(L.lvl_off.data(), 4, L.lvl_off.size()) &&
              rd(L.dn_first.data(), 4, L.dn_first.size()) && rd(L.up_first.data(), 4, L.up_first.size()) &&
              rd(L.dn_arc.data(), 8, L.dn_arc.size()) && rd(L.up_arc.data(), 8, L.up_arc.size());
+        uint64_t n_in = 0;
+        ok = ok && rd(&n_in, 8, 1) && n_in < 0xFFFFFFFEull;
+        if (ok) {
+            try {
+                L.in_first.resize((size_t)h->n + 1);
+                L.in_arc.resize(n_in);
+            } catch (const std::bad_alloc&) {
+                std::fclose(f);
+                return PHAST_ENOMEM;
+            }
+            ok = rd(L.in_first.data(), 4, L.in_first.size()) && rd(L.in_arc.data(), 8, n_in) &&
+                 L.in_first[h->n] == n_in;
+        }
     }
     std::fclose(f);
     if (!ok) return PHAST_EIO;

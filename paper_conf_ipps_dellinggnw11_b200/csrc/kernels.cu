@@ -18,6 +18,7 @@
 //                        §VII-B "making each core keep track of the maximum label it
 //                        encounters").
 // No tensor cores: the loop is an integer (min,+) gather with no reuse.
+#include <algorithm>
 #include <atomic>
 #include <cstdio>
 #include <cstdlib>
@@ -395,6 +396,70 @@ cudaError_t sweep_k(const DevImage& g, uint32_t vbeg, uint32_t vend, uint32_t* d
     }
     return last ? sweep_launch<K, false, true, true, false>(g, vbeg, vend, dist, diam, st)
                 : sweep_launch<K, false, true, false, false>(g, vbeg, vend, dist, diam, st);
+}
+
+// ------------------------------------------------------------------ NEXT-1 parent pointers
+// After a sweep every label is final, so the parent pass has no dependencies: one
+// grid-stride pass over (vertex, 16-byte lane) items.  Each lane owns W trees of the
+// row; it scans v's original in-arcs in input order and keeps, per tree, the tail of
+// the first tight arc (§VII-A).  The identity is tested as d(u) <= d(v)
+// and d(v) - d(u) = l, which equals d(u) + l = d(v) exactly (no 32-bit overflow).
+// The scan stops once every finite tree of the lane has its parent.
+template <int K>
+__global__ void __launch_bounds__(SWEEP_THREADS) parents_kernel(const uint32_t* __restrict__ in_first,
+                                                                const uint2* __restrict__ in_arc,
+                                                                const uint32_t* __restrict__ d,
+                                                                uint32_t* __restrict__ parent, uint32_t n,
+                                                                Sources src) {
+    constexpr uint32_t W = RowT<K>::W;
+    constexpr uint32_t G = K / W;
+    using T = typename RowT<K>::T;
+    const uint64_t total = (uint64_t)n * G;
+    for (uint64_t t = (uint64_t)blockIdx.x * SWEEP_THREADS + threadIdx.x; t < total;
+         t += (uint64_t)gridDim.x * SWEEP_THREADS) {
+        const uint32_t v = (uint32_t)(t / G), lane = (uint32_t)(t % G);
+        const T rv = __ldg(reinterpret_cast<const T*>(d + (size_t)v * K) + lane);
+        const uint32_t* dv = reinterpret_cast<const uint32_t*>(&rv);
+        uint32_t p[W];
+        uint32_t need = 0;
+#pragma unroll
+        for (uint32_t q = 0; q < W; q++) {
+            p[q] = INF;
+            if (dv[q] != INF) need |= 1u << q;
+        }
+        const uint32_t e1 = __ldg(&in_first[v + 1]);
+        for (uint32_t e = __ldg(&in_first[v]); need && e < e1; e++) {
+            const uint2 a = __ldg(&in_arc[e]);
+            const T ru = __ldg(reinterpret_cast<const T*>(d + (size_t)a.x * K) + lane);
+            const uint32_t* du = reinterpret_cast<const uint32_t*>(&ru);
+#pragma unroll
+            for (uint32_t q = 0; q < W; q++)
+                if (((need >> q) & 1u) && du[q] <= dv[q] && dv[q] - du[q] == a.y) {
+                    p[q] = a.x;
+                    need &= ~(1u << q);
+                }
+        }
+#pragma unroll
+        for (uint32_t q = 0; q < W; q++)
+            if (src.s[lane * W + q] == v) p[q] = v;   // the root of tree lane*W+q
+        T out;
+        uint32_t* po = reinterpret_cast<uint32_t*>(&out);
+#pragma unroll
+        for (uint32_t q = 0; q < W; q++) po[q] = p[q];
+        reinterpret_cast<T*>(parent + (size_t)v * K)[lane] = out;
+    }
+}
+
+template <int K>
+cudaError_t parents_k(const uint32_t* in_first, const uint2* in_arc, uint32_t n, const Sources& src,
+                      const uint32_t* dist, uint32_t* parent, cudaStream_t st) {
+    constexpr uint32_t G = K / RowT<K>::W;
+    uint64_t blocks = ((uint64_t)n * G + SWEEP_THREADS - 1) / SWEEP_THREADS;
+    blocks = std::min<uint64_t>(blocks, (uint64_t)num_sms() * 8);
+    if (blocks == 0) return cudaSuccess;
+    parents_kernel<K><<<(unsigned)blocks, SWEEP_THREADS, 0, st>>>(in_first, in_arc, dist, parent, n, src);
+    g_launches++;
+    return cudaGetLastError();
 }
 
 // ------------------------------------------------------------------ a3+a4 persistent sweep
@@ -1667,6 +1732,13 @@ cudaError_t launch_sweep_persistent(const DevImage& g, const SweepPlan& p, uint3
 #define CALL_PS(K) persistent_k<K>(g, p, epoch, dist, diam, st)
     PHAST_K_SWITCH(p.k, CALL_PS)
 #undef CALL_PS
+}
+
+cudaError_t launch_parents(const uint32_t* in_first, const uint2* in_arc, uint32_t n, const Sources& src,
+                           uint32_t k, const uint32_t* dist, uint32_t* parent, cudaStream_t st) {
+#define CALL_PA(K) parents_k<K>(in_first, in_arc, n, src, dist, parent, st)
+    PHAST_K_SWITCH(k, CALL_PA)
+#undef CALL_PA
 }
 
 cudaError_t launch_clear_flags(const DevImage& g, uint32_t k, uint32_t slot, cudaStream_t st) {

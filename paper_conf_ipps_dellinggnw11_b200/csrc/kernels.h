@@ -85,6 +85,14 @@ int sweep_blocks_per_sm(uint32_t k, bool diam, uint32_t variant);
 cudaError_t launch_sweep_persistent(const DevImage& g, const SweepPlan& p, uint32_t epoch, uint32_t* dist,
                                     uint32_t* diam, cudaStream_t st);
 
+// NEXT-1 parent pointers (§VII-A "we check whether the identity d(v) =
+// d(u) + l(u,v) holds"): parent[r*k + i] = internal id of the tail of the first
+// (smallest input index) original arc (u, v) with d_i(u) + l = d_i(v); the source's
+// own row entry is itself; INF where d_i(v) = INF.  in_first/in_arc: the original
+// graph's in-CSR in internal ids (Layout::in_first / in_arc).
+cudaError_t launch_parents(const uint32_t* in_first, const uint2* in_arc, uint32_t n, const Sources& src,
+                           uint32_t k, const uint32_t* dist, uint32_t* parent, cudaStream_t st);
+
 // after the sweep: clear the visited bits of every search-space vertex ("After
 // scanning v we unmark the vertex", §IV-C).
 cudaError_t launch_clear_flags(const DevImage& g, uint32_t k, uint32_t slot, cudaStream_t st);

@@ -230,6 +230,22 @@ int layout_build(const ChResult& R, const uint64_t* first, const uint32_t* head,
     return ok ? 0 : kEinternal;
 }
 
+int build_in_csr(Layout& L, uint32_t n, const uint64_t* first, const uint32_t* head, const uint32_t* len) {
+    std::vector<uint64_t> cnt((size_t)n + 1, 0);
+    for (uint32_t u = 0; u < n; u++)
+        for (uint64_t e = first[u]; e < first[u + 1]; e++)
+            if (head[e] != u && len[e] != 0xFFFFFFFFu) cnt[L.perm[head[e]] + 1]++;
+    for (uint32_t r = 0; r < n; r++) cnt[r + 1] += cnt[r];
+    if (cnt[n] >= 0xFFFFFFFEull) return kErange;
+    L.in_first.assign(cnt.begin(), cnt.end());
+    L.in_arc.resize(cnt[n]);
+    std::vector<uint64_t> fill(cnt.begin(), cnt.end() - 1);
+    for (uint32_t u = 0; u < n; u++)          // increasing input arc index
+        for (uint64_t e = first[u]; e < first[u + 1]; e++)
+            if (head[e] != u && len[e] != 0xFFFFFFFFu) L.in_arc[fill[L.perm[head[e]]]++] = Arc{L.perm[u], len[e]};
+    return 0;
+}
+
 int plan_warp_chunks(const Layout& L, uint32_t cap, uint32_t workers, WarpPlan& P, uint32_t cap_arcs) {
     const uint32_t n = (uint32_t)L.perm.size();
     if (cap == 0 || workers == 0) return kEinternal;

@@ -34,7 +34,16 @@ struct Layout {
     uint32_t cut = 0;                // LAYOUT_DIAGONAL: levels >= cut form the top part
     std::vector<uint32_t> dn_first, up_first;   // [n+1]
     std::vector<Arc> dn_arc, up_arc;
+    // The ORIGINAL graph's in-arcs in internal ids (parent pointers, PAPER.md:20
+    // §VII-A): in_first[n+1] by head, in_arc = {tail, len} in increasing input arc
+    // index per head; self-loops and length-0xFFFFFFFF arcs (never tight) dropped.
+    std::vector<uint32_t> in_first;
+    std::vector<Arc> in_arc;
 };
+
+// Fills L.in_first / L.in_arc from the input CSR (after layout_build).  Returns 0 or
+// PHAST_ERANGE (more than 2^32-2 kept arcs).
+int build_in_csr(Layout& L, uint32_t n, const uint64_t* first, const uint32_t* head, const uint32_t* len);
 
 // Builds the renumbering from the CH result.  first/head: the input graph (used
 // for the BFS that gives the spatial rank in LAYOUT_WAVEFRONT).  Returns 0,

@@ -102,6 +102,38 @@ def test_edge_case_graphs(name):
             assert np.array_equal(gpu_trees(h, src), oracle.sssp_many(g, src)), k
 
 
+def gpu_parents(h, src):
+    src = np.asarray(src, np.uint32)
+    d = h.trees(src)
+    p = h.parents(src, d)
+    h.sync()
+    return h.to_original(d.cpu().numpy()), h.parents_to_original(p.cpu().numpy())
+
+
+@pytest.mark.parametrize("k", (1, 4, 16, 64))
+def test_parents_bit_exact(c1, road, k):
+    """NEXT-1 parent pointers (§VII-A tight-arc identity, reading R14):
+    bit-exact with the oracle's canonical parents, C1 and a road graph."""
+    for g, h in (c1, road):
+        src = phastgen.sources(g.n, k, seed=600 + k, distinct=False)
+        d, par = gpu_parents(h, src)
+        for i, s in enumerate(src):
+            assert np.array_equal(d[i], oracle.sssp(g, s)), (k, i)
+            assert np.array_equal(par[i], oracle.parents(g, s)), (k, i)
+
+
+@pytest.mark.parametrize("name", sorted(EDGE_GRAPHS))
+def test_parents_edge_case_graphs(name):
+    """Zero lengths (ties, zero cycles), saturating lengths, unreachable parts."""
+    g = EDGE_GRAPHS[name]()
+    with P.Phast.from_graph(g) as h:
+        for k in (2, 64):
+            src = phastgen.sources(g.n, k, seed=17 + k)
+            _, par = gpu_parents(h, src)
+            for i, s in enumerate(src):
+                assert np.array_equal(par[i], oracle.parents(g, s)), (k, i)
+
+
 def test_upward_global_fallback_and_overflow(monkeypatch):
     """A shared-memory table too small for the search space falls back to the global
     table (same labels); a per-source capacity too small is reported as ERANGE by

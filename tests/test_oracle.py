@@ -166,7 +166,7 @@ def test_star_and_metric_complete_graph():
 
 
 # ---------------------------------------------------------------- golden
-def load_golden(path):
+def load_golden(path, parents=None):
     n, arcs, dists, diam = None, [], {}, None
     for line in open(path):
         line = line.split("#")[0].split()
@@ -180,6 +180,8 @@ def load_golden(path):
             dists[int(line[1])] = [INF if x == "INF" else int(x) for x in line[2:]]
         elif line[0] == "diameter":
             diam = int(line[1])
+        elif line[0] == "parent" and parents is not None:
+            parents[int(line[1])] = [INF if x == "INF" else int(x) for x in line[2:]]
     return csr_from_arcs(n, arcs), dists, diam
 
 
@@ -193,6 +195,60 @@ def test_golden(name):
         assert list(oracle.sssp(g, s)) == want, (name, s)
         assert oracle.certify(g, s, np.array(want, np.uint32)) == 0
     assert oracle.diameter(g, list(dists)) == diam
+
+
+@pytest.mark.parametrize("name", GOLDEN_FILES)
+def test_golden_parents(name):
+    want = {}
+    g, dists, _ = load_golden(os.path.join(GOLDEN, name), want)
+    for s, p in want.items():
+        assert list(oracle.parents(g, s)) == p, (name, s)
+
+
+# ---------------------------------------------------------------- parents
+def _random_graph(rng, n, lo, hi, density=3):
+    m = int(rng.integers(0, density * n + 1))
+    arcs = [(int(rng.integers(n)), int(rng.integers(n)), int(rng.integers(lo, hi))) for _ in range(m)]
+    return csr_from_arcs(n, arcs)
+
+
+@pytest.mark.parametrize("lenrange", [(1, 4), (1, 1000), (0, 3)])
+def test_parents_vs_floyd_warshall(lenrange):
+    """Parents computed from Floyd-Warshall labels (independent of the oracle's
+    Dijkstra): every parent arc exists and is tight; unreached <-> INF; with
+    positive lengths, following parents from any reached vertex ends at s after
+    < n steps with total length d(v) (a shortest-path tree, §VII-A)."""
+    rng = np.random.default_rng(77 + lenrange[1])
+    for trial in range(150):
+        n = int(rng.integers(1, 24))
+        g = _random_graph(rng, n, *lenrange)
+        D = floyd_warshall(g)
+        tails = g.tails()
+        arcs = {}
+        for e, (t, h, l) in enumerate(zip(tails, g.head, g.len)):
+            arcs.setdefault((int(t), int(h)), []).append(int(l))
+        for s in range(n):
+            d = D[s]
+            p = oracle.parents(g, s, d)
+            assert np.array_equal(oracle.parents(g, s), p)      # same labels from the oracle's own sssp
+            assert p[s] == s
+            for v in range(n):
+                if v == s:
+                    continue
+                if d[v] == INF:
+                    assert p[v] == INF
+                    continue
+                u = int(p[v])
+                assert u != v and (u, v) in arcs
+                assert any(int(d[u]) + l == int(d[v]) for l in arcs[(u, v)])
+                if lenrange[0] > 0:
+                    x, tot, steps = v, 0, 0
+                    while x != s:
+                        y = int(p[x])
+                        tot += min(l for l in arcs[(y, x)] if int(d[y]) + l == int(d[x]))
+                        x, steps = y, steps + 1
+                        assert steps < n
+                    assert tot == int(d[v])
 
 
 # ---------------------------------------------------------------- diameter
