@@ -256,8 +256,9 @@ def main():
     try:
         prof = json.load(open(os.path.join(ROOT, "profiles", "sweep_traffic.json")))
         key = f"{args.config}_k{k}"
-        if key in prof:
-            traffic = prof[key]["dram_bytes_per_sweep"]
+        if key in prof and prof[key].get("layout") == P.LAYOUT_NAMES[info.layout] and \
+                os.environ.get("PHAST_SWEEP", "levels") == prof[key].get("sweep"):
+            traffic = prof[key]["dram_bytes_per_sweep"]   # ncu launch list of this configuration
     except Exception:
         pass
 
