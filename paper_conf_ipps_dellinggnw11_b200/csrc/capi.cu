@@ -42,6 +42,7 @@ struct phast_ctx {
         SweepPlan p;
         uint32_t epoch = 0;
         uint32_t top_levels = 0;   // hybrid (per-level mode): levels [0, top_levels) run as one persistent launch
+        uint32_t bottom_from = 0;  // diagonal layout: segments [bottom_from, end) run as one lagged persistent launch
         bool ok = false;
     };
     std::map<uint32_t, Plan> plans;
@@ -249,8 +250,15 @@ phast_ctx::Plan* get_plan(phast_ctx* h, uint32_t k) {
     p.k = k;
     p.variant = h->sweep_mode == 2 ? 0u : h->sweep_mode == 3 ? 1u : h->sweep_mode == 4 && k >= 4 ? 3u
               : h->sweep_mode == 5 ? 2u : h->sweep_mode == 6 ? 5u : h->sweep_mode == 7 ? 6u : 4u;
-    uint32_t nseg_top = 0;
-    if (h->sweep_mode == 1) {   // hybrid: the small top segments as one segment-barrier launch, big ones one launch each
+    uint32_t nseg_top = 0, seg_from = 0;
+    const char* bseg = std::getenv("PHAST_BOTTOM_SEG");
+    if (h->sweep_mode == 1 && L.mode == LAYOUT_DIAGONAL && bseg && std::atoi(bseg)) {
+        // the diagonals of the bottom levels in ONE launch; segment j waits only for
+        // segment j - lag (the layout's guarantee), the top levels stay one launch each
+        seg_from = L.levels - L.cut;
+        P.bottom_from = seg_from;
+        p.variant = 6;
+    } else if (h->sweep_mode == 1) {   // hybrid: the small top segments as one segment-barrier launch, big ones one launch each
         uint32_t thresh = 0;
         if (const char* e = std::getenv("PHAST_TOP_THRESH")) thresh = (uint32_t)std::atoi(e);
         uint32_t J = 0;
@@ -271,15 +279,16 @@ phast_ctx::Plan* get_plan(phast_ctx* h, uint32_t k) {
         int per_sm = nseg_top ? 4 : 8;
         if (const char* e = std::getenv(nseg_top ? "PHAST_TOP_CTAS" : "PHAST_SEG_CTAS")) per_sm = std::max(1, std::atoi(e));
         p.grid = (uint32_t)std::max(1, std::min(occ, per_sm) * num_sms());
-        const uint32_t nseg = nseg_top ? nseg_top : (uint32_t)L.lvl_off.size() - 1;
+        const uint32_t nseg = nseg_top ? nseg_top : (uint32_t)L.lvl_off.size() - 1 - seg_from;
         p.nchunks = p.iters = nseg;
-        p.chunk_cap = L.mode == LAYOUT_DIAGONAL ? L.levels - L.cut : nseg;   // diagonals: store by tail bit
+        p.chunk_cap = seg_from ? 0u : L.mode == LAYOUT_DIAGONAL ? L.levels - L.cut : nseg;   // diagonals: by tail bit
         p.stream_last = nseg_top ? 0u : 1u;   // the layout's last segment is nobody's tail
+        p.seg_lag = seg_from ? L.lag : 1u;
         uint32_t *a, *w;
         if (dmalloc(&a, nseg + 1) || dmalloc(&w, nseg)) return nullptr;
         p.chunk_v = a;
         p.wave_done = w;
-        if (cudaMemcpy(a, L.lvl_off.data(), (size_t)(nseg + 1) * 4, cudaMemcpyHostToDevice) != cudaSuccess ||
+        if (cudaMemcpy(a, L.lvl_off.data() + seg_from, (size_t)(nseg + 1) * 4, cudaMemcpyHostToDevice) != cudaSuccess ||
             cudaMemset(w, 0, (size_t)nseg * 4) != cudaSuccess) {
             cudaGetLastError();
             return nullptr;
@@ -437,7 +446,18 @@ int run_query(phast_ctx* h, const Sources& S, uint32_t k, uint32_t* dist, uint32
     if (launch_seed(h->g, k, slot, dist, st) != cudaSuccess) return PHAST_ECUDA;
     if (e1) cudaEventRecord(e1, st);
     phast_ctx::Plan* plan = get_plan(h, k);
-    if (plan && plan->top_levels == 0) {   // a3 + a4: one persistent launch, dataflow over chunks
+    if (plan && plan->bottom_from) {   // top levels one launch each, then the bottom diagonals in one launch
+        for (uint32_t j = 0; j < plan->bottom_from; j++)
+            if (launch_sweep_level(h->g, k, h->L.lvl_off[j], h->L.lvl_off[j + 1], dist, diam, true, false, false,
+                                   st) != cudaSuccess)
+                return PHAST_ECUDA;
+        if ((uint64_t)(plan->epoch + 1) * plan->p.grid >= 0x7FFFFFFFull) {
+            if (cudaMemsetAsync(plan->p.wave_done, 0, (size_t)plan->p.iters * 4, st) != cudaSuccess) return PHAST_ECUDA;
+            plan->epoch = 0;
+        }
+        plan->epoch++;
+        if (launch_sweep_persistent(h->g, plan->p, plan->epoch, dist, diam, st) != cudaSuccess) return PHAST_ECUDA;
+    } else if (plan && plan->top_levels == 0) {   // a3 + a4: one persistent launch, dataflow over chunks
         if ((plan->p.variant < 2 || plan->p.variant == 6) && (uint64_t)(plan->epoch + 1) * plan->p.grid >= 0x7FFFFFFFull) {
             if (cudaMemsetAsync(plan->p.wave_done, 0, (size_t)plan->p.iters * 4, st) != cudaSuccess) return PHAST_ECUDA;
             plan->epoch = 0;
@@ -730,7 +750,7 @@ int phast_save(const phast_ctx* h, const char* path) {
     if (!f) return PHAST_EIO;
     const Layout& L = h->L;
     uint64_t hdr[10] = {h->n, L.levels, h->m, h->shortcuts, h->rounds, L.dn_arc.size(), L.up_arc.size(),
-                        L.mode | ((uint64_t)L.cut << 32), L.delta, L.lvl_off.size()};
+                        L.mode | ((uint64_t)L.cut << 32) | ((uint64_t)L.lag << 56), L.delta, L.lvl_off.size()};
     auto wr = [&](const void* p, size_t sz, size_t cnt) { return std::fwrite(p, sz, cnt, f) == cnt; };
     bool ok = wr(MAGIC, 1, 8) && wr(hdr, 8, 10) && wr(&h->build_seconds, 8, 1) && wr(L.perm.data(), 4, h->n) &&
               wr(L.level.data(), 4, h->n) && wr(L.lvl_off.data(), 4, L.lvl_off.size()) &&
@@ -758,7 +778,8 @@ int phast_load(const char* path, uint32_t flags, phast_ctx** out) {
         try {
             h->n = (uint32_t)hdr[0]; L.levels = (uint32_t)hdr[1]; h->m = hdr[2];
             h->shortcuts = hdr[3]; h->rounds = (uint32_t)hdr[4];
-            L.mode = (uint32_t)hdr[7]; L.cut = (uint32_t)(hdr[7] >> 32); L.delta = (uint32_t)hdr[8];
+            L.mode = (uint32_t)hdr[7]; L.cut = (uint32_t)((hdr[7] >> 32) & 0xFFFFFFu);
+            L.lag = std::max(1u, (uint32_t)(hdr[7] >> 56)); L.delta = (uint32_t)hdr[8];
             L.perm.resize(h->n); L.iperm.resize(h->n); L.level.resize(h->n);
             L.lvl_off.resize(hdr[9]);
             L.dn_first.resize((size_t)h->n + 1); L.up_first.resize((size_t)h->n + 1);

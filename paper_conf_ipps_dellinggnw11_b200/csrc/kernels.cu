@@ -1234,16 +1234,18 @@ __global__ void __launch_bounds__(SWEEP_THREADS, BATCH ? 6 : 8) sweep_seg_kernel
             }
             if constexpr (DIAM) mx = max(mx, fmax_of(acc));
         }
-        if (j + 1 < nseg) {   // grid barrier: segment j complete and visible
+        if (j + 1 < nseg) {   // segment j done here; segment j + 1 needs segment j + 1 - lag everywhere
             __syncthreads();
             if (threadIdx.x == 0) {
                 asm volatile("red.release.gpu.global.add.u32 [%0], 1;" ::"l"(&p.wave_done[j]) : "memory");
-                // relaxed spin (an acquire load per poll would drop the L1 lines of the
-                // CTAs still working on this SM), then one acquire fence
-                if (ld_flag(&p.wave_done[j]) < target) {
+                // lag 1: a grid barrier on segment j; relaxed spin (an acquire load per
+                // poll would drop the L1 lines of the CTAs still working on this SM), then
+                // one acquire fence
+                const uint32_t w = j + 1 >= p.seg_lag ? j + 1 - p.seg_lag : j;
+                if (j + 1 >= p.seg_lag && ld_flag(&p.wave_done[w]) < target) {
                     uint32_t ns = 32;
                     const uint64_t t0 = globaltimer_ns();
-                    while (ld_flag(&p.wave_done[j]) < target) {
+                    while (ld_flag(&p.wave_done[w]) < target) {
                         __nanosleep(ns);
                         ns = min(ns * 2, 256u);
                         if ((*(volatile uint32_t*)p.err & 2u) || globaltimer_ns() - t0 > 4000000000ull) {

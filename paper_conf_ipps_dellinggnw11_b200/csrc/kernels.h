@@ -67,6 +67,7 @@ struct SweepPlan {
     const uint4* wdesc = nullptr;           // variant 5: [iters * workers] chunk descriptors (plan_waves)
     uint32_t* err = nullptr;                // sticky device error word (bit 1: dependency watchdog)
     uint32_t stream_last = 1;               // variant 6: the last segment's rows are nobody's tail
+    uint32_t seg_lag = 1;                   // variant 6: segment j waits for segment j - seg_lag (1: barrier)
 };
 // vertices per chunk and CTAs per SM the persistent sweep uses for this k
 uint32_t sweep_chunk_vertices(uint32_t k);   // max vertices per chunk

@@ -34,6 +34,7 @@
 #include "layout.h"
 
 #include <algorithm>
+#include <cstdlib>
 #include <numeric>
 
 namespace phast {
@@ -125,7 +126,13 @@ int layout_build(const ChResult& R, const uint64_t* first, const uint32_t* head,
             uint64_t above = 0;
             while (cut > 1 && above + cnt[cut - 1] <= n / 256) above += cnt[--cut];
         }
+        // experiment knobs: the cut level, and the lag (key(tail) <= key(head) - lag, so
+        // that a persistent sweep may run diagonal j while diagonals > j - lag finish)
+        if (const char* e = std::getenv("PHAST_DIAG_CUT")) cut = std::max(1u, std::min<uint32_t>(levels, std::atoi(e)));
+        uint32_t lag = 1;
+        if (const char* e = std::getenv("PHAST_DIAG_LAG")) lag = std::max(1, std::min(8, std::atoi(e)));
         L.cut = cut;
+        L.lag = lag;
         const uint32_t band_w = std::max(1u, delta);
         auto band = [&](uint32_t v) { return (int64_t)(rank[v] / band_w); };
         std::vector<int64_t> o(levels, 0);
@@ -137,7 +144,7 @@ int layout_build(const ChResult& R, const uint64_t* first, const uint32_t* head,
                 for (uint32_t v : by_level[l])
                     for (uint64_t e = R.dn_first[v]; e < R.dn_first[v + 1]; e++) {
                         const uint32_t t = R.dn_tail[e];
-                        if (R.level[t] < cut) o[l] = std::max(o[l], o[R.level[t]] + band(t) - band(v) + 1);
+                        if (R.level[t] < cut) o[l] = std::max(o[l], o[R.level[t]] + band(t) - band(v) + lag);
                     }
         }
         std::iota(order.begin(), order.end(), 0u);

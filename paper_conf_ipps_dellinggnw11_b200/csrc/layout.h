@@ -32,6 +32,7 @@ struct Layout {
     // one each, then one per diagonal.  Empty for LAYOUT_WAVEFRONT.
     std::vector<uint32_t> lvl_off;
     uint32_t cut = 0;                // LAYOUT_DIAGONAL: levels >= cut form the top part
+    uint32_t lag = 1;                // LAYOUT_DIAGONAL: key(tail) <= key(head) - lag on bottom arcs
     std::vector<uint32_t> dn_first, up_first;   // [n+1]
     std::vector<Arc> dn_arc, up_arc;
     // The ORIGINAL graph's in-arcs in internal ids (parent pointers, PAPER.md:20

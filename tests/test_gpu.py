@@ -159,6 +159,9 @@ def test_upward_global_fallback_and_overflow(monkeypatch):
                                                      ("levels-ab1", "bfs", 0), ("levels-ab3", "bfs", 0),
                                                      ("levels-ab4", "bfs", 0), ("levels-ab8", "bfs", 0),
                                                      ("levels-ab8", "diagonal", 0),
+                                                     ("bottomseg2-2", "diagonal", 0), ("bottomseg2-2", "diagonal", 3000),
+                                                     ("bottomseg3-2", "diagonal", 0), ("bottomsegauto-3", "diagonal", 500),
+                                                     ("bottomseg2-1", "diagonal", 2000),
                                                      ("warp", True, 0), ("staged", True, 0),
                                                      ("warp", False, 0), ("persistent", False, 0),
                                                      ("wpipe", False, 0), ("wpipe", False, 300), ("wpipe", True, 0),
@@ -174,7 +177,14 @@ def test_sweep_modes(monkeypatch, mode, level_layout, delta):
     (§VI); the single persistent launch as warp dataflow (default) or CTA
     waves (with and without bulk-staged arcs), on both layouts, including a small
     wavefront skew (many short dependencies)."""
-    if mode.startswith("levels-ab"):            # per-level launches, other arc batch (1, 3, 4, 8 = cp.async staged)
+    if mode.startswith("bottomseg"):            # diagonal layout, bottom diagonals in one lagged launch
+        cut, lag = mode[len("bottomseg"):].split("-")
+        monkeypatch.setenv("PHAST_BOTTOM_SEG", "1")
+        monkeypatch.setenv("PHAST_DIAG_LAG", lag)
+        if cut != "auto":
+            monkeypatch.setenv("PHAST_DIAG_CUT", cut)
+        mode = "levels"
+    elif mode.startswith("levels-ab"):            # per-level launches, other arc batch (1, 3, 4, 8 = cp.async staged)
         monkeypatch.setenv("PHAST_ARC_BATCH", mode[len("levels-ab"):])
         mode = "levels"
     elif mode == "levels-hybrid":                # a few small top levels fused, the rest one launch each
