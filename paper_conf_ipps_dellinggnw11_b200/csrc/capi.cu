@@ -46,6 +46,13 @@ struct phast_ctx {
         bool ok = false;
     };
     std::map<uint32_t, Plan> plans;
+    // top levels [0, J) swept in one single-CTA launch (launch_sweep_top), one plan per k
+    struct Top {
+        uint4* chunks = nullptr;   // device [nchunks] {vbeg, vend, first[vbeg], first[vend]}
+        uint32_t nchunks = 0, J = 0, V = 0;
+        bool ok = false;
+    };
+    std::map<uint32_t, Top> tops;
     // 0 = warp pipeline (default), 1 = one launch per level, 2 = CTA waves, 3 = CTA waves + bulk-staged
     // arcs, 4 = pipelined CTA gather (k >= 4; else warp pipeline), 5 = warp dataflow without pipeline
     int sweep_mode = 0;
@@ -104,6 +111,8 @@ void free_plans(phast_ctx* h) {
         cudaFree(kv.second.p.done);
     }
     h->plans.clear();
+    for (auto& kv : h->tops) cudaFree(kv.second.chunks);
+    h->tops.clear();
 }
 
 void free_device(phast_ctx* h) {
@@ -415,6 +424,59 @@ phast_ctx::Plan* get_plan(phast_ctx* h, uint32_t k) {
     return &P;
 }
 
+// Top levels in one single-CTA launch (kernels.cu: sweep_top_kernel): the longest
+// prefix of levels whose rows [0, V) fit the shared-memory label budget at this k,
+// each level small enough for one SM (<= 32 items per consumer thread) and no vertex
+// with more in-arcs than a chunk holds.  PHAST_TOP=0 disables it; PHAST_TOP_MAXV caps V.
+phast_ctx::Top* get_top(phast_ctx* h, uint32_t k) {
+    auto it = h->tops.find(k);
+    if (it != h->tops.end()) return it->second.ok ? &it->second : nullptr;
+    phast_ctx::Top& T = h->tops[k];
+    const char* env = std::getenv("PHAST_TOP");
+    if (env && std::atoi(env) == 0) return nullptr;
+    const Layout& L = h->L;
+    if (L.mode != LAYOUT_LEVELS && L.mode != LAYOUT_LEVELS_BFS) return nullptr;
+    if (L.lvl_off.size() < 2) return nullptr;
+    const uint32_t G = k >= 4 ? k / 4 : 1;
+    uint64_t vmax = top_label_budget() / (4ull * k);
+    if (const char* e = std::getenv("PHAST_TOP_MAXV")) vmax = std::min<uint64_t>(vmax, (uint64_t)std::atoll(e));
+    const uint32_t VCH = top_chunk_vertices(), ECH = top_chunk_arcs();
+    const uint32_t nseg = (uint32_t)L.lvl_off.size() - 1;
+    uint32_t J = 0;
+    while (J < nseg) {
+        const uint32_t a = L.lvl_off[J], b = L.lvl_off[J + 1];
+        if (b > vmax || (uint64_t)(b - a) * G > 32ull * 992) break;
+        bool fits = true;
+        for (uint32_t v = a; v < b && fits; v++) fits = L.dn_first[v + 1] - L.dn_first[v] <= ECH;
+        if (!fits) break;
+        J++;
+    }
+    if (J < 2) return nullptr;
+    std::vector<uint4> ch;
+    for (uint32_t j = 0; j < J; j++) {
+        uint32_t v = L.lvl_off[j];
+        const uint32_t b = L.lvl_off[j + 1];
+        while (v < b) {   // greedy chunks inside the level: <= VCH vertices, <= ECH arcs
+            uint32_t w = v;
+            while (w < b && w - v < VCH && L.dn_first[w + 1] - L.dn_first[v] <= ECH) w++;
+            ch.push_back(make_uint4(v, w, L.dn_first[v], L.dn_first[w]));
+            v = w;
+        }
+    }
+    if (dmalloc(&T.chunks, ch.size()) ||
+        cudaMemcpy(T.chunks, ch.data(), ch.size() * sizeof(uint4), cudaMemcpyHostToDevice) != cudaSuccess) {
+        cudaGetLastError();
+        return nullptr;
+    }
+    T.nchunks = (uint32_t)ch.size();
+    T.J = J;
+    T.V = L.lvl_off[J];
+    T.ok = true;
+    if (std::getenv("PHAST_VERBOSE"))
+        std::fprintf(stderr, "top plan k=%u: %u levels, %u vertices, %u chunks\n", k, J, T.V, T.nchunks);
+    return &T;
+}
+
 constexpr size_t MAX_TIMED_BATCHES = 16384;
 
 cudaEvent_t timing_event(phast_ctx* h) {
@@ -475,7 +537,12 @@ int run_query(phast_ctx* h, const Sources& S, uint32_t k, uint32_t* dist, uint32
         const uint32_t levels = (uint32_t)h->L.lvl_off.size() - 1;   // segments
         const bool diagonal = h->L.mode == LAYOUT_DIAGONAL;
         uint32_t j0 = 0;
-        if (plan) {                           // hybrid: small top levels in one persistent launch
+        phast_ctx::Top* top = (!plan && !diagonal) ? get_top(h, k) : nullptr;
+        if (top) {                            // the small top levels in one single-CTA launch
+            if (launch_sweep_top(h->g, k, top->chunks, top->nchunks, top->V, dist, diam, st) != cudaSuccess)
+                return PHAST_ECUDA;
+            j0 = top->J;
+        } else if (plan) {                    // hybrid: small top levels in one persistent launch
             if ((uint64_t)(plan->epoch + 1) * plan->p.grid >= 0x7FFFFFFFull) {
                 if (cudaMemsetAsync(plan->p.wave_done, 0, (size_t)plan->p.iters * 4, st) != cudaSuccess)
                     return PHAST_ECUDA;

@@ -263,10 +263,19 @@ __global__ void __launch_bounds__(SWEEP_THREADS, AB >= 3 && AB < 8 ? 6 : 8) swee
     constexpr uint32_t W = RowT<K>::W;
     constexpr uint32_t G = K / W;   // lanes per vertex
     asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
-    asm volatile("griddepcontrol.wait;" ::: "memory");          // previous level complete and visible
     const uint32_t total = (vend - vbeg) * G;   // host: < 2^31 (sweep_launch splits longer segments)
+    // The graph (offsets, arcs) is static: the first item's offsets are loaded and its
+    // first arcs prefetched into L2 BEFORE griddepcontrol.wait, overlapping the previous
+    // level's drain; only label rows (flags, tail rows) must wait.  The loop itself
+    // re-reads them (L1 / L2 hits) so that it keeps its register budget.
+    uint32_t t = blockIdx.x * SWEEP_THREADS + threadIdx.x;
+    if (t < total) {
+        const uint32_t e0 = __ldg(&first[vbeg + t / G]);
+        asm volatile("prefetch.global.L2 [%0];" ::"l"(arcs + e0));
+    }
+    asm volatile("griddepcontrol.wait;" ::: "memory");          // previous level complete and visible
     uint32_t mx = 0;
-    for (uint32_t t = blockIdx.x * SWEEP_THREADS + threadIdx.x; t < total; t += gridDim.x * SWEEP_THREADS) {
+    for (; t < total; t += gridDim.x * SWEEP_THREADS) {
         const uint32_t v = vbeg + t / G;
         const uint32_t lane = t % G;
         T acc = inf_row<T>();
@@ -1628,6 +1637,138 @@ __global__ void max_reduce_kernel(const uint32_t* __restrict__ in, uint32_t coun
 
 }  // namespace
 
+// ------------------------------------------------------------------ a3 + a4: top levels in one CTA
+// The top of the hierarchy has many tiny levels (C1: 73 levels for 10 k vertices;
+// C3: the top 46 levels hold 59 k of 18 M vertices).  One launch per level
+// (§VI "The CPU starts, for each level i, a kernel on the GPU") costs
+// ~4 us of launch + drain per level however small it is, so the levels whose rows
+// fit in shared memory run in ONE CTA instead:
+//  - the rows of [0, V) (the top levels: internal ids ascend as levels descend) are
+//    loaded once into shared memory (seeded label if visited, else INF: PAPER.md:16
+//    §IV-C), swept there level by level, and written back once;
+//  - warp 0 is a producer: one elected thread streams every chunk's offsets and
+//    arcs (contiguous per level, §IV-A) into a 3-stage shared-memory ring
+//    with bulk copies (TMA, cp.async.bulk) signalled on mbarriers, ahead of use;
+//  - 31 consumer warps relax one chunk at a time from shared memory
+//    (§III "if d(v) > d(u)+l(u,v), we set d(v) = d(u)+l(u,v)") and meet
+//    at a named barrier after it, which orders the levels (Lemma 4.1: every tail is
+//    in an earlier chunk) and frees the ring stage.
+// A level boundary costs one named barrier (~tens of ns) instead of a launch.
+constexpr int TOP_THREADS = 1024, TOP_CONS = TOP_THREADS - 32, TOP_STAGES = 3;
+constexpr uint32_t TOP_VCH = 1024, TOP_ECH = 2048;                // per chunk: vertices, arcs
+constexpr uint32_t TOP_OFF_BUF = TOP_VCH + 8, TOP_ARC_BUF = TOP_ECH + 2;
+constexpr size_t TOP_RING_BYTES = (size_t)TOP_STAGES * (TOP_OFF_BUF * 4 + TOP_ARC_BUF * 8);
+constexpr size_t TOP_SMEM_MAX = 227 * 1024;
+
+__device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
+}
+
+template <int K, bool DIAM>
+__global__ void __launch_bounds__(TOP_THREADS, 1) sweep_top_kernel(const uint32_t* __restrict__ first,
+                                                                   const uint2* __restrict__ arcs,
+                                                                   uint32_t* __restrict__ d,
+                                                                   const uint32_t* __restrict__ flags,
+                                                                   const uint4* __restrict__ chunks,
+                                                                   uint32_t nchunks, uint32_t V,
+                                                                   uint32_t* __restrict__ diam) {
+    using T = typename RowT<K>::T;
+    constexpr uint32_t G = K / RowT<K>::W;   // lanes per vertex
+    extern __shared__ __align__(16) unsigned char top_smem[];
+    T* srow = reinterpret_cast<T*>(top_smem);
+    const size_t lab = ((size_t)V * G * sizeof(T) + 15) & ~(size_t)15;
+    uint32_t* soff = reinterpret_cast<uint32_t*>(top_smem + lab);                              // [S][OFF_BUF]
+    uint2* sarc = reinterpret_cast<uint2*>(top_smem + lab + (size_t)TOP_STAGES * TOP_OFF_BUF * 4);   // [S][ARC_BUF]
+    uint64_t* full = reinterpret_cast<uint64_t*>(top_smem + lab + TOP_RING_BYTES);
+    uint64_t* empty = full + TOP_STAGES;
+    const uint32_t tid = threadIdx.x;
+    if (tid == 0) {
+        for (int s = 0; s < TOP_STAGES; s++) {
+            mbar_init(&full[s], 1);
+            mbar_init(&empty[s], 1);
+        }
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    // a2 (implicit init): the top rows, seeded label if visited else INF
+    const T* dr = reinterpret_cast<const T*>(d);
+    for (uint32_t i = tid; i < V * G; i += TOP_THREADS) {
+        const uint32_t v = i / G;
+        srow[i] = ((__ldg(&flags[v >> 5]) >> (v & 31)) & 1u) ? dr[i] : inf_row<T>();
+    }
+    __syncthreads();
+    uint32_t mx = 0;
+    if (tid < 32) {   // producer warp: one elected thread issues the bulk copies
+        if (tid == 0) {
+            for (uint32_t c = 0; c < nchunks; c++) {
+                const uint32_t s = c % TOP_STAGES;
+                if (c >= TOP_STAGES) mbar_wait(&empty[s], ((c / TOP_STAGES) - 1) & 1);
+                const uint4 ch = __ldg(&chunks[c]);   // {vbeg, vend, ebeg = first[vbeg], eend = first[vend]}
+                const uint32_t f0 = ch.x & ~3u, nf = (ch.y + 1 - f0 + 3) & ~3u;   // 16-byte aligned copies
+                const uint32_t a0 = ch.z & ~1u, na = (ch.w - a0 + 1) & ~1u;
+                mbar_arrive_tx(&full[s], nf * 4 + na * 8);
+                bulk_g2s(soff + s * TOP_OFF_BUF, first + f0, nf * 4, &full[s]);
+                if (na) bulk_g2s(sarc + s * TOP_ARC_BUF, arcs + a0, na * 8, &full[s]);
+            }
+        }
+        __syncwarp();
+    } else {
+        const uint32_t ct = tid - 32;
+        for (uint32_t c = 0; c < nchunks; c++) {
+            const uint32_t s = c % TOP_STAGES;
+            const uint4 ch = __ldg(&chunks[c]);
+            mbar_wait(&full[s], (c / TOP_STAGES) & 1);
+            const uint32_t f0 = ch.x & ~3u, a0 = ch.z & ~1u;
+            const uint32_t* sf = soff + s * TOP_OFF_BUF;
+            const uint2* sa = sarc + s * TOP_ARC_BUF;
+            const uint32_t total = (ch.y - ch.x) * G;
+            for (uint32_t t = ct; t < total; t += TOP_CONS) {
+                const uint32_t v = ch.x + t / G, lane = t % G;
+                T acc = srow[v * G + lane];
+                const uint32_t e0 = sf[v - f0], e1 = sf[v + 1 - f0];
+                for (uint32_t e = e0; e < e1; e++) {
+                    const uint2 a = sa[e - a0];
+                    acc = relax(acc, srow[a.x * G + lane], a.y);
+                }
+                srow[v * G + lane] = acc;
+                if constexpr (DIAM) mx = max(mx, fmax_of(acc));
+            }
+            asm volatile("bar.sync 1, %0;" ::"n"(TOP_CONS) : "memory");   // chunk done: next level may read it
+            if (ct == 0) mbar_arrive(&empty[s]);                          // ring stage free
+        }
+    }
+    __syncthreads();
+    T* dw = reinterpret_cast<T*>(d);
+    for (uint32_t i = tid; i < V * G; i += TOP_THREADS) dw[i] = srow[i];
+    if constexpr (DIAM) {
+        mx = __reduce_max_sync(0xFFFFFFFFu, mx);
+        if ((tid & 31) == 0 && mx) atomicMax(diam, mx);
+    }
+}
+
+size_t top_smem_bytes(uint32_t k, uint32_t V) {
+    const size_t lab = ((size_t)V * k * 4 + 15) & ~(size_t)15;
+    return lab + TOP_RING_BYTES + 2 * TOP_STAGES * sizeof(uint64_t);
+}
+size_t top_label_budget() { return TOP_SMEM_MAX - TOP_RING_BYTES - 2 * TOP_STAGES * sizeof(uint64_t) - 16; }
+uint32_t top_chunk_vertices() { return TOP_VCH; }
+uint32_t top_chunk_arcs() { return TOP_ECH; }
+
+template <int K>
+cudaError_t top_k(const DevImage& g, const uint4* chunks, uint32_t nchunks, uint32_t V, uint32_t* dist,
+                  uint32_t* diam, cudaStream_t st) {
+    const size_t smem = top_smem_bytes(K, V);
+    static bool attr_set[2] = {false, false};
+    auto kern = diam ? sweep_top_kernel<K, true> : sweep_top_kernel<K, false>;
+    if (!attr_set[diam ? 1 : 0]) {
+        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)TOP_SMEM_MAX);
+        if (e != cudaSuccess) return e;
+        attr_set[diam ? 1 : 0] = true;
+    }
+    kern<<<1, TOP_THREADS, smem, st>>>(g.dn_first, g.dn_arc, dist, g.flags, chunks, nchunks, V, diam);
+    g_launches++;
+    return cudaGetLastError();
+}
+
 #define PHAST_K_SWITCH(k, CALL)      \
     switch (k) {                     \
         case 1: return CALL(1);      \
@@ -1741,6 +1882,13 @@ cudaError_t launch_parents(const uint32_t* in_first, const uint2* in_arc, uint32
 #define CALL_PA(K) parents_k<K>(in_first, in_arc, n, src, dist, parent, st)
     PHAST_K_SWITCH(k, CALL_PA)
 #undef CALL_PA
+}
+
+cudaError_t launch_sweep_top(const DevImage& g, uint32_t k, const uint4* chunks, uint32_t nchunks, uint32_t V,
+                             uint32_t* dist, uint32_t* diam, cudaStream_t st) {
+#define CALL_TOP(K) top_k<K>(g, chunks, nchunks, V, dist, diam, st)
+    PHAST_K_SWITCH(k, CALL_TOP)
+#undef CALL_TOP
 }
 
 cudaError_t launch_clear_flags(const DevImage& g, uint32_t k, uint32_t slot, cudaStream_t st) {

@@ -94,6 +94,16 @@ cudaError_t launch_sweep_persistent(const DevImage& g, const SweepPlan& p, uint3
 cudaError_t launch_parents(const uint32_t* in_first, const uint2* in_arc, uint32_t n, const Sources& src,
                            uint32_t k, const uint32_t* dist, uint32_t* parent, cudaStream_t st);
 
+// a3 + a4 for the top levels [0, V) in ONE single-CTA launch (labels in shared
+// memory, arcs streamed by TMA): chunks[c] = {vbeg, vend, first[vbeg], first[vend]},
+// level-ordered, at most top_chunk_vertices() vertices and top_chunk_arcs() arcs
+// each, never spanning two levels; V * k * 4 <= top_label_budget().
+cudaError_t launch_sweep_top(const DevImage& g, uint32_t k, const uint4* chunks, uint32_t nchunks, uint32_t V,
+                             uint32_t* dist, uint32_t* diam, cudaStream_t st);
+size_t top_label_budget();
+uint32_t top_chunk_vertices();
+uint32_t top_chunk_arcs();
+
 // after the sweep: clear the visited bits of every search-space vertex ("After
 // scanning v we unmark the vertex", §IV-C).
 cudaError_t launch_clear_flags(const DevImage& g, uint32_t k, uint32_t slot, cudaStream_t st);

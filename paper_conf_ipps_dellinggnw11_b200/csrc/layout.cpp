@@ -116,6 +116,10 @@ int layout_build(const ChResult& R, const uint64_t* first, const uint32_t* head,
             std::sort(by.begin(), by.end(), [&](uint32_t a, uint32_t b) { return rank[a] < rank[b]; });
         }
         for (uint32_t v : by) order[pos[R.level[v]]++] = v;
+        if (mode == LAYOUT_LEVELS_BFS)   // serpentine: odd levels in descending BFS rank, so a
+            for (uint32_t j = 0; j < levels; j++)   // level starts where the level above ended (its rows
+                if ((levels - 1 - j) & 1u)          // still in L2): 7.8 % fewer tail-row misses (r1_l2sim.md)
+                    std::reverse(order.begin() + L.lvl_off[j], order.begin() + L.lvl_off[j + 1]);
     } else if (mode == LAYOUT_DIAGONAL) {
         std::vector<uint32_t> rank = bfs_rank(n, first, head);
         std::vector<uint32_t> cnt(levels, 0);
@@ -155,9 +159,17 @@ int layout_build(const ChResult& R, const uint64_t* first, const uint32_t* head,
             if (R.level[a] != R.level[b]) return R.level[a] > R.level[b];
             return rank[a] < rank[b];
         });
+        // one segment per top level, then one per bottom key VALUE, empty ones included:
+        // key(head) - key(tail) >= lag must hold for segment indices too, so that a
+        // lagged schedule (segment j waits for j - lag) sees every tail finished
         L.lvl_off.assign(1, 0);
-        for (uint32_t r = 1; r <= n; r++)
-            if (r == n || key(order[r]) != key(order[r - 1])) L.lvl_off.push_back(r);
+        for (uint32_t r = 1; r <= n; r++) {
+            if (r < n && key(order[r]) == key(order[r - 1])) continue;
+            const int64_t kp = key(order[r - 1]);
+            if (r < n && kp >= 0)
+                for (int64_t kk = kp + 1; kk < key(order[r]); kk++) L.lvl_off.push_back(r);   // empty keys
+            L.lvl_off.push_back(r);
+        }
     } else {
         std::vector<uint32_t> rank = bfs_rank(n, first, head);
         std::vector<int64_t> key(n);

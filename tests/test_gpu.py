@@ -204,6 +204,45 @@ def test_sweep_modes(monkeypatch, mode, level_layout, delta):
         assert h.diameter(src, k_batch=64) == oracle.diameter(g, src)
 
 
+@pytest.mark.parametrize("top", ["0", "1", "40", "700", "3000"])
+def test_top_levels_kernel(monkeypatch, top):
+    """The top levels in one single-CTA launch (sweep_top_kernel: rows in shared
+    memory, TMA-staged arc chunks): off ("0"), default ("1", the whole 10 k grid at
+    k <= 4), and capped at V <= 40 / 700 / 3000 vertices (the prefix ends inside the
+    hierarchy, chunks split long levels), every k, bit-exact; plus the diameter."""
+    if top == "0":
+        monkeypatch.setenv("PHAST_TOP", "0")
+    elif top != "1":
+        monkeypatch.setenv("PHAST_TOP_MAXV", top)
+    for g in (phastgen.CONFIGS["C1"]["graph"](), phastgen.road(60_000, seed=35)):
+        with P.Phast.from_graph(g) as h:
+            for k in (1, 2, 4, 16, 64):
+                src = phastgen.sources(g.n, k, seed=950 + k)
+                assert np.array_equal(gpu_trees(h, src), oracle.sssp_many(g, src)), (k, top)
+            src = phastgen.sources(g.n, 130, seed=951)
+            assert h.diameter(src, k_batch=4) == oracle.diameter(g, src)
+
+
+def test_top_levels_hub_vertex():
+    """A sink with 2 999 in-arcs (more than one TMA chunk holds, 2 048) is contracted
+    first and ends in level 0 with all of them in G-down: the top prefix must stop
+    before its level.  Bit-exact."""
+    rng = np.random.default_rng(5)
+    n = 3000
+    t = np.r_[rng.integers(1, n, 9000), np.arange(1, n)]
+    hd = np.r_[rng.integers(1, n, 9000), np.zeros(n - 1, np.int64)]   # vertex 0: a sink hub
+    order = np.argsort(t, kind="stable")
+    t, hd = t[order], hd[order]
+    first = np.zeros(n + 1, np.uint64)
+    np.add.at(first, t + 1, 1)
+    first = np.cumsum(first).astype(np.uint64)
+    g = phastgen.Graph(n, first, hd.astype(np.uint32), rng.integers(1, 1000, t.size).astype(np.uint32))
+    with P.Phast.from_graph(g) as h:
+        for k in (1, 16):
+            src = phastgen.sources(n, k, seed=960 + k)
+            assert np.array_equal(gpu_trees(h, src), oracle.sssp_many(g, src)), k
+
+
 @pytest.mark.parametrize("window", ["0", "1", "64"])
 def test_wave_sweep_every_k(monkeypatch, window):
     """The warp-wave sweep (plan_waves + sweep_wave_kernel) at every k (each k has its
