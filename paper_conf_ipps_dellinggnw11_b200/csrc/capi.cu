@@ -49,10 +49,15 @@ struct phast_ctx {
     // top levels [0, J) swept in one single-CTA launch (launch_sweep_top), one plan per k
     struct Top {
         uint4* chunks = nullptr;   // device [nchunks] {vbeg, vend, first[vbeg], first[vend]}
-        uint32_t nchunks = 0, J = 0, V = 0;
+        TopArgs a;                 // a.fused: the whole query in this one launch
+        uint32_t J = 0;            // segments [0, J) covered
         bool ok = false;
     };
     std::map<uint32_t, Top> tops;
+    // A-up in-arcs by head {tail, len} (fused single-launch queries on small graphs)
+    uint32_t* d_upin_first = nullptr;
+    uint2* d_upin_arc = nullptr;
+    bool upin_tried = false;
     // 0 = warp pipeline (default), 1 = one launch per level, 2 = CTA waves, 3 = CTA waves + bulk-staged
     // arcs, 4 = pipelined CTA gather (k >= 4; else warp pipeline), 5 = warp dataflow without pipeline
     int sweep_mode = 0;
@@ -131,6 +136,7 @@ void free_device(phast_ctx* h) {
     if (h->side) cudaStreamDestroy(h->side);
     h->side = nullptr;
     cudaFree((void*)h->g.dn_first); cudaFree((void*)h->g.dn_arc);
+    cudaFree((void*)h->g.dn_rec); cudaFree((void*)h->g.dn_ovf);
     cudaFree((void*)h->g.up_first); cudaFree((void*)h->g.up_arc);
     cudaFree(h->g.flags); cudaFree((void*)h->g.tail_bits);
     cudaFree(h->g.seed_v); cudaFree(h->g.seed_d); cudaFree(h->g.seed_cnt);
@@ -138,6 +144,9 @@ void free_device(phast_ctx* h) {
     cudaFree(h->dist_scratch); cudaFree(h->batch_max_scratch);
     cudaFree(h->d_in_first); cudaFree(h->d_in_arc);
     h->d_in_first = nullptr; h->d_in_arc = nullptr;
+    cudaFree(h->d_upin_first); cudaFree(h->d_upin_arc);
+    h->d_upin_first = nullptr; h->d_upin_arc = nullptr;
+    h->upin_tried = false;
     h->g = DevImage();
     h->dist_scratch = nullptr; h->batch_max_scratch = nullptr;
     h->dist_scratch_elems = 0; h->batch_max_elems = 0;
@@ -195,6 +204,38 @@ int upload(phast_ctx* h) {
         return rc;
     }
     g.dn_first = dnf; g.dn_arc = dna; g.up_first = upf; g.up_arc = upa; g.tail_bits = tb;
+    // G-down as ELL-2 records + overflow lists (kernels.h: DevImage::dn_rec)
+    {
+        std::vector<uint4> rec(h->n);
+        std::vector<Arc> ovf;
+        for (uint32_t v = 0; v < h->n; v++) {
+            const uint32_t e0 = L.dn_first[v], deg = L.dn_first[v + 1] - e0;
+            uint4 r = make_uint4(INF, INF, INF, INF);
+            if (deg >= 1) { r.x = L.dn_arc[e0].x; r.y = L.dn_arc[e0].y; }
+            if (deg == 2) { r.z = L.dn_arc[e0 + 1].x; r.w = L.dn_arc[e0 + 1].y; }
+            if (deg > 2) {
+                r.z = (uint32_t)ovf.size();
+                ovf.push_back(Arc{deg - 1, 0});
+                for (uint32_t e = e0 + 1; e < e0 + deg; e++) ovf.push_back(L.dn_arc[e]);
+            }
+            rec[v] = r;
+        }
+        uint4* dr = nullptr;
+        uint2* dov = nullptr;
+        if (ovf.size() >= INF || (rc = dmalloc(&dr, rec.size())) || (rc = dmalloc(&dov, ovf.size()))) {
+            cudaFree(dr);
+            free_device(h);
+            return rc ? rc : PHAST_ERANGE;
+        }
+        g.dn_rec = dr;
+        g.dn_ovf = dov;
+        if (cudaMemcpy(dr, rec.data(), rec.size() * sizeof(uint4), cudaMemcpyHostToDevice) != cudaSuccess ||
+            (!ovf.empty() && cudaMemcpy(dov, ovf.data(), ovf.size() * 8, cudaMemcpyHostToDevice) != cudaSuccess)) {
+            cudaGetLastError();
+            free_device(h);
+            return PHAST_ECUDA;
+        }
+    }
     bool ok = cudaMemset(dnf, 0, (L.dn_first.size() + 4) * 4) == cudaSuccess &&
               cudaMemset(dna, 0, (L.dn_arc.size() + 2) * 8) == cudaSuccess &&
               cudaMemcpy(dnf, L.dn_first.data(), L.dn_first.size() * 4, cudaMemcpyHostToDevice) == cudaSuccess &&
@@ -424,56 +465,125 @@ phast_ctx::Plan* get_plan(phast_ctx* h, uint32_t k) {
     return &P;
 }
 
-// Top levels in one single-CTA launch (kernels.cu: sweep_top_kernel): the longest
-// prefix of levels whose rows [0, V) fit the shared-memory label budget at this k,
-// each level small enough for one SM (<= 32 items per consumer thread) and no vertex
-// with more in-arcs than a chunk holds.  PHAST_TOP=0 disables it; PHAST_TOP_MAXV caps V.
+// Chunks of one segment [a, b) over a CSR (offsets `f`): <= VCH vertices and <= ECH
+// arcs each; chunks without arcs change nothing and are skipped.
+void push_chunks(std::vector<uint4>& ch, const uint32_t* f, uint32_t a, uint32_t b) {
+    const uint32_t VCH = top_chunk_vertices(), ECH = top_chunk_arcs();
+    uint32_t v = a;
+    while (v < b) {
+        uint32_t w = v;
+        while (w < b && w - v < VCH && f[w + 1] - f[v] <= ECH) w++;
+        if (f[w] > f[v]) ch.push_back(make_uint4(v, w, f[v], f[w]));
+        v = w;
+    }
+}
+
+// A-up in-arcs by head, uploaded once (graphs small enough for a fused query).
+bool ensure_upin(phast_ctx* h) {
+    if (h->d_upin_first) return true;
+    if (h->upin_tried) return false;
+    h->upin_tried = true;
+    const Layout& L = h->L;
+    const uint32_t n = h->n;
+    std::vector<uint32_t> f((size_t)n + 1, 0);
+    for (const Arc& a : L.up_arc) f[a.x + 1]++;
+    for (uint32_t v = 0; v < n; v++) f[v + 1] += f[v];
+    std::vector<Arc> arc(L.up_arc.size());
+    std::vector<uint32_t> pos(f.begin(), f.end() - 1);
+    for (uint32_t u = 0; u < n; u++)
+        for (uint32_t e = L.up_first[u]; e < L.up_first[u + 1]; e++) arc[pos[L.up_arc[e].x]++] = Arc{u, L.up_arc[e].y};
+    for (uint32_t v = 0; v < n; v++)
+        if (f[v + 1] - f[v] > top_chunk_arcs()) return false;
+    uint32_t* df = nullptr;
+    uint2* da = nullptr;
+    // +4 / +2 elements: the 16-byte aligned bulk copies may read past the end
+    if (dmalloc(&df, f.size() + 4) || dmalloc(&da, arc.size() + 2)) {
+        cudaFree(df);
+        return false;
+    }
+    if (cudaMemset(df, 0, (f.size() + 4) * 4) != cudaSuccess || cudaMemset(da, 0, (arc.size() + 2) * 8) != cudaSuccess ||
+        cudaMemcpy(df, f.data(), f.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess ||
+        (!arc.empty() && cudaMemcpy(da, arc.data(), arc.size() * 8, cudaMemcpyHostToDevice) != cudaSuccess)) {
+        cudaGetLastError();
+        cudaFree(df);
+        cudaFree(da);
+        return false;
+    }
+    h->d_upin_first = df;
+    h->d_upin_arc = da;
+    return true;
+}
+
+// Shared-memory sweep plans (kernels.cu: sweep_top_kernel), one per k:
+//  - fused: the whole graph's rows fit the label budget -> the whole query (G-up
+//    pull sweep, then the G-down sweep) in one launch.  PHAST_FUSED=0 disables it;
+//  - top: the longest prefix of levels whose rows [0, V) fit, each level small
+//    enough for one SM (<= 32 items per consumer thread); the rest one launch per
+//    level.  PHAST_TOP=0 disables it; PHAST_TOP_MAXV caps V.
+// Both need every vertex to have at most top_chunk_arcs() in-arcs.
 phast_ctx::Top* get_top(phast_ctx* h, uint32_t k) {
     auto it = h->tops.find(k);
     if (it != h->tops.end()) return it->second.ok ? &it->second : nullptr;
     phast_ctx::Top& T = h->tops[k];
-    const char* env = std::getenv("PHAST_TOP");
-    if (env && std::atoi(env) == 0) return nullptr;
     const Layout& L = h->L;
     if (L.mode != LAYOUT_LEVELS && L.mode != LAYOUT_LEVELS_BFS) return nullptr;
     if (L.lvl_off.size() < 2) return nullptr;
-    const uint32_t G = k >= 4 ? k / 4 : 1;
-    uint64_t vmax = top_label_budget() / (4ull * k);
-    if (const char* e = std::getenv("PHAST_TOP_MAXV")) vmax = std::min<uint64_t>(vmax, (uint64_t)std::atoll(e));
-    const uint32_t VCH = top_chunk_vertices(), ECH = top_chunk_arcs();
     const uint32_t nseg = (uint32_t)L.lvl_off.size() - 1;
-    uint32_t J = 0;
-    while (J < nseg) {
-        const uint32_t a = L.lvl_off[J], b = L.lvl_off[J + 1];
-        if (b > vmax || (uint64_t)(b - a) * G > 32ull * 992) break;
-        bool fits = true;
-        for (uint32_t v = a; v < b && fits; v++) fits = L.dn_first[v + 1] - L.dn_first[v] <= ECH;
-        if (!fits) break;
-        J++;
-    }
-    if (J < 2) return nullptr;
+    const uint32_t G = k >= 4 ? k / 4 : 1;
+    const uint32_t ECH = top_chunk_arcs();
+    const uint64_t vmax_budget = top_label_budget() / (4ull * k);
     std::vector<uint4> ch;
-    for (uint32_t j = 0; j < J; j++) {
-        uint32_t v = L.lvl_off[j];
-        const uint32_t b = L.lvl_off[j + 1];
-        while (v < b) {   // greedy chunks inside the level: <= VCH vertices, <= ECH arcs
-            uint32_t w = v;
-            while (w < b && w - v < VCH && L.dn_first[w + 1] - L.dn_first[v] <= ECH) w++;
-            ch.push_back(make_uint4(v, w, L.dn_first[v], L.dn_first[w]));
-            v = w;
+    const char* fe = std::getenv("PHAST_FUSED");
+    bool fused = !(fe && std::atoi(fe) == 0) && h->n <= vmax_budget;
+    for (uint32_t v = 0; fused && v < h->n; v++) fused = L.dn_first[v + 1] - L.dn_first[v] <= ECH;
+    if (fused && ensure_upin(h)) {
+        std::vector<uint32_t> f((size_t)h->n + 1);
+        if (cudaMemcpy(f.data(), h->d_upin_first, f.size() * 4, cudaMemcpyDeviceToHost) != cudaSuccess) {
+            cudaGetLastError();
+            return nullptr;
         }
+        for (uint32_t j = nseg; j-- > 0;) push_chunks(ch, f.data(), L.lvl_off[j], L.lvl_off[j + 1]);   // ascending levels
+        T.a.split = (uint32_t)ch.size();
+        for (uint32_t j = 0; j < nseg; j++) push_chunks(ch, L.dn_first.data(), L.lvl_off[j], L.lvl_off[j + 1]);
+        T.a.first[0] = h->d_upin_first;
+        T.a.arcs[0] = h->d_upin_arc;
+        T.a.fused = 1;
+        T.J = nseg;
+        T.a.V = h->n;
+    } else {
+        const char* env = std::getenv("PHAST_TOP");
+        if (env && std::atoi(env) == 0) return nullptr;
+        uint64_t vmax = vmax_budget;
+        if (const char* e = std::getenv("PHAST_TOP_MAXV")) vmax = std::min<uint64_t>(vmax, (uint64_t)std::atoll(e));
+        uint32_t J = 0;
+        while (J < nseg) {
+            const uint32_t a = L.lvl_off[J], b = L.lvl_off[J + 1];
+            if (b > vmax || (uint64_t)(b - a) * G > 32ull * 992) break;
+            bool fits = true;
+            for (uint32_t v = a; v < b && fits; v++) fits = L.dn_first[v + 1] - L.dn_first[v] <= ECH;
+            if (!fits) break;
+            J++;
+        }
+        if (J < 2) return nullptr;
+        for (uint32_t j = 0; j < J; j++) push_chunks(ch, L.dn_first.data(), L.lvl_off[j], L.lvl_off[j + 1]);
+        T.a.split = 0;
+        T.J = J;
+        T.a.V = L.lvl_off[J];
     }
+    if (ch.empty()) ch.push_back(make_uint4(0, 0, 0, 0));   // keep a valid device array
     if (dmalloc(&T.chunks, ch.size()) ||
         cudaMemcpy(T.chunks, ch.data(), ch.size() * sizeof(uint4), cudaMemcpyHostToDevice) != cudaSuccess) {
         cudaGetLastError();
         return nullptr;
     }
-    T.nchunks = (uint32_t)ch.size();
-    T.J = J;
-    T.V = L.lvl_off[J];
+    T.a.chunks = T.chunks;
+    T.a.nchunks = (ch.size() == 1 && ch[0].y == 0) ? 0u : (uint32_t)ch.size();
+    T.a.first[1] = h->g.dn_first;
+    T.a.arcs[1] = h->g.dn_arc;
     T.ok = true;
     if (std::getenv("PHAST_VERBOSE"))
-        std::fprintf(stderr, "top plan k=%u: %u levels, %u vertices, %u chunks\n", k, J, T.V, T.nchunks);
+        std::fprintf(stderr, "%s plan k=%u: %u levels, %u vertices, %u chunks (%u up)\n",
+                     T.a.fused ? "fused" : "top", k, T.J, T.a.V, T.a.nchunks, T.a.split);
     return &T;
 }
 
@@ -497,6 +607,13 @@ int run_query(phast_ctx* h, const Sources& S, uint32_t k, uint32_t* dist, uint32
         e0 = timing_event(h); e1 = timing_event(h); e2 = timing_event(h);
         if (!e0 || !e1 || !e2) return PHAST_ECUDA;
         cudaEventRecord(e0, st);
+    }
+    phast_ctx::Top* top = get_top(h, k);
+    if (top && top->a.fused) {   // small graph: the whole query (a1-a3, a5) in one launch
+        if (launch_sweep_top(top->a, k, S, dist, h->g.flags, diam, st) != cudaSuccess) return PHAST_ECUDA;
+        if (e1) cudaEventRecord(e1, st);   // no separate upward stage: all of it counts as the sweep
+        if (e2) cudaEventRecord(e2, st);
+        return PHAST_OK;
     }
     // a1 on the side stream (overlaps the previous batch's sweep), a2 on the caller's stream
     const uint32_t slot = h->slot_next;
@@ -537,10 +654,9 @@ int run_query(phast_ctx* h, const Sources& S, uint32_t k, uint32_t* dist, uint32
         const uint32_t levels = (uint32_t)h->L.lvl_off.size() - 1;   // segments
         const bool diagonal = h->L.mode == LAYOUT_DIAGONAL;
         uint32_t j0 = 0;
-        phast_ctx::Top* top = (!plan && !diagonal) ? get_top(h, k) : nullptr;
+        if (plan || diagonal) top = nullptr;
         if (top) {                            // the small top levels in one single-CTA launch
-            if (launch_sweep_top(h->g, k, top->chunks, top->nchunks, top->V, dist, diam, st) != cudaSuccess)
-                return PHAST_ECUDA;
+            if (launch_sweep_top(top->a, k, S, dist, h->g.flags, diam, st) != cudaSuccess) return PHAST_ECUDA;
             j0 = top->J;
         } else if (plan) {                    // hybrid: small top levels in one persistent launch
             if ((uint64_t)(plan->epoch + 1) * plan->p.grid >= 0x7FFFFFFFull) {

@@ -239,6 +239,7 @@ template <> __device__ __forceinline__ uint4 inf_row<uint4>() { return make_uint
 template <class T> __device__ __forceinline__ void st_stream(T* p, T v) { __stcs(p, v); }
 
 constexpr int SWEEP_THREADS = 256;
+constexpr int ELL = 16;   // sweep_kernel AB value: ELL-2 records (DevImage::dn_rec) instead of the CSR
 
 // One level [vbeg, vend) (§VI "The CPU starts, for each level i, a kernel on
 // the GPU").  One (vertex, 16-byte lane) item per thread per grid-stride step; the
@@ -254,6 +255,8 @@ constexpr int SWEEP_THREADS = 256;
 template <int K, bool DIAM, bool STORE, bool STREAM, bool TB, int AB>
 __global__ void __launch_bounds__(SWEEP_THREADS, AB >= 3 && AB < 8 ? 6 : 8) sweep_kernel(const uint32_t* __restrict__ first,
                                                                const uint2* __restrict__ arcs,
+                                                               const uint4* __restrict__ rec,
+                                                               const uint2* __restrict__ ovf,
                                                                uint32_t* __restrict__ d,
                                                                const uint32_t* __restrict__ flags,
                                                                const uint32_t* __restrict__ tail_bits,
@@ -270,8 +273,12 @@ __global__ void __launch_bounds__(SWEEP_THREADS, AB >= 3 && AB < 8 ? 6 : 8) swee
     // re-reads them (L1 / L2 hits) so that it keeps its register budget.
     uint32_t t = blockIdx.x * SWEEP_THREADS + threadIdx.x;
     if (t < total) {
-        const uint32_t e0 = __ldg(&first[vbeg + t / G]);
-        asm volatile("prefetch.global.L2 [%0];" ::"l"(arcs + e0));
+        if constexpr (AB == ELL) {
+            asm volatile("prefetch.global.L2 [%0];" ::"l"(rec + vbeg + t / G));
+        } else {
+            const uint32_t e0 = __ldg(&first[vbeg + t / G]);
+            asm volatile("prefetch.global.L2 [%0];" ::"l"(arcs + e0));
+        }
     }
     asm volatile("griddepcontrol.wait;" ::: "memory");          // previous level complete and visible
     uint32_t mx = 0;
@@ -281,6 +288,25 @@ __global__ void __launch_bounds__(SWEEP_THREADS, AB >= 3 && AB < 8 ? 6 : 8) swee
         T acc = inf_row<T>();
         if ((__ldg(&flags[v >> 5]) >> (v & 31)) & 1u)   // visited by an upward search
             acc = __ldg(reinterpret_cast<const T*>(d + (size_t)v * K) + lane);
+        if constexpr (AB == ELL) {
+            // one 16-byte record: the vertex's first two in-arcs (97 % of level-0 and
+            // 92 % of level-1 vertices have at most two), so the gather depends on ONE
+            // load instead of offsets -> arcs
+            // (a missing arc has len INF: relaxing an INF row by it changes nothing)
+            const uint4 r = __ldg(&rec[v]);
+            T x0 = inf_row<T>(), x1 = inf_row<T>();
+            if (r.y != INF) x0 = __ldg(reinterpret_cast<const T*>(d + (size_t)r.x * K) + lane);
+            if (r.w != INF) x1 = __ldg(reinterpret_cast<const T*>(d + (size_t)r.z * K) + lane);
+            acc = relax(relax(acc, x0, r.y), x1, r.w);
+            if (r.w == INF && r.z != INF) {   // more than two in-arcs: the rest in the overflow list
+                const uint2* o = ovf + r.z;
+                const uint32_t cnt = __ldg(&o->x);
+                for (uint32_t j = 1; j <= cnt; j++) {
+                    const uint2 a = __ldg(&o[j]);
+                    acc = relax(acc, __ldg(reinterpret_cast<const T*>(d + (size_t)a.x * K) + lane), a.y);
+                }
+            }
+        } else {
         const uint32_t e0 = __ldg(&first[v]), e1 = __ldg(&first[v + 1]);
         if constexpr (AB == 1) {
 #pragma unroll 4
@@ -326,6 +352,7 @@ __global__ void __launch_bounds__(SWEEP_THREADS, AB >= 3 && AB < 8 ? 6 : 8) swee
                     if (e + r < e1) acc = relax(acc, x[r], a[r].y);
             }
         }
+        }   // CSR path
         if constexpr (TB) {
             T* p = reinterpret_cast<T*>(d + (size_t)v * K) + lane;
             if ((__ldg(&tail_bits[v >> 5]) >> (v & 31)) & 1u) *p = acc;
@@ -349,10 +376,10 @@ __global__ void __launch_bounds__(SWEEP_THREADS, AB >= 3 && AB < 8 ? 6 : 8) swee
     }
 }
 
-int arc_batch() {   // PHAST_ARC_BATCH: 1, 2 (default), 3, 4 or 8 (staged; sweep_kernel AB), read per launch
+int arc_batch() {   // PHAST_ARC_BATCH: 1, 2, 3, 4, 8 (staged) or 16 (ELL-2 records, default); read per launch
     const char* e = std::getenv("PHAST_ARC_BATCH");
-    int b = e ? std::atoi(e) : 2;
-    if (b != 8 && (b < 1 || b > 4)) b = 2;
+    int b = e ? std::atoi(e) : ELL;
+    if (b != 8 && b != ELL && (b < 1 || b > 4)) b = ELL;
     return b;
 }
 
@@ -380,14 +407,16 @@ cudaError_t sweep_launch(const DevImage& g, uint32_t vbeg, uint32_t vend, uint32
     attr[0].val.programmaticStreamSerializationAllowed = 1;
     cfg.attrs = attr;
     cfg.numAttrs = 1;
-    const int ab = arc_batch();
-    cudaError_t e = cudaLaunchKernelEx(&cfg, ab == 8 ? sweep_kernel<K, DIAM, STORE, STREAM, TB, 8>
+    int ab = arc_batch();
+    if (ab == ELL && !g.dn_rec) ab = 2;
+    cudaError_t e = cudaLaunchKernelEx(&cfg, ab == ELL ? sweep_kernel<K, DIAM, STORE, STREAM, TB, ELL>
+                                             : ab == 8 ? sweep_kernel<K, DIAM, STORE, STREAM, TB, 8>
                                              : ab == 4 ? sweep_kernel<K, DIAM, STORE, STREAM, TB, 4>
                                              : ab == 3 ? sweep_kernel<K, DIAM, STORE, STREAM, TB, 3>
                                              : ab == 2 ? sweep_kernel<K, DIAM, STORE, STREAM, TB, 2>
                                                        : sweep_kernel<K, DIAM, STORE, STREAM, TB, 1>,
-                                       g.dn_first, g.dn_arc, dist, (const uint32_t*)g.flags, g.tail_bits, vbeg, vend,
-                                       diam);
+                                       g.dn_first, g.dn_arc, g.dn_rec, g.dn_ovf, dist, (const uint32_t*)g.flags,
+                                       g.tail_bits, vbeg, vend, diam);
     g_launches++;
     return e;
 }
@@ -1643,21 +1672,33 @@ __global__ void max_reduce_kernel(const uint32_t* __restrict__ in, uint32_t coun
 // (§VI "The CPU starts, for each level i, a kernel on the GPU") costs
 // ~4 us of launch + drain per level however small it is, so the levels whose rows
 // fit in shared memory run in ONE CTA instead:
-//  - the rows of [0, V) (the top levels: internal ids ascend as levels descend) are
-//    loaded once into shared memory (seeded label if visited, else INF: PAPER.md:16
-//    §IV-C), swept there level by level, and written back once;
+//  - the rows of [0, V) (the top levels: internal ids ascend as levels descend) live
+//    in shared memory for the whole launch and are written back once;
 //  - warp 0 is a producer: one elected thread streams every chunk's offsets and
-//    arcs (contiguous per level, §IV-A) into a 3-stage shared-memory ring
-//    with bulk copies (TMA, cp.async.bulk) signalled on mbarriers, ahead of use;
+//    arcs (contiguous per level, §IV-A) into a ring of `stages`
+//    shared-memory stages with bulk copies (TMA, cp.async.bulk) signalled on
+//    mbarriers, as far ahead as the ring allows (the copies, not the relaxations,
+//    are the latency: the ring is as deep as shared memory permits);
 //  - 31 consumer warps relax one chunk at a time from shared memory
 //    (§III "if d(v) > d(u)+l(u,v), we set d(v) = d(u)+l(u,v)") and meet
 //    at a named barrier after it, which orders the levels (Lemma 4.1: every tail is
 //    in an earlier chunk) and frees the ring stage.
-// A level boundary costs one named barrier (~tens of ns) instead of a launch.
-constexpr int TOP_THREADS = 1024, TOP_CONS = TOP_THREADS - 32, TOP_STAGES = 3;
-constexpr uint32_t TOP_VCH = 1024, TOP_ECH = 2048;                // per chunk: vertices, arcs
+// Two initialisations:
+//  - top mode (fused = 0): rows = seeded label if visited, else INF (PAPER.md:16
+//    §IV-C); the upward searches and the seeding ran before;
+//  - fused mode (fused = 1, V = n, the whole graph): rows = INF except d_i(s_i) = 0,
+//    and the chunks [0, split) are a PULL sweep of G-up in ascending level order
+//    (in-arcs of A-up by head): afterwards every row holds the exact G-up distance
+//    from its source, INF where G-up does not reach -- the result of the upward CH
+//    search run to exhaustion (§III "it runs Dijkstra s algorithm from s
+//    in G, stopping when the priority queue becomes empty"; reading R9), for every
+//    vertex at once.  The chunks [split, nchunks) are then the downward sweep.  One
+//    launch per query: no upward kernel, no seeding, no visited bits.
+constexpr int TOP_THREADS = 1024, TOP_CONS = TOP_THREADS - 32;
+constexpr uint32_t TOP_VCH = 256, TOP_ECH = 1024;                 // per chunk: vertices, arcs
 constexpr uint32_t TOP_OFF_BUF = TOP_VCH + 8, TOP_ARC_BUF = TOP_ECH + 2;
-constexpr size_t TOP_RING_BYTES = (size_t)TOP_STAGES * (TOP_OFF_BUF * 4 + TOP_ARC_BUF * 8);
+constexpr size_t TOP_STAGE_BYTES = 16 + TOP_OFF_BUF * 4 + TOP_ARC_BUF * 8;   // {descriptor, offsets, arcs}: 9 280
+constexpr uint32_t TOP_MAX_STAGES = 24, TOP_MIN_STAGES = 4;
 constexpr size_t TOP_SMEM_MAX = 227 * 1024;
 
 __device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
@@ -1665,61 +1706,81 @@ __device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
 }
 
 template <int K, bool DIAM>
-__global__ void __launch_bounds__(TOP_THREADS, 1) sweep_top_kernel(const uint32_t* __restrict__ first,
-                                                                   const uint2* __restrict__ arcs,
-                                                                   uint32_t* __restrict__ d,
+__global__ void __launch_bounds__(TOP_THREADS, 1) sweep_top_kernel(TopArgs A, Sources src, uint32_t* __restrict__ d,
                                                                    const uint32_t* __restrict__ flags,
-                                                                   const uint4* __restrict__ chunks,
-                                                                   uint32_t nchunks, uint32_t V,
                                                                    uint32_t* __restrict__ diam) {
     using T = typename RowT<K>::T;
-    constexpr uint32_t G = K / RowT<K>::W;   // lanes per vertex
+    constexpr uint32_t W = RowT<K>::W;
+    constexpr uint32_t G = K / W;   // lanes per vertex
     extern __shared__ __align__(16) unsigned char top_smem[];
+    const uint32_t V = A.V, S = A.stages;
     T* srow = reinterpret_cast<T*>(top_smem);
     const size_t lab = ((size_t)V * G * sizeof(T) + 15) & ~(size_t)15;
-    uint32_t* soff = reinterpret_cast<uint32_t*>(top_smem + lab);                              // [S][OFF_BUF]
-    uint2* sarc = reinterpret_cast<uint2*>(top_smem + lab + (size_t)TOP_STAGES * TOP_OFF_BUF * 4);   // [S][ARC_BUF]
-    uint64_t* full = reinterpret_cast<uint64_t*>(top_smem + lab + TOP_RING_BYTES);
-    uint64_t* empty = full + TOP_STAGES;
+    unsigned char* ring = top_smem + lab;                                   // [S] {offsets, arcs}
+    uint64_t* full = reinterpret_cast<uint64_t*>(ring + (size_t)S * TOP_STAGE_BYTES);
+    uint64_t* empty = full + S;
     const uint32_t tid = threadIdx.x;
     if (tid == 0) {
-        for (int s = 0; s < TOP_STAGES; s++) {
+        for (uint32_t s = 0; s < S; s++) {
             mbar_init(&full[s], 1);
             mbar_init(&empty[s], 1);
         }
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
-    // a2 (implicit init): the top rows, seeded label if visited else INF
     const T* dr = reinterpret_cast<const T*>(d);
-    for (uint32_t i = tid; i < V * G; i += TOP_THREADS) {
-        const uint32_t v = i / G;
-        srow[i] = ((__ldg(&flags[v >> 5]) >> (v & 31)) & 1u) ? dr[i] : inf_row<T>();
+    if (A.fused) {   // every row INF, then d_i(s_i) = 0
+        for (uint32_t i = tid; i < V * G; i += TOP_THREADS) srow[i] = inf_row<T>();
+        __syncthreads();
+        if (tid < K) reinterpret_cast<uint32_t*>(srow)[(size_t)src.s[tid] * K + tid] = 0u;
+    } else {         // a2 (implicit init): seeded label if visited, else INF
+        for (uint32_t i = tid; i < V * G; i += TOP_THREADS) {
+            const uint32_t v = i / G;
+            srow[i] = ((__ldg(&flags[v >> 5]) >> (v & 31)) & 1u) ? dr[i] : inf_row<T>();
+        }
     }
     __syncthreads();
     uint32_t mx = 0;
-    if (tid < 32) {   // producer warp: one elected thread issues the bulk copies
-        if (tid == 0) {
-            for (uint32_t c = 0; c < nchunks; c++) {
-                const uint32_t s = c % TOP_STAGES;
-                if (c >= TOP_STAGES) mbar_wait(&empty[s], ((c / TOP_STAGES) - 1) & 1);
-                const uint4 ch = __ldg(&chunks[c]);   // {vbeg, vend, ebeg = first[vbeg], eend = first[vend]}
+    if (tid < 32) {   // producer warp: lane 0 issues the bulk copies
+        // descriptors: each lane holds one of the current 32 and one of the next 32
+        // (loaded a batch ahead), so the issue loop never waits on a global load
+        const uint32_t lane = tid;
+        uint4 cur = make_uint4(0, 0, 0, 0), nxt = make_uint4(0, 0, 0, 0);
+        if (lane < A.nchunks) cur = __ldg(&A.chunks[lane]);
+        if (32 + lane < A.nchunks) nxt = __ldg(&A.chunks[32 + lane]);
+        for (uint32_t c = 0; c < A.nchunks; c++) {
+            const uint32_t s = c % S;
+            if ((c & 31) == 0 && c) {
+                cur = nxt;
+                if (c + 32 + lane < A.nchunks) nxt = __ldg(&A.chunks[c + 32 + lane]);
+            }
+            uint4 ch;   // {vbeg, vend, ebeg = first[vbeg], eend = first[vend]}
+            ch.x = __shfl_sync(0xFFFFFFFFu, cur.x, c & 31);
+            ch.y = __shfl_sync(0xFFFFFFFFu, cur.y, c & 31);
+            ch.z = __shfl_sync(0xFFFFFFFFu, cur.z, c & 31);
+            ch.w = __shfl_sync(0xFFFFFFFFu, cur.w, c & 31);
+            if (lane == 0) {
+                if (c >= S) mbar_wait(&empty[s], ((c / S) - 1) & 1);
+                const bool up = c < A.split;
                 const uint32_t f0 = ch.x & ~3u, nf = (ch.y + 1 - f0 + 3) & ~3u;   // 16-byte aligned copies
                 const uint32_t a0 = ch.z & ~1u, na = (ch.w - a0 + 1) & ~1u;
-                mbar_arrive_tx(&full[s], nf * 4 + na * 8);
-                bulk_g2s(soff + s * TOP_OFF_BUF, first + f0, nf * 4, &full[s]);
-                if (na) bulk_g2s(sarc + s * TOP_ARC_BUF, arcs + a0, na * 8, &full[s]);
+                unsigned char* st = ring + (size_t)s * TOP_STAGE_BYTES;
+                mbar_arrive_tx(&full[s], 16 + nf * 4 + na * 8);
+                bulk_g2s(st, A.chunks + c, 16, &full[s]);   // the consumers read the descriptor here
+                bulk_g2s(st + 16, (up ? A.first[0] : A.first[1]) + f0, nf * 4, &full[s]);
+                if (na) bulk_g2s(st + 16 + TOP_OFF_BUF * 4, (up ? A.arcs[0] : A.arcs[1]) + a0, na * 8, &full[s]);
             }
+            __syncwarp();
         }
-        __syncwarp();
     } else {
         const uint32_t ct = tid - 32;
-        for (uint32_t c = 0; c < nchunks; c++) {
-            const uint32_t s = c % TOP_STAGES;
-            const uint4 ch = __ldg(&chunks[c]);
-            mbar_wait(&full[s], (c / TOP_STAGES) & 1);
+        for (uint32_t c = 0; c < A.nchunks; c++) {
+            const uint32_t s = c % S;
+            mbar_wait(&full[s], (c / S) & 1);
+            const unsigned char* st = ring + (size_t)s * TOP_STAGE_BYTES;
+            const uint4 ch = *reinterpret_cast<const uint4*>(st);
             const uint32_t f0 = ch.x & ~3u, a0 = ch.z & ~1u;
-            const uint32_t* sf = soff + s * TOP_OFF_BUF;
-            const uint2* sa = sarc + s * TOP_ARC_BUF;
+            const uint32_t* sf = reinterpret_cast<const uint32_t*>(st + 16);
+            const uint2* sa = reinterpret_cast<const uint2*>(st + 16 + TOP_OFF_BUF * 4);
             const uint32_t total = (ch.y - ch.x) * G;
             for (uint32_t t = ct; t < total; t += TOP_CONS) {
                 const uint32_t v = ch.x + t / G, lane = t % G;
@@ -1730,7 +1791,6 @@ __global__ void __launch_bounds__(TOP_THREADS, 1) sweep_top_kernel(const uint32_
                     acc = relax(acc, srow[a.x * G + lane], a.y);
                 }
                 srow[v * G + lane] = acc;
-                if constexpr (DIAM) mx = max(mx, fmax_of(acc));
             }
             asm volatile("bar.sync 1, %0;" ::"n"(TOP_CONS) : "memory");   // chunk done: next level may read it
             if (ct == 0) mbar_arrive(&empty[s]);                          // ring stage free
@@ -1738,25 +1798,28 @@ __global__ void __launch_bounds__(TOP_THREADS, 1) sweep_top_kernel(const uint32_
     }
     __syncthreads();
     T* dw = reinterpret_cast<T*>(d);
-    for (uint32_t i = tid; i < V * G; i += TOP_THREADS) dw[i] = srow[i];
+    for (uint32_t i = tid; i < V * G; i += TOP_THREADS) {   // final rows (a5: the fused max over them)
+        dw[i] = srow[i];
+        if constexpr (DIAM) mx = max(mx, fmax_of(srow[i]));
+    }
     if constexpr (DIAM) {
         mx = __reduce_max_sync(0xFFFFFFFFu, mx);
         if ((tid & 31) == 0 && mx) atomicMax(diam, mx);
     }
 }
 
-size_t top_smem_bytes(uint32_t k, uint32_t V) {
-    const size_t lab = ((size_t)V * k * 4 + 15) & ~(size_t)15;
-    return lab + TOP_RING_BYTES + 2 * TOP_STAGES * sizeof(uint64_t);
-}
-size_t top_label_budget() { return TOP_SMEM_MAX - TOP_RING_BYTES - 2 * TOP_STAGES * sizeof(uint64_t) - 16; }
+size_t top_ring_min() { return TOP_MIN_STAGES * TOP_STAGE_BYTES + 2 * TOP_MIN_STAGES * sizeof(uint64_t); }
+size_t top_label_budget() { return TOP_SMEM_MAX - top_ring_min() - 16; }
 uint32_t top_chunk_vertices() { return TOP_VCH; }
 uint32_t top_chunk_arcs() { return TOP_ECH; }
 
 template <int K>
-cudaError_t top_k(const DevImage& g, const uint4* chunks, uint32_t nchunks, uint32_t V, uint32_t* dist,
-                  uint32_t* diam, cudaStream_t st) {
-    const size_t smem = top_smem_bytes(K, V);
+cudaError_t top_k(TopArgs A, const Sources& src, uint32_t* dist, const uint32_t* flags, uint32_t* diam,
+                  cudaStream_t st) {
+    const size_t lab = ((size_t)A.V * K * 4 + 15) & ~(size_t)15;
+    if (lab > top_label_budget()) return cudaErrorInvalidValue;
+    A.stages = (uint32_t)std::min<size_t>(TOP_MAX_STAGES, (TOP_SMEM_MAX - lab) / (TOP_STAGE_BYTES + 16));
+    const size_t smem = lab + A.stages * (TOP_STAGE_BYTES + 16);
     static bool attr_set[2] = {false, false};
     auto kern = diam ? sweep_top_kernel<K, true> : sweep_top_kernel<K, false>;
     if (!attr_set[diam ? 1 : 0]) {
@@ -1764,7 +1827,7 @@ cudaError_t top_k(const DevImage& g, const uint4* chunks, uint32_t nchunks, uint
         if (e != cudaSuccess) return e;
         attr_set[diam ? 1 : 0] = true;
     }
-    kern<<<1, TOP_THREADS, smem, st>>>(g.dn_first, g.dn_arc, dist, g.flags, chunks, nchunks, V, diam);
+    kern<<<1, TOP_THREADS, smem, st>>>(A, src, dist, flags, diam);
     g_launches++;
     return cudaGetLastError();
 }
@@ -1884,9 +1947,9 @@ cudaError_t launch_parents(const uint32_t* in_first, const uint2* in_arc, uint32
 #undef CALL_PA
 }
 
-cudaError_t launch_sweep_top(const DevImage& g, uint32_t k, const uint4* chunks, uint32_t nchunks, uint32_t V,
-                             uint32_t* dist, uint32_t* diam, cudaStream_t st) {
-#define CALL_TOP(K) top_k<K>(g, chunks, nchunks, V, dist, diam, st)
+cudaError_t launch_sweep_top(const TopArgs& A, uint32_t k, const Sources& src, uint32_t* dist,
+                             const uint32_t* flags, uint32_t* diam, cudaStream_t st) {
+#define CALL_TOP(K) top_k<K>(A, src, dist, flags, diam, st)
     PHAST_K_SWITCH(k, CALL_TOP)
 #undef CALL_TOP
 }

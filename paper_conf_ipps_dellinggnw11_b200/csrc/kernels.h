@@ -14,6 +14,12 @@ struct DevImage {
     uint32_t n = 0;
     const uint32_t* dn_first = nullptr;  // [n+1]   G-down in-arcs by head (internal ids)
     const uint2* dn_arc = nullptr;       // [m_down] {tail, len}
+    // G-down as ELL-2 records (the per-level sweep's default): rec[v] = {tail0, len0,
+    // tail1, len1}; len = INF marks "no arc" (arcs of length INF never exist in G-down,
+    // reading R1); len1 = INF with tail1 != INF: more than two in-arcs, tail1 indexes
+    // dn_ovf = {count, 0} followed by the remaining count arcs {tail, len}
+    const uint4* dn_rec = nullptr;       // [n]
+    const uint2* dn_ovf = nullptr;       // [overflow entries]
     const uint32_t* up_first = nullptr;  // [n+1]   G-up out-arcs by tail
     const uint2* up_arc = nullptr;       // [m_up]   {head, len}
     uint32_t* flags = nullptr;           // [ceil(n/32)] visited bits (§IV-C), zero between calls
@@ -95,11 +101,22 @@ cudaError_t launch_parents(const uint32_t* in_first, const uint2* in_arc, uint32
                            uint32_t k, const uint32_t* dist, uint32_t* parent, cudaStream_t st);
 
 // a3 + a4 for the top levels [0, V) in ONE single-CTA launch (labels in shared
-// memory, arcs streamed by TMA): chunks[c] = {vbeg, vend, first[vbeg], first[vend]},
-// level-ordered, at most top_chunk_vertices() vertices and top_chunk_arcs() arcs
+// memory, arcs streamed by TMA through an mbarrier ring).  chunks[c] = {vbeg, vend,
+// first[vbeg], first[vend]} over CSR first[0]/arcs[0] for c < split (fused mode: the
+// G-up pull sweep, ascending levels) and CSR first[1]/arcs[1] after (G-down,
+// descending levels); at most top_chunk_vertices() vertices and top_chunk_arcs() arcs
 // each, never spanning two levels; V * k * 4 <= top_label_budget().
-cudaError_t launch_sweep_top(const DevImage& g, uint32_t k, const uint4* chunks, uint32_t nchunks, uint32_t V,
-                             uint32_t* dist, uint32_t* diam, cudaStream_t st);
+//   fused = 0: rows start from the seeded rows / visited bits (after a1, a2);
+//   fused = 1: V = n, rows start at INF with d_i(src.s[i]) = 0 -- the whole query
+//   (a1 as a pull sweep of G-up, a2, a3) in one launch.
+struct TopArgs {
+    const uint32_t* first[2] = {nullptr, nullptr};
+    const uint2* arcs[2] = {nullptr, nullptr};
+    const uint4* chunks = nullptr;
+    uint32_t split = 0, nchunks = 0, V = 0, stages = 0, fused = 0;
+};
+cudaError_t launch_sweep_top(const TopArgs& A, uint32_t k, const Sources& src, uint32_t* dist,
+                             const uint32_t* flags, uint32_t* diam, cudaStream_t st);
 size_t top_label_budget();
 uint32_t top_chunk_vertices();
 uint32_t top_chunk_arcs();

@@ -50,7 +50,7 @@ def _load():
                                 ctypes.c_uint64, P]
         lib.pg_road.argtypes = [ctypes.c_uint32, ctypes.c_uint32, ctypes.c_double,
                                 ctypes.POINTER(ctypes.c_double), ctypes.c_double, ctypes.c_uint32,
-                                ctypes.c_uint64, P]
+                                ctypes.c_uint64, ctypes.c_uint32, P]
         lib.pg_random_digraph.argtypes = [ctypes.c_uint32, ctypes.c_uint64, ctypes.c_uint32,
                                           ctypes.c_uint32, ctypes.c_uint64, P]
         lib.pg_sources.argtypes = [ctypes.c_uint32, ctypes.c_uint64, ctypes.c_int, ctypes.c_uint64,
@@ -108,16 +108,22 @@ _ROAD_PRESETS = {
 }
 
 
-def road(n_target: int, seed: int, preset: str = "europe", base: int = 1000) -> Graph:
-    """Road-like graph with about n_target vertices in DFS layout (see gen.c)."""
+def road(n_target: int, seed: int, preset: str = "europe", base: int = 1000, metric: str = "time") -> Graph:
+    """Road-like graph with about n_target vertices in DFS layout (see gen.c).
+    metric "time" (travel times, road classes 1/2/4/8x faster) or "distance" (every
+    class speed 1: the paper's travel-distance metric, deeper hierarchies,
+    PAPER.md:26 §VIII-G)."""
     p = _ROAD_PRESETS[preset]
     side = max(2, int(round(math.sqrt(n_target / p["per_int"]))))
     shape = (ctypes.c_double * 4)(*p["shape"])
     g = _PgGraph()
-    rc = _load().pg_road(side, side, p["p_keep"], shape, p["oneway"], base, seed, ctypes.byref(g))
+    if metric not in ("time", "distance"):
+        raise ValueError("metric must be 'time' or 'distance'")
+    rc = _load().pg_road(side, side, p["p_keep"], shape, p["oneway"], base, seed, int(metric == "distance"),
+                         ctypes.byref(g))
     if rc != 0:
         raise ValueError(f"pg_road failed: {rc}")
-    return _take(g, f"road-{preset}-{n_target}-s{seed}")
+    return _take(g, f"road-{preset}-{metric}-{n_target}-s{seed}")
 
 
 def random_digraph(n: int, m: int, lo: int, hi: int, seed: int) -> Graph:
@@ -149,4 +155,7 @@ CONFIGS = {
                desc="road-like ~24M vertices / ~58M arcs (USA-scale), 8192 sources"),
     "C5": dict(graph=lambda: road(1_000_000, seed=5), src_seed=105, k=64,
                desc="road-like ~1M vertices, diameter over all sources"),
+    # NEXT-4: the travel-DISTANCE metric (deeper hierarchy, §VIII-G)
+    "C2D": dict(graph=lambda: road(1_000_000, seed=2, metric="distance"), src_seed=102, k=16,
+                desc="road-like ~1M vertices, travel-distance metric, k=16"),
 }

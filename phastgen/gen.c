@@ -100,7 +100,9 @@ int pg_grid(uint32_t W, uint32_t H, uint32_t lo, uint32_t hi, uint64_t seed, pg_
  *   class-0 edges become one-way (random direction) with probability oneway.
  *   Each kept edge is subdivided by s shape vertices, P(s=j) = shape_p[j], j<4.
  *   Edge travel time T = round(base * U(0.8,1.2) / speed), split over the s+1
- *   segments with weights U(0.5,1.5), every segment >= 1.
+ *   segments with weights U(0.5,1.5), every segment >= 1.  metric = 1 (travel
+ *   DISTANCE, §VIII-G "generating upwards and downwards graphs with 410
+ *   levels"): every class has speed 1, so the length is the geometric length.
  *   Finally ids are relabelled in DFS discovery order from a seeded random vertex
  *   (undirected DFS, neighbours in stored order).
  */
@@ -119,7 +121,7 @@ static int road_class(uint32_t i) {
 }
 
 int pg_road(uint32_t W, uint32_t H, double p_keep, const double *shape_p, double oneway,
-            uint32_t base, uint64_t seed, pg_graph *g) {
+            uint32_t base, uint64_t seed, uint32_t metric, pg_graph *g) {
     memset(g, 0, sizeof(*g));
     if (W < 2 || H < 2) return -1;
     uint64_t NI = (uint64_t)W * H;
@@ -196,7 +198,7 @@ int pg_road(uint32_t W, uint32_t H, double p_keep, const double *shape_p, double
     for (uint64_t i = 0; i < NE; i++) {
         if (!E[i].keep) continue;
         int s = ns[i];
-        double T = (double)base * (0.8 + 0.4 * rndu(seed, 7, i)) / speed[E[i].cls];
+        double T = (double)base * (0.8 + 0.4 * rndu(seed, 7, i)) / (metric ? 1.0 : speed[E[i].cls]);
         double w[4], ws = 0;
         for (int j = 0; j <= s; j++) { w[j] = 0.5 + rndu(seed, 8, i * 4 + j); ws += w[j]; }
         uint32_t chain[5];

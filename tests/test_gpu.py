@@ -141,6 +141,7 @@ def test_upward_global_fallback_and_overflow(monkeypatch):
     g = phastgen.grid(100, 100, 1, 1 << 20, seed=1)   # upward spaces ~200-300 vertices
     src = phastgen.sources(g.n, 16, seed=3)
     want = oracle.sssp_many(g, src)
+    monkeypatch.setenv("PHAST_FUSED", "0")             # the upward-search kernel, not the fused pull sweep
     monkeypatch.setenv("PHAST_UP_SMEM_CAP", "32")
     with P.Phast.from_graph(g) as h:
         assert np.array_equal(gpu_trees(h, src), want)
@@ -204,23 +205,45 @@ def test_sweep_modes(monkeypatch, mode, level_layout, delta):
         assert h.diameter(src, k_batch=64) == oracle.diameter(g, src)
 
 
-@pytest.mark.parametrize("top", ["0", "1", "40", "700", "3000"])
+@pytest.mark.parametrize("top", ["off", "default", "nofused", "40", "700", "3000"])
 def test_top_levels_kernel(monkeypatch, top):
-    """The top levels in one single-CTA launch (sweep_top_kernel: rows in shared
-    memory, TMA-staged arc chunks): off ("0"), default ("1", the whole 10 k grid at
-    k <= 4), and capped at V <= 40 / 700 / 3000 vertices (the prefix ends inside the
-    hierarchy, chunks split long levels), every k, bit-exact; plus the diameter."""
-    if top == "0":
+    """The shared-memory sweep (sweep_top_kernel: rows in shared memory, TMA-staged
+    arc chunks): off (one launch per level), default (C1 at k <= 4: the whole query
+    fused in one launch, G-up as a pull sweep; larger k / the road graph: the top
+    levels), top levels only ("nofused"), and top levels capped at V <= 40 / 700 /
+    3000 vertices (the prefix ends inside the hierarchy, chunks split long levels);
+    every k, bit-exact; plus the diameter (fused max over the final rows)."""
+    if top == "off":
         monkeypatch.setenv("PHAST_TOP", "0")
-    elif top != "1":
+        monkeypatch.setenv("PHAST_FUSED", "0")
+    elif top == "nofused":
+        monkeypatch.setenv("PHAST_FUSED", "0")
+    elif top != "default":
+        monkeypatch.setenv("PHAST_FUSED", "0")
         monkeypatch.setenv("PHAST_TOP_MAXV", top)
-    for g in (phastgen.CONFIGS["C1"]["graph"](), phastgen.road(60_000, seed=35)):
+    for g in (phastgen.CONFIGS["C1"]["graph"](), phastgen.road(60_000, seed=35), phastgen.road(9_000, seed=36)):
         with P.Phast.from_graph(g) as h:
             for k in (1, 2, 4, 16, 64):
                 src = phastgen.sources(g.n, k, seed=950 + k)
                 assert np.array_equal(gpu_trees(h, src), oracle.sssp_many(g, src)), (k, top)
-            src = phastgen.sources(g.n, 130, seed=951)
-            assert h.diameter(src, k_batch=4) == oracle.diameter(g, src)
+            for kb in (1, 4, 16):
+                src = phastgen.sources(g.n, 130, seed=951)
+                assert h.diameter(src, k_batch=kb) == oracle.diameter(g, src), kb
+
+
+def test_fused_query_edge_cases(monkeypatch):
+    """The fused single-launch query on graphs with unreachable parts, one-way arcs,
+    zero and near-2^32 lengths (random digraphs), duplicate sources; bit-exact, and
+    again with the per-level path for comparison."""
+    for seed in range(6):
+        g = phastgen.random_digraph(400 + 50 * seed, 1500 + 300 * seed, 0 if seed % 2 else 1,
+                                    (1 << 32) - 1 if seed == 5 else 1 << 20, seed=70 + seed)
+        for fused in ("1", "0"):
+            monkeypatch.setenv("PHAST_FUSED", fused)
+            with P.Phast.from_graph(g) as h:
+                for k in (1, 4, 16):
+                    src = phastgen.sources(g.n, k, seed=seed, distinct=False)
+                    assert np.array_equal(gpu_trees(h, src), oracle.sssp_many(g, src)), (seed, fused, k)
 
 
 def test_top_levels_hub_vertex():
@@ -310,6 +333,19 @@ def test_diameter_road_and_unreachable(road):
     with P.Phast.from_graph(g2) as h2:
         src = np.arange(0, g2.n, 7, dtype=np.uint32)
         assert h2.diameter(src, k_batch=64) == oracle.diameter(g2, src)
+
+
+def test_distance_metric_deep_hierarchy():
+    """NEXT-4: the travel-distance metric (§VIII-G: 410 levels instead of
+    140 on Europe) gives a much deeper hierarchy; every schedule stays bit-exact."""
+    g = phastgen.road(40_000, seed=37, metric="distance")
+    with P.Phast.from_graph(g) as h:
+        assert h.levels > 60
+        for k in (1, 16, 64):
+            src = phastgen.sources(g.n, k, seed=970 + k)
+            assert np.array_equal(gpu_trees(h, src), oracle.sssp_many(g, src)), k
+        src = phastgen.sources(g.n, 100, seed=971)
+        assert h.diameter(src, k_batch=16) == oracle.diameter(g, src)
 
 
 def test_c2_1m_k16():

@@ -43,6 +43,7 @@ GRAPHS = {
     "grid": lambda: phastgen.grid(60, 40, 1, 1 << 20, seed=1),
     "unit_grid": lambda: phastgen.grid(50, 50, 1, 2, seed=2),
     "road": lambda: phastgen.road(60_000, seed=9),
+    "road_distance": lambda: phastgen.road(20_000, seed=9, metric="distance"),
     "rand_zero": lambda: phastgen.random_digraph(400, 1400, 0, 4, seed=3),
     "grid_zero": lambda: phastgen.grid(40, 30, 0, 4, seed=6),
     "rand_sat": lambda: phastgen.random_digraph(800, 4000, 1 << 30, 0xFFFFFFFF, seed=4),
@@ -110,6 +111,15 @@ def test_every_layout_sweep_equals_oracle(layout):
     h = P.Phast.from_graph(g, host_only=True, delta=5000, **LAYOUTS[layout])
     src = phastgen.sources(g.n, 5, seed=3)
     assert np.array_equal(chref.phast_cpu(h, h.export(), src), oracle.sssp_many(g, src))
+
+
+def test_distance_metric_is_deeper():
+    """NEXT-4 generator variant: the travel-distance metric (all road classes speed
+    1) yields a deeper hierarchy than travel times on the same lattice, as in the
+    paper (§VIII-G: 410 vs 140 levels on Europe)."""
+    lv = {m: P.Phast.from_graph(phastgen.road(20_000, seed=9, metric=m), host_only=True).levels
+          for m in ("time", "distance")}
+    assert lv["distance"] > 1.5 * lv["time"], lv
 
 
 def test_shortcut_lengths_dominate_distances():

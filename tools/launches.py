@@ -25,6 +25,8 @@ def load(path):
 def main(path, verbose=False):
     L = load(path)
     starts = [j for j, x in enumerate(L) if 'upward' in x['name']]
+    if not starts:   # fused single-launch queries: one launch per step
+        starts = [j for j, x in enumerate(L) if 'sweep_top' in x['name']]
     starts.append(len(L))
     for a, b in zip(starts[:-1], starts[1:]):
         grp = L[a:b]
