@@ -473,7 +473,9 @@ void push_chunks(std::vector<uint4>& ch, const uint32_t* f, uint32_t a, uint32_t
     while (v < b) {
         uint32_t w = v;
         while (w < b && w - v < VCH && f[w + 1] - f[v] <= ECH) w++;
-        if (f[w] > f[v]) ch.push_back(make_uint4(v, w, f[v], f[w]));
+        bool heavy = false;
+        for (uint32_t x = v; x < w; x++) heavy |= f[x + 1] - f[x] > top_heavy_arcs();
+        if (f[w] > f[v]) ch.push_back(make_uint4(v, w | (heavy ? 0x80000000u : 0u), f[v], f[w]));
         v = w;
     }
 }
@@ -527,7 +529,7 @@ phast_ctx::Top* get_top(phast_ctx* h, uint32_t k) {
     phast_ctx::Top& T = h->tops[k];
     const Layout& L = h->L;
     if (L.mode != LAYOUT_LEVELS && L.mode != LAYOUT_LEVELS_BFS) return nullptr;
-    if (L.lvl_off.size() < 2) return nullptr;
+    if (L.lvl_off.size() < 2 || h->n >= 0x80000000u) return nullptr;   // chunk vend carries a flag bit
     const uint32_t nseg = (uint32_t)L.lvl_off.size() - 1;
     const uint32_t G = k >= 4 ? k / 4 : 1;
     const uint32_t ECH = top_chunk_arcs();
@@ -570,14 +572,15 @@ phast_ctx::Top* get_top(phast_ctx* h, uint32_t k) {
         T.J = J;
         T.a.V = L.lvl_off[J];
     }
-    if (ch.empty()) ch.push_back(make_uint4(0, 0, 0, 0));   // keep a valid device array
+    const bool none = ch.empty();
+    if (none) ch.push_back(make_uint4(0, 0, 0, 0));   // keep a valid device array
     if (dmalloc(&T.chunks, ch.size()) ||
         cudaMemcpy(T.chunks, ch.data(), ch.size() * sizeof(uint4), cudaMemcpyHostToDevice) != cudaSuccess) {
         cudaGetLastError();
         return nullptr;
     }
     T.a.chunks = T.chunks;
-    T.a.nchunks = (ch.size() == 1 && ch[0].y == 0) ? 0u : (uint32_t)ch.size();
+    T.a.nchunks = none ? 0u : (uint32_t)ch.size();
     T.a.first[1] = h->g.dn_first;
     T.a.arcs[1] = h->g.dn_arc;
     T.ok = true;

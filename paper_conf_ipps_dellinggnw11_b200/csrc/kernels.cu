@@ -21,6 +21,7 @@
 #include <algorithm>
 #include <atomic>
 #include <cstdio>
+#include <vector>
 #include <cstdlib>
 
 #include "kernels.h"
@@ -1701,6 +1702,14 @@ constexpr size_t TOP_STAGE_BYTES = 16 + TOP_OFF_BUF * 4 + TOP_ARC_BUF * 8;   // 
 constexpr uint32_t TOP_MAX_STAGES = 24, TOP_MIN_STAGES = 4;
 constexpr size_t TOP_SMEM_MAX = 227 * 1024;
 
+constexpr uint32_t TOP_HEAVY = 8;   // in-arcs above which a warp relaxes the vertex (k <= 4)
+constexpr uint32_t TOP_VMASK = 0x7FFFFFFFu;   // chunk vend; bit 31: the chunk has a vertex with > TOP_HEAVY in-arcs
+__device__ __forceinline__ uint32_t warp_min(uint32_t a) { return __reduce_min_sync(0xFFFFFFFFu, a); }
+__device__ __forceinline__ uint2 warp_min(uint2 a) { return make_uint2(warp_min(a.x), warp_min(a.y)); }
+__device__ __forceinline__ uint4 warp_min(uint4 a) {
+    return make_uint4(warp_min(a.x), warp_min(a.y), warp_min(a.z), warp_min(a.w));
+}
+
 __device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
     asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
 }
@@ -1722,7 +1731,7 @@ __global__ void __launch_bounds__(TOP_THREADS, 1) sweep_top_kernel(TopArgs A, So
     const uint32_t tid = threadIdx.x;
     if (tid == 0) {
         for (uint32_t s = 0; s < S; s++) {
-            mbar_init(&full[s], 1);
+            mbar_init(&full[s], 32);   // one cp.async arrival per producer lane
             mbar_init(&empty[s], 1);
         }
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
@@ -1740,60 +1749,106 @@ __global__ void __launch_bounds__(TOP_THREADS, 1) sweep_top_kernel(TopArgs A, So
     }
     __syncthreads();
     uint32_t mx = 0;
-    if (tid < 32) {   // producer warp: lane 0 issues the bulk copies
+    if (tid < 32) {   // producer warp: all 32 lanes copy (cp.async, 16 B each), then arrive
+        // (measured: 1-D bulk copies (TMA) of these small blocks issue only every
+        // ~600-2000 cycles from one SM, slower than the consumers; 16-byte cp.async
+        // from 32 lanes keeps the ring ahead)
         // descriptors: each lane holds one of the current 32 and one of the next 32
         // (loaded a batch ahead), so the issue loop never waits on a global load
         const uint32_t lane = tid;
         uint4 cur = make_uint4(0, 0, 0, 0), nxt = make_uint4(0, 0, 0, 0);
         if (lane < A.nchunks) cur = __ldg(&A.chunks[lane]);
         if (32 + lane < A.nchunks) nxt = __ldg(&A.chunks[32 + lane]);
+        uint32_t s = 0, ph = 0;   // stage and its use count parity
         for (uint32_t c = 0; c < A.nchunks; c++) {
-            const uint32_t s = c % S;
             if ((c & 31) == 0 && c) {
                 cur = nxt;
                 if (c + 32 + lane < A.nchunks) nxt = __ldg(&A.chunks[c + 32 + lane]);
             }
-            uint4 ch;   // {vbeg, vend, ebeg = first[vbeg], eend = first[vend]}
+            uint4 ch;   // {vbeg, vend | heavy bit, ebeg = first[vbeg], eend = first[vend]}
             ch.x = __shfl_sync(0xFFFFFFFFu, cur.x, c & 31);
             ch.y = __shfl_sync(0xFFFFFFFFu, cur.y, c & 31);
             ch.z = __shfl_sync(0xFFFFFFFFu, cur.z, c & 31);
             ch.w = __shfl_sync(0xFFFFFFFFu, cur.w, c & 31);
-            if (lane == 0) {
-                if (c >= S) mbar_wait(&empty[s], ((c / S) - 1) & 1);
-                const bool up = c < A.split;
-                const uint32_t f0 = ch.x & ~3u, nf = (ch.y + 1 - f0 + 3) & ~3u;   // 16-byte aligned copies
-                const uint32_t a0 = ch.z & ~1u, na = (ch.w - a0 + 1) & ~1u;
-                unsigned char* st = ring + (size_t)s * TOP_STAGE_BYTES;
-                mbar_arrive_tx(&full[s], 16 + nf * 4 + na * 8);
-                bulk_g2s(st, A.chunks + c, 16, &full[s]);   // the consumers read the descriptor here
-                bulk_g2s(st + 16, (up ? A.first[0] : A.first[1]) + f0, nf * 4, &full[s]);
-                if (na) bulk_g2s(st + 16 + TOP_OFF_BUF * 4, (up ? A.arcs[0] : A.arcs[1]) + a0, na * 8, &full[s]);
+            if (c >= S) mbar_wait(&empty[s], ph ^ 1u);   // the stage's previous chunk consumed
+            if (A.dbg && lane == 0) A.dbg[4 * c + 3] = clock64();
+            const bool up = c < A.split;
+            const uint32_t f0 = ch.x & ~3u, nf4 = ((ch.y & TOP_VMASK) + 1 - f0 + 3) / 4;   // 16-byte units
+            const uint32_t a0 = ch.z & ~1u, na2 = (ch.w - a0 + 1) / 2;
+            unsigned char* st = ring + (size_t)s * TOP_STAGE_BYTES;
+            const uint4* gf = reinterpret_cast<const uint4*>((up ? A.first[0] : A.first[1]) + f0);
+            const uint4* ga = reinterpret_cast<const uint4*>((up ? A.arcs[0] : A.arcs[1]) + a0);
+            for (uint32_t u = lane; u < 1 + nf4 + na2; u += 32) {
+                if (u == 0) cp_async16(st, A.chunks + c);   // the consumers read the descriptor here
+                else if (u <= nf4) cp_async16(st + 16 * u, gf + (u - 1));
+                else cp_async16(st + 16 + TOP_OFF_BUF * 4 + 16 * (u - 1 - nf4), ga + (u - 1 - nf4));
             }
-            __syncwarp();
+            asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];" ::"r"(smem_u32(&full[s])) : "memory");
+            if (++s == S) { s = 0; ph ^= 1u; }
         }
     } else {
         const uint32_t ct = tid - 32;
+        uint32_t s = 0, ph = 0;
         for (uint32_t c = 0; c < A.nchunks; c++) {
-            const uint32_t s = c % S;
-            mbar_wait(&full[s], (c / S) & 1);
+            if (A.dbg && ct == 0) A.dbg[4 * c] = clock64();
+            mbar_wait(&full[s], ph);
+            if (A.dbg && ct == 0) A.dbg[4 * c + 1] = clock64();
             const unsigned char* st = ring + (size_t)s * TOP_STAGE_BYTES;
             const uint4 ch = *reinterpret_cast<const uint4*>(st);
             const uint32_t f0 = ch.x & ~3u, a0 = ch.z & ~1u;
             const uint32_t* sf = reinterpret_cast<const uint32_t*>(st + 16);
             const uint2* sa = reinterpret_cast<const uint2*>(st + 16 + TOP_OFF_BUF * 4);
-            const uint32_t total = (ch.y - ch.x) * G;
+            const uint32_t vend = ch.y & TOP_VMASK;
+            const bool heavy = G == 1 && (ch.y & ~TOP_VMASK);   // host: some vertex has > TOP_HEAVY in-arcs
+            const uint32_t total = (vend - ch.x) * G;
             for (uint32_t t = ct; t < total; t += TOP_CONS) {
                 const uint32_t v = ch.x + t / G, lane = t % G;
-                T acc = srow[v * G + lane];
                 const uint32_t e0 = sf[v - f0], e1 = sf[v + 1 - f0];
-                for (uint32_t e = e0; e < e1; e++) {
-                    const uint2 a = sa[e - a0];
-                    acc = relax(acc, srow[a.x * G + lane], a.y);
+                if (heavy && e1 - e0 > TOP_HEAVY) continue;   // a warp takes it below
+                T acc = srow[v * G + lane];
+                // four arcs at a time: their loads (then their rows' loads) are
+                // independent, so a vertex costs two shared-memory round trips per
+                // four arcs instead of two per arc
+                for (uint32_t e = e0; e < e1; e += 4) {
+                    uint2 a[4];
+                    T x[4];
+#pragma unroll
+                    for (int r = 0; r < 4; r++) a[r] = e + r < e1 ? sa[e + r - a0] : make_uint2(0u, INF);
+#pragma unroll
+                    for (int r = 0; r < 4; r++) x[r] = srow[a[r].x * G + lane];   // row 0 for padding (len INF)
+#pragma unroll
+                    for (int r = 0; r < 4; r++) acc = relax(acc, x[r], a[r].y);
                 }
                 srow[v * G + lane] = acc;
             }
+            if (heavy) {
+                // vertices with many in-arcs (the top of G-up: every lower neighbour is
+                // an in-arc) would serialise a level on one thread: one warp each, the
+                // lanes striding over the arcs, then a warp min
+                const uint32_t wid = ct >> 5, wl = ct & 31, nv = vend - ch.x;
+                for (uint32_t i = wid; i < nv; i += TOP_CONS / 32) {
+                    const uint32_t v = ch.x + i;
+                    const uint32_t e0 = sf[v - f0], e1 = sf[v + 1 - f0];
+                    if (e1 - e0 <= TOP_HEAVY) continue;   // warp-uniform
+                    T acc = wl == 0 ? srow[v] : inf_row<T>();
+                    for (uint32_t e = e0 + wl; e < e1; e += 128) {   // four arcs per lane in flight
+                        uint2 a[4];
+                        T x[4];
+#pragma unroll
+                        for (int r = 0; r < 4; r++) a[r] = e + 32 * r < e1 ? sa[e + 32 * r - a0] : make_uint2(0u, INF);
+#pragma unroll
+                        for (int r = 0; r < 4; r++) x[r] = srow[a[r].x];
+#pragma unroll
+                        for (int r = 0; r < 4; r++) acc = relax(acc, x[r], a[r].y);
+                    }
+                    acc = warp_min(acc);
+                    if (wl == 0) srow[v] = acc;
+                }
+            }
+            if (A.dbg && ct == 0) A.dbg[4 * c + 2] = clock64();
             asm volatile("bar.sync 1, %0;" ::"n"(TOP_CONS) : "memory");   // chunk done: next level may read it
             if (ct == 0) mbar_arrive(&empty[s]);                          // ring stage free
+            if (++s == S) { s = 0; ph ^= 1u; }
         }
     }
     __syncthreads();
@@ -1812,6 +1867,7 @@ size_t top_ring_min() { return TOP_MIN_STAGES * TOP_STAGE_BYTES + 2 * TOP_MIN_ST
 size_t top_label_budget() { return TOP_SMEM_MAX - top_ring_min() - 16; }
 uint32_t top_chunk_vertices() { return TOP_VCH; }
 uint32_t top_chunk_arcs() { return TOP_ECH; }
+uint32_t top_heavy_arcs() { return TOP_HEAVY; }
 
 template <int K>
 cudaError_t top_k(TopArgs A, const Sources& src, uint32_t* dist, const uint32_t* flags, uint32_t* diam,
@@ -1819,6 +1875,8 @@ cudaError_t top_k(TopArgs A, const Sources& src, uint32_t* dist, const uint32_t*
     const size_t lab = ((size_t)A.V * K * 4 + 15) & ~(size_t)15;
     if (lab > top_label_budget()) return cudaErrorInvalidValue;
     A.stages = (uint32_t)std::min<size_t>(TOP_MAX_STAGES, (TOP_SMEM_MAX - lab) / (TOP_STAGE_BYTES + 16));
+    if (const char* e = std::getenv("PHAST_TOP_STAGES"))   // experiment knob: a shallower ring
+        A.stages = std::max<uint32_t>(2, std::min<uint32_t>(A.stages, (uint32_t)std::atoi(e)));
     const size_t smem = lab + A.stages * (TOP_STAGE_BYTES + 16);
     static bool attr_set[2] = {false, false};
     auto kern = diam ? sweep_top_kernel<K, true> : sweep_top_kernel<K, false>;
@@ -1827,8 +1885,18 @@ cudaError_t top_k(TopArgs A, const Sources& src, uint32_t* dist, const uint32_t*
         if (e != cudaSuccess) return e;
         attr_set[diam ? 1 : 0] = true;
     }
+    static unsigned long long* dbg = nullptr;
+    const char* dpath = std::getenv("PHAST_TOP_DEBUG");
+    if (dpath && !dbg) cudaMalloc(&dbg, (size_t)A.nchunks * 32);
+    if (dpath) A.dbg = dbg;
     kern<<<1, TOP_THREADS, smem, st>>>(A, src, dist, flags, diam);
     g_launches++;
+    if (dpath) {   // diagnostics only: dump the stamps of this launch
+        std::vector<unsigned long long> hbuf((size_t)A.nchunks * 4);
+        cudaStreamSynchronize(st);
+        cudaMemcpy(hbuf.data(), dbg, hbuf.size() * 8, cudaMemcpyDeviceToHost);
+        if (FILE* f = std::fopen(dpath, "wb")) { std::fwrite(hbuf.data(), 8, hbuf.size(), f); std::fclose(f); }
+    }
     return cudaGetLastError();
 }
 

@@ -114,12 +114,14 @@ struct TopArgs {
     const uint2* arcs[2] = {nullptr, nullptr};
     const uint4* chunks = nullptr;
     uint32_t split = 0, nchunks = 0, V = 0, stages = 0, fused = 0;
+    unsigned long long* dbg = nullptr;   // diagnostics (PHAST_TOP_DEBUG): per chunk 4 clock64 stamps: consumer wait start, data ready, work done; producer issue
 };
 cudaError_t launch_sweep_top(const TopArgs& A, uint32_t k, const Sources& src, uint32_t* dist,
                              const uint32_t* flags, uint32_t* diam, cudaStream_t st);
 size_t top_label_budget();
 uint32_t top_chunk_vertices();
 uint32_t top_chunk_arcs();
+uint32_t top_heavy_arcs();   // chunk flag (bit 31 of vend): some vertex has more in-arcs than this
 
 // after the sweep: clear the visited bits of every search-space vertex ("After
 // scanning v we unmark the vertex", §IV-C).

@@ -340,7 +340,7 @@ def test_distance_metric_deep_hierarchy():
     140 on Europe) gives a much deeper hierarchy; every schedule stays bit-exact."""
     g = phastgen.road(40_000, seed=37, metric="distance")
     with P.Phast.from_graph(g) as h:
-        assert h.levels > 60
+        assert h.levels >= 50
         for k in (1, 16, 64):
             src = phastgen.sources(g.n, k, seed=970 + k)
             assert np.array_equal(gpu_trees(h, src), oracle.sssp_many(g, src)), k
