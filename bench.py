@@ -268,9 +268,11 @@ def main():
     try:
         prof = json.load(open(os.path.join(ROOT, "profiles", "sweep_traffic.json")))
         key = f"{args.config}_k{k}"
-        if key in prof and prof[key].get("layout") == P.LAYOUT_NAMES[info.layout] and \
-                os.environ.get("PHAST_SWEEP", "levels") == prof[key].get("sweep"):
-            traffic = prof[key]["dram_bytes_per_sweep"]   # ncu launch list of this configuration
+        e = prof.get(key, {})
+        default_path = not any(os.environ.get(v) for v in ("PHAST_SWEEP", "PHAST_ARC_BATCH", "PHAST_TOP",
+                                                            "PHAST_FUSED", "PHAST_TOP_MAXV"))
+        if e.get("layout") == P.LAYOUT_NAMES[info.layout] and default_path and e.get("arc_batch") == "ell":
+            traffic = e["dram_bytes_per_sweep"]   # ncu launch list of this configuration (warm L2)
     except Exception:
         pass
 
@@ -339,7 +341,7 @@ def main():
                        "us_per_tree": ms * 1e3 / (args.steps * k),
                        "ch_build_s": round(info.build_seconds, 1)},
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
-                         "traffic": traffic, "kernel": "sweep_kernel (all levels of one sweep)",
+                         "traffic": traffic, "kernel": "sweep_top_kernel + sweep_kernel (all levels of one sweep)",
                          "alg_bytes_per_sweep": B_alg, "sweep_ms": sweep_ms, "upward_ms": ms_up / max(nb, 1),
                          "peak_source": peak_src},
             "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": launches, "clocks": clk.summary(),

@@ -50,7 +50,12 @@ struct phast_ctx {
     struct Top {
         uint4* chunks = nullptr;   // device [nchunks] {vbeg, vend, first[vbeg], first[vend]}
         TopArgs a;                 // a.fused: the whole query in this one launch
-        uint32_t J = 0;            // segments [0, J) covered
+        uint32_t J = 0;            // segments [0, J) in the shared-memory launch (0: none)
+        uint32_t J2 = 0;           // segments [J, J2) in one cluster launch (launch_sweep_cluster)
+        uint32_t* cl_seg = nullptr;   // device [J2 - J + 1] offsets
+        uint32_t vtop = 0;            // upward searches stop expanding below this id (0: full searches)
+        uint32_t* up_f = nullptr;     // top mode with vtop: A-up in-arcs by head inside [0, V)
+        uint2* up_a = nullptr;
         bool ok = false;
     };
     std::map<uint32_t, Top> tops;
@@ -116,7 +121,10 @@ void free_plans(phast_ctx* h) {
         cudaFree(kv.second.p.done);
     }
     h->plans.clear();
-    for (auto& kv : h->tops) cudaFree(kv.second.chunks);
+    for (auto& kv : h->tops) {
+        cudaFree(kv.second.chunks); cudaFree(kv.second.cl_seg);
+        cudaFree(kv.second.up_f); cudaFree(kv.second.up_a);
+    }
     h->tops.clear();
 }
 
@@ -550,11 +558,10 @@ phast_ctx::Top* get_top(phast_ctx* h, uint32_t k) {
         T.a.first[0] = h->d_upin_first;
         T.a.arcs[0] = h->d_upin_arc;
         T.a.fused = 1;
-        T.J = nseg;
+        T.J = T.J2 = nseg;
         T.a.V = h->n;
     } else {
-        const char* env = std::getenv("PHAST_TOP");
-        if (env && std::atoi(env) == 0) return nullptr;
+        const char* env = std::getenv("PHAST_TOP");   // PHAST_TOP=0: no shared-memory top launch
         uint64_t vmax = vmax_budget;
         if (const char* e = std::getenv("PHAST_TOP_MAXV")) vmax = std::min<uint64_t>(vmax, (uint64_t)std::atoll(e));
         uint32_t J = 0;
@@ -566,11 +573,62 @@ phast_ctx::Top* get_top(phast_ctx* h, uint32_t k) {
             if (!fits) break;
             J++;
         }
-        if (J < 2) return nullptr;
+        if (J < 2 || (env && std::atoi(env) == 0)) J = 0;
+        // hybrid upward search (PHAST_UP_HYBRID=0 disables): the upward kernel expands
+        // only vertices below the top levels; the top kernel finishes G-up inside
+        // [0, V) with a pull pass in ascending level order (reading R9), then sweeps
+        // G-down.  Exact: a G-up path only climbs, so it enters [0, V) once and its part
+        // below V is found by the search, its part inside by the pull pass.
+        const char* he = std::getenv("PHAST_UP_HYBRID");
+        const uint32_t V = L.lvl_off[J];
+        if (J && !(he && std::atoi(he) == 0)) {
+            std::vector<uint32_t> f((size_t)V + 1, 0);
+            for (uint32_t u = 0; u < V; u++)
+                for (uint32_t e = L.up_first[u]; e < L.up_first[u + 1]; e++) f[L.up_arc[e].x + 1]++;
+            for (uint32_t v = 0; v < V; v++) f[v + 1] += f[v];
+            std::vector<Arc> arc(f[V]);
+            std::vector<uint32_t> pos(f.begin(), f.end() - 1);
+            for (uint32_t u = 0; u < V; u++)
+                for (uint32_t e = L.up_first[u]; e < L.up_first[u + 1]; e++)
+                    arc[pos[L.up_arc[e].x]++] = Arc{u, L.up_arc[e].y};
+            bool fits = true;
+            for (uint32_t v = 0; v < V && fits; v++) fits = f[v + 1] - f[v] <= ECH;
+            if (fits && !dmalloc(&T.up_f, f.size() + 4) && !dmalloc(&T.up_a, arc.size() + 2) &&
+                cudaMemset(T.up_f, 0, (f.size() + 4) * 4) == cudaSuccess &&
+                cudaMemset(T.up_a, 0, (arc.size() + 2) * 8) == cudaSuccess &&
+                cudaMemcpy(T.up_f, f.data(), f.size() * 4, cudaMemcpyHostToDevice) == cudaSuccess &&
+                (arc.empty() || cudaMemcpy(T.up_a, arc.data(), arc.size() * 8, cudaMemcpyHostToDevice) == cudaSuccess)) {
+                for (uint32_t j = J; j-- > 0;) push_chunks(ch, f.data(), L.lvl_off[j], L.lvl_off[j + 1]);
+                T.a.first[0] = T.up_f;
+                T.a.arcs[0] = T.up_a;
+                T.vtop = V;
+            } else {
+                cudaGetLastError();
+            }
+        }
+        T.a.split = (uint32_t)ch.size();
         for (uint32_t j = 0; j < J; j++) push_chunks(ch, L.dn_first.data(), L.lvl_off[j], L.lvl_off[j + 1]);
-        T.a.split = 0;
         T.J = J;
-        T.a.V = L.lvl_off[J];
+        T.a.V = V;
+        // the next levels, while small, in one cluster launch (PHAST_CL_SIZE=0 disables;
+        // PHAST_CL_PASSES: max grid-stride passes of the cluster per level, default 8)
+        uint32_t J2 = J;
+        const uint64_t CT = cluster_threads();
+        uint64_t passes = 8;
+        if (const char* e = std::getenv("PHAST_CL_PASSES")) passes = (uint64_t)std::max(1, std::atoi(e));
+        if (CT && h->g.dn_rec)
+            while (J2 + 1 < nseg && (uint64_t)(L.lvl_off[J2 + 1] - L.lvl_off[J2]) * G <= CT * passes) J2++;
+        if (J2 - J < 2) J2 = J;   // not worth a launch
+        if (J == 0 && J2 == 0) return nullptr;
+        if (J2 > J) {
+            if (dmalloc(&T.cl_seg, J2 - J + 1) ||
+                cudaMemcpy(T.cl_seg, L.lvl_off.data() + J, (size_t)(J2 - J + 1) * 4, cudaMemcpyHostToDevice) !=
+                    cudaSuccess) {
+                cudaGetLastError();
+                return nullptr;
+            }
+        }
+        T.J2 = J2;
     }
     const bool none = ch.empty();
     if (none) ch.push_back(make_uint4(0, 0, 0, 0));   // keep a valid device array
@@ -585,8 +643,8 @@ phast_ctx::Top* get_top(phast_ctx* h, uint32_t k) {
     T.a.arcs[1] = h->g.dn_arc;
     T.ok = true;
     if (std::getenv("PHAST_VERBOSE"))
-        std::fprintf(stderr, "%s plan k=%u: %u levels, %u vertices, %u chunks (%u up)\n",
-                     T.a.fused ? "fused" : "top", k, T.J, T.a.V, T.a.nchunks, T.a.split);
+        std::fprintf(stderr, "%s plan k=%u: %u levels, %u vertices, %u chunks (%u up); cluster levels [%u, %u)\n",
+                     T.a.fused ? "fused" : "top", k, T.J, T.a.V, T.a.nchunks, T.a.split, T.J, T.J2);
     return &T;
 }
 
@@ -622,12 +680,15 @@ int run_query(phast_ctx* h, const Sources& S, uint32_t k, uint32_t* dist, uint32
     const uint32_t slot = h->slot_next;
     h->slot_next = (h->slot_next + 1) % SEED_SLOTS;
     if (cudaStreamWaitEvent(h->side, h->slot_free[slot], 0) != cudaSuccess) return PHAST_ECUDA;
-    if (launch_upward(h->g, S, k, slot, h->side) != cudaSuccess) return PHAST_ECUDA;
+    phast_ctx::Plan* plan = get_plan(h, k);
+    // the top / cluster launches run only on the per-level path (no persistent plan)
+    if (plan || h->L.mode == LAYOUT_DIAGONAL || h->L.lvl_off.empty()) top = nullptr;
+    const uint32_t vtop = (top && top->J) ? top->vtop : 0u;
+    if (launch_upward(h->g, S, k, slot, vtop, h->side) != cudaSuccess) return PHAST_ECUDA;
     if (cudaEventRecord(h->up_done[slot], h->side) != cudaSuccess) return PHAST_ECUDA;
     if (cudaStreamWaitEvent(st, h->up_done[slot], 0) != cudaSuccess) return PHAST_ECUDA;
     if (launch_seed(h->g, k, slot, dist, st) != cudaSuccess) return PHAST_ECUDA;
     if (e1) cudaEventRecord(e1, st);
-    phast_ctx::Plan* plan = get_plan(h, k);
     if (plan && plan->bottom_from) {   // top levels one launch each, then the bottom diagonals in one launch
         for (uint32_t j = 0; j < plan->bottom_from; j++)
             if (launch_sweep_level(h->g, k, h->L.lvl_off[j], h->L.lvl_off[j + 1], dist, diam, true, false, false,
@@ -657,10 +718,13 @@ int run_query(phast_ctx* h, const Sources& S, uint32_t k, uint32_t* dist, uint32
         const uint32_t levels = (uint32_t)h->L.lvl_off.size() - 1;   // segments
         const bool diagonal = h->L.mode == LAYOUT_DIAGONAL;
         uint32_t j0 = 0;
-        if (plan || diagonal) top = nullptr;
-        if (top) {                            // the small top levels in one single-CTA launch
-            if (launch_sweep_top(top->a, k, S, dist, h->g.flags, diam, st) != cudaSuccess) return PHAST_ECUDA;
-            j0 = top->J;
+        if (top) {                            // the small top levels in one single-CTA launch,
+            if (top->J && launch_sweep_top(top->a, k, S, dist, h->g.flags, diam, st) != cudaSuccess)
+                return PHAST_ECUDA;
+            if (top->J2 > top->J &&           // the next small ones in one cluster launch
+                launch_sweep_cluster(h->g, k, top->cl_seg, top->J2 - top->J, dist, diam, st) != cudaSuccess)
+                return PHAST_ECUDA;
+            j0 = top->J2;
         } else if (plan) {                    // hybrid: small top levels in one persistent launch
             if ((uint64_t)(plan->epoch + 1) * plan->p.grid >= 0x7FFFFFFFull) {
                 if (cudaMemsetAsync(plan->p.wave_done, 0, (size_t)plan->p.iters * 4, st) != cudaSuccess)

@@ -92,15 +92,17 @@ __device__ __forceinline__ uint32_t up_insert(const UpTable& t, uint32_t w, UpSh
 // Label-correcting relaxation of G-up from s, wave-synchronous; on return the
 // table holds exact G-up distances of every vertex reachable from s (Bellman-Ford
 // fixed point with saturating sums).  Returns false on table overflow.
+// vtop > 0: vertices < vtop (the top levels, swept by sweep_top_kernel's G-up pull
+// pass) get their labels from the arcs entering them but are not expanded.
 __device__ bool up_search(const uint32_t* __restrict__ up_first, const uint2* __restrict__ up_arc,
-                          uint32_t s, UpTable t, UpShared& c) {
+                          uint32_t s, UpTable t, UpShared& c, uint32_t vtop) {
     const uint32_t tid = threadIdx.x;
     for (uint32_t i = tid; i < t.cap; i += blockDim.x) { t.keys[i] = EMPTY; t.vals[i] = INF; t.inq[i] = 0; }
     __syncthreads();
     if (tid == 0) {
         uint32_t h = hash32(s) & (t.cap - 1);
         t.keys[h] = s; t.vals[h] = 0; t.inq[h] = 1; t.qa[0] = h;
-        c.qn = 1; c.nn = 0; c.used = 1; c.over = 0; c.cnt = 0;
+        c.qn = s >= vtop ? 1u : 0u; c.nn = 0; c.used = 1; c.over = 0; c.cnt = 0;
     }
     __syncthreads();
     uint32_t* qa = t.qa;
@@ -122,7 +124,7 @@ __device__ bool up_search(const uint32_t* __restrict__ up_first, const uint2* __
                 uint32_t ws = up_insert(t, a.x, c);
                 if (ws == EMPTY) { c.over = 1; break; }
                 uint32_t old = atomicMin(&t.vals[ws], nd);
-                if (nd < old) {
+                if (nd < old && a.x >= vtop) {
                     __threadfence_block();
                     if (atomicExch(&t.inq[ws], 1u) == 0u) qb[atomicAdd(&c.nn, 1u)] = ws;
                 }
@@ -141,7 +143,7 @@ __device__ bool up_search(const uint32_t* __restrict__ up_first, const uint2* __
 // a1: search only; the search space goes to seed slot `slot` (the sweep of the
 // previous batch may still be running on the main stream: nothing here touches the
 // visited bits or the label rows).
-__global__ void __launch_bounds__(UP_THREADS) upward_kernel(DevImage g, Sources src, uint32_t slot) {
+__global__ void __launch_bounds__(UP_THREADS) upward_kernel(DevImage g, Sources src, uint32_t slot, uint32_t vtop) {
     extern __shared__ uint32_t smem[];
     __shared__ UpShared c;
     const uint32_t i = blockIdx.x;
@@ -149,13 +151,13 @@ __global__ void __launch_bounds__(UP_THREADS) upward_kernel(DevImage g, Sources 
     const uint32_t sc = g.smem_cap;
     const size_t so = ((size_t)slot * KMAX + i) * g.seed_cap;
     UpTable t{smem, smem + sc, smem + 2 * sc, smem + 3 * sc, smem + 4 * sc, sc};
-    bool ok = up_search(g.up_first, g.up_arc, s, t, c);
+    bool ok = up_search(g.up_first, g.up_arc, s, t, c, vtop);
     if (!ok) {   // global-memory fallback with the per-source capacity
         uint32_t* base = g.gscratch + (size_t)i * g.seed_cap * 5;
         UpTable gt{base, base + g.seed_cap, base + 2 * (size_t)g.seed_cap, base + 3 * (size_t)g.seed_cap,
                    base + 4 * (size_t)g.seed_cap, g.seed_cap};
         t = gt;
-        ok = up_search(g.up_first, g.up_arc, s, t, c);
+        ok = up_search(g.up_first, g.up_arc, s, t, c, vtop);
         if (!ok) {
             if (threadIdx.x == 0) { atomicOr(g.err, 1u); g.seed_cnt[slot * KMAX + i] = 0; }
             return;
@@ -1630,7 +1632,8 @@ cudaError_t persistent_k(const DevImage& g, const SweepPlan& p, uint32_t epoch, 
                           : persistent_k2<K, false>(g, p, epoch, dist, diam, st);
 }
 
-cudaError_t upward_launch(const DevImage& g, const Sources& src, uint32_t k, uint32_t slot, cudaStream_t st) {
+cudaError_t upward_launch(const DevImage& g, const Sources& src, uint32_t k, uint32_t slot, uint32_t vtop,
+                          cudaStream_t st) {
     static bool attr = false;
     size_t smem = 5 * (size_t)g.smem_cap * sizeof(uint32_t);
     if (!attr) {
@@ -1639,7 +1642,7 @@ cudaError_t upward_launch(const DevImage& g, const Sources& src, uint32_t k, uin
         if (e != cudaSuccess) return e;
         attr = true;
     }
-    upward_kernel<<<k, UP_THREADS, smem, st>>>(g, src, slot);
+    upward_kernel<<<k, UP_THREADS, smem, st>>>(g, src, slot, vtop);
     g_launches++;
     return cudaGetLastError();
 }
@@ -1900,6 +1903,122 @@ cudaError_t top_k(TopArgs A, const Sources& src, uint32_t* dist, const uint32_t*
     return cudaGetLastError();
 }
 
+// ------------------------------------------------------------------ a3 + a4: mid levels in one cluster
+// After the shared-memory top levels come levels of a few thousand vertices: too big
+// for one SM, too small to amortise a launch (~4-5 us each with programmatic
+// dependent launch).  They run in ONE launch of a thread-block cluster (C CTAs of
+// 1 024 threads on C SMs): each level is a grid-stride pass over (vertex, 16-byte
+// lane) items exactly like sweep_kernel's ELL path, and the level boundary
+// (§VI: a kernel boundary in the paper) is a hardware cluster barrier
+// with release/acquire semantics (barrier.cluster.arrive.release / wait.acquire),
+// which orders the rows written by every CTA of the cluster before the next level
+// reads them (Lemma 4.1: tails are in earlier levels).  Tail rows are read with
+// ld.global.cg (L2): another SM wrote them in this launch.  The next level's first
+// record is prefetched into L2 before the barrier (static data).
+constexpr int CL_THREADS = 1024;
+
+__device__ __forceinline__ void cluster_sync_acqrel() {
+    asm volatile("barrier.cluster.arrive.release.aligned;\nbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+}
+
+template <int K, bool DIAM>
+__global__ void __launch_bounds__(CL_THREADS, 1) sweep_cluster_kernel(const uint4* __restrict__ rec,
+                                                                      const uint2* __restrict__ ovf,
+                                                                      uint32_t* __restrict__ d,
+                                                                      const uint32_t* __restrict__ flags,
+                                                                      const uint32_t* __restrict__ seg,
+                                                                      uint32_t nseg, uint32_t* __restrict__ diam) {
+    using T = typename RowT<K>::T;
+    constexpr uint32_t G = K / RowT<K>::W;   // lanes per vertex
+    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+    const uint32_t stride = gridDim.x * CL_THREADS;
+    const uint32_t t0 = blockIdx.x * CL_THREADS + threadIdx.x;
+    if (t0 < (__ldg(&seg[1]) - __ldg(&seg[0])) * G) asm volatile("prefetch.global.L2 [%0];" ::"l"(rec + __ldg(&seg[0]) + t0 / G));
+    asm volatile("griddepcontrol.wait;" ::: "memory");   // the previous launch (top levels) complete
+    uint32_t mx = 0;
+    uint32_t vb = __ldg(&seg[0]);
+    for (uint32_t j = 0; j < nseg; j++) {
+        const uint32_t ve = __ldg(&seg[j + 1]);
+        const uint32_t total = (ve - vb) * G;
+        for (uint32_t t = t0; t < total; t += stride) {
+            const uint32_t v = vb + t / G, lane = t % G;
+            T acc = inf_row<T>();
+            if ((__ldg(&flags[v >> 5]) >> (v & 31)) & 1u)   // visited by an upward search
+                acc = __ldcg(reinterpret_cast<const T*>(d + (size_t)v * K) + lane);
+            const uint4 r = __ldg(&rec[v]);
+            T x0 = inf_row<T>(), x1 = inf_row<T>();
+            if (r.y != INF) x0 = __ldcg(reinterpret_cast<const T*>(d + (size_t)r.x * K) + lane);
+            if (r.w != INF) x1 = __ldcg(reinterpret_cast<const T*>(d + (size_t)r.z * K) + lane);
+            acc = relax(relax(acc, x0, r.y), x1, r.w);
+            if (r.w == INF && r.z != INF) {   // more than two in-arcs
+                const uint2* o = ovf + r.z;
+                const uint32_t cnt = __ldg(&o->x);
+                for (uint32_t i = 1; i <= cnt; i++) {
+                    const uint2 a = __ldg(&o[i]);
+                    acc = relax(acc, __ldcg(reinterpret_cast<const T*>(d + (size_t)a.x * K) + lane), a.y);
+                }
+            }
+            reinterpret_cast<T*>(d + (size_t)v * K)[lane] = acc;
+            if constexpr (DIAM) mx = max(mx, fmax_of(acc));
+        }
+        if (j + 1 < nseg) {
+            const uint32_t nb = __ldg(&seg[j + 2]);
+            if (t0 < (nb - ve) * G) asm volatile("prefetch.global.L2 [%0];" ::"l"(rec + ve + t0 / G));
+            cluster_sync_acqrel();   // level j final everywhere in the cluster
+        }
+        vb = ve;
+    }
+    if constexpr (DIAM) {
+        mx = __reduce_max_sync(0xFFFFFFFFu, mx);
+        if ((threadIdx.x & 31) == 0 && mx) atomicMax(diam, mx);
+    }
+}
+
+// PHAST_CL_SIZE: CTAs per cluster (16 non-portable, 8 portable); default 0 = off:
+// measured slower than per-level launches (C3 k=64 sweep 2.06-2.12 vs 2.03 ms; C2
+// k=16 0.160 vs 0.132 ms; C2D 0.357 vs 0.377 ms, r42): a level inside the cluster
+// costs about what a programmatic-dependent launch costs, on 16 SMs instead of 148.
+int cluster_size() {
+    const char* e = std::getenv("PHAST_CL_SIZE");
+    int c = e ? std::atoi(e) : 0;
+    return c <= 0 ? 0 : c > 16 ? 16 : c;
+}
+
+template <int K>
+cudaError_t cluster_k(const DevImage& g, const uint32_t* seg, uint32_t nseg, uint32_t* dist, uint32_t* diam,
+                      cudaStream_t st) {
+    const int C = cluster_size();
+    auto kern = diam ? sweep_cluster_kernel<K, true> : sweep_cluster_kernel<K, false>;
+    static bool attr_set[2] = {false, false};
+    if (!attr_set[diam ? 1 : 0]) {
+        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
+        if (e != cudaSuccess) return e;
+        attr_set[diam ? 1 : 0] = true;
+    }
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3((unsigned)C);
+    cfg.blockDim = dim3(CL_THREADS);
+    cfg.stream = st;
+    cudaLaunchAttribute attr[2];
+    attr[0].id = cudaLaunchAttributeClusterDimension;
+    attr[0].val.clusterDim.x = (unsigned)C;
+    attr[0].val.clusterDim.y = 1;
+    attr[0].val.clusterDim.z = 1;
+    attr[1].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[1].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 2;
+    cudaError_t e = cudaLaunchKernelEx(&cfg, kern, g.dn_rec, g.dn_ovf, dist, (const uint32_t*)g.flags, seg, nseg, diam);
+    if (e != cudaSuccess && C > 8) {   // a 16-CTA cluster may not fit this GPU's GPCs: portable size 8
+        cudaGetLastError();
+        cfg.gridDim = dim3(8u);
+        attr[0].val.clusterDim.x = 8u;
+        e = cudaLaunchKernelEx(&cfg, kern, g.dn_rec, g.dn_ovf, dist, (const uint32_t*)g.flags, seg, nseg, diam);
+    }
+    g_launches++;
+    return e;
+}
+
 #define PHAST_K_SWITCH(k, CALL)      \
     switch (k) {                     \
         case 1: return CALL(1);      \
@@ -1912,8 +2031,9 @@ cudaError_t top_k(TopArgs A, const Sources& src, uint32_t* dist, const uint32_t*
         default: return cudaErrorInvalidValue; \
     }
 
-cudaError_t launch_upward(const DevImage& g, const Sources& src, uint32_t k, uint32_t slot, cudaStream_t st) {
-    return upward_launch(g, src, k, slot, st);
+cudaError_t launch_upward(const DevImage& g, const Sources& src, uint32_t k, uint32_t slot, uint32_t vtop,
+                          cudaStream_t st) {
+    return upward_launch(g, src, k, slot, vtop, st);
 }
 
 cudaError_t launch_seed(const DevImage& g, uint32_t k, uint32_t slot, uint32_t* dist, cudaStream_t st) {
@@ -2021,6 +2141,14 @@ cudaError_t launch_sweep_top(const TopArgs& A, uint32_t k, const Sources& src, u
     PHAST_K_SWITCH(k, CALL_TOP)
 #undef CALL_TOP
 }
+
+cudaError_t launch_sweep_cluster(const DevImage& g, uint32_t k, const uint32_t* seg, uint32_t nseg, uint32_t* dist,
+                                 uint32_t* diam, cudaStream_t st) {
+#define CALL_CL(K) cluster_k<K>(g, seg, nseg, dist, diam, st)
+    PHAST_K_SWITCH(k, CALL_CL)
+#undef CALL_CL
+}
+uint32_t cluster_threads() { return cluster_size() > 0 ? (uint32_t)cluster_size() * CL_THREADS : 0u; }
 
 cudaError_t launch_clear_flags(const DevImage& g, uint32_t k, uint32_t slot, cudaStream_t st) {
     clear_flags_kernel<<<k, 256, 0, st>>>(g, slot);

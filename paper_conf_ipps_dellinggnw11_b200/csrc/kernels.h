@@ -39,7 +39,10 @@ struct Sources {
 
 // a1: one CTA per source; exact G-up labels; the search space goes to seed slot `slot`
 // (SEED_SLOTS slots, so the next batch's searches can run beside this batch's sweep).
-cudaError_t launch_upward(const DevImage& g, const Sources& src, uint32_t k, uint32_t slot, cudaStream_t st);
+// vtop > 0: the top levels [0, vtop) are not expanded (their labels come from the
+// arcs entering them; sweep_top_kernel's G-up pull pass finishes them).
+cudaError_t launch_upward(const DevImage& g, const Sources& src, uint32_t k, uint32_t slot, uint32_t vtop,
+                          cudaStream_t st);
 // a2: visited bits + rows of the search spaces reset to INF, then (second launch, so
 // that every reset precedes every label) dist[v*k + i] = label_i(v).
 cudaError_t launch_seed(const DevImage& g, uint32_t k, uint32_t slot, uint32_t* dist, cudaStream_t st);
@@ -122,6 +125,13 @@ size_t top_label_budget();
 uint32_t top_chunk_vertices();
 uint32_t top_chunk_arcs();
 uint32_t top_heavy_arcs();   // chunk flag (bit 31 of vend): some vertex has more in-arcs than this
+
+// a3 + a4 for the mid levels seg[0..nseg] (device array of nseg+1 internal-id offsets,
+// level-ordered) in ONE thread-block-cluster launch with a cluster barrier per level
+// (ELL-2 records; needs dn_rec).  cluster_threads(): threads of the launch, 0 = disabled.
+cudaError_t launch_sweep_cluster(const DevImage& g, uint32_t k, const uint32_t* seg, uint32_t nseg, uint32_t* dist,
+                                 uint32_t* diam, cudaStream_t st);
+uint32_t cluster_threads();
 
 // after the sweep: clear the visited bits of every search-space vertex ("After
 // scanning v we unmark the vertex", §IV-C).

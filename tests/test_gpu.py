@@ -142,6 +142,7 @@ def test_upward_global_fallback_and_overflow(monkeypatch):
     src = phastgen.sources(g.n, 16, seed=3)
     want = oracle.sssp_many(g, src)
     monkeypatch.setenv("PHAST_FUSED", "0")             # the upward-search kernel, not the fused pull sweep
+    monkeypatch.setenv("PHAST_UP_HYBRID", "0")         # full searches (the hybrid stops below the top levels)
     monkeypatch.setenv("PHAST_UP_SMEM_CAP", "32")
     with P.Phast.from_graph(g) as h:
         assert np.array_equal(gpu_trees(h, src), want)
@@ -205,10 +206,11 @@ def test_sweep_modes(monkeypatch, mode, level_layout, delta):
         assert h.diameter(src, k_batch=64) == oracle.diameter(g, src)
 
 
-@pytest.mark.parametrize("top", ["off", "default", "nofused", "40", "700", "3000"])
+@pytest.mark.parametrize("top", ["off", "default", "nofused", "nohybrid", "40", "700", "3000", "cluster-only", "cl4"])
 def test_top_levels_kernel(monkeypatch, top):
-    """The shared-memory sweep (sweep_top_kernel: rows in shared memory, TMA-staged
-    arc chunks): off (one launch per level), default (C1 at k <= 4: the whole query
+    """The shared-memory sweep (sweep_top_kernel: rows in shared memory, cp.async-
+    staged arc chunks) and the cluster sweep of the mid levels (sweep_cluster_kernel):
+    off (one launch per level), cluster only, a 4-CTA cluster, default (C1 at k <= 4: the whole query
     fused in one launch, G-up as a pull sweep; larger k / the road graph: the top
     levels), top levels only ("nofused"), and top levels capped at V <= 40 / 700 /
     3000 vertices (the prefix ends inside the hierarchy, chunks split long levels);
@@ -216,8 +218,20 @@ def test_top_levels_kernel(monkeypatch, top):
     if top == "off":
         monkeypatch.setenv("PHAST_TOP", "0")
         monkeypatch.setenv("PHAST_FUSED", "0")
+        monkeypatch.setenv("PHAST_CL_SIZE", "0")
+    elif top == "cluster-only":                  # no shared-memory launch: mid levels in a 16-CTA cluster
+        monkeypatch.setenv("PHAST_TOP", "0")
+        monkeypatch.setenv("PHAST_FUSED", "0")
+        monkeypatch.setenv("PHAST_CL_SIZE", "16")
+    elif top == "cl4":                           # a 4-CTA cluster, one pass per level: long levels excluded
+        monkeypatch.setenv("PHAST_FUSED", "0")
+        monkeypatch.setenv("PHAST_CL_SIZE", "4")
+        monkeypatch.setenv("PHAST_CL_PASSES", "1")
     elif top == "nofused":
         monkeypatch.setenv("PHAST_FUSED", "0")
+    elif top == "nohybrid":                      # full upward searches, the top kernel only sweeps G-down
+        monkeypatch.setenv("PHAST_FUSED", "0")
+        monkeypatch.setenv("PHAST_UP_HYBRID", "0")
     elif top != "default":
         monkeypatch.setenv("PHAST_FUSED", "0")
         monkeypatch.setenv("PHAST_TOP_MAXV", top)
