@@ -325,6 +325,9 @@ def main():
         cpu = {"value": v, "unit": "trees/s", "cores": threads, "kind": "oracle",
                "sample": f"{threads} uniform sources of the full {args.config} graph, one per thread, "
                          f"binary-heap Dijkstra, {dt:.1f}s wall"}
+        if k == 1:   # latency configs (C1): one tree on one core, against the GPU's us/tree
+            v1, dt1, _ = oracle_sample(g, cfg, 1, 8)
+            cpu["us_per_tree_1thread"] = dt1 / 8 * 1e6
 
     if rank == 0:
         line = {

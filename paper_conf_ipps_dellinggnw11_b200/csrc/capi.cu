@@ -579,9 +579,17 @@ phast_ctx::Top* get_top(phast_ctx* h, uint32_t k) {
         // [0, V) with a pull pass in ascending level order (reading R9), then sweeps
         // G-down.  Exact: a G-up path only climbs, so it enters [0, V) once and its part
         // below V is found by the search, its part inside by the pull pass.
+        // When: the upward searches run beside the previous batch's sweep (side stream),
+        // so moving work from them into the top kernel only pays when they are the
+        // critical path, i.e. when a sweep is shorter than the searches: estimated sweep
+        // 8kn B at ~5 TB/s vs ~2 us per search wave (<= one per level).  Measured (r43):
+        // C2 k=16 14.1 vs 14.9 us/tree, C2D 50.9 vs 61.5 (hybrid); C2 k=64 3.87 vs 3.60,
+        // C3 k=64 2.069 vs 2.058 ms/step (full searches).  PHAST_UP_HYBRID=0/1 forces it.
         const char* he = std::getenv("PHAST_UP_HYBRID");
         const uint32_t V = L.lvl_off[J];
-        if (J && !(he && std::atoi(he) == 0)) {
+        const double sweep_us = 8.0 * k * h->n / 5e6, search_us = 2.0 * L.levels;
+        const bool hybrid = he ? std::atoi(he) != 0 : sweep_us < search_us;
+        if (J && hybrid) {
             std::vector<uint32_t> f((size_t)V + 1, 0);
             for (uint32_t u = 0; u < V; u++)
                 for (uint32_t e = L.up_first[u]; e < L.up_first[u + 1]; e++) f[L.up_arc[e].x + 1]++;

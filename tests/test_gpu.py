@@ -227,8 +227,9 @@ def test_top_levels_kernel(monkeypatch, top):
         monkeypatch.setenv("PHAST_FUSED", "0")
         monkeypatch.setenv("PHAST_CL_SIZE", "4")
         monkeypatch.setenv("PHAST_CL_PASSES", "1")
-    elif top == "nofused":
+    elif top == "nofused":                       # top levels; the hybrid upward search forced on
         monkeypatch.setenv("PHAST_FUSED", "0")
+        monkeypatch.setenv("PHAST_UP_HYBRID", "1")
     elif top == "nohybrid":                      # full upward searches, the top kernel only sweeps G-down
         monkeypatch.setenv("PHAST_FUSED", "0")
         monkeypatch.setenv("PHAST_UP_HYBRID", "0")
