@@ -243,6 +243,7 @@ template <class T> __device__ __forceinline__ void st_stream(T* p, T v) { __stcs
 
 constexpr int SWEEP_THREADS = 256;
 constexpr int ELL = 16;   // sweep_kernel AB value: ELL-2 records (DevImage::dn_rec) instead of the CSR
+constexpr int ELLP = 17;  // ELL-2 records, the next item's record loaded one item ahead
 
 // One level [vbeg, vend) (§VI "The CPU starts, for each level i, a kernel on
 // the GPU").  One (vertex, 16-byte lane) item per thread per grid-stride step; the
@@ -275,8 +276,11 @@ __global__ void __launch_bounds__(SWEEP_THREADS, AB >= 3 && AB < 8 ? 6 : 8) swee
     // level's drain; only label rows (flags, tail rows) must wait.  The loop itself
     // re-reads them (L1 / L2 hits) so that it keeps its register budget.
     uint32_t t = blockIdx.x * SWEEP_THREADS + threadIdx.x;
+    uint4 rn = make_uint4(INF, INF, INF, INF);   // ELLP: the next item's record, loaded one item ahead
     if (t < total) {
-        if constexpr (AB == ELL) {
+        if constexpr (AB == ELLP) {
+            rn = __ldg(&rec[vbeg + t / G]);
+        } else if constexpr (AB == ELL) {
             asm volatile("prefetch.global.L2 [%0];" ::"l"(rec + vbeg + t / G));
         } else {
             const uint32_t e0 = __ldg(&first[vbeg + t / G]);
@@ -291,12 +295,19 @@ __global__ void __launch_bounds__(SWEEP_THREADS, AB >= 3 && AB < 8 ? 6 : 8) swee
         T acc = inf_row<T>();
         if ((__ldg(&flags[v >> 5]) >> (v & 31)) & 1u)   // visited by an upward search
             acc = __ldg(reinterpret_cast<const T*>(d + (size_t)v * K) + lane);
-        if constexpr (AB == ELL) {
+        if constexpr (AB == ELL || AB == ELLP) {
             // one 16-byte record: the vertex's first two in-arcs (97 % of level-0 and
             // 92 % of level-1 vertices have at most two), so the gather depends on ONE
             // load instead of offsets -> arcs
             // (a missing arc has len INF: relaxing an INF row by it changes nothing)
-            const uint4 r = __ldg(&rec[v]);
+            uint4 r;
+            if constexpr (AB == ELLP) {   // record loaded one item ahead: the gathers wait on nothing
+                r = rn;
+                const uint32_t tn = t + gridDim.x * SWEEP_THREADS;
+                if (tn < total) rn = __ldg(&rec[vbeg + tn / G]);
+            } else {
+                r = __ldg(&rec[v]);
+            }
             T x0 = inf_row<T>(), x1 = inf_row<T>();
             if (r.y != INF) x0 = __ldg(reinterpret_cast<const T*>(d + (size_t)r.x * K) + lane);
             if (r.w != INF) x1 = __ldg(reinterpret_cast<const T*>(d + (size_t)r.z * K) + lane);
@@ -382,7 +393,7 @@ __global__ void __launch_bounds__(SWEEP_THREADS, AB >= 3 && AB < 8 ? 6 : 8) swee
 int arc_batch() {   // PHAST_ARC_BATCH: 1, 2, 3, 4, 8 (staged) or 16 (ELL-2 records, default); read per launch
     const char* e = std::getenv("PHAST_ARC_BATCH");
     int b = e ? std::atoi(e) : ELL;
-    if (b != 8 && b != ELL && (b < 1 || b > 4)) b = ELL;
+    if (b != 8 && b != ELL && b != ELLP && (b < 1 || b > 4)) b = ELL;
     return b;
 }
 
@@ -397,7 +408,10 @@ cudaError_t sweep_launch(const DevImage& g, uint32_t vbeg, uint32_t vend, uint32
     }
     uint64_t total = (uint64_t)(vend - vbeg) * G;
     uint64_t blocks = (total + SWEEP_THREADS - 1) / SWEEP_THREADS;
-    uint64_t cap = (uint64_t)num_sms() * 8;
+    int ab = arc_batch();
+    if ((ab == ELL || ab == ELLP) && !g.dn_rec) ab = 2;
+    // one full wave of resident CTAs (the kernels' launch bounds: 8, 6 for AB 3-4)
+    const uint64_t cap = (uint64_t)num_sms() * ((ab == 3 || ab == 4) ? 6 : 8);
     if (blocks > cap) blocks = cap;
     if (blocks == 0) return cudaSuccess;
     cudaLaunchConfig_t cfg = {};
@@ -410,9 +424,8 @@ cudaError_t sweep_launch(const DevImage& g, uint32_t vbeg, uint32_t vend, uint32
     attr[0].val.programmaticStreamSerializationAllowed = 1;
     cfg.attrs = attr;
     cfg.numAttrs = 1;
-    int ab = arc_batch();
-    if (ab == ELL && !g.dn_rec) ab = 2;
-    cudaError_t e = cudaLaunchKernelEx(&cfg, ab == ELL ? sweep_kernel<K, DIAM, STORE, STREAM, TB, ELL>
+    cudaError_t e = cudaLaunchKernelEx(&cfg, ab == ELLP ? sweep_kernel<K, DIAM, STORE, STREAM, TB, ELLP>
+                                             : ab == ELL ? sweep_kernel<K, DIAM, STORE, STREAM, TB, ELL>
                                              : ab == 8 ? sweep_kernel<K, DIAM, STORE, STREAM, TB, 8>
                                              : ab == 4 ? sweep_kernel<K, DIAM, STORE, STREAM, TB, 4>
                                              : ab == 3 ? sweep_kernel<K, DIAM, STORE, STREAM, TB, 3>

@@ -160,7 +160,8 @@ def test_upward_global_fallback_and_overflow(monkeypatch):
                                                      ("levels-hybrid", "bfs", 0), ("levels-hybrid", "diagonal", 0),
                                                      ("levels-ab1", "bfs", 0), ("levels-ab3", "bfs", 0),
                                                      ("levels-ab4", "bfs", 0), ("levels-ab8", "bfs", 0),
-                                                     ("levels-ab8", "diagonal", 0),
+                                                     ("levels-ab8", "diagonal", 0), ("levels-ab16", "bfs", 0),
+                                                     ("levels-ab17", "bfs", 0), ("levels-ab17", True, 0),
                                                      ("bottomseg2-2", "diagonal", 0), ("bottomseg2-2", "diagonal", 3000),
                                                      ("bottomseg3-2", "diagonal", 0), ("bottomsegauto-3", "diagonal", 500),
                                                      ("bottomseg2-1", "diagonal", 2000),
@@ -186,7 +187,8 @@ def test_sweep_modes(monkeypatch, mode, level_layout, delta):
         if cut != "auto":
             monkeypatch.setenv("PHAST_DIAG_CUT", cut)
         mode = "levels"
-    elif mode.startswith("levels-ab"):            # per-level launches, other arc batch (1, 3, 4, 8 = cp.async staged)
+    elif mode.startswith("levels-ab"):            # per-level launches, other arc batch (1-4, 8 = cp.async staged,
+                                                 # 16 = ELL-2 records, 17 = ELL-2 with the next record loaded ahead)
         monkeypatch.setenv("PHAST_ARC_BATCH", mode[len("levels-ab"):])
         mode = "levels"
     elif mode == "levels-hybrid":                # a few small top levels fused, the rest one launch each
