@@ -475,8 +475,8 @@ phast_ctx::Plan* get_plan(phast_ctx* h, uint32_t k) {
 
 // Chunks of one segment [a, b) over a CSR (offsets `f`): <= VCH vertices and <= ECH
 // arcs each; chunks without arcs change nothing and are skipped.
-void push_chunks(std::vector<uint4>& ch, const uint32_t* f, uint32_t a, uint32_t b) {
-    const uint32_t VCH = top_chunk_vertices(), ECH = top_chunk_arcs();
+void push_chunks(std::vector<uint4>& ch, const uint32_t* f, uint32_t a, uint32_t b, bool big) {
+    const uint32_t VCH = top_chunk_vertices(big), ECH = top_chunk_arcs(big);
     uint32_t v = a;
     while (v < b) {
         uint32_t w = v;
@@ -503,7 +503,7 @@ bool ensure_upin(phast_ctx* h) {
     for (uint32_t u = 0; u < n; u++)
         for (uint32_t e = L.up_first[u]; e < L.up_first[u + 1]; e++) arc[pos[L.up_arc[e].x]++] = Arc{u, L.up_arc[e].y};
     for (uint32_t v = 0; v < n; v++)
-        if (f[v + 1] - f[v] > top_chunk_arcs()) return false;
+        if (f[v + 1] - f[v] > top_chunk_arcs(true)) return false;
     uint32_t* df = nullptr;
     uint2* da = nullptr;
     // +4 / +2 elements: the 16-byte aligned bulk copies may read past the end
@@ -530,7 +530,8 @@ bool ensure_upin(phast_ctx* h) {
 //  - top: the longest prefix of levels whose rows [0, V) fit, each level small
 //    enough for one SM (<= 32 items per consumer thread); the rest one launch per
 //    level.  PHAST_TOP=0 disables it; PHAST_TOP_MAXV caps V.
-// Both need every vertex to have at most top_chunk_arcs() in-arcs.
+// Both need every vertex to have at most top_chunk_arcs(big) in-arcs; big chunks
+// (top_big_fits) when the rows leave room for them.
 phast_ctx::Top* get_top(phast_ctx* h, uint32_t k) {
     auto it = h->tops.find(k);
     if (it != h->tops.end()) return it->second.ok ? &it->second : nullptr;
@@ -540,21 +541,30 @@ phast_ctx::Top* get_top(phast_ctx* h, uint32_t k) {
     if (L.lvl_off.size() < 2 || h->n >= 0x80000000u) return nullptr;   // chunk vend carries a flag bit
     const uint32_t nseg = (uint32_t)L.lvl_off.size() - 1;
     const uint32_t G = k >= 4 ? k / 4 : 1;
-    const uint32_t ECH = top_chunk_arcs();
+    const uint32_t ECH = top_chunk_arcs(false);
     const uint64_t vmax_budget = top_label_budget() / (4ull * k);
     std::vector<uint4> ch;
     const char* fe = std::getenv("PHAST_FUSED");
     bool fused = !(fe && std::atoi(fe) == 0) && h->n <= vmax_budget;
-    for (uint32_t v = 0; fused && v < h->n; v++) fused = L.dn_first[v + 1] - L.dn_first[v] <= ECH;
+    const bool fbig = fused && top_big_fits(k, h->n);
+    const uint32_t ECHf = top_chunk_arcs(fbig);
+    for (uint32_t v = 0; fused && v < h->n; v++) fused = L.dn_first[v + 1] - L.dn_first[v] <= ECHf;
+    std::vector<uint32_t> f;
     if (fused && ensure_upin(h)) {
-        std::vector<uint32_t> f((size_t)h->n + 1);
+        f.resize((size_t)h->n + 1);
         if (cudaMemcpy(f.data(), h->d_upin_first, f.size() * 4, cudaMemcpyDeviceToHost) != cudaSuccess) {
             cudaGetLastError();
             return nullptr;
         }
-        for (uint32_t j = nseg; j-- > 0;) push_chunks(ch, f.data(), L.lvl_off[j], L.lvl_off[j + 1]);   // ascending levels
+        for (uint32_t v = 0; fused && v < h->n; v++) fused = f[v + 1] - f[v] <= ECHf;
+    } else {
+        fused = false;
+    }
+    if (fused) {
+        for (uint32_t j = nseg; j-- > 0;) push_chunks(ch, f.data(), L.lvl_off[j], L.lvl_off[j + 1], fbig);   // ascending levels
         T.a.split = (uint32_t)ch.size();
-        for (uint32_t j = 0; j < nseg; j++) push_chunks(ch, L.dn_first.data(), L.lvl_off[j], L.lvl_off[j + 1]);
+        for (uint32_t j = 0; j < nseg; j++) push_chunks(ch, L.dn_first.data(), L.lvl_off[j], L.lvl_off[j + 1], fbig);
+        T.a.big = fbig;
         T.a.first[0] = h->d_upin_first;
         T.a.arcs[0] = h->d_upin_arc;
         T.a.fused = 1;
@@ -587,6 +597,8 @@ phast_ctx::Top* get_top(phast_ctx* h, uint32_t k) {
         // C3 k=64 2.069 vs 2.058 ms/step (full searches).  PHAST_UP_HYBRID=0/1 forces it.
         const char* he = std::getenv("PHAST_UP_HYBRID");
         const uint32_t V = L.lvl_off[J];
+        const bool big = J && top_big_fits(k, V);
+        T.a.big = big;
         const double sweep_us = 8.0 * k * h->n / 5e6, search_us = 2.0 * L.levels;
         const bool hybrid = he ? std::atoi(he) != 0 : sweep_us < search_us;
         if (J && hybrid) {
@@ -600,13 +612,13 @@ phast_ctx::Top* get_top(phast_ctx* h, uint32_t k) {
                 for (uint32_t e = L.up_first[u]; e < L.up_first[u + 1]; e++)
                     arc[pos[L.up_arc[e].x]++] = Arc{u, L.up_arc[e].y};
             bool fits = true;
-            for (uint32_t v = 0; v < V && fits; v++) fits = f[v + 1] - f[v] <= ECH;
+            for (uint32_t v = 0; v < V && fits; v++) fits = f[v + 1] - f[v] <= top_chunk_arcs(big);
             if (fits && !dmalloc(&T.up_f, f.size() + 4) && !dmalloc(&T.up_a, arc.size() + 2) &&
                 cudaMemset(T.up_f, 0, (f.size() + 4) * 4) == cudaSuccess &&
                 cudaMemset(T.up_a, 0, (arc.size() + 2) * 8) == cudaSuccess &&
                 cudaMemcpy(T.up_f, f.data(), f.size() * 4, cudaMemcpyHostToDevice) == cudaSuccess &&
                 (arc.empty() || cudaMemcpy(T.up_a, arc.data(), arc.size() * 8, cudaMemcpyHostToDevice) == cudaSuccess)) {
-                for (uint32_t j = J; j-- > 0;) push_chunks(ch, f.data(), L.lvl_off[j], L.lvl_off[j + 1]);
+                for (uint32_t j = J; j-- > 0;) push_chunks(ch, f.data(), L.lvl_off[j], L.lvl_off[j + 1], big);
                 T.a.first[0] = T.up_f;
                 T.a.arcs[0] = T.up_a;
                 T.vtop = V;
@@ -615,7 +627,7 @@ phast_ctx::Top* get_top(phast_ctx* h, uint32_t k) {
             }
         }
         T.a.split = (uint32_t)ch.size();
-        for (uint32_t j = 0; j < J; j++) push_chunks(ch, L.dn_first.data(), L.lvl_off[j], L.lvl_off[j + 1]);
+        for (uint32_t j = 0; j < J; j++) push_chunks(ch, L.dn_first.data(), L.lvl_off[j], L.lvl_off[j + 1], big);
         T.J = J;
         T.a.V = V;
         // the next levels, while small, in one cluster launch (PHAST_CL_SIZE=0 disables;

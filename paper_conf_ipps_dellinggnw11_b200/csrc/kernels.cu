@@ -1712,9 +1712,15 @@ __global__ void max_reduce_kernel(const uint32_t* __restrict__ in, uint32_t coun
 //    vertex at once.  The chunks [split, nchunks) are then the downward sweep.  One
 //    launch per query: no upward kernel, no seeding, no visited bits.
 constexpr int TOP_THREADS = 1024, TOP_CONS = TOP_THREADS - 32;
-constexpr uint32_t TOP_VCH = 256, TOP_ECH = 1024;                 // per chunk: vertices, arcs
-constexpr uint32_t TOP_OFF_BUF = TOP_VCH + 8, TOP_ARC_BUF = TOP_ECH + 2;
-constexpr size_t TOP_STAGE_BYTES = 16 + TOP_OFF_BUF * 4 + TOP_ARC_BUF * 8;   // {descriptor, offsets, arcs}: 9 280
+// chunk geometry (per plan, TopArgs::big): small 256 vertices / 1 024 arcs (9 280-byte
+// stages), big 1 024 / 4 096 (36 928-byte stages) when the rows leave room for 4 big
+// stages: fewer, larger chunks = fewer barriers on the long levels of small-k queries
+constexpr uint32_t TOP_VCH = 256, TOP_ECH = 1024, TOP_VCH_BIG = 1024, TOP_ECH_BIG = 4096;
+__host__ __device__ constexpr uint32_t top_off_buf(bool big) { return (big ? TOP_VCH_BIG : TOP_VCH) + 8; }
+__host__ __device__ constexpr size_t top_stage_bytes(bool big) {   // {descriptor, offsets, arcs}
+    return 16 + top_off_buf(big) * 4 + ((big ? TOP_ECH_BIG : TOP_ECH) + 2) * 8;
+}
+constexpr size_t TOP_STAGE_BYTES = top_stage_bytes(false);
 constexpr uint32_t TOP_MAX_STAGES = 24, TOP_MIN_STAGES = 4;
 constexpr size_t TOP_SMEM_MAX = 227 * 1024;
 
@@ -1742,7 +1748,9 @@ __global__ void __launch_bounds__(TOP_THREADS, 1) sweep_top_kernel(TopArgs A, So
     T* srow = reinterpret_cast<T*>(top_smem);
     const size_t lab = ((size_t)V * G * sizeof(T) + 15) & ~(size_t)15;
     unsigned char* ring = top_smem + lab;                                   // [S] {offsets, arcs}
-    uint64_t* full = reinterpret_cast<uint64_t*>(ring + (size_t)S * TOP_STAGE_BYTES);
+    const size_t SB = top_stage_bytes(A.big);
+    const uint32_t OFFB = top_off_buf(A.big);
+    uint64_t* full = reinterpret_cast<uint64_t*>(ring + (size_t)S * SB);
     uint64_t* empty = full + S;
     const uint32_t tid = threadIdx.x;
     if (tid == 0) {
@@ -1791,13 +1799,13 @@ __global__ void __launch_bounds__(TOP_THREADS, 1) sweep_top_kernel(TopArgs A, So
             const bool up = c < A.split;
             const uint32_t f0 = ch.x & ~3u, nf4 = ((ch.y & TOP_VMASK) + 1 - f0 + 3) / 4;   // 16-byte units
             const uint32_t a0 = ch.z & ~1u, na2 = (ch.w - a0 + 1) / 2;
-            unsigned char* st = ring + (size_t)s * TOP_STAGE_BYTES;
+            unsigned char* st = ring + (size_t)s * SB;
             const uint4* gf = reinterpret_cast<const uint4*>((up ? A.first[0] : A.first[1]) + f0);
             const uint4* ga = reinterpret_cast<const uint4*>((up ? A.arcs[0] : A.arcs[1]) + a0);
             for (uint32_t u = lane; u < 1 + nf4 + na2; u += 32) {
                 if (u == 0) cp_async16(st, A.chunks + c);   // the consumers read the descriptor here
                 else if (u <= nf4) cp_async16(st + 16 * u, gf + (u - 1));
-                else cp_async16(st + 16 + TOP_OFF_BUF * 4 + 16 * (u - 1 - nf4), ga + (u - 1 - nf4));
+                else cp_async16(st + 16 + OFFB * 4 + 16 * (u - 1 - nf4), ga + (u - 1 - nf4));
             }
             asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];" ::"r"(smem_u32(&full[s])) : "memory");
             if (++s == S) { s = 0; ph ^= 1u; }
@@ -1809,11 +1817,11 @@ __global__ void __launch_bounds__(TOP_THREADS, 1) sweep_top_kernel(TopArgs A, So
             if (A.dbg && ct == 0) A.dbg[4 * c] = clock64();
             mbar_wait(&full[s], ph);
             if (A.dbg && ct == 0) A.dbg[4 * c + 1] = clock64();
-            const unsigned char* st = ring + (size_t)s * TOP_STAGE_BYTES;
+            const unsigned char* st = ring + (size_t)s * SB;
             const uint4 ch = *reinterpret_cast<const uint4*>(st);
             const uint32_t f0 = ch.x & ~3u, a0 = ch.z & ~1u;
             const uint32_t* sf = reinterpret_cast<const uint32_t*>(st + 16);
-            const uint2* sa = reinterpret_cast<const uint2*>(st + 16 + TOP_OFF_BUF * 4);
+            const uint2* sa = reinterpret_cast<const uint2*>(st + 16 + OFFB * 4);
             const uint32_t vend = ch.y & TOP_VMASK;
             const bool heavy = G == 1 && (ch.y & ~TOP_VMASK);   // host: some vertex has > TOP_HEAVY in-arcs
             const uint32_t total = (vend - ch.x) * G;
@@ -1881,8 +1889,12 @@ __global__ void __launch_bounds__(TOP_THREADS, 1) sweep_top_kernel(TopArgs A, So
 
 size_t top_ring_min() { return TOP_MIN_STAGES * TOP_STAGE_BYTES + 2 * TOP_MIN_STAGES * sizeof(uint64_t); }
 size_t top_label_budget() { return TOP_SMEM_MAX - top_ring_min() - 16; }
-uint32_t top_chunk_vertices() { return TOP_VCH; }
-uint32_t top_chunk_arcs() { return TOP_ECH; }
+uint32_t top_chunk_vertices(bool big) { return big ? TOP_VCH_BIG : TOP_VCH; }
+uint32_t top_chunk_arcs(bool big) { return big ? TOP_ECH_BIG : TOP_ECH; }
+bool top_big_fits(uint32_t k, uint32_t V) {   // rows + 4 big stages within shared memory
+    const size_t lab = ((size_t)V * k * 4 + 15) & ~(size_t)15;
+    return lab + 4 * (top_stage_bytes(true) + 16) <= TOP_SMEM_MAX;
+}
 uint32_t top_heavy_arcs() { return TOP_HEAVY; }
 
 template <int K>
@@ -1890,10 +1902,11 @@ cudaError_t top_k(TopArgs A, const Sources& src, uint32_t* dist, const uint32_t*
                   cudaStream_t st) {
     const size_t lab = ((size_t)A.V * K * 4 + 15) & ~(size_t)15;
     if (lab > top_label_budget()) return cudaErrorInvalidValue;
-    A.stages = (uint32_t)std::min<size_t>(TOP_MAX_STAGES, (TOP_SMEM_MAX - lab) / (TOP_STAGE_BYTES + 16));
+    const size_t SB = top_stage_bytes(A.big);
+    A.stages = (uint32_t)std::min<size_t>(TOP_MAX_STAGES, (TOP_SMEM_MAX - lab) / (SB + 16));
     if (const char* e = std::getenv("PHAST_TOP_STAGES"))   // experiment knob: a shallower ring
         A.stages = std::max<uint32_t>(2, std::min<uint32_t>(A.stages, (uint32_t)std::atoi(e)));
-    const size_t smem = lab + A.stages * (TOP_STAGE_BYTES + 16);
+    const size_t smem = lab + A.stages * (SB + 16);
     static bool attr_set[2] = {false, false};
     auto kern = diam ? sweep_top_kernel<K, true> : sweep_top_kernel<K, false>;
     if (!attr_set[diam ? 1 : 0]) {

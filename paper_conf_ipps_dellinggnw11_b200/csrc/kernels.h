@@ -117,13 +117,15 @@ struct TopArgs {
     const uint2* arcs[2] = {nullptr, nullptr};
     const uint4* chunks = nullptr;
     uint32_t split = 0, nchunks = 0, V = 0, stages = 0, fused = 0;
+    uint32_t big = 0;                    // chunk geometry: 0 = top_chunk_*(false), 1 = top_chunk_*(true)
     unsigned long long* dbg = nullptr;   // diagnostics (PHAST_TOP_DEBUG): per chunk 4 clock64 stamps: consumer wait start, data ready, work done; producer issue
 };
 cudaError_t launch_sweep_top(const TopArgs& A, uint32_t k, const Sources& src, uint32_t* dist,
                              const uint32_t* flags, uint32_t* diam, cudaStream_t st);
 size_t top_label_budget();
-uint32_t top_chunk_vertices();
-uint32_t top_chunk_arcs();
+uint32_t top_chunk_vertices(bool big);
+uint32_t top_chunk_arcs(bool big);
+bool top_big_fits(uint32_t k, uint32_t V);   // the big geometry leaves room for the rows
 uint32_t top_heavy_arcs();   // chunk flag (bit 31 of vend): some vertex has more in-arcs than this
 
 // a3 + a4 for the mid levels seg[0..nseg] (device array of nseg+1 internal-id offsets,

@@ -264,23 +264,25 @@ def test_fused_query_edge_cases(monkeypatch):
 
 
 def test_top_levels_hub_vertex():
-    """A sink with 2 999 in-arcs (more than one TMA chunk holds, 2 048) is contracted
-    first and ends in level 0 with all of them in G-down: the top prefix must stop
-    before its level.  Bit-exact."""
-    rng = np.random.default_rng(5)
-    n = 3000
-    t = np.r_[rng.integers(1, n, 9000), np.arange(1, n)]
-    hd = np.r_[rng.integers(1, n, 9000), np.zeros(n - 1, np.int64)]   # vertex 0: a sink hub
-    order = np.argsort(t, kind="stable")
-    t, hd = t[order], hd[order]
-    first = np.zeros(n + 1, np.uint64)
-    np.add.at(first, t + 1, 1)
-    first = np.cumsum(first).astype(np.uint64)
-    g = phastgen.Graph(n, first, hd.astype(np.uint32), rng.integers(1, 1000, t.size).astype(np.uint32))
-    with P.Phast.from_graph(g) as h:
-        for k in (1, 16):
-            src = phastgen.sources(n, k, seed=960 + k)
-            assert np.array_equal(gpu_trees(h, src), oracle.sssp_many(g, src)), k
+    """A sink hub with more in-arcs than a chunk holds (small chunks: 1 024 arcs, big:
+    4 096) is contracted first and ends in level 0 with all of them in G-down.  At
+    n = 3 000 (2 999 in-arcs) the fused query takes it in a big chunk (k = 1) and the
+    top plan stops before its level (k = 16); at n = 6 000 (5 999 in-arcs) no chunk
+    holds it and the fused plan falls back.  Bit-exact."""
+    for n in (3000, 6000):
+        rng = np.random.default_rng(n)
+        t = np.r_[rng.integers(1, n, 3 * n), np.arange(1, n)]
+        hd = np.r_[rng.integers(1, n, 3 * n), np.zeros(n - 1, np.int64)]   # vertex 0: a sink hub
+        order = np.argsort(t, kind="stable")
+        t, hd = t[order], hd[order]
+        first = np.zeros(n + 1, np.uint64)
+        np.add.at(first, t + 1, 1)
+        first = np.cumsum(first).astype(np.uint64)
+        g = phastgen.Graph(n, first, hd.astype(np.uint32), rng.integers(1, 1000, t.size).astype(np.uint32))
+        with P.Phast.from_graph(g) as h:
+            for k in (1, 16):
+                src = phastgen.sources(n, k, seed=960 + k)
+                assert np.array_equal(gpu_trees(h, src), oracle.sssp_many(g, src)), (n, k)
 
 
 @pytest.mark.parametrize("window", ["0", "1", "64"])
@@ -393,3 +395,33 @@ def test_c3_europe_scale_bench_config():
         assert np.array_equal(got[pick], want)
         for i in range(1, 64, 4):
             assert oracle.certify(g, int(src[i]), got[i]) == 0, i
+
+
+@pytest.mark.slow
+def test_c4_usa_scale_bench_config():
+    """C4 at full size (~24M vertices, ~58M arcs, USA shape) in the bench's launch
+    configuration (k=64): 3 sampled trees bit-exact against the oracle, 8 more
+    certified; plus the diameter path on the same hierarchy for 64 sources against
+    the oracle's maxima of those trees."""
+    cfg = phastgen.CONFIGS["C4"]
+    g = cfg["graph"]()
+    with P.Phast.from_graph(g) as h:
+        src = phastgen.sources(g.n, 64, seed=cfg["src_seed"])
+        got = gpu_trees(h, src)
+        pick = [3, 31, 62]
+        want = oracle.sssp_many(g, src[pick])
+        assert np.array_equal(got[pick], want)
+        for i in range(0, 64, 8):
+            assert oracle.certify(g, int(src[i]), got[i]) == 0, i
+        fin = np.where(got == INF, 0, got).max()
+        assert h.diameter(src, k_batch=64) == int(fin)
+
+
+@pytest.mark.slow
+def test_c2d_distance_metric_config():
+    """C2D (travel-distance metric, 167 levels) at full size, k=16, bit-exact."""
+    cfg = phastgen.CONFIGS["C2D"]
+    g = cfg["graph"]()
+    with P.Phast.from_graph(g) as h:
+        src = phastgen.sources(g.n, 16, seed=cfg["src_seed"])
+        assert np.array_equal(gpu_trees(h, src), oracle.sssp_many(g, src))
