@@ -189,6 +189,8 @@ int upload(phast_ctx* h) {
     uint32_t seed_cap = SEED_CAP, smem_cap = 4096;
     if (const char* e = std::getenv("PHAST_SEED_CAP"))
         seed_cap = std::max(16u, std::min<uint32_t>(SEED_CAP, (uint32_t)std::atoi(e)));
+    if (const char* e = std::getenv("PHAST_L2_PERSIST_MB"))   // experiment knob
+        set_l2_persist((size_t)std::max(0, std::atoi(e)) << 20);
     if (const char* e = std::getenv("PHAST_UP_SMEM_CAP"))
         smem_cap = std::max(16u, std::min<uint32_t>(4096u, (uint32_t)std::atoi(e)));
     auto pow2 = [](uint32_t x) { uint32_t p = 1; while (p * 2 <= x) p *= 2; return p; };

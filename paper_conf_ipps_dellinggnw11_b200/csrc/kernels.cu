@@ -29,7 +29,30 @@
 namespace phast {
 
 static std::atomic<uint64_t> g_launches{0};
+// L2 persistence window over the first rows of the label array (the top levels, which
+// a level-by-level sweep re-reads once per lower level holding one of their heads):
+// bytes, 0 = off (set_l2_persist)
+static size_t g_persist_bytes = 0;
 uint64_t launches() { return g_launches.load(); }
+
+int set_l2_persist(size_t bytes) {
+    if (bytes) {
+        int dev = 0, maxw = 0, maxp = 0;
+        if (cudaGetDevice(&dev) != cudaSuccess ||
+            cudaDeviceGetAttribute(&maxw, cudaDevAttrMaxAccessPolicyWindowSize, dev) != cudaSuccess ||
+            cudaDeviceGetAttribute(&maxp, cudaDevAttrMaxPersistingL2CacheSize, dev) != cudaSuccess) {
+            cudaGetLastError();
+            return -1;
+        }
+        bytes = std::min<size_t>(bytes, std::min<size_t>((size_t)maxw, (size_t)maxp));
+        if (cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, bytes) != cudaSuccess) {
+            cudaGetLastError();
+            return -1;
+        }
+    }
+    g_persist_bytes = bytes;
+    return 0;
+}
 
 int num_sms() {
     static int sms = 0;
@@ -419,11 +442,20 @@ cudaError_t sweep_launch(const DevImage& g, uint32_t vbeg, uint32_t vend, uint32
     cfg.blockDim = dim3(SWEEP_THREADS);
     cfg.dynamicSmemBytes = 0;
     cfg.stream = st;
-    cudaLaunchAttribute attr[1];
+    cudaLaunchAttribute attr[2];
     attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
     attr[0].val.programmaticStreamSerializationAllowed = 1;
     cfg.attrs = attr;
     cfg.numAttrs = 1;
+    if (g_persist_bytes) {   // the top levels' rows (ids [0, ...): re-read by many lower levels) persist in L2
+        attr[1].id = cudaLaunchAttributeAccessPolicyWindow;
+        attr[1].val.accessPolicyWindow.base_ptr = dist;
+        attr[1].val.accessPolicyWindow.num_bytes = std::min<size_t>(g_persist_bytes, (size_t)vend * K * 4);
+        attr[1].val.accessPolicyWindow.hitRatio = 1.0f;
+        attr[1].val.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
+        attr[1].val.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
+        cfg.numAttrs = 2;
+    }
     cudaError_t e = cudaLaunchKernelEx(&cfg, ab == ELLP ? sweep_kernel<K, DIAM, STORE, STREAM, TB, ELLP>
                                              : ab == ELL ? sweep_kernel<K, DIAM, STORE, STREAM, TB, ELL>
                                              : ab == 8 ? sweep_kernel<K, DIAM, STORE, STREAM, TB, 8>

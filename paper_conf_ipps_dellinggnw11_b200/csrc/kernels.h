@@ -143,5 +143,9 @@ cudaError_t launch_max_reduce(const uint32_t* in, uint32_t count, uint32_t* out,
 
 uint64_t launches();
 int num_sms();
+// L2 persistence for the sweep launches: the first `bytes` of each label array (the
+// top levels' rows) are accessed with the persisting property; sets the device's
+// persisting-L2 limit (process-wide).  0 = off.  Returns 0, or -1 if unsupported.
+int set_l2_persist(size_t bytes);
 
 }  // namespace phast

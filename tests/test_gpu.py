@@ -285,6 +285,23 @@ def test_top_levels_hub_vertex():
                 assert np.array_equal(gpu_trees(h, src), oracle.sssp_many(g, src)), (n, k)
 
 
+def test_l2_persistence_window(monkeypatch):
+    """The per-level sweep with an L2 persistence window over the top levels' rows
+    (PHAST_L2_PERSIST_MB) is bit-exact; the setting is process-wide, so the test
+    switches it off again at the end."""
+    g = phastgen.road(120_000, seed=39)
+    try:
+        monkeypatch.setenv("PHAST_L2_PERSIST_MB", "8")
+        with P.Phast.from_graph(g) as h:
+            for k in (1, 16, 64):
+                src = phastgen.sources(g.n, k, seed=980 + k)
+                assert np.array_equal(gpu_trees(h, src), oracle.sssp_many(g, src)), k
+    finally:
+        monkeypatch.setenv("PHAST_L2_PERSIST_MB", "0")
+        with P.Phast.from_graph(phastgen.grid(8, 8)):
+            pass
+
+
 @pytest.mark.parametrize("window", ["0", "1", "64"])
 def test_wave_sweep_every_k(monkeypatch, window):
     """The warp-wave sweep (plan_waves + sweep_wave_kernel) at every k (each k has its
