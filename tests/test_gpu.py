@@ -238,7 +238,7 @@ def test_top_levels_kernel(monkeypatch, top):
     elif top != "default":
         monkeypatch.setenv("PHAST_FUSED", "0")
         monkeypatch.setenv("PHAST_TOP_MAXV", top)
-    for g in (phastgen.CONFIGS["C1"]["graph"](), phastgen.road(60_000, seed=35), phastgen.road(9_000, seed=36)):
+    for g in (phastgen.CONFIGS["C1"]["graph"](), phastgen.road(40_000, seed=35), phastgen.road(9_000, seed=36)):
         with P.Phast.from_graph(g) as h:
             for k in (1, 2, 4, 16, 64):
                 src = phastgen.sources(g.n, k, seed=950 + k)
@@ -265,20 +265,30 @@ def test_fused_query_edge_cases(monkeypatch):
 
 def test_top_levels_hub_vertex():
     """A sink hub with more in-arcs than a chunk holds (small chunks: 1 024 arcs, big:
-    4 096) is contracted first and ends in level 0 with all of them in G-down.  At
-    n = 3 000 (2 999 in-arcs) the fused query takes it in a big chunk (k = 1) and the
-    top plan stops before its level (k = 16); at n = 6 000 (5 999 in-arcs) no chunk
-    holds it and the fused plan falls back.  Bit-exact."""
-    for n in (3000, 6000):
-        rng = np.random.default_rng(n)
-        t = np.r_[rng.integers(1, n, 3 * n), np.arange(1, n)]
-        hd = np.r_[rng.integers(1, n, 3 * n), np.zeros(n - 1, np.int64)]   # vertex 0: a sink hub
-        order = np.argsort(t, kind="stable")
-        t, hd = t[order], hd[order]
+    4 096): a grid plus one extra vertex that every grid vertex points to.  The hub
+    has no out-arcs, so it is contracted first and keeps all its in-arcs in G-down.
+    With 3 000 in-arcs, the fused query takes it in a big chunk (k = 1) and the top
+    plan stops before its level (k = 16).  With 4 500 in-arcs no chunk holds it, and
+    the fused plan falls back.  Bit-exact."""
+    for W, H in ((60, 50), (75, 60)):
+        base = phastgen.grid(W, H, 1, 1000, seed=W)
+        n = base.n + 1
+        hub = base.n
+        rng = np.random.default_rng(W)
+        deg = np.diff(base.first).astype(np.int64) + 1          # every grid vertex: one more arc, to the hub
         first = np.zeros(n + 1, np.uint64)
-        np.add.at(first, t + 1, 1)
-        first = np.cumsum(first).astype(np.uint64)
-        g = phastgen.Graph(n, first, hd.astype(np.uint32), rng.integers(1, 1000, t.size).astype(np.uint32))
+        first[1:base.n + 1] = np.cumsum(deg)
+        first[n] = first[base.n]
+        head = np.empty(int(first[n]), np.uint32)
+        length = np.empty(int(first[n]), np.uint32)
+        for_v = np.repeat(np.arange(base.n), np.diff(base.first).astype(np.int64))
+        pos = first[:-2].astype(np.int64)[for_v] + (np.arange(base.m) - base.first[:-1].astype(np.int64)[for_v])
+        head[pos] = base.head
+        length[pos] = base.len
+        last = first[1:base.n + 1].astype(np.int64) - 1
+        head[last] = hub
+        length[last] = rng.integers(1, 1000, base.n).astype(np.uint32)
+        g = phastgen.Graph(n, first, head, length)
         with P.Phast.from_graph(g) as h:
             for k in (1, 16):
                 src = phastgen.sources(n, k, seed=960 + k)
