@@ -663,27 +663,6 @@ phast_ctx::Top* get_top(phast_ctx* h, uint32_t k) {
     T.a.nchunks = none ? 0u : (uint32_t)ch.size();
     T.a.first[1] = h->g.dn_first;
     T.a.arcs[1] = h->g.dn_arc;
-    {   // L2 prefetch ranges: the G-down CSR of [0, V), and the G-up CSR the up chunks use
-        const uint32_t V = T.a.V;
-        T.a.pf_ptr[0] = h->g.dn_first;
-        T.a.pf_bytes[0] = (V + 1) * 4;
-        T.a.pf_ptr[1] = h->g.dn_arc;
-        T.a.pf_bytes[1] = (uint32_t)std::min<uint64_t>(0xFFFFFFFFull, (uint64_t)L.dn_first[V] * 8);
-        if (T.a.split) {
-            const uint32_t* uf = T.a.first[0];
-            std::vector<uint32_t> last(1);
-            if (cudaMemcpy(last.data(), uf + V, 4, cudaMemcpyDeviceToHost) != cudaSuccess) {
-                cudaGetLastError();
-                last[0] = 0;
-            }
-            T.a.pf_ptr[2] = uf;
-            T.a.pf_bytes[2] = (V + 1) * 4;
-            T.a.pf_ptr[3] = T.a.arcs[0];
-            T.a.pf_bytes[3] = (uint32_t)std::min<uint64_t>(0xFFFFFFFFull, (uint64_t)last[0] * 8);
-        }
-        if (const char* e = std::getenv("PHAST_TOP_PREFETCH"))   // experiment knob: 0 = no L2 prefetch
-            if (std::atoi(e) == 0) for (int q = 0; q < 4; q++) T.a.pf_bytes[q] = 0;
-    }
     T.ok = true;
     if (std::getenv("PHAST_VERBOSE"))
         std::fprintf(stderr, "%s plan k=%u: %u levels, %u vertices, %u chunks (%u up); cluster levels [%u, %u)\n",

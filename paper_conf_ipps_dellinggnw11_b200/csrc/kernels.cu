@@ -1723,15 +1723,15 @@ __global__ void max_reduce_kernel(const uint32_t* __restrict__ in, uint32_t coun
 // fit in shared memory run in ONE CTA instead:
 //  - the rows of [0, V) (the top levels: internal ids ascend as levels descend) live
 //    in shared memory for the whole launch and are written back once;
-//  - every thread copies its share of the offsets and arcs of the chunk D-1 ahead
-//    (contiguous per level, §IV-A) into a ring of D shared-memory
-//    stages with 16-byte cp.async, one commit group per chunk (a single producer
-//    warp, with bulk copies or cp.async, issued a chunk only every 3 000-6 000 cycles:
-//    PHAST_TOP_DEBUG stamps, r39/r46/r48);
-//  - all 32 warps relax one chunk at a time from shared memory (§III
-//    "if d(v) > d(u)+l(u,v), we set d(v) = d(u)+l(u,v)"); one barrier per chunk orders
-//    the levels (Lemma 4.1: every tail is in an earlier chunk), publishes the chunk's
-//    copies and frees the stage of the chunk before it.
+//  - warp 0 is a producer: one elected thread streams every chunk's offsets and
+//    arcs (contiguous per level, §IV-A) into a ring of `stages`
+//    shared-memory stages with bulk copies (TMA, cp.async.bulk) signalled on
+//    mbarriers, as far ahead as the ring allows (the copies, not the relaxations,
+//    are the latency: the ring is as deep as shared memory permits);
+//  - 31 consumer warps relax one chunk at a time from shared memory
+//    (§III "if d(v) > d(u)+l(u,v), we set d(v) = d(u)+l(u,v)") and meet
+//    at a named barrier after it, which orders the levels (Lemma 4.1: every tail is
+//    in an earlier chunk) and frees the ring stage.
 // Two initialisations:
 //  - top mode (fused = 0): rows = seeded label if visited, else INF (PAPER.md:16
 //    §IV-C); the upward searches and the seeding ran before;
@@ -1743,20 +1743,20 @@ __global__ void max_reduce_kernel(const uint32_t* __restrict__ in, uint32_t coun
 //    in G, stopping when the priority queue becomes empty"; reading R9), for every
 //    vertex at once.  The chunks [split, nchunks) are then the downward sweep.  One
 //    launch per query: no upward kernel, no seeding, no visited bits.
-constexpr int TOP_THREADS = 1024;
+constexpr int TOP_THREADS = 1024, TOP_CONS = TOP_THREADS - 32;
 // chunk geometry (per plan, TopArgs::big): small 256 vertices / 1 024 arcs (9 280-byte
 // stages), big 1 024 / 4 096 (36 928-byte stages) when the rows leave room for 4 big
 // stages: fewer, larger chunks = fewer barriers on the long levels of small-k queries
 constexpr uint32_t TOP_VCH = 256, TOP_ECH = 1024, TOP_VCH_BIG = 1024, TOP_ECH_BIG = 4096;
 __host__ __device__ constexpr uint32_t top_off_buf(bool big) { return (big ? TOP_VCH_BIG : TOP_VCH) + 8; }
-__host__ __device__ constexpr size_t top_stage_bytes(bool big) {   // {offsets, arcs}
-    return top_off_buf(big) * 4 + ((big ? TOP_ECH_BIG : TOP_ECH) + 2) * 8;
+__host__ __device__ constexpr size_t top_stage_bytes(bool big) {   // {descriptor, offsets, arcs}
+    return 16 + top_off_buf(big) * 4 + ((big ? TOP_ECH_BIG : TOP_ECH) + 2) * 8;
 }
-__host__ __device__ constexpr uint32_t top_stages(bool big) { return big ? 4u : 6u; }   // ring depth D
-constexpr uint32_t TOP_DESC_CAP = 512;   // chunk descriptors kept in shared memory (the rest read from L2)
+constexpr size_t TOP_STAGE_BYTES = top_stage_bytes(false);
+constexpr uint32_t TOP_MAX_STAGES = 24, TOP_MIN_STAGES = 4;
 constexpr size_t TOP_SMEM_MAX = 227 * 1024;
 
-constexpr uint32_t TOP_HEAVY = 48;   // in-arcs above which a warp relaxes the vertex (k <= 4); below, one thread (r49: at 8, most G-up vertices of levels >= 2 went to the warp path, one vertex per warp at a time)
+constexpr uint32_t TOP_HEAVY = 8;   // in-arcs above which a warp relaxes the vertex (k <= 4)
 constexpr uint32_t TOP_VMASK = 0x7FFFFFFFu;   // chunk vend; bit 31: the chunk has a vertex with > TOP_HEAVY in-arcs
 __device__ __forceinline__ uint32_t warp_min(uint32_t a) { return __reduce_min_sync(0xFFFFFFFFu, a); }
 __device__ __forceinline__ uint2 warp_min(uint2 a) { return make_uint2(warp_min(a.x), warp_min(a.y)); }
@@ -1773,27 +1773,25 @@ __global__ void __launch_bounds__(TOP_THREADS, 1) sweep_top_kernel(TopArgs A, So
                                                                    const uint32_t* __restrict__ flags,
                                                                    uint32_t* __restrict__ diam) {
     using T = typename RowT<K>::T;
-    constexpr uint32_t G = K / RowT<K>::W;   // lanes per vertex
+    constexpr uint32_t W = RowT<K>::W;
+    constexpr uint32_t G = K / W;   // lanes per vertex
     extern __shared__ __align__(16) unsigned char top_smem[];
-    const uint32_t V = A.V, nch = A.nchunks;
-    const bool big = A.big != 0;
-    const uint32_t D = top_stages(big);
-    const size_t SB = top_stage_bytes(big);
-    const uint32_t OFFB = top_off_buf(big);
+    const uint32_t V = A.V, S = A.stages;
     T* srow = reinterpret_cast<T*>(top_smem);
     const size_t lab = ((size_t)V * G * sizeof(T) + 15) & ~(size_t)15;
-    uint4* sdesc = reinterpret_cast<uint4*>(top_smem + lab);
-    const uint32_t ndesc = min(nch, TOP_DESC_CAP);
-    unsigned char* ring = top_smem + lab + (size_t)ndesc * 16;
+    unsigned char* ring = top_smem + lab;                                   // [S] {offsets, arcs}
+    const size_t SB = top_stage_bytes(A.big);
+    const uint32_t OFFB = top_off_buf(A.big);
+    uint64_t* full = reinterpret_cast<uint64_t*>(ring + (size_t)S * SB);
+    uint64_t* empty = full + S;
     const uint32_t tid = threadIdx.x;
-    // everything the ring will stream: DRAM -> L2 now
-#pragma unroll
-    for (int q = 0; q < 4; q++) {
-        const char* base = static_cast<const char*>(A.pf_ptr[q]);
-        for (uint32_t off = tid * 128u; off < A.pf_bytes[q]; off += TOP_THREADS * 128u)
-            asm volatile("prefetch.global.L2 [%0];" ::"l"(base + off));
+    if (tid == 0) {
+        for (uint32_t s = 0; s < S; s++) {
+            mbar_init(&full[s], 32);   // one cp.async arrival per producer lane
+            mbar_init(&empty[s], 1);
+        }
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
-    for (uint32_t i = tid; i < ndesc; i += TOP_THREADS) sdesc[i] = __ldg(&A.chunks[i]);
     const T* dr = reinterpret_cast<const T*>(d);
     if (A.fused) {   // every row INF, then d_i(s_i) = 0
         for (uint32_t i = tid; i < V * G; i += TOP_THREADS) srow[i] = inf_row<T>();
@@ -1806,86 +1804,109 @@ __global__ void __launch_bounds__(TOP_THREADS, 1) sweep_top_kernel(TopArgs A, So
         }
     }
     __syncthreads();
-    // {vbeg, vend | heavy bit, ebeg = first[vbeg], eend = first[vend]}
-    auto desc = [&](uint32_t c) { return c < ndesc ? sdesc[c] : __ldg(&A.chunks[c]); };
-    auto issue = [&](uint32_t c) {   // this thread's share of chunk c's copies; one commit group per chunk
-        if (c < nch && !(A.dbg_skip & 1u)) {
-            const uint4 ch = desc(c);
+    uint32_t mx = 0;
+    if (tid < 32) {   // producer warp: all 32 lanes copy (cp.async, 16 B each), then arrive
+        // (measured: 1-D bulk copies (TMA) of these small blocks issue only every
+        // ~600-2000 cycles from one SM, slower than the consumers; 16-byte cp.async
+        // from 32 lanes keeps the ring ahead)
+        // descriptors: each lane holds one of the current 32 and one of the next 32
+        // (loaded a batch ahead), so the issue loop never waits on a global load
+        const uint32_t lane = tid;
+        uint4 cur = make_uint4(0, 0, 0, 0), nxt = make_uint4(0, 0, 0, 0);
+        if (lane < A.nchunks) cur = __ldg(&A.chunks[lane]);
+        if (32 + lane < A.nchunks) nxt = __ldg(&A.chunks[32 + lane]);
+        uint32_t s = 0, ph = 0;   // stage and its use count parity
+        for (uint32_t c = 0; c < A.nchunks; c++) {
+            if ((c & 31) == 0 && c) {
+                cur = nxt;
+                if (c + 32 + lane < A.nchunks) nxt = __ldg(&A.chunks[c + 32 + lane]);
+            }
+            uint4 ch;   // {vbeg, vend | heavy bit, ebeg = first[vbeg], eend = first[vend]}
+            ch.x = __shfl_sync(0xFFFFFFFFu, cur.x, c & 31);
+            ch.y = __shfl_sync(0xFFFFFFFFu, cur.y, c & 31);
+            ch.z = __shfl_sync(0xFFFFFFFFu, cur.z, c & 31);
+            ch.w = __shfl_sync(0xFFFFFFFFu, cur.w, c & 31);
+            if (c >= S) mbar_wait(&empty[s], ph ^ 1u);   // the stage's previous chunk consumed
+            if (A.dbg && lane == 0) A.dbg[4 * c + 3] = clock64();
             const bool up = c < A.split;
             const uint32_t f0 = ch.x & ~3u, nf4 = ((ch.y & TOP_VMASK) + 1 - f0 + 3) / 4;   // 16-byte units
             const uint32_t a0 = ch.z & ~1u, na2 = (ch.w - a0 + 1) / 2;
-            unsigned char* st = ring + (size_t)(c % D) * SB;
+            unsigned char* st = ring + (size_t)s * SB;
             const uint4* gf = reinterpret_cast<const uint4*>((up ? A.first[0] : A.first[1]) + f0);
             const uint4* ga = reinterpret_cast<const uint4*>((up ? A.arcs[0] : A.arcs[1]) + a0);
-            for (uint32_t u = tid; u < nf4 + na2; u += TOP_THREADS) {
-                if (u < nf4) cp_async16(st + 16 * u, gf + u);
-                else cp_async16(st + OFFB * 4 + 16 * (u - nf4), ga + (u - nf4));
+            for (uint32_t u = lane; u < 1 + nf4 + na2; u += 32) {
+                if (u == 0) cp_async16(st, A.chunks + c);   // the consumers read the descriptor here
+                else if (u <= nf4) cp_async16(st + 16 * u, gf + (u - 1));
+                else cp_async16(st + 16 + OFFB * 4 + 16 * (u - 1 - nf4), ga + (u - 1 - nf4));
             }
+            asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];" ::"r"(smem_u32(&full[s])) : "memory");
+            if (++s == S) { s = 0; ph ^= 1u; }
         }
-        cp_async_commit();
-    };
-    for (uint32_t c = 0; c + 1 < D; c++) issue(c);   // prologue: D - 1 chunks in flight
-    uint32_t mx = 0;
-    for (uint32_t c = 0; c < nch; c++) {
-        if (A.dbg && tid == 0) A.dbg[4 * c] = clock64();
-        if (big) asm volatile("cp.async.wait_group 2;" ::: "memory");   // my copies of chunk c landed
-        else asm volatile("cp.async.wait_group 4;" ::: "memory");
-        __syncthreads();   // everyone's copies of chunk c visible; chunk c-1 relaxed, its stage free
-        if (A.dbg && tid == 0) A.dbg[4 * c + 1] = clock64();
-        issue(c + D - 1);  // into the stage of chunk c-1
-        const uint4 ch = desc(c);
-        const unsigned char* st = ring + (size_t)(c % D) * SB;
-        const uint32_t f0 = ch.x & ~3u, a0 = ch.z & ~1u;
-        const uint32_t* sf = reinterpret_cast<const uint32_t*>(st);
-        const uint2* sa = reinterpret_cast<const uint2*>(st + OFFB * 4);
-        const uint32_t vend = ch.y & TOP_VMASK;
-        const bool heavy = G == 1 && (ch.y & ~TOP_VMASK);   // host: some vertex has > TOP_HEAVY in-arcs
-        const uint32_t total = (A.dbg_skip & 2u) ? 0u : (vend - ch.x) * G;
-        for (uint32_t t = tid; t < total; t += TOP_THREADS) {
-            const uint32_t v = ch.x + t / G, lane = t % G;
-            const uint32_t e0 = sf[v - f0], e1 = sf[v + 1 - f0];
-            if (heavy && e1 - e0 > TOP_HEAVY) continue;   // a warp takes it below
-            T acc = srow[v * G + lane];
-            // four arcs at a time: their loads (then their rows' loads) are independent
-            for (uint32_t e = e0; e < e1; e += 4) {
-                uint2 a[4];
-                T x[4];
-#pragma unroll
-                for (int r = 0; r < 4; r++) a[r] = e + r < e1 ? sa[e + r - a0] : make_uint2(0u, INF);
-#pragma unroll
-                for (int r = 0; r < 4; r++) x[r] = srow[a[r].x * G + lane];   // row 0 for padding (len INF)
-#pragma unroll
-                for (int r = 0; r < 4; r++) acc = relax(acc, x[r], a[r].y);
-            }
-            srow[v * G + lane] = acc;
-        }
-        if (heavy && !(A.dbg_skip & 2u)) {
-            // vertices with many in-arcs (the top of G-up: every lower neighbour is an
-            // in-arc) would serialise a level on one thread: one warp each, the lanes
-            // striding over the arcs, then a warp min
-            const uint32_t wid = tid >> 5, wl = tid & 31, nv = vend - ch.x;
-            for (uint32_t i = wid; i < nv; i += TOP_THREADS / 32) {
-                const uint32_t v = ch.x + i;
+    } else {
+        const uint32_t ct = tid - 32;
+        uint32_t s = 0, ph = 0;
+        for (uint32_t c = 0; c < A.nchunks; c++) {
+            if (A.dbg && ct == 0) A.dbg[4 * c] = clock64();
+            mbar_wait(&full[s], ph);
+            if (A.dbg && ct == 0) A.dbg[4 * c + 1] = clock64();
+            const unsigned char* st = ring + (size_t)s * SB;
+            const uint4 ch = *reinterpret_cast<const uint4*>(st);
+            const uint32_t f0 = ch.x & ~3u, a0 = ch.z & ~1u;
+            const uint32_t* sf = reinterpret_cast<const uint32_t*>(st + 16);
+            const uint2* sa = reinterpret_cast<const uint2*>(st + 16 + OFFB * 4);
+            const uint32_t vend = ch.y & TOP_VMASK;
+            const bool heavy = G == 1 && (ch.y & ~TOP_VMASK);   // host: some vertex has > TOP_HEAVY in-arcs
+            const uint32_t total = (vend - ch.x) * G;
+            for (uint32_t t = ct; t < total; t += TOP_CONS) {
+                const uint32_t v = ch.x + t / G, lane = t % G;
                 const uint32_t e0 = sf[v - f0], e1 = sf[v + 1 - f0];
-                if (e1 - e0 <= TOP_HEAVY) continue;   // warp-uniform
-                T acc = wl == 0 ? srow[v] : inf_row<T>();
-                for (uint32_t e = e0 + wl; e < e1; e += 128) {   // four arcs per lane in flight
+                if (heavy && e1 - e0 > TOP_HEAVY) continue;   // a warp takes it below
+                T acc = srow[v * G + lane];
+                // four arcs at a time: their loads (then their rows' loads) are
+                // independent, so a vertex costs two shared-memory round trips per
+                // four arcs instead of two per arc
+                for (uint32_t e = e0; e < e1; e += 4) {
                     uint2 a[4];
                     T x[4];
 #pragma unroll
-                    for (int r = 0; r < 4; r++) a[r] = e + 32 * r < e1 ? sa[e + 32 * r - a0] : make_uint2(0u, INF);
+                    for (int r = 0; r < 4; r++) a[r] = e + r < e1 ? sa[e + r - a0] : make_uint2(0u, INF);
 #pragma unroll
-                    for (int r = 0; r < 4; r++) x[r] = srow[a[r].x];
+                    for (int r = 0; r < 4; r++) x[r] = srow[a[r].x * G + lane];   // row 0 for padding (len INF)
 #pragma unroll
                     for (int r = 0; r < 4; r++) acc = relax(acc, x[r], a[r].y);
                 }
-                acc = warp_min(acc);
-                if (wl == 0) srow[v] = acc;
+                srow[v * G + lane] = acc;
             }
+            if (heavy) {
+                // vertices with many in-arcs (the top of G-up: every lower neighbour is
+                // an in-arc) would serialise a level on one thread: one warp each, the
+                // lanes striding over the arcs, then a warp min
+                const uint32_t wid = ct >> 5, wl = ct & 31, nv = vend - ch.x;
+                for (uint32_t i = wid; i < nv; i += TOP_CONS / 32) {
+                    const uint32_t v = ch.x + i;
+                    const uint32_t e0 = sf[v - f0], e1 = sf[v + 1 - f0];
+                    if (e1 - e0 <= TOP_HEAVY) continue;   // warp-uniform
+                    T acc = wl == 0 ? srow[v] : inf_row<T>();
+                    for (uint32_t e = e0 + wl; e < e1; e += 128) {   // four arcs per lane in flight
+                        uint2 a[4];
+                        T x[4];
+#pragma unroll
+                        for (int r = 0; r < 4; r++) a[r] = e + 32 * r < e1 ? sa[e + 32 * r - a0] : make_uint2(0u, INF);
+#pragma unroll
+                        for (int r = 0; r < 4; r++) x[r] = srow[a[r].x];
+#pragma unroll
+                        for (int r = 0; r < 4; r++) acc = relax(acc, x[r], a[r].y);
+                    }
+                    acc = warp_min(acc);
+                    if (wl == 0) srow[v] = acc;
+                }
+            }
+            if (A.dbg && ct == 0) A.dbg[4 * c + 2] = clock64();
+            asm volatile("bar.sync 1, %0;" ::"n"(TOP_CONS) : "memory");   // chunk done: next level may read it
+            if (ct == 0) mbar_arrive(&empty[s]);                          // ring stage free
+            if (++s == S) { s = 0; ph ^= 1u; }
         }
-        if (A.dbg && tid == 0) A.dbg[4 * c + 2] = clock64();
     }
-    asm volatile("cp.async.wait_group 0;" ::: "memory");
     __syncthreads();
     T* dw = reinterpret_cast<T*>(d);
     for (uint32_t i = tid; i < V * G; i += TOP_THREADS) {   // final rows (a5: the fused max over them)
@@ -1898,13 +1919,13 @@ __global__ void __launch_bounds__(TOP_THREADS, 1) sweep_top_kernel(TopArgs A, So
     }
 }
 
-size_t top_fixed_bytes(bool big) { return (size_t)TOP_DESC_CAP * 16 + top_stages(big) * top_stage_bytes(big); }
-size_t top_label_budget() { return TOP_SMEM_MAX - top_fixed_bytes(false) - 16; }
+size_t top_ring_min() { return TOP_MIN_STAGES * TOP_STAGE_BYTES + 2 * TOP_MIN_STAGES * sizeof(uint64_t); }
+size_t top_label_budget() { return TOP_SMEM_MAX - top_ring_min() - 16; }
 uint32_t top_chunk_vertices(bool big) { return big ? TOP_VCH_BIG : TOP_VCH; }
 uint32_t top_chunk_arcs(bool big) { return big ? TOP_ECH_BIG : TOP_ECH; }
-bool top_big_fits(uint32_t k, uint32_t V) {   // rows + descriptors + the big ring within shared memory
+bool top_big_fits(uint32_t k, uint32_t V) {   // rows + 4 big stages within shared memory
     const size_t lab = ((size_t)V * k * 4 + 15) & ~(size_t)15;
-    return lab + top_fixed_bytes(true) <= TOP_SMEM_MAX;
+    return lab + 4 * (top_stage_bytes(true) + 16) <= TOP_SMEM_MAX;
 }
 uint32_t top_heavy_arcs() { return TOP_HEAVY; }
 
@@ -1912,11 +1933,12 @@ template <int K>
 cudaError_t top_k(TopArgs A, const Sources& src, uint32_t* dist, const uint32_t* flags, uint32_t* diam,
                   cudaStream_t st) {
     const size_t lab = ((size_t)A.V * K * 4 + 15) & ~(size_t)15;
-    const bool big = A.big != 0;
-    const size_t smem = lab + (size_t)std::min<uint32_t>(A.nchunks, TOP_DESC_CAP) * 16 +
-                        top_stages(big) * top_stage_bytes(big);
-    if (smem > TOP_SMEM_MAX) return cudaErrorInvalidValue;
-    A.stages = top_stages(big);
+    if (lab > top_label_budget()) return cudaErrorInvalidValue;
+    const size_t SB = top_stage_bytes(A.big);
+    A.stages = (uint32_t)std::min<size_t>(TOP_MAX_STAGES, (TOP_SMEM_MAX - lab) / (SB + 16));
+    if (const char* e = std::getenv("PHAST_TOP_STAGES"))   // experiment knob: a shallower ring
+        A.stages = std::max<uint32_t>(2, std::min<uint32_t>(A.stages, (uint32_t)std::atoi(e)));
+    const size_t smem = lab + A.stages * (SB + 16);
     static bool attr_set[2] = {false, false};
     auto kern = diam ? sweep_top_kernel<K, true> : sweep_top_kernel<K, false>;
     if (!attr_set[diam ? 1 : 0]) {
@@ -1926,7 +1948,6 @@ cudaError_t top_k(TopArgs A, const Sources& src, uint32_t* dist, const uint32_t*
     }
     static unsigned long long* dbg = nullptr;
     const char* dpath = std::getenv("PHAST_TOP_DEBUG");
-    if (const char* e = std::getenv("PHAST_TOP_SKIP")) A.dbg_skip = (uint32_t)std::atoi(e);   // diagnostics only
     if (dpath && !dbg) cudaMalloc(&dbg, (size_t)A.nchunks * 32);
     if (dpath) A.dbg = dbg;
     kern<<<1, TOP_THREADS, smem, st>>>(A, src, dist, flags, diam);

@@ -118,11 +118,6 @@ struct TopArgs {
     const uint4* chunks = nullptr;
     uint32_t split = 0, nchunks = 0, V = 0, stages = 0, fused = 0;
     uint32_t big = 0;                    // chunk geometry: 0 = top_chunk_*(false), 1 = top_chunk_*(true)
-    // static byte ranges the chunks read (offsets and arcs of both CSRs), prefetched into
-    // L2 by every thread at launch: one SM alone pulls them from DRAM far too slowly
-    const void* pf_ptr[4] = {nullptr, nullptr, nullptr, nullptr};
-    uint32_t pf_bytes[4] = {0, 0, 0, 0};
-    uint32_t dbg_skip = 0;               // diagnostics only (PHAST_TOP_SKIP): 1 = no copies, 2 = no relaxing (wrong labels)
     unsigned long long* dbg = nullptr;   // diagnostics (PHAST_TOP_DEBUG): per chunk 4 clock64 stamps: consumer wait start, data ready, work done; producer issue
 };
 cudaError_t launch_sweep_top(const TopArgs& A, uint32_t k, const Sources& src, uint32_t* dist,
