@@ -1723,11 +1723,11 @@ __global__ void max_reduce_kernel(const uint32_t* __restrict__ in, uint32_t coun
 // fit in shared memory run in ONE CTA instead:
 //  - the rows of [0, V) (the top levels: internal ids ascend as levels descend) live
 //    in shared memory for the whole launch and are written back once;
-//  - warp 0 is a producer: one elected thread streams every chunk's offsets and
-//    arcs (contiguous per level, §IV-A) into a ring of `stages`
-//    shared-memory stages with bulk copies (TMA, cp.async.bulk) signalled on
-//    mbarriers, as far ahead as the ring allows (the copies, not the relaxations,
-//    are the latency: the ring is as deep as shared memory permits);
+//  - warp 0 is a producer: its 32 lanes stream every chunk's offsets and arcs
+//    (contiguous per level, §IV-A) into a ring of `stages` shared-memory
+//    stages with 16-byte cp.async, arriving on the stage's mbarrier, as far ahead as
+//    the ring allows (DESIGN.md §6 lists the fills measured slower: TMA from one
+//    lane, every thread's share, TMA after an L2 prefetch);
 //  - 31 consumer warps relax one chunk at a time from shared memory
 //    (§III "if d(v) > d(u)+l(u,v), we set d(v) = d(u)+l(u,v)") and meet
 //    at a named barrier after it, which orders the levels (Lemma 4.1: every tail is

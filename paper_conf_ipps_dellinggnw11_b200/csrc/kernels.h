@@ -104,7 +104,7 @@ cudaError_t launch_parents(const uint32_t* in_first, const uint2* in_arc, uint32
                            uint32_t k, const uint32_t* dist, uint32_t* parent, cudaStream_t st);
 
 // a3 + a4 for the top levels [0, V) in ONE single-CTA launch (labels in shared
-// memory, arcs streamed by TMA through an mbarrier ring).  chunks[c] = {vbeg, vend,
+// memory, arcs streamed by cp.async through an mbarrier ring).  chunks[c] = {vbeg, vend,
 // first[vbeg], first[vend]} over CSR first[0]/arcs[0] for c < split (fused mode: the
 // G-up pull sweep, ascending levels) and CSR first[1]/arcs[1] after (G-down,
 // descending levels); at most top_chunk_vertices() vertices and top_chunk_arcs() arcs
