@@ -130,3 +130,51 @@ def parents(g, s: int, d=None) -> np.ndarray:
     if rc:
         raise ValueError(f"oracle_parents: {rc}")
     return out
+
+
+def betweenness(g, sources) -> np.ndarray:
+    """float64[n]: partial betweenness c_B(v) = sum over s in `sources`, t in V,
+    s != v != t, of sigma_st(v) / sigma_st (§VII-B "c_B(v) = sum_{s != v
+    != t in V} sigma_st(v)/sigma_st, where sigma_st is the number of shortest paths
+    between two vertices s and t"); with sources = V it is the exact betweenness.
+
+    SURVEY.md §8(f) NEXT-3.  Readings (DESIGN.md R16): directed graph, ordered pairs;
+    a path is a sequence of arcs, so parallel tight arcs are distinct paths; all
+    lengths must be > 0 (zero-length cycles make sigma unbounded; §VII-A
+    "As long as all original arc lengths are strictly positive").
+
+    Written step by step after Brandes' accumulation, the method PAPER.md:20 cites
+    for "Computing exact betweenness relies on n shortest path tree computations
+    [28]": per source, the tree of `sssp` (pinned Dijkstra); sigma in nondecreasing
+    distance order over tight arcs d(u) + l = d(w); then
+    delta(u) = sum over tight (u, w) of sigma(u)/sigma(w) * (1 + delta(w)) in
+    nonincreasing distance order; c_B(w) += delta(w) for w != s.  Plain Python
+    loops: small graphs only.  Pins: tests/test_oracle.py (brute-force path
+    enumeration, closed forms on paths and stars)."""
+    n = g.n
+    first = np.asarray(g.first, dtype=np.int64).tolist()
+    head = np.asarray(g.head, dtype=np.int64).tolist()
+    ln = np.asarray(g.len, dtype=np.int64).tolist()
+    if head and min(ln) == 0:
+        raise ValueError("betweenness needs all arc lengths > 0")
+    cb = np.zeros(n, dtype=np.float64)
+    for s in np.asarray(sources, dtype=np.int64).ravel():
+        d = sssp(g, int(s)).astype(np.int64)
+        order = [int(v) for v in np.argsort(d, kind="stable") if d[v] != INF]
+        d = d.tolist()
+        sigma = [0.0] * n
+        sigma[s] = 1.0
+        for u in order:                               # nondecreasing d(u)
+            for e in range(first[u], first[u + 1]):
+                w = head[e]
+                if w != u and d[w] != INF and d[u] + ln[e] == d[w]:
+                    sigma[w] += sigma[u]
+        delta = [0.0] * n
+        for w in reversed(order):                      # nonincreasing d(w)
+            for e in range(first[w], first[w + 1]):
+                x = head[e]
+                if x != w and d[x] != INF and d[w] + ln[e] == d[x]:
+                    delta[w] += sigma[w] / sigma[x] * (1.0 + delta[x])
+            if w != s:
+                cb[w] += delta[w]
+    return cb

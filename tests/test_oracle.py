@@ -307,3 +307,91 @@ def test_oracle_rejects_bad_input():
     bad = Graph(3, g.first, np.array([7], np.uint32), g.len)
     with pytest.raises(ValueError):
         oracle.sssp(bad, 0)
+
+
+# ---------------------------------------------------------------- NEXT-3 betweenness
+def brute_betweenness(n, arcs, sources):
+    """c_B by definition (§VII-B): enumerate every simple arc path s -> t
+    by DFS (with lengths > 0 every shortest path is simple), keep the shortest ones
+    per (s, t), and add sigma_st(v)/sigma_st for each interior v.  Parallel arcs are
+    distinct arcs, so distinct paths (reading R16).  Independent of Brandes."""
+    out = [[] for _ in range(n)]
+    for t, h, l in arcs:
+        if t != h:
+            out[t].append((h, l))
+    cb = np.zeros(n)
+    for s in sources:
+        paths = {}                     # t -> list of (length, interior vertex list)
+
+        def dfs(v, length, seen, interior):
+            for h, l in out[v]:
+                if h in seen:
+                    continue
+                paths.setdefault(h, []).append((length + l, list(interior)))
+                dfs(h, length + l, seen | {h}, interior + [h])
+        dfs(s, 0, {s}, [])
+        for t, ps in paths.items():
+            best = min(p[0] for p in ps)
+            sp = [p[1] for p in ps if p[0] == best]
+            for inter in sp:
+                for v in inter:            # the vertices strictly between s and t
+                    cb[v] += 1.0 / len(sp)
+    return cb
+
+
+@pytest.mark.parametrize("seed", range(6))
+def test_betweenness_vs_brute_force(seed):
+    rng = np.random.default_rng(100 + seed)
+    n = 6
+    arcs = []
+    for _ in range(14):
+        t, h = rng.integers(0, n, 2)
+        arcs.append((int(t), int(h), int(rng.integers(1, 4))))   # small lengths: many ties
+    arcs.append((0, 1, 2))
+    arcs.append((0, 1, 2))            # a parallel pair
+    g = csr_from_arcs(n, arcs)
+    src = list(range(n))
+    np.testing.assert_allclose(oracle.betweenness(g, src), brute_betweenness(n, arcs, src),
+                               rtol=1e-12, atol=1e-12)
+    # partial sums over a source subset add up (the batching reading)
+    a = oracle.betweenness(g, [0, 2, 4]) + oracle.betweenness(g, [1, 3, 5])
+    np.testing.assert_allclose(a, oracle.betweenness(g, src), rtol=1e-12)
+
+
+def test_betweenness_unit_grid_vs_brute_force():
+    """3x3 bidirected unit grid: many equal-length paths (sigma up to 6)."""
+    W = 3
+    arcs = []
+    for y in range(W):
+        for x in range(W):
+            v = y * W + x
+            if x + 1 < W:
+                arcs += [(v, v + 1, 1), (v + 1, v, 1)]
+            if y + 1 < W:
+                arcs += [(v, v + W, 1), (v + W, v, 1)]
+    g = csr_from_arcs(W * W, arcs)
+    cb = oracle.betweenness(g, range(W * W))
+    np.testing.assert_allclose(cb, brute_betweenness(W * W, arcs, range(W * W)), rtol=1e-12)
+    assert cb[4] == max(cb)           # the centre is the most central
+
+
+def test_betweenness_closed_forms():
+    # bidirected path v0 - ... - v(n-1): c_B(v_i) = 2 i (n-1-i) over ordered pairs
+    n = 9
+    arcs = [(i, i + 1, 3) for i in range(n - 1)] + [(i + 1, i, 3) for i in range(n - 1)]
+    cb = oracle.betweenness(csr_from_arcs(n, arcs), range(n))
+    np.testing.assert_array_equal(cb, [2.0 * i * (n - 1 - i) for i in range(n)])
+    # bidirected star: centre (n-1)(n-2), leaves 0
+    arcs = [(0, j, 5) for j in range(1, n)] + [(j, 0, 7) for j in range(1, n)]
+    cb = oracle.betweenness(csr_from_arcs(n, arcs), range(n))
+    np.testing.assert_array_equal(cb, [float((n - 1) * (n - 2))] + [0.0] * (n - 1))
+    # a diamond with doubled middle: 0->1->3, 0->2->3, plus a parallel 0->1:
+    # sigma_03 = 3, of which 2 pass through 1 and 1 through 2
+    arcs = [(0, 1, 1), (0, 1, 1), (0, 2, 1), (1, 3, 1), (2, 3, 1)]
+    cb = oracle.betweenness(csr_from_arcs(4, arcs), [0])
+    np.testing.assert_allclose(cb, [0.0, 2.0 / 3.0, 1.0 / 3.0, 0.0], rtol=1e-15)
+
+
+def test_betweenness_rejects_zero_length():
+    with pytest.raises(ValueError):
+        oracle.betweenness(csr_from_arcs(2, [(0, 1, 0)]), [0])
