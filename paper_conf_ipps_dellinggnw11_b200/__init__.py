@@ -67,6 +67,7 @@ def _load_lib():
         "phast_parents": ([vp, vp, u32, vp, vp, vp], ctypes.c_int),
         "phast_sync": ([vp, vp], ctypes.c_int),
         "phast_diameter": ([vp, vp, u64, u32, vp, vp, vp], ctypes.c_int),
+        "phast_betweenness": ([vp, vp, u64, u32, vp, vp], ctypes.c_int),
         "phast_info": ([vp, ctypes.POINTER(_Info)], ctypes.c_int),
         "phast_level_sizes": ([vp, vp], ctypes.c_int),
         "phast_order": ([vp, vp], ctypes.c_int),
@@ -89,7 +90,7 @@ def _load_lib():
 
 
 _lib = _load_lib()
-EXPORTED = ("phast_build", "phast_trees", "phast_trees_host", "phast_parents", "phast_sync", "phast_diameter", "phast_info",
+EXPORTED = ("phast_build", "phast_trees", "phast_trees_host", "phast_parents", "phast_sync", "phast_diameter", "phast_betweenness", "phast_info",
             "phast_level_sizes", "phast_order", "phast_export", "phast_save", "phast_load", "phast_free",
             "phast_strerror", "phast_launch_count", "phast_timing", "phast_timing_read",
             "phast_plan_stats")
@@ -253,6 +254,22 @@ class Phast:
         bm_ptr = None if batch_max is None else batch_max.data_ptr()
         _check("phast_diameter", _lib.phast_diameter(self._h, src.ctypes.data, src.size, k_batch,
                                                      max_out.data_ptr(), bm_ptr, _stream_ptr(stream)))
+
+    def betweenness(self, sources, k_batch=16, out=None, stream=None):
+        """Partial betweenness over `sources` (phast_betweenness):
+        device float64 tensor [n] in internal order (see vertex_to_original).  The call
+        is synchronous on `stream`."""
+        import torch
+        src = np.ascontiguousarray(sources, dtype=np.uint32)
+        if out is None:
+            out = torch.empty(self.n, dtype=torch.float64, device="cuda")
+        _check("phast_betweenness", _lib.phast_betweenness(self._h, src.ctypes.data, src.size, k_batch,
+                                                           out.data_ptr(), _stream_ptr(stream)))
+        return out
+
+    def vertex_to_original(self, vec: np.ndarray) -> np.ndarray:
+        """[n] per-vertex values in internal order -> original order."""
+        return np.ascontiguousarray(np.asarray(vec)[self.order()])
 
     def plan_stats(self, k: int, grid: int) -> dict:
         out = np.zeros(5, np.uint64)

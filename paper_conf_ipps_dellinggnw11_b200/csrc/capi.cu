@@ -37,6 +37,16 @@ struct phast_ctx {
     size_t batch_max_elems = 0;
     uint32_t* d_in_first = nullptr;     // original in-CSR on the device (parents; uploaded on first use)
     uint2* d_in_arc = nullptr;
+    // NEXT-3 betweenness: original out-CSR {head, len} by tail (internal ids), sigma/delta
+    // rows [n][k] fp64, per-pass change words (device + pinned host)
+    uint32_t* d_out_first = nullptr;
+    uint2* d_out_arc = nullptr;
+    double* bc_sigma = nullptr;
+    double* bc_delta = nullptr;
+    size_t bc_elems = 0;
+    uint32_t* bc_changed = nullptr;
+    uint32_t* bc_changed_host = nullptr;
+    int bc_len_ok = 0;                  // 0 unknown, 1 all original lengths > 0, -1 not
     // persistent-sweep plans, one per k (built on first use)
     struct Plan {
         SweepPlan p;
@@ -152,6 +162,10 @@ void free_device(phast_ctx* h) {
     cudaFree(h->dist_scratch); cudaFree(h->batch_max_scratch);
     cudaFree(h->d_in_first); cudaFree(h->d_in_arc);
     h->d_in_first = nullptr; h->d_in_arc = nullptr;
+    cudaFree(h->d_out_first); cudaFree(h->d_out_arc); cudaFree(h->bc_sigma); cudaFree(h->bc_delta);
+    cudaFree(h->bc_changed); cudaFreeHost(h->bc_changed_host);
+    h->d_out_first = nullptr; h->d_out_arc = nullptr; h->bc_sigma = h->bc_delta = nullptr;
+    h->bc_elems = 0; h->bc_changed = nullptr; h->bc_changed_host = nullptr;
     cudaFree(h->d_upin_first); cudaFree(h->d_upin_arc);
     h->d_upin_first = nullptr; h->d_upin_arc = nullptr;
     h->upin_tried = false;
@@ -787,6 +801,62 @@ ChOptions to_ch_options(const phast_opts* o) {
     return c;
 }
 
+int ensure_in_csr(phast_ctx* h) {
+    int rc;
+    if (!h->d_in_first) {   // upload the original in-CSR on first use (parents, betweenness)
+        uint32_t* f = nullptr;
+        uint2* a = nullptr;
+        if ((rc = dmalloc(&f, h->L.in_first.size())) || (rc = dmalloc(&a, h->L.in_arc.size() + 1))) {
+            cudaFree(f);
+            return rc;
+        }
+        if (cudaMemcpy(f, h->L.in_first.data(), h->L.in_first.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess ||
+            (!h->L.in_arc.empty() &&
+             cudaMemcpy(a, h->L.in_arc.data(), h->L.in_arc.size() * 8, cudaMemcpyHostToDevice) != cudaSuccess)) {
+            cudaGetLastError();
+            cudaFree(f);
+            cudaFree(a);
+            return PHAST_ECUDA;
+        }
+        h->d_in_first = f;
+        h->d_in_arc = a;
+    }
+    return PHAST_OK;
+}
+
+// Original out-arcs by tail {head, len} in internal ids: the transpose of L.in_arc
+// (betweenness delta pass), uploaded on first use.
+int ensure_out_csr(phast_ctx* h) {
+    if (h->d_out_first) return PHAST_OK;
+    const uint32_t n = h->n;
+    const auto& F = h->L.in_first;
+    const auto& A = h->L.in_arc;
+    std::vector<uint32_t> of(n + 1, 0);
+    for (const auto& a : A) of[a.x + 1]++;
+    for (uint32_t v = 0; v < n; v++) of[v + 1] += of[v];
+    std::vector<uint32_t> fill(of.begin(), of.end() - 1);
+    std::vector<Arc> oa(A.size());
+    for (uint32_t w = 0; w < n; w++)
+        for (uint32_t e = F[w]; e < F[w + 1]; e++) oa[fill[A[e].x]++] = Arc{w, A[e].y};
+    uint32_t* f = nullptr;
+    uint2* a = nullptr;
+    int rc;
+    if ((rc = dmalloc(&f, of.size())) || (rc = dmalloc(&a, oa.size() + 1))) {
+        cudaFree(f);
+        return rc;
+    }
+    if (cudaMemcpy(f, of.data(), of.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess ||
+        (!oa.empty() && cudaMemcpy(a, oa.data(), oa.size() * 8, cudaMemcpyHostToDevice) != cudaSuccess)) {
+        cudaGetLastError();
+        cudaFree(f);
+        cudaFree(a);
+        return PHAST_ECUDA;
+    }
+    h->d_out_first = f;
+    h->d_out_arc = a;
+    return PHAST_OK;
+}
+
 int ensure_scratch(phast_ctx* h, size_t elems) {
     if (h->dist_scratch_elems >= elems) return PHAST_OK;
     cudaFree(h->dist_scratch);
@@ -899,24 +969,7 @@ int phast_parents(phast_ctx* h, const uint32_t* sources, uint32_t k, const uint3
     int rc = map_sources(h, sources, k, S);
     if (rc) return rc;
     DeviceGuard dg(h->device);
-    if (!h->d_in_first) {   // upload the original in-CSR on first use
-        uint32_t* f = nullptr;
-        uint2* a = nullptr;
-        if ((rc = dmalloc(&f, h->L.in_first.size())) || (rc = dmalloc(&a, h->L.in_arc.size() + 1))) {
-            cudaFree(f);
-            return rc;
-        }
-        if (cudaMemcpy(f, h->L.in_first.data(), h->L.in_first.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess ||
-            (!h->L.in_arc.empty() &&
-             cudaMemcpy(a, h->L.in_arc.data(), h->L.in_arc.size() * 8, cudaMemcpyHostToDevice) != cudaSuccess)) {
-            cudaGetLastError();
-            cudaFree(f);
-            cudaFree(a);
-            return PHAST_ECUDA;
-        }
-        h->d_in_first = f;
-        h->d_in_arc = a;
-    }
+    if ((rc = ensure_in_csr(h))) return rc;
     if (launch_parents(h->d_in_first, h->d_in_arc, h->n, S, k, dist, parent, (cudaStream_t)stream) != cudaSuccess)
         return PHAST_ECUDA;
     return PHAST_OK;
@@ -960,6 +1013,81 @@ int phast_diameter(phast_ctx* h, const uint32_t* sources, uint64_t count, uint32
     }
     if (launch_max_reduce(bm, (uint32_t)nb, max_dev, st) != cudaSuccess) return PHAST_ECUDA;
     return PHAST_OK;
+}
+
+int phast_betweenness(phast_ctx* h, const uint32_t* sources, uint64_t count, uint32_t k_batch, double* cb_dev,
+                      void* stream) {
+    if (!h || !sources || !cb_dev || count == 0 || !k_ok(k_batch)) return PHAST_EINVAL;
+    if (h->device < 0) return PHAST_ESTATE;
+    if (h->L.in_first.size() != (size_t)h->n + 1) return PHAST_ESTATE;
+    for (uint64_t i = 0; i < count; i++)
+        if (sources[i] >= h->n) return PHAST_ERANGE;
+    if (h->bc_len_ok == 0) {   // reading R16: every original length > 0 (self-loops excepted)
+        h->bc_len_ok = 1;
+        for (const auto& a : h->L.in_arc)
+            if (a.y == 0) h->bc_len_ok = -1;
+    }
+    if (h->bc_len_ok < 0) return PHAST_EINVAL;
+    DeviceGuard dg(h->device);
+    if (!dg.ok) return PHAST_ECUDA;
+    cudaStream_t st = (cudaStream_t)stream;
+    const uint32_t n = h->n, k = k_batch;
+    const size_t elems = (size_t)n * k;
+    int rc = ensure_scratch(h, elems);
+    if (!rc) rc = ensure_in_csr(h);
+    if (!rc) rc = ensure_out_csr(h);
+    if (rc) return rc;
+    constexpr uint32_t R = 8;   // passes between host convergence checks
+    if (!h->bc_changed) {
+        if ((rc = dmalloc(&h->bc_changed, R))) return rc;
+        if (cudaMallocHost(&h->bc_changed_host, R * 4) != cudaSuccess) {
+            cudaGetLastError();
+            return PHAST_ENOMEM;
+        }
+    }
+    if (h->bc_elems < elems) {
+        cudaFree(h->bc_sigma);
+        cudaFree(h->bc_delta);
+        h->bc_sigma = h->bc_delta = nullptr;
+        h->bc_elems = 0;
+        if ((rc = dmalloc(&h->bc_sigma, elems)) || (rc = dmalloc(&h->bc_delta, elems))) return rc;
+        h->bc_elems = elems;
+    }
+    if (cudaMemsetAsync(cb_dev, 0, (size_t)n * 8, st) != cudaSuccess) return PHAST_ECUDA;
+    // repeat a relaxation pass until one changes nothing (<= hop depth + 1 passes)
+    auto fixpoint = [&](auto pass) -> int {
+        for (uint64_t it = 0; it <= (uint64_t)n + R; it += R) {
+            if (cudaMemsetAsync(h->bc_changed, 0, R * 4, st) != cudaSuccess) return PHAST_ECUDA;
+            for (uint32_t j = 0; j < R; j++)
+                if (pass(h->bc_changed + j) != cudaSuccess) return PHAST_ECUDA;
+            if (cudaMemcpyAsync(h->bc_changed_host, h->bc_changed, R * 4, cudaMemcpyDeviceToHost, st) != cudaSuccess ||
+                cudaStreamSynchronize(st) != cudaSuccess)
+                return PHAST_ECUDA;
+            for (uint32_t j = 0; j < R; j++)
+                if (h->bc_changed_host[j] == 0) return PHAST_OK;
+        }
+        return PHAST_EINTERNAL;   // cannot happen with lengths > 0
+    };
+    for (uint64_t base = 0; base < count; base += k) {
+        Sources S;
+        const uint32_t kv = (uint32_t)std::min<uint64_t>(k, count - base);
+        for (uint32_t i = 0; i < k; i++) S.s[i] = h->L.perm[sources[base + (i < kv ? i : 0)]];
+        if ((rc = run_query(h, S, k, h->dist_scratch, nullptr, st))) return rc;
+        if (cudaMemsetAsync(h->bc_sigma, 0, elems * 8, st) != cudaSuccess ||
+            cudaMemsetAsync(h->bc_delta, 0, elems * 8, st) != cudaSuccess)
+            return PHAST_ECUDA;
+        rc = fixpoint([&](uint32_t* ch) {
+            return launch_bc_sigma(h->d_in_first, h->d_in_arc, h->dist_scratch, h->bc_sigma, n, k, S, ch, st);
+        });
+        if (rc) return rc;
+        rc = fixpoint([&](uint32_t* ch) {
+            return launch_bc_delta(h->d_out_first, h->d_out_arc, h->dist_scratch, h->bc_sigma, h->bc_delta, n, k,
+                                   ch, st);
+        });
+        if (rc) return rc;
+        if (launch_bc_accum(h->bc_delta, cb_dev, n, k, kv, S, st) != cudaSuccess) return PHAST_ECUDA;
+    }
+    return phast_sync(h, stream);
 }
 
 int phast_info(const phast_ctx* h, phast_info_t* o) {

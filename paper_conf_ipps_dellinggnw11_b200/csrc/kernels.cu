@@ -2221,3 +2221,118 @@ cudaError_t launch_max_reduce(const uint32_t* in, uint32_t count, uint32_t* out,
 }
 
 }  // namespace phast
+
+// ------------------------------------------------------------------ NEXT-3 betweenness
+// Exact (partial) betweenness on top of k finished trees (§VII-B "c_B(v) =
+// sum_{s != v != t} sigma_st(v)/sigma_st").  Rows are [n][k]
+// like the labels.  With lengths > 0 the tight arcs d(u) + l = d(w) of a tree form a
+// DAG, and sigma (path counts) and delta (Brandes' dependencies) are the unique
+// solutions of
+//   sigma(v) = [v = s] + sum_{tight (u, v)} sigma(u)
+//   delta(v) = sum_{tight (v, w)} sigma(v) / sigma(w) * (1 + delta(w)).
+// Both kernels are one in-place (chaotic) relaxation pass over every (vertex, tree);
+// the host repeats a pass until one changes nothing, which is then the fixpoint.  Each
+// value is a fixed function of its inputs summed in a fixed arc order, so the result
+// does not depend on the schedule.  sigma is an integer in fp64 (exact below 2^53).
+// The in-place reads race benignly with writes of other threads (aligned 8-byte
+// stores); plain loads (not __ldg) so a pass sees writes of earlier passes.
+namespace phast {
+namespace {
+__device__ __forceinline__ bool tight(uint32_t du, uint32_t dv, uint32_t l) {
+    return du <= dv && dv - du == l;   // du + l == dv without 32-bit overflow
+}
+}  // namespace
+
+__global__ void __launch_bounds__(256) bc_sigma_kernel(const uint32_t* __restrict__ in_first,
+                                                       const uint2* __restrict__ in_arc,
+                                                       const uint32_t* __restrict__ d, double* sigma, uint32_t n,
+                                                       uint32_t k, Sources src, uint32_t* changed) {
+    const uint64_t total = (uint64_t)n * k;
+    bool ch = false;
+    for (uint64_t t = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; t < total;
+         t += (uint64_t)gridDim.x * blockDim.x) {
+        const uint32_t v = (uint32_t)(t / k), i = (uint32_t)(t % k);
+        const uint32_t dv = __ldg(&d[t]);
+        if (dv == INF) continue;
+        double acc = src.s[i] == v ? 1.0 : 0.0;
+        const uint32_t e1 = __ldg(&in_first[v + 1]);
+        for (uint32_t e = __ldg(&in_first[v]); e < e1; e++) {
+            const uint2 a = __ldg(&in_arc[e]);
+            const size_t u = (size_t)a.x * k + i;
+            if (tight(__ldg(&d[u]), dv, a.y)) acc += sigma[u];
+        }
+        if (acc != sigma[t]) {
+            sigma[t] = acc;
+            ch = true;
+        }
+    }
+    if (__syncthreads_or(ch) && threadIdx.x == 0) *changed = 1;
+}
+
+__global__ void __launch_bounds__(256) bc_delta_kernel(const uint32_t* __restrict__ out_first,
+                                                       const uint2* __restrict__ out_arc,
+                                                       const uint32_t* __restrict__ d,
+                                                       const double* __restrict__ sigma, double* delta, uint32_t n,
+                                                       uint32_t k, uint32_t* changed) {
+    const uint64_t total = (uint64_t)n * k;
+    bool ch = false;
+    for (uint64_t t = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; t < total;
+         t += (uint64_t)gridDim.x * blockDim.x) {
+        const uint32_t v = (uint32_t)(t / k), i = (uint32_t)(t % k);
+        const uint32_t dv = __ldg(&d[t]);
+        if (dv == INF) continue;
+        const double sv = __ldg(&sigma[t]);
+        double acc = 0.0;
+        const uint32_t e1 = __ldg(&out_first[v + 1]);
+        for (uint32_t e = __ldg(&out_first[v]); e < e1; e++) {
+            const uint2 a = __ldg(&out_arc[e]);
+            const size_t w = (size_t)a.x * k + i;
+            const uint32_t dw = __ldg(&d[w]);
+            if (dw != INF && tight(dv, dw, a.y)) acc += sv / __ldg(&sigma[w]) * (1.0 + delta[w]);
+        }
+        if (acc != delta[t]) {
+            delta[t] = acc;
+            ch = true;
+        }
+    }
+    if (__syncthreads_or(ch) && threadIdx.x == 0) *changed = 1;
+}
+
+// c_B(v) += sum over the first kv trees i (in order) with sources[i] != v of delta_i(v)
+__global__ void __launch_bounds__(256) bc_accum_kernel(const double* __restrict__ delta, double* __restrict__ cb,
+                                                       uint32_t n, uint32_t k, uint32_t kv, Sources src) {
+    for (uint32_t v = blockIdx.x * blockDim.x + threadIdx.x; v < n; v += gridDim.x * blockDim.x) {
+        double s = 0.0;
+        for (uint32_t i = 0; i < kv; i++)
+            if (src.s[i] != v) s += __ldg(&delta[(size_t)v * k + i]);
+        cb[v] += s;
+    }
+}
+
+static unsigned bc_blocks(uint64_t items) {
+    uint64_t b = (items + 255) / 256;
+    return (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(b, (uint64_t)num_sms() * 8));
+}
+
+cudaError_t launch_bc_sigma(const uint32_t* in_first, const uint2* in_arc, const uint32_t* d, double* sigma,
+                            uint32_t n, uint32_t k, const Sources& src, uint32_t* changed, cudaStream_t st) {
+    bc_sigma_kernel<<<bc_blocks((uint64_t)n * k), 256, 0, st>>>(in_first, in_arc, d, sigma, n, k, src, changed);
+    g_launches++;
+    return cudaGetLastError();
+}
+
+cudaError_t launch_bc_delta(const uint32_t* out_first, const uint2* out_arc, const uint32_t* d, const double* sigma,
+                            double* delta, uint32_t n, uint32_t k, uint32_t* changed, cudaStream_t st) {
+    bc_delta_kernel<<<bc_blocks((uint64_t)n * k), 256, 0, st>>>(out_first, out_arc, d, sigma, delta, n, k, changed);
+    g_launches++;
+    return cudaGetLastError();
+}
+
+cudaError_t launch_bc_accum(const double* delta, double* cb, uint32_t n, uint32_t k, uint32_t kv, const Sources& src,
+                            cudaStream_t st) {
+    bc_accum_kernel<<<bc_blocks(n), 256, 0, st>>>(delta, cb, n, k, kv, src);
+    g_launches++;
+    return cudaGetLastError();
+}
+
+}  // namespace phast

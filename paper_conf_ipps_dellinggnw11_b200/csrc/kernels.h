@@ -141,6 +141,15 @@ cudaError_t launch_clear_flags(const DevImage& g, uint32_t k, uint32_t slot, cud
 // max of per-batch maxima (diameter)
 cudaError_t launch_max_reduce(const uint32_t* in, uint32_t count, uint32_t* out, cudaStream_t st);
 
+// NEXT-3 betweenness (kernels.cu): one in-place relaxation pass each; *changed := 1 if
+// the pass wrote anything.  accum: cb[v] += sum_{i < kv, src.s[i] != v} delta[v*k+i].
+cudaError_t launch_bc_sigma(const uint32_t* in_first, const uint2* in_arc, const uint32_t* d, double* sigma,
+                            uint32_t n, uint32_t k, const Sources& src, uint32_t* changed, cudaStream_t st);
+cudaError_t launch_bc_delta(const uint32_t* out_first, const uint2* out_arc, const uint32_t* d, const double* sigma,
+                            double* delta, uint32_t n, uint32_t k, uint32_t* changed, cudaStream_t st);
+cudaError_t launch_bc_accum(const double* delta, double* cb, uint32_t n, uint32_t k, uint32_t kv, const Sources& src,
+                            cudaStream_t st);
+
 uint64_t launches();
 int num_sms();
 // L2 persistence for the sweep launches: the first `bytes` of each label array (the

@@ -452,3 +452,55 @@ def test_c2d_distance_metric_config():
     with P.Phast.from_graph(g) as h:
         src = phastgen.sources(g.n, 16, seed=cfg["src_seed"])
         assert np.array_equal(gpu_trees(h, src), oracle.sssp_many(g, src))
+
+
+# ---------------------------------------------------------------- NEXT-3 betweenness
+BC_GRAPHS = {
+    "grid": lambda: phastgen.grid(40, 30, 1, 100, seed=81),
+    "unit_grid": lambda: phastgen.grid(30, 20, 1, 2, seed=82),      # sigma ~ binomials: many ties
+    "small_lengths": lambda: phastgen.random_digraph(900, 3600, 1, 4, seed=83),
+    "unreachable": lambda: phastgen.random_digraph(1200, 1000, 1, 50, seed=84),
+    "road": lambda: phastgen.road(3000, seed=85),
+}
+
+
+def bc_close(got, want):
+    scale = max(1.0, float(np.abs(want).max()))
+    np.testing.assert_allclose(got, want, rtol=1e-9, atol=1e-12 * scale)
+
+
+@pytest.mark.parametrize("name", sorted(BC_GRAPHS))
+@pytest.mark.parametrize("k_batch", (1, 16, 64))
+def test_betweenness_vs_oracle(name, k_batch):
+    """Partial betweenness over 37 sources (ragged last batch, one duplicate) against
+    the oracle (§VII-B; fp64, tolerance: summation order only)."""
+    g = BC_GRAPHS[name]()
+    src = phastgen.sources(g.n, 37, seed=90 + k_batch, distinct=False)
+    src[5] = src[4]
+    want = oracle.betweenness(g, src)
+    with P.Phast.from_graph(g) as h:
+        got = h.vertex_to_original(h.betweenness(src, k_batch=k_batch).cpu().numpy())
+    bc_close(got, want)
+
+
+def test_betweenness_exact_all_sources_and_additivity():
+    """count = n: the exact betweenness; disjoint source shards add up (the multi-GPU
+    all_reduce(SUM) reading)."""
+    g = phastgen.grid(12, 10, 1, 6, seed=86)
+    allv = np.arange(g.n, dtype=np.uint32)
+    want = oracle.betweenness(g, allv)
+    with P.Phast.from_graph(g) as h:
+        got = h.vertex_to_original(h.betweenness(allv, k_batch=64).cpu().numpy())
+        a = h.vertex_to_original(h.betweenness(allv[::2], k_batch=32).cpu().numpy())
+        b = h.vertex_to_original(h.betweenness(allv[1::2], k_batch=8).cpu().numpy())
+    bc_close(got, want)
+    bc_close(a + b, want)
+
+
+def test_betweenness_rejects_zero_lengths():
+    g = phastgen.grid(10, 10, 0, 3, seed=87)
+    assert int(np.asarray(g.len).min()) == 0
+    with P.Phast.from_graph(g) as h:
+        with pytest.raises(P.PhastError) as e:
+            h.betweenness([0, 1])
+        assert e.value.status == -1
