@@ -46,6 +46,7 @@ struct phast_ctx {
     size_t bc_elems = 0;
     uint32_t* bc_changed = nullptr;
     uint32_t* bc_changed_host = nullptr;
+    uint8_t* bc_mark = nullptr;         // [3][n] rotating frontier marks
     int bc_len_ok = 0;                  // 0 unknown, 1 all original lengths > 0, -1 not
     // persistent-sweep plans, one per k (built on first use)
     struct Plan {
@@ -163,7 +164,8 @@ void free_device(phast_ctx* h) {
     cudaFree(h->d_in_first); cudaFree(h->d_in_arc);
     h->d_in_first = nullptr; h->d_in_arc = nullptr;
     cudaFree(h->d_out_first); cudaFree(h->d_out_arc); cudaFree(h->bc_sigma); cudaFree(h->bc_delta);
-    cudaFree(h->bc_changed); cudaFreeHost(h->bc_changed_host);
+    cudaFree(h->bc_changed); cudaFreeHost(h->bc_changed_host); cudaFree(h->bc_mark);
+    h->bc_mark = nullptr;
     h->d_out_first = nullptr; h->d_out_arc = nullptr; h->bc_sigma = h->bc_delta = nullptr;
     h->bc_elems = 0; h->bc_changed = nullptr; h->bc_changed_host = nullptr;
     cudaFree(h->d_upin_first); cudaFree(h->d_upin_arc);
@@ -1039,7 +1041,7 @@ int phast_betweenness(phast_ctx* h, const uint32_t* sources, uint64_t count, uin
     if (rc) return rc;
     constexpr uint32_t R = 8;   // passes between host convergence checks
     if (!h->bc_changed) {
-        if ((rc = dmalloc(&h->bc_changed, R))) return rc;
+        if ((rc = dmalloc(&h->bc_changed, R)) || (rc = dmalloc(&h->bc_mark, (size_t)3 * n))) return rc;
         if (cudaMallocHost(&h->bc_changed_host, R * 4) != cudaSuccess) {
             cudaGetLastError();
             return PHAST_ENOMEM;
@@ -1055,11 +1057,18 @@ int phast_betweenness(phast_ctx* h, const uint32_t* sources, uint64_t count, uin
     }
     if (cudaMemsetAsync(cb_dev, 0, (size_t)n * 8, st) != cudaSuccess) return PHAST_ECUDA;
     // repeat a relaxation pass until one changes nothing (<= hop depth + 1 passes)
+    // pass p reads marks buf[p%3], marks buf[(p+1)%3], zeroes buf[(p+2)%3]
+    const BcGraph G{h->d_in_first, h->d_in_arc, h->d_out_first, h->d_out_arc};
     auto fixpoint = [&](auto pass) -> int {
+        uint8_t* buf[3] = {h->bc_mark, h->bc_mark + n, h->bc_mark + 2 * (size_t)n};
+        if (cudaMemsetAsync(buf[0], 1, n, st) != cudaSuccess || cudaMemsetAsync(buf[1], 0, n, st) != cudaSuccess)
+            return PHAST_ECUDA;
+        uint64_t p = 0;
         for (uint64_t it = 0; it <= (uint64_t)n + R; it += R) {
             if (cudaMemsetAsync(h->bc_changed, 0, R * 4, st) != cudaSuccess) return PHAST_ECUDA;
-            for (uint32_t j = 0; j < R; j++)
-                if (pass(h->bc_changed + j) != cudaSuccess) return PHAST_ECUDA;
+            for (uint32_t j = 0; j < R; j++, p++)
+                if (pass(buf[p % 3], buf[(p + 1) % 3], buf[(p + 2) % 3], h->bc_changed + j) != cudaSuccess)
+                    return PHAST_ECUDA;
             if (cudaMemcpyAsync(h->bc_changed_host, h->bc_changed, R * 4, cudaMemcpyDeviceToHost, st) != cudaSuccess ||
                 cudaStreamSynchronize(st) != cudaSuccess)
                 return PHAST_ECUDA;
@@ -1076,13 +1085,12 @@ int phast_betweenness(phast_ctx* h, const uint32_t* sources, uint64_t count, uin
         if (cudaMemsetAsync(h->bc_sigma, 0, elems * 8, st) != cudaSuccess ||
             cudaMemsetAsync(h->bc_delta, 0, elems * 8, st) != cudaSuccess)
             return PHAST_ECUDA;
-        rc = fixpoint([&](uint32_t* ch) {
-            return launch_bc_sigma(h->d_in_first, h->d_in_arc, h->dist_scratch, h->bc_sigma, n, k, S, ch, st);
+        rc = fixpoint([&](const uint8_t* cur, uint8_t* nxt, uint8_t* clr, uint32_t* ch) {
+            return launch_bc_sigma(G, h->dist_scratch, h->bc_sigma, n, k, S, cur, nxt, clr, ch, st);
         });
         if (rc) return rc;
-        rc = fixpoint([&](uint32_t* ch) {
-            return launch_bc_delta(h->d_out_first, h->d_out_arc, h->dist_scratch, h->bc_sigma, h->bc_delta, n, k,
-                                   ch, st);
+        rc = fixpoint([&](const uint8_t* cur, uint8_t* nxt, uint8_t* clr, uint32_t* ch) {
+            return launch_bc_delta(G, h->dist_scratch, h->bc_sigma, h->bc_delta, n, k, cur, nxt, clr, ch, st);
         });
         if (rc) return rc;
         if (launch_bc_accum(h->bc_delta, cb_dev, n, k, kv, S, st) != cudaSuccess) return PHAST_ECUDA;

@@ -2243,15 +2243,25 @@ __device__ __forceinline__ bool tight(uint32_t du, uint32_t dv, uint32_t l) {
 }
 }  // namespace
 
+// Frontier (reading of the passes, not of the method): a pass only recomputes the
+// vertices marked in `cur`; a vertex whose value changed in some tree marks its
+// dependents (σ: out-neighbours, δ: in-neighbours) in `nxt`.  Three byte arrays
+// rotate: pass p reads buf[p%3], marks buf[(p+1)%3] and zeroes buf[(p+2)%3] (read by
+// pass p-1, marked by pass p+1).  The first pass has every vertex marked.
 __global__ void __launch_bounds__(256) bc_sigma_kernel(const uint32_t* __restrict__ in_first,
                                                        const uint2* __restrict__ in_arc,
+                                                       const uint32_t* __restrict__ out_first,
+                                                       const uint2* __restrict__ out_arc,
                                                        const uint32_t* __restrict__ d, double* sigma, uint32_t n,
-                                                       uint32_t k, Sources src, uint32_t* changed) {
+                                                       uint32_t k, Sources src, const uint8_t* __restrict__ cur,
+                                                       uint8_t* nxt, uint8_t* clr, uint32_t* changed) {
     const uint64_t total = (uint64_t)n * k;
+    const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
     bool ch = false;
-    for (uint64_t t = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; t < total;
-         t += (uint64_t)gridDim.x * blockDim.x) {
+    for (uint64_t v = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += stride) clr[v] = 0;
+    for (uint64_t t = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; t < total; t += stride) {
         const uint32_t v = (uint32_t)(t / k), i = (uint32_t)(t % k);
+        if (!cur[v]) continue;
         const uint32_t dv = __ldg(&d[t]);
         if (dv == INF) continue;
         double acc = src.s[i] == v ? 1.0 : 0.0;
@@ -2264,6 +2274,8 @@ __global__ void __launch_bounds__(256) bc_sigma_kernel(const uint32_t* __restric
         if (acc != sigma[t]) {
             sigma[t] = acc;
             ch = true;
+            const uint32_t f1 = __ldg(&out_first[v + 1]);
+            for (uint32_t e = __ldg(&out_first[v]); e < f1; e++) nxt[__ldg(&out_arc[e]).x] = 1;
         }
     }
     if (__syncthreads_or(ch) && threadIdx.x == 0) *changed = 1;
@@ -2271,14 +2283,19 @@ __global__ void __launch_bounds__(256) bc_sigma_kernel(const uint32_t* __restric
 
 __global__ void __launch_bounds__(256) bc_delta_kernel(const uint32_t* __restrict__ out_first,
                                                        const uint2* __restrict__ out_arc,
+                                                       const uint32_t* __restrict__ in_first,
+                                                       const uint2* __restrict__ in_arc,
                                                        const uint32_t* __restrict__ d,
                                                        const double* __restrict__ sigma, double* delta, uint32_t n,
-                                                       uint32_t k, uint32_t* changed) {
+                                                       uint32_t k, const uint8_t* __restrict__ cur, uint8_t* nxt,
+                                                       uint8_t* clr, uint32_t* changed) {
     const uint64_t total = (uint64_t)n * k;
+    const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
     bool ch = false;
-    for (uint64_t t = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; t < total;
-         t += (uint64_t)gridDim.x * blockDim.x) {
+    for (uint64_t v = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += stride) clr[v] = 0;
+    for (uint64_t t = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; t < total; t += stride) {
         const uint32_t v = (uint32_t)(t / k), i = (uint32_t)(t % k);
+        if (!cur[v]) continue;
         const uint32_t dv = __ldg(&d[t]);
         if (dv == INF) continue;
         const double sv = __ldg(&sigma[t]);
@@ -2293,6 +2310,8 @@ __global__ void __launch_bounds__(256) bc_delta_kernel(const uint32_t* __restric
         if (acc != delta[t]) {
             delta[t] = acc;
             ch = true;
+            const uint32_t f1 = __ldg(&in_first[v + 1]);
+            for (uint32_t e = __ldg(&in_first[v]); e < f1; e++) nxt[__ldg(&in_arc[e]).x] = 1;
         }
     }
     if (__syncthreads_or(ch) && threadIdx.x == 0) *changed = 1;
@@ -2314,16 +2333,20 @@ static unsigned bc_blocks(uint64_t items) {
     return (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(b, (uint64_t)num_sms() * 8));
 }
 
-cudaError_t launch_bc_sigma(const uint32_t* in_first, const uint2* in_arc, const uint32_t* d, double* sigma,
-                            uint32_t n, uint32_t k, const Sources& src, uint32_t* changed, cudaStream_t st) {
-    bc_sigma_kernel<<<bc_blocks((uint64_t)n * k), 256, 0, st>>>(in_first, in_arc, d, sigma, n, k, src, changed);
+cudaError_t launch_bc_sigma(const BcGraph& G, const uint32_t* d, double* sigma, uint32_t n, uint32_t k,
+                            const Sources& src, const uint8_t* cur, uint8_t* nxt, uint8_t* clr, uint32_t* changed,
+                            cudaStream_t st) {
+    bc_sigma_kernel<<<bc_blocks((uint64_t)n * k), 256, 0, st>>>(G.in_first, G.in_arc, G.out_first, G.out_arc, d, sigma,
+                                                                 n, k, src, cur, nxt, clr, changed);
     g_launches++;
     return cudaGetLastError();
 }
 
-cudaError_t launch_bc_delta(const uint32_t* out_first, const uint2* out_arc, const uint32_t* d, const double* sigma,
-                            double* delta, uint32_t n, uint32_t k, uint32_t* changed, cudaStream_t st) {
-    bc_delta_kernel<<<bc_blocks((uint64_t)n * k), 256, 0, st>>>(out_first, out_arc, d, sigma, delta, n, k, changed);
+cudaError_t launch_bc_delta(const BcGraph& G, const uint32_t* d, const double* sigma, double* delta, uint32_t n,
+                            uint32_t k, const uint8_t* cur, uint8_t* nxt, uint8_t* clr, uint32_t* changed,
+                            cudaStream_t st) {
+    bc_delta_kernel<<<bc_blocks((uint64_t)n * k), 256, 0, st>>>(G.out_first, G.out_arc, G.in_first, G.in_arc, d, sigma,
+                                                                 delta, n, k, cur, nxt, clr, changed);
     g_launches++;
     return cudaGetLastError();
 }

@@ -143,10 +143,20 @@ cudaError_t launch_max_reduce(const uint32_t* in, uint32_t count, uint32_t* out,
 
 // NEXT-3 betweenness (kernels.cu): one in-place relaxation pass each; *changed := 1 if
 // the pass wrote anything.  accum: cb[v] += sum_{i < kv, src.s[i] != v} delta[v*k+i].
-cudaError_t launch_bc_sigma(const uint32_t* in_first, const uint2* in_arc, const uint32_t* d, double* sigma,
-                            uint32_t n, uint32_t k, const Sources& src, uint32_t* changed, cudaStream_t st);
-cudaError_t launch_bc_delta(const uint32_t* out_first, const uint2* out_arc, const uint32_t* d, const double* sigma,
-                            double* delta, uint32_t n, uint32_t k, uint32_t* changed, cudaStream_t st);
+// Frontier: a pass recomputes the vertices marked in cur, marks the dependents of changed
+// vertices in nxt and zeroes clr (byte arrays [n]).
+struct BcGraph {
+    const uint32_t* in_first;   // original in-arcs by head {tail, len}, internal ids
+    const uint2* in_arc;
+    const uint32_t* out_first;  // original out-arcs by tail {head, len}
+    const uint2* out_arc;
+};
+cudaError_t launch_bc_sigma(const BcGraph& G, const uint32_t* d, double* sigma, uint32_t n, uint32_t k,
+                            const Sources& src, const uint8_t* cur, uint8_t* nxt, uint8_t* clr, uint32_t* changed,
+                            cudaStream_t st);
+cudaError_t launch_bc_delta(const BcGraph& G, const uint32_t* d, const double* sigma, double* delta, uint32_t n,
+                            uint32_t k, const uint8_t* cur, uint8_t* nxt, uint8_t* clr, uint32_t* changed,
+                            cudaStream_t st);
 cudaError_t launch_bc_accum(const double* delta, double* cb, uint32_t n, uint32_t k, uint32_t kv, const Sources& src,
                             cudaStream_t st);
 
