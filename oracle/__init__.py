@@ -178,3 +178,38 @@ def betweenness(g, sources) -> np.ndarray:
             if w != s:
                 cb[w] += delta[w]
     return cb
+
+
+def reach(g, sources) -> np.ndarray:
+    """uint32[n]: partial exact reach r(v) = max over s in `sources`, t in V and shortest
+    s-t paths P containing v of min(dist(s, v), dist(v, t)) (§VII-B "The
+    reach of v is defined as the maximum, over all shortest s t paths containing v, of
+    min{dist(s, v), dist(v, t)}"); 0 where v lies on no such path.  With sources = V
+    it is the exact reach.  Readings (R17): every shortest path counts (ties
+    included); dist(v, t) along P equals dist(s, t) - dist(s, v); lengths > 0.
+
+    Per source: the tree of `sssp`; v lies on a shortest s-t path iff t is reachable
+    from v over tight arcs, so the largest dist(v, t) is the height
+    h(v) = max(0, max over tight (v, w) of l + h(w)), taken in nonincreasing distance
+    order; r(v) = max over s of min(d_s(v), h_s(v)).  Plain Python loops: small
+    graphs only.  Pins: tests/test_oracle.py (brute-force path enumeration, path
+    closed form)."""
+    n = g.n
+    first = np.asarray(g.first, dtype=np.int64).tolist()
+    head = np.asarray(g.head, dtype=np.int64).tolist()
+    ln = np.asarray(g.len, dtype=np.int64).tolist()
+    if head and min(ln) == 0:
+        raise ValueError("reach needs all arc lengths > 0")
+    r = [0] * n
+    for s in np.asarray(sources, dtype=np.int64).ravel():
+        d = sssp(g, int(s)).astype(np.int64)
+        order = [int(v) for v in np.argsort(d, kind="stable") if d[v] != INF]
+        d = d.tolist()
+        h = [0] * n
+        for v in reversed(order):                      # nonincreasing d(v)
+            for e in range(first[v], first[v + 1]):
+                w = head[e]
+                if w != v and d[w] != INF and d[v] + ln[e] == d[w]:
+                    h[v] = max(h[v], ln[e] + h[w])
+            r[v] = max(r[v], min(d[v], h[v]))
+    return np.array(r, dtype=np.uint32)

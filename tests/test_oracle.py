@@ -310,6 +310,42 @@ def test_oracle_rejects_bad_input():
 
 
 # ---------------------------------------------------------------- NEXT-3 betweenness
+def brute_shortest_paths(n, arcs, s):
+    """{t: (shortest length, [list of prefix lengths along each shortest path, one
+    (vertex, length from s) pair per vertex after s])} by enumerating every simple arc
+    path from s (lengths > 0, so shortest paths are simple)."""
+    out = [[] for _ in range(n)]
+    for t, h, l in arcs:
+        if t != h:
+            out[t].append((h, l))
+    paths = {}
+
+    def dfs(v, length, seen, pre):
+        for h, l in out[v]:
+            if h in seen:
+                continue
+            paths.setdefault(h, []).append((length + l, pre + [(h, length + l)]))
+            dfs(h, length + l, seen | {h}, pre + [(h, length + l)])
+    dfs(s, 0, {s}, [])
+    res = {}
+    for t, ps in paths.items():
+        best = min(p[0] for p in ps)
+        res[t] = (best, [p[1] for p in ps if p[0] == best])
+    return res
+
+
+def brute_reach(n, arcs, sources):
+    """reach by definition (§VII-B): over every shortest s-t path and every
+    vertex v on it (s and t included, where the min is 0), min(len to v, len from v)."""
+    r = np.zeros(n, np.int64)
+    for s in sources:
+        for t, (best, sp) in brute_shortest_paths(n, arcs, s).items():
+            for p in sp:
+                for v, dv in p:
+                    r[v] = max(r[v], min(dv, best - dv))
+    return r
+
+
 def brute_betweenness(n, arcs, sources):
     """c_B by definition (§VII-B): enumerate every simple arc path s -> t
     by DFS (with lengths > 0 every shortest path is simple), keep the shortest ones
@@ -395,3 +431,27 @@ def test_betweenness_closed_forms():
 def test_betweenness_rejects_zero_length():
     with pytest.raises(ValueError):
         oracle.betweenness(csr_from_arcs(2, [(0, 1, 0)]), [0])
+
+
+@pytest.mark.parametrize("seed", range(6))
+def test_reach_vs_brute_force(seed):
+    rng = np.random.default_rng(200 + seed)
+    n = 7
+    arcs = [(int(t), int(h), int(rng.integers(1, 5))) for t, h in rng.integers(0, n, (16, 2))]
+    g = csr_from_arcs(n, arcs)
+    src = list(range(n))
+    np.testing.assert_array_equal(oracle.reach(g, src), brute_reach(n, arcs, src))
+    np.testing.assert_array_equal(np.maximum(oracle.reach(g, [0, 1, 2]), oracle.reach(g, [3, 4, 5, 6])),
+                                  oracle.reach(g, src))
+
+
+def test_reach_closed_forms():
+    # bidirected path with length-c arcs: r(v_i) = c * min(i, n-1-i)
+    n, c = 10, 7
+    arcs = [(i, i + 1, c) for i in range(n - 1)] + [(i + 1, i, c) for i in range(n - 1)]
+    np.testing.assert_array_equal(oracle.reach(csr_from_arcs(n, arcs), range(n)),
+                                  [c * min(i, n - 1 - i) for i in range(n)])
+    # a tie: 0->1->3 and 0->2->3 both shortest (length 2+3 = 4+1); reach counts every
+    # shortest path: r(1) = min(2, 3), r(2) = min(4, 1)
+    arcs = [(0, 1, 2), (1, 3, 3), (0, 2, 4), (2, 3, 1)]
+    np.testing.assert_array_equal(oracle.reach(csr_from_arcs(4, arcs), [0]), [0, 2, 1, 0])
