@@ -7,7 +7,8 @@ reference` legs may import this package.  The product path
 Plain binary-heap Dijkstra on the ORIGINAL graph (§II-A), exact by
 Theorem 3.1 (§III) for what PHAST computes; diameter (PAPER.md:20
 §VII-B); O(n+m) optimality certificate; canonical parent
-pointers by the tight-arc identity (§VII-A, reading R14).  See oracle.c for the
+pointers by the tight-arc identity (§VII-A, reading R14); exact betweenness
+and reach (§VII-B, readings R16/R17, plain Python below).  See oracle.c for the
 passage each function follows.  Pins: tests/test_oracle.py.  Parity status of
 every function: pinned.
 """

@@ -68,6 +68,7 @@ def _load_lib():
         "phast_sync": ([vp, vp], ctypes.c_int),
         "phast_diameter": ([vp, vp, u64, u32, vp, vp, vp], ctypes.c_int),
         "phast_betweenness": ([vp, vp, u64, u32, vp, vp], ctypes.c_int),
+        "phast_reach": ([vp, vp, u64, u32, vp, vp], ctypes.c_int),
         "phast_info": ([vp, ctypes.POINTER(_Info)], ctypes.c_int),
         "phast_level_sizes": ([vp, vp], ctypes.c_int),
         "phast_order": ([vp, vp], ctypes.c_int),
@@ -90,7 +91,7 @@ def _load_lib():
 
 
 _lib = _load_lib()
-EXPORTED = ("phast_build", "phast_trees", "phast_trees_host", "phast_parents", "phast_sync", "phast_diameter", "phast_betweenness", "phast_info",
+EXPORTED = ("phast_build", "phast_trees", "phast_trees_host", "phast_parents", "phast_sync", "phast_diameter", "phast_betweenness", "phast_reach", "phast_info",
             "phast_level_sizes", "phast_order", "phast_export", "phast_save", "phast_load", "phast_free",
             "phast_strerror", "phast_launch_count", "phast_timing", "phast_timing_read",
             "phast_plan_stats")
@@ -265,6 +266,17 @@ class Phast:
             out = torch.empty(self.n, dtype=torch.float64, device="cuda")
         _check("phast_betweenness", _lib.phast_betweenness(self._h, src.ctypes.data, src.size, k_batch,
                                                            out.data_ptr(), _stream_ptr(stream)))
+        return out
+
+    def reach(self, sources, k_batch=16, out=None, stream=None):
+        """Partial exact reach over `sources` (phast_reach):
+        device tensor [n] (uint32 bits in int32) in internal order.  Synchronous."""
+        import torch
+        src = np.ascontiguousarray(sources, dtype=np.uint32)
+        if out is None:
+            out = torch.empty(self.n, dtype=torch.int32, device="cuda")
+        _check("phast_reach", _lib.phast_reach(self._h, src.ctypes.data, src.size, k_batch, out.data_ptr(),
+                                               _stream_ptr(stream)))
         return out
 
     def vertex_to_original(self, vec: np.ndarray) -> np.ndarray:

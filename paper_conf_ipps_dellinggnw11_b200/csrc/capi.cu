@@ -1017,14 +1017,19 @@ int phast_diameter(phast_ctx* h, const uint32_t* sources, uint64_t count, uint32
     return PHAST_OK;
 }
 
-int phast_betweenness(phast_ctx* h, const uint32_t* sources, uint64_t count, uint32_t k_batch, double* cb_dev,
-                      void* stream) {
-    if (!h || !sources || !cb_dev || count == 0 || !k_ok(k_batch)) return PHAST_EINVAL;
+}  // extern "C"
+
+namespace {
+// NEXT-3 driver shared by phast_betweenness (out = double cb[n]) and phast_reach
+// (out = uint32 r[n]): per batch the trees, then the fixpoint(s), then the accumulation.
+int centrality(phast_ctx* h, const uint32_t* sources, uint64_t count, uint32_t k_batch, void* out, bool reach,
+               void* stream) {
+    if (!h || !sources || !out || count == 0 || !k_ok(k_batch)) return PHAST_EINVAL;
     if (h->device < 0) return PHAST_ESTATE;
     if (h->L.in_first.size() != (size_t)h->n + 1) return PHAST_ESTATE;
     for (uint64_t i = 0; i < count; i++)
         if (sources[i] >= h->n) return PHAST_ERANGE;
-    if (h->bc_len_ok == 0) {   // reading R16: every original length > 0 (self-loops excepted)
+    if (h->bc_len_ok == 0) {   // readings R16/R17: every original length > 0 (self-loops excepted)
         h->bc_len_ok = 1;
         for (const auto& a : h->L.in_arc)
             if (a.y == 0) h->bc_len_ok = -1;
@@ -1039,7 +1044,7 @@ int phast_betweenness(phast_ctx* h, const uint32_t* sources, uint64_t count, uin
     if (!rc) rc = ensure_in_csr(h);
     if (!rc) rc = ensure_out_csr(h);
     if (rc) return rc;
-    constexpr uint32_t R = 8;   // passes between host convergence checks
+    constexpr uint32_t R = 32;   // passes between host convergence checks
     if (!h->bc_changed) {
         if ((rc = dmalloc(&h->bc_changed, R)) || (rc = dmalloc(&h->bc_mark, (size_t)3 * n))) return rc;
         if (cudaMallocHost(&h->bc_changed_host, R * 4) != cudaSuccess) {
@@ -1055,9 +1060,9 @@ int phast_betweenness(phast_ctx* h, const uint32_t* sources, uint64_t count, uin
         if ((rc = dmalloc(&h->bc_sigma, elems)) || (rc = dmalloc(&h->bc_delta, elems))) return rc;
         h->bc_elems = elems;
     }
-    if (cudaMemsetAsync(cb_dev, 0, (size_t)n * 8, st) != cudaSuccess) return PHAST_ECUDA;
-    // repeat a relaxation pass until one changes nothing (<= hop depth + 1 passes)
-    // pass p reads marks buf[p%3], marks buf[(p+1)%3], zeroes buf[(p+2)%3]
+    if (cudaMemsetAsync(out, 0, (size_t)n * (reach ? 4 : 8), st) != cudaSuccess) return PHAST_ECUDA;
+    // pass p reads marks buf[p%3], marks buf[(p+1)%3], zeroes buf[(p+2)%3]; repeat until a
+    // pass changes nothing (<= hop depth of the tight DAG + 1 passes)
     const BcGraph G{h->d_in_first, h->d_in_arc, h->d_out_first, h->d_out_arc};
     auto fixpoint = [&](auto pass) -> int {
         uint8_t* buf[3] = {h->bc_mark, h->bc_mark + n, h->bc_mark + 2 * (size_t)n};
@@ -1077,11 +1082,22 @@ int phast_betweenness(phast_ctx* h, const uint32_t* sources, uint64_t count, uin
         }
         return PHAST_EINTERNAL;   // cannot happen with lengths > 0
     };
+    uint32_t* hgt = reinterpret_cast<uint32_t*>(h->bc_delta);
     for (uint64_t base = 0; base < count; base += k) {
         Sources S;
         const uint32_t kv = (uint32_t)std::min<uint64_t>(k, count - base);
         for (uint32_t i = 0; i < k; i++) S.s[i] = h->L.perm[sources[base + (i < kv ? i : 0)]];
         if ((rc = run_query(h, S, k, h->dist_scratch, nullptr, st))) return rc;
+        if (reach) {
+            if (cudaMemsetAsync(hgt, 0, elems * 4, st) != cudaSuccess) return PHAST_ECUDA;
+            rc = fixpoint([&](const uint8_t* cur, uint8_t* nxt, uint8_t* clr, uint32_t* ch) {
+                return launch_bc_height(G, h->dist_scratch, hgt, n, k, cur, nxt, clr, ch, st);
+            });
+            if (rc) return rc;
+            if (launch_reach_accum(h->dist_scratch, hgt, (uint32_t*)out, n, k, kv, st) != cudaSuccess)
+                return PHAST_ECUDA;
+            continue;
+        }
         if (cudaMemsetAsync(h->bc_sigma, 0, elems * 8, st) != cudaSuccess ||
             cudaMemsetAsync(h->bc_delta, 0, elems * 8, st) != cudaSuccess)
             return PHAST_ECUDA;
@@ -1093,9 +1109,22 @@ int phast_betweenness(phast_ctx* h, const uint32_t* sources, uint64_t count, uin
             return launch_bc_delta(G, h->dist_scratch, h->bc_sigma, h->bc_delta, n, k, cur, nxt, clr, ch, st);
         });
         if (rc) return rc;
-        if (launch_bc_accum(h->bc_delta, cb_dev, n, k, kv, S, st) != cudaSuccess) return PHAST_ECUDA;
+        if (launch_bc_accum(h->bc_delta, (double*)out, n, k, kv, S, st) != cudaSuccess) return PHAST_ECUDA;
     }
     return phast_sync(h, stream);
+}
+}  // namespace
+
+extern "C" {
+
+int phast_betweenness(phast_ctx* h, const uint32_t* sources, uint64_t count, uint32_t k_batch, double* cb_dev,
+                      void* stream) {
+    return centrality(h, sources, count, k_batch, cb_dev, false, stream);
+}
+
+int phast_reach(phast_ctx* h, const uint32_t* sources, uint64_t count, uint32_t k_batch, uint32_t* reach_dev,
+                void* stream) {
+    return centrality(h, sources, count, k_batch, reach_dev, true, stream);
 }
 
 int phast_info(const phast_ctx* h, phast_info_t* o) {

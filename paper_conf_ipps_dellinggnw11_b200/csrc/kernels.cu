@@ -2243,75 +2243,118 @@ __device__ __forceinline__ bool tight(uint32_t du, uint32_t dv, uint32_t l) {
 }
 }  // namespace
 
-// Frontier (reading of the passes, not of the method): a pass only recomputes the
-// vertices marked in `cur`; a vertex whose value changed in some tree marks its
-// dependents (σ: out-neighbours, δ: in-neighbours) in `nxt`.  Three byte arrays
+// Frontier (a schedule choice, not part of the method): a pass only recomputes the
+// vertices marked in `cur`, one thread per vertex looping over its k trees (the
+// frontier is small after the first pass, so scanning n marks is the pass's fixed
+// cost); a vertex whose value changed in some tree marks its dependents (sigma:
+// out-neighbours; delta and height: in-neighbours) in `nxt`.  Three byte arrays
 // rotate: pass p reads buf[p%3], marks buf[(p+1)%3] and zeroes buf[(p+2)%3] (read by
 // pass p-1, marked by pass p+1).  The first pass has every vertex marked.
-__global__ void __launch_bounds__(256) bc_sigma_kernel(const uint32_t* __restrict__ in_first,
-                                                       const uint2* __restrict__ in_arc,
-                                                       const uint32_t* __restrict__ out_first,
-                                                       const uint2* __restrict__ out_arc,
-                                                       const uint32_t* __restrict__ d, double* sigma, uint32_t n,
-                                                       uint32_t k, Sources src, const uint8_t* __restrict__ cur,
-                                                       uint8_t* nxt, uint8_t* clr, uint32_t* changed) {
-    const uint64_t total = (uint64_t)n * k;
-    const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+__device__ __forceinline__ void bc_mark(const uint32_t* __restrict__ f, const uint2* __restrict__ a, uint32_t v,
+                                        uint8_t* nxt) {
+    const uint32_t e1 = __ldg(&f[v + 1]);
+    for (uint32_t e = __ldg(&f[v]); e < e1; e++) nxt[__ldg(&a[e]).x] = 1;
+}
+
+__global__ void __launch_bounds__(256) bc_sigma_kernel(BcGraph G, const uint32_t* __restrict__ d, double* sigma,
+                                                       uint32_t n, uint32_t k, Sources src,
+                                                       const uint8_t* __restrict__ cur, uint8_t* nxt, uint8_t* clr,
+                                                       uint32_t* changed) {
     bool ch = false;
-    for (uint64_t v = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += stride) clr[v] = 0;
-    for (uint64_t t = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; t < total; t += stride) {
-        const uint32_t v = (uint32_t)(t / k), i = (uint32_t)(t % k);
+    for (uint32_t v = blockIdx.x * blockDim.x + threadIdx.x; v < n; v += gridDim.x * blockDim.x) {
+        clr[v] = 0;
         if (!cur[v]) continue;
-        const uint32_t dv = __ldg(&d[t]);
-        if (dv == INF) continue;
-        double acc = src.s[i] == v ? 1.0 : 0.0;
-        const uint32_t e1 = __ldg(&in_first[v + 1]);
-        for (uint32_t e = __ldg(&in_first[v]); e < e1; e++) {
-            const uint2 a = __ldg(&in_arc[e]);
-            const size_t u = (size_t)a.x * k + i;
-            if (tight(__ldg(&d[u]), dv, a.y)) acc += sigma[u];
+        const uint32_t e0 = __ldg(&G.in_first[v]), e1 = __ldg(&G.in_first[v + 1]);
+        bool any = false;
+        for (uint32_t i = 0; i < k; i++) {
+            const size_t t = (size_t)v * k + i;
+            const uint32_t dv = __ldg(&d[t]);
+            if (dv == INF) continue;
+            double acc = src.s[i] == v ? 1.0 : 0.0;
+            for (uint32_t e = e0; e < e1; e++) {
+                const uint2 a = __ldg(&G.in_arc[e]);
+                const size_t u = (size_t)a.x * k + i;
+                if (tight(__ldg(&d[u]), dv, a.y)) acc += sigma[u];
+            }
+            if (acc != sigma[t]) {
+                sigma[t] = acc;
+                any = true;
+            }
         }
-        if (acc != sigma[t]) {
-            sigma[t] = acc;
+        if (any) {
             ch = true;
-            const uint32_t f1 = __ldg(&out_first[v + 1]);
-            for (uint32_t e = __ldg(&out_first[v]); e < f1; e++) nxt[__ldg(&out_arc[e]).x] = 1;
+            bc_mark(G.out_first, G.out_arc, v, nxt);
         }
     }
     if (__syncthreads_or(ch) && threadIdx.x == 0) *changed = 1;
 }
 
-__global__ void __launch_bounds__(256) bc_delta_kernel(const uint32_t* __restrict__ out_first,
-                                                       const uint2* __restrict__ out_arc,
-                                                       const uint32_t* __restrict__ in_first,
-                                                       const uint2* __restrict__ in_arc,
-                                                       const uint32_t* __restrict__ d,
+__global__ void __launch_bounds__(256) bc_delta_kernel(BcGraph G, const uint32_t* __restrict__ d,
                                                        const double* __restrict__ sigma, double* delta, uint32_t n,
                                                        uint32_t k, const uint8_t* __restrict__ cur, uint8_t* nxt,
                                                        uint8_t* clr, uint32_t* changed) {
-    const uint64_t total = (uint64_t)n * k;
-    const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
     bool ch = false;
-    for (uint64_t v = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += stride) clr[v] = 0;
-    for (uint64_t t = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; t < total; t += stride) {
-        const uint32_t v = (uint32_t)(t / k), i = (uint32_t)(t % k);
+    for (uint32_t v = blockIdx.x * blockDim.x + threadIdx.x; v < n; v += gridDim.x * blockDim.x) {
+        clr[v] = 0;
         if (!cur[v]) continue;
-        const uint32_t dv = __ldg(&d[t]);
-        if (dv == INF) continue;
-        const double sv = __ldg(&sigma[t]);
-        double acc = 0.0;
-        const uint32_t e1 = __ldg(&out_first[v + 1]);
-        for (uint32_t e = __ldg(&out_first[v]); e < e1; e++) {
-            const uint2 a = __ldg(&out_arc[e]);
-            const size_t w = (size_t)a.x * k + i;
-            const uint32_t dw = __ldg(&d[w]);
-            if (dw != INF && tight(dv, dw, a.y)) acc += sv / __ldg(&sigma[w]) * (1.0 + delta[w]);
+        const uint32_t e0 = __ldg(&G.out_first[v]), e1 = __ldg(&G.out_first[v + 1]);
+        bool any = false;
+        for (uint32_t i = 0; i < k; i++) {
+            const size_t t = (size_t)v * k + i;
+            const uint32_t dv = __ldg(&d[t]);
+            if (dv == INF) continue;
+            const double sv = __ldg(&sigma[t]);
+            double acc = 0.0;
+            for (uint32_t e = e0; e < e1; e++) {
+                const uint2 a = __ldg(&G.out_arc[e]);
+                const size_t w = (size_t)a.x * k + i;
+                const uint32_t dw = __ldg(&d[w]);
+                if (dw != INF && tight(dv, dw, a.y)) acc += sv / __ldg(&sigma[w]) * (1.0 + delta[w]);
+            }
+            if (acc != delta[t]) {
+                delta[t] = acc;
+                any = true;
+            }
         }
-        if (acc != delta[t]) {
-            delta[t] = acc;
+        if (any) {
             ch = true;
-            const uint32_t f1 = __ldg(&in_first[v + 1]);
-            for (uint32_t e = __ldg(&in_first[v]); e < f1; e++) nxt[__ldg(&in_arc[e]).x] = 1;
+            bc_mark(G.in_first, G.in_arc, v, nxt);
+        }
+    }
+    if (__syncthreads_or(ch) && threadIdx.x == 0) *changed = 1;
+}
+
+// reach: height h(v) = max(0, max over tight (v, w) of l + h(w)) (the largest
+// dist(v, t) over the t whose shortest s-t paths pass v).  l + h(w) <= d(w) + h(w) - d(v)
+// is at most the largest finite label, so it never wraps.
+__global__ void __launch_bounds__(256) bc_height_kernel(BcGraph G, const uint32_t* __restrict__ d, uint32_t* hgt,
+                                                        uint32_t n, uint32_t k, const uint8_t* __restrict__ cur,
+                                                        uint8_t* nxt, uint8_t* clr, uint32_t* changed) {
+    bool ch = false;
+    for (uint32_t v = blockIdx.x * blockDim.x + threadIdx.x; v < n; v += gridDim.x * blockDim.x) {
+        clr[v] = 0;
+        if (!cur[v]) continue;
+        const uint32_t e0 = __ldg(&G.out_first[v]), e1 = __ldg(&G.out_first[v + 1]);
+        bool any = false;
+        for (uint32_t i = 0; i < k; i++) {
+            const size_t t = (size_t)v * k + i;
+            const uint32_t dv = __ldg(&d[t]);
+            if (dv == INF) continue;
+            uint32_t acc = 0;
+            for (uint32_t e = e0; e < e1; e++) {
+                const uint2 a = __ldg(&G.out_arc[e]);
+                const size_t w = (size_t)a.x * k + i;
+                const uint32_t dw = __ldg(&d[w]);
+                if (dw != INF && tight(dv, dw, a.y)) acc = max(acc, a.y + hgt[w]);
+            }
+            if (acc != hgt[t]) {
+                hgt[t] = acc;
+                any = true;
+            }
+        }
+        if (any) {
+            ch = true;
+            bc_mark(G.in_first, G.in_arc, v, nxt);
         }
     }
     if (__syncthreads_or(ch) && threadIdx.x == 0) *changed = 1;
@@ -2328,6 +2371,20 @@ __global__ void __launch_bounds__(256) bc_accum_kernel(const double* __restrict_
     }
 }
 
+// r(v) = max(r(v), max over the first kv trees of min(d_i(v), h_i(v)))
+__global__ void __launch_bounds__(256) reach_accum_kernel(const uint32_t* __restrict__ d,
+                                                          const uint32_t* __restrict__ hgt, uint32_t* __restrict__ r,
+                                                          uint32_t n, uint32_t k, uint32_t kv) {
+    for (uint32_t v = blockIdx.x * blockDim.x + threadIdx.x; v < n; v += gridDim.x * blockDim.x) {
+        uint32_t m = r[v];
+        for (uint32_t i = 0; i < kv; i++) {
+            const uint32_t dv = __ldg(&d[(size_t)v * k + i]);
+            if (dv != INF) m = max(m, min(dv, __ldg(&hgt[(size_t)v * k + i])));
+        }
+        r[v] = m;
+    }
+}
+
 static unsigned bc_blocks(uint64_t items) {
     uint64_t b = (items + 255) / 256;
     return (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(b, (uint64_t)num_sms() * 8));
@@ -2336,8 +2393,7 @@ static unsigned bc_blocks(uint64_t items) {
 cudaError_t launch_bc_sigma(const BcGraph& G, const uint32_t* d, double* sigma, uint32_t n, uint32_t k,
                             const Sources& src, const uint8_t* cur, uint8_t* nxt, uint8_t* clr, uint32_t* changed,
                             cudaStream_t st) {
-    bc_sigma_kernel<<<bc_blocks((uint64_t)n * k), 256, 0, st>>>(G.in_first, G.in_arc, G.out_first, G.out_arc, d, sigma,
-                                                                 n, k, src, cur, nxt, clr, changed);
+    bc_sigma_kernel<<<bc_blocks(n), 256, 0, st>>>(G, d, sigma, n, k, src, cur, nxt, clr, changed);
     g_launches++;
     return cudaGetLastError();
 }
@@ -2345,8 +2401,21 @@ cudaError_t launch_bc_sigma(const BcGraph& G, const uint32_t* d, double* sigma, 
 cudaError_t launch_bc_delta(const BcGraph& G, const uint32_t* d, const double* sigma, double* delta, uint32_t n,
                             uint32_t k, const uint8_t* cur, uint8_t* nxt, uint8_t* clr, uint32_t* changed,
                             cudaStream_t st) {
-    bc_delta_kernel<<<bc_blocks((uint64_t)n * k), 256, 0, st>>>(G.out_first, G.out_arc, G.in_first, G.in_arc, d, sigma,
-                                                                 delta, n, k, cur, nxt, clr, changed);
+    bc_delta_kernel<<<bc_blocks(n), 256, 0, st>>>(G, d, sigma, delta, n, k, cur, nxt, clr, changed);
+    g_launches++;
+    return cudaGetLastError();
+}
+
+cudaError_t launch_bc_height(const BcGraph& G, const uint32_t* d, uint32_t* hgt, uint32_t n, uint32_t k,
+                             const uint8_t* cur, uint8_t* nxt, uint8_t* clr, uint32_t* changed, cudaStream_t st) {
+    bc_height_kernel<<<bc_blocks(n), 256, 0, st>>>(G, d, hgt, n, k, cur, nxt, clr, changed);
+    g_launches++;
+    return cudaGetLastError();
+}
+
+cudaError_t launch_reach_accum(const uint32_t* d, const uint32_t* hgt, uint32_t* r, uint32_t n, uint32_t k, uint32_t kv,
+                               cudaStream_t st) {
+    reach_accum_kernel<<<bc_blocks(n), 256, 0, st>>>(d, hgt, r, n, k, kv);
     g_launches++;
     return cudaGetLastError();
 }

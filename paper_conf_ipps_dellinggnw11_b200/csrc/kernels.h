@@ -157,6 +157,10 @@ cudaError_t launch_bc_sigma(const BcGraph& G, const uint32_t* d, double* sigma, 
 cudaError_t launch_bc_delta(const BcGraph& G, const uint32_t* d, const double* sigma, double* delta, uint32_t n,
                             uint32_t k, const uint8_t* cur, uint8_t* nxt, uint8_t* clr, uint32_t* changed,
                             cudaStream_t st);
+cudaError_t launch_bc_height(const BcGraph& G, const uint32_t* d, uint32_t* hgt, uint32_t n, uint32_t k,
+                             const uint8_t* cur, uint8_t* nxt, uint8_t* clr, uint32_t* changed, cudaStream_t st);
+cudaError_t launch_reach_accum(const uint32_t* d, const uint32_t* hgt, uint32_t* r, uint32_t n, uint32_t k, uint32_t kv,
+                               cudaStream_t st);
 cudaError_t launch_bc_accum(const double* delta, double* cb, uint32_t n, uint32_t k, uint32_t kv, const Sources& src,
                             cudaStream_t st);
 

@@ -504,3 +504,32 @@ def test_betweenness_rejects_zero_lengths():
         with pytest.raises(P.PhastError) as e:
             h.betweenness([0, 1])
         assert e.value.status == -1
+
+
+@pytest.mark.parametrize("name", sorted(BC_GRAPHS))
+@pytest.mark.parametrize("k_batch", (1, 16, 64))
+def test_reach_bit_exact(name, k_batch):
+    """NEXT-3 exact reach (§VII-B, reading R17) over 37 sources with a
+    ragged last batch and a duplicate: integer, bit-exact with the oracle."""
+    g = BC_GRAPHS[name]()
+    src = phastgen.sources(g.n, 37, seed=190 + k_batch, distinct=False)
+    src[5] = src[4]
+    want = oracle.reach(g, src)
+    with P.Phast.from_graph(g) as h:
+        got = h.vertex_to_original(h.reach(src, k_batch=k_batch).cpu().numpy().view(np.uint32))
+    assert np.array_equal(got, want)
+
+
+def test_reach_exact_all_sources_and_max_shards():
+    g = phastgen.grid(12, 10, 1, 6, seed=186)
+    allv = np.arange(g.n, dtype=np.uint32)
+    want = oracle.reach(g, allv)
+    with P.Phast.from_graph(g) as h:
+        got = h.vertex_to_original(h.reach(allv, k_batch=64).cpu().numpy().view(np.uint32))
+        a = h.vertex_to_original(h.reach(allv[:50], k_batch=4).cpu().numpy().view(np.uint32))
+        b = h.vertex_to_original(h.reach(allv[50:], k_batch=32).cpu().numpy().view(np.uint32))
+        # betweenness and reach share scratch: interleaving them must not leak state
+        cb = h.vertex_to_original(h.betweenness(allv[:20], k_batch=16).cpu().numpy())
+    assert np.array_equal(got, want)
+    assert np.array_equal(np.maximum(a, b), want)
+    bc_close(cb, oracle.betweenness(g, allv[:20]))
