@@ -46,7 +46,8 @@ struct phast_ctx {
     size_t bc_elems = 0;
     uint32_t* bc_changed = nullptr;
     uint32_t* bc_changed_host = nullptr;
-    uint8_t* bc_mark = nullptr;         // [3][n] rotating frontier marks
+    uint32_t* bc_q = nullptr;           // [3][n*k]: two item queues + unfinished-input counts
+    uint32_t* bc_qs = nullptr;          // [3] rotating queue sizes
     int bc_len_ok = 0;                  // 0 unknown, 1 all original lengths > 0, -1 not
     // persistent-sweep plans, one per k (built on first use)
     struct Plan {
@@ -164,8 +165,8 @@ void free_device(phast_ctx* h) {
     cudaFree(h->d_in_first); cudaFree(h->d_in_arc);
     h->d_in_first = nullptr; h->d_in_arc = nullptr;
     cudaFree(h->d_out_first); cudaFree(h->d_out_arc); cudaFree(h->bc_sigma); cudaFree(h->bc_delta);
-    cudaFree(h->bc_changed); cudaFreeHost(h->bc_changed_host); cudaFree(h->bc_mark);
-    h->bc_mark = nullptr;
+    cudaFree(h->bc_changed); cudaFreeHost(h->bc_changed_host); cudaFree(h->bc_q); cudaFree(h->bc_qs);
+    h->bc_q = nullptr; h->bc_qs = nullptr;
     h->d_out_first = nullptr; h->d_out_arc = nullptr; h->bc_sigma = h->bc_delta = nullptr;
     h->bc_elems = 0; h->bc_changed = nullptr; h->bc_changed_host = nullptr;
     cudaFree(h->d_upin_first); cudaFree(h->d_upin_arc);
@@ -1040,13 +1041,14 @@ int centrality(phast_ctx* h, const uint32_t* sources, uint64_t count, uint32_t k
     cudaStream_t st = (cudaStream_t)stream;
     const uint32_t n = h->n, k = k_batch;
     const size_t elems = (size_t)n * k;
+    if (elems >= 0xFFFFFFFFull) return PHAST_ERANGE;   // items are 32-bit
     int rc = ensure_scratch(h, elems);
     if (!rc) rc = ensure_in_csr(h);
     if (!rc) rc = ensure_out_csr(h);
     if (rc) return rc;
     constexpr uint32_t R = 32;   // passes between host convergence checks
     if (!h->bc_changed) {
-        if ((rc = dmalloc(&h->bc_changed, R)) || (rc = dmalloc(&h->bc_mark, (size_t)3 * n))) return rc;
+        if ((rc = dmalloc(&h->bc_changed, R)) || (rc = dmalloc(&h->bc_qs, 3))) return rc;
         if (cudaMallocHost(&h->bc_changed_host, R * 4) != cudaSuccess) {
             cudaGetLastError();
             return PHAST_ENOMEM;
@@ -1055,25 +1057,34 @@ int centrality(phast_ctx* h, const uint32_t* sources, uint64_t count, uint32_t k
     if (h->bc_elems < elems) {
         cudaFree(h->bc_sigma);
         cudaFree(h->bc_delta);
+        cudaFree(h->bc_q);
         h->bc_sigma = h->bc_delta = nullptr;
+        h->bc_q = nullptr;
         h->bc_elems = 0;
-        if ((rc = dmalloc(&h->bc_sigma, elems)) || (rc = dmalloc(&h->bc_delta, elems))) return rc;
+        if ((rc = dmalloc(&h->bc_sigma, elems)) || (rc = dmalloc(&h->bc_delta, elems)) ||
+            (rc = dmalloc(&h->bc_q, 3 * elems)))
+            return rc;
         h->bc_elems = elems;
     }
     if (cudaMemsetAsync(out, 0, (size_t)n * (reach ? 4 : 8), st) != cudaSuccess) return PHAST_ECUDA;
-    // pass p reads marks buf[p%3], marks buf[(p+1)%3], zeroes buf[(p+2)%3]; repeat until a
-    // pass changes nothing (<= hop depth of the tight DAG + 1 passes)
+    // Kahn order (kernels.cu): the count kernel fills queue 0; pass p reads queue p%2 with
+    // size qs[p%3], appends to queue (p+1)%2 with qs[(p+1)%3], zeroes qs[(p+2)%3]; stop
+    // after a pass that readied nothing (<= hop depth of the tight DAG + 1 passes)
     const BcGraph G{h->d_in_first, h->d_in_arc, h->d_out_first, h->d_out_arc};
-    auto fixpoint = [&](auto pass) -> int {
-        uint8_t* buf[3] = {h->bc_mark, h->bc_mark + n, h->bc_mark + 2 * (size_t)n};
-        if (cudaMemsetAsync(buf[0], 1, n, st) != cudaSuccess || cudaMemsetAsync(buf[1], 0, n, st) != cudaSuccess)
+    uint32_t* qbuf[2] = {h->bc_q, h->bc_q + elems};
+    uint32_t* cnt = h->bc_q + 2 * elems;
+    auto kahn = [&](int backward, auto pass) -> int {
+        if (cudaMemsetAsync(h->bc_qs, 0, 12, st) != cudaSuccess) return PHAST_ECUDA;
+        if (launch_bc_count(G, h->dist_scratch, n, k, backward, cnt, qbuf[0], h->bc_qs, st) != cudaSuccess)
             return PHAST_ECUDA;
         uint64_t p = 0;
         for (uint64_t it = 0; it <= (uint64_t)n + R; it += R) {
             if (cudaMemsetAsync(h->bc_changed, 0, R * 4, st) != cudaSuccess) return PHAST_ECUDA;
-            for (uint32_t j = 0; j < R; j++, p++)
-                if (pass(buf[p % 3], buf[(p + 1) % 3], buf[(p + 2) % 3], h->bc_changed + j) != cudaSuccess)
-                    return PHAST_ECUDA;
+            for (uint32_t j = 0; j < R; j++, p++) {
+                BcQueue Q{qbuf[p % 2], h->bc_qs + p % 3, qbuf[(p + 1) % 2], h->bc_qs + (p + 1) % 3,
+                          h->bc_qs + (p + 2) % 3, cnt};
+                if (pass(Q, h->bc_changed + j) != cudaSuccess) return PHAST_ECUDA;
+            }
             if (cudaMemcpyAsync(h->bc_changed_host, h->bc_changed, R * 4, cudaMemcpyDeviceToHost, st) != cudaSuccess ||
                 cudaStreamSynchronize(st) != cudaSuccess)
                 return PHAST_ECUDA;
@@ -1090,8 +1101,8 @@ int centrality(phast_ctx* h, const uint32_t* sources, uint64_t count, uint32_t k
         if ((rc = run_query(h, S, k, h->dist_scratch, nullptr, st))) return rc;
         if (reach) {
             if (cudaMemsetAsync(hgt, 0, elems * 4, st) != cudaSuccess) return PHAST_ECUDA;
-            rc = fixpoint([&](const uint8_t* cur, uint8_t* nxt, uint8_t* clr, uint32_t* ch) {
-                return launch_bc_height(G, h->dist_scratch, hgt, n, k, cur, nxt, clr, ch, st);
+            rc = kahn(1, [&](const BcQueue& Q, uint32_t* ch) {
+                return launch_bc_back(G, h->dist_scratch, nullptr, hgt, n, k, 1, Q, ch, st);
             });
             if (rc) return rc;
             if (launch_reach_accum(h->dist_scratch, hgt, (uint32_t*)out, n, k, kv, st) != cudaSuccess)
@@ -1101,12 +1112,12 @@ int centrality(phast_ctx* h, const uint32_t* sources, uint64_t count, uint32_t k
         if (cudaMemsetAsync(h->bc_sigma, 0, elems * 8, st) != cudaSuccess ||
             cudaMemsetAsync(h->bc_delta, 0, elems * 8, st) != cudaSuccess)
             return PHAST_ECUDA;
-        rc = fixpoint([&](const uint8_t* cur, uint8_t* nxt, uint8_t* clr, uint32_t* ch) {
-            return launch_bc_sigma(G, h->dist_scratch, h->bc_sigma, n, k, S, cur, nxt, clr, ch, st);
+        rc = kahn(0, [&](const BcQueue& Q, uint32_t* ch) {
+            return launch_bc_sigma(G, h->dist_scratch, h->bc_sigma, n, k, S, Q, ch, st);
         });
         if (rc) return rc;
-        rc = fixpoint([&](const uint8_t* cur, uint8_t* nxt, uint8_t* clr, uint32_t* ch) {
-            return launch_bc_delta(G, h->dist_scratch, h->bc_sigma, h->bc_delta, n, k, cur, nxt, clr, ch, st);
+        rc = kahn(1, [&](const BcQueue& Q, uint32_t* ch) {
+            return launch_bc_back(G, h->dist_scratch, h->bc_sigma, h->bc_delta, n, k, 0, Q, ch, st);
         });
         if (rc) return rc;
         if (launch_bc_accum(h->bc_delta, (double*)out, n, k, kv, S, st) != cudaSuccess) return PHAST_ECUDA;

@@ -2243,121 +2243,123 @@ __device__ __forceinline__ bool tight(uint32_t du, uint32_t dv, uint32_t l) {
 }
 }  // namespace
 
-// Frontier (a schedule choice, not part of the method): a pass only recomputes the
-// vertices marked in `cur`, one thread per vertex looping over its k trees (the
-// frontier is small after the first pass, so scanning n marks is the pass's fixed
-// cost); a vertex whose value changed in some tree marks its dependents (sigma:
-// out-neighbours; delta and height: in-neighbours) in `nxt`.  Three byte arrays
-// rotate: pass p reads buf[p%3], marks buf[(p+1)%3] and zeroes buf[(p+2)%3] (read by
-// pass p-1, marked by pass p+1).  The first pass has every vertex marked.
-__device__ __forceinline__ void bc_mark(const uint32_t* __restrict__ f, const uint2* __restrict__ a, uint32_t v,
-                                        uint8_t* nxt) {
-    const uint32_t e1 = __ldg(&f[v + 1]);
-    for (uint32_t e = __ldg(&f[v]); e < e1; e++) nxt[__ldg(&a[e]).x] = 1;
+// Schedule (not part of the method): Kahn's topological order of each tree's tight DAG.
+// An item t = v*k + i is computed ONCE, when all its inputs are final: cnt[t] counts the
+// item's unfinished inputs (forward: tight in-arcs; backward: tight out-arcs); a pass
+// computes the items of its queue and, for each dependent whose count drops to zero,
+// appends it to the next queue.  Passes = hop depth of the tight DAG + 1; each pass
+// touches only its frontier.  Queue sizes rotate over three counters: pass p reads
+// qs[p%3], appends with qs[(p+1)%3] and zeroes qs[(p+2)%3].
+__device__ __forceinline__ void bc_push(uint32_t t, uint32_t* q, uint32_t* qs, bool& pushed) {
+    q[atomicAdd(qs, 1u)] = t;
+    pushed = true;
 }
 
-__global__ void __launch_bounds__(256) bc_sigma_kernel(BcGraph G, const uint32_t* __restrict__ d, double* sigma,
-                                                       uint32_t n, uint32_t k, Sources src,
-                                                       const uint8_t* __restrict__ cur, uint8_t* nxt, uint8_t* clr,
-                                                       uint32_t* changed) {
-    bool ch = false;
-    for (uint32_t v = blockIdx.x * blockDim.x + threadIdx.x; v < n; v += gridDim.x * blockDim.x) {
-        clr[v] = 0;
-        if (!cur[v]) continue;
-        const uint32_t e0 = __ldg(&G.in_first[v]), e1 = __ldg(&G.in_first[v + 1]);
-        bool any = false;
-        for (uint32_t i = 0; i < k; i++) {
-            const size_t t = (size_t)v * k + i;
-            const uint32_t dv = __ldg(&d[t]);
-            if (dv == INF) continue;
-            double acc = src.s[i] == v ? 1.0 : 0.0;
-            for (uint32_t e = e0; e < e1; e++) {
+// cnt[t] = number of inputs of item t; items with none start the first queue
+__global__ void __launch_bounds__(256) bc_count_kernel(BcGraph G, const uint32_t* __restrict__ d, uint32_t n,
+                                                       uint32_t k, int backward, uint32_t* cnt, uint32_t* q,
+                                                       uint32_t* qs) {
+    const uint64_t total = (uint64_t)n * k;
+    bool pushed = false;
+    for (uint64_t t = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; t < total;
+         t += (uint64_t)gridDim.x * blockDim.x) {
+        const uint32_t v = (uint32_t)(t / k), i = (uint32_t)(t % k);
+        const uint32_t dv = __ldg(&d[t]);
+        if (dv == INF) continue;
+        uint32_t c = 0;
+        if (!backward) {
+            const uint32_t e1 = __ldg(&G.in_first[v + 1]);
+            for (uint32_t e = __ldg(&G.in_first[v]); e < e1; e++) {
                 const uint2 a = __ldg(&G.in_arc[e]);
-                const size_t u = (size_t)a.x * k + i;
-                if (tight(__ldg(&d[u]), dv, a.y)) acc += sigma[u];
+                c += tight(__ldg(&d[(size_t)a.x * k + i]), dv, a.y);
             }
-            if (acc != sigma[t]) {
-                sigma[t] = acc;
-                any = true;
+        } else {
+            const uint32_t e1 = __ldg(&G.out_first[v + 1]);
+            for (uint32_t e = __ldg(&G.out_first[v]); e < e1; e++) {
+                const uint2 a = __ldg(&G.out_arc[e]);
+                const uint32_t dw = __ldg(&d[(size_t)a.x * k + i]);
+                c += dw != INF && tight(dv, dw, a.y);
             }
         }
-        if (any) {
-            ch = true;
-            bc_mark(G.out_first, G.out_arc, v, nxt);
+        cnt[t] = c;
+        if (c == 0) bc_push((uint32_t)t, q, qs, pushed);
+    }
+    (void)pushed;
+}
+
+// forward pass: sigma(v) = [v = s] + sum over tight (u, v) of sigma(u)
+__global__ void __launch_bounds__(256) bc_sigma_kernel(BcGraph G, const uint32_t* __restrict__ d, double* sigma,
+                                                       uint32_t k, Sources src, BcQueue Q, uint32_t* changed) {
+    const uint32_t size = *Q.qs_in;
+    if (blockIdx.x == 0 && threadIdx.x == 0) *Q.qs_clr = 0;
+    bool pushed = false;
+    for (uint32_t x = blockIdx.x * blockDim.x + threadIdx.x; x < size; x += gridDim.x * blockDim.x) {
+        const uint32_t t = Q.q_in[x];
+        const uint32_t v = t / k, i = t % k;
+        const uint32_t dv = __ldg(&d[t]);
+        double acc = src.s[i] == v ? 1.0 : 0.0;
+        const uint32_t e1 = __ldg(&G.in_first[v + 1]);
+        for (uint32_t e = __ldg(&G.in_first[v]); e < e1; e++) {
+            const uint2 a = __ldg(&G.in_arc[e]);
+            const size_t u = (size_t)a.x * k + i;
+            if (tight(__ldg(&d[u]), dv, a.y)) acc += sigma[u];
+        }
+        sigma[t] = acc;
+        const uint32_t f1 = __ldg(&G.out_first[v + 1]);
+        for (uint32_t e = __ldg(&G.out_first[v]); e < f1; e++) {
+            const uint2 a = __ldg(&G.out_arc[e]);
+            const uint32_t w = a.x * k + i;
+            const uint32_t dw = __ldg(&d[w]);
+            if (dw != INF && tight(dv, dw, a.y) && atomicSub(&Q.cnt[w], 1u) == 1u) bc_push(w, Q.q_out, Q.qs_out, pushed);
         }
     }
-    if (__syncthreads_or(ch) && threadIdx.x == 0) *changed = 1;
+    if (__syncthreads_or(pushed) && threadIdx.x == 0) *changed = 1;
 }
 
-__global__ void __launch_bounds__(256) bc_delta_kernel(BcGraph G, const uint32_t* __restrict__ d,
-                                                       const double* __restrict__ sigma, double* delta, uint32_t n,
-                                                       uint32_t k, const uint8_t* __restrict__ cur, uint8_t* nxt,
-                                                       uint8_t* clr, uint32_t* changed) {
-    bool ch = false;
-    for (uint32_t v = blockIdx.x * blockDim.x + threadIdx.x; v < n; v += gridDim.x * blockDim.x) {
-        clr[v] = 0;
-        if (!cur[v]) continue;
-        const uint32_t e0 = __ldg(&G.out_first[v]), e1 = __ldg(&G.out_first[v + 1]);
-        bool any = false;
-        for (uint32_t i = 0; i < k; i++) {
-            const size_t t = (size_t)v * k + i;
-            const uint32_t dv = __ldg(&d[t]);
-            if (dv == INF) continue;
+// backward pass; mode 0: delta(v) = sum over tight (v, w) of sigma(v)/sigma(w) (1 + delta(w));
+// mode 1 (reach): height h(v) = max over tight (v, w) of l + h(w), stored as uint32 in
+// `val` (l + h(w) <= d(w) + h(w) - d(v) is at most the largest finite label: no wrap)
+__global__ void __launch_bounds__(256) bc_back_kernel(BcGraph G, const uint32_t* __restrict__ d,
+                                                      const double* __restrict__ sigma, void* val, uint32_t k,
+                                                      int mode, BcQueue Q, uint32_t* changed) {
+    const uint32_t size = *Q.qs_in;
+    if (blockIdx.x == 0 && threadIdx.x == 0) *Q.qs_clr = 0;
+    bool pushed = false;
+    double* delta = static_cast<double*>(val);
+    uint32_t* hgt = static_cast<uint32_t*>(val);
+    for (uint32_t x = blockIdx.x * blockDim.x + threadIdx.x; x < size; x += gridDim.x * blockDim.x) {
+        const uint32_t t = Q.q_in[x];
+        const uint32_t v = t / k, i = t % k;
+        const uint32_t dv = __ldg(&d[t]);
+        const uint32_t e1 = __ldg(&G.out_first[v + 1]);
+        if (mode == 0) {
             const double sv = __ldg(&sigma[t]);
             double acc = 0.0;
-            for (uint32_t e = e0; e < e1; e++) {
+            for (uint32_t e = __ldg(&G.out_first[v]); e < e1; e++) {
                 const uint2 a = __ldg(&G.out_arc[e]);
                 const size_t w = (size_t)a.x * k + i;
                 const uint32_t dw = __ldg(&d[w]);
                 if (dw != INF && tight(dv, dw, a.y)) acc += sv / __ldg(&sigma[w]) * (1.0 + delta[w]);
             }
-            if (acc != delta[t]) {
-                delta[t] = acc;
-                any = true;
-            }
-        }
-        if (any) {
-            ch = true;
-            bc_mark(G.in_first, G.in_arc, v, nxt);
-        }
-    }
-    if (__syncthreads_or(ch) && threadIdx.x == 0) *changed = 1;
-}
-
-// reach: height h(v) = max(0, max over tight (v, w) of l + h(w)) (the largest
-// dist(v, t) over the t whose shortest s-t paths pass v).  l + h(w) <= d(w) + h(w) - d(v)
-// is at most the largest finite label, so it never wraps.
-__global__ void __launch_bounds__(256) bc_height_kernel(BcGraph G, const uint32_t* __restrict__ d, uint32_t* hgt,
-                                                        uint32_t n, uint32_t k, const uint8_t* __restrict__ cur,
-                                                        uint8_t* nxt, uint8_t* clr, uint32_t* changed) {
-    bool ch = false;
-    for (uint32_t v = blockIdx.x * blockDim.x + threadIdx.x; v < n; v += gridDim.x * blockDim.x) {
-        clr[v] = 0;
-        if (!cur[v]) continue;
-        const uint32_t e0 = __ldg(&G.out_first[v]), e1 = __ldg(&G.out_first[v + 1]);
-        bool any = false;
-        for (uint32_t i = 0; i < k; i++) {
-            const size_t t = (size_t)v * k + i;
-            const uint32_t dv = __ldg(&d[t]);
-            if (dv == INF) continue;
+            delta[t] = acc;
+        } else {
             uint32_t acc = 0;
-            for (uint32_t e = e0; e < e1; e++) {
+            for (uint32_t e = __ldg(&G.out_first[v]); e < e1; e++) {
                 const uint2 a = __ldg(&G.out_arc[e]);
                 const size_t w = (size_t)a.x * k + i;
                 const uint32_t dw = __ldg(&d[w]);
                 if (dw != INF && tight(dv, dw, a.y)) acc = max(acc, a.y + hgt[w]);
             }
-            if (acc != hgt[t]) {
-                hgt[t] = acc;
-                any = true;
-            }
+            hgt[t] = acc;
         }
-        if (any) {
-            ch = true;
-            bc_mark(G.in_first, G.in_arc, v, nxt);
+        const uint32_t f1 = __ldg(&G.in_first[v + 1]);
+        for (uint32_t e = __ldg(&G.in_first[v]); e < f1; e++) {
+            const uint2 a = __ldg(&G.in_arc[e]);
+            const uint32_t u = a.x * k + i;
+            if (tight(__ldg(&d[u]), dv, a.y) && atomicSub(&Q.cnt[u], 1u) == 1u) bc_push(u, Q.q_out, Q.qs_out, pushed);
         }
     }
-    if (__syncthreads_or(ch) && threadIdx.x == 0) *changed = 1;
+    if (__syncthreads_or(pushed) && threadIdx.x == 0) *changed = 1;
 }
 
 // c_B(v) += sum over the first kv trees i (in order) with sources[i] != v of delta_i(v)
@@ -2390,25 +2392,23 @@ static unsigned bc_blocks(uint64_t items) {
     return (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(b, (uint64_t)num_sms() * 8));
 }
 
+cudaError_t launch_bc_count(const BcGraph& G, const uint32_t* d, uint32_t n, uint32_t k, int backward, uint32_t* cnt,
+                            uint32_t* q, uint32_t* qs, cudaStream_t st) {
+    bc_count_kernel<<<bc_blocks((uint64_t)n * k), 256, 0, st>>>(G, d, n, k, backward, cnt, q, qs);
+    g_launches++;
+    return cudaGetLastError();
+}
+
 cudaError_t launch_bc_sigma(const BcGraph& G, const uint32_t* d, double* sigma, uint32_t n, uint32_t k,
-                            const Sources& src, const uint8_t* cur, uint8_t* nxt, uint8_t* clr, uint32_t* changed,
-                            cudaStream_t st) {
-    bc_sigma_kernel<<<bc_blocks(n), 256, 0, st>>>(G, d, sigma, n, k, src, cur, nxt, clr, changed);
+                            const Sources& src, const BcQueue& Q, uint32_t* changed, cudaStream_t st) {
+    bc_sigma_kernel<<<bc_blocks((uint64_t)n * k), 256, 0, st>>>(G, d, sigma, k, src, Q, changed);
     g_launches++;
     return cudaGetLastError();
 }
 
-cudaError_t launch_bc_delta(const BcGraph& G, const uint32_t* d, const double* sigma, double* delta, uint32_t n,
-                            uint32_t k, const uint8_t* cur, uint8_t* nxt, uint8_t* clr, uint32_t* changed,
-                            cudaStream_t st) {
-    bc_delta_kernel<<<bc_blocks(n), 256, 0, st>>>(G, d, sigma, delta, n, k, cur, nxt, clr, changed);
-    g_launches++;
-    return cudaGetLastError();
-}
-
-cudaError_t launch_bc_height(const BcGraph& G, const uint32_t* d, uint32_t* hgt, uint32_t n, uint32_t k,
-                             const uint8_t* cur, uint8_t* nxt, uint8_t* clr, uint32_t* changed, cudaStream_t st) {
-    bc_height_kernel<<<bc_blocks(n), 256, 0, st>>>(G, d, hgt, n, k, cur, nxt, clr, changed);
+cudaError_t launch_bc_back(const BcGraph& G, const uint32_t* d, const double* sigma, void* val, uint32_t n, uint32_t k,
+                           int mode, const BcQueue& Q, uint32_t* changed, cudaStream_t st) {
+    bc_back_kernel<<<bc_blocks((uint64_t)n * k), 256, 0, st>>>(G, d, sigma, val, k, mode, Q, changed);
     g_launches++;
     return cudaGetLastError();
 }

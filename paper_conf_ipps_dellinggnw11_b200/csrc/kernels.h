@@ -143,22 +143,27 @@ cudaError_t launch_max_reduce(const uint32_t* in, uint32_t count, uint32_t* out,
 
 // NEXT-3 betweenness (kernels.cu): one in-place relaxation pass each; *changed := 1 if
 // the pass wrote anything.  accum: cb[v] += sum_{i < kv, src.s[i] != v} delta[v*k+i].
-// Frontier: a pass recomputes the vertices marked in cur, marks the dependents of changed
-// vertices in nxt and zeroes clr (byte arrays [n]).
+// Passes in Kahn order of each tree's tight DAG (kernels.cu): items t = v*k + i (n*k < 2^32).
 struct BcGraph {
     const uint32_t* in_first;   // original in-arcs by head {tail, len}, internal ids
     const uint2* in_arc;
     const uint32_t* out_first;  // original out-arcs by tail {head, len}
     const uint2* out_arc;
 };
+struct BcQueue {
+    const uint32_t* q_in;       // items of this pass
+    const uint32_t* qs_in;      // their count
+    uint32_t* q_out;            // items that become ready
+    uint32_t* qs_out;
+    uint32_t* qs_clr;           // counter zeroed for the pass after next
+    uint32_t* cnt;              // [n*k] unfinished inputs per item
+};
+cudaError_t launch_bc_count(const BcGraph& G, const uint32_t* d, uint32_t n, uint32_t k, int backward, uint32_t* cnt,
+                            uint32_t* q, uint32_t* qs, cudaStream_t st);
 cudaError_t launch_bc_sigma(const BcGraph& G, const uint32_t* d, double* sigma, uint32_t n, uint32_t k,
-                            const Sources& src, const uint8_t* cur, uint8_t* nxt, uint8_t* clr, uint32_t* changed,
-                            cudaStream_t st);
-cudaError_t launch_bc_delta(const BcGraph& G, const uint32_t* d, const double* sigma, double* delta, uint32_t n,
-                            uint32_t k, const uint8_t* cur, uint8_t* nxt, uint8_t* clr, uint32_t* changed,
-                            cudaStream_t st);
-cudaError_t launch_bc_height(const BcGraph& G, const uint32_t* d, uint32_t* hgt, uint32_t n, uint32_t k,
-                             const uint8_t* cur, uint8_t* nxt, uint8_t* clr, uint32_t* changed, cudaStream_t st);
+                            const Sources& src, const BcQueue& Q, uint32_t* changed, cudaStream_t st);
+cudaError_t launch_bc_back(const BcGraph& G, const uint32_t* d, const double* sigma, void* val, uint32_t n, uint32_t k,
+                           int mode, const BcQueue& Q, uint32_t* changed, cudaStream_t st);
 cudaError_t launch_reach_accum(const uint32_t* d, const uint32_t* hgt, uint32_t* r, uint32_t n, uint32_t k, uint32_t kv,
                                cudaStream_t st);
 cudaError_t launch_bc_accum(const double* delta, double* cb, uint32_t n, uint32_t k, uint32_t kv, const Sources& src,
