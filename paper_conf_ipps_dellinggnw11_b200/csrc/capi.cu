@@ -48,6 +48,8 @@ struct phast_ctx {
     uint32_t* bc_changed_host = nullptr;
     uint32_t* bc_q = nullptr;           // [3][n*k]: two item queues + unfinished-input counts
     uint32_t* bc_qs = nullptr;          // [3] rotating queue sizes
+    cudaStream_t bc_stream = nullptr;   // private stream the pass graphs run on
+    cudaEvent_t bc_ev = nullptr;
     int bc_len_ok = 0;                  // 0 unknown, 1 all original lengths > 0, -1 not
     // persistent-sweep plans, one per k (built on first use)
     struct Plan {
@@ -167,6 +169,9 @@ void free_device(phast_ctx* h) {
     cudaFree(h->d_out_first); cudaFree(h->d_out_arc); cudaFree(h->bc_sigma); cudaFree(h->bc_delta);
     cudaFree(h->bc_changed); cudaFreeHost(h->bc_changed_host); cudaFree(h->bc_q); cudaFree(h->bc_qs);
     h->bc_q = nullptr; h->bc_qs = nullptr;
+    if (h->bc_stream) cudaStreamDestroy(h->bc_stream);
+    if (h->bc_ev) cudaEventDestroy(h->bc_ev);
+    h->bc_stream = nullptr; h->bc_ev = nullptr;
     h->d_out_first = nullptr; h->d_out_arc = nullptr; h->bc_sigma = h->bc_delta = nullptr;
     h->bc_elems = 0; h->bc_changed = nullptr; h->bc_changed_host = nullptr;
     cudaFree(h->d_upin_first); cudaFree(h->d_upin_arc);
@@ -1046,7 +1051,7 @@ int centrality(phast_ctx* h, const uint32_t* sources, uint64_t count, uint32_t k
     if (!rc) rc = ensure_in_csr(h);
     if (!rc) rc = ensure_out_csr(h);
     if (rc) return rc;
-    constexpr uint32_t R = 32;   // passes between host convergence checks
+    constexpr uint32_t R = 30;   // passes per graph launch / host convergence check (multiple of 6)
     if (!h->bc_changed) {
         if ((rc = dmalloc(&h->bc_changed, R)) || (rc = dmalloc(&h->bc_qs, 3))) return rc;
         if (cudaMallocHost(&h->bc_changed_host, R * 4) != cudaSuccess) {
@@ -1073,23 +1078,61 @@ int centrality(phast_ctx* h, const uint32_t* sources, uint64_t count, uint32_t k
     const BcGraph G{h->d_in_first, h->d_in_arc, h->d_out_first, h->d_out_arc};
     uint32_t* qbuf[2] = {h->bc_q, h->bc_q + elems};
     uint32_t* cnt = h->bc_q + 2 * elems;
-    auto kahn = [&](int backward, auto pass) -> int {
-        if (cudaMemsetAsync(h->bc_qs, 0, 12, st) != cudaSuccess) return PHAST_ECUDA;
-        if (launch_bc_count(G, h->dist_scratch, n, k, backward, cnt, qbuf[0], h->bc_qs, st) != cudaSuccess)
-            return PHAST_ECUDA;
-        uint64_t p = 0;
-        for (uint64_t it = 0; it <= (uint64_t)n + R; it += R) {
-            if (cudaMemsetAsync(h->bc_changed, 0, R * 4, st) != cudaSuccess) return PHAST_ECUDA;
-            for (uint32_t j = 0; j < R; j++, p++) {
+    // R passes (+ clearing the change words before, reading them back after) are one CUDA
+    // graph, captured once per call and direction on a private stream (the caller's stream
+    // may be the legacy default stream, which cannot be captured); R is a multiple of 6,
+    // so every chunk starts with the same queue/counter rotation.
+    if ((!h->bc_ev && cudaEventCreateWithFlags(&h->bc_ev, cudaEventDisableTiming) != cudaSuccess) ||
+        (!h->bc_stream && cudaStreamCreateWithFlags(&h->bc_stream, cudaStreamNonBlocking) != cudaSuccess)) {
+        cudaGetLastError();
+        return PHAST_ECUDA;
+    }
+    cudaStream_t gs = h->bc_stream;
+    cudaGraphExec_t execs[3] = {nullptr, nullptr, nullptr};   // sigma, delta, height
+    struct ExecGuard {
+        cudaGraphExec_t* e;
+        ~ExecGuard() {
+            for (int j = 0; j < 3; j++)
+                if (e[j]) cudaGraphExecDestroy(e[j]);
+        }
+    } eg{execs};
+    auto kahn = [&](int which, int backward, auto pass) -> int {
+        if (!execs[which]) {
+            cudaGraph_t graph = nullptr;
+            if (cudaStreamBeginCapture(gs, cudaStreamCaptureModeThreadLocal) != cudaSuccess) return PHAST_ECUDA;
+            bool ok = cudaMemsetAsync(h->bc_changed, 0, R * 4, gs) == cudaSuccess;
+            for (uint32_t p = 0; ok && p < R; p++) {
                 BcQueue Q{qbuf[p % 2], h->bc_qs + p % 3, qbuf[(p + 1) % 2], h->bc_qs + (p + 1) % 3,
                           h->bc_qs + (p + 2) % 3, cnt};
-                if (pass(Q, h->bc_changed + j) != cudaSuccess) return PHAST_ECUDA;
+                ok = pass(Q, h->bc_changed + p, gs) == cudaSuccess;
             }
-            if (cudaMemcpyAsync(h->bc_changed_host, h->bc_changed, R * 4, cudaMemcpyDeviceToHost, st) != cudaSuccess ||
-                cudaStreamSynchronize(st) != cudaSuccess)
+            ok = ok && cudaMemcpyAsync(h->bc_changed_host, h->bc_changed, R * 4, cudaMemcpyDeviceToHost, gs) ==
+                           cudaSuccess;
+            add_launches(-(int64_t)R);   // captured, not launched
+            if (cudaStreamEndCapture(gs, &graph) != cudaSuccess || !ok) {
+                cudaGetLastError();
+                if (graph) cudaGraphDestroy(graph);
                 return PHAST_ECUDA;
+            }
+            cudaError_t ie = cudaGraphInstantiate(&execs[which], graph, 0);
+            cudaGraphDestroy(graph);
+            if (ie != cudaSuccess) {
+                cudaGetLastError();
+                execs[which] = nullptr;
+                return PHAST_ECUDA;
+            }
+        }
+        // the count kernel and the chunks run on gs after everything queued on st so far
+        if (cudaEventRecord(h->bc_ev, st) != cudaSuccess || cudaStreamWaitEvent(gs, h->bc_ev, 0) != cudaSuccess ||
+            cudaMemsetAsync(h->bc_qs, 0, 12, gs) != cudaSuccess ||
+            launch_bc_count(G, h->dist_scratch, n, k, backward, cnt, qbuf[0], h->bc_qs, gs) != cudaSuccess)
+            return PHAST_ECUDA;
+        for (uint64_t it = 0; it <= (uint64_t)n + R; it += R) {
+            if (cudaGraphLaunch(execs[which], gs) != cudaSuccess || cudaStreamSynchronize(gs) != cudaSuccess)
+                return PHAST_ECUDA;
+            add_launches(R);
             for (uint32_t j = 0; j < R; j++)
-                if (h->bc_changed_host[j] == 0) return PHAST_OK;
+                if (h->bc_changed_host[j] == 0) return PHAST_OK;   // st waits for nothing: gs is idle
         }
         return PHAST_EINTERNAL;   // cannot happen with lengths > 0
     };
@@ -1101,8 +1144,8 @@ int centrality(phast_ctx* h, const uint32_t* sources, uint64_t count, uint32_t k
         if ((rc = run_query(h, S, k, h->dist_scratch, nullptr, st))) return rc;
         if (reach) {
             if (cudaMemsetAsync(hgt, 0, elems * 4, st) != cudaSuccess) return PHAST_ECUDA;
-            rc = kahn(1, [&](const BcQueue& Q, uint32_t* ch) {
-                return launch_bc_back(G, h->dist_scratch, nullptr, hgt, n, k, 1, Q, ch, st);
+            rc = kahn(2, 1, [&](const BcQueue& Q, uint32_t* ch, cudaStream_t s2) {
+                return launch_bc_back(G, h->dist_scratch, nullptr, hgt, n, k, 1, Q, ch, s2);
             });
             if (rc) return rc;
             if (launch_reach_accum(h->dist_scratch, hgt, (uint32_t*)out, n, k, kv, st) != cudaSuccess)
@@ -1112,12 +1155,12 @@ int centrality(phast_ctx* h, const uint32_t* sources, uint64_t count, uint32_t k
         if (cudaMemsetAsync(h->bc_sigma, 0, elems * 8, st) != cudaSuccess ||
             cudaMemsetAsync(h->bc_delta, 0, elems * 8, st) != cudaSuccess)
             return PHAST_ECUDA;
-        rc = kahn(0, [&](const BcQueue& Q, uint32_t* ch) {
-            return launch_bc_sigma(G, h->dist_scratch, h->bc_sigma, n, k, S, Q, ch, st);
+        rc = kahn(0, 0, [&](const BcQueue& Q, uint32_t* ch, cudaStream_t s2) {
+            return launch_bc_sigma(G, h->dist_scratch, h->bc_sigma, n, k, Q, ch, s2);
         });
         if (rc) return rc;
-        rc = kahn(1, [&](const BcQueue& Q, uint32_t* ch) {
-            return launch_bc_back(G, h->dist_scratch, h->bc_sigma, h->bc_delta, n, k, 0, Q, ch, st);
+        rc = kahn(1, 1, [&](const BcQueue& Q, uint32_t* ch, cudaStream_t s2) {
+            return launch_bc_back(G, h->dist_scratch, h->bc_sigma, h->bc_delta, n, k, 0, Q, ch, s2);
         });
         if (rc) return rc;
         if (launch_bc_accum(h->bc_delta, (double*)out, n, k, kv, S, st) != cudaSuccess) return PHAST_ECUDA;

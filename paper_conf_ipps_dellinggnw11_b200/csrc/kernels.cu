@@ -34,6 +34,7 @@ static std::atomic<uint64_t> g_launches{0};
 // bytes, 0 = off (set_l2_persist)
 static size_t g_persist_bytes = 0;
 uint64_t launches() { return g_launches.load(); }
+void add_launches(int64_t d) { g_launches += (uint64_t)d; }
 
 int set_l2_persist(size_t bytes) {
     if (bytes) {
@@ -2287,9 +2288,11 @@ __global__ void __launch_bounds__(256) bc_count_kernel(BcGraph G, const uint32_t
     (void)pushed;
 }
 
-// forward pass: sigma(v) = [v = s] + sum over tight (u, v) of sigma(u)
+// forward pass: sigma(v) = [v = s] + sum over tight (u, v) of sigma(u).  With lengths > 0
+// the source is the only finite item without a tight in-arc, so [v = s] is "no tight
+// in-arc" (no source list in the parameters: the passes are graph-captured once per call)
 __global__ void __launch_bounds__(256) bc_sigma_kernel(BcGraph G, const uint32_t* __restrict__ d, double* sigma,
-                                                       uint32_t k, Sources src, BcQueue Q, uint32_t* changed) {
+                                                       uint32_t k, BcQueue Q, uint32_t* changed) {
     const uint32_t size = *Q.qs_in;
     if (blockIdx.x == 0 && threadIdx.x == 0) *Q.qs_clr = 0;
     bool pushed = false;
@@ -2297,14 +2300,18 @@ __global__ void __launch_bounds__(256) bc_sigma_kernel(BcGraph G, const uint32_t
         const uint32_t t = Q.q_in[x];
         const uint32_t v = t / k, i = t % k;
         const uint32_t dv = __ldg(&d[t]);
-        double acc = src.s[i] == v ? 1.0 : 0.0;
+        double acc = 0.0;
+        bool any = false;
         const uint32_t e1 = __ldg(&G.in_first[v + 1]);
         for (uint32_t e = __ldg(&G.in_first[v]); e < e1; e++) {
             const uint2 a = __ldg(&G.in_arc[e]);
             const size_t u = (size_t)a.x * k + i;
-            if (tight(__ldg(&d[u]), dv, a.y)) acc += sigma[u];
+            if (tight(__ldg(&d[u]), dv, a.y)) {
+                acc += sigma[u];
+                any = true;
+            }
         }
-        sigma[t] = acc;
+        sigma[t] = any ? acc : 1.0;
         const uint32_t f1 = __ldg(&G.out_first[v + 1]);
         for (uint32_t e = __ldg(&G.out_first[v]); e < f1; e++) {
             const uint2 a = __ldg(&G.out_arc[e]);
@@ -2399,16 +2406,19 @@ cudaError_t launch_bc_count(const BcGraph& G, const uint32_t* d, uint32_t n, uin
     return cudaGetLastError();
 }
 
+// the passes touch only their queue: a small fixed grid (queue sizes are read on the device)
+static unsigned bc_pass_blocks(uint64_t items) { return std::min<unsigned>(bc_blocks(items), (unsigned)num_sms() * 2); }
+
 cudaError_t launch_bc_sigma(const BcGraph& G, const uint32_t* d, double* sigma, uint32_t n, uint32_t k,
-                            const Sources& src, const BcQueue& Q, uint32_t* changed, cudaStream_t st) {
-    bc_sigma_kernel<<<bc_blocks((uint64_t)n * k), 256, 0, st>>>(G, d, sigma, k, src, Q, changed);
+                            const BcQueue& Q, uint32_t* changed, cudaStream_t st) {
+    bc_sigma_kernel<<<bc_pass_blocks((uint64_t)n * k), 256, 0, st>>>(G, d, sigma, k, Q, changed);
     g_launches++;
     return cudaGetLastError();
 }
 
 cudaError_t launch_bc_back(const BcGraph& G, const uint32_t* d, const double* sigma, void* val, uint32_t n, uint32_t k,
                            int mode, const BcQueue& Q, uint32_t* changed, cudaStream_t st) {
-    bc_back_kernel<<<bc_blocks((uint64_t)n * k), 256, 0, st>>>(G, d, sigma, val, k, mode, Q, changed);
+    bc_back_kernel<<<bc_pass_blocks((uint64_t)n * k), 256, 0, st>>>(G, d, sigma, val, k, mode, Q, changed);
     g_launches++;
     return cudaGetLastError();
 }

@@ -161,7 +161,7 @@ struct BcQueue {
 cudaError_t launch_bc_count(const BcGraph& G, const uint32_t* d, uint32_t n, uint32_t k, int backward, uint32_t* cnt,
                             uint32_t* q, uint32_t* qs, cudaStream_t st);
 cudaError_t launch_bc_sigma(const BcGraph& G, const uint32_t* d, double* sigma, uint32_t n, uint32_t k,
-                            const Sources& src, const BcQueue& Q, uint32_t* changed, cudaStream_t st);
+                            const BcQueue& Q, uint32_t* changed, cudaStream_t st);
 cudaError_t launch_bc_back(const BcGraph& G, const uint32_t* d, const double* sigma, void* val, uint32_t n, uint32_t k,
                            int mode, const BcQueue& Q, uint32_t* changed, cudaStream_t st);
 cudaError_t launch_reach_accum(const uint32_t* d, const uint32_t* hgt, uint32_t* r, uint32_t n, uint32_t k, uint32_t kv,
@@ -170,6 +170,8 @@ cudaError_t launch_bc_accum(const double* delta, double* cb, uint32_t n, uint32_
                             cudaStream_t st);
 
 uint64_t launches();
+// kernels replayed from a CUDA graph (counted at launch, not at capture)
+void add_launches(int64_t d);
 int num_sms();
 // L2 persistence for the sweep launches: the first `bytes` of each label array (the
 // top levels' rows) are accessed with the persisting property; sets the device's
