@@ -41,7 +41,7 @@ def main():
     import torch.distributed as dist
 
     import paper_conf_ipps_dellinggnw11_b200 as P
-    from paper_conf_ipps_dellinggnw11_b200.parallel import shard, share_hierarchy
+    from paper_conf_ipps_dellinggnw11_b200.parallel import combine_centrality, shard, share_hierarchy
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
@@ -72,7 +72,7 @@ def main():
     ms = t0.elapsed_time(t1)
     launches = P.launch_count() - launches0
     if world > 1:
-        dist.all_reduce(cb, op=dist.ReduceOp.MAX if args.reach else dist.ReduceOp.SUM)
+        combine_centrality(cb, args.reach)
         tt = torch.tensor([ms], dtype=torch.float64, device="cuda")
         dist.all_reduce(tt, op=dist.ReduceOp.MAX)
         ms = float(tt.item())

@@ -62,3 +62,21 @@ def diameter_distributed(h, sources, k_batch: int = 64) -> int:
         h.sync()
         local = int(out.cpu().numpy().view(np.uint32)[0])
     return allreduce_max_u32(local, device="cuda")
+
+
+def combine_centrality(t, reach: bool):
+    """Combine per-rank partial centrality over disjoint source shards, in place:
+    betweenness (fp64) adds up over sources, reach (uint32 bits in int32, values
+    < 2^31 never assumed) is a max -- carried as int64 so the unsigned order holds
+    (R16/R17).  No-op without an initialised process group."""
+    import torch
+    import torch.distributed as dist
+    if not (dist.is_available() and dist.is_initialized()) or dist.get_world_size() == 1:
+        return t
+    if not reach:
+        dist.all_reduce(t, op=dist.ReduceOp.SUM)
+        return t
+    wide = (t.to(torch.int64) & 0xFFFFFFFF)
+    dist.all_reduce(wide, op=dist.ReduceOp.MAX)
+    t.copy_(wide.to(torch.int32))
+    return t

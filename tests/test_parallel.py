@@ -72,3 +72,48 @@ def test_two_rank_gloo_sharing_and_allreduce(tmp_path):
     assert all(r[5] == 0xFFFFFFF0 for r in res)
     assert all(r[6] == 1007 for r in res)
     assert not os.path.exists(tmp_path / "h.phast")               # rank 0 cleaned up
+
+
+def _centrality_worker(rank, world, port, q):
+    import torch
+    import torch.distributed as dist
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        import oracle
+        import phastgen
+        from paper_conf_ipps_dellinggnw11_b200.parallel import combine_centrality, shard
+        g = phastgen.grid(9, 7, 1, 5, seed=12)
+        lo, hi = shard(g.n, world, rank)
+        src = np.arange(lo, hi, dtype=np.uint32)
+        cb = torch.from_numpy(oracle.betweenness(g, src))
+        r = torch.from_numpy(oracle.reach(g, src).view(np.int32).copy())
+        combine_centrality(cb, reach=False)
+        combine_centrality(r, reach=True)
+        q.put((rank, cb.numpy(), r.numpy().view(np.uint32)))
+    finally:
+        dist.destroy_process_group()
+
+
+def test_two_rank_centrality_shards_combine():
+    """Betweenness / reach over disjoint source shards (NEXT-3): SUM and MAX over the
+    ranks give the all-sources values (the combine bench_betweenness.py uses)."""
+    import oracle
+    import phastgen
+    world = 2
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_centrality_worker, args=(r, world, port, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    for p in procs:
+        p.join(timeout=300)
+        assert p.exitcode == 0
+    res = sorted((q.get(timeout=10) for _ in range(world)), key=lambda x: x[0])
+    g = phastgen.grid(9, 7, 1, 5, seed=12)
+    allv = np.arange(g.n)
+    for _, cb, r in res:
+        np.testing.assert_allclose(cb, oracle.betweenness(g, allv), rtol=1e-12)
+        assert np.array_equal(r, oracle.reach(g, allv))
