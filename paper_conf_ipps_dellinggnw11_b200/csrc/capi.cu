@@ -1096,7 +1096,25 @@ int centrality(phast_ctx* h, const uint32_t* sources, uint64_t count, uint32_t k
                 if (e[j]) cudaGraphExecDestroy(e[j]);
         }
     } eg{execs};
+    // default: graph-captured chunks of R pass launches; PHAST_BC_PERSIST=1 runs every pass
+    // of a direction in ONE cooperative launch with a grid barrier between passes
+    // (measured slower: the passes are bound by their dependent-load
+    // chains, not by launches)
+    const char* pe = std::getenv("PHAST_BC_PERSIST");
+    const bool persist = pe && pe[0] == '1';
     auto kahn = [&](int which, int backward, auto pass) -> int {
+        if (persist) {
+            if (cudaMemsetAsync(h->bc_qs, 0, 12, st) != cudaSuccess ||
+                launch_bc_count(G, h->dist_scratch, n, k, backward, cnt, qbuf[0], h->bc_qs, st) != cudaSuccess)
+                return PHAST_ECUDA;
+            void* val = which == 0 ? (void*)h->bc_sigma : (void*)h->bc_delta;
+            if (launch_bc_persistent(G, h->dist_scratch, h->bc_sigma, val, k, which, qbuf[0], qbuf[1], h->bc_qs, cnt,
+                                     n + 2, h->g.err, st) != cudaSuccess) {
+                cudaGetLastError();
+                return PHAST_ECUDA;
+            }
+            return PHAST_OK;
+        }
         if (!execs[which]) {
             cudaGraph_t graph = nullptr;
             if (cudaStreamBeginCapture(gs, cudaStreamCaptureModeThreadLocal) != cudaSuccess) return PHAST_ECUDA;

@@ -24,6 +24,7 @@
 #include <vector>
 #include <cstdlib>
 
+#include <cooperative_groups.h>
 #include "kernels.h"
 
 namespace phast {
@@ -2369,6 +2370,90 @@ __global__ void __launch_bounds__(256) bc_back_kernel(BcGraph G, const uint32_t*
     if (__syncthreads_or(pushed) && threadIdx.x == 0) *changed = 1;
 }
 
+// Persistent form of the Kahn passes: ONE cooperative launch runs every pass of one
+// direction, moving to the next pass on a grid-wide barrier (no launch or host check
+// per pass).  Values written in earlier passes by other SMs are read with ld.global.cg
+// (L2, not the incoherent L1); the queue size of a pass is final at the barrier before
+// it, so every thread sees the same size and leaves the loop together.
+// mode 0: sigma (forward); 1: delta (backward); 2: height (backward).
+__global__ void __launch_bounds__(256) bc_kahn_persistent_kernel(BcGraph G, const uint32_t* __restrict__ d,
+                                                                 double* sigma, void* val, uint32_t k, int mode,
+                                                                 uint32_t* q0, uint32_t* q1, uint32_t* qs,
+                                                                 uint32_t* cnt, uint32_t max_passes, uint32_t* err) {
+    namespace cg = cooperative_groups;
+    cg::grid_group grid = cg::this_grid();
+    double* delta = static_cast<double*>(val);
+    uint32_t* hgt = static_cast<uint32_t*>(val);
+    const uint32_t gtid = blockIdx.x * blockDim.x + threadIdx.x, gthreads = gridDim.x * blockDim.x;
+    for (uint32_t p = 0;; p++) {
+        const uint32_t* q_in = (p & 1) ? q1 : q0;
+        uint32_t* q_out = (p & 1) ? q0 : q1;
+        uint32_t* qs_out = qs + (p + 1) % 3;
+        const uint32_t size = __ldcg(qs + p % 3);
+        if (size == 0) break;
+        if (p >= max_passes) {   // cannot happen with lengths > 0
+            if (gtid == 0) atomicOr(err, 2u);
+            break;
+        }
+        if (gtid == 0) qs[(p + 2) % 3] = 0;
+        for (uint32_t x = gtid; x < size; x += gthreads) {
+            const uint32_t t = __ldcg(q_in + x);
+            const uint32_t v = t / k, i = t % k;
+            const uint32_t dv = __ldg(&d[t]);
+            if (mode == 0) {
+                double acc = 0.0;
+                bool any = false;
+                const uint32_t e1 = __ldg(&G.in_first[v + 1]);
+                for (uint32_t e = __ldg(&G.in_first[v]); e < e1; e++) {
+                    const uint2 a = __ldg(&G.in_arc[e]);
+                    const size_t u = (size_t)a.x * k + i;
+                    if (tight(__ldg(&d[u]), dv, a.y)) {
+                        acc += __ldcg(sigma + u);
+                        any = true;
+                    }
+                }
+                sigma[t] = any ? acc : 1.0;
+                const uint32_t f1 = __ldg(&G.out_first[v + 1]);
+                for (uint32_t e = __ldg(&G.out_first[v]); e < f1; e++) {
+                    const uint2 a = __ldg(&G.out_arc[e]);
+                    const uint32_t w = a.x * k + i;
+                    const uint32_t dw = __ldg(&d[w]);
+                    if (dw != INF && tight(dv, dw, a.y) && atomicSub(&cnt[w], 1u) == 1u) q_out[atomicAdd(qs_out, 1u)] = w;
+                }
+            } else {
+                const uint32_t e1 = __ldg(&G.out_first[v + 1]);
+                if (mode == 1) {
+                    const double sv = __ldg(&sigma[t]);
+                    double acc = 0.0;
+                    for (uint32_t e = __ldg(&G.out_first[v]); e < e1; e++) {
+                        const uint2 a = __ldg(&G.out_arc[e]);
+                        const size_t w = (size_t)a.x * k + i;
+                        const uint32_t dw = __ldg(&d[w]);
+                        if (dw != INF && tight(dv, dw, a.y)) acc += sv / __ldg(&sigma[w]) * (1.0 + __ldcg(delta + w));
+                    }
+                    delta[t] = acc;
+                } else {
+                    uint32_t acc = 0;
+                    for (uint32_t e = __ldg(&G.out_first[v]); e < e1; e++) {
+                        const uint2 a = __ldg(&G.out_arc[e]);
+                        const size_t w = (size_t)a.x * k + i;
+                        const uint32_t dw = __ldg(&d[w]);
+                        if (dw != INF && tight(dv, dw, a.y)) acc = max(acc, a.y + __ldcg(hgt + w));
+                    }
+                    hgt[t] = acc;
+                }
+                const uint32_t f1 = __ldg(&G.in_first[v + 1]);
+                for (uint32_t e = __ldg(&G.in_first[v]); e < f1; e++) {
+                    const uint2 a = __ldg(&G.in_arc[e]);
+                    const uint32_t u = a.x * k + i;
+                    if (tight(__ldg(&d[u]), dv, a.y) && atomicSub(&cnt[u], 1u) == 1u) q_out[atomicAdd(qs_out, 1u)] = u;
+                }
+            }
+        }
+        grid.sync();
+    }
+}
+
 // c_B(v) += sum over the first kv trees i (in order) with sources[i] != v of delta_i(v)
 __global__ void __launch_bounds__(256) bc_accum_kernel(const double* __restrict__ delta, double* __restrict__ cb,
                                                        uint32_t n, uint32_t k, uint32_t kv, Sources src) {
@@ -2421,6 +2506,24 @@ cudaError_t launch_bc_back(const BcGraph& G, const uint32_t* d, const double* si
     bc_back_kernel<<<bc_pass_blocks((uint64_t)n * k), 256, 0, st>>>(G, d, sigma, val, k, mode, Q, changed);
     g_launches++;
     return cudaGetLastError();
+}
+
+cudaError_t launch_bc_persistent(const BcGraph& G, const uint32_t* d, double* sigma, void* val, uint32_t k, int mode,
+                                 uint32_t* q0, uint32_t* q1, uint32_t* qs, uint32_t* cnt, uint32_t max_passes,
+                                 uint32_t* err, cudaStream_t st) {
+    static int per_sm = -1;
+    if (per_sm < 0) {
+        int b = 0;
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, bc_kahn_persistent_kernel, 256, 0) != cudaSuccess) b = 0;
+        per_sm = std::min(b, 2);
+    }
+    if (per_sm <= 0) return cudaErrorCooperativeLaunchTooLarge;
+    void* args[] = {(void*)&G, (void*)&d, (void*)&sigma, (void*)&val, (void*)&k, (void*)&mode, (void*)&q0,
+                    (void*)&q1, (void*)&qs, (void*)&cnt, (void*)&max_passes, (void*)&err};
+    cudaError_t e = cudaLaunchCooperativeKernel((const void*)bc_kahn_persistent_kernel, dim3(num_sms() * per_sm),
+                                                dim3(256), args, 0, st);
+    g_launches++;
+    return e;
 }
 
 cudaError_t launch_reach_accum(const uint32_t* d, const uint32_t* hgt, uint32_t* r, uint32_t n, uint32_t k, uint32_t kv,

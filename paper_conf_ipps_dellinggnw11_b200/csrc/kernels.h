@@ -164,6 +164,11 @@ cudaError_t launch_bc_sigma(const BcGraph& G, const uint32_t* d, double* sigma, 
                             const BcQueue& Q, uint32_t* changed, cudaStream_t st);
 cudaError_t launch_bc_back(const BcGraph& G, const uint32_t* d, const double* sigma, void* val, uint32_t n, uint32_t k,
                            int mode, const BcQueue& Q, uint32_t* changed, cudaStream_t st);
+// all passes of one direction in one cooperative launch (mode 0 sigma, 1 delta, 2 height);
+// queue 0 / qs[0] hold the count kernel's items; err bit 1 if max_passes is exceeded
+cudaError_t launch_bc_persistent(const BcGraph& G, const uint32_t* d, double* sigma, void* val, uint32_t k, int mode,
+                                 uint32_t* q0, uint32_t* q1, uint32_t* qs, uint32_t* cnt, uint32_t max_passes,
+                                 uint32_t* err, cudaStream_t st);
 cudaError_t launch_reach_accum(const uint32_t* d, const uint32_t* hgt, uint32_t* r, uint32_t n, uint32_t k, uint32_t kv,
                                cudaStream_t st);
 cudaError_t launch_bc_accum(const double* delta, double* cb, uint32_t n, uint32_t k, uint32_t kv, const Sources& src,

@@ -533,3 +533,17 @@ def test_reach_exact_all_sources_and_max_shards():
     assert np.array_equal(got, want)
     assert np.array_equal(np.maximum(a, b), want)
     bc_close(cb, oracle.betweenness(g, allv[:20]))
+
+
+@pytest.mark.parametrize("persist", ("0", "1"))
+def test_centrality_both_pass_drivers(monkeypatch, persist):
+    """The graph-captured pass chunks (default) and the persistent cooperative Kahn
+    kernel (PHAST_BC_PERSIST=1) give the oracle's values."""
+    monkeypatch.setenv("PHAST_BC_PERSIST", persist)
+    g = BC_GRAPHS["unit_grid"]()
+    src = phastgen.sources(g.n, 21, seed=77)
+    with P.Phast.from_graph(g) as h:
+        cb = h.vertex_to_original(h.betweenness(src, k_batch=8).cpu().numpy())
+        r = h.vertex_to_original(h.reach(src, k_batch=16).cpu().numpy().view(np.uint32))
+    bc_close(cb, oracle.betweenness(g, src))
+    assert np.array_equal(r, oracle.reach(g, src))
