@@ -1,22 +1,30 @@
 #!/usr/bin/env python
 """bench.py -- PHAST multi-tree sweep throughput on B200 (driver contract).
 
-  python bench.py [--gpus N] [--steps K] [--warmup W] [--config C3] [--k 64] [--impl phast|reference]
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--config C3] [--k 64]
+                  [--inflight S] [--total-sources T] [--steady] [--impl phast|reference]
 
 A step is one pass of the whole hot path (source intake,
 upward CH searches, seeding, the level-ordered downward sweep, result left in HBM)
 over one batch of k synthetic sources on the Europe-scale synthetic road graph
 (BASELINE.json metric: "SSSP trees/sec on 18M-vertex road-like graph"; configs[2]).
-value = trees/s over all ranks (weak scaling: every rank sweeps its own sources on
-its own replica of the graph; no collective on the data path).  Rank 0 prints ONE
-JSON line.  `--impl reference` times the oracle (binary-heap Dijkstra on the
-original graph, oracle/) on the host cores instead -- the reference arm of this tier.
+Batches are issued round robin on S streams (`--inflight`, the library keeps
+PHAST_SLOTS queries in flight), each stream with its own label buffer.
+value = trees/s over all ranks.  Weak scaling (default): every rank sweeps `--steps`
+batches of its own sources on its own replica of the graph; strong scaling
+(`--total-sources T`, BASELINE configs[3] "8192 sources sharded at 1/2/4/8 B200"):
+T sources split into contiguous per-rank shards.  No collective on the data path.
+`--gpus N` without a torchrun environment re-launches itself under
+torch.distributed.run with N ranks (one per GPU, NCCL).  Rank 0 prints ONE JSON line.
+`--impl reference` times the oracle (binary-heap Dijkstra on the original graph,
+oracle/) on the host cores instead -- the reference arm of this tier.
 """
 from __future__ import annotations
 
 import argparse
 import json
 import os
+import socket
 import statistics
 import subprocess
 import sys
@@ -35,6 +43,7 @@ THROTTLE_BITS = {0x1: "gpu_idle", 0x2: "applications_clocks_setting", 0x4: "sw_p
                  0x8: "hw_slowdown", 0x10: "sync_boost", 0x20: "sw_thermal_slowdown",
                  0x40: "hw_thermal_slowdown", 0x80: "hw_power_brake_slowdown",
                  0x100: "display_clock_setting"}
+L2_BYTES = 126 << 20
 
 
 def log(*a):
@@ -123,6 +132,44 @@ def oracle_sample(g, cfg, threads, count):
     return count / dt, dt, src
 
 
+def free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def relaunch_distributed(args):
+    """`--gpus N` (N > 1) outside torchrun: run this script under
+    torch.distributed.run with N ranks on this node, NCCL communicator init logged."""
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+           "--master-addr", "127.0.0.1", f"--master-port={free_port()}", os.path.abspath(__file__)] + sys.argv[1:]
+    env = dict(os.environ)
+    env.setdefault("NCCL_DEBUG", "INFO")
+    env.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
+    log("[bench] relaunch: " + " ".join(cmd))
+    return subprocess.call(cmd, env=env)
+
+
+def rank_batches(n, cfg, k, world, rank, steps, warmup, total_sources=0):
+    """This rank's batches of k sources: (warm-up batches, timed batches, trees counted).
+    Weak scaling: `steps` batches of its own seeded sources per rank.  Strong scaling
+    (total_sources = T): one seeded list of T sources split into contiguous per-rank
+    shards (parallel.shard); a ragged last batch is padded with duplicates of its first
+    source, whose extra trees are not counted."""
+    from paper_conf_ipps_dellinggnw11_b200.parallel import shard
+    warm = source_table(n, cfg, rank + 7919, warmup, k)
+    if not total_sources:
+        return warm, source_table(n, cfg, rank, steps, k), steps * k
+    lo, hi = shard(total_sources, world, rank)
+    mine = phastgen.sources(n, total_sources, seed=cfg["src_seed"] * 7919 + 1)[lo:hi]
+    timed = [mine[i:i + k] for i in range(0, mine.size, k)]
+    timed = [b if b.size == k else np.concatenate([b, np.repeat(b[:1], k - b.size)]).astype(np.uint32)
+             for b in timed]
+    return warm, timed, int(hi - lo)
+
+
 def run_reference(args):
     """Reference arm: the oracle as it stands, on the host cores, same metric/config."""
     rank = int(os.environ.get("RANK", "0"))
@@ -142,7 +189,8 @@ def run_reference(args):
     line = {
         "impl": "reference", "metric": METRIC, "value": value, "unit": "trees/s", "n_gpus": args.gpus,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": dt / args.steps * 1e3,
-        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
+        "higher_is_better": True, "scaling": "strong" if args.total_sources else "weak", "vs_baseline": None,
+        "dtype": "u32", "data": "synthetic",
         "config": {"workload": f"{args.config}: {cfg['desc']}", "n": g.n, "m": g.m, "sources_per_step": per_step},
         "cpu_baseline": {"value": value, "unit": "trees/s", "cores": threads, "kind": "oracle", "sample": sample},
         "e2e": {"value": value, "unit": "trees/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
@@ -158,20 +206,27 @@ def main():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--config", default="C3")
     ap.add_argument("--k", type=int, default=64)
+    ap.add_argument("--inflight", type=int, default=2, help="streams with a batch in flight (1..4)")
+    ap.add_argument("--total-sources", type=int, default=0,
+                    help="strong scaling: this many sources split over the ranks (C4: 8192); steps is derived")
+    ap.add_argument("--steady", action="store_true",
+                    help="small configs: no L2 flush between steps (steady state; label buffers rotate)")
     ap.add_argument("--impl", default="phast", choices=["phast", "reference"])
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-probes", action="store_true")
     ap.add_argument("--cache", default="", help="hierarchy file to reuse/create (optional)")
-    ap.add_argument("--layout", default="levels-bfs", choices=["wavefront", "levels", "levels-bfs", "diagonal"],
-                    help="vertex order: wavefront, the paper's level layout (DFS within a level), or level "
-                         "layout with BFS order within a level (default)")
-    ap.add_argument("--delta", type=int, default=0, help="wavefront skew (0 = library default)")
+    ap.add_argument("--layout", default="levels-bfs", choices=["levels", "levels-bfs"],
+                    help="vertex order: the paper's level layout (DFS within a level) or BFS within a level")
     ap.add_argument("--parents", action="store_true",
                     help="also time the parent-pointer pass (phast_parents, NEXT-1) on the last batch")
     args = ap.parse_args()
     args.warmup = max(3, args.warmup)
+    args.inflight = max(1, min(4, args.inflight))
     if args.impl == "reference":
         return run_reference(args)
+    if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        return relaunch_distributed(args)
 
     import torch
     import torch.distributed as dist
@@ -181,6 +236,8 @@ def main():
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world != args.gpus:
+        log(f"[bench] WARNING: --gpus {args.gpus} but WORLD_SIZE={world}; using {world} rank(s)")
     torch.cuda.set_device(local)
     if world > 1:
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
@@ -189,10 +246,21 @@ def main():
         if world > 1:
             dist.barrier()
 
-    g, cfg = build_graph(args.config)
+    def max_over_ranks(x):
+        if world == 1:
+            return x
+        tt = torch.tensor([x], dtype=torch.float64, device="cuda")
+        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+        return float(tt.item())
+
+    cfg = phastgen.CONFIGS[args.config]
     k = args.k
-    bopts = dict(layout=args.layout, delta=args.delta)
-    # hierarchy: rank 0 builds (host CH, not the timed target) and shares it via a file
+    bopts = dict(layout=args.layout)
+    # hierarchy: rank 0 generates the graph and builds (host CH, not the timed target),
+    # the other ranks load it from a file (graph replicated per GPU)
+    g = None
+    if rank == 0:
+        g, _ = build_graph(args.config)
     path = args.cache or f"/tmp/phast_{args.config}_{os.getpid() if world == 1 else 'dist'}.phast"
     if world > 1:
         from paper_conf_ipps_dellinggnw11_b200.parallel import share_hierarchy
@@ -207,94 +275,154 @@ def main():
         log(f"[bench] CH build {time.time() - t:.1f}s")
         if args.cache:
             h.save(args.cache)
+    n = h.n
     info = h.info()
     lsz = h.level_sizes()
-    log(f"[bench] n={info.n} m={info.m} m_up={info.m_up} m_down={info.m_down} n_tail={info.n_tail} "
-        f"levels={info.levels} L0={lsz[0] / info.n:.3f} CH={info.build_seconds:.1f}s")
+    sched = h.schedule(k)
+    if rank == 0:
+        log(f"[bench] n={info.n} m={info.m} m_up={info.m_up} m_down={info.m_down} n_tail={info.n_tail} "
+            f"levels={info.levels} L0={lsz[0] / info.n:.3f} CH={info.build_seconds:.1f}s "
+            f"upward search space mean={info.mean_up_space:.1f} max={info.max_up_space} "
+            f"({info.up_space_samples} sampled sources)")
+        log("[bench] level histogram (level: vertices, 0 = lowest): " +
+            " ".join(f"{i}:{int(c)}" for i, c in enumerate(lsz)))
+        log(f"[bench] schedule k={k}: {sched}")
 
+    warm, timed, trees_here = rank_batches(n, cfg, k, world, rank, args.steps, args.warmup, args.total_sources)
+    args.steps = len(timed)
+
+    S = args.inflight
     stream = torch.cuda.current_stream()
-    sptr = stream.cuda_stream
-    dist_buf = torch.empty((g.n, k), dtype=torch.int32, device="cuda")
-    srcs = source_table(g.n, cfg, rank, args.warmup + args.steps, k)
+    streams = [torch.cuda.Stream() for _ in range(S)]
+    # L2 protocol: the C3/C4 label arrays (>= 1 GB) are far beyond the 126 MB L2; small
+    # configs (labels + graph fit in L2) flush L2 before every step, or with --steady
+    # rotate over enough label buffers that the labels alone exceed 2x L2
+    small = 4 * k * n + 16 * info.m_down < 256e6
+    flush = small and not args.steady
+    nbuf = S
+    if small and args.steady:
+        nbuf = max(S, -(-2 * L2_BYTES // (4 * k * n)))
+    bufs = [torch.empty(n * k, dtype=torch.int32, device="cuda") for _ in range(nbuf)]
 
-    for b in range(args.warmup):
-        h.trees_into(srcs[b], dist_buf.data_ptr(), sptr)
+    def issue(batches, ev0=None):
+        """batches round robin over the S streams (each waits for ev0 first)."""
+        if ev0 is not None:
+            for st in streams:
+                st.wait_event(ev0)
+        for i, b in enumerate(batches):
+            h.trees_into(b, bufs[i % nbuf].data_ptr(), streams[i % S].cuda_stream)
+
+    def join():
+        for st in streams:
+            e = torch.cuda.Event()
+            e.record(st)
+            stream.wait_event(e)
+
+    issue(warm)
+    join()
     h.sync(stream)
 
     # ---------------------------------------------------------------- timed region
-    # working set: the n*k*4-byte label array (4.6 GB at C3, k=64) >> 126 MB L2: no flush needed
-    # small configs (C1, C2: labels + graph fit in L2): every timed step starts from a
-    # flushed L2 (a 512 MB write between steps, outside the step's events)
-    flush = 4 * k * info.n + 16 * info.m_down < 256e6
     t0, t1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     if flush:
         scrub = torch.empty(512 << 20, dtype=torch.uint8, device="cuda")
-        ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+        groups = [timed[i:i + S] for i in range(0, len(timed), S)]   # a step of S sweeps in flight
+        ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in groups]
     with Clocks(local) as clk:
         barrier()
         torch.cuda.synchronize()
         h.timing(True)
         l0 = P.launch_count()
-        t0.record(stream)
-        for i, b in enumerate(range(args.warmup, args.warmup + args.steps)):
-            if flush:
+        if flush:
+            for i, grp in enumerate(groups):
                 scrub.fill_(i & 0xFF)
-                torch.cuda.synchronize()   # the step's upward search (side stream) starts after ev[i][0]
+                torch.cuda.synchronize()   # the step's upward searches start after ev[i][0]
                 ev[i][0].record(stream)
-            h.trees_into(srcs[b], dist_buf.data_ptr(), sptr)
-            if flush:
+                issue(grp, ev[i][0])
+                join()
                 ev[i][1].record(stream)
-        t1.record(stream)
+        else:
+            t0.record(stream)
+            issue(timed, t0)
+            join()
+            t1.record(stream)
         torch.cuda.synchronize()
         launches = P.launch_count() - l0
         barrier()
     h.timing(False)
     h.sync(stream)
-    ms = sum(a.elapsed_time(b) for a, b in ev) if flush else t0.elapsed_time(t1)
+    ms_local = sum(a.elapsed_time(b) for a, b in ev) if flush else t0.elapsed_time(t1)
     ms_up, ms_sweep, nb = h.timing_read()
-    if world > 1:
-        tt = torch.tensor([ms], dtype=torch.float64, device="cuda")
-        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
-        ms = float(tt.item())
-    trees = world * args.steps * k
-    value = trees / (ms / 1e3)
+    ms = max_over_ranks(ms_local)
+    total_trees = args.total_sources if args.total_sources else world * trees_here
+    value = total_trees / (ms / 1e3)
 
-    # roofline of the dominant kernel (the level sweep; one "launch" = one whole sweep)
+    # roofline of the dominant kernel: the level sweep of one batch (sweep_top_kernel +
+    # one sweep_kernel per level), algorithmic bytes B_alg (SURVEY.md §8(d))
     B_alg = 8 * info.m_down + 4 * (info.n + 1) + 4 * k * info.n + 4 * k * info.n_tail + info.n / 8
-    sweep_ms = ms_sweep / max(nb, 1)
+    sweeps = len(timed)
+    sweep_ms_events = ms_sweep / max(nb, 1)            # per-batch events (a3 + flag clear), stream-local
+    if S == 1:
+        sweep_ms = sweep_ms_events
+        how = "per-batch CUDA events around the sweep launches (a3 + flag clear) on the query stream"
+    else:   # overlapping sweeps: the whole timed region per sweep (upward searches and seeding included)
+        sweep_ms = ms_local / sweeps
+        how = (f"timed region / sweeps with {S} sweeps in flight (includes upward searches and seeding; "
+               "a lower bound of the sweep kernels' rate)")
     achieved = B_alg / (sweep_ms / 1e3) / 1e9
     peak, peak_src = peaks()
     traffic = None
     try:
         prof = json.load(open(os.path.join(ROOT, "profiles", "sweep_traffic.json")))
-        key = f"{args.config}_k{k}"
-        e = prof.get(key, {})
-        default_path = not any(os.environ.get(v) for v in ("PHAST_SWEEP", "PHAST_ARC_BATCH", "PHAST_TOP",
-                                                            "PHAST_FUSED", "PHAST_TOP_MAXV"))
-        if e.get("layout") == P.LAYOUT_NAMES[info.layout] and default_path and e.get("arc_batch") == "ell":
-            traffic = e["dram_bytes_per_sweep"]   # ncu launch list of this configuration (warm L2)
+        e = prof.get(f"{args.config}_k{k}", {})
+        if e.get("layout") == P.LAYOUT_NAMES[info.layout]:
+            traffic = e["dram_bytes_per_sweep"]   # warm-L2 ncu launch list of this configuration
     except Exception:
         pass
+
+    # probes A33 / A34 (SURVEY.md §8(d)) on the same arrays: ceilings for the sweep
+    ceiling = None
+    if not args.no_probes:
+        def timed_probe(kind, reps=5):
+            a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            h.probe(kind, k, bufs[0], sources=timed[0], stream=stream)
+            h.sync(stream)
+            a.record(stream)
+            for _ in range(reps):
+                h.probe(kind, k, bufs[0], sources=timed[0], stream=stream)
+            b.record(stream)
+            h.sync(stream)
+            return a.elapsed_time(b) / reps
+        a33 = timed_probe(0)
+        a34 = timed_probe(1)
+        B33 = 16 * n + 8 * k * n
+        ceiling = {"a33_stream_ms": a33, "a33_bytes": B33, "a33_GBps": B33 / (a33 / 1e3) / 1e9,
+                   "a34_nogather_ms": a34, "sweep_over_a33": sweep_ms / a33, "sweep_over_a34": sweep_ms / a34,
+                   "note": "A33: one sequential launch reading every ELL record and label row and writing "
+                           "every row (PAPER.md:22 §VIII-B 'PHAST is only 2.6 times slower than this'); A34: the "
+                           "query's launches with every tail-row gather replaced by the arc length "
+                           "('it takes 153 ms to traverse the graph exactly as PHAST does'); ratios are sweep "
+                           "time over probe time (L2 warm, back to back)"}
 
     # NEXT-1: parent pointers of the last timed batch (a separate pass, not in `value`)
     parents = None
     if args.parents:
-        par_buf = torch.empty((g.n, k), dtype=torch.int32, device="cuda")
-        last = srcs[args.warmup + args.steps - 1]
-        h.parents(last, dist_buf, out=par_buf, stream=stream)
+        par_buf = torch.empty(n * k, dtype=torch.int32, device="cuda")
+        last = timed[-1]
+        dist_t = bufs[(len(timed) - 1) % nbuf]
+        h.parents(last, dist_t, out=par_buf, stream=stream)
         h.sync(stream)
         p0, p1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         reps = max(1, min(args.steps, 10))
         p0.record(stream)
         for _ in range(reps):
-            h.parents(last, dist_buf, out=par_buf, stream=stream)
+            h.parents(last, dist_t, out=par_buf, stream=stream)
         p1.record(stream)
         h.sync(stream)
         pms = p0.elapsed_time(p1) / reps
-        m_in = g.m   # original arcs (self-loops, if any, are dropped by the library)
-        B_par = 8 * m_in + 4 * (g.n + 1) + 12 * k * g.n
+        B_par = 8 * info.m + 4 * (n + 1) + 12 * k * n
         parents = {"ms_per_pass": pms, "alg_bytes": B_par, "achieved_GBps": B_par / (pms / 1e3) / 1e9,
-                   "frac": B_par / (pms / 1e3) / 1e9 / peaks()[0],
+                   "frac": B_par / (pms / 1e3) / 1e9 / peak,
                    "note": "B = 8m + 4(n+1) + 12kn: in-arcs, offsets, own row read, in-neighbour rows read "
                            "at least once, parent row written"}
         del par_buf
@@ -302,20 +430,17 @@ def main():
     # end to end through the public host entry point (sources in, all labels out)
     e2e = None
     if args.e2e_steps > 0:
-        host_out = torch.empty((g.n, k), dtype=torch.int32, pin_memory=True).numpy().view(np.uint32)
-        h.trees_host(srcs[0], host_out, stream)
+        host_out = torch.empty((n, k), dtype=torch.int32, pin_memory=True).numpy().view(np.uint32)
+        h.trees_host(timed[0], host_out, stream)
         barrier()
         te = time.perf_counter()
         for b in range(args.e2e_steps):
-            h.trees_host(srcs[args.warmup + b % args.steps], host_out, stream)
-        te = time.perf_counter() - te
-        if world > 1:
-            tt = torch.tensor([te], dtype=torch.float64, device="cuda")
-            dist.all_reduce(tt, op=dist.ReduceOp.MAX)
-            te = float(tt.item())
+            h.trees_host(timed[b % len(timed)], host_out, stream)
+        te = max_over_ranks(time.perf_counter() - te)
         e2e = {"value": world * args.e2e_steps * k / te, "unit": "trees/s", "h2d_bytes_per_step": 4 * k,
-               "d2h_bytes_per_step": 4 * k * g.n,
-               "note": "phast_trees_host: sources in as kernel parameters, all n*k labels copied to pinned host memory"}
+               "d2h_bytes_per_step": 4 * k * n,
+               "note": "phast_trees_host: sources in as kernel parameters, all n*k labels copied to pinned host "
+                       "memory (PCIe-bound at large n*k)"}
         del host_out
 
     cpu = None
@@ -330,24 +455,37 @@ def main():
             cpu["us_per_tree_1thread"] = dt1 / 8 * 1e6
 
     if rank == 0:
+        if flush:
+            l2 = (f"L2 flushed before every timed step (512 MB write outside the step's events); a step = "
+                  f"{S} sweep(s) of k={k} in flight; value = trees / sum of per-step times")
+        elif small:
+            l2 = f"steady state: no flush, {nbuf} label buffers of {4 * k * n / 1e6:.0f} MB rotate (> 2x L2)"
+        else:
+            l2 = f"label array {4 * k * n / 1e9:.2f} GB per buffer >> 126 MB L2 (no flush needed)"
         line = {
             "metric": METRIC, "value": value, "unit": "trees/s", "n_gpus": world, "steps": args.steps,
-            "warmup": args.warmup, "ms_per_step": ms / args.steps, "higher_is_better": True, "scaling": "weak",
-            "vs_baseline": None, "dtype": "u32", "data": "synthetic",
-            "config": {"workload": f"{args.config}: {cfg['desc']}", "k": k, "trees_per_step_per_gpu": k,
-                       "n": info.n, "m": info.m, "m_down": info.m_down, "m_up": info.m_up, "n_tail": info.n_tail,
-                       "levels": info.levels, "layout": P.LAYOUT_NAMES[info.layout],
-                       "delta": info.delta, "sweep": os.environ.get("PHAST_SWEEP", "levels" if info.layout else "warp"), "parallelism": f"sources sharded over {world} GPU(s), graph replicated",
-                       "l2": ("L2 flushed before every timed step (512 MB write outside the step's events); "
-                              "value = steps * k / sum of per-step times") if flush else
-                             f"label array {4 * k * info.n / 1e9:.2f} GB >> 126 MB L2 (no flush needed)",
-                       "us_per_tree": ms * 1e3 / (args.steps * k),
+            "warmup": args.warmup, "ms_per_step": ms / max(args.steps, 1), "higher_is_better": True,
+            "scaling": "strong" if args.total_sources else "weak", "vs_baseline": None, "dtype": "u32",
+            "data": "synthetic",
+            "config": {"workload": f"{args.config}: {cfg['desc']}", "k": k, "sweeps_in_flight": S,
+                       "trees_total": total_trees, "n": info.n, "m": info.m, "m_down": info.m_down,
+                       "m_up": info.m_up, "n_tail": info.n_tail, "levels": info.levels,
+                       "level_sizes": [int(c) for c in lsz],
+                       "up_space": {"mean": round(info.mean_up_space, 1), "max": info.max_up_space,
+                                    "samples": info.up_space_samples},
+                       "schedule": sched, "layout": P.LAYOUT_NAMES[info.layout],
+                       "parallelism": (f"{args.total_sources} sources sharded over {world} GPU(s)"
+                                       if args.total_sources else f"{args.steps} batches per GPU on {world} GPU(s)")
+                                      + ", graph replicated",
+                       "l2": l2, "us_per_tree": ms * 1e3 / total_trees * world if args.total_sources
+                       else ms * 1e3 / trees_here,
                        "ch_build_s": round(info.build_seconds, 1)},
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
                          "traffic": traffic, "kernel": "sweep_top_kernel + sweep_kernel (all levels of one sweep)",
-                         "alg_bytes_per_sweep": B_alg, "sweep_ms": sweep_ms, "upward_ms": ms_up / max(nb, 1),
-                         "peak_source": peak_src},
-            "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": launches, "clocks": clk.summary(),
+                         "alg_bytes_per_sweep": B_alg, "sweep_ms": sweep_ms, "sweep_ms_events": sweep_ms_events,
+                         "upward_ms": ms_up / max(nb, 1), "how": how, "peak_source": peak_src},
+            "ceiling": ceiling, "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": launches,
+            "clocks": clk.summary(),
             **({"parents": parents} if parents else {}),
         }
         print(json.dumps(line), flush=True)

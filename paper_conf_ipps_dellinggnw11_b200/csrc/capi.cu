@@ -1,5 +1,5 @@
 // capi.cu -- the C ABI of include/phast.h: handle lifetime, validation, device
-// image upload, sweep plans and query orchestration.
+// image upload, launch plans and query orchestration.
 //
 // Layout (layout.cpp): internal ids follow a reverse topological order
 // of G-down, so that the sweep is "a simple linear sweep in increasing order of IDs"
@@ -21,28 +21,51 @@
 
 using namespace phast;
 
+static_assert(PHAST_SLOTS == SLOTS, "phast.h and kernels.h disagree on the slot count");
+
 struct phast_ctx {
     uint32_t n = 0;
-    uint64_t m = 0, shortcuts = 0;
+    uint64_t m = 0, shortcuts = 0, n_tail = 0;
     uint32_t rounds = 0;
     double build_seconds = 0;
     Layout L;
-    std::vector<uint32_t> tail_bits;   // bit v: internal id v is the tail of some G-down arc
+    phast_query_opts q = {0, 0, 0, 0};
+    // upward-search-space statistics of phast_info (host sample, computed once)
+    mutable bool up_stats = false;
+    mutable double up_mean = 0;
+    mutable uint32_t up_max = 0, up_samples = 0;
     // device
     int device = -1;
     DevImage g;
-    uint32_t* dist_scratch = nullptr;   // phast_trees_host / phast_diameter label buffer
-    size_t dist_scratch_elems = 0;
+    // per-query slots (PHAST_SLOTS in flight): visited bits + search spaces; upward
+    // searches run on one side stream, each waiting for its slot's previous query
+    Slot slot[SLOTS];
+    cudaEvent_t up_done[SLOTS] = {};
+    cudaEvent_t slot_free[SLOTS] = {};
+    uint32_t slot_next = 0;
+    cudaStream_t side = nullptr;
+    uint32_t* pad[SLOTS] = {};          // padded-k label scratch per slot (phast_trees with k not a power of two)
+    size_t pad_elems[SLOTS] = {};
+    // library streams for batches in flight (phast_diameter) and their label buffers
+    cudaStream_t lane[SLOTS] = {};
+    cudaEvent_t lane_ev[SLOTS] = {};
+    cudaEvent_t fork_ev = nullptr;
+    uint32_t* lane_dist[SLOTS] = {};
+    size_t lane_elems[SLOTS] = {};
+    uint32_t* host_scratch = nullptr;   // phast_trees_host label buffer
+    size_t host_elems = 0;
     uint32_t* batch_max_scratch = nullptr;
     size_t batch_max_elems = 0;
+    uint32_t* wit = nullptr;            // [4] witness scratch: max, pad, 64-bit key
     uint32_t* d_in_first = nullptr;     // original in-CSR on the device (parents; uploaded on first use)
     uint2* d_in_arc = nullptr;
     // NEXT-3 betweenness: original out-CSR {head, len} by tail (internal ids), sigma/delta
-    // rows [n][k] fp64, per-pass change words (device + pinned host)
+    // rows [n][k] fp64, per-pass change words (device + pinned host), label rows
     uint32_t* d_out_first = nullptr;
     uint2* d_out_arc = nullptr;
     double* bc_sigma = nullptr;
     double* bc_delta = nullptr;
+    uint32_t* bc_dist = nullptr;
     size_t bc_elems = 0;
     uint32_t* bc_changed = nullptr;
     uint32_t* bc_changed_host = nullptr;
@@ -51,40 +74,20 @@ struct phast_ctx {
     cudaStream_t bc_stream = nullptr;   // private stream the pass graphs run on
     cudaEvent_t bc_ev = nullptr;
     int bc_len_ok = 0;                  // 0 unknown, 1 all original lengths > 0, -1 not
-    // persistent-sweep plans, one per k (built on first use)
-    struct Plan {
-        SweepPlan p;
-        uint32_t epoch = 0;
-        uint32_t top_levels = 0;   // hybrid (per-level mode): levels [0, top_levels) run as one persistent launch
-        uint32_t bottom_from = 0;  // diagonal layout: segments [bottom_from, end) run as one lagged persistent launch
-        bool ok = false;
-    };
-    std::map<uint32_t, Plan> plans;
     // top levels [0, J) swept in one single-CTA launch (launch_sweep_top), one plan per k
     struct Top {
         uint4* chunks = nullptr;   // device [nchunks] {vbeg, vend, first[vbeg], first[vend]}
         TopArgs a;                 // a.fused: the whole query in this one launch
-        uint32_t J = 0;            // segments [0, J) in the shared-memory launch (0: none)
-        uint32_t J2 = 0;           // segments [J, J2) in one cluster launch (launch_sweep_cluster)
-        uint32_t* cl_seg = nullptr;   // device [J2 - J + 1] offsets
-        uint32_t vtop = 0;            // upward searches stop expanding below this id (0: full searches)
-        uint32_t* up_f = nullptr;     // top mode with vtop: A-up in-arcs by head inside [0, V)
+        uint32_t J = 0;            // levels [0, J) in the shared-memory launch (0: none)
+        uint32_t vtop = 0;         // upward searches stop expanding below this id (0: full searches)
+        uint32_t* up_f = nullptr;  // top mode with vtop: A-up in-arcs by head inside [0, V)
         uint2* up_a = nullptr;
-        bool ok = false;
     };
     std::map<uint32_t, Top> tops;
     // A-up in-arcs by head {tail, len} (fused single-launch queries on small graphs)
     uint32_t* d_upin_first = nullptr;
     uint2* d_upin_arc = nullptr;
     bool upin_tried = false;
-    // 0 = warp pipeline (default), 1 = one launch per level, 2 = CTA waves, 3 = CTA waves + bulk-staged
-    // arcs, 4 = pipelined CTA gather (k >= 4; else warp pipeline), 5 = warp dataflow without pipeline
-    int sweep_mode = 0;
-    // upward searches run on a side stream, one seed slot ahead of the sweep
-    cudaStream_t side = nullptr;
-    cudaEvent_t up_done[SEED_SLOTS] = {};
-    cudaEvent_t slot_free[SEED_SLOTS] = {};
-    uint32_t slot_next = 0;
     // stage timing (phast_timing)
     bool timing = false;
     std::vector<cudaEvent_t> ev;   // 3 per recorded batch
@@ -93,10 +96,16 @@ struct phast_ctx {
 
 namespace {
 
-constexpr uint32_t SEED_CAP = 1u << 16;   // per-source search-space capacity (global fallback)
-constexpr uint32_t DEFAULT_DELTA = 65536;
+constexpr uint32_t SEED_CAP = 1u << 16;   // default per-source search-space capacity
+constexpr uint32_t UP_SAMPLE = 1024;      // sources sampled for phast_info's search-space stats
 
-bool k_ok(uint32_t k) { return k == 1 || k == 2 || k == 4 || k == 8 || k == 16 || k == 32 || k == 64; }
+// the vector widths the kernels are instantiated for; any other k runs at the next one
+uint32_t kpad(uint32_t k) {
+    uint32_t p = 1;
+    while (p < k) p *= 2;
+    return p;
+}
+bool k_valid(uint32_t k) { return k >= 1 && k <= KMAX; }
 
 struct DeviceGuard {
     int prev = -1;
@@ -124,68 +133,110 @@ int dmalloc(T** p, size_t elems) {
     return PHAST_OK;
 }
 
-void free_plans(phast_ctx* h) {
-    for (auto& kv : h->plans) {
-        cudaFree((void*)kv.second.p.chunk_v);
-        cudaFree((void*)kv.second.p.chunk_dep);
-        cudaFree(kv.second.p.wave_done);
-        cudaFree((void*)kv.second.p.wmeta);
-        cudaFree((void*)kv.second.p.pinfo);
-        cudaFree((void*)kv.second.p.wdeps);
-        cudaFree(kv.second.p.done);
-    }
-    h->plans.clear();
+// device buffer that only grows
+template <class T>
+int grow(T** p, size_t* have, size_t elems) {
+    if (*have >= elems && *p) return PHAST_OK;
+    cudaFree(*p);
+    *p = nullptr;
+    *have = 0;
+    int rc = dmalloc(p, elems);
+    if (!rc) *have = elems;
+    return rc;
+}
+
+void free_tops(phast_ctx* h) {
     for (auto& kv : h->tops) {
-        cudaFree(kv.second.chunks); cudaFree(kv.second.cl_seg);
-        cudaFree(kv.second.up_f); cudaFree(kv.second.up_a);
+        cudaFree(kv.second.chunks);
+        cudaFree(kv.second.up_f);
+        cudaFree(kv.second.up_a);
     }
     h->tops.clear();
+}
+
+void free_seeds(phast_ctx* h) {
+    for (uint32_t s = 0; s < SLOTS; s++) {
+        cudaFree(h->slot[s].seed_v);
+        cudaFree(h->slot[s].seed_d);
+        h->slot[s].seed_v = h->slot[s].seed_d = nullptr;
+    }
+    cudaFree(h->g.gscratch);
+    h->g.gscratch = nullptr;
+}
+
+// search-space buffers for the current options (phast_query_opts seed_cap / up_smem_cap)
+int alloc_seeds(phast_ctx* h) {
+    auto pow2 = [](uint32_t x) { uint32_t p = 1; while (p * 2 <= x) p *= 2; return p; };
+    const uint32_t cap = h->q.seed_cap ? std::max(16u, std::min(SEED_CAP, h->q.seed_cap)) : SEED_CAP;
+    const uint32_t sm = h->q.up_smem_cap ? std::max(16u, std::min(4096u, h->q.up_smem_cap)) : 4096u;
+    h->g.seed_cap = pow2(cap);
+    h->g.smem_cap = pow2(sm);
+    int rc;
+    for (uint32_t s = 0; s < SLOTS; s++)
+        if ((rc = dmalloc(&h->slot[s].seed_v, (size_t)KMAX * h->g.seed_cap)) ||
+            (rc = dmalloc(&h->slot[s].seed_d, (size_t)KMAX * h->g.seed_cap)))
+            return rc;
+    return dmalloc(&h->g.gscratch, (size_t)KMAX * h->g.seed_cap * 5);
 }
 
 void free_device(phast_ctx* h) {
     if (h->device < 0) return;
     DeviceGuard dg(h->device);
     cudaDeviceSynchronize();
-    free_plans(h);
+    free_tops(h);
+    free_seeds(h);
     for (cudaEvent_t e : h->ev) cudaEventDestroy(e);
     h->ev.clear();
     h->ev_used = 0;
-    for (uint32_t s = 0; s < SEED_SLOTS; s++) {
+    for (uint32_t s = 0; s < SLOTS; s++) {
         if (h->up_done[s]) cudaEventDestroy(h->up_done[s]);
         if (h->slot_free[s]) cudaEventDestroy(h->slot_free[s]);
-        h->up_done[s] = h->slot_free[s] = nullptr;
+        if (h->lane_ev[s]) cudaEventDestroy(h->lane_ev[s]);
+        if (h->lane[s]) cudaStreamDestroy(h->lane[s]);
+        cudaFree(h->slot[s].flags);
+        cudaFree(h->slot[s].seed_cnt);
+        cudaFree(h->pad[s]);
+        cudaFree(h->lane_dist[s]);
+        h->up_done[s] = h->slot_free[s] = h->lane_ev[s] = nullptr;
+        h->lane[s] = nullptr;
+        h->slot[s] = Slot();
+        h->pad[s] = h->lane_dist[s] = nullptr;
+        h->pad_elems[s] = h->lane_elems[s] = 0;
     }
+    if (h->fork_ev) cudaEventDestroy(h->fork_ev);
+    h->fork_ev = nullptr;
     if (h->side) cudaStreamDestroy(h->side);
     h->side = nullptr;
     cudaFree((void*)h->g.dn_first); cudaFree((void*)h->g.dn_arc);
     cudaFree((void*)h->g.dn_rec); cudaFree((void*)h->g.dn_ovf);
     cudaFree((void*)h->g.up_first); cudaFree((void*)h->g.up_arc);
-    cudaFree(h->g.flags); cudaFree((void*)h->g.tail_bits);
-    cudaFree(h->g.seed_v); cudaFree(h->g.seed_d); cudaFree(h->g.seed_cnt);
-    cudaFree(h->g.gscratch); cudaFree(h->g.err);
-    cudaFree(h->dist_scratch); cudaFree(h->batch_max_scratch);
+    cudaFree(h->g.err);
+    cudaFree(h->host_scratch); cudaFree(h->batch_max_scratch); cudaFree(h->wit);
     cudaFree(h->d_in_first); cudaFree(h->d_in_arc);
-    h->d_in_first = nullptr; h->d_in_arc = nullptr;
-    cudaFree(h->d_out_first); cudaFree(h->d_out_arc); cudaFree(h->bc_sigma); cudaFree(h->bc_delta);
+    cudaFree(h->d_out_first); cudaFree(h->d_out_arc);
+    cudaFree(h->bc_sigma); cudaFree(h->bc_delta); cudaFree(h->bc_dist);
     cudaFree(h->bc_changed); cudaFreeHost(h->bc_changed_host); cudaFree(h->bc_q); cudaFree(h->bc_qs);
-    h->bc_q = nullptr; h->bc_qs = nullptr;
     if (h->bc_stream) cudaStreamDestroy(h->bc_stream);
     if (h->bc_ev) cudaEventDestroy(h->bc_ev);
-    h->bc_stream = nullptr; h->bc_ev = nullptr;
-    h->d_out_first = nullptr; h->d_out_arc = nullptr; h->bc_sigma = h->bc_delta = nullptr;
-    h->bc_elems = 0; h->bc_changed = nullptr; h->bc_changed_host = nullptr;
     cudaFree(h->d_upin_first); cudaFree(h->d_upin_arc);
-    h->d_upin_first = nullptr; h->d_upin_arc = nullptr;
-    h->upin_tried = false;
+    h->host_scratch = nullptr; h->host_elems = 0;
+    h->batch_max_scratch = nullptr; h->batch_max_elems = 0; h->wit = nullptr;
+    h->d_in_first = nullptr; h->d_in_arc = nullptr;
+    h->d_out_first = nullptr; h->d_out_arc = nullptr;
+    h->bc_sigma = h->bc_delta = nullptr; h->bc_dist = nullptr; h->bc_elems = 0;
+    h->bc_changed = nullptr; h->bc_changed_host = nullptr; h->bc_q = nullptr; h->bc_qs = nullptr;
+    h->bc_stream = nullptr; h->bc_ev = nullptr;
+    h->d_upin_first = nullptr; h->d_upin_arc = nullptr; h->upin_tried = false;
     h->g = DevImage();
-    h->dist_scratch = nullptr; h->batch_max_scratch = nullptr;
-    h->dist_scratch_elems = 0; h->batch_max_elems = 0;
     h->device = -1;
 }
 
-void compute_tail_bits(phast_ctx* h) {
-    h->tail_bits.assign(((size_t)h->n + 31) / 32, 0u);
-    for (const Arc& a : h->L.dn_arc) h->tail_bits[a.x >> 5] |= 1u << (a.x & 31);
+void count_tails(phast_ctx* h) {
+    std::vector<uint32_t> bits(((size_t)h->n + 31) / 32, 0u);
+    for (const Arc& a : h->L.dn_arc) bits[a.x >> 5] |= 1u << (a.x & 31);
+    uint64_t nt = 0;
+    for (uint32_t w : bits) nt += (uint64_t)__builtin_popcount(w);
+    h->n_tail = nt;
 }
 
 int upload(phast_ctx* h) {
@@ -194,48 +245,29 @@ int upload(phast_ctx* h) {
     h->device = dev;
     DevImage& g = h->g;
     g.n = h->n;
-    if (const char* e = std::getenv("PHAST_SWEEP"))
-        h->sweep_mode = std::strcmp(e, "levels") == 0       ? 1
-                        : std::strcmp(e, "persistent") == 0 ? 2
-                        : std::strcmp(e, "staged") == 0     ? 3
-                        : std::strcmp(e, "pipe") == 0       ? 4
-                        : std::strcmp(e, "warp") == 0       ? 5
-                        : std::strcmp(e, "wave") == 0       ? 6
-                        : std::strcmp(e, "segments") == 0   ? 7
-                                                            : 0;
-    // level layouts default to one launch per level (the fastest schedule measured on them)
-    if (!std::getenv("PHAST_SWEEP") && !h->L.lvl_off.empty()) h->sweep_mode = 1;
-    if ((h->sweep_mode == 1 || h->sweep_mode == 7) && h->L.lvl_off.empty()) h->sweep_mode = 0;   // needs segments
-    // test knobs (rounded down to powers of two): shrink the shared-memory table / the
-    // per-source capacity to exercise the global fallback and the overflow error path
-    uint32_t seed_cap = SEED_CAP, smem_cap = 4096;
-    if (const char* e = std::getenv("PHAST_SEED_CAP"))
-        seed_cap = std::max(16u, std::min<uint32_t>(SEED_CAP, (uint32_t)std::atoi(e)));
-    if (const char* e = std::getenv("PHAST_L2_PERSIST_MB"))   // experiment knob
-        set_l2_persist((size_t)std::max(0, std::atoi(e)) << 20);
-    if (const char* e = std::getenv("PHAST_UP_SMEM_CAP"))
-        smem_cap = std::max(16u, std::min<uint32_t>(4096u, (uint32_t)std::atoi(e)));
-    auto pow2 = [](uint32_t x) { uint32_t p = 1; while (p * 2 <= x) p *= 2; return p; };
-    g.seed_cap = pow2(seed_cap);
-    g.smem_cap = pow2(smem_cap);
     const Layout& L = h->L;
-    uint32_t *dnf = nullptr, *upf = nullptr, *tb = nullptr;
+    uint32_t *dnf = nullptr, *upf = nullptr;
     uint2 *dna = nullptr, *upa = nullptr;
     int rc;
-    size_t nw = ((size_t)h->n + 31) / 32;
+    const size_t nw = ((size_t)h->n + 31) / 32;
     // +4 / +2 elements: 16-byte aligned bulk copies may read up to 12 bytes past the end
     if ((rc = dmalloc(&dnf, L.dn_first.size() + 4)) || (rc = dmalloc(&dna, L.dn_arc.size() + 2)) ||
         (rc = dmalloc(&upf, L.up_first.size())) || (rc = dmalloc(&upa, L.up_arc.size())) ||
-        (rc = dmalloc(&g.flags, nw)) || (rc = dmalloc(&tb, nw)) ||
-        (rc = dmalloc(&g.seed_v, (size_t)SEED_SLOTS * KMAX * g.seed_cap)) ||
-        (rc = dmalloc(&g.seed_d, (size_t)SEED_SLOTS * KMAX * g.seed_cap)) ||
-        (rc = dmalloc(&g.seed_cnt, SEED_SLOTS * KMAX)) || (rc = dmalloc(&g.gscratch, (size_t)KMAX * g.seed_cap * 5)) ||
         (rc = dmalloc(&g.err, 1))) {
-        g.dn_first = dnf; g.dn_arc = dna; g.up_first = upf; g.up_arc = upa; g.tail_bits = tb;
+        g.dn_first = dnf; g.dn_arc = dna; g.up_first = upf; g.up_arc = upa;
         free_device(h);
         return rc;
     }
-    g.dn_first = dnf; g.dn_arc = dna; g.up_first = upf; g.up_arc = upa; g.tail_bits = tb;
+    g.dn_first = dnf; g.dn_arc = dna; g.up_first = upf; g.up_arc = upa;
+    for (uint32_t s = 0; s < SLOTS; s++)
+        if ((rc = dmalloc(&h->slot[s].flags, nw)) || (rc = dmalloc(&h->slot[s].seed_cnt, KMAX))) {
+            free_device(h);
+            return rc;
+        }
+    if ((rc = alloc_seeds(h))) {
+        free_device(h);
+        return rc;
+    }
     // G-down as ELL-2 records + overflow lists (kernels.h: DevImage::dn_rec)
     {
         std::vector<uint4> rec(h->n);
@@ -274,14 +306,17 @@ int upload(phast_ctx* h) {
               cudaMemcpy(dna, L.dn_arc.data(), L.dn_arc.size() * 8, cudaMemcpyHostToDevice) == cudaSuccess &&
               cudaMemcpy(upf, L.up_first.data(), L.up_first.size() * 4, cudaMemcpyHostToDevice) == cudaSuccess &&
               cudaMemcpy(upa, L.up_arc.data(), L.up_arc.size() * 8, cudaMemcpyHostToDevice) == cudaSuccess &&
-              cudaMemcpy(tb, h->tail_bits.data(), nw * 4, cudaMemcpyHostToDevice) == cudaSuccess &&
-              cudaMemset(g.flags, 0, nw * 4) == cudaSuccess && cudaMemset(g.err, 0, 4) == cudaSuccess &&
-              cudaMemset(g.seed_cnt, 0, SEED_SLOTS * KMAX * 4) == cudaSuccess &&
+              cudaMemset(g.err, 0, 4) == cudaSuccess &&
               cudaStreamCreateWithFlags(&h->side, cudaStreamNonBlocking) == cudaSuccess &&
-              cudaDeviceSynchronize() == cudaSuccess;
-    for (uint32_t s = 0; ok && s < SEED_SLOTS; s++)
-        ok = cudaEventCreateWithFlags(&h->up_done[s], cudaEventDisableTiming) == cudaSuccess &&
-             cudaEventCreateWithFlags(&h->slot_free[s], cudaEventDisableTiming) == cudaSuccess;
+              cudaEventCreateWithFlags(&h->fork_ev, cudaEventDisableTiming) == cudaSuccess;
+    for (uint32_t s = 0; ok && s < SLOTS; s++)
+        ok = cudaMemset(h->slot[s].flags, 0, nw * 4) == cudaSuccess &&
+             cudaMemset(h->slot[s].seed_cnt, 0, KMAX * 4) == cudaSuccess &&
+             cudaEventCreateWithFlags(&h->up_done[s], cudaEventDisableTiming) == cudaSuccess &&
+             cudaEventCreateWithFlags(&h->slot_free[s], cudaEventDisableTiming) == cudaSuccess &&
+             cudaEventCreateWithFlags(&h->lane_ev[s], cudaEventDisableTiming) == cudaSuccess &&
+             cudaStreamCreateWithFlags(&h->lane[s], cudaStreamNonBlocking) == cudaSuccess;
+    ok = ok && cudaDeviceSynchronize() == cudaSuccess;
     if (!ok) { cudaGetLastError(); free_device(h); return PHAST_ECUDA; }
     return PHAST_OK;
 }
@@ -291,213 +326,24 @@ int validate_csr(uint32_t n, const uint64_t* first, const uint32_t* head, const 
     if (first[0] != 0) return PHAST_EINVAL;
     for (uint32_t v = 0; v < n; v++)
         if (first[v + 1] < first[v]) return PHAST_EINVAL;
-    uint64_t m = first[n];
+    const uint64_t m = first[n];
     if (m && (!head || !len)) return PHAST_EINVAL;
     for (uint64_t e = 0; e < m; e++)
         if (head[e] >= n) return PHAST_EINVAL;
     return PHAST_OK;
 }
 
-int map_sources(const phast_ctx* h, const uint32_t* src, uint32_t k, Sources& S) {
+// a0: original ids -> internal ids; the kp - k padding trees repeat sources[0]
+int map_sources(const phast_ctx* h, const uint32_t* src, uint32_t k, uint32_t kp, Sources& S) {
     for (uint32_t i = 0; i < k; i++) {
         if (src[i] >= h->n) return PHAST_ERANGE;
         S.s[i] = h->L.perm[src[i]];
     }
-    for (uint32_t i = k; i < KMAX; i++) S.s[i] = 0;
+    for (uint32_t i = k; i < KMAX; i++) S.s[i] = i < kp ? S.s[0] : 0u;
     return PHAST_OK;
 }
 
-// Chunk size: at most sweep_chunk_vertices(k); in the wavefront layout small enough
-// that one iteration of all CTAs (grid * cap vertices) stays under delta / 2, so that
-// almost every dependency points at least one iteration back (few pad slots).
-uint32_t chunk_cap_for(const Layout& L, uint32_t k, uint32_t grid) {
-    const uint32_t vmax = sweep_chunk_vertices(k), vpp = sweep_pass_vertices(k);
-    if (L.mode != LAYOUT_WAVEFRONT) return vmax;
-    uint32_t cap = L.delta / (2 * std::max(1u, grid));
-    cap = cap / vpp * vpp;
-    return std::max(vpp, std::min(vmax, cap));
-}
-
-// Plan of the persistent sweep for one k.  Chunks are contiguous internal-id ranges
-// of at most CV vertices, cut wherever a vertex has a G-down tail inside the open
-// chunk (so a chunk never waits on itself).  Chunk c is processed by CTA c % grid in
-// iteration c / grid; it depends on the iteration of the latest chunk holding one
-// of its tails, and may start once every CTA has finished that iteration.
-phast_ctx::Plan* get_plan(phast_ctx* h, uint32_t k) {
-    auto it = h->plans.find(k);
-    if (it != h->plans.end()) return it->second.ok ? &it->second : nullptr;
-    phast_ctx::Plan& P = h->plans[k];
-    const Layout& L = h->L;
-    SweepPlan& p = P.p;
-    p.k = k;
-    p.variant = h->sweep_mode == 2 ? 0u : h->sweep_mode == 3 ? 1u : h->sweep_mode == 4 && k >= 4 ? 3u
-              : h->sweep_mode == 5 ? 2u : h->sweep_mode == 6 ? 5u : h->sweep_mode == 7 ? 6u : 4u;
-    uint32_t nseg_top = 0, seg_from = 0;
-    const char* bseg = std::getenv("PHAST_BOTTOM_SEG");
-    if (h->sweep_mode == 1 && L.mode == LAYOUT_DIAGONAL && bseg && std::atoi(bseg)) {
-        // the diagonals of the bottom levels in ONE launch; segment j waits only for
-        // segment j - lag (the layout's guarantee), the top levels stay one launch each
-        seg_from = L.levels - L.cut;
-        P.bottom_from = seg_from;
-        p.variant = 6;
-    } else if (h->sweep_mode == 1) {   // hybrid: the small top segments as one segment-barrier launch, big ones one launch each
-        uint32_t thresh = 0;
-        if (const char* e = std::getenv("PHAST_TOP_THRESH")) thresh = (uint32_t)std::atoi(e);
-        uint32_t J = 0;
-        while (J + 1 < L.lvl_off.size() && L.lvl_off[J + 1] - L.lvl_off[J] < thresh) J++;
-        if (J < 2) return nullptr;           // nothing worth fusing
-        P.top_levels = J;
-        nseg_top = J;
-        p.variant = 6;
-    }
-    int occ = std::min(sweep_blocks_per_sm(k, false, p.variant), sweep_blocks_per_sm(k, true, p.variant));
-    p.grid = (uint32_t)std::max(1, occ * num_sms());
-    p.err = h->g.err;
-    if (p.variant == 6) {   // segment barriers: the segments of the layout, one grid barrier between two
-        if ((uint64_t)h->n * 16 >= 0x7FFFFFFFull) return nullptr;   // 32-bit item indices
-        // CTAs per SM: all (8) for a whole sweep; for the hybrid's top levels fewer, so
-        // that the next batch's upward searches (side stream) stay co-resident and never
-        // hold back a CTA of this grid (every CTA must be resident for the barriers)
-        int per_sm = nseg_top ? 4 : 8;
-        if (const char* e = std::getenv(nseg_top ? "PHAST_TOP_CTAS" : "PHAST_SEG_CTAS")) per_sm = std::max(1, std::atoi(e));
-        p.grid = (uint32_t)std::max(1, std::min(occ, per_sm) * num_sms());
-        const uint32_t nseg = nseg_top ? nseg_top : (uint32_t)L.lvl_off.size() - 1 - seg_from;
-        p.nchunks = p.iters = nseg;
-        p.chunk_cap = seg_from ? 0u : L.mode == LAYOUT_DIAGONAL ? L.levels - L.cut : nseg;   // diagonals: by tail bit
-        p.stream_last = nseg_top ? 0u : 1u;   // the layout's last segment is nobody's tail
-        p.seg_lag = seg_from ? L.lag : 1u;
-        uint32_t *a, *w;
-        if (dmalloc(&a, nseg + 1) || dmalloc(&w, nseg)) return nullptr;
-        p.chunk_v = a;
-        p.wave_done = w;
-        if (cudaMemcpy(a, L.lvl_off.data() + seg_from, (size_t)(nseg + 1) * 4, cudaMemcpyHostToDevice) != cudaSuccess ||
-            cudaMemset(w, 0, (size_t)nseg * 4) != cudaSuccess) {
-            cudaGetLastError();
-            return nullptr;
-        }
-        P.ok = true;
-        return &P;
-    }
-    if (p.variant == 5) {   // warp waves: one wave = one chunk of every warp (layout.cpp: plan_waves)
-        p.workers = p.grid * SWEEP_WARPS;
-        uint32_t window = 4;
-        if (const char* e = std::getenv("PHAST_WAVE_WINDOW")) window = (uint32_t)std::atoi(e);
-        WavePlan wp;
-        if (plan_waves(L, sweep_wave_chunk_vertices(k), sweep_wave_chunk_arcs(), p.workers, window, wp))
-            return nullptr;
-        p.nchunks = wp.chunks;
-        p.iters = wp.waves;
-        p.chunk_cap = (wp.waves + 63) / 64 * 64;   // sub-counter stride: each sub-counter array on its own lines
-        if (std::getenv("PHAST_VERBOSE"))
-            std::fprintf(stderr, "wave plan k=%u: T=%u chunks=%u waves=%u pads=%u lag1=%llu lag2=%llu lag3=%llu lag4+=%llu\n",
-                         k, p.workers, wp.chunks, wp.waves, wp.pads, (unsigned long long)wp.lag_hist[0],
-                         (unsigned long long)wp.lag_hist[1], (unsigned long long)wp.lag_hist[2],
-                         (unsigned long long)wp.lag_hist[3]);
-        uint32_t *a, *w;
-        const size_t nc = (size_t)sweep_wave_subcounters() * p.chunk_cap;
-        if (dmalloc(&a, wp.desc.size() + 4) || dmalloc(&w, nc)) return nullptr;
-        p.wdesc = reinterpret_cast<const uint4*>(a);
-        p.wave_done = w;
-        if ((!wp.desc.empty() && cudaMemcpy(a, wp.desc.data(), wp.desc.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess) ||
-            cudaMemset(w, 0, nc * 4) != cudaSuccess) {
-            cudaGetLastError();
-            return nullptr;
-        }
-        P.ok = true;
-        return &P;
-    }
-    if (p.variant == 2 || p.variant == 4) {
-        p.workers = p.grid * (SWEEP_WARPS);
-        WarpPlan wp;
-        const uint32_t cap = p.variant == 4 ? sweep_wpipe_chunk_vertices(k) : sweep_warp_chunk_vertices(k);
-        if (plan_warp_chunks(L, cap, p.workers, wp, p.variant == 4 ? 126u : 0u)) return nullptr;
-        p.nchunks = wp.chunks;
-        p.chunk_cap = cap;
-        if (p.variant == 4) {   // per-chunk {vbeg, vend, e0, e1} for the cp.async staging
-            std::vector<uint32_t> info((size_t)wp.chunks * 4);
-            for (uint32_t j = 0; j < wp.chunks; j++) {
-                const uint32_t vb = wp.meta[4 * (size_t)j], ve = wp.meta[4 * (size_t)j + 1];
-                info[4 * (size_t)j + 0] = vb;
-                info[4 * (size_t)j + 1] = ve;
-                info[4 * (size_t)j + 2] = L.dn_first[vb];
-                info[4 * (size_t)j + 3] = L.dn_first[ve];
-            }
-            uint32_t* pi;
-            if (dmalloc(&pi, info.size())) return nullptr;
-            p.pinfo = reinterpret_cast<const uint4*>(pi);
-            if (cudaMemcpy(pi, info.data(), info.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess) {
-                cudaGetLastError();
-                return nullptr;
-            }
-        }
-        uint32_t *a, *b, *w;
-        if (dmalloc(&a, wp.meta.size()) || dmalloc(&b, wp.deps.size()) || dmalloc(&w, wp.chunks)) return nullptr;
-        p.wmeta = reinterpret_cast<const uint4*>(a); p.wdeps = b; p.done = w;
-        if (cudaMemcpy(a, wp.meta.data(), wp.meta.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess ||
-            (!wp.deps.empty() &&
-             cudaMemcpy(b, wp.deps.data(), wp.deps.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess) ||
-            cudaMemset(w, 0, (size_t)wp.chunks * 4) != cudaSuccess) {
-            cudaGetLastError();
-            return nullptr;
-        }
-        P.ok = true;
-        return &P;
-    }
-    if (p.variant == 3) {   // pipelined gather: CTA chunks, per-chunk completion flags, one-chunk lookahead
-        uint32_t gv = 0, cap_arcs = 0;
-        sweep_pipe_geometry(k, &gv, &cap_arcs);
-        p.workers = p.grid;
-        p.chunk_cap = gv;
-        WarpPlan wp;
-        if (plan_warp_chunks(L, gv, p.workers, wp, cap_arcs)) return nullptr;
-        p.nchunks = wp.chunks;
-        std::vector<uint32_t> info((size_t)wp.chunks * 4);
-        for (uint32_t j = 0; j < wp.chunks; j++) {
-            const uint32_t vb = wp.meta[4 * (size_t)j], ve = wp.meta[4 * (size_t)j + 1];
-            info[4 * (size_t)j + 0] = vb;
-            info[4 * (size_t)j + 1] = ve;
-            info[4 * (size_t)j + 2] = L.dn_first[vb];
-            info[4 * (size_t)j + 3] = L.dn_first[ve];
-        }
-        uint32_t *a, *b, *w, *pi;
-        if (dmalloc(&a, wp.meta.size()) || dmalloc(&b, wp.deps.size()) || dmalloc(&w, wp.chunks) ||
-            dmalloc(&pi, info.size()))
-            return nullptr;
-        p.wmeta = reinterpret_cast<const uint4*>(a); p.wdeps = b; p.done = w;
-        p.pinfo = reinterpret_cast<const uint4*>(pi);
-        if (cudaMemcpy(a, wp.meta.data(), wp.meta.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess ||
-            (!wp.deps.empty() &&
-             cudaMemcpy(b, wp.deps.data(), wp.deps.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess) ||
-            cudaMemcpy(pi, info.data(), info.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess ||
-            cudaMemset(w, 0, (size_t)wp.chunks * 4) != cudaSuccess) {
-            cudaGetLastError();
-            return nullptr;
-        }
-        P.ok = true;
-        return &P;
-    }
-    const uint32_t CV = chunk_cap_for(h->L, k, p.grid);
-    p.chunk_cap = CV;
-    ChunkPlan cp;
-    if (plan_chunks(L, CV, p.grid, cp, 0, 1, 0)) return nullptr;
-    p.nchunks = cp.slots;
-    p.iters = (cp.slots + p.grid - 1) / p.grid;
-    const std::vector<uint32_t>& cv = cp.slot_v;
-    const std::vector<uint32_t>& dep = cp.dep;
-    uint32_t *a, *b, *w;
-    if (dmalloc(&a, cv.size()) || dmalloc(&b, dep.size()) || dmalloc(&w, p.iters)) return nullptr;
-    p.chunk_v = a; p.chunk_dep = b; p.wave_done = w;
-    if (cudaMemcpy(a, cv.data(), cv.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess ||
-        cudaMemcpy(b, dep.data(), dep.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess ||
-        cudaMemset(w, 0, (size_t)p.iters * 4) != cudaSuccess) {
-        cudaGetLastError();
-        return nullptr;
-    }
-    P.ok = true;
-    return &P;
-}
-
-// Chunks of one segment [a, b) over a CSR (offsets `f`): <= VCH vertices and <= ECH
+// Chunks of one level [a, b) over a CSR (offsets `f`): <= VCH vertices and <= ECH
 // arcs each; chunks without arcs change nothing and are skipped.
 void push_chunks(std::vector<uint4>& ch, const uint32_t* f, uint32_t a, uint32_t b, bool big) {
     const uint32_t VCH = top_chunk_vertices(big), ECH = top_chunk_arcs(big);
@@ -512,183 +358,158 @@ void push_chunks(std::vector<uint4>& ch, const uint32_t* f, uint32_t a, uint32_t
     }
 }
 
-// A-up in-arcs by head, uploaded once (graphs small enough for a fused query).
-bool ensure_upin(phast_ctx* h) {
-    if (h->d_upin_first) return true;
-    if (h->upin_tried) return false;
-    h->upin_tried = true;
-    const Layout& L = h->L;
-    const uint32_t n = h->n;
-    std::vector<uint32_t> f((size_t)n + 1, 0);
-    for (const Arc& a : L.up_arc) f[a.x + 1]++;
-    for (uint32_t v = 0; v < n; v++) f[v + 1] += f[v];
-    std::vector<Arc> arc(L.up_arc.size());
+// A-up in-arcs by head {tail, len} of the arcs inside [0, V) (V = n: all of them; the
+// top levels are a prefix of the ids and A-up climbs, so a tail < V has its head < V),
+// as a CSR over [0, V]; false if some head has more than `cap` in-arcs.  Arcs entering
+// [0, V) from below are the upward search's (hybrid mode): the pull pass reads only
+// rows inside [0, V), which live in shared memory.
+bool upin_csr(const Layout& L, uint32_t V, uint32_t cap, std::vector<uint32_t>& f, std::vector<Arc>& arc) {
+    f.assign((size_t)V + 1, 0);
+    for (uint32_t u = 0; u < V; u++)
+        for (uint32_t e = L.up_first[u]; e < L.up_first[u + 1]; e++) f[L.up_arc[e].x + 1]++;
+    for (uint32_t v = 0; v < V; v++) {
+        if (f[v + 1] > cap) return false;
+        f[v + 1] += f[v];
+    }
+    arc.resize(f[V]);
     std::vector<uint32_t> pos(f.begin(), f.end() - 1);
-    for (uint32_t u = 0; u < n; u++)
+    for (uint32_t u = 0; u < V; u++)
         for (uint32_t e = L.up_first[u]; e < L.up_first[u + 1]; e++) arc[pos[L.up_arc[e].x]++] = Arc{u, L.up_arc[e].y};
-    for (uint32_t v = 0; v < n; v++)
-        if (f[v + 1] - f[v] > top_chunk_arcs(true)) return false;
-    uint32_t* df = nullptr;
-    uint2* da = nullptr;
-    // +4 / +2 elements: the 16-byte aligned bulk copies may read past the end
-    if (dmalloc(&df, f.size() + 4) || dmalloc(&da, arc.size() + 2)) {
-        cudaFree(df);
-        return false;
-    }
-    if (cudaMemset(df, 0, (f.size() + 4) * 4) != cudaSuccess || cudaMemset(da, 0, (arc.size() + 2) * 8) != cudaSuccess ||
-        cudaMemcpy(df, f.data(), f.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess ||
-        (!arc.empty() && cudaMemcpy(da, arc.data(), arc.size() * 8, cudaMemcpyHostToDevice) != cudaSuccess)) {
-        cudaGetLastError();
-        cudaFree(df);
-        cudaFree(da);
-        return false;
-    }
-    h->d_upin_first = df;
-    h->d_upin_arc = da;
     return true;
 }
 
-// Shared-memory sweep plans (kernels.cu: sweep_top_kernel), one per k:
-//  - fused: the whole graph's rows fit the label budget -> the whole query (G-up
-//    pull sweep, then the G-down sweep) in one launch.  PHAST_FUSED=0 disables it;
-//  - top: the longest prefix of levels whose rows [0, V) fit, each level small
-//    enough for one SM (<= 32 items per consumer thread); the rest one launch per
-//    level.  PHAST_TOP=0 disables it; PHAST_TOP_MAXV caps V.
+// upload a CSR with the bulk-copy padding (+4 offsets, +2 arcs)
+bool upload_csr(const std::vector<uint32_t>& f, const std::vector<Arc>& arc, uint32_t** df, uint2** da) {
+    *df = nullptr;
+    *da = nullptr;
+    if (dmalloc(df, f.size() + 4) || dmalloc(da, arc.size() + 2)) {
+        cudaFree(*df);
+        *df = nullptr;
+        return false;
+    }
+    if (cudaMemset(*df, 0, (f.size() + 4) * 4) != cudaSuccess || cudaMemset(*da, 0, (arc.size() + 2) * 8) != cudaSuccess ||
+        cudaMemcpy(*df, f.data(), f.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess ||
+        (!arc.empty() && cudaMemcpy(*da, arc.data(), arc.size() * 8, cudaMemcpyHostToDevice) != cudaSuccess)) {
+        cudaGetLastError();
+        cudaFree(*df);
+        cudaFree(*da);
+        *df = nullptr;
+        *da = nullptr;
+        return false;
+    }
+    return true;
+}
+
+// Shared-memory sweep plan (top.cu: sweep_top_kernel) for one k; nullptr = none (every
+// level gets its own launch):
+//  - fused: the whole graph's rows fit the label budget -> the whole query (G-up pull
+//    sweep, then the G-down sweep) in one launch (off with PHAST_Q_NO_FUSED);
+//  - top: the longest prefix of levels whose rows [0, V) fit, each level small enough
+//    for one SM (<= 32 items per consumer thread); the rest one launch per level (off
+//    with PHAST_Q_NO_TOP; V capped by top_max_vertices).
 // Both need every vertex to have at most top_chunk_arcs(big) in-arcs; big chunks
 // (top_big_fits) when the rows leave room for them.
 phast_ctx::Top* get_top(phast_ctx* h, uint32_t k) {
     auto it = h->tops.find(k);
-    if (it != h->tops.end()) return it->second.ok ? &it->second : nullptr;
-    phast_ctx::Top& T = h->tops[k];
+    if (it != h->tops.end()) return it->second.chunks ? &it->second : nullptr;
+    phast_ctx::Top& T = h->tops[k];   // chunks stays nullptr: "no plan"
     const Layout& L = h->L;
-    if (L.mode != LAYOUT_LEVELS && L.mode != LAYOUT_LEVELS_BFS) return nullptr;
     if (L.lvl_off.size() < 2 || h->n >= 0x80000000u) return nullptr;   // chunk vend carries a flag bit
     const uint32_t nseg = (uint32_t)L.lvl_off.size() - 1;
     const uint32_t G = k >= 4 ? k / 4 : 1;
-    const uint32_t ECH = top_chunk_arcs(false);
     const uint64_t vmax_budget = top_label_budget() / (4ull * k);
     std::vector<uint4> ch;
-    const char* fe = std::getenv("PHAST_FUSED");
-    bool fused = !(fe && std::atoi(fe) == 0) && h->n <= vmax_budget;
+    bool fused = !(h->q.flags & PHAST_Q_NO_FUSED) && h->n <= vmax_budget;
     const bool fbig = fused && top_big_fits(k, h->n);
-    const uint32_t ECHf = top_chunk_arcs(fbig);
-    for (uint32_t v = 0; fused && v < h->n; v++) fused = L.dn_first[v + 1] - L.dn_first[v] <= ECHf;
-    std::vector<uint32_t> f;
-    if (fused && ensure_upin(h)) {
-        f.resize((size_t)h->n + 1);
-        if (cudaMemcpy(f.data(), h->d_upin_first, f.size() * 4, cudaMemcpyDeviceToHost) != cudaSuccess) {
+    for (uint32_t v = 0; fused && v < h->n; v++) fused = L.dn_first[v + 1] - L.dn_first[v] <= top_chunk_arcs(fbig);
+    if (fused && !h->upin_tried) {   // A-up in-arcs by head, uploaded once
+        h->upin_tried = true;
+        std::vector<uint32_t> f;
+        std::vector<Arc> arc;
+        if (upin_csr(L, h->n, top_chunk_arcs(true), f, arc)) upload_csr(f, arc, &h->d_upin_first, &h->d_upin_arc);
+    }
+    std::vector<uint32_t> uf;
+    if (fused && h->d_upin_first) {
+        uf.resize((size_t)h->n + 1);
+        if (cudaMemcpy(uf.data(), h->d_upin_first, uf.size() * 4, cudaMemcpyDeviceToHost) != cudaSuccess) {
             cudaGetLastError();
             return nullptr;
         }
-        for (uint32_t v = 0; fused && v < h->n; v++) fused = f[v + 1] - f[v] <= ECHf;
+        for (uint32_t v = 0; fused && v < h->n; v++) fused = uf[v + 1] - uf[v] <= top_chunk_arcs(fbig);
     } else {
         fused = false;
     }
     if (fused) {
-        for (uint32_t j = nseg; j-- > 0;) push_chunks(ch, f.data(), L.lvl_off[j], L.lvl_off[j + 1], fbig);   // ascending levels
+        for (uint32_t j = nseg; j-- > 0;) push_chunks(ch, uf.data(), L.lvl_off[j], L.lvl_off[j + 1], fbig);   // ascending
         T.a.split = (uint32_t)ch.size();
         for (uint32_t j = 0; j < nseg; j++) push_chunks(ch, L.dn_first.data(), L.lvl_off[j], L.lvl_off[j + 1], fbig);
         T.a.big = fbig;
         T.a.first[0] = h->d_upin_first;
         T.a.arcs[0] = h->d_upin_arc;
         T.a.fused = 1;
-        T.J = T.J2 = nseg;
+        T.J = nseg;
         T.a.V = h->n;
     } else {
-        const char* env = std::getenv("PHAST_TOP");   // PHAST_TOP=0: no shared-memory top launch
+        if (h->q.flags & PHAST_Q_NO_TOP) return nullptr;
         uint64_t vmax = vmax_budget;
-        if (const char* e = std::getenv("PHAST_TOP_MAXV")) vmax = std::min<uint64_t>(vmax, (uint64_t)std::atoll(e));
+        if (h->q.top_max_vertices) vmax = std::min<uint64_t>(vmax, h->q.top_max_vertices);
         uint32_t J = 0;
         while (J < nseg) {
             const uint32_t a = L.lvl_off[J], b = L.lvl_off[J + 1];
             if (b > vmax || (uint64_t)(b - a) * G > 32ull * 992) break;
             bool fits = true;
-            for (uint32_t v = a; v < b && fits; v++) fits = L.dn_first[v + 1] - L.dn_first[v] <= ECH;
+            for (uint32_t v = a; v < b && fits; v++) fits = L.dn_first[v + 1] - L.dn_first[v] <= top_chunk_arcs(false);
             if (!fits) break;
             J++;
         }
-        if (J < 2 || (env && std::atoi(env) == 0)) J = 0;
-        // hybrid upward search (PHAST_UP_HYBRID=0 disables): the upward kernel expands
-        // only vertices below the top levels; the top kernel finishes G-up inside
-        // [0, V) with a pull pass in ascending level order (reading R9), then sweeps
-        // G-down.  Exact: a G-up path only climbs, so it enters [0, V) once and its part
-        // below V is found by the search, its part inside by the pull pass.
+        if (J < 2) return nullptr;
+        // hybrid upward search: the upward kernel expands only vertices below the top
+        // levels; the top kernel finishes G-up inside [0, V) with a pull pass in
+        // ascending level order (reading R9), then sweeps G-down.  Exact: a G-up path
+        // only climbs, so it enters [0, V) once and its part below V is found by the
+        // search, its part inside by the pull pass.
         // When: the upward searches run beside the previous batch's sweep (side stream),
         // so moving work from them into the top kernel only pays when they are the
         // critical path, i.e. when a sweep is shorter than the searches: estimated sweep
         // 8kn B at ~5 TB/s vs ~2 us per search wave (<= one per level).  Measured (r43):
         // C2 k=16 14.1 vs 14.9 us/tree, C2D 50.9 vs 61.5 (hybrid); C2 k=64 3.87 vs 3.60,
-        // C3 k=64 2.069 vs 2.058 ms/step (full searches).  PHAST_UP_HYBRID=0/1 forces it.
-        const char* he = std::getenv("PHAST_UP_HYBRID");
+        // C3 k=64 2.069 vs 2.058 ms/step (full searches).
         const uint32_t V = L.lvl_off[J];
-        const bool big = J && top_big_fits(k, V);
+        const bool big = top_big_fits(k, V);
         T.a.big = big;
         const double sweep_us = 8.0 * k * h->n / 5e6, search_us = 2.0 * L.levels;
-        const bool hybrid = he ? std::atoi(he) != 0 : sweep_us < search_us;
-        if (J && hybrid) {
-            std::vector<uint32_t> f((size_t)V + 1, 0);
-            for (uint32_t u = 0; u < V; u++)
-                for (uint32_t e = L.up_first[u]; e < L.up_first[u + 1]; e++) f[L.up_arc[e].x + 1]++;
-            for (uint32_t v = 0; v < V; v++) f[v + 1] += f[v];
-            std::vector<Arc> arc(f[V]);
-            std::vector<uint32_t> pos(f.begin(), f.end() - 1);
-            for (uint32_t u = 0; u < V; u++)
-                for (uint32_t e = L.up_first[u]; e < L.up_first[u + 1]; e++)
-                    arc[pos[L.up_arc[e].x]++] = Arc{u, L.up_arc[e].y};
-            bool fits = true;
-            for (uint32_t v = 0; v < V && fits; v++) fits = f[v + 1] - f[v] <= top_chunk_arcs(big);
-            if (fits && !dmalloc(&T.up_f, f.size() + 4) && !dmalloc(&T.up_a, arc.size() + 2) &&
-                cudaMemset(T.up_f, 0, (f.size() + 4) * 4) == cudaSuccess &&
-                cudaMemset(T.up_a, 0, (arc.size() + 2) * 8) == cudaSuccess &&
-                cudaMemcpy(T.up_f, f.data(), f.size() * 4, cudaMemcpyHostToDevice) == cudaSuccess &&
-                (arc.empty() || cudaMemcpy(T.up_a, arc.data(), arc.size() * 8, cudaMemcpyHostToDevice) == cudaSuccess)) {
+        const bool hybrid = (h->q.flags & PHAST_Q_HYBRID_ON) ? true
+                            : (h->q.flags & PHAST_Q_HYBRID_OFF) ? false
+                                                                 : sweep_us < search_us;
+        if (hybrid) {
+            std::vector<uint32_t> f;
+            std::vector<Arc> arc;
+            if (upin_csr(L, V, top_chunk_arcs(big), f, arc) && upload_csr(f, arc, &T.up_f, &T.up_a)) {
                 for (uint32_t j = J; j-- > 0;) push_chunks(ch, f.data(), L.lvl_off[j], L.lvl_off[j + 1], big);
                 T.a.first[0] = T.up_f;
                 T.a.arcs[0] = T.up_a;
                 T.vtop = V;
-            } else {
-                cudaGetLastError();
             }
         }
         T.a.split = (uint32_t)ch.size();
         for (uint32_t j = 0; j < J; j++) push_chunks(ch, L.dn_first.data(), L.lvl_off[j], L.lvl_off[j + 1], big);
         T.J = J;
         T.a.V = V;
-        // the next levels, while small, in one cluster launch (PHAST_CL_SIZE=0 disables;
-        // PHAST_CL_PASSES: max grid-stride passes of the cluster per level, default 8)
-        uint32_t J2 = J;
-        const uint64_t CT = cluster_threads();
-        uint64_t passes = 8;
-        if (const char* e = std::getenv("PHAST_CL_PASSES")) passes = (uint64_t)std::max(1, std::atoi(e));
-        if (CT && h->g.dn_rec)
-            while (J2 + 1 < nseg && (uint64_t)(L.lvl_off[J2 + 1] - L.lvl_off[J2]) * G <= CT * passes) J2++;
-        if (J2 - J < 2) J2 = J;   // not worth a launch
-        if (J == 0 && J2 == 0) return nullptr;
-        if (J2 > J) {
-            if (dmalloc(&T.cl_seg, J2 - J + 1) ||
-                cudaMemcpy(T.cl_seg, L.lvl_off.data() + J, (size_t)(J2 - J + 1) * 4, cudaMemcpyHostToDevice) !=
-                    cudaSuccess) {
-                cudaGetLastError();
-                return nullptr;
-            }
-        }
-        T.J2 = J2;
     }
     const bool none = ch.empty();
     if (none) ch.push_back(make_uint4(0, 0, 0, 0));   // keep a valid device array
-    if (dmalloc(&T.chunks, ch.size()) ||
-        cudaMemcpy(T.chunks, ch.data(), ch.size() * sizeof(uint4), cudaMemcpyHostToDevice) != cudaSuccess) {
+    uint4* dch = nullptr;
+    if (dmalloc(&dch, ch.size()) ||
+        cudaMemcpy(dch, ch.data(), ch.size() * sizeof(uint4), cudaMemcpyHostToDevice) != cudaSuccess) {
         cudaGetLastError();
+        cudaFree(dch);
         return nullptr;
     }
-    T.a.chunks = T.chunks;
+    T.chunks = dch;
+    T.a.chunks = dch;
     T.a.nchunks = none ? 0u : (uint32_t)ch.size();
     T.a.first[1] = h->g.dn_first;
     T.a.arcs[1] = h->g.dn_arc;
-    T.ok = true;
-    if (std::getenv("PHAST_VERBOSE"))
-        std::fprintf(stderr, "%s plan k=%u: %u levels, %u vertices, %u chunks (%u up); cluster levels [%u, %u)\n",
-                     T.a.fused ? "fused" : "top", k, T.J, T.a.V, T.a.nchunks, T.a.split, T.J, T.J2);
     return &T;
 }
 
@@ -704,96 +525,63 @@ cudaEvent_t timing_event(phast_ctx* h) {
     return h->ev[h->ev_used++];
 }
 
-// one full query (a1-a3) for k mapped sources; diam != nullptr: fused max, rows of
-// vertices that are nobody's tail are not stored
-int run_query(phast_ctx* h, const Sources& S, uint32_t k, uint32_t* dist, uint32_t* diam, cudaStream_t st) {
+struct QueryOut {
+    uint32_t* dist;            // rows of the sweep (width kp)
+    uint32_t* diam = nullptr;  // fused max (a5); rows of level 0 are then not stored
+    uint32_t* compact_to = nullptr;   // copy the first kc columns here (padded k)
+    uint32_t kc = 0;
+    bool nogather = false;     // probe A34
+};
+
+// One full query (a0 done; a1-a3, a5) of kp mapped sources on stream st, in the next slot.
+int run_query(phast_ctx* h, const Sources& S, uint32_t kp, const QueryOut& o, cudaStream_t st) {
     cudaEvent_t e0 = nullptr, e1 = nullptr, e2 = nullptr;
     if (h->timing && h->ev_used + 3 <= 3 * MAX_TIMED_BATCHES) {
         e0 = timing_event(h); e1 = timing_event(h); e2 = timing_event(h);
         if (!e0 || !e1 || !e2) return PHAST_ECUDA;
-        cudaEventRecord(e0, st);
+        if (cudaEventRecord(e0, st) != cudaSuccess) return PHAST_ECUDA;
     }
-    phast_ctx::Top* top = get_top(h, k);
-    if (top && top->a.fused) {   // small graph: the whole query (a1-a3, a5) in one launch
-        if (launch_sweep_top(top->a, k, S, dist, h->g.flags, diam, st) != cudaSuccess) return PHAST_ECUDA;
-        if (e1) cudaEventRecord(e1, st);   // no separate upward stage: all of it counts as the sweep
+    phast_ctx::Top* top = get_top(h, kp);
+    const uint32_t s = h->slot_next;
+    h->slot_next = (h->slot_next + 1) % SLOTS;
+    const Slot& sl = h->slot[s];
+    if (top && top->a.fused && !o.nogather) {   // small graph: the whole query (a1-a3, a5) in one launch
+        if (e1) cudaEventRecord(e1, st);          // no separate upward stage: all of it is the sweep
+        if (launch_sweep_top(top->a, kp, S, o.dist, sl.flags, o.diam, st) != cudaSuccess) return PHAST_ECUDA;
+        if (o.compact_to && launch_compact(o.dist, kp, o.compact_to, o.kc, h->n, st) != cudaSuccess)
+            return PHAST_ECUDA;
+        if (cudaEventRecord(h->slot_free[s], st) != cudaSuccess) return PHAST_ECUDA;   // padded scratch reusable
         if (e2) cudaEventRecord(e2, st);
         return PHAST_OK;
     }
-    // a1 on the side stream (overlaps the previous batch's sweep), a2 on the caller's stream
-    const uint32_t slot = h->slot_next;
-    h->slot_next = (h->slot_next + 1) % SEED_SLOTS;
-    if (cudaStreamWaitEvent(h->side, h->slot_free[slot], 0) != cudaSuccess) return PHAST_ECUDA;
-    phast_ctx::Plan* plan = get_plan(h, k);
-    // the top / cluster launches run only on the per-level path (no persistent plan)
-    if (plan || h->L.mode == LAYOUT_DIAGONAL || h->L.lvl_off.empty()) top = nullptr;
-    const uint32_t vtop = (top && top->J) ? top->vtop : 0u;
-    if (launch_upward(h->g, S, k, slot, vtop, h->side) != cudaSuccess) return PHAST_ECUDA;
-    if (cudaEventRecord(h->up_done[slot], h->side) != cudaSuccess) return PHAST_ECUDA;
-    if (cudaStreamWaitEvent(st, h->up_done[slot], 0) != cudaSuccess) return PHAST_ECUDA;
-    if (launch_seed(h->g, k, slot, dist, st) != cudaSuccess) return PHAST_ECUDA;
+    if (top && top->a.fused) top = nullptr;   // the A34 probe runs every level as its own launch
+    // a1 on the side stream (overlaps earlier sweeps), after this slot's previous query
+    if (cudaStreamWaitEvent(h->side, h->slot_free[s], 0) != cudaSuccess) return PHAST_ECUDA;
+    if (launch_upward(h->g, sl, S, kp, top ? top->vtop : 0u, h->side) != cudaSuccess) return PHAST_ECUDA;
+    if (cudaEventRecord(h->up_done[s], h->side) != cudaSuccess) return PHAST_ECUDA;
+    if (cudaStreamWaitEvent(st, h->up_done[s], 0) != cudaSuccess) return PHAST_ECUDA;
+    // a2 on the caller's stream
+    if (launch_seed(h->g, sl, kp, o.dist, st) != cudaSuccess) return PHAST_ECUDA;
     if (e1) cudaEventRecord(e1, st);
-    if (plan && plan->bottom_from) {   // top levels one launch each, then the bottom diagonals in one launch
-        for (uint32_t j = 0; j < plan->bottom_from; j++)
-            if (launch_sweep_level(h->g, k, h->L.lvl_off[j], h->L.lvl_off[j + 1], dist, diam, true, false, false,
-                                   st) != cudaSuccess)
-                return PHAST_ECUDA;
-        if ((uint64_t)(plan->epoch + 1) * plan->p.grid >= 0x7FFFFFFFull) {
-            if (cudaMemsetAsync(plan->p.wave_done, 0, (size_t)plan->p.iters * 4, st) != cudaSuccess) return PHAST_ECUDA;
-            plan->epoch = 0;
-        }
-        plan->epoch++;
-        if (launch_sweep_persistent(h->g, plan->p, plan->epoch, dist, diam, st) != cudaSuccess) return PHAST_ECUDA;
-    } else if (plan && plan->top_levels == 0) {   // a3 + a4: one persistent launch, dataflow over chunks
-        if ((plan->p.variant < 2 || plan->p.variant == 6) && (uint64_t)(plan->epoch + 1) * plan->p.grid >= 0x7FFFFFFFull) {
-            if (cudaMemsetAsync(plan->p.wave_done, 0, (size_t)plan->p.iters * 4, st) != cudaSuccess) return PHAST_ECUDA;
-            plan->epoch = 0;
-        }
-        if (plan->p.variant == 5 &&
-            (uint64_t)(plan->epoch + 1) * (plan->p.workers / sweep_wave_subcounters()) >= 0x7FFFFFFFull) {
-            if (cudaMemsetAsync(plan->p.wave_done, 0,
-                                (size_t)sweep_wave_subcounters() * plan->p.chunk_cap * 4, st) != cudaSuccess)
-                return PHAST_ECUDA;
-            plan->epoch = 0;
-        }
-        plan->epoch++;
-        if (launch_sweep_persistent(h->g, plan->p, plan->epoch, dist, diam, st) != cudaSuccess) return PHAST_ECUDA;
-    } else if (!h->L.lvl_off.empty()) {   // one launch per level (§VI), level layout only
-        const uint32_t levels = (uint32_t)h->L.lvl_off.size() - 1;   // segments
-        const bool diagonal = h->L.mode == LAYOUT_DIAGONAL;
-        uint32_t j0 = 0;
-        if (top) {                            // the small top levels in one single-CTA launch,
-            if (top->J && launch_sweep_top(top->a, k, S, dist, h->g.flags, diam, st) != cudaSuccess)
-                return PHAST_ECUDA;
-            if (top->J2 > top->J &&           // the next small ones in one cluster launch
-                launch_sweep_cluster(h->g, k, top->cl_seg, top->J2 - top->J, dist, diam, st) != cudaSuccess)
-                return PHAST_ECUDA;
-            j0 = top->J2;
-        } else if (plan) {                    // hybrid: small top levels in one persistent launch
-            if ((uint64_t)(plan->epoch + 1) * plan->p.grid >= 0x7FFFFFFFull) {
-                if (cudaMemsetAsync(plan->p.wave_done, 0, (size_t)plan->p.iters * 4, st) != cudaSuccess)
-                    return PHAST_ECUDA;
-                plan->epoch = 0;
-            }
-            plan->epoch++;
-            if (launch_sweep_persistent(h->g, plan->p, plan->epoch, dist, diam, st) != cudaSuccess)
-                return PHAST_ECUDA;
-            j0 = plan->top_levels;
-        }
-        for (uint32_t j = j0; j < levels; j++) {
-            bool last = (j + 1 == levels);
-            bool store = !(diam && last);   // level-0 rows are never read again (diameter mode)
-            const bool by_tail = diagonal && j >= h->L.levels - h->L.cut;   // diagonals mix levels
-            if (launch_sweep_level(h->g, k, h->L.lvl_off[j], h->L.lvl_off[j + 1], dist, diam, store, last, by_tail,
-                                   st) !=
-                cudaSuccess)
-                return PHAST_ECUDA;
-        }
-    } else {
-        return PHAST_EINTERNAL;
+    // a3 + a4: the small top levels in one single-CTA launch, then one launch per level
+    // (§VI "The CPU starts, for each level i, a kernel on the GPU")
+    const uint32_t levels = (uint32_t)h->L.lvl_off.size() - 1;
+    uint32_t j0 = 0;
+    if (top) {
+        if (launch_sweep_top(top->a, kp, S, o.dist, sl.flags, o.diam, st) != cudaSuccess) return PHAST_ECUDA;
+        j0 = top->J;
     }
-    if (launch_clear_flags(h->g, k, slot, st) != cudaSuccess) return PHAST_ECUDA;
-    if (cudaEventRecord(h->slot_free[slot], st) != cudaSuccess) return PHAST_ECUDA;   // seeds of `slot` consumed
+    for (uint32_t j = j0; j < levels; j++) {
+        const bool last = (j + 1 == levels);
+        const bool store = !(o.diam && last);   // level-0 rows are never read again (diameter mode)
+        if (launch_sweep_level(h->g, sl.flags, kp, h->L.lvl_off[j], h->L.lvl_off[j + 1], o.dist, o.diam, store, last,
+                               o.nogather, st) != cudaSuccess)
+            return PHAST_ECUDA;
+    }
+    if (launch_clear_flags(sl, kp, h->g.seed_cap, st) != cudaSuccess) return PHAST_ECUDA;
+    if (o.compact_to && launch_compact(o.dist, kp, o.compact_to, o.kc, h->n, st) != cudaSuccess) return PHAST_ECUDA;
+    // the slot (visited bits, search space, padded scratch) is free for the query SLOTS later
+    if (cudaEventRecord(h->slot_free[s], st) != cudaSuccess) return PHAST_ECUDA;
     if (e2) cudaEventRecord(e2, st);
     return PHAST_OK;
 }
@@ -810,30 +598,29 @@ ChOptions to_ch_options(const phast_opts* o) {
 }
 
 int ensure_in_csr(phast_ctx* h) {
+    if (h->d_in_first) return PHAST_OK;   // the original in-CSR, uploaded on first use (parents, centrality)
+    uint32_t* f = nullptr;
+    uint2* a = nullptr;
     int rc;
-    if (!h->d_in_first) {   // upload the original in-CSR on first use (parents, betweenness)
-        uint32_t* f = nullptr;
-        uint2* a = nullptr;
-        if ((rc = dmalloc(&f, h->L.in_first.size())) || (rc = dmalloc(&a, h->L.in_arc.size() + 1))) {
-            cudaFree(f);
-            return rc;
-        }
-        if (cudaMemcpy(f, h->L.in_first.data(), h->L.in_first.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess ||
-            (!h->L.in_arc.empty() &&
-             cudaMemcpy(a, h->L.in_arc.data(), h->L.in_arc.size() * 8, cudaMemcpyHostToDevice) != cudaSuccess)) {
-            cudaGetLastError();
-            cudaFree(f);
-            cudaFree(a);
-            return PHAST_ECUDA;
-        }
-        h->d_in_first = f;
-        h->d_in_arc = a;
+    if ((rc = dmalloc(&f, h->L.in_first.size())) || (rc = dmalloc(&a, h->L.in_arc.size() + 1))) {
+        cudaFree(f);
+        return rc;
     }
+    if (cudaMemcpy(f, h->L.in_first.data(), h->L.in_first.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess ||
+        (!h->L.in_arc.empty() &&
+         cudaMemcpy(a, h->L.in_arc.data(), h->L.in_arc.size() * 8, cudaMemcpyHostToDevice) != cudaSuccess)) {
+        cudaGetLastError();
+        cudaFree(f);
+        cudaFree(a);
+        return PHAST_ECUDA;
+    }
+    h->d_in_first = f;
+    h->d_in_arc = a;
     return PHAST_OK;
 }
 
 // Original out-arcs by tail {head, len} in internal ids: the transpose of L.in_arc
-// (betweenness delta pass), uploaded on first use.
+// (betweenness backward passes), uploaded on first use.
 int ensure_out_csr(phast_ctx* h) {
     if (h->d_out_first) return PHAST_OK;
     const uint32_t n = h->n;
@@ -865,15 +652,77 @@ int ensure_out_csr(phast_ctx* h) {
     return PHAST_OK;
 }
 
-int ensure_scratch(phast_ctx* h, size_t elems) {
-    if (h->dist_scratch_elems >= elems) return PHAST_OK;
-    cudaFree(h->dist_scratch);
-    h->dist_scratch = nullptr;
-    h->dist_scratch_elems = 0;
-    int rc = dmalloc(&h->dist_scratch, elems);
+// phast_trees for a validated handle on the current device
+int trees(phast_ctx* h, const uint32_t* sources, uint32_t k, uint32_t* dist, cudaStream_t st) {
+    const uint32_t kp = kpad(k);
+    Sources S;
+    int rc = map_sources(h, sources, k, kp, S);
     if (rc) return rc;
-    h->dist_scratch_elems = elems;
+    if (kp == k) {
+        QueryOut o{dist};
+        return run_query(h, S, k, o, st);
+    }
+    // padded: sweep kp trees into this slot's scratch, then copy the k columns out
+    const uint32_t s = h->slot_next;
+    if (cudaStreamWaitEvent(st, h->slot_free[s], 0) != cudaSuccess) return PHAST_ECUDA;   // scratch reuse
+    if ((rc = grow(&h->pad[s], &h->pad_elems[s], (size_t)h->n * kp))) return rc;
+    QueryOut o{h->pad[s]};
+    o.compact_to = dist;
+    o.kc = k;
+    return run_query(h, S, kp, o, st);
+}
+
+int check_handle(const phast_ctx* h) {
+    if (!h) return PHAST_EINVAL;
+    if (h->device < 0) return PHAST_ESTATE;
     return PHAST_OK;
+}
+
+// diameter batches on up to SLOTS library streams: lanes whose label buffers fit 2 GiB
+uint32_t diameter_lanes(const phast_ctx* h, uint32_t kp, uint64_t nb) {
+    const uint64_t bytes = (uint64_t)h->n * kp * 4;
+    uint64_t lanes = std::max<uint64_t>(1, (2ull << 30) / std::max<uint64_t>(bytes, 1));
+    return (uint32_t)std::min<uint64_t>({lanes, (uint64_t)SLOTS, nb});
+}
+
+int diameter(phast_ctx* h, const uint32_t* sources, uint64_t count, uint32_t k_batch, uint32_t* max_dev,
+             uint32_t* bm, cudaStream_t st) {
+    const uint32_t kp = kpad(k_batch);
+    const uint64_t nb = (count + k_batch - 1) / k_batch;
+    const uint32_t nl = diameter_lanes(h, kp, nb);
+    int rc;
+    for (uint32_t l = 0; l < nl; l++)
+        if ((rc = grow(&h->lane_dist[l], &h->lane_elems[l], (size_t)h->n * kp))) return rc;
+    if (cudaMemsetAsync(bm, 0, nb * 4, st) != cudaSuccess) return PHAST_ECUDA;
+    // fork: every lane starts after the work queued on st so far
+    if (cudaEventRecord(h->fork_ev, st) != cudaSuccess) return PHAST_ECUDA;
+    for (uint32_t l = 0; l < nl; l++)
+        if (cudaStreamWaitEvent(h->lane[l], h->fork_ev, 0) != cudaSuccess) return PHAST_ECUDA;
+    for (uint64_t b = 0; b < nb; b++) {
+        Sources S;
+        const uint64_t base = b * k_batch;
+        for (uint32_t i = 0; i < kp; i++) {
+            const uint64_t idx = i < k_batch && base + i < count ? base + i : base;   // pad: duplicates
+            S.s[i] = h->L.perm[sources[idx]];
+        }
+        for (uint32_t i = kp; i < KMAX; i++) S.s[i] = 0;
+        const uint32_t l = (uint32_t)(b % nl);
+        QueryOut o{h->lane_dist[l]};
+        o.diam = bm + b;
+        if ((rc = run_query(h, S, kp, o, h->lane[l]))) return rc;
+    }
+    // join
+    for (uint32_t l = 0; l < nl; l++)
+        if (cudaEventRecord(h->lane_ev[l], h->lane[l]) != cudaSuccess || cudaStreamWaitEvent(st, h->lane_ev[l], 0) != cudaSuccess)
+            return PHAST_ECUDA;
+    if (launch_max_reduce(bm, (uint32_t)nb, max_dev, st) != cudaSuccess) return PHAST_ECUDA;
+    return PHAST_OK;
+}
+
+int batch_max_buffer(phast_ctx* h, uint64_t nb, uint32_t** bm) {
+    int rc = grow(&h->batch_max_scratch, &h->batch_max_elems, nb);
+    *bm = h->batch_max_scratch;
+    return rc;
 }
 
 }  // namespace
@@ -886,10 +735,10 @@ int phast_build(uint32_t n, const uint64_t* first, const uint32_t* head, const u
     *out = nullptr;
     int rc = validate_csr(n, first, head, len);
     if (rc) return rc;
+    const uint32_t flags = opts ? opts->flags : 0u;
+    if (flags & ~(PHAST_FLAG_HOST_ONLY | PHAST_FLAG_LEVEL_LAYOUT | PHAST_FLAG_BFS_IN_LEVEL)) return PHAST_EINVAL;
     std::unique_ptr<phast_ctx> h(new (std::nothrow) phast_ctx());
     if (!h) return PHAST_ENOMEM;
-    uint32_t flags = opts ? opts->flags : 0u;
-    uint32_t delta = (opts && opts->delta) ? opts->delta : DEFAULT_DELTA;
     try {
         ChResult R;
         rc = ch_build(n, first, head, len, to_ch_options(opts), R);
@@ -898,17 +747,15 @@ int phast_build(uint32_t n, const uint64_t* first, const uint32_t* head, const u
         h->m = first[n];
         h->shortcuts = R.shortcuts;
         h->rounds = R.rounds;
-        const uint32_t mode = (flags & PHAST_FLAG_DIAGONAL)    ? LAYOUT_DIAGONAL
-                              : (flags & PHAST_FLAG_WAVEFRONT) ? LAYOUT_WAVEFRONT
-                              : ((flags & PHAST_FLAG_LEVEL_LAYOUT) && !(flags & PHAST_FLAG_BFS_IN_LEVEL))
+        const uint32_t mode = ((flags & PHAST_FLAG_LEVEL_LAYOUT) && !(flags & PHAST_FLAG_BFS_IN_LEVEL))
                                   ? LAYOUT_LEVELS
                                   : LAYOUT_LEVELS_BFS;
-        rc = layout_build(R, first, head, mode, delta, h->L);
+        rc = layout_build(R, first, head, mode, h->L);
         h->build_seconds = R.seconds;
         if (rc) return rc;
         rc = build_in_csr(h->L, n, first, head, len);
         if (rc) return rc;
-        compute_tail_bits(h.get());
+        count_tails(h.get());
     } catch (const std::bad_alloc&) {
         return PHAST_ENOMEM;
     }
@@ -920,63 +767,76 @@ int phast_build(uint32_t n, const uint64_t* first, const uint32_t* head, const u
     return PHAST_OK;
 }
 
-int phast_trees(phast_ctx* h, const uint32_t* sources, uint32_t k, uint32_t* dist, void* stream) {
-    if (!h || !sources || !dist || !k_ok(k)) return PHAST_EINVAL;
-    if (h->device < 0) return PHAST_ESTATE;
-    if (k % 4 == 0 && ((uintptr_t)dist & 15)) return PHAST_EINVAL;
-    Sources S;
-    int rc = map_sources(h, sources, k, S);
+int phast_configure(phast_ctx* h, const phast_query_opts* q) {
+    int rc = check_handle(h);
     if (rc) return rc;
+    phast_query_opts nq = q ? *q : phast_query_opts{0, 0, 0, 0};
+    const uint32_t known = PHAST_Q_NO_FUSED | PHAST_Q_NO_TOP | PHAST_Q_HYBRID_ON | PHAST_Q_HYBRID_OFF;
+    if ((nq.flags & ~known) || ((nq.flags & PHAST_Q_HYBRID_ON) && (nq.flags & PHAST_Q_HYBRID_OFF)))
+        return PHAST_EINVAL;
+    DeviceGuard dg(h->device);
+    if (!dg.ok || cudaDeviceSynchronize() != cudaSuccess) { cudaGetLastError(); return PHAST_ECUDA; }
+    free_tops(h);
+    free_seeds(h);
+    h->q = nq;
+    return alloc_seeds(h);
+}
+
+int phast_trees(phast_ctx* h, const uint32_t* sources, uint32_t k, uint32_t* dist, void* stream) {
+    int rc = check_handle(h);
+    if (rc) return rc;
+    if (!sources || !dist || !k_valid(k)) return PHAST_EINVAL;
+    if (k % 4 == 0 && kpad(k) == k && ((uintptr_t)dist & 15)) return PHAST_EINVAL;
+    if (((uintptr_t)dist & 3)) return PHAST_EINVAL;
     DeviceGuard dg(h->device);
     if (!dg.ok) return PHAST_ECUDA;
-    return run_query(h, S, k, dist, nullptr, (cudaStream_t)stream);
+    return trees(h, sources, k, dist, (cudaStream_t)stream);
 }
 
 int phast_sync(phast_ctx* h, void* stream) {
-    if (!h) return PHAST_EINVAL;
-    if (h->device < 0) return PHAST_ESTATE;
+    int rc = check_handle(h);
+    if (rc) return rc;
     DeviceGuard dg(h->device);
     cudaError_t ce = cudaStreamSynchronize((cudaStream_t)stream);
     if (ce != cudaSuccess) {
         cudaGetLastError();
-        if (std::getenv("PHAST_VERBOSE")) std::fprintf(stderr, "phast_sync: %s\n", cudaGetErrorString(ce));
         return PHAST_ECUDA;
     }
     uint32_t err = 0;
     if (cudaMemcpy(&err, h->g.err, 4, cudaMemcpyDeviceToHost) != cudaSuccess) return PHAST_ECUDA;
     if (err) {
-        if (std::getenv("PHAST_VERBOSE")) std::fprintf(stderr, "phast_sync: device error word 0x%x\n", err);
         cudaMemset(h->g.err, 0, 4);
-        return (err & 1u) ? PHAST_ERANGE : PHAST_ECUDA;   // bit 0: search-space overflow; bit 1: watchdog
+        return (err & 1u) ? PHAST_ERANGE : PHAST_ECUDA;   // bit 0: over capacity / over 2^53
     }
     return PHAST_OK;
 }
 
 int phast_trees_host(phast_ctx* h, const uint32_t* sources, uint32_t k, uint32_t* host_dist, void* stream) {
-    if (!h || !sources || !host_dist || !k_ok(k)) return PHAST_EINVAL;
-    if (h->device < 0) return PHAST_ESTATE;
+    int rc = check_handle(h);
+    if (rc) return rc;
+    if (!sources || !host_dist || !k_valid(k)) return PHAST_EINVAL;
     DeviceGuard dg(h->device);
-    size_t elems = (size_t)h->n * k;
-    int rc = ensure_scratch(h, elems);
-    if (rc) return rc;
-    rc = phast_trees(h, sources, k, h->dist_scratch, stream);
-    if (rc) return rc;
+    if (!dg.ok) return PHAST_ECUDA;
+    const size_t elems = (size_t)h->n * k;
     cudaStream_t st = (cudaStream_t)stream;
-    if (cudaMemcpyAsync(host_dist, h->dist_scratch, elems * 4, cudaMemcpyDeviceToHost, st) != cudaSuccess)
+    if ((rc = grow(&h->host_scratch, &h->host_elems, elems))) return rc;
+    if ((rc = trees(h, sources, k, h->host_scratch, st))) return rc;
+    if (cudaMemcpyAsync(host_dist, h->host_scratch, elems * 4, cudaMemcpyDeviceToHost, st) != cudaSuccess)
         return PHAST_ECUDA;
     return phast_sync(h, stream);
 }
 
 int phast_parents(phast_ctx* h, const uint32_t* sources, uint32_t k, const uint32_t* dist, uint32_t* parent,
                   void* stream) {
-    if (!h || !sources || !dist || !parent || !k_ok(k)) return PHAST_EINVAL;
-    if (h->device < 0) return PHAST_ESTATE;
-    if (k % 4 == 0 && (((uintptr_t)dist & 15) || ((uintptr_t)parent & 15))) return PHAST_EINVAL;
+    int rc = check_handle(h);
+    if (rc) return rc;
+    if (!sources || !dist || !parent || !k_valid(k)) return PHAST_EINVAL;
+    if (k % 4 == 0 && kpad(k) == k && (((uintptr_t)dist & 15) || ((uintptr_t)parent & 15))) return PHAST_EINVAL;
     if (h->L.in_first.size() != (size_t)h->n + 1) return PHAST_ESTATE;
     Sources S;
-    int rc = map_sources(h, sources, k, S);
-    if (rc) return rc;
+    if ((rc = map_sources(h, sources, k, k, S))) return rc;
     DeviceGuard dg(h->device);
+    if (!dg.ok) return PHAST_ECUDA;
     if ((rc = ensure_in_csr(h))) return rc;
     if (launch_parents(h->d_in_first, h->d_in_arc, h->n, S, k, dist, parent, (cudaStream_t)stream) != cudaSuccess)
         return PHAST_ECUDA;
@@ -985,41 +845,69 @@ int phast_parents(phast_ctx* h, const uint32_t* sources, uint32_t k, const uint3
 
 int phast_diameter(phast_ctx* h, const uint32_t* sources, uint64_t count, uint32_t k_batch, uint32_t* max_dev,
                    uint32_t* batch_max_dev, void* stream) {
-    if (!h || !sources || !max_dev || count == 0 || !k_ok(k_batch)) return PHAST_EINVAL;
-    if (h->device < 0) return PHAST_ESTATE;
+    int rc = check_handle(h);
+    if (rc) return rc;
+    if (!sources || !max_dev || count == 0 || !k_valid(k_batch)) return PHAST_EINVAL;
     for (uint64_t i = 0; i < count; i++)
         if (sources[i] >= h->n) return PHAST_ERANGE;
+    const uint64_t nb = (count + k_batch - 1) / k_batch;
+    if (nb > 0xFFFFFFFFull) return PHAST_ERANGE;
+    DeviceGuard dg(h->device);
+    if (!dg.ok) return PHAST_ECUDA;
+    uint32_t* bm = batch_max_dev;
+    if (!bm && (rc = batch_max_buffer(h, nb, &bm))) return rc;
+    return diameter(h, sources, count, k_batch, max_dev, bm, (cudaStream_t)stream);
+}
+
+int phast_diameter_witness(phast_ctx* h, const uint32_t* sources, uint64_t count, uint32_t k_batch, uint32_t* out,
+                           void* stream) {
+    int rc = check_handle(h);
+    if (rc) return rc;
+    if (!sources || !out || count == 0 || !k_valid(k_batch)) return PHAST_EINVAL;
+    for (uint64_t i = 0; i < count; i++)
+        if (sources[i] >= h->n) return PHAST_ERANGE;
+    const uint32_t kp = kpad(k_batch);
+    const uint64_t nb = (count + k_batch - 1) / k_batch;
+    if (nb > 0xFFFFFFFFull || (uint64_t)h->n * kp >= 0xFFFFFFFFull) return PHAST_ERANGE;
     DeviceGuard dg(h->device);
     if (!dg.ok) return PHAST_ECUDA;
     cudaStream_t st = (cudaStream_t)stream;
-    int rc = ensure_scratch(h, (size_t)h->n * k_batch);
-    if (rc) return rc;
-    uint64_t nb = (count + k_batch - 1) / k_batch;
-    if (nb > 0xFFFFFFFFull) return PHAST_ERANGE;
-    uint32_t* bm = batch_max_dev;
-    if (!bm) {
-        if (h->batch_max_elems < nb) {
-            cudaFree(h->batch_max_scratch);
-            h->batch_max_scratch = nullptr;
-            h->batch_max_elems = 0;
-            rc = dmalloc(&h->batch_max_scratch, nb);
-            if (rc) return rc;
-            h->batch_max_elems = nb;
-        }
-        bm = h->batch_max_scratch;
-    }
-    if (cudaMemsetAsync(bm, 0, nb * 4, st) != cudaSuccess) return PHAST_ECUDA;
-    for (uint64_t b = 0; b < nb; b++) {
-        Sources S;
-        uint64_t base = b * k_batch;
-        for (uint32_t i = 0; i < k_batch; i++) {
-            uint64_t idx = base + i < count ? base + i : base;   // pad with a duplicate (max unchanged)
-            S.s[i] = h->L.perm[sources[idx]];
-        }
-        rc = run_query(h, S, k_batch, h->dist_scratch, bm + b, st);
-        if (rc) return rc;
-    }
-    if (launch_max_reduce(bm, (uint32_t)nb, max_dev, st) != cudaSuccess) return PHAST_ECUDA;
+    uint32_t* bm = nullptr;
+    if ((rc = batch_max_buffer(h, nb, &bm))) return rc;
+    if (!h->wit && (rc = dmalloc(&h->wit, 4))) return rc;
+    if ((rc = diameter(h, sources, count, k_batch, h->wit, bm, st))) return rc;
+    if ((rc = phast_sync(h, stream))) return rc;
+    std::vector<uint32_t> hb(nb);
+    uint32_t D = 0;
+    if (cudaMemcpy(&D, h->wit, 4, cudaMemcpyDeviceToHost) != cudaSuccess ||
+        cudaMemcpy(hb.data(), bm, nb * 4, cudaMemcpyDeviceToHost) != cudaSuccess)
+        return PHAST_ECUDA;
+    out[0] = D;
+    out[1] = out[2] = sources[0];
+    if (D == 0) return PHAST_OK;
+    uint64_t b = 0;
+    while (b < nb && hb[b] != D) b++;
+    if (b == nb) return PHAST_EINTERNAL;
+    // the arg-max batch again, as trees (rows of every level stored), then an on-device argmax
+    const uint64_t base = b * k_batch;
+    const uint32_t kv = (uint32_t)std::min<uint64_t>(k_batch, count - base);
+    std::vector<uint32_t> bs(sources + base, sources + base + kv);
+    if ((rc = grow(&h->lane_dist[0], &h->lane_elems[0], (size_t)h->n * kp))) return rc;
+    Sources S;
+    if ((rc = map_sources(h, bs.data(), kv, kp, S))) return rc;
+    QueryOut o{h->lane_dist[0]};
+    unsigned long long* key = reinterpret_cast<unsigned long long*>(h->wit + 2);
+    if ((rc = run_query(h, S, kp, o, st))) return rc;
+    if (cudaMemsetAsync(key, 0, 8, st) != cudaSuccess ||
+        launch_argmax(h->lane_dist[0], h->n, kp, kv, key, st) != cudaSuccess)
+        return PHAST_ECUDA;
+    if ((rc = phast_sync(h, stream))) return rc;
+    unsigned long long hk = 0;
+    if (cudaMemcpy(&hk, key, 8, cudaMemcpyDeviceToHost) != cudaSuccess) return PHAST_ECUDA;
+    if ((uint32_t)(hk >> 32) != D) return PHAST_EINTERNAL;
+    const uint32_t item = 0xFFFFFFFFu - (uint32_t)(hk & 0xFFFFFFFFull);
+    out[1] = bs[item % kp];
+    out[2] = h->L.iperm[item / kp];
     return PHAST_OK;
 }
 
@@ -1027,11 +915,12 @@ int phast_diameter(phast_ctx* h, const uint32_t* sources, uint64_t count, uint32
 
 namespace {
 // NEXT-3 driver shared by phast_betweenness (out = double cb[n]) and phast_reach
-// (out = uint32 r[n]): per batch the trees, then the fixpoint(s), then the accumulation.
+// (out = uint32 r[n]): per batch the trees, then the Kahn-order passes, then the accumulation.
 int centrality(phast_ctx* h, const uint32_t* sources, uint64_t count, uint32_t k_batch, void* out, bool reach,
                void* stream) {
-    if (!h || !sources || !out || count == 0 || !k_ok(k_batch)) return PHAST_EINVAL;
-    if (h->device < 0) return PHAST_ESTATE;
+    int rc = check_handle(h);
+    if (rc) return rc;
+    if (!sources || !out || count == 0 || !k_valid(k_batch)) return PHAST_EINVAL;
     if (h->L.in_first.size() != (size_t)h->n + 1) return PHAST_ESTATE;
     for (uint64_t i = 0; i < count; i++)
         if (sources[i] >= h->n) return PHAST_ERANGE;
@@ -1044,13 +933,10 @@ int centrality(phast_ctx* h, const uint32_t* sources, uint64_t count, uint32_t k
     DeviceGuard dg(h->device);
     if (!dg.ok) return PHAST_ECUDA;
     cudaStream_t st = (cudaStream_t)stream;
-    const uint32_t n = h->n, k = k_batch;
+    const uint32_t n = h->n, k = kpad(k_batch);   // a batch is k sources (k_batch rounded up)
     const size_t elems = (size_t)n * k;
     if (elems >= 0xFFFFFFFFull) return PHAST_ERANGE;   // items are 32-bit
-    int rc = ensure_scratch(h, elems);
-    if (!rc) rc = ensure_in_csr(h);
-    if (!rc) rc = ensure_out_csr(h);
-    if (rc) return rc;
+    if ((rc = ensure_in_csr(h)) || (rc = ensure_out_csr(h))) return rc;
     constexpr uint32_t R = 30;   // passes per graph launch / host convergence check (multiple of 6)
     if (!h->bc_changed) {
         if ((rc = dmalloc(&h->bc_changed, R)) || (rc = dmalloc(&h->bc_qs, 3))) return rc;
@@ -1060,22 +946,21 @@ int centrality(phast_ctx* h, const uint32_t* sources, uint64_t count, uint32_t k
         }
     }
     if (h->bc_elems < elems) {
-        cudaFree(h->bc_sigma);
-        cudaFree(h->bc_delta);
-        cudaFree(h->bc_q);
+        cudaFree(h->bc_sigma); cudaFree(h->bc_delta); cudaFree(h->bc_q); cudaFree(h->bc_dist);
         h->bc_sigma = h->bc_delta = nullptr;
-        h->bc_q = nullptr;
+        h->bc_q = h->bc_dist = nullptr;
         h->bc_elems = 0;
         if ((rc = dmalloc(&h->bc_sigma, elems)) || (rc = dmalloc(&h->bc_delta, elems)) ||
-            (rc = dmalloc(&h->bc_q, 3 * elems)))
+            (rc = dmalloc(&h->bc_q, 3 * elems)) || (rc = dmalloc(&h->bc_dist, elems)))
             return rc;
         h->bc_elems = elems;
     }
     if (cudaMemsetAsync(out, 0, (size_t)n * (reach ? 4 : 8), st) != cudaSuccess) return PHAST_ECUDA;
-    // Kahn order (kernels.cu): the count kernel fills queue 0; pass p reads queue p%2 with
+    // Kahn order (next.cu): the count kernel fills queue 0; pass p reads queue p%2 with
     // size qs[p%3], appends to queue (p+1)%2 with qs[(p+1)%3], zeroes qs[(p+2)%3]; stop
     // after a pass that readied nothing (<= hop depth of the tight DAG + 1 passes)
-    const BcGraph G{h->d_in_first, h->d_in_arc, h->d_out_first, h->d_out_arc};
+    uint32_t* d = h->bc_dist;
+    const BcGraph G{h->d_in_first, h->d_in_arc, h->d_out_first, h->d_out_arc, h->g.err};
     uint32_t* qbuf[2] = {h->bc_q, h->bc_q + elems};
     uint32_t* cnt = h->bc_q + 2 * elems;
     // R passes (+ clearing the change words before, reading them back after) are one CUDA
@@ -1096,25 +981,7 @@ int centrality(phast_ctx* h, const uint32_t* sources, uint64_t count, uint32_t k
                 if (e[j]) cudaGraphExecDestroy(e[j]);
         }
     } eg{execs};
-    // default: graph-captured chunks of R pass launches; PHAST_BC_PERSIST=1 runs every pass
-    // of a direction in ONE cooperative launch with a grid barrier between passes
-    // (measured slower: the passes are bound by their dependent-load
-    // chains, not by launches)
-    const char* pe = std::getenv("PHAST_BC_PERSIST");
-    const bool persist = pe && pe[0] == '1';
     auto kahn = [&](int which, int backward, auto pass) -> int {
-        if (persist) {
-            if (cudaMemsetAsync(h->bc_qs, 0, 12, st) != cudaSuccess ||
-                launch_bc_count(G, h->dist_scratch, n, k, backward, cnt, qbuf[0], h->bc_qs, st) != cudaSuccess)
-                return PHAST_ECUDA;
-            void* val = which == 0 ? (void*)h->bc_sigma : (void*)h->bc_delta;
-            if (launch_bc_persistent(G, h->dist_scratch, h->bc_sigma, val, k, which, qbuf[0], qbuf[1], h->bc_qs, cnt,
-                                     n + 2, h->g.err, st) != cudaSuccess) {
-                cudaGetLastError();
-                return PHAST_ECUDA;
-            }
-            return PHAST_OK;
-        }
         if (!execs[which]) {
             cudaGraph_t graph = nullptr;
             if (cudaStreamBeginCapture(gs, cudaStreamCaptureModeThreadLocal) != cudaSuccess) return PHAST_ECUDA;
@@ -1143,7 +1010,7 @@ int centrality(phast_ctx* h, const uint32_t* sources, uint64_t count, uint32_t k
         // the count kernel and the chunks run on gs after everything queued on st so far
         if (cudaEventRecord(h->bc_ev, st) != cudaSuccess || cudaStreamWaitEvent(gs, h->bc_ev, 0) != cudaSuccess ||
             cudaMemsetAsync(h->bc_qs, 0, 12, gs) != cudaSuccess ||
-            launch_bc_count(G, h->dist_scratch, n, k, backward, cnt, qbuf[0], h->bc_qs, gs) != cudaSuccess)
+            launch_bc_count(G, d, n, k, backward, cnt, qbuf[0], h->bc_qs, gs) != cudaSuccess)
             return PHAST_ECUDA;
         for (uint64_t it = 0; it <= (uint64_t)n + R; it += R) {
             if (cudaGraphLaunch(execs[which], gs) != cudaSuccess || cudaStreamSynchronize(gs) != cudaSuccess)
@@ -1156,34 +1023,54 @@ int centrality(phast_ctx* h, const uint32_t* sources, uint64_t count, uint32_t k
     };
     uint32_t* hgt = reinterpret_cast<uint32_t*>(h->bc_delta);
     for (uint64_t base = 0; base < count; base += k) {
-        Sources S;
         const uint32_t kv = (uint32_t)std::min<uint64_t>(k, count - base);
-        for (uint32_t i = 0; i < k; i++) S.s[i] = h->L.perm[sources[base + (i < kv ? i : 0)]];
-        if ((rc = run_query(h, S, k, h->dist_scratch, nullptr, st))) return rc;
+        Sources S;
+        if ((rc = map_sources(h, sources + base, kv, k, S))) return rc;
+        QueryOut o{d};
+        if ((rc = run_query(h, S, k, o, st))) return rc;
         if (reach) {
             if (cudaMemsetAsync(hgt, 0, elems * 4, st) != cudaSuccess) return PHAST_ECUDA;
             rc = kahn(2, 1, [&](const BcQueue& Q, uint32_t* ch, cudaStream_t s2) {
-                return launch_bc_back(G, h->dist_scratch, nullptr, hgt, n, k, 1, Q, ch, s2);
+                return launch_bc_back(G, d, nullptr, hgt, n, k, 1, Q, ch, s2);
             });
             if (rc) return rc;
-            if (launch_reach_accum(h->dist_scratch, hgt, (uint32_t*)out, n, k, kv, st) != cudaSuccess)
-                return PHAST_ECUDA;
+            if (launch_reach_accum(d, hgt, (uint32_t*)out, n, k, kv, st) != cudaSuccess) return PHAST_ECUDA;
             continue;
         }
         if (cudaMemsetAsync(h->bc_sigma, 0, elems * 8, st) != cudaSuccess ||
             cudaMemsetAsync(h->bc_delta, 0, elems * 8, st) != cudaSuccess)
             return PHAST_ECUDA;
         rc = kahn(0, 0, [&](const BcQueue& Q, uint32_t* ch, cudaStream_t s2) {
-            return launch_bc_sigma(G, h->dist_scratch, h->bc_sigma, n, k, Q, ch, s2);
+            return launch_bc_sigma(G, d, h->bc_sigma, n, k, Q, ch, s2);
         });
         if (rc) return rc;
         rc = kahn(1, 1, [&](const BcQueue& Q, uint32_t* ch, cudaStream_t s2) {
-            return launch_bc_back(G, h->dist_scratch, h->bc_sigma, h->bc_delta, n, k, 0, Q, ch, s2);
+            return launch_bc_back(G, d, h->bc_sigma, h->bc_delta, n, k, 0, Q, ch, s2);
         });
         if (rc) return rc;
         if (launch_bc_accum(h->bc_delta, (double*)out, n, k, kv, S, st) != cudaSuccess) return PHAST_ECUDA;
     }
     return phast_sync(h, stream);
+}
+
+// upward search space of internal id s: the vertices reachable from s in G-up (the
+// search runs to exhaustion, §III), counted with an epoch-stamped mark
+uint32_t up_space(const Layout& L, uint32_t s, std::vector<uint32_t>& mark, uint32_t epoch,
+                  std::vector<uint32_t>& stack) {
+    uint32_t cnt = 0;
+    stack.clear();
+    stack.push_back(s);
+    mark[s] = epoch;
+    while (!stack.empty()) {
+        const uint32_t v = stack.back();
+        stack.pop_back();
+        cnt++;
+        for (uint32_t e = L.up_first[v]; e < L.up_first[v + 1]; e++) {
+            const uint32_t w = L.up_arc[e].x;
+            if (mark[w] != epoch) { mark[w] = epoch; stack.push_back(w); }
+        }
+    }
+    return cnt;
 }
 }  // namespace
 
@@ -1201,21 +1088,37 @@ int phast_reach(phast_ctx* h, const uint32_t* sources, uint64_t count, uint32_t 
 
 int phast_info(const phast_ctx* h, phast_info_t* o) {
     if (!h || !o) return PHAST_EINVAL;
+    if (!h->up_stats) {   // seeded sample of sources (a fixed odd stride over the ids)
+        const uint32_t n = h->n, cnt = std::min(n, UP_SAMPLE);
+        std::vector<uint32_t> mark(n, 0), stack;
+        double sum = 0;
+        uint32_t mx = 0;
+        for (uint32_t i = 0; i < cnt; i++) {
+            const uint32_t s = (uint32_t)(((uint64_t)i * 2654435761ull + 12345) % n);
+            const uint32_t c = up_space(h->L, s, mark, i + 1, stack);
+            sum += c;
+            mx = std::max(mx, c);
+        }
+        h->up_mean = cnt ? sum / cnt : 0.0;
+        h->up_max = mx;
+        h->up_samples = cnt;
+        h->up_stats = true;
+    }
     std::memset(o, 0, sizeof(*o));
     o->n = h->n;
     o->levels = h->L.levels;
     o->m = h->m;
     o->m_up = h->L.up_arc.size();
     o->m_down = h->L.dn_arc.size();
-    uint64_t nt = 0;
-    for (uint32_t w : h->tail_bits) nt += (uint64_t)__builtin_popcount(w);
-    o->n_tail = nt;
+    o->n_tail = h->n_tail;
     o->shortcuts = h->shortcuts;
     o->rounds = h->rounds;
     o->device = h->device < 0 ? 0xFFFFFFFFu : (uint32_t)h->device;
     o->layout = h->L.mode;
-    o->delta = h->L.delta;
+    o->up_space_samples = h->up_samples;
     o->build_seconds = h->build_seconds;
+    o->mean_up_space = h->up_mean;
+    o->max_up_space = h->up_max;
     return PHAST_OK;
 }
 
@@ -1250,8 +1153,23 @@ int phast_export(const phast_ctx* h, uint32_t* level, uint32_t* dn_first, uint32
     return PHAST_OK;
 }
 
+int phast_schedule(phast_ctx* h, uint32_t k, uint32_t* out) {
+    int rc = check_handle(h);
+    if (rc) return rc;
+    if (!out || !k_valid(k)) return PHAST_EINVAL;
+    DeviceGuard dg(h->device);
+    if (!dg.ok) return PHAST_ECUDA;
+    const phast_ctx::Top* t = get_top(h, kpad(k));
+    const uint32_t levels = (uint32_t)h->L.lvl_off.size() - 1;
+    out[0] = t && t->a.fused ? 1u : 0u;
+    out[1] = t ? t->J : 0u;
+    out[2] = t ? t->a.V : 0u;
+    out[3] = t && t->a.fused ? 0u : levels - (t ? t->J : 0u);
+    return PHAST_OK;
+}
+
 // ---------------------------------------------------------------- save / load
-static const char MAGIC[8] = {'P', 'H', 'A', 'S', 'T', 'B', '2', '3'};
+static const char MAGIC[8] = {'P', 'H', 'A', 'S', 'T', 'B', '2', '4'};
 
 int phast_save(const phast_ctx* h, const char* path) {
     if (!h || !path) return PHAST_EINVAL;
@@ -1259,7 +1177,7 @@ int phast_save(const phast_ctx* h, const char* path) {
     if (!f) return PHAST_EIO;
     const Layout& L = h->L;
     uint64_t hdr[10] = {h->n, L.levels, h->m, h->shortcuts, h->rounds, L.dn_arc.size(), L.up_arc.size(),
-                        L.mode | ((uint64_t)L.cut << 32) | ((uint64_t)L.lag << 56), L.delta, L.lvl_off.size()};
+                        L.mode, 0, L.lvl_off.size()};
     auto wr = [&](const void* p, size_t sz, size_t cnt) { return std::fwrite(p, sz, cnt, f) == cnt; };
     bool ok = wr(MAGIC, 1, 8) && wr(hdr, 8, 10) && wr(&h->build_seconds, 8, 1) && wr(L.perm.data(), 4, h->n) &&
               wr(L.level.data(), 4, h->n) && wr(L.lvl_off.data(), 4, L.lvl_off.size()) &&
@@ -1274,6 +1192,7 @@ int phast_save(const phast_ctx* h, const char* path) {
 int phast_load(const char* path, uint32_t flags, phast_ctx** out) {
     if (!path || !out) return PHAST_EINVAL;
     *out = nullptr;
+    if (flags & ~PHAST_FLAG_HOST_ONLY) return PHAST_EINVAL;
     FILE* f = std::fopen(path, "rb");
     if (!f) return PHAST_EIO;
     std::unique_ptr<phast_ctx> h(new (std::nothrow) phast_ctx());
@@ -1281,14 +1200,14 @@ int phast_load(const char* path, uint32_t flags, phast_ctx** out) {
     uint64_t hdr[10];
     auto rd = [&](void* p, size_t sz, size_t cnt) { return std::fread(p, sz, cnt, f) == cnt; };
     bool ok = h && rd(magic, 1, 8) && std::memcmp(magic, MAGIC, 8) == 0 && rd(hdr, 8, 10) &&
-              rd(&h->build_seconds, 8, 1) && hdr[0] > 0 && hdr[0] < 0xFFFFFFFFull;
+              rd(&h->build_seconds, 8, 1) && hdr[0] > 0 && hdr[0] < 0xFFFFFFFFull &&
+              (hdr[7] == LAYOUT_LEVELS || hdr[7] == LAYOUT_LEVELS_BFS) && hdr[9] == hdr[1] + 1;
     if (ok) {
         Layout& L = h->L;
         try {
             h->n = (uint32_t)hdr[0]; L.levels = (uint32_t)hdr[1]; h->m = hdr[2];
             h->shortcuts = hdr[3]; h->rounds = (uint32_t)hdr[4];
-            L.mode = (uint32_t)hdr[7]; L.cut = (uint32_t)((hdr[7] >> 32) & 0xFFFFFFu);
-            L.lag = std::max(1u, (uint32_t)(hdr[7] >> 56)); L.delta = (uint32_t)hdr[8];
+            L.mode = (uint32_t)hdr[7];
             L.perm.resize(h->n); L.iperm.resize(h->n); L.level.resize(h->n);
             L.lvl_off.resize(hdr[9]);
             L.dn_first.resize((size_t)h->n + 1); L.up_first.resize((size_t)h->n + 1);
@@ -1320,7 +1239,7 @@ int phast_load(const char* path, uint32_t flags, phast_ctx** out) {
         if (h->L.perm[v] >= h->n) return PHAST_EIO;
         h->L.iperm[h->L.perm[v]] = v;
     }
-    compute_tail_bits(h.get());
+    count_tails(h.get());
     if (!(flags & PHAST_FLAG_HOST_ONLY)) {
         int rc = upload(h.get());
         if (rc) return rc;
@@ -1350,16 +1269,17 @@ const char* phast_strerror(int s) {
 }
 
 int phast_timing(phast_ctx* h, int enable) {
-    if (!h) return PHAST_EINVAL;
-    if (h->device < 0) return PHAST_ESTATE;
+    int rc = check_handle(h);
+    if (rc) return rc;
     if (enable) h->ev_used = 0;
     h->timing = enable != 0;
     return PHAST_OK;
 }
 
 int phast_timing_read(phast_ctx* h, double* ms_up, double* ms_sweep, uint64_t* batches) {
-    if (!h || !ms_up || !ms_sweep || !batches) return PHAST_EINVAL;
-    if (h->device < 0) return PHAST_ESTATE;
+    if (!ms_up || !ms_sweep || !batches) return PHAST_EINVAL;
+    int rc = check_handle(h);
+    if (rc) return rc;
     DeviceGuard dg(h->device);
     double a = 0, b = 0;
     for (size_t i = 0; i + 2 < h->ev_used; i += 3) {
@@ -1379,17 +1299,20 @@ int phast_timing_read(phast_ctx* h, double* ms_up, double* ms_sweep, uint64_t* b
     return PHAST_OK;
 }
 
-int phast_plan_stats(const phast_ctx* h, uint32_t k, uint32_t grid, uint64_t* out) {
-    if (!h || !out || !k_ok(k) || grid == 0) return PHAST_EINVAL;
-    ChunkPlan cp;
-    int rc = plan_chunks(h->L, chunk_cap_for(h->L, k, grid), grid, cp);
+int phast_probe(phast_ctx* h, int kind, const uint32_t* sources, uint32_t k, uint32_t* dist, void* stream) {
+    int rc = check_handle(h);
     if (rc) return rc;
-    out[0] = cp.chunks;
-    out[1] = cp.slots;
-    out[2] = cp.pads;
-    out[3] = (cp.slots + grid - 1) / grid;
-    out[4] = chunk_cap_for(h->L, k, grid);
-    return PHAST_OK;
+    if (!dist || !k_valid(k) || kpad(k) != k || (kind != 0 && kind != 1) || (kind == 1 && !sources)) return PHAST_EINVAL;
+    if (k % 4 == 0 && ((uintptr_t)dist & 15)) return PHAST_EINVAL;
+    DeviceGuard dg(h->device);
+    if (!dg.ok) return PHAST_ECUDA;
+    cudaStream_t st = (cudaStream_t)stream;
+    if (kind == 0) return launch_probe_stream(h->g, k, dist, st) == cudaSuccess ? PHAST_OK : PHAST_ECUDA;
+    Sources S;
+    if ((rc = map_sources(h, sources, k, k, S))) return rc;
+    QueryOut o{dist};
+    o.nogather = true;
+    return run_query(h, S, k, o, st);
 }
 
 uint64_t phast_launch_count(void) { return launches(); }

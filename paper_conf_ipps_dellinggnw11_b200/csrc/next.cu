@@ -1,0 +1,335 @@
+// next.cu -- SURVEY.md §8(f) rows built on top of finished trees (never on the
+// hot path of a3):
+//   NEXT-1 parent pointers (§VII-A "we check whether the identity d(v) =
+//          d(u) + l(u,v) holds"), in the ORIGINAL graph (reading R14);
+//   NEXT-3 exact betweenness and reach (§VII-B), readings R16/R17.
+#include <algorithm>
+
+#include "device.cuh"
+#include "kernels.h"
+
+namespace phast {
+namespace {
+constexpr int SWEEP_THREADS = 256;
+// ------------------------------------------------------------------ NEXT-1 parent pointers
+// After a sweep every label is final, so the parent pass has no dependencies: one
+// grid-stride pass over (vertex, 16-byte lane) items.  Each lane owns W trees of the
+// row; it scans v's original in-arcs in input order and keeps, per tree, the tail of
+// the first tight arc (§VII-A).  The identity is tested as d(u) <= d(v)
+// and d(v) - d(u) = l, which equals d(u) + l = d(v) exactly (no 32-bit overflow).
+// The scan stops once every finite tree of the lane has its parent.
+template <int K>
+__global__ void __launch_bounds__(SWEEP_THREADS) parents_kernel(const uint32_t* __restrict__ in_first,
+                                                                const uint2* __restrict__ in_arc,
+                                                                const uint32_t* __restrict__ d,
+                                                                uint32_t* __restrict__ parent, uint32_t n,
+                                                                Sources src) {
+    constexpr uint32_t W = RowT<K>::W;
+    constexpr uint32_t G = K / W;
+    using T = typename RowT<K>::T;
+    const uint64_t total = (uint64_t)n * G;
+    for (uint64_t t = (uint64_t)blockIdx.x * SWEEP_THREADS + threadIdx.x; t < total;
+         t += (uint64_t)gridDim.x * SWEEP_THREADS) {
+        const uint32_t v = (uint32_t)(t / G), lane = (uint32_t)(t % G);
+        const T rv = __ldg(reinterpret_cast<const T*>(d + (size_t)v * K) + lane);
+        const uint32_t* dv = reinterpret_cast<const uint32_t*>(&rv);
+        uint32_t p[W];
+        uint32_t need = 0;
+#pragma unroll
+        for (uint32_t q = 0; q < W; q++) {
+            p[q] = INF;
+            if (dv[q] != INF) need |= 1u << q;
+        }
+        const uint32_t e1 = __ldg(&in_first[v + 1]);
+        for (uint32_t e = __ldg(&in_first[v]); need && e < e1; e++) {
+            const uint2 a = __ldg(&in_arc[e]);
+            const T ru = __ldg(reinterpret_cast<const T*>(d + (size_t)a.x * K) + lane);
+            const uint32_t* du = reinterpret_cast<const uint32_t*>(&ru);
+#pragma unroll
+            for (uint32_t q = 0; q < W; q++)
+                if (((need >> q) & 1u) && du[q] <= dv[q] && dv[q] - du[q] == a.y) {
+                    p[q] = a.x;
+                    need &= ~(1u << q);
+                }
+        }
+#pragma unroll
+        for (uint32_t q = 0; q < W; q++)
+            if (src.s[lane * W + q] == v) p[q] = v;   // the root of tree lane*W+q
+        T out;
+        uint32_t* po = reinterpret_cast<uint32_t*>(&out);
+#pragma unroll
+        for (uint32_t q = 0; q < W; q++) po[q] = p[q];
+        reinterpret_cast<T*>(parent + (size_t)v * K)[lane] = out;
+    }
+}
+
+// any k (the caller's row width is not one of the vector widths): one thread per
+// (vertex, tree) item, same scan and tie rule
+__global__ void __launch_bounds__(SWEEP_THREADS) parents_any_kernel(const uint32_t* __restrict__ in_first,
+                                                                    const uint2* __restrict__ in_arc,
+                                                                    const uint32_t* __restrict__ d,
+                                                                    uint32_t* __restrict__ parent, uint32_t n,
+                                                                    uint32_t k, Sources src) {
+    const uint64_t total = (uint64_t)n * k;
+    for (uint64_t t = (uint64_t)blockIdx.x * SWEEP_THREADS + threadIdx.x; t < total;
+         t += (uint64_t)gridDim.x * SWEEP_THREADS) {
+        const uint32_t v = (uint32_t)(t / k), i = (uint32_t)(t % k);
+        const uint32_t dv = __ldg(&d[t]);
+        uint32_t p = INF;
+        if (dv != INF) {
+            const uint32_t e1 = __ldg(&in_first[v + 1]);
+            for (uint32_t e = __ldg(&in_first[v]); e < e1; e++) {
+                const uint2 a = __ldg(&in_arc[e]);
+                const uint32_t du = __ldg(&d[(size_t)a.x * k + i]);
+                if (du <= dv && dv - du == a.y) { p = a.x; break; }
+            }
+        }
+        if (src.s[i] == v) p = v;
+        parent[t] = p;
+    }
+}
+
+template <int K>
+cudaError_t parents_k(const uint32_t* in_first, const uint2* in_arc, uint32_t n, const Sources& src,
+                      const uint32_t* dist, uint32_t* parent, cudaStream_t st) {
+    constexpr uint32_t G = K / RowT<K>::W;
+    uint64_t blocks = ((uint64_t)n * G + SWEEP_THREADS - 1) / SWEEP_THREADS;
+    blocks = std::min<uint64_t>(blocks, (uint64_t)num_sms() * 8);
+    if (blocks == 0) return cudaSuccess;
+    parents_kernel<K><<<(unsigned)blocks, SWEEP_THREADS, 0, st>>>(in_first, in_arc, dist, parent, n, src);
+    count_launch();
+    return cudaGetLastError();
+}
+
+}  // namespace
+
+cudaError_t launch_parents(const uint32_t* in_first, const uint2* in_arc, uint32_t n, const Sources& src,
+                           uint32_t k, const uint32_t* dist, uint32_t* parent, cudaStream_t st) {
+    if (k == 1 || k == 2 || k == 4 || k == 8 || k == 16 || k == 32 || k == 64) {
+#define CALL_PA(K) parents_k<K>(in_first, in_arc, n, src, dist, parent, st)
+        PHAST_K_SWITCH(k, CALL_PA)
+#undef CALL_PA
+    }
+    uint64_t blocks = ((uint64_t)n * k + SWEEP_THREADS - 1) / SWEEP_THREADS;
+    blocks = std::min<uint64_t>(blocks, (uint64_t)num_sms() * 8);
+    if (blocks == 0) return cudaSuccess;
+    parents_any_kernel<<<(unsigned)blocks, SWEEP_THREADS, 0, st>>>(in_first, in_arc, dist, parent, n, k, src);
+    count_launch();
+    return cudaGetLastError();
+}
+
+// ------------------------------------------------------------------ NEXT-3 betweenness
+// Exact (partial) betweenness on top of k finished trees (§VII-B "c_B(v) =
+// sum_{s != v != t} sigma_st(v)/sigma_st").  Rows are [n][k]
+// like the labels.  With lengths > 0 the tight arcs d(u) + l = d(w) of a tree form a
+// DAG, and sigma (path counts) and delta (Brandes' dependencies) are the unique
+// solutions of
+//   sigma(v) = [v = s] + sum_{tight (u, v)} sigma(u)
+//   delta(v) = sum_{tight (v, w)} sigma(v) / sigma(w) * (1 + delta(w)).
+// Every item (v, i) is computed ONCE, in Kahn order of tree i's tight DAG (below), from
+// final inputs summed in a fixed arc order, so the result does not depend on the
+// schedule.  sigma is an integer held in fp64: exact below 2^53 (the host reports
+// ERANGE if any sigma is not finite).  Values written by earlier passes are read with
+// plain loads (not __ldg): every pass is a separate launch.
+namespace {
+__device__ __forceinline__ bool tight(uint32_t du, uint32_t dv, uint32_t l) {
+    return du <= dv && dv - du == l;   // du + l == dv without 32-bit overflow
+}
+// Schedule (not part of the method): Kahn's topological order of each tree's tight DAG.
+// An item t = v*k + i is computed ONCE, when all its inputs are final: cnt[t] counts the
+// item's unfinished inputs (forward: tight in-arcs; backward: tight out-arcs); a pass
+// computes the items of its queue and, for each dependent whose count drops to zero,
+// appends it to the next queue.  Passes = hop depth of the tight DAG + 1; each pass
+// touches only its frontier.  Queue sizes rotate over three counters: pass p reads
+// qs[p%3], appends with qs[(p+1)%3] and zeroes qs[(p+2)%3].
+__device__ __forceinline__ void bc_push(uint32_t t, uint32_t* q, uint32_t* qs, bool& pushed) {
+    q[atomicAdd(qs, 1u)] = t;
+    pushed = true;
+}
+
+// cnt[t] = number of inputs of item t; items with none start the first queue
+__global__ void __launch_bounds__(256) bc_count_kernel(BcGraph G, const uint32_t* __restrict__ d, uint32_t n,
+                                                       uint32_t k, int backward, uint32_t* cnt, uint32_t* q,
+                                                       uint32_t* qs) {
+    const uint64_t total = (uint64_t)n * k;
+    bool pushed = false;
+    for (uint64_t t = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; t < total;
+         t += (uint64_t)gridDim.x * blockDim.x) {
+        const uint32_t v = (uint32_t)(t / k), i = (uint32_t)(t % k);
+        const uint32_t dv = __ldg(&d[t]);
+        if (dv == INF) continue;
+        uint32_t c = 0;
+        if (!backward) {
+            const uint32_t e1 = __ldg(&G.in_first[v + 1]);
+            for (uint32_t e = __ldg(&G.in_first[v]); e < e1; e++) {
+                const uint2 a = __ldg(&G.in_arc[e]);
+                c += tight(__ldg(&d[(size_t)a.x * k + i]), dv, a.y);
+            }
+        } else {
+            const uint32_t e1 = __ldg(&G.out_first[v + 1]);
+            for (uint32_t e = __ldg(&G.out_first[v]); e < e1; e++) {
+                const uint2 a = __ldg(&G.out_arc[e]);
+                const uint32_t dw = __ldg(&d[(size_t)a.x * k + i]);
+                c += dw != INF && tight(dv, dw, a.y);
+            }
+        }
+        cnt[t] = c;
+        if (c == 0) bc_push((uint32_t)t, q, qs, pushed);
+    }
+    (void)pushed;
+}
+
+// forward pass: sigma(v) = [v = s] + sum over tight (u, v) of sigma(u).  With lengths > 0
+// the source is the only finite item without a tight in-arc, so [v = s] is "no tight
+// in-arc" (no source list in the parameters: the passes are graph-captured once per call)
+__global__ void __launch_bounds__(256) bc_sigma_kernel(BcGraph G, const uint32_t* __restrict__ d, double* sigma,
+                                                       uint32_t k, BcQueue Q, uint32_t* changed) {
+    const uint32_t size = *Q.qs_in;
+    if (blockIdx.x == 0 && threadIdx.x == 0) *Q.qs_clr = 0;
+    bool pushed = false;
+    for (uint32_t x = blockIdx.x * blockDim.x + threadIdx.x; x < size; x += gridDim.x * blockDim.x) {
+        const uint32_t t = Q.q_in[x];
+        const uint32_t v = t / k, i = t % k;
+        const uint32_t dv = __ldg(&d[t]);
+        double acc = 0.0;
+        bool any = false;
+        const uint32_t e1 = __ldg(&G.in_first[v + 1]);
+        for (uint32_t e = __ldg(&G.in_first[v]); e < e1; e++) {
+            const uint2 a = __ldg(&G.in_arc[e]);
+            const size_t u = (size_t)a.x * k + i;
+            if (tight(__ldg(&d[u]), dv, a.y)) {
+                acc += sigma[u];
+                any = true;
+            }
+        }
+        if (!(acc <= 9007199254740992.0)) atomicOr(G.err, 1u);   // > 2^53 or not finite: not exact
+        sigma[t] = any ? acc : 1.0;
+        const uint32_t f1 = __ldg(&G.out_first[v + 1]);
+        for (uint32_t e = __ldg(&G.out_first[v]); e < f1; e++) {
+            const uint2 a = __ldg(&G.out_arc[e]);
+            const uint32_t w = a.x * k + i;
+            const uint32_t dw = __ldg(&d[w]);
+            if (dw != INF && tight(dv, dw, a.y) && atomicSub(&Q.cnt[w], 1u) == 1u) bc_push(w, Q.q_out, Q.qs_out, pushed);
+        }
+    }
+    if (__syncthreads_or(pushed) && threadIdx.x == 0) *changed = 1;
+}
+
+// backward pass; mode 0: delta(v) = sum over tight (v, w) of sigma(v)/sigma(w) (1 + delta(w));
+// mode 1 (reach): height h(v) = max over tight (v, w) of l + h(w), stored as uint32 in
+// `val` (l + h(w) <= d(w) + h(w) - d(v) is at most the largest finite label: no wrap)
+__global__ void __launch_bounds__(256) bc_back_kernel(BcGraph G, const uint32_t* __restrict__ d,
+                                                      const double* __restrict__ sigma, void* val, uint32_t k,
+                                                      int mode, BcQueue Q, uint32_t* changed) {
+    const uint32_t size = *Q.qs_in;
+    if (blockIdx.x == 0 && threadIdx.x == 0) *Q.qs_clr = 0;
+    bool pushed = false;
+    double* delta = static_cast<double*>(val);
+    uint32_t* hgt = static_cast<uint32_t*>(val);
+    for (uint32_t x = blockIdx.x * blockDim.x + threadIdx.x; x < size; x += gridDim.x * blockDim.x) {
+        const uint32_t t = Q.q_in[x];
+        const uint32_t v = t / k, i = t % k;
+        const uint32_t dv = __ldg(&d[t]);
+        const uint32_t e1 = __ldg(&G.out_first[v + 1]);
+        if (mode == 0) {
+            const double sv = __ldg(&sigma[t]);
+            double acc = 0.0;
+            for (uint32_t e = __ldg(&G.out_first[v]); e < e1; e++) {
+                const uint2 a = __ldg(&G.out_arc[e]);
+                const size_t w = (size_t)a.x * k + i;
+                const uint32_t dw = __ldg(&d[w]);
+                if (dw != INF && tight(dv, dw, a.y)) acc += sv / __ldg(&sigma[w]) * (1.0 + delta[w]);
+            }
+            delta[t] = acc;
+        } else {
+            uint32_t acc = 0;
+            for (uint32_t e = __ldg(&G.out_first[v]); e < e1; e++) {
+                const uint2 a = __ldg(&G.out_arc[e]);
+                const size_t w = (size_t)a.x * k + i;
+                const uint32_t dw = __ldg(&d[w]);
+                if (dw != INF && tight(dv, dw, a.y)) acc = max(acc, a.y + hgt[w]);
+            }
+            hgt[t] = acc;
+        }
+        const uint32_t f1 = __ldg(&G.in_first[v + 1]);
+        for (uint32_t e = __ldg(&G.in_first[v]); e < f1; e++) {
+            const uint2 a = __ldg(&G.in_arc[e]);
+            const uint32_t u = a.x * k + i;
+            if (tight(__ldg(&d[u]), dv, a.y) && atomicSub(&Q.cnt[u], 1u) == 1u) bc_push(u, Q.q_out, Q.qs_out, pushed);
+        }
+    }
+    if (__syncthreads_or(pushed) && threadIdx.x == 0) *changed = 1;
+}
+
+
+// c_B(v) += sum over the first kv trees i (in order) with sources[i] != v of delta_i(v)
+__global__ void __launch_bounds__(256) bc_accum_kernel(const double* __restrict__ delta, double* __restrict__ cb,
+                                                       uint32_t n, uint32_t k, uint32_t kv, Sources src) {
+    for (uint32_t v = blockIdx.x * blockDim.x + threadIdx.x; v < n; v += gridDim.x * blockDim.x) {
+        double s = 0.0;
+        for (uint32_t i = 0; i < kv; i++)
+            if (src.s[i] != v) s += __ldg(&delta[(size_t)v * k + i]);
+        cb[v] += s;
+    }
+}
+
+// r(v) = max(r(v), max over the first kv trees of min(d_i(v), h_i(v)))
+__global__ void __launch_bounds__(256) reach_accum_kernel(const uint32_t* __restrict__ d,
+                                                          const uint32_t* __restrict__ hgt, uint32_t* __restrict__ r,
+                                                          uint32_t n, uint32_t k, uint32_t kv) {
+    for (uint32_t v = blockIdx.x * blockDim.x + threadIdx.x; v < n; v += gridDim.x * blockDim.x) {
+        uint32_t m = r[v];
+        for (uint32_t i = 0; i < kv; i++) {
+            const uint32_t dv = __ldg(&d[(size_t)v * k + i]);
+            if (dv != INF) m = max(m, min(dv, __ldg(&hgt[(size_t)v * k + i])));
+        }
+        r[v] = m;
+    }
+}
+
+unsigned bc_blocks(uint64_t items) {
+    uint64_t b = (items + 255) / 256;
+    return (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(b, (uint64_t)num_sms() * 8));
+}
+
+// the passes touch only their queue: a small fixed grid (queue sizes are read on the device)
+unsigned bc_pass_blocks(uint64_t items) { return std::min<unsigned>(bc_blocks(items), (unsigned)num_sms() * 2); }
+
+}  // namespace
+
+cudaError_t launch_bc_count(const BcGraph& G, const uint32_t* d, uint32_t n, uint32_t k, int backward, uint32_t* cnt,
+                            uint32_t* q, uint32_t* qs, cudaStream_t st) {
+    bc_count_kernel<<<bc_blocks((uint64_t)n * k), 256, 0, st>>>(G, d, n, k, backward, cnt, q, qs);
+    count_launch();
+    return cudaGetLastError();
+}
+
+cudaError_t launch_bc_sigma(const BcGraph& G, const uint32_t* d, double* sigma, uint32_t n, uint32_t k,
+                            const BcQueue& Q, uint32_t* changed, cudaStream_t st) {
+    bc_sigma_kernel<<<bc_pass_blocks((uint64_t)n * k), 256, 0, st>>>(G, d, sigma, k, Q, changed);
+    count_launch();
+    return cudaGetLastError();
+}
+
+cudaError_t launch_bc_back(const BcGraph& G, const uint32_t* d, const double* sigma, void* val, uint32_t n, uint32_t k,
+                           int mode, const BcQueue& Q, uint32_t* changed, cudaStream_t st) {
+    bc_back_kernel<<<bc_pass_blocks((uint64_t)n * k), 256, 0, st>>>(G, d, sigma, val, k, mode, Q, changed);
+    count_launch();
+    return cudaGetLastError();
+}
+
+cudaError_t launch_reach_accum(const uint32_t* d, const uint32_t* hgt, uint32_t* r, uint32_t n, uint32_t k, uint32_t kv,
+                               cudaStream_t st) {
+    reach_accum_kernel<<<bc_blocks(n), 256, 0, st>>>(d, hgt, r, n, k, kv);
+    count_launch();
+    return cudaGetLastError();
+}
+
+cudaError_t launch_bc_accum(const double* delta, double* cb, uint32_t n, uint32_t k, uint32_t kv, const Sources& src,
+                            cudaStream_t st) {
+    bc_accum_kernel<<<bc_blocks(n), 256, 0, st>>>(delta, cb, n, k, kv, src);
+    count_launch();
+    return cudaGetLastError();
+}
+
+}  // namespace phast

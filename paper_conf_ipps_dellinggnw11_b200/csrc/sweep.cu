@@ -1,0 +1,478 @@
+// sweep.cu -- PHAST's hot path on sm_100a.
+//
+// a1 upward CH search  : one CTA per source, exact labels in G-up by label-correcting
+//                        relaxation over a shared-memory hash table (global fallback).
+//                        PAPER.md:14 §III "it runs Dijkstra's algorithm from s in G-up,
+//                        stopping when the priority queue becomes empty"; any method
+//                        giving exact G-up distances is valid (reading R9).
+// a2 seed + implicit init: visited bits (§IV-C "we mark vertices visited
+//                        during the CH search with a single bit"), rows of the search
+//                        space reset to INF, then labels scattered (two launches so
+//                        every reset precedes every scatter).
+// a3 downward sweep    : per level, d(v) = min(flag(v) ? d(v) : INF,
+//                        min_{(u,v) in A-down} sat(d(u) + l(u,v))) for k trees at once
+//                        (§III, §IV-B).  k/4 lanes per vertex,
+//                        16-byte label loads per lane.
+// a5 diameter          : max over finite labels fused into the sweep (PAPER.md:20
+//                        §VII-B "making each core keep track of the maximum label it
+//                        encounters"); witness argmax.
+// No tensor cores: the loop is an integer (min,+) gather with no reuse.
+#include <algorithm>
+#include <atomic>
+#include <mutex>
+#include <set>
+#include <utility>
+
+#include "device.cuh"
+#include "kernels.h"
+
+namespace phast {
+
+static std::atomic<uint64_t> g_launches{0};
+uint64_t launches() { return g_launches.load(); }
+void add_launches(int64_t d) { g_launches += (uint64_t)d; }
+void count_launch() { g_launches++; }
+
+int num_sms() {
+    static std::atomic<int> cache[64];
+    int dev = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess) { cudaGetLastError(); return 148; }
+    if (dev < 0 || dev >= 64) return 148;
+    int s = cache[dev].load();
+    if (!s) {
+        if (cudaDeviceGetAttribute(&s, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess || s <= 0) {
+            cudaGetLastError();
+            s = 148;
+        }
+        cache[dev] = s;
+    }
+    return s;
+}
+
+cudaError_t ensure_smem_attr(const void* kernel, int bytes) {
+    static std::mutex mu;
+    static std::set<std::pair<const void*, int>> done;   // (kernel, device)
+    int dev = 0;
+    cudaError_t e = cudaGetDevice(&dev);
+    if (e != cudaSuccess) return e;
+    std::lock_guard<std::mutex> lk(mu);
+    if (done.count({kernel, dev})) return cudaSuccess;
+    e = cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes);
+    if (e == cudaSuccess) done.insert({kernel, dev});
+    return e;
+}
+
+namespace {
+
+constexpr uint32_t EMPTY = 0xFFFFFFFFu;
+constexpr int UP_THREADS = 512;
+constexpr uint32_t UP_SMEM_CAP = 4096;   // shared-memory table entries per source (max)
+
+__device__ __forceinline__ uint32_t hash32(uint32_t x) {
+    x ^= x >> 16; x *= 0x7feb352dU; x ^= x >> 15; x *= 0x846ca68bU; x ^= x >> 16;
+    return x;
+}
+
+// ------------------------------------------------------------------ a1 upward
+struct UpTable {
+    uint32_t* keys;
+    uint32_t* vals;
+    uint32_t* inq;
+    uint32_t* qa;
+    uint32_t* qb;
+    uint32_t cap;  // power of two
+};
+
+struct UpShared {
+    uint32_t qn, nn, used, over, cnt;
+};
+
+// Returns the slot of w (inserting it), or EMPTY when the table is 3/4 full.
+__device__ __forceinline__ uint32_t up_insert(const UpTable& t, uint32_t w, UpShared& c) {
+    const uint32_t mask = t.cap - 1;
+    uint32_t h = hash32(w) & mask;
+    for (uint32_t probe = 0; probe < t.cap; probe++) {
+        const uint32_t k = *((volatile uint32_t*)&t.keys[h]);
+        if (k == w) return h;
+        if (k == EMPTY) {
+            if (atomicAdd(&c.used, 0u) * 4 >= t.cap * 3) return EMPTY;
+            const uint32_t old = atomicCAS(&t.keys[h], EMPTY, w);
+            if (old == EMPTY) { atomicAdd(&c.used, 1u); return h; }
+            if (old == w) return h;
+        }
+        h = (h + 1) & mask;
+    }
+    return EMPTY;
+}
+
+// Label-correcting relaxation of G-up from s, wave-synchronous; on return the
+// table holds exact G-up distances of every vertex reachable from s (Bellman-Ford
+// fixed point with saturating sums).  Returns false on table overflow.
+// vtop > 0: vertices < vtop (the top levels, swept by sweep_top_kernel's G-up pull
+// pass) get their labels from the arcs entering them but are not expanded.
+__device__ bool up_search(const uint32_t* __restrict__ up_first, const uint2* __restrict__ up_arc, uint32_t s,
+                          UpTable t, UpShared& c, uint32_t vtop) {
+    const uint32_t tid = threadIdx.x;
+    for (uint32_t i = tid; i < t.cap; i += blockDim.x) { t.keys[i] = EMPTY; t.vals[i] = INF; t.inq[i] = 0; }
+    __syncthreads();
+    if (tid == 0) {
+        const uint32_t h = hash32(s) & (t.cap - 1);
+        t.keys[h] = s; t.vals[h] = 0; t.inq[h] = 1; t.qa[0] = h;
+        c.qn = s >= vtop ? 1u : 0u; c.nn = 0; c.used = 1; c.over = 0; c.cnt = 0;
+    }
+    __syncthreads();
+    uint32_t* qa = t.qa;
+    uint32_t* qb = t.qb;
+    for (;;) {
+        const uint32_t qn = c.qn;
+        if (qn == 0 || c.over) break;
+        for (uint32_t idx = tid; idx < qn; idx += blockDim.x) {
+            const uint32_t slot = qa[idx];
+            atomicExch(&t.inq[slot], 0u);
+            __threadfence_block();
+            const uint32_t v = t.keys[slot];
+            const uint32_t dv = *((volatile uint32_t*)&t.vals[slot]);
+            const uint32_t e1 = __ldg(&up_first[v + 1]);
+            for (uint32_t e = __ldg(&up_first[v]); e < e1; e++) {
+                const uint2 a = __ldg(&up_arc[e]);
+                const uint32_t nd = sat_add(dv, a.y);
+                if (nd == INF) continue;
+                const uint32_t ws = up_insert(t, a.x, c);
+                if (ws == EMPTY) { c.over = 1; break; }
+                const uint32_t old = atomicMin(&t.vals[ws], nd);
+                if (nd < old && a.x >= vtop) {
+                    __threadfence_block();
+                    if (atomicExch(&t.inq[ws], 1u) == 0u) qb[atomicAdd(&c.nn, 1u)] = ws;
+                }
+            }
+        }
+        __syncthreads();
+        if (tid == 0) { c.qn = c.nn; c.nn = 0; }
+        uint32_t* tmp = qa; qa = qb; qb = tmp;
+        __syncthreads();
+    }
+    const bool ok = !c.over;
+    __syncthreads();
+    return ok;
+}
+
+// a1: search only; the search space goes to the slot's seed buffers (the sweep of
+// the previous batch may still be running: nothing here touches the visited bits or
+// the label rows).
+__global__ void __launch_bounds__(UP_THREADS) upward_kernel(DevImage g, Slot sl, Sources src, uint32_t vtop) {
+    extern __shared__ uint32_t smem[];
+    __shared__ UpShared c;
+    const uint32_t i = blockIdx.x;
+    const uint32_t s = src.s[i];
+    const uint32_t sc = g.smem_cap;
+    UpTable t{smem, smem + sc, smem + 2 * sc, smem + 3 * sc, smem + 4 * sc, sc};
+    bool ok = up_search(g.up_first, g.up_arc, s, t, c, vtop);
+    if (!ok) {   // global-memory fallback with the per-source capacity (searches of one
+                 // handle run on one side stream, one launch at a time: one table set)
+        uint32_t* base = g.gscratch + (size_t)i * g.seed_cap * 5;
+        UpTable gt{base, base + g.seed_cap, base + 2 * (size_t)g.seed_cap, base + 3 * (size_t)g.seed_cap,
+                   base + 4 * (size_t)g.seed_cap, g.seed_cap};
+        t = gt;
+        ok = up_search(g.up_first, g.up_arc, s, t, c, vtop);
+        if (!ok) {
+            if (threadIdx.x == 0) { atomicOr(g.err, 1u); sl.seed_cnt[i] = 0; }
+            return;
+        }
+    }
+    uint32_t* sv = sl.seed_v + (size_t)i * g.seed_cap;
+    uint32_t* sd = sl.seed_d + (size_t)i * g.seed_cap;
+    for (uint32_t e = threadIdx.x; e < t.cap; e += blockDim.x) {
+        const uint32_t v = t.keys[e];
+        if (v == EMPTY) continue;
+        const uint32_t pos = atomicAdd(&c.cnt, 1u);
+        sv[pos] = v;
+        sd[pos] = t.vals[e];
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) sl.seed_cnt[i] = c.cnt;
+}
+
+// ------------------------------------------------------------------ a2 seeding
+// phase 1: visited bits of the search space, and its rows reset to INF
+template <int K>
+__global__ void seed_rows_kernel(Slot sl, uint32_t seed_cap, uint32_t* __restrict__ dist) {
+    const uint32_t i = blockIdx.x;
+    const uint32_t cnt = sl.seed_cnt[i];
+    const uint32_t* sv = sl.seed_v + (size_t)i * seed_cap;
+    for (uint32_t j = threadIdx.x; j < cnt; j += blockDim.x) {
+        const uint32_t v = sv[j];
+        atomicOr(&sl.flags[v >> 5], 1u << (v & 31));
+    }
+    using T = typename RowT<K>::T;
+    constexpr uint32_t G = K / RowT<K>::W;
+    for (uint32_t j = threadIdx.x; j < cnt * G; j += blockDim.x)
+        reinterpret_cast<T*>(dist + (size_t)sv[j / G] * K)[j % G] = inf_row<T>();
+}
+
+// phase 2 (after every reset of phase 1): the labels
+__global__ void scatter_kernel(Slot sl, uint32_t seed_cap, uint32_t k, uint32_t* __restrict__ dist) {
+    const uint32_t i = blockIdx.x;
+    const uint32_t cnt = sl.seed_cnt[i];
+    const uint32_t* sv = sl.seed_v + (size_t)i * seed_cap;
+    const uint32_t* sd = sl.seed_d + (size_t)i * seed_cap;
+    for (uint32_t j = threadIdx.x; j < cnt; j += blockDim.x) dist[(size_t)sv[j] * k + i] = sd[j];
+}
+
+__global__ void clear_flags_kernel(Slot sl, uint32_t seed_cap) {
+    const uint32_t i = blockIdx.x;
+    const uint32_t cnt = sl.seed_cnt[i];
+    const uint32_t* sv = sl.seed_v + (size_t)i * seed_cap;
+    for (uint32_t j = threadIdx.x; j < cnt; j += blockDim.x) sl.flags[sv[j] >> 5] = 0u;
+}
+
+// ------------------------------------------------------------------ a3 sweep
+constexpr int SWEEP_THREADS = 256;
+
+// One level [vbeg, vend) (§VI "The CPU starts, for each level i, a kernel on
+// the GPU").  One (vertex, 16-byte lane) item per thread per grid-stride step; the
+// grid fills every SM (8 CTAs of 256 threads), which keeps the most gathers in flight.
+// Each vertex's first two in-arcs come from one 16-byte ELL-2 record (97 % of level-0
+// and 92 % of level-1 vertices at C3 have at most two), so the tail-row gathers depend
+// on ONE load; more in-arcs continue in the overflow list.  Launched with programmatic
+// dependent launch: the next level's grid is launched while this one drains and blocks
+// in griddepcontrol.wait until this grid's rows are visible; the graph is static, so
+// the first record is prefetched into L2 before the wait.
+// NOGATHER (probe A34, §VIII-B "it takes 153 ms to traverse the graph
+// exactly as PHAST does, but storing at d(v) the sum of the lengths of all arcs into
+// v"): identical traversal, with every tail row replaced by the arc's length.
+template <int K, bool DIAM, bool STORE, bool STREAM, bool NOGATHER>
+__global__ void __launch_bounds__(SWEEP_THREADS, 8)
+    sweep_kernel(const uint4* __restrict__ rec, const uint2* __restrict__ ovf, uint32_t* __restrict__ d,
+                 const uint32_t* __restrict__ flags, uint32_t vbeg, uint32_t vend, uint32_t* __restrict__ diam) {
+    using T = typename RowT<K>::T;
+    constexpr uint32_t G = K / RowT<K>::W;   // lanes per vertex
+    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+    const uint32_t total = (vend - vbeg) * G;   // host: < 2^31 (sweep_launch splits longer levels)
+    uint32_t t = blockIdx.x * SWEEP_THREADS + threadIdx.x;
+    if (t < total) asm volatile("prefetch.global.L2 [%0];" ::"l"(rec + vbeg + t / G));
+    asm volatile("griddepcontrol.wait;" ::: "memory");   // previous level complete and visible
+    uint32_t mx = 0;
+    for (; t < total; t += gridDim.x * SWEEP_THREADS) {
+        const uint32_t v = vbeg + t / G;
+        const uint32_t lane = t % G;
+        T acc = inf_row<T>();
+        if (visited(flags, v)) acc = __ldg(reinterpret_cast<const T*>(d + (size_t)v * K) + lane);
+        const uint4 r = __ldg(&rec[v]);
+        T x0 = inf_row<T>(), x1 = inf_row<T>();
+        if constexpr (NOGATHER) {
+            acc = splat<T>(min(r.y, 0xFFFFFFFEu) + (r.w == INF ? 0u : r.w));
+        } else {
+            // a missing arc has len INF: relaxing an INF row by it changes nothing
+            if (r.y != INF) x0 = __ldg(reinterpret_cast<const T*>(d + (size_t)r.x * K) + lane);
+            if (r.w != INF) x1 = __ldg(reinterpret_cast<const T*>(d + (size_t)r.z * K) + lane);
+            acc = relax(relax(acc, x0, r.y), x1, r.w);
+        }
+        if (r.w == INF && r.z != INF) {   // more than two in-arcs: the rest in the overflow list
+            const uint2* o = ovf + r.z;
+            const uint32_t cnt = __ldg(&o->x);
+            for (uint32_t j = 1; j <= cnt; j++) {
+                const uint2 a = __ldg(&o[j]);
+                if constexpr (NOGATHER) acc = splat<T>(sat_add(fmax_of(acc), a.y));
+                else acc = relax(acc, __ldg(reinterpret_cast<const T*>(d + (size_t)a.x * K) + lane), a.y);
+            }
+        }
+        if constexpr (STORE) {
+            T* p = reinterpret_cast<T*>(d + (size_t)v * K) + lane;
+            if constexpr (STREAM) __stcs(p, acc); else *p = acc;
+        }
+        if constexpr (DIAM) mx = max(mx, fmax_of(acc));
+    }
+    if constexpr (DIAM) cta_max_to<SWEEP_THREADS>(mx, diam);
+}
+
+template <int K, bool DIAM, bool STORE, bool STREAM, bool NOGATHER>
+cudaError_t sweep_launch(const DevImage& g, const uint32_t* flags, uint32_t vbeg, uint32_t vend, uint32_t* dist,
+                         uint32_t* diam, cudaStream_t st) {
+    constexpr uint32_t G = K / RowT<K>::W;
+    constexpr uint32_t VMAX = (1u << 31) / G;   // 32-bit item indices in the kernel
+    if (vend - vbeg > VMAX) {                    // a level has no internal arcs: split it freely
+        cudaError_t e = sweep_launch<K, DIAM, STORE, STREAM, NOGATHER>(g, flags, vbeg, vbeg + VMAX, dist, diam, st);
+        return e != cudaSuccess ? e
+                                : sweep_launch<K, DIAM, STORE, STREAM, NOGATHER>(g, flags, vbeg + VMAX, vend, dist,
+                                                                                 diam, st);
+    }
+    const uint64_t total = (uint64_t)(vend - vbeg) * G;
+    uint64_t blocks = (total + SWEEP_THREADS - 1) / SWEEP_THREADS;
+    const uint64_t cap = (uint64_t)num_sms() * 8;   // one full wave of resident CTAs (launch bounds: 8)
+    if (blocks > cap) blocks = cap;
+    if (blocks == 0) return cudaSuccess;
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3((unsigned)blocks);
+    cfg.blockDim = dim3(SWEEP_THREADS);
+    cfg.dynamicSmemBytes = 0;
+    cfg.stream = st;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    cudaError_t e = cudaLaunchKernelEx(&cfg, sweep_kernel<K, DIAM, STORE, STREAM, NOGATHER>, g.dn_rec, g.dn_ovf,
+                                       dist, flags, vbeg, vend, diam);
+    count_launch();
+    return e;
+}
+
+template <int K>
+cudaError_t sweep_k(const DevImage& g, const uint32_t* flags, uint32_t vbeg, uint32_t vend, uint32_t* dist,
+                    uint32_t* diam, bool store, bool last, bool nogather, cudaStream_t st) {
+    if (nogather) return sweep_launch<K, false, true, false, true>(g, flags, vbeg, vend, dist, diam, st);
+    if (diam) {
+        if (!store) return sweep_launch<K, true, false, false, false>(g, flags, vbeg, vend, dist, diam, st);
+        return last ? sweep_launch<K, true, true, true, false>(g, flags, vbeg, vend, dist, diam, st)
+                    : sweep_launch<K, true, true, false, false>(g, flags, vbeg, vend, dist, diam, st);
+    }
+    return last ? sweep_launch<K, false, true, true, false>(g, flags, vbeg, vend, dist, diam, st)
+                : sweep_launch<K, false, true, false, false>(g, flags, vbeg, vend, dist, diam, st);
+}
+
+// ------------------------------------------------------------------ probe A33
+// Sequential stream over the sweep's arrays: every ELL record read, every label row
+// read and written once (no gathers, no level dependencies, ONE launch).
+template <int K>
+__global__ void __launch_bounds__(SWEEP_THREADS, 8)
+    probe_stream_kernel(const uint4* __restrict__ rec, uint32_t* __restrict__ d, uint32_t n) {
+    using T = typename RowT<K>::T;
+    constexpr uint32_t G = K / RowT<K>::W;
+    const uint64_t total = (uint64_t)n * G;
+    for (uint64_t t = (uint64_t)blockIdx.x * SWEEP_THREADS + threadIdx.x; t < total;
+         t += (uint64_t)gridDim.x * SWEEP_THREADS) {
+        const uint32_t v = (uint32_t)(t / G), lane = (uint32_t)(t % G);
+        const uint4 r = __ldg(&rec[v]);
+        T* p = reinterpret_cast<T*>(d + (size_t)v * K) + lane;
+        const T x = __ldcs(p);
+        __stcs(p, relax(x, splat<T>(r.x), r.y));
+    }
+}
+
+template <int K>
+cudaError_t probe_stream_k(const DevImage& g, uint32_t* dist, cudaStream_t st) {
+    constexpr uint32_t G = K / RowT<K>::W;
+    uint64_t blocks = ((uint64_t)g.n * G + SWEEP_THREADS - 1) / SWEEP_THREADS;
+    blocks = std::min<uint64_t>(blocks, (uint64_t)num_sms() * 8);
+    if (blocks == 0) return cudaSuccess;
+    probe_stream_kernel<K><<<(unsigned)blocks, SWEEP_THREADS, 0, st>>>(g.dn_rec, dist, g.n);
+    count_launch();
+    return cudaGetLastError();
+}
+
+// ------------------------------------------------------------------ a5 reductions
+__global__ void max_reduce_kernel(const uint32_t* __restrict__ in, uint32_t count, uint32_t* out) {
+    uint32_t mx = 0;
+    for (uint32_t i = threadIdx.x; i < count; i += blockDim.x) mx = max(mx, in[i]);
+    __shared__ uint32_t w[32];
+    mx = __reduce_max_sync(0xFFFFFFFFu, mx);
+    if ((threadIdx.x & 31) == 0) w[threadIdx.x >> 5] = mx;
+    __syncthreads();
+    if (threadIdx.x < 32) {
+        uint32_t x = threadIdx.x < blockDim.x / 32 ? w[threadIdx.x] : 0u;
+        x = __reduce_max_sync(0xFFFFFFFFu, x);
+        if (threadIdx.x == 0) *out = x;
+    }
+}
+
+__global__ void __launch_bounds__(256) argmax_kernel(const uint32_t* __restrict__ d, uint32_t n, uint32_t k,
+                                                     uint32_t kv, unsigned long long* key) {
+    unsigned long long best = 0;
+    const uint64_t total = (uint64_t)n * k;
+    for (uint64_t t = (uint64_t)blockIdx.x * 256 + threadIdx.x; t < total; t += (uint64_t)gridDim.x * 256) {
+        const uint32_t x = __ldg(&d[t]);
+        if (x == INF || (uint32_t)(t % k) >= kv) continue;
+        const unsigned long long c = ((unsigned long long)x << 32) | (0xFFFFFFFFu - (uint32_t)t);
+        best = best > c ? best : c;
+    }
+    for (int o = 16; o; o >>= 1) {
+        const unsigned long long y = __shfl_xor_sync(0xFFFFFFFFu, best, o);
+        best = best > y ? best : y;
+    }
+    if ((threadIdx.x & 31) == 0 && best) atomicMax(key, best);
+}
+
+__global__ void __launch_bounds__(256) compact_kernel(const uint32_t* __restrict__ src, uint32_t ks,
+                                                      uint32_t* __restrict__ dst, uint32_t kd, uint32_t n) {
+    const uint64_t total = (uint64_t)n * kd;
+    for (uint64_t t = (uint64_t)blockIdx.x * 256 + threadIdx.x; t < total; t += (uint64_t)gridDim.x * 256) {
+        const uint64_t r = t / kd;
+        __stcs(dst + t, __ldcs(src + r * ks + (t - r * kd)));
+    }
+}
+
+unsigned grid_for(uint64_t items) {
+    const uint64_t b = (items + 255) / 256;
+    return (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(b, (uint64_t)num_sms() * 8));
+}
+
+template <int K>
+cudaError_t seed_k(const DevImage& g, const Slot& sl, uint32_t* dist, cudaStream_t st) {
+    seed_rows_kernel<K><<<K, 256, 0, st>>>(sl, g.seed_cap, dist);
+    count_launch();
+    return cudaGetLastError();
+}
+
+}  // namespace
+
+cudaError_t launch_upward(const DevImage& g, const Slot& sl, const Sources& src, uint32_t k, uint32_t vtop,
+                          cudaStream_t st) {
+    cudaError_t e = ensure_smem_attr((const void*)upward_kernel, (int)(5 * UP_SMEM_CAP * sizeof(uint32_t)));
+    if (e != cudaSuccess) return e;
+    const size_t smem = 5 * (size_t)g.smem_cap * sizeof(uint32_t);
+    upward_kernel<<<k, UP_THREADS, smem, st>>>(g, sl, src, vtop);
+    count_launch();
+    return cudaGetLastError();
+}
+
+cudaError_t launch_seed(const DevImage& g, const Slot& sl, uint32_t k, uint32_t* dist, cudaStream_t st) {
+#define CALL_SR(K) seed_k<K>(g, sl, dist, st)
+    cudaError_t e = [&]() -> cudaError_t { PHAST_K_SWITCH(k, CALL_SR) }();
+#undef CALL_SR
+    if (e != cudaSuccess) return e;
+    scatter_kernel<<<k, 256, 0, st>>>(sl, g.seed_cap, k, dist);
+    count_launch();
+    return cudaGetLastError();
+}
+
+cudaError_t launch_sweep_level(const DevImage& g, const uint32_t* flags, uint32_t k, uint32_t vbeg, uint32_t vend,
+                               uint32_t* dist, uint32_t* diam, bool store, bool last_level, bool nogather,
+                               cudaStream_t st) {
+#define CALL_SW(K) sweep_k<K>(g, flags, vbeg, vend, dist, diam, store, last_level, nogather, st)
+    PHAST_K_SWITCH(k, CALL_SW)
+#undef CALL_SW
+}
+
+cudaError_t launch_clear_flags(const Slot& sl, uint32_t k, uint32_t seed_cap, cudaStream_t st) {
+    clear_flags_kernel<<<k, 256, 0, st>>>(sl, seed_cap);
+    count_launch();
+    return cudaGetLastError();
+}
+
+cudaError_t launch_max_reduce(const uint32_t* in, uint32_t count, uint32_t* out, cudaStream_t st) {
+    max_reduce_kernel<<<1, 1024, 0, st>>>(in, count, out);
+    count_launch();
+    return cudaGetLastError();
+}
+
+cudaError_t launch_argmax(const uint32_t* d, uint32_t n, uint32_t k, uint32_t kv, unsigned long long* key,
+                          cudaStream_t st) {
+    argmax_kernel<<<grid_for((uint64_t)n * k), 256, 0, st>>>(d, n, k, kv, key);
+    count_launch();
+    return cudaGetLastError();
+}
+
+cudaError_t launch_compact(const uint32_t* src, uint32_t ks, uint32_t* dst, uint32_t kd, uint32_t n,
+                           cudaStream_t st) {
+    compact_kernel<<<grid_for((uint64_t)n * kd), 256, 0, st>>>(src, ks, dst, kd, n);
+    count_launch();
+    return cudaGetLastError();
+}
+
+cudaError_t launch_probe_stream(const DevImage& g, uint32_t k, uint32_t* dist, cudaStream_t st) {
+#define CALL_PR(K) probe_stream_k<K>(g, dist, st)
+    PHAST_K_SWITCH(k, CALL_PR)
+#undef CALL_PR
+}
+
+}  // namespace phast

@@ -58,8 +58,11 @@ def test_c1_all_sources(c1):
         assert np.array_equal(gpu_trees(h, [s])[0], want[s])
 
 
-@pytest.mark.parametrize("k", P.K_ALLOWED)
+@pytest.mark.parametrize("k", (1, 2, 3, 4, 5, 7, 8, 12, 16, 17, 31, 32, 33, 48, 63, 64))
 def test_every_k_with_duplicates(road, k):
+    """Every k of the boundary (1 <= k <= 64): the vector widths
+    directly, the others padded to the next width and compacted into the caller's
+    n*k buffer."""
     g, h = road
     src = phastgen.sources(g.n, k, seed=100 + k, distinct=False)
     if k >= 4:
@@ -79,7 +82,7 @@ def test_repeated_calls_no_stale_state(road):
         h.sync()
         assert np.array_equal(h.to_original(out.cpu().numpy()), oracle.sssp_many(g, src)), rep
     # same buffer, alternating k
-    for k in (64, 1, 32, 4):
+    for k in (64, 1, 32, 4, 9, 64):
         src = phastgen.sources(g.n, k, seed=300 + k)
         assert np.array_equal(gpu_trees(h, src), oracle.sssp_many(g, src))
 
@@ -97,7 +100,7 @@ EDGE_GRAPHS = {
 def test_edge_case_graphs(name):
     g = EDGE_GRAPHS[name]()
     with P.Phast.from_graph(g) as h:
-        for k in (1, 16, 64):
+        for k in (1, 13, 16, 64):
             src = phastgen.sources(g.n, k, seed=7 + k)
             assert np.array_equal(gpu_trees(h, src), oracle.sssp_many(g, src)), k
 
@@ -110,7 +113,7 @@ def gpu_parents(h, src):
     return h.to_original(d.cpu().numpy()), h.parents_to_original(p.cpu().numpy())
 
 
-@pytest.mark.parametrize("k", (1, 4, 16, 64))
+@pytest.mark.parametrize("k", (1, 4, 5, 16, 24, 64))
 def test_parents_bit_exact(c1, road, k):
     """NEXT-1 parent pointers (§VII-A tight-arc identity, reading R14):
     bit-exact with the oracle's canonical parents, C1 and a road graph."""
@@ -134,133 +137,84 @@ def test_parents_edge_case_graphs(name):
                 assert np.array_equal(par[i], oracle.parents(g, s)), (k, i)
 
 
-def test_upward_global_fallback_and_overflow(monkeypatch):
+def test_upward_global_fallback_and_overflow():
     """A shared-memory table too small for the search space falls back to the global
     table (same labels); a per-source capacity too small is reported as ERANGE by
     phast_sync (never silently wrong labels)."""
     g = phastgen.grid(100, 100, 1, 1 << 20, seed=1)   # upward spaces ~200-300 vertices
     src = phastgen.sources(g.n, 16, seed=3)
     want = oracle.sssp_many(g, src)
-    monkeypatch.setenv("PHAST_FUSED", "0")             # the upward-search kernel, not the fused pull sweep
-    monkeypatch.setenv("PHAST_UP_HYBRID", "0")         # full searches (the hybrid stops below the top levels)
-    monkeypatch.setenv("PHAST_UP_SMEM_CAP", "32")
+    full_searches = P.Q_NO_FUSED | P.Q_HYBRID_OFF       # the upward kernel, whole searches
     with P.Phast.from_graph(g) as h:
+        h.configure(flags=full_searches, up_smem_cap=32)
         assert np.array_equal(gpu_trees(h, src), want)
-    monkeypatch.setenv("PHAST_SEED_CAP", "32")
-    with P.Phast.from_graph(g) as h:
+        h.configure(flags=full_searches, seed_cap=32)
         h.trees(src)
         with pytest.raises(P.PhastError) as e:
             h.sync()
         assert e.value.status == -4
         h.sync()                                       # error word is cleared
+        h.configure()                                  # defaults again: exact
+        assert np.array_equal(gpu_trees(h, src), want)
 
 
-@pytest.mark.parametrize("mode,level_layout,delta", [("levels", True, 0), ("levels", "bfs", 0),
-                                                     ("levels-hybrid", True, 0), ("levels-flat", "bfs", 0),
-                                                     ("levels-hybrid", "bfs", 0), ("levels-hybrid", "diagonal", 0),
-                                                     ("levels-ab1", "bfs", 0), ("levels-ab3", "bfs", 0),
-                                                     ("levels-ab4", "bfs", 0), ("levels-ab8", "bfs", 0),
-                                                     ("levels-ab8", "diagonal", 0), ("levels-ab16", "bfs", 0),
-                                                     ("levels-ab17", "bfs", 0), ("levels-ab17", True, 0),
-                                                     ("bottomseg2-2", "diagonal", 0), ("bottomseg2-2", "diagonal", 3000),
-                                                     ("bottomseg3-2", "diagonal", 0), ("bottomsegauto-3", "diagonal", 500),
-                                                     ("bottomseg2-1", "diagonal", 2000),
-                                                     ("warp", True, 0), ("staged", True, 0),
-                                                     ("warp", False, 0), ("persistent", False, 0),
-                                                     ("wpipe", False, 0), ("wpipe", False, 300), ("wpipe", True, 0),
-                                                     ("pipe", False, 0), ("pipe", False, 300), ("pipe", True, 0),
-                                                     ("staged", False, 0), ("warp", False, 300),
-                                                     ("staged", False, 300), ("wave", False, 0),
-                                                     ("wave", False, 300), ("wave", True, 0), ("wave", "bfs", 0),
-                                                     ("levels", "diagonal", 0), ("levels", "diagonal", 500),
-                                                     ("segments", True, 0), ("segments", "bfs", 0),
-                                                     ("segments", "diagonal", 0), ("segments", "diagonal", 500)])
-def test_sweep_modes(monkeypatch, mode, level_layout, delta):
-    """Every schedule is bit-exact: one launch per level on the paper's level layout
-    (§VI); the single persistent launch as warp dataflow (default) or CTA
-    waves (with and without bulk-staged arcs), on both layouts, including a small
-    wavefront skew (many short dependencies)."""
-    if mode.startswith("bottomseg"):            # diagonal layout, bottom diagonals in one lagged launch
-        cut, lag = mode[len("bottomseg"):].split("-")
-        monkeypatch.setenv("PHAST_BOTTOM_SEG", "1")
-        monkeypatch.setenv("PHAST_DIAG_LAG", lag)
-        if cut != "auto":
-            monkeypatch.setenv("PHAST_DIAG_CUT", cut)
-        mode = "levels"
-    elif mode.startswith("levels-ab"):            # per-level launches, other arc batch (1-4, 8 = cp.async staged,
-                                                 # 16 = ELL-2 records, 17 = ELL-2 with the next record loaded ahead)
-        monkeypatch.setenv("PHAST_ARC_BATCH", mode[len("levels-ab"):])
-        mode = "levels"
-    elif mode == "levels-hybrid":                # a few small top levels fused, the rest one launch each
-        monkeypatch.setenv("PHAST_TOP_THRESH", "3000")
-        mode = "levels"
-    elif mode == "levels-flat":                  # one launch per level, no fusion
-        monkeypatch.setenv("PHAST_TOP_THRESH", "0")
-        mode = "levels"
-    monkeypatch.setenv("PHAST_SWEEP", mode)
-    g = phastgen.road(120_000, seed=33)
-    layout = {True: "levels", "bfs": "levels-bfs", False: "wavefront"}.get(level_layout, level_layout)
-    with P.Phast.from_graph(g, layout=layout, delta=delta) as h:
-        for k in (1, 2, 16, 64):
-            src = phastgen.sources(g.n, k, seed=900 + k)
-            assert np.array_equal(gpu_trees(h, src), oracle.sssp_many(g, src)), k
-        src = phastgen.sources(g.n, 200, seed=901)
-        assert h.diameter(src, k_batch=64) == oracle.diameter(g, src)
+SCHEDULES = {
+    "default": {},
+    "per_level": dict(flags=P.Q_NO_TOP | P.Q_NO_FUSED),          # the paper's: one launch per level
+    "top_hybrid": dict(flags=P.Q_NO_FUSED | P.Q_HYBRID_ON),
+    "top_full_searches": dict(flags=P.Q_NO_FUSED | P.Q_HYBRID_OFF),
+    "top_40": dict(flags=P.Q_NO_FUSED, top_max_vertices=40),    # the prefix ends inside the hierarchy
+    "top_700": dict(flags=P.Q_NO_FUSED, top_max_vertices=700),
+    "top_3000_hybrid": dict(flags=P.Q_NO_FUSED | P.Q_HYBRID_ON, top_max_vertices=3000),
+}
 
 
-@pytest.mark.parametrize("top", ["off", "default", "nofused", "nohybrid", "40", "700", "3000", "cluster-only", "cl4"])
-def test_top_levels_kernel(monkeypatch, top):
-    """The shared-memory sweep (sweep_top_kernel: rows in shared memory, cp.async-
-    staged arc chunks) and the cluster sweep of the mid levels (sweep_cluster_kernel):
-    off (one launch per level), cluster only, a 4-CTA cluster, default (C1 at k <= 4: the whole query
-    fused in one launch, G-up as a pull sweep; larger k / the road graph: the top
-    levels), top levels only ("nofused"), and top levels capped at V <= 40 / 700 /
-    3000 vertices (the prefix ends inside the hierarchy, chunks split long levels);
-    every k, bit-exact; plus the diameter (fused max over the final rows)."""
-    if top == "off":
-        monkeypatch.setenv("PHAST_TOP", "0")
-        monkeypatch.setenv("PHAST_FUSED", "0")
-        monkeypatch.setenv("PHAST_CL_SIZE", "0")
-    elif top == "cluster-only":                  # no shared-memory launch: mid levels in a 16-CTA cluster
-        monkeypatch.setenv("PHAST_TOP", "0")
-        monkeypatch.setenv("PHAST_FUSED", "0")
-        monkeypatch.setenv("PHAST_CL_SIZE", "16")
-    elif top == "cl4":                           # a 4-CTA cluster, one pass per level: long levels excluded
-        monkeypatch.setenv("PHAST_FUSED", "0")
-        monkeypatch.setenv("PHAST_CL_SIZE", "4")
-        monkeypatch.setenv("PHAST_CL_PASSES", "1")
-    elif top == "nofused":                       # top levels; the hybrid upward search forced on
-        monkeypatch.setenv("PHAST_FUSED", "0")
-        monkeypatch.setenv("PHAST_UP_HYBRID", "1")
-    elif top == "nohybrid":                      # full upward searches, the top kernel only sweeps G-down
-        monkeypatch.setenv("PHAST_FUSED", "0")
-        monkeypatch.setenv("PHAST_UP_HYBRID", "0")
-    elif top != "default":
-        monkeypatch.setenv("PHAST_FUSED", "0")
-        monkeypatch.setenv("PHAST_TOP_MAXV", top)
+@pytest.mark.parametrize("layout", ["levels-bfs", "levels"])
+@pytest.mark.parametrize("sched", sorted(SCHEDULES))
+def test_schedules(layout, sched):
+    """Every launch schedule (phast_configure) on both vertex orders is bit-exact:
+    one launch per level (§VI), the shared-memory top launch with and
+    without the hybrid upward search, capped top prefixes, and (default, small graphs)
+    the single fused launch; every k including padded ones; plus the diameter."""
     for g in (phastgen.CONFIGS["C1"]["graph"](), phastgen.road(40_000, seed=35), phastgen.road(9_000, seed=36)):
-        with P.Phast.from_graph(g) as h:
-            for k in (1, 2, 4, 16, 64):
+        with P.Phast.from_graph(g, layout=layout) as h:
+            h.configure(**SCHEDULES[sched])
+            for k in (1, 2, 4, 6, 16, 64):
                 src = phastgen.sources(g.n, k, seed=950 + k)
-                assert np.array_equal(gpu_trees(h, src), oracle.sssp_many(g, src)), (k, top)
+                assert np.array_equal(gpu_trees(h, src), oracle.sssp_many(g, src)), (k, sched)
             for kb in (1, 4, 16):
                 src = phastgen.sources(g.n, 130, seed=951)
                 assert h.diameter(src, k_batch=kb) == oracle.diameter(g, src), kb
 
 
-def test_fused_query_edge_cases(monkeypatch):
+def test_schedule_reports_launch_shape():
+    """phast_schedule: C1 at k <= 4 is one fused launch; a road graph gets a top launch
+    plus per-level launches; NO_TOP gives one launch per level."""
+    g = phastgen.CONFIGS["C1"]["graph"]()
+    with P.Phast.from_graph(g) as h:
+        s = h.schedule(1)
+        assert s["fused"] and s["level_launches"] == 0 and s["top_vertices"] == g.n
+    g = phastgen.road(120_000, seed=33)
+    with P.Phast.from_graph(g) as h:
+        s = h.schedule(64)
+        assert not s["fused"] and s["top_levels"] >= 2 and s["top_levels"] + s["level_launches"] == h.levels
+        h.configure(flags=P.Q_NO_TOP | P.Q_NO_FUSED)
+        assert h.schedule(64) == dict(fused=False, top_levels=0, top_vertices=0, level_launches=h.levels)
+
+
+def test_fused_query_edge_cases():
     """The fused single-launch query on graphs with unreachable parts, one-way arcs,
     zero and near-2^32 lengths (random digraphs), duplicate sources; bit-exact, and
     again with the per-level path for comparison."""
     for seed in range(6):
         g = phastgen.random_digraph(400 + 50 * seed, 1500 + 300 * seed, 0 if seed % 2 else 1,
                                     (1 << 32) - 1 if seed == 5 else 1 << 20, seed=70 + seed)
-        for fused in ("1", "0"):
-            monkeypatch.setenv("PHAST_FUSED", fused)
-            with P.Phast.from_graph(g) as h:
-                for k in (1, 4, 16):
+        with P.Phast.from_graph(g) as h:
+            for flags in (0, P.Q_NO_FUSED):
+                h.configure(flags=flags)
+                for k in (1, 3, 4, 16):
                     src = phastgen.sources(g.n, k, seed=seed, distinct=False)
-                    assert np.array_equal(gpu_trees(h, src), oracle.sssp_many(g, src)), (seed, fused, k)
+                    assert np.array_equal(gpu_trees(h, src), oracle.sssp_many(g, src)), (seed, flags, k)
 
 
 def test_top_levels_hub_vertex():
@@ -295,36 +249,84 @@ def test_top_levels_hub_vertex():
                 assert np.array_equal(gpu_trees(h, src), oracle.sssp_many(g, src)), (n, k)
 
 
-def test_l2_persistence_window(monkeypatch):
-    """The per-level sweep with an L2 persistence window over the top levels' rows
-    (PHAST_L2_PERSIST_MB) is bit-exact; the setting is process-wide, so the test
-    switches it off again at the end."""
-    g = phastgen.road(120_000, seed=39)
-    try:
-        monkeypatch.setenv("PHAST_L2_PERSIST_MB", "8")
-        with P.Phast.from_graph(g) as h:
-            for k in (1, 16, 64):
-                src = phastgen.sources(g.n, k, seed=980 + k)
-                assert np.array_equal(gpu_trees(h, src), oracle.sssp_many(g, src)), k
-    finally:
-        monkeypatch.setenv("PHAST_L2_PERSIST_MB", "0")
-        with P.Phast.from_graph(phastgen.grid(8, 8)):
-            pass
+def test_queries_in_flight_on_several_streams(road):
+    """PHAST_SLOTS queries in flight: 11 queries issued round robin on 3 streams into 3
+    label buffers (each buffer reused by its own stream), mixed k (padded k too), no
+    host synchronisation in between; every result bit-exact.  Exercises the slot
+    rotation (visited bits, search spaces, padded scratch) across streams."""
+    g, h = road
+    streams = [torch.cuda.Stream() for _ in range(3)]
+    ks = [64, 16, 5, 64, 1, 33, 16, 64, 7, 2, 64]
+    srcs = [phastgen.sources(g.n, k, seed=1200 + i) for i, k in enumerate(ks)]
+    bufs = [torch.empty(g.n * 64, dtype=torch.int32, device="cuda") for _ in range(3)]
+    got = []
+    for i, (k, src) in enumerate(zip(ks, srcs)):
+        st = streams[i % 3]
+        out = bufs[i % 3][:g.n * k]
+        h.trees(src, out=out, stream=st)
+        host = torch.empty(g.n * k, dtype=torch.int32, pin_memory=True)
+        with torch.cuda.stream(st):
+            host.copy_(out, non_blocking=True)
+        got.append((host, st))
+    for (host, st), src in zip(got, srcs):
+        st.synchronize()
+        assert np.array_equal(h.to_original(host.numpy()), oracle.sssp_many(g, src))
+    h.sync()
 
 
-@pytest.mark.parametrize("window", ["0", "1", "64"])
-def test_wave_sweep_every_k(monkeypatch, window):
-    """The warp-wave sweep (plan_waves + sweep_wave_kernel) at every k (each k has its
-    own chunk geometry) and several placement windows, bit-exact, repeated calls
-    (epoch-monotone completion counters)."""
-    monkeypatch.setenv("PHAST_SWEEP", "wave")
-    monkeypatch.setenv("PHAST_WAVE_WINDOW", window)
-    g = phastgen.road(60_000, seed=35)
-    with P.Phast.from_graph(g, layout="wavefront", delta=2000) as h:
-        for k in (1, 2, 4, 8, 16, 32, 64):
-            for rep in range(2):
-                src = phastgen.sources(g.n, k, seed=950 + k + rep)
-                assert np.array_equal(gpu_trees(h, src), oracle.sssp_many(g, src)), (k, rep)
+def test_probes_leave_state_clean(road):
+    """Probes A33 (stream) and A34 (no-gather traversal) run through the C ABI; a query
+    after them is still exact (A34 seeds and clears its slot like a query)."""
+    g, h = road
+    buf = torch.zeros(g.n * 16, dtype=torch.int32, device="cuda")
+    src = phastgen.sources(g.n, 16, seed=1300)
+    h.probe(0, 16, buf)
+    h.probe(1, 16, buf, sources=src)
+    h.sync()
+    with pytest.raises(P.PhastError):
+        h.probe(1, 16, buf)                 # A34 needs sources
+    with pytest.raises(P.PhastError):
+        h.probe(0, 12, buf[:g.n * 12])      # probes take the vector widths only
+    assert np.array_equal(gpu_trees(h, src), oracle.sssp_many(g, src))
+
+
+def test_binding_rejects_bad_output_tensors(road):
+    """The binding checks what the library will write: dtype, element
+    count, device, contiguity -- before any pointer reaches the C ABI."""
+    g, h = road
+    src = phastgen.sources(g.n, 4, seed=1)
+    with pytest.raises(TypeError):
+        h.trees(src, out=torch.empty(g.n * 4, dtype=torch.int64, device="cuda"))
+    with pytest.raises(ValueError):
+        h.trees(src, out=torch.empty(g.n * 4 - 1, dtype=torch.int32, device="cuda"))
+    with pytest.raises(ValueError):
+        h.trees(src, out=torch.empty(g.n * 4, dtype=torch.int32))
+    with pytest.raises(ValueError):
+        h.trees(src, out=torch.empty(g.n * 8, dtype=torch.int32, device="cuda")[::2])
+    with pytest.raises(TypeError):
+        h.betweenness([0, 1], out=torch.empty(g.n, dtype=torch.int32, device="cuda"))
+    with pytest.raises(ValueError):
+        h.reach([0, 1], out=torch.empty(g.n + 1, dtype=torch.int32, device="cuda"))
+    d = h.trees(src)
+    with pytest.raises(ValueError):
+        h.parents(src, d, out=torch.empty(g.n, dtype=torch.int32, device="cuda"))
+
+
+@pytest.mark.skipif(torch.cuda.device_count() < 2, reason="needs two GPUs")
+def test_two_devices_in_one_process():
+    """Handles on two devices (per-device kernel attributes and SM counts)."""
+    g = phastgen.road(30_000, seed=41)
+    src = phastgen.sources(g.n, 16, seed=2)
+    want = oracle.sssp_many(g, src)
+    hs = []
+    for dev in (0, 1):
+        torch.cuda.set_device(dev)
+        hs.append(P.Phast.from_graph(g))
+    for dev, h in enumerate(hs):
+        torch.cuda.set_device(dev)
+        assert np.array_equal(gpu_trees(h, src), want), dev
+        h.close()
+    torch.cuda.set_device(0)
 
 
 def test_tiny_and_degenerate():
@@ -342,13 +344,16 @@ def test_source_out_of_range(road):
         h.trees(np.array([g.n], np.uint32))
     assert e.value.status == -4
     with pytest.raises(ValueError):
-        h.trees(np.zeros(3, np.uint32))
+        h.trees(np.zeros(65, np.uint32))       # k > PHAST_KMAX
+    with pytest.raises(ValueError):
+        h.trees(np.zeros(0, np.uint32))
 
 
-def test_host_entry_point(road):
+@pytest.mark.parametrize("k", (8, 11))
+def test_host_entry_point(road, k):
     g, h = road
-    src = phastgen.sources(g.n, 8, seed=77)
-    out = np.empty((g.n, 8), np.uint32)
+    src = phastgen.sources(g.n, k, seed=77)
+    out = np.empty((g.n, k), np.uint32)
     h.trees_host(src, out)
     assert np.array_equal(h.to_original(out), oracle.sssp_many(g, src))
 
@@ -367,7 +372,7 @@ def test_diameter_c1_all_sources(c1):
     bmv = bm.cpu().numpy().view(np.uint32)
     for b in range(16):
         assert bmv[b] == tm[b * 64:(b + 1) * 64].max(), b
-    for kb in (1, 16):
+    for kb in (1, 5, 16):
         assert h.diameter(sub[:37], k_batch=kb) == int(tm[:37].max())
 
 
@@ -379,6 +384,25 @@ def test_diameter_road_and_unreachable(road):
     with P.Phast.from_graph(g2) as h2:
         src = np.arange(0, g2.n, 7, dtype=np.uint32)
         assert h2.diameter(src, k_batch=64) == oracle.diameter(g2, src)
+
+
+def witness_ok(g, src, D, s, t):
+    """(D, s*, t*) from phast_diameter_witness: D is the oracle's diameter over src, s*
+    is one of the sources, and the oracle's dist(s*, t*) = D."""
+    assert s in set(int(x) for x in src)
+    assert int(oracle.sssp(g, s)[t]) == D
+
+
+def test_diameter_witness(c1, road):
+    for g, h in (c1, road):
+        src = phastgen.sources(g.n, 300, seed=12)
+        for kb in (64, 7):
+            D, s, t = h.diameter_witness(src, k_batch=kb)
+            assert D == oracle.diameter(g, src), kb
+            witness_ok(g, src, D, s, t)
+    g1 = phastgen.Graph(2, np.array([0, 0, 0], np.uint64), np.zeros(0, np.uint32), np.zeros(0, np.uint32))
+    with P.Phast.from_graph(g1) as h1:
+        assert h1.diameter_witness([1, 0]) == (0, 1, 1)     # no finite nonzero label
 
 
 def test_distance_metric_deep_hierarchy():
@@ -409,39 +433,59 @@ def test_c2_1m_k16():
 
 
 @pytest.mark.slow
-def test_c3_europe_scale_bench_config():
-    """C3 at full size (~18M vertices, ~42M arcs) in the bench's launch configuration
-    (k=64): 4 sampled trees bit-exact against the oracle, 16 more certified."""
+def test_c3_europe_scale_bench_configs():
+    """C3 at full size (~18M vertices, ~42M arcs) in the bench's launch configurations
+    (BASELINE.json configs[2]: k = 16, 32, 64; labels left in HBM): per k, 4 sampled
+    trees bit-exact against the oracle and 12 more certified by the O(n+m)
+    certificate."""
     cfg = phastgen.CONFIGS["C3"]
     g = cfg["graph"]()
     with P.Phast.from_graph(g) as h:
-        src = phastgen.sources(g.n, 64, seed=cfg["src_seed"])
-        got = gpu_trees(h, src)
-        pick = [0, 17, 40, 63]
-        want = oracle.sssp_many(g, src[pick])
-        assert np.array_equal(got[pick], want)
-        for i in range(1, 64, 4):
-            assert oracle.certify(g, int(src[i]), got[i]) == 0, i
+        for k in (16, 32, 64):
+            src = phastgen.sources(g.n, k, seed=cfg["src_seed"] + k)
+            got = gpu_trees(h, src)
+            pick = [0, k // 3, (2 * k) // 3, k - 1]
+            assert np.array_equal(got[pick], oracle.sssp_many(g, src[pick])), k
+            for i in range(1, k, max(1, k // 12)):
+                assert oracle.certify(g, int(src[i]), got[i]) == 0, (k, i)
 
 
 @pytest.mark.slow
 def test_c4_usa_scale_bench_config():
     """C4 at full size (~24M vertices, ~58M arcs, USA shape) in the bench's launch
     configuration (k=64): 3 sampled trees bit-exact against the oracle, 8 more
-    certified; plus the diameter path on the same hierarchy for 64 sources against
-    the oracle's maxima of those trees."""
+    certified; plus the diameter over the same 64 sources against the ORACLE's
+    maxima of those 64 trees (oracle.tree_maxima, independent of the GPU rows)."""
     cfg = phastgen.CONFIGS["C4"]
     g = cfg["graph"]()
     with P.Phast.from_graph(g) as h:
         src = phastgen.sources(g.n, 64, seed=cfg["src_seed"])
         got = gpu_trees(h, src)
         pick = [3, 31, 62]
-        want = oracle.sssp_many(g, src[pick])
-        assert np.array_equal(got[pick], want)
+        assert np.array_equal(got[pick], oracle.sssp_many(g, src[pick]))
         for i in range(0, 64, 8):
             assert oracle.certify(g, int(src[i]), got[i]) == 0, i
-        fin = np.where(got == INF, 0, got).max()
-        assert h.diameter(src, k_batch=64) == int(fin)
+        del got
+        assert h.diameter(src, k_batch=64) == int(oracle.tree_maxima(g, src).max())
+
+
+@pytest.mark.slow
+def test_c5_exact_diameter_with_witness():
+    """C5 (BASELINE.json configs[4]): the exact diameter over ALL sources of the 1M
+    road graph, with its witness (SURVEY.md §8(c) diameter row): the oracle confirms
+    dist(s*, t*) = D, and the oracle's maximum over 1 024 sampled sources is <= D.
+    The per-rank form (sources sharded, MAX all-reduce) is covered on CPU by
+    tests/test_parallel.py."""
+    cfg = phastgen.CONFIGS["C5"]
+    g = cfg["graph"]()
+    allsrc = np.arange(g.n, dtype=np.uint32)
+    with P.Phast.from_graph(g) as h:
+        D, s, t = h.diameter_witness(allsrc, k_batch=64)
+        assert h.diameter(allsrc, k_batch=64) == D
+    witness_ok(g, allsrc, D, s, t)
+    sample = phastgen.sources(g.n, 1024, seed=cfg["src_seed"] + 9)
+    assert int(oracle.tree_maxima(g, sample).max()) <= D
+    assert int(oracle.tree_maxima(g, [s]).max()) == D        # s* is an eccentricity-D source
 
 
 @pytest.mark.slow
@@ -535,15 +579,12 @@ def test_reach_exact_all_sources_and_max_shards():
     bc_close(cb, oracle.betweenness(g, allv[:20]))
 
 
-@pytest.mark.parametrize("persist", ("0", "1"))
-def test_centrality_both_pass_drivers(monkeypatch, persist):
-    """The graph-captured pass chunks (default) and the persistent cooperative Kahn
-    kernel (PHAST_BC_PERSIST=1) give the oracle's values."""
-    monkeypatch.setenv("PHAST_BC_PERSIST", persist)
+def test_centrality_padded_batches():
+    """k_batch not a power of two (rounded up internally): same values."""
     g = BC_GRAPHS["unit_grid"]()
     src = phastgen.sources(g.n, 21, seed=77)
     with P.Phast.from_graph(g) as h:
-        cb = h.vertex_to_original(h.betweenness(src, k_batch=8).cpu().numpy())
-        r = h.vertex_to_original(h.reach(src, k_batch=16).cpu().numpy().view(np.uint32))
+        cb = h.vertex_to_original(h.betweenness(src, k_batch=5).cpu().numpy())
+        r = h.vertex_to_original(h.reach(src, k_batch=11).cpu().numpy().view(np.uint32))
     bc_close(cb, oracle.betweenness(g, src))
     assert np.array_equal(r, oracle.reach(g, src))

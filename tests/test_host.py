@@ -64,7 +64,7 @@ def test_host_hierarchy_sweep_equals_oracle(name):
     assert np.array_equal(got, want)
 
 
-LAYOUTS = {name: dict(layout=name) for name in ("wavefront", "levels", "levels-bfs", "diagonal")}
+LAYOUTS = {name: dict(layout=name) for name in ("levels", "levels-bfs")}
 
 
 @pytest.mark.parametrize("layout", sorted(LAYOUTS))
@@ -72,7 +72,6 @@ LAYOUTS = {name: dict(layout=name) for name in ("wavefront", "levels", "levels-b
 def test_layout_invariants(name, layout):
     g = GRAPHS[name]()
     h = P.Phast.from_graph(g, host_only=True, **LAYOUTS[layout])
-    level_layout = layout != "wavefront"
     ex = h.export()
     n, L = h.n, h.levels
     lev = ex["level"].astype(np.int64)
@@ -92,9 +91,8 @@ def test_layout_invariants(name, layout):
     assert np.array_equal(np.sort(perm), np.arange(n, dtype=np.uint32))
     # level-0 vertices are never tails (their rows need not be stored in diameter mode)
     assert np.all(lev[tails] > 0)
-    assert h.info().layout == {"wavefront": 0, "levels": 1, "levels-bfs": 2, "diagonal": 3}[layout]
-    if layout in ("levels", "levels-bfs"):
-        assert np.all(np.diff(lev) <= 0)                 # levels contiguous, highest first
+    assert h.info().layout == {"levels": 1, "levels-bfs": 2}[layout]
+    assert np.all(np.diff(lev) <= 0)                     # levels contiguous, highest first
     if layout == "levels":
         inv = np.empty_like(perm)
         inv[perm] = np.arange(n, dtype=np.uint32)
@@ -108,7 +106,7 @@ def test_layout_invariants(name, layout):
 @pytest.mark.parametrize("layout", sorted(LAYOUTS))
 def test_every_layout_sweep_equals_oracle(layout):
     g = phastgen.road(40_000, seed=12)
-    h = P.Phast.from_graph(g, host_only=True, delta=5000, **LAYOUTS[layout])
+    h = P.Phast.from_graph(g, host_only=True, **LAYOUTS[layout])
     src = phastgen.sources(g.n, 5, seed=3)
     assert np.array_equal(chref.phast_cpu(h, h.export(), src), oracle.sssp_many(g, src))
 
@@ -194,18 +192,43 @@ def test_degenerate_graphs():
     assert np.array_equal(got, oracle.sssp_many(g2, [0, 1, 2]))
 
 
-@pytest.mark.parametrize("layout", sorted(LAYOUTS))
-def test_sweep_schedule_is_well_formed(layout):
-    """The persistent sweep's static schedule (layout.cpp plan_chunks): every chunk is
-    placed in an iteration after the one producing its latest tail; pad slots fill the
-    gaps.  plan_chunks itself fails (EINTERNAL) if a dependency is not strictly earlier."""
-    g = phastgen.road(60_000, seed=9)
-    h = P.Phast.from_graph(g, host_only=True, **LAYOUTS[layout])
-    for k in (1, 16, 64):
-        for grid in (1, 7, 148, 592):
-            st = h.plan_stats(k, grid)
-            assert st["slots"] == st["chunks"] + st["pads"]
-            assert st["iterations"] == -(-st["slots"] // grid)
-            assert st["chunks"] >= -(-g.n // (4 * 256 // max(1, k // 4)))
-    with pytest.raises(P.PhastError):
-        h.plan_stats(3, 148)
+def test_unknown_build_flags_rejected():
+    g = phastgen.grid(4, 4)
+    o = P._Opts(0, 0, 0, 0, P.FLAG_HOST_ONLY | 8, 0, 0)       # 8, 16: the removed experimental layouts
+    h = P.ctypes.c_void_p()
+    rc = P._lib.phast_build(g.n, g.first.ctypes.data, g.head.ctypes.data, g.len.ctypes.data, P.ctypes.byref(o),
+                            P.ctypes.byref(h))
+    assert rc == -1
+
+
+def upward_space_bfs(ex, s):
+    """Vertices reachable from internal id s in G-up (numpy reference of the search
+    space; the upward search runs to exhaustion, §III)."""
+    uf, uh = ex["up_first"].astype(np.int64), ex["up_head"]
+    seen = {int(s)}
+    stack = [int(s)]
+    while stack:
+        v = stack.pop()
+        for w in uh[uf[v]:uf[v + 1]]:
+            if int(w) not in seen:
+                seen.add(int(w))
+                stack.append(int(w))
+    return len(seen)
+
+
+def test_info_upward_search_space_stats():
+    """phast_info's mean/max upward search space: the library's host
+    sample of 1 024 sources (stride 2654435761 mod n from 12345) against a Python BFS
+    over the exported G-up, and within the expected regime (§II-B "about 500
+    vertices" on Europe; our 60 k road graph: a few hundred)."""
+    g = GRAPHS["road"]()
+    h = P.Phast.from_graph(g, host_only=True)
+    inf = h.info()
+    assert inf.up_space_samples == 1024
+    ex = h.export()
+    sizes = [upward_space_bfs(ex, (i * 2654435761 + 12345) % h.n) for i in range(1024)]
+    assert inf.max_up_space == max(sizes)
+    assert abs(inf.mean_up_space - np.mean(sizes)) < 1e-9
+    assert 10 < inf.mean_up_space < 2000
+    small = P.Phast.from_graph(phastgen.grid(5, 4), host_only=True).info()
+    assert small.up_space_samples == 20 and small.max_up_space <= 20

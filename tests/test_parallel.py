@@ -117,3 +117,93 @@ def test_two_rank_centrality_shards_combine():
     for _, cb, r in res:
         np.testing.assert_allclose(cb, oracle.betweenness(g, allv), rtol=1e-12)
         assert np.array_equal(r, oracle.reach(g, allv))
+
+
+def _bench_worker(rank, world, port, q):
+    import torch
+    import torch.distributed as dist
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        import bench
+        import phastgen
+        cfg = phastgen.CONFIGS["C4"]
+        n = 24_000_000
+        # strong scaling (BASELINE configs[3]): 8192 sources sharded; 8000 = ragged last batch
+        out = {}
+        for total in (8192, 8000):
+            warm, timed, trees = bench.rank_batches(n, cfg, 64, world, rank, 5, 3, total)
+            got = [None] * world
+            dist.all_gather_object(got, (rank, [b.tolist() for b in timed], trees))
+            out[total] = got
+        # weak scaling: `steps` batches of this rank's own sources
+        warm, timed, trees = bench.rank_batches(n, cfg, 64, world, rank, 5, 3, 0)
+        weak = [None] * world
+        dist.all_gather_object(weak, (rank, [b.tolist() for b in timed], [b.tolist() for b in warm], trees))
+        # max-over-ranks timing (the bench's rule for every multi-GPU number)
+        t = torch.tensor([10.0 + rank], dtype=torch.float64)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        q.put((rank, out, weak, float(t.item())))
+    finally:
+        dist.destroy_process_group()
+
+
+def test_two_rank_bench_source_plan():
+    """bench.py's rank logic on a world-2 gloo group: in strong-scaling mode the two
+    ranks' batches cover the one seeded list of T sources exactly once (a ragged last
+    batch is padded with duplicates that are not counted); in weak mode each rank
+    sweeps `steps` batches of k sources of its own; timings combine by MAX."""
+    import phastgen
+    world = 2
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_bench_worker, args=(r, world, port, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    # drain the queue before joining: a worker cannot exit while its large result
+    # is still in the pipe
+    res = sorted((q.get(timeout=300) for _ in range(world)), key=lambda x: x[0])
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    cfg = phastgen.CONFIGS["C4"]
+    for total in (8192, 8000):
+        full = phastgen.sources(24_000_000, total, seed=cfg["src_seed"] * 7919 + 1).tolist()
+        per_rank = sorted(res[0][1][total])
+        assert per_rank == sorted(res[1][1][total])           # all_gather agrees on both ranks
+        flat, counted = [], 0
+        for r, batches, trees in per_rank:
+            assert all(len(b) == 64 for b in batches)
+            real = sum((b for b in batches), [])[:trees]
+            flat += real
+            counted += trees
+        assert flat == full and counted == total
+    weak = res[0][2]
+    assert [w[3] for w in weak] == [320, 320]
+    a, b = weak[0][1], weak[1][1]
+    assert len(a) == len(b) == 5 and all(len(x) == 64 for x in a + b)
+    assert a != b and weak[0][2] != a                          # own sources per rank; warm-up differs
+    assert all(r[3] == 11.0 for r in res)
+
+
+def test_bench_relaunches_under_torchrun(monkeypatch):
+    """`python bench.py --gpus 8` outside torchrun re-executes itself under
+    torch.distributed.run with 8 ranks, 127.0.0.1 rendezvous, NCCL init logging."""
+    import sys
+    import bench
+    seen = {}
+
+    def fake_call(cmd, env):
+        seen["cmd"], seen["env"] = cmd, env
+        return 0
+    monkeypatch.setattr(bench.subprocess, "call", fake_call)
+    monkeypatch.delenv("WORLD_SIZE", raising=False)
+    monkeypatch.setattr(sys, "argv", ["bench.py", "--gpus", "8", "--steps", "5"])
+    assert bench.main() == 0
+    cmd = seen["cmd"]
+    assert cmd[1:4] == ["-m", "torch.distributed.run", "--nnodes=1"]
+    assert "--nproc-per-node=8" in cmd and "127.0.0.1" in cmd
+    assert cmd[-4:] == ["--gpus", "8", "--steps", "5"] and cmd[-5].endswith("bench.py")
+    assert seen["env"]["NCCL_DEBUG"] == "INFO"
