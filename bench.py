@@ -206,7 +206,9 @@ def main():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--config", default="C3")
     ap.add_argument("--k", type=int, default=64)
-    ap.add_argument("--inflight", type=int, default=2, help="streams with a batch in flight (1..4)")
+    ap.add_argument("--inflight", type=int, default=0,
+                    help="streams with a batch in flight (1..4; 0 = auto: 4 on small graphs whose labels fit L2, "
+                         "1 on large ones, where overlapping sweeps thrash L2: measured slower, DESIGN.md §6)")
     ap.add_argument("--total-sources", type=int, default=0,
                     help="strong scaling: this many sources split over the ranks (C4: 8192); steps is derived")
     ap.add_argument("--steady", action="store_true",
@@ -218,11 +220,13 @@ def main():
     ap.add_argument("--cache", default="", help="hierarchy file to reuse/create (optional)")
     ap.add_argument("--layout", default="levels-bfs", choices=["levels", "levels-bfs"],
                     help="vertex order: the paper's level layout (DFS within a level) or BFS within a level")
+    ap.add_argument("--no-band", action="store_true",
+                    help="one launch per level below the top launch instead of the band dataflow launch")
     ap.add_argument("--parents", action="store_true",
                     help="also time the parent-pointer pass (phast_parents, NEXT-1) on the last batch")
     args = ap.parse_args()
     args.warmup = max(3, args.warmup)
-    args.inflight = max(1, min(4, args.inflight))
+    args.inflight = max(0, min(4, args.inflight))
     if args.impl == "reference":
         return run_reference(args)
     if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
@@ -275,6 +279,8 @@ def main():
         log(f"[bench] CH build {time.time() - t:.1f}s")
         if args.cache:
             h.save(args.cache)
+    if args.no_band:
+        h.configure(flags=P.Q_NO_BAND)
     n = h.n
     info = h.info()
     lsz = h.level_sizes()
@@ -291,13 +297,13 @@ def main():
     warm, timed, trees_here = rank_batches(n, cfg, k, world, rank, args.steps, args.warmup, args.total_sources)
     args.steps = len(timed)
 
-    S = args.inflight
+    small = 4 * k * n + 16 * info.m_down < 256e6
+    S = args.inflight or (4 if small else 1)
     stream = torch.cuda.current_stream()
     streams = [torch.cuda.Stream() for _ in range(S)]
     # L2 protocol: the C3/C4 label arrays (>= 1 GB) are far beyond the 126 MB L2; small
     # configs (labels + graph fit in L2) flush L2 before every step, or with --steady
     # rotate over enough label buffers that the labels alone exceed 2x L2
-    small = 4 * k * n + 16 * info.m_down < 256e6
     flush = small and not args.steady
     nbuf = S
     if small and args.steady:

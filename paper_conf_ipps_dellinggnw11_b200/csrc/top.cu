@@ -46,7 +46,9 @@ __host__ __device__ constexpr size_t top_stage_bytes(bool big) {   // {descripto
 }
 constexpr size_t TOP_STAGE_BYTES = top_stage_bytes(false);
 constexpr uint32_t TOP_MAX_STAGES = 24, TOP_MIN_STAGES = 4;
-constexpr size_t TOP_SMEM_MAX = 227 * 1024;
+// dynamic shared memory: the 227 KB per-CTA maximum less the static heavy-vertex lists
+constexpr size_t TOP_STATIC = 2 * 2 * 1024 + 64;
+constexpr size_t TOP_SMEM_MAX = 227 * 1024 - TOP_STATIC;
 
 constexpr uint32_t TOP_HEAVY = 8;              // in-arcs above which a warp relaxes the vertex (k <= 4)
 constexpr uint32_t TOP_VMASK = 0x7FFFFFFFu;    // chunk vend; bit 31: the chunk has a vertex with > TOP_HEAVY in-arcs
@@ -119,8 +121,16 @@ __global__ void __launch_bounds__(TOP_THREADS, 1) sweep_top_kernel(TopArgs A, So
         }
     } else {
         const uint32_t ct = tid - 32;
+        __shared__ uint32_t hcnt[2];            // heavy vertices of the chunk (double-buffered)
+        __shared__ uint16_t hlist[2][TOP_VCH_BIG];   // as offsets from the chunk's first vertex
+        static_assert(sizeof(hcnt) + sizeof(hlist) <= TOP_STATIC, "static shared memory");
+        if (ct < 2) hcnt[ct] = 0;
+        asm volatile("bar.sync 1, %0;" ::"n"(TOP_CONS) : "memory");
         uint32_t s = 0, ph = 0;
         for (uint32_t c = 0; c < A.nchunks; c++) {
+            // the other count was last used by chunk c - 1, whose readers all passed its
+            // end barrier; chunk c + 1's writers wait for chunk c's end barrier
+            if (ct == 0) hcnt[(c + 1) & 1] = 0;
             mbar_wait(&full[s], ph);
             const unsigned char* st = ring + (size_t)s * SB;
             const uint4 ch = *reinterpret_cast<const uint4*>(st);
@@ -133,7 +143,10 @@ __global__ void __launch_bounds__(TOP_THREADS, 1) sweep_top_kernel(TopArgs A, So
             for (uint32_t t = ct; t < total; t += TOP_CONS) {
                 const uint32_t v = ch.x + t / G, lane = t % G;
                 const uint32_t e0 = sf[v - f0], e1 = sf[v + 1 - f0];
-                if (heavy && e1 - e0 > TOP_HEAVY) continue;   // a warp takes it below
+                if (heavy && e1 - e0 > TOP_HEAVY) {   // a warp takes it below
+                    hlist[c & 1][atomicAdd(&hcnt[c & 1], 1u)] = (uint16_t)(v - ch.x);
+                    continue;
+                }
                 T acc = srow[v * G + lane];
                 // four arcs at a time: their loads (then their rows' loads) are
                 // independent, so a vertex costs two shared-memory round trips per
@@ -153,12 +166,13 @@ __global__ void __launch_bounds__(TOP_THREADS, 1) sweep_top_kernel(TopArgs A, So
             if (heavy) {
                 // vertices with many in-arcs (the top of G-up: every lower neighbour is
                 // an in-arc) would serialise a level on one thread: one warp each, the
-                // lanes striding over the arcs, then a warp min
-                const uint32_t wid = ct >> 5, wl = ct & 31, nv = vend - ch.x;
-                for (uint32_t i = wid; i < nv; i += TOP_CONS / 32) {
-                    const uint32_t v = ch.x + i;
+                // lanes striding over the arcs, then a warp min.  The light pass listed
+                // them; the list is complete after this barrier (heavy chunks only).
+                asm volatile("bar.sync 1, %0;" ::"n"(TOP_CONS) : "memory");
+                const uint32_t wid = ct >> 5, wl = ct & 31, nh = hcnt[c & 1];
+                for (uint32_t i = wid; i < nh; i += TOP_CONS / 32) {
+                    const uint32_t v = ch.x + hlist[c & 1][i];
                     const uint32_t e0 = sf[v - f0], e1 = sf[v + 1 - f0];
-                    if (e1 - e0 <= TOP_HEAVY) continue;   // warp-uniform
                     T acc = wl == 0 ? srow[v] : inf_row<T>();
                     for (uint32_t e = e0 + wl; e < e1; e += 128) {   // four arcs per lane in flight
                         uint2 a[4];

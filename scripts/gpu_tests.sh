@@ -6,8 +6,8 @@ cd "${GRAFT_REPO_ROOT:-/root/repo}"
 mkdir -p gpurun_out
 nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm --format=csv > gpurun_out/gpu.txt 2>&1
 python -c "import __graft_entry__ as g; g.build()" > gpurun_out/build.log 2>&1 || { tail -30 gpurun_out/build.log; exit 1; }
-K=${1:+-k "$1"}
-timeout 2400 python -m pytest tests -m "gpu and not slow" -x -q $K > gpurun_out/pytest_gpu.log 2>&1; echo "fast rc=$?" >> gpurun_out/pytest_gpu.log
+if [ -n "$1" ]; then K=(-k "$1"); else K=(); fi
+timeout 2400 python -m pytest tests -m "gpu and not slow" -x -q "${K[@]}" > gpurun_out/pytest_gpu.log 2>&1; echo "fast rc=$?" >> gpurun_out/pytest_gpu.log
 tail -5 gpurun_out/pytest_gpu.log
 if [ -z "$1" ]; then
   timeout 2400 python -m pytest tests -m "gpu and slow" -x -q > gpurun_out/pytest_slow.log 2>&1; echo "slow rc=$?" >> gpurun_out/pytest_slow.log
