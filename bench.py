@@ -220,8 +220,6 @@ def main():
     ap.add_argument("--cache", default="", help="hierarchy file to reuse/create (optional)")
     ap.add_argument("--layout", default="levels-bfs", choices=["levels", "levels-bfs"],
                     help="vertex order: the paper's level layout (DFS within a level) or BFS within a level")
-    ap.add_argument("--no-band", action="store_true",
-                    help="one launch per level below the top launch instead of the band dataflow launch")
     ap.add_argument("--parents", action="store_true",
                     help="also time the parent-pointer pass (phast_parents, NEXT-1) on the last batch")
     args = ap.parse_args()
@@ -279,8 +277,6 @@ def main():
         log(f"[bench] CH build {time.time() - t:.1f}s")
         if args.cache:
             h.save(args.cache)
-    if args.no_band:
-        h.configure(flags=P.Q_NO_BAND)
     n = h.n
     info = h.info()
     lsz = h.level_sizes()

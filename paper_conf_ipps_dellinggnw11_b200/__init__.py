@@ -28,7 +28,7 @@ FLAG_LEVEL_LAYOUT = 2
 FLAG_BFS_IN_LEVEL = 4
 LAYOUT_FLAGS = {"levels-bfs": 0, "levels": FLAG_LEVEL_LAYOUT}
 LAYOUT_NAMES = {1: "levels", 2: "levels-bfs"}   # phast_info_t.layout
-Q_NO_FUSED, Q_NO_TOP, Q_HYBRID_ON, Q_HYBRID_OFF, Q_NO_BAND = 1, 2, 4, 8, 16
+Q_NO_FUSED, Q_NO_TOP, Q_HYBRID_ON, Q_HYBRID_OFF = 1, 2, 4, 8
 
 STATUS = {0: "OK", -1: "EINVAL", -2: "ENOMEM", -3: "ECUDA", -4: "ERANGE", -5: "ESTATE", -6: "EIO",
           -7: "EINTERNAL"}
@@ -48,9 +48,7 @@ class _Opts(ctypes.Structure):
 
 class _QOpts(ctypes.Structure):
     _fields_ = [("flags", ctypes.c_uint32), ("top_max_vertices", ctypes.c_uint32),
-                ("seed_cap", ctypes.c_uint32), ("up_smem_cap", ctypes.c_uint32),
-                ("band_levels", ctypes.c_uint32), ("bands", ctypes.c_uint32),
-                ("band_lag", ctypes.c_uint32), ("band_chunk", ctypes.c_uint32)]
+                ("seed_cap", ctypes.c_uint32), ("up_smem_cap", ctypes.c_uint32)]
 
 
 class _Info(ctypes.Structure):
@@ -83,7 +81,7 @@ def _load_lib():
         "phast_info": ([vp, ctypes.POINTER(_Info)], ci),
         "phast_level_sizes": ([vp, vp], ci),
         "phast_order": ([vp, vp], ci),
-        "phast_export": ([vp, vp, vp, vp, vp, vp, vp, vp, vp], ci),
+        "phast_export": ([vp, vp, vp, vp, vp, vp, vp, vp], ci),
         "phast_schedule": ([vp, u32, vp], ci),
         "phast_save": ([vp, ctypes.c_char_p], ci),
         "phast_load": ([ctypes.c_char_p, u32, pp], ci),
@@ -218,10 +216,9 @@ class Phast:
     def save(self, path):
         _check("phast_save", _lib.phast_save(self._h, path.encode()))
 
-    def configure(self, flags=0, top_max_vertices=0, seed_cap=0, up_smem_cap=0, band_levels=0, bands=0,
-                  band_lag=0, band_chunk=0):
+    def configure(self, flags=0, top_max_vertices=0, seed_cap=0, up_smem_cap=0):
         """Query-path options (phast_configure): schedule choices only, same labels."""
-        q = _QOpts(flags, top_max_vertices, seed_cap, up_smem_cap, band_levels, bands, band_lag, band_chunk)
+        q = _QOpts(flags, top_max_vertices, seed_cap, up_smem_cap)
         _check("phast_configure", _lib.phast_configure(self._h, ctypes.byref(q)))
         return self
 
@@ -364,11 +361,10 @@ class Phast:
 
     def schedule(self, k: int) -> dict:
         """Launch schedule of a k-tree query (phast_schedule)."""
-        out = np.zeros(7, np.uint32)
+        out = np.zeros(4, np.uint32)
         _check("phast_schedule", _lib.phast_schedule(self._h, k, out.ctypes.data))
         return dict(fused=bool(out[0]), top_levels=int(out[1]), top_vertices=int(out[2]),
-                    level_launches=int(out[3]), band_levels=int(out[4]), band_tasks=int(out[5]),
-                    band_chunks=int(out[6]))
+                    level_launches=int(out[3]))
 
     def timing(self, enable: bool):
         _check("phast_timing", _lib.phast_timing(self._h, 1 if enable else 0))
@@ -402,13 +398,12 @@ class Phast:
 
     def export(self) -> dict:
         inf = self.info()
-        a = dict(level=np.empty(inf.n, np.uint32), rank=np.empty(inf.n, np.uint32),
-                 dn_first=np.empty(inf.n + 1, np.uint32),
+        a = dict(level=np.empty(inf.n, np.uint32), dn_first=np.empty(inf.n + 1, np.uint32),
                  dn_tail=np.empty(max(inf.m_down, 1), np.uint32), dn_len=np.empty(max(inf.m_down, 1), np.uint32),
                  up_first=np.empty(inf.n + 1, np.uint32), up_head=np.empty(max(inf.m_up, 1), np.uint32),
                  up_len=np.empty(max(inf.m_up, 1), np.uint32))
         _check("phast_export", _lib.phast_export(self._h, *[a[k].ctypes.data for k in
-                                                           ("level", "rank", "dn_first", "dn_tail", "dn_len", "up_first",
+                                                           ("level", "dn_first", "dn_tail", "dn_len", "up_first",
                                                             "up_head", "up_len")]))
         a["dn_tail"] = a["dn_tail"][:inf.m_down]
         a["dn_len"] = a["dn_len"][:inf.m_down]

@@ -6,7 +6,6 @@
 // (§IV-A).  G-down: in-arcs by head, {tail, len} (§IV-A),
 // sentinel dn_first[n].  G-up: out-arcs by tail, {head, len}.
 #include <algorithm>
-#include <cmath>
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
@@ -30,7 +29,7 @@ struct phast_ctx {
     uint32_t rounds = 0;
     double build_seconds = 0;
     Layout L;
-    phast_query_opts q = {};
+    phast_query_opts q = {0, 0, 0, 0};
     // upward-search-space statistics of phast_info (host sample, computed once)
     mutable bool up_stats = false;
     mutable double up_mean = 0;
@@ -85,27 +84,6 @@ struct phast_ctx {
         uint2* up_a = nullptr;
     };
     std::map<uint32_t, Top> tops;
-    // band dataflow plan of the levels below the top launch (k-independent part; built
-    // on first use for a given first banded level jb) and its per-k chunk tables
-    struct Band {
-        uint32_t jb = 0;                 // first banded level index (top-down); vertices [lvl_off[jb], n)
-        uint32_t ntasks = 0;
-        std::vector<uint32_t> vbeg, vend, last;   // per task (sequence order)
-        std::vector<uint32_t> dep_first, dep_list;
-        uint32_t* d_dep_first = nullptr;
-        uint32_t* d_dep_list = nullptr;
-        struct PerK {
-            uint4* chunks = nullptr;
-            uint32_t* task_nch = nullptr;
-            uint32_t nchunks = 0;
-        };
-        std::map<uint32_t, PerK> perk;
-        uint32_t* counters[SLOTS] = {};  // per slot: [ntasks] done + [1] next (zeroed by the seed launch)
-        uint32_t chunk_lanes = 1024;     // (vertex, 16-byte lane) items per chunk
-        uint32_t unroll = 4;
-        bool ok = false;
-    };
-    std::map<uint32_t, Band> bands;      // by jb (the top prefix may differ between k)
     // A-up in-arcs by head {tail, len} (fused single-launch queries on small graphs)
     uint32_t* d_upin_first = nullptr;
     uint2* d_upin_arc = nullptr;
@@ -167,20 +145,6 @@ int grow(T** p, size_t* have, size_t elems) {
     return rc;
 }
 
-void free_bands(phast_ctx* h) {
-    for (auto& bk : h->bands) {
-        phast_ctx::Band& B = bk.second;
-        cudaFree(B.d_dep_first);
-        cudaFree(B.d_dep_list);
-        for (auto& kv : B.perk) {
-            cudaFree(kv.second.chunks);
-            cudaFree(kv.second.task_nch);
-        }
-        for (uint32_t s = 0; s < SLOTS; s++) cudaFree(B.counters[s]);
-    }
-    h->bands.clear();
-}
-
 void free_tops(phast_ctx* h) {
     for (auto& kv : h->tops) {
         cudaFree(kv.second.chunks);
@@ -188,7 +152,6 @@ void free_tops(phast_ctx* h) {
         cudaFree(kv.second.up_a);
     }
     h->tops.clear();
-    free_bands(h);
 }
 
 void free_seeds(phast_ctx* h) {
@@ -552,175 +515,6 @@ phast_ctx::Top* get_top(phast_ctx* h, uint32_t k) {
     return &T;
 }
 
-// Band dataflow plan (kernels.h: BandArgs) for levels [jb, L) (top-down level index).
-// Every vertex v of the banded levels gets a key
-//     K(v) = floor(rank(v) / bw + o(L(v))),   bw = n / bands,
-// rank = the spatial order each level is sorted by (Layout::rank), o(l) a per-level
-// offset in band units computed top-down:
-//     o(l) = max over G-down arcs (t, v) with L(v) = l, t banded, of
-//            o(L(t)) + (rank(t) - rank(v)) / bw + lag
-// so every arc has K(t) <= K(v) - lag + 1: a diagonal through the levels, skewed by
-// how far (in rank) the arcs into each level reach.  A task = the vertices of one level
-// with one key (a contiguous id range: each level is sorted by rank); the sequence
-// sorts tasks by (key, level descending), which is topological.  Dependencies (the
-// tasks holding a vertex's tails) are exact; one implied by another (u in D(v), v in
-// D(t)) is dropped.  Band b of every level covers about the same region, so a tail row
-// is written shortly before its heads read it and is read from L2
-// (profiles/r2_bandsim.md); lag >= 2 keeps `lag - 1` keys of independent tasks between
-// a task and its dependencies, so many chunks run at once.
-struct BandParams { uint32_t bands, lag, chunk_lanes, levels, unroll; };
-
-BandParams band_params(const phast_ctx* h) {
-    BandParams p;
-    p.bands = h->q.bands ? h->q.bands : 512u;
-    p.lag = h->q.band_lag ? h->q.band_lag : 2u;
-    p.unroll = h->q.band_chunk == 512 ? 2u : 4u;   // band_chunk: items per chunk, 512 or 1024
-    p.chunk_lanes = band_chunk_lanes(p.unroll);
-    p.levels = h->q.band_levels ? h->q.band_levels : 12u;
-    return p;
-}
-
-bool build_band(phast_ctx* h, phast_ctx::Band& B, uint32_t jb) {
-    const Layout& L = h->L;
-    const BandParams bp = band_params(h);
-    const uint32_t nseg = (uint32_t)L.lvl_off.size() - 1, n = h->n;
-    const uint32_t vb = L.lvl_off[jb];
-    const double bw = std::max(1.0, (double)n / bp.bands);
-    // per-level offsets, top-down (j ascending = level descending)
-    std::vector<double> o(nseg, 0.0);
-    for (uint32_t j = jb; j < nseg; j++) {
-        double oj = j > jb ? o[j - 1] : 0.0;
-        bool any = false;
-        double best = 0.0;
-        for (uint32_t v = L.lvl_off[j]; v < L.lvl_off[j + 1]; v++)
-            for (uint32_t e = L.dn_first[v]; e < L.dn_first[v + 1]; e++) {
-                const uint32_t t = L.dn_arc[e].x;
-                if (t < vb) continue;
-                const uint32_t jt = nseg - 1 - L.level[t];
-                const double x = o[jt] + ((double)L.rank[t] - (double)L.rank[v]) / bw + bp.lag;
-                best = any ? std::max(best, x) : x;
-                any = true;
-            }
-        o[j] = any ? best : oj;
-    }
-    struct Task { uint32_t vbeg, vend, level; int64_t key; };
-    std::vector<Task> tasks;
-    std::vector<uint32_t> task_of(n - vb);
-    for (uint32_t j = jb; j < nseg; j++) {
-        const uint32_t a = L.lvl_off[j], b = L.lvl_off[j + 1], lv = nseg - 1 - j;
-        uint32_t v = a;
-        while (v < b) {
-            const int64_t key = (int64_t)std::floor(L.rank[v] / bw + o[j]);
-            uint32_t w = v + 1;
-            while (w < b && (int64_t)std::floor(L.rank[w] / bw + o[j]) == key) w++;
-            for (uint32_t x = v; x < w; x++) task_of[x - vb] = (uint32_t)tasks.size();
-            tasks.push_back(Task{v, w, lv, key});
-            v = w;
-        }
-    }
-    const uint32_t T = (uint32_t)tasks.size();
-    std::vector<uint32_t> seq(T), seq_of(T);
-    for (uint32_t t = 0; t < T; t++) seq[t] = t;
-    std::stable_sort(seq.begin(), seq.end(), [&](uint32_t x, uint32_t y) {
-        if (tasks[x].key != tasks[y].key) return tasks[x].key < tasks[y].key;
-        return tasks[x].level > tasks[y].level;
-    });
-    for (uint32_t i = 0; i < T; i++) seq_of[seq[i]] = i;
-    std::vector<std::vector<uint32_t>> dep(T);   // in sequence indices
-    for (uint32_t i = 0; i < T; i++) {
-        const Task& tk = tasks[seq[i]];
-        std::vector<uint32_t>& d = dep[i];
-        for (uint32_t v = tk.vbeg; v < tk.vend; v++)
-            for (uint32_t e = L.dn_first[v]; e < L.dn_first[v + 1]; e++)
-                if (L.dn_arc[e].x >= vb) d.push_back(seq_of[task_of[L.dn_arc[e].x - vb]]);
-        std::sort(d.begin(), d.end());
-        d.erase(std::unique(d.begin(), d.end()), d.end());
-        if (!d.empty() && d.back() >= i) return false;   // not topological: cannot happen (Lemma 4.1)
-    }
-    B.jb = jb;
-    B.ntasks = T;
-    B.vbeg.resize(T); B.vend.resize(T); B.last.resize(T);
-    B.dep_first.assign(1, 0);
-    B.dep_list.clear();
-    for (uint32_t i = 0; i < T; i++) {
-        const Task& tk = tasks[seq[i]];
-        B.vbeg[i] = tk.vbeg;
-        B.vend[i] = tk.vend;
-        B.last[i] = tk.level == 0 ? 1u : 0u;
-        for (uint32_t u : dep[i]) {   // one-step transitive reduction
-            bool implied = false;
-            for (uint32_t w : dep[i])
-                if (w != u && std::binary_search(dep[w].begin(), dep[w].end(), u)) { implied = true; break; }
-            if (!implied) B.dep_list.push_back(u);
-        }
-        B.dep_first.push_back((uint32_t)B.dep_list.size());
-    }
-    B.chunk_lanes = bp.chunk_lanes;
-    B.unroll = bp.unroll;
-    if (dmalloc(&B.d_dep_first, B.dep_first.size()) || dmalloc(&B.d_dep_list, B.dep_list.size()) ||
-        cudaMemcpy(B.d_dep_first, B.dep_first.data(), B.dep_first.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess ||
-        (!B.dep_list.empty() &&
-         cudaMemcpy(B.d_dep_list, B.dep_list.data(), B.dep_list.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess)) {
-        cudaGetLastError();
-        return false;
-    }
-    for (uint32_t sl = 0; sl < SLOTS; sl++)
-        if (dmalloc(&B.counters[sl], (size_t)T + 1)) return false;
-    return true;
-}
-
-// first banded level: the bottom `levels` levels (band_params), never above the top launch
-uint32_t band_first_level(const phast_ctx* h, uint32_t j0) {
-    const uint32_t nseg = (uint32_t)h->L.lvl_off.size() - 1, m = band_params(h).levels;
-    return std::max(j0, nseg > m ? nseg - m : 0u);
-}
-
-// The band plan for k trees with the banded region starting at level jb, or nullptr
-// (then every level below the top launch gets its own launch).
-phast_ctx::Band* get_band(phast_ctx* h, uint32_t jb) {
-    const uint32_t nseg = (uint32_t)h->L.lvl_off.size() - 1;
-    if ((h->q.flags & PHAST_Q_NO_BAND) || jb + 2 > nseg) return nullptr;   // fewer than two levels to band
-    auto bt = h->bands.find(jb);
-    if (bt == h->bands.end()) {
-        phast_ctx::Band& B = h->bands[jb];
-        B.jb = jb;
-        B.ok = build_band(h, B, jb);
-        if (!B.ok) cudaGetLastError();
-        return B.ok ? &B : nullptr;
-    }
-    return bt->second.ok ? &bt->second : nullptr;
-}
-
-// its chunk table for k trees
-const phast_ctx::Band::PerK* get_band_k(phast_ctx::Band& B, uint32_t k) {
-    auto it = B.perk.find(k);
-    if (it != B.perk.end()) return it->second.chunks ? &it->second : nullptr;
-    phast_ctx::Band::PerK& P = B.perk[k];
-    const uint32_t G = k >= 4 ? k / 4 : 1;
-    const uint32_t CV = std::max(1u, B.chunk_lanes / G);   // vertices per chunk
-    std::vector<uint4> ch;
-    std::vector<uint32_t> nch(B.ntasks);
-    for (uint32_t t = 0; t < B.ntasks; t++) {
-        for (uint32_t v = B.vbeg[t]; v < B.vend[t]; v += CV)
-            ch.push_back(make_uint4(v, std::min(B.vend[t], v + CV), t, B.last[t]));
-        nch[t] = (uint32_t)((B.vend[t] - B.vbeg[t] + CV - 1) / CV);
-    }
-    uint4* dch = nullptr;
-    uint32_t* dn = nullptr;
-    if (dmalloc(&dch, ch.size()) || dmalloc(&dn, nch.size()) ||
-        cudaMemcpy(dch, ch.data(), ch.size() * sizeof(uint4), cudaMemcpyHostToDevice) != cudaSuccess ||
-        cudaMemcpy(dn, nch.data(), nch.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess) {
-        cudaGetLastError();
-        cudaFree(dch);
-        cudaFree(dn);
-        return nullptr;
-    }
-    P.chunks = dch;
-    P.task_nch = dn;
-    P.nchunks = (uint32_t)ch.size();
-    return &P;
-}
-
 constexpr size_t MAX_TIMED_BATCHES = 16384;
 
 cudaEvent_t timing_event(phast_ctx* h) {
@@ -769,39 +563,22 @@ int run_query(phast_ctx* h, const Sources& S, uint32_t kp, const QueryOut& o, cu
     if (cudaEventRecord(h->up_done[s], h->side) != cudaSuccess) return PHAST_ECUDA;
     if (cudaStreamWaitEvent(st, h->up_done[s], 0) != cudaSuccess) return PHAST_ECUDA;
     // a2 on the caller's stream
-    // a3 + a4: the small top levels in one single-CTA launch; below them, the band
-    // dataflow launch, or (PHAST_Q_NO_BAND, the A34 probe) one launch per level
+    if (launch_seed(h->g, sl, kp, o.dist, st) != cudaSuccess) return PHAST_ECUDA;
+    if (e1) cudaEventRecord(e1, st);
+    // a3 + a4: the small top levels in one single-CTA launch, then one launch per level
     // (§VI "The CPU starts, for each level i, a kernel on the GPU")
     const uint32_t levels = (uint32_t)h->L.lvl_off.size() - 1;
-    const uint32_t j0 = top ? top->J : 0u;
-    const uint32_t jb = band_first_level(h, j0);
-    phast_ctx::Band* bp = o.nogather ? nullptr : get_band(h, jb);
-    const phast_ctx::Band::PerK* band = bp ? get_band_k(*bp, kp) : nullptr;
-    const uint32_t jend = band ? jb : levels;
-    if (launch_seed(h->g, sl, kp, o.dist, band ? bp->counters[s] : nullptr, band ? bp->ntasks + 1 : 0u, st) !=
-        cudaSuccess)
-        return PHAST_ECUDA;
-    if (e1) cudaEventRecord(e1, st);
-    if (top && launch_sweep_top(top->a, kp, S, o.dist, sl.flags, o.diam, st) != cudaSuccess) return PHAST_ECUDA;
-    for (uint32_t j = j0; j < jend; j++) {
+    uint32_t j0 = 0;
+    if (top) {
+        if (launch_sweep_top(top->a, kp, S, o.dist, sl.flags, o.diam, st) != cudaSuccess) return PHAST_ECUDA;
+        j0 = top->J;
+    }
+    for (uint32_t j = j0; j < levels; j++) {
         const bool last = (j + 1 == levels);
         const bool store = !(o.diam && last);   // level-0 rows are never read again (diameter mode)
         if (launch_sweep_level(h->g, sl.flags, kp, h->L.lvl_off[j], h->L.lvl_off[j + 1], o.dist, o.diam, store, last,
                                o.nogather, st) != cudaSuccess)
             return PHAST_ECUDA;
-    }
-    if (band) {
-        BandArgs A;
-        A.chunks = band->chunks;
-        A.task_nch = band->task_nch;
-        A.dep_first = bp->d_dep_first;
-        A.dep_list = bp->d_dep_list;
-        A.done = bp->counters[s];
-        A.next = bp->counters[s] + bp->ntasks;
-        A.nchunks = band->nchunks;
-        A.grid = 0;   // the launcher sizes the grid for the unroll's occupancy
-        A.unroll = bp->unroll;
-        if (launch_sweep_band(h->g, A, kp, o.dist, sl.flags, o.diam, st) != cudaSuccess) return PHAST_ECUDA;
     }
     if (launch_clear_flags(sl, kp, h->g.seed_cap, st) != cudaSuccess) return PHAST_ECUDA;
     if (o.compact_to && launch_compact(o.dist, kp, o.compact_to, o.kc, h->n, st) != cudaSuccess) return PHAST_ECUDA;
@@ -995,8 +772,8 @@ int phast_build(uint32_t n, const uint64_t* first, const uint32_t* head, const u
 int phast_configure(phast_ctx* h, const phast_query_opts* q) {
     int rc = check_handle(h);
     if (rc) return rc;
-    phast_query_opts nq = q ? *q : phast_query_opts{};
-    const uint32_t known = PHAST_Q_NO_FUSED | PHAST_Q_NO_TOP | PHAST_Q_HYBRID_ON | PHAST_Q_HYBRID_OFF | PHAST_Q_NO_BAND;
+    phast_query_opts nq = q ? *q : phast_query_opts{0, 0, 0, 0};
+    const uint32_t known = PHAST_Q_NO_FUSED | PHAST_Q_NO_TOP | PHAST_Q_HYBRID_ON | PHAST_Q_HYBRID_OFF;
     if ((nq.flags & ~known) || ((nq.flags & PHAST_Q_HYBRID_ON) && (nq.flags & PHAST_Q_HYBRID_OFF)))
         return PHAST_EINVAL;
     DeviceGuard dg(h->device);
@@ -1360,12 +1137,11 @@ int phast_order(const phast_ctx* h, uint32_t* o) {
     return PHAST_OK;
 }
 
-int phast_export(const phast_ctx* h, uint32_t* level, uint32_t* rank, uint32_t* dn_first, uint32_t* dn_tail,
-                 uint32_t* dn_len, uint32_t* up_first, uint32_t* up_head, uint32_t* up_len) {
+int phast_export(const phast_ctx* h, uint32_t* level, uint32_t* dn_first, uint32_t* dn_tail, uint32_t* dn_len,
+                 uint32_t* up_first, uint32_t* up_head, uint32_t* up_len) {
     if (!h) return PHAST_EINVAL;
     const Layout& L = h->L;
     if (level) std::memcpy(level, L.level.data(), L.level.size() * 4);
-    if (rank) std::memcpy(rank, L.rank.data(), L.rank.size() * 4);
     if (dn_first) std::memcpy(dn_first, L.dn_first.data(), L.dn_first.size() * 4);
     if (up_first) std::memcpy(up_first, L.up_first.data(), L.up_first.size() * 4);
     for (size_t i = 0; i < L.dn_arc.size(); i++) {
@@ -1385,26 +1161,17 @@ int phast_schedule(phast_ctx* h, uint32_t k, uint32_t* out) {
     if (!out || !k_valid(k)) return PHAST_EINVAL;
     DeviceGuard dg(h->device);
     if (!dg.ok) return PHAST_ECUDA;
-    const uint32_t kp = kpad(k);
-    const phast_ctx::Top* t = get_top(h, kp);
+    const phast_ctx::Top* t = get_top(h, kpad(k));
     const uint32_t levels = (uint32_t)h->L.lvl_off.size() - 1;
-    const bool fused = t && t->a.fused;
-    const uint32_t j0 = t ? t->J : 0u;
-    const uint32_t jb = band_first_level(h, j0);
-    phast_ctx::Band* bp = fused ? nullptr : get_band(h, jb);
-    const phast_ctx::Band::PerK* band = bp ? get_band_k(*bp, kp) : nullptr;
-    out[0] = fused ? 1u : 0u;
+    out[0] = t && t->a.fused ? 1u : 0u;
     out[1] = t ? t->J : 0u;
     out[2] = t ? t->a.V : 0u;
-    out[3] = fused ? 0u : (band ? jb : levels) - j0;
-    out[4] = band ? levels - jb : 0u;
-    out[5] = band ? bp->ntasks : 0u;
-    out[6] = band ? band->nchunks : 0u;
+    out[3] = t && t->a.fused ? 0u : levels - (t ? t->J : 0u);
     return PHAST_OK;
 }
 
 // ---------------------------------------------------------------- save / load
-static const char MAGIC[8] = {'P', 'H', 'A', 'S', 'T', 'B', '2', '5'};
+static const char MAGIC[8] = {'P', 'H', 'A', 'S', 'T', 'B', '2', '4'};
 
 int phast_save(const phast_ctx* h, const char* path) {
     if (!h || !path) return PHAST_EINVAL;
@@ -1415,7 +1182,7 @@ int phast_save(const phast_ctx* h, const char* path) {
                         L.mode, 0, L.lvl_off.size()};
     auto wr = [&](const void* p, size_t sz, size_t cnt) { return std::fwrite(p, sz, cnt, f) == cnt; };
     bool ok = wr(MAGIC, 1, 8) && wr(hdr, 8, 10) && wr(&h->build_seconds, 8, 1) && wr(L.perm.data(), 4, h->n) &&
-              wr(L.level.data(), 4, h->n) && wr(L.rank.data(), 4, h->n) && wr(L.lvl_off.data(), 4, L.lvl_off.size()) &&
+              wr(L.level.data(), 4, h->n) && wr(L.lvl_off.data(), 4, L.lvl_off.size()) &&
               wr(L.dn_first.data(), 4, L.dn_first.size()) && wr(L.up_first.data(), 4, L.up_first.size()) &&
               wr(L.dn_arc.data(), 8, L.dn_arc.size()) && wr(L.up_arc.data(), 8, L.up_arc.size());
     const uint64_t n_in = L.in_arc.size();
@@ -1443,7 +1210,7 @@ int phast_load(const char* path, uint32_t flags, phast_ctx** out) {
             h->n = (uint32_t)hdr[0]; L.levels = (uint32_t)hdr[1]; h->m = hdr[2];
             h->shortcuts = hdr[3]; h->rounds = (uint32_t)hdr[4];
             L.mode = (uint32_t)hdr[7];
-            L.perm.resize(h->n); L.iperm.resize(h->n); L.level.resize(h->n); L.rank.resize(h->n);
+            L.perm.resize(h->n); L.iperm.resize(h->n); L.level.resize(h->n);
             L.lvl_off.resize(hdr[9]);
             L.dn_first.resize((size_t)h->n + 1); L.up_first.resize((size_t)h->n + 1);
             L.dn_arc.resize(hdr[5]); L.up_arc.resize(hdr[6]);
@@ -1451,8 +1218,7 @@ int phast_load(const char* path, uint32_t flags, phast_ctx** out) {
             std::fclose(f);
             return PHAST_ENOMEM;
         }
-        ok = rd(L.perm.data(), 4, h->n) && rd(L.level.data(), 4, h->n) && rd(L.rank.data(), 4, h->n) &&
-             rd(L.lvl_off.data(), 4, L.lvl_off.size()) &&
+        ok = rd(L.perm.data(), 4, h->n) && rd(L.level.data(), 4, h->n) && rd(L.lvl_off.data(), 4, L.lvl_off.size()) &&
              rd(L.dn_first.data(), 4, L.dn_first.size()) && rd(L.up_first.data(), 4, L.up_first.size()) &&
              rd(L.dn_arc.data(), 8, L.dn_arc.size()) && rd(L.up_arc.data(), 8, L.up_arc.size());
         uint64_t n_in = 0;

@@ -53,9 +53,7 @@ cudaError_t launch_upward(const DevImage& g, const Slot& sl, const Sources& src,
                           cudaStream_t st);
 // a2: visited bits + rows of the search spaces reset to INF, then (second launch, so
 // that every reset precedes every label) dist[v*k + i] = label_i(v).
-// zero[0..nzero): the slot's band counters (BandArgs::done / next), zeroed here for free
-cudaError_t launch_seed(const DevImage& g, const Slot& sl, uint32_t k, uint32_t* dist, uint32_t* zero, uint32_t nzero,
-                        cudaStream_t st);
+cudaError_t launch_seed(const DevImage& g, const Slot& sl, uint32_t k, uint32_t* dist, cudaStream_t st);
 // a3: one level [vbeg, vend) of the downward sweep; diam != nullptr fuses the max (a5);
 // store == false skips the row stores (diameter mode: level-0 rows are never read);
 // last_level: rows are stored evict-first (nobody reads them again).
@@ -90,30 +88,6 @@ uint32_t top_chunk_vertices(bool big);
 uint32_t top_chunk_arcs(bool big);
 bool top_big_fits(uint32_t k, uint32_t V);   // the big geometry leaves room for the rows
 uint32_t top_heavy_arcs();   // chunk flag (bit 31 of vend): some vertex has more in-arcs than this
-
-// a3 + a4 for the bottom levels [vb, n) in ONE launch (band dataflow, capi.cu: get_band):
-// every level below the shared-memory top launch is cut into spatially aligned bands
-// (band b of each level covers the same quantile of its within-level order); a task
-// = one band of one level = a contiguous id range, and the tasks are sequenced
-// topologically (a task after the tasks holding its tails).  A chunk (<= 4096 lanes
-// of one task) is handed out in sequence order by an atomic counter; before its items
-// the CTA waits until every task the chunk's task depends on has all its chunks done
-// (acquire), after them it counts the chunk done (release).  Tail rows are written
-// shortly before their heads read them, so they are read from L2 instead of being
-// re-read from HBM once per level holding a head.
-struct BandArgs {
-    const uint4* chunks = nullptr;      // [nchunks] {vbeg, vend, task, last-level flag}
-    const uint32_t* task_nch = nullptr; // [ntasks] chunks per task
-    const uint32_t* dep_first = nullptr;// [ntasks+1] CSR of task dependencies (sequence indices)
-    const uint32_t* dep_list = nullptr;
-    uint32_t* done = nullptr;           // [ntasks] completed chunks (slot's; zeroed by launch_seed)
-    uint32_t* next = nullptr;           // [1] chunk dispenser (slot's; zeroed by launch_seed)
-    uint32_t nchunks = 0, grid = 0;
-    uint32_t unroll = 4;                // items per thread per chunk in flight together (2 or 4)
-};
-cudaError_t launch_sweep_band(const DevImage& g, const BandArgs& A, uint32_t k, uint32_t* dist, const uint32_t* flags,
-                              uint32_t* diam, cudaStream_t st);
-uint32_t band_chunk_lanes(uint32_t unroll);   // (vertex, lane) items per chunk: unroll x the CTA size
 
 // a5: max of `count` per-batch maxima into *out
 cudaError_t launch_max_reduce(const uint32_t* in, uint32_t count, uint32_t* out, cudaStream_t st);

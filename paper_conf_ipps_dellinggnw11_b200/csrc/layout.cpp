@@ -88,26 +88,17 @@ int layout_build(const ChResult& R, const uint64_t* first, const uint32_t* head,
         for (uint32_t j = 0; j < levels; j++) pos[levels - 1 - j] = L.lvl_off[j];
         std::vector<uint32_t> by(n);                 // within-level order: input id, or BFS rank
         std::iota(by.begin(), by.end(), 0u);
-        std::vector<uint32_t> rank(n);
-        std::iota(rank.begin(), rank.end(), 0u);
         if (mode == LAYOUT_LEVELS_BFS) {
-            rank = bfs_rank(n, first, head);
+            std::vector<uint32_t> rank = bfs_rank(n, first, head);
             std::sort(by.begin(), by.end(), [&](uint32_t a, uint32_t b) { return rank[a] < rank[b]; });
         }
-        L.rank.resize(n);
         for (uint32_t v : by) order[pos[R.level[v]]++] = v;
-        for (uint32_t v = 0; v < n; v++) L.rank[v] = rank[v];   // by ORIGINAL id; permuted below
         if (mode == LAYOUT_LEVELS_BFS)   // serpentine: odd levels in descending BFS rank, so a
             for (uint32_t j = 0; j < levels; j++)   // level starts where the level above ended (its rows
                 if ((levels - 1 - j) & 1u)          // still in L2): 7.8 % fewer tail-row misses (r1_l2sim.md)
                     std::reverse(order.begin() + L.lvl_off[j], order.begin() + L.lvl_off[j + 1]);
     } else {
         return kEinval;
-    }
-    {   // spatial keys by internal id
-        std::vector<uint32_t> by_orig(std::move(L.rank));
-        L.rank.resize(n);
-        for (uint32_t r = 0; r < n; r++) L.rank[r] = by_orig[order[r]];
     }
     L.perm.assign(n, 0);
     L.iperm = order;

@@ -23,10 +23,6 @@ struct Layout {
     std::vector<uint32_t> perm;      // internal_of_original
     std::vector<uint32_t> iperm;     // original_of_internal
     std::vector<uint32_t> level;     // CH level L of every internal id (0 = lowest)
-    // spatial key of every internal id: BFS rank (LAYOUT_LEVELS_BFS) or input id
-    // (LAYOUT_LEVELS); each level is sorted by it (the odd levels of the serpentine
-    // order backwards), so an interval of keys is a contiguous id range of a level
-    std::vector<uint32_t> rank;
     // Level offsets in processing order: [levels+1] internal ids, j = 0 the top level;
     // no G-down arc has both ends in one level (Lemma 4.1).
     std::vector<uint32_t> lvl_off;

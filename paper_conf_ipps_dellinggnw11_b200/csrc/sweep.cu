@@ -195,10 +195,8 @@ __global__ void __launch_bounds__(UP_THREADS) upward_kernel(DevImage g, Slot sl,
 // ------------------------------------------------------------------ a2 seeding
 // phase 1: visited bits of the search space, and its rows reset to INF
 template <int K>
-__global__ void seed_rows_kernel(Slot sl, uint32_t seed_cap, uint32_t* __restrict__ dist, uint32_t* zero,
-                                 uint32_t nzero) {
+__global__ void seed_rows_kernel(Slot sl, uint32_t seed_cap, uint32_t* __restrict__ dist) {
     const uint32_t i = blockIdx.x;
-    for (uint32_t j = i * blockDim.x + threadIdx.x; j < nzero; j += gridDim.x * blockDim.x) zero[j] = 0u;
     const uint32_t cnt = sl.seed_cnt[i];
     const uint32_t* sv = sl.seed_v + (size_t)i * seed_cap;
     for (uint32_t j = threadIdx.x; j < cnt; j += blockDim.x) {
@@ -332,123 +330,6 @@ cudaError_t sweep_k(const DevImage& g, const uint32_t* flags, uint32_t vbeg, uin
                 : sweep_launch<K, false, true, false, false>(g, flags, vbeg, vend, dist, diam, st);
 }
 
-// ------------------------------------------------------------------ a3 + a4 band dataflow
-
-__device__ __forceinline__ uint32_t ld_acquire_gpu(const uint32_t* p) {
-    uint32_t v;
-    asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
-    return v;
-}
-__device__ __forceinline__ void red_release_gpu_add(uint32_t* p, uint32_t v) {
-    asm volatile("red.release.gpu.global.add.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
-}
-
-// See kernels.h (BandArgs).  Per chunk: wait for the task's dependencies (one thread
-// per dependency spins on an acquire load; then a CTA barrier), relax the chunk's items
-// exactly as sweep_kernel does (§III) with U items per thread in flight
-// together, CTA barrier, one release add.  The chunk's ELL records are loaded before the
-// wait and the next chunk index is fetched while the current chunk runs.  Rows written
-// by other CTAs of this launch are read with ld.global.cg (L2, the coherence point; L1
-// is not coherent and a 128-byte line may hold a row of a band not yet finished).
-// Chunks are handed out in sequence order and every dependency is earlier in the
-// sequence, so the smallest unfinished chunk is always some running CTA's current chunk
-// with its dependencies done: no deadlock, whatever the number of resident CTAs (a CTA
-// takes chunks only while it runs).
-template <int K, bool DIAM, int U>
-__global__ void __launch_bounds__(SWEEP_THREADS, U == 2 ? 6 : 4)
-    band_kernel(BandArgs A, const uint4* __restrict__ rec, const uint2* __restrict__ ovf, uint32_t* __restrict__ d,
-                const uint32_t* __restrict__ flags, uint32_t* __restrict__ diam) {
-    using T = typename RowT<K>::T;
-    constexpr uint32_t G = K / RowT<K>::W;   // lanes per vertex
-    __shared__ uint32_t s_c[2];
-    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
-    asm volatile("griddepcontrol.wait;" ::: "memory");   // the levels above complete and visible
-    const uint32_t tid = threadIdx.x;
-    if (tid == 0) s_c[0] = atomicAdd(A.next, 1u);
-    __syncthreads();
-    uint32_t c = s_c[0], it = 0, mx = 0;
-    while (c < A.nchunks) {
-        const uint4 ch = __ldg(&A.chunks[c]);   // {vbeg, vend, task, last level}
-        uint32_t nxt = 0;
-        if (tid == 0) nxt = atomicAdd(A.next, 1u);   // the next chunk, in flight meanwhile
-        const uint32_t total = (ch.y - ch.x) * G;     // <= U * SWEEP_THREADS (host: chunk geometry)
-        uint4 r[U];
-#pragma unroll
-        for (uint32_t u = 0; u < U; u++) {
-            const uint32_t t = tid + u * SWEEP_THREADS;
-            r[u] = t < total ? __ldg(&rec[ch.x + t / G]) : make_uint4(0u, INF, 0u, INF);
-        }
-        const uint32_t d1 = __ldg(&A.dep_first[ch.z + 1]);
-        for (uint32_t i = __ldg(&A.dep_first[ch.z]) + tid; i < d1; i += SWEEP_THREADS) {
-            const uint32_t u = __ldg(&A.dep_list[i]);
-            const uint32_t need = __ldg(&A.task_nch[u]);
-            while (ld_acquire_gpu(&A.done[u]) < need) __nanosleep(64);
-        }
-        __syncthreads();   // every dependency complete, for every thread of the CTA
-        T x0[U], x1[U];
-#pragma unroll
-        for (uint32_t u = 0; u < U; u++) {   // all tail-row gathers of the thread in flight at once
-            const uint32_t lane = (tid + u * SWEEP_THREADS) % G;
-            x0[u] = r[u].y != INF ? __ldcg(reinterpret_cast<const T*>(d + (size_t)r[u].x * K) + lane) : inf_row<T>();
-            x1[u] = r[u].w != INF ? __ldcg(reinterpret_cast<const T*>(d + (size_t)r[u].z * K) + lane) : inf_row<T>();
-        }
-#pragma unroll
-        for (uint32_t u = 0; u < U; u++) {
-            const uint32_t t = tid + u * SWEEP_THREADS;
-            if (t >= total) break;
-            const uint32_t v = ch.x + t / G, lane = t % G;
-            T acc = inf_row<T>();
-            if (visited(flags, v)) acc = __ldcg(reinterpret_cast<const T*>(d + (size_t)v * K) + lane);
-            acc = relax(relax(acc, x0[u], r[u].y), x1[u], r[u].w);
-            if (r[u].w == INF && r[u].z != INF) {   // more than two in-arcs: the rest in the overflow list
-                const uint2* o = ovf + r[u].z;
-                const uint32_t cnt = __ldg(&o->x);
-                for (uint32_t j = 1; j <= cnt; j++) {
-                    const uint2 a = __ldg(&o[j]);
-                    acc = relax(acc, __ldcg(reinterpret_cast<const T*>(d + (size_t)a.x * K) + lane), a.y);
-                }
-            }
-            T* p = reinterpret_cast<T*>(d + (size_t)v * K) + lane;
-            if (ch.w) {                                  // level 0: nobody's tail
-                if constexpr (!DIAM) __stcs(p, acc);     // diameter mode: not stored at all
-            } else {
-                *p = acc;
-            }
-            if constexpr (DIAM) mx = max(mx, fmax_of(acc));
-        }
-        it ^= 1u;
-        if (tid == 0) s_c[it] = nxt;
-        __syncthreads();   // the chunk's rows are written (and the next index published)
-        if (tid == 0) red_release_gpu_add(&A.done[ch.z], 1u);
-        c = s_c[it];
-    }
-    if constexpr (DIAM) cta_max_to<SWEEP_THREADS>(mx, diam);
-}
-
-template <int K, int U>
-cudaError_t band_ku(const DevImage& g, const BandArgs& A, uint32_t* dist, const uint32_t* flags, uint32_t* diam,
-                    cudaStream_t st) {
-    cudaLaunchConfig_t cfg = {};
-    cfg.gridDim = dim3(std::min<uint32_t>(A.nchunks, (U == 2 ? 6u : 4u) * (uint32_t)num_sms()));
-    cfg.blockDim = dim3(SWEEP_THREADS);
-    cfg.stream = st;
-    cudaLaunchAttribute attr[1];
-    attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
-    attr[0].val.programmaticStreamSerializationAllowed = 1;
-    cfg.attrs = attr;
-    cfg.numAttrs = 1;
-    cudaError_t e = diam ? cudaLaunchKernelEx(&cfg, band_kernel<K, true, U>, A, g.dn_rec, g.dn_ovf, dist, flags, diam)
-                         : cudaLaunchKernelEx(&cfg, band_kernel<K, false, U>, A, g.dn_rec, g.dn_ovf, dist, flags, diam);
-    count_launch();
-    return e;
-}
-
-template <int K>
-cudaError_t band_k(const DevImage& g, const BandArgs& A, uint32_t* dist, const uint32_t* flags, uint32_t* diam,
-                   cudaStream_t st) {
-    return A.unroll == 2 ? band_ku<K, 2>(g, A, dist, flags, diam, st) : band_ku<K, 4>(g, A, dist, flags, diam, st);
-}
-
 // ------------------------------------------------------------------ probe A33
 // Sequential stream over the sweep's arrays: every ELL record read, every label row
 // read and written once (no gathers, no level dependencies, ONE launch).
@@ -526,8 +407,8 @@ unsigned grid_for(uint64_t items) {
 }
 
 template <int K>
-cudaError_t seed_k(const DevImage& g, const Slot& sl, uint32_t* dist, uint32_t* zero, uint32_t nzero, cudaStream_t st) {
-    seed_rows_kernel<K><<<K, 256, 0, st>>>(sl, g.seed_cap, dist, zero, nzero);
+cudaError_t seed_k(const DevImage& g, const Slot& sl, uint32_t* dist, cudaStream_t st) {
+    seed_rows_kernel<K><<<K, 256, 0, st>>>(sl, g.seed_cap, dist);
     count_launch();
     return cudaGetLastError();
 }
@@ -544,9 +425,8 @@ cudaError_t launch_upward(const DevImage& g, const Slot& sl, const Sources& src,
     return cudaGetLastError();
 }
 
-cudaError_t launch_seed(const DevImage& g, const Slot& sl, uint32_t k, uint32_t* dist, uint32_t* zero, uint32_t nzero,
-                        cudaStream_t st) {
-#define CALL_SR(K) seed_k<K>(g, sl, dist, zero, nzero, st)
+cudaError_t launch_seed(const DevImage& g, const Slot& sl, uint32_t k, uint32_t* dist, cudaStream_t st) {
+#define CALL_SR(K) seed_k<K>(g, sl, dist, st)
     cudaError_t e = [&]() -> cudaError_t { PHAST_K_SWITCH(k, CALL_SR) }();
 #undef CALL_SR
     if (e != cudaSuccess) return e;
@@ -561,15 +441,6 @@ cudaError_t launch_sweep_level(const DevImage& g, const uint32_t* flags, uint32_
 #define CALL_SW(K) sweep_k<K>(g, flags, vbeg, vend, dist, diam, store, last_level, nogather, st)
     PHAST_K_SWITCH(k, CALL_SW)
 #undef CALL_SW
-}
-
-uint32_t band_chunk_lanes(uint32_t unroll) { return unroll * SWEEP_THREADS; }
-
-cudaError_t launch_sweep_band(const DevImage& g, const BandArgs& A, uint32_t k, uint32_t* dist, const uint32_t* flags,
-                              uint32_t* diam, cudaStream_t st) {
-#define CALL_BD(K) band_k<K>(g, A, dist, flags, diam, st)
-    PHAST_K_SWITCH(k, CALL_BD)
-#undef CALL_BD
 }
 
 cudaError_t launch_clear_flags(const Slot& sl, uint32_t k, uint32_t seed_cap, cudaStream_t st) {

@@ -160,9 +160,7 @@ def test_upward_global_fallback_and_overflow():
 
 SCHEDULES = {
     "default": {},
-    "per_level": dict(flags=P.Q_NO_TOP | P.Q_NO_FUSED | P.Q_NO_BAND),   # the paper's: one launch per level
-    "band_all": dict(flags=P.Q_NO_TOP | P.Q_NO_FUSED),                  # every level in the band launch
-    "top_then_levels": dict(flags=P.Q_NO_FUSED | P.Q_NO_BAND),
+    "per_level": dict(flags=P.Q_NO_TOP | P.Q_NO_FUSED),          # the paper's: one launch per level
     "top_hybrid": dict(flags=P.Q_NO_FUSED | P.Q_HYBRID_ON),
     "top_full_searches": dict(flags=P.Q_NO_FUSED | P.Q_HYBRID_OFF),
     "top_40": dict(flags=P.Q_NO_FUSED, top_max_vertices=40),    # the prefix ends inside the hierarchy
@@ -199,11 +197,9 @@ def test_schedule_reports_launch_shape():
     g = phastgen.road(120_000, seed=33)
     with P.Phast.from_graph(g) as h:
         s = h.schedule(64)
-        assert not s["fused"] and s["top_levels"] >= 2 and s["level_launches"] == 0
-        assert s["top_levels"] + s["band_levels"] == h.levels and s["band_tasks"] > 0
-        h.configure(flags=P.Q_NO_TOP | P.Q_NO_FUSED | P.Q_NO_BAND)
-        s = h.schedule(64)
-        assert (s["fused"], s["top_levels"], s["level_launches"], s["band_levels"]) == (False, 0, h.levels, 0)
+        assert not s["fused"] and s["top_levels"] >= 2 and s["top_levels"] + s["level_launches"] == h.levels
+        h.configure(flags=P.Q_NO_TOP | P.Q_NO_FUSED)
+        assert h.schedule(64) == dict(fused=False, top_levels=0, top_vertices=0, level_launches=h.levels)
 
 
 def test_fused_query_edge_cases():
