@@ -29,6 +29,7 @@ struct phast_ctx {
     uint32_t rounds = 0;
     double build_seconds = 0;
     Layout L;
+    std::vector<uint8_t> wide;          // per level (top-down): the two-record ELL format (DevImage::dn_rec2)
     phast_query_opts q = {0, 0, 0, 0};
     // upward-search-space statistics of phast_info (host sample, computed once)
     mutable bool up_stats = false;
@@ -98,6 +99,9 @@ namespace {
 
 constexpr uint32_t SEED_CAP = 1u << 16;   // default per-source search-space capacity
 constexpr uint32_t UP_SAMPLE = 1024;      // sources sampled for phast_info's search-space stats
+// a level gets the two-record ELL format when more than this share of its vertices have
+// more than two in-arcs (C3: levels 2-11 and 14-; 35-81 % of their vertices)
+constexpr double WIDE_SHARE = 0.15;
 
 // the vector widths the kernels are instantiated for; any other k runs at the next one
 uint32_t kpad(uint32_t k) {
@@ -210,7 +214,7 @@ void free_device(phast_ctx* h) {
     if (h->side) cudaStreamDestroy(h->side);
     h->side = nullptr;
     cudaFree((void*)h->g.dn_first); cudaFree((void*)h->g.dn_arc);
-    cudaFree((void*)h->g.dn_rec); cudaFree((void*)h->g.dn_ovf);
+    cudaFree((void*)h->g.dn_rec); cudaFree((void*)h->g.dn_rec2); cudaFree((void*)h->g.dn_ovf);
     cudaFree((void*)h->g.up_first); cudaFree((void*)h->g.up_arc);
     cudaFree(h->g.err);
     cudaFree(h->host_scratch); cudaFree(h->batch_max_scratch); cudaFree(h->wit);
@@ -270,32 +274,61 @@ int upload(phast_ctx* h) {
         free_device(h);
         return rc;
     }
-    // G-down as ELL-2 records + overflow lists (kernels.h: DevImage::dn_rec)
+    // G-down as ELL records + overflow lists (kernels.h: DevImage::dn_rec / dn_rec2); a
+    // level is "wide" when more than WIDE_SHARE of its vertices have more than two in-arcs
     {
-        std::vector<uint4> rec(h->n);
-        std::vector<Arc> ovf;
-        for (uint32_t v = 0; v < h->n; v++) {
-            const uint32_t e0 = L.dn_first[v], deg = L.dn_first[v + 1] - e0;
-            uint4 r = make_uint4(INF, INF, INF, INF);
-            if (deg >= 1) { r.x = L.dn_arc[e0].x; r.y = L.dn_arc[e0].y; }
-            if (deg == 2) { r.z = L.dn_arc[e0 + 1].x; r.w = L.dn_arc[e0 + 1].y; }
-            if (deg > 2) {
-                r.z = (uint32_t)ovf.size();
-                ovf.push_back(Arc{deg - 1, 0});
-                for (uint32_t e = e0 + 1; e < e0 + deg; e++) ovf.push_back(L.dn_arc[e]);
-            }
-            rec[v] = r;
+        const uint32_t nseg = (uint32_t)L.lvl_off.size() - 1;
+        h->wide.assign(nseg, 0);
+        bool any_wide = false;
+        for (uint32_t j = 0; j < nseg; j++) {
+            uint32_t many = 0;
+            for (uint32_t v = L.lvl_off[j]; v < L.lvl_off[j + 1]; v++) many += L.dn_first[v + 1] - L.dn_first[v] > 2;
+            h->wide[j] = (double)many > WIDE_SHARE * (L.lvl_off[j + 1] - L.lvl_off[j]) ? 1 : 0;
+            any_wide |= h->wide[j] != 0;
         }
-        uint4* dr = nullptr;
+        std::vector<uint4> rec(h->n), rec2(any_wide ? h->n : 0, make_uint4(INF, INF, INF, INF));
+        std::vector<Arc> ovf;
+        for (uint32_t j = 0; j < nseg; j++)
+            for (uint32_t v = L.lvl_off[j]; v < L.lvl_off[j + 1]; v++) {
+                const uint32_t e0 = L.dn_first[v], deg = L.dn_first[v + 1] - e0;
+                const Arc* a = L.dn_arc.data() + e0;
+                uint4 r = make_uint4(INF, INF, INF, INF);
+                if (deg >= 1) { r.x = a[0].x; r.y = a[0].y; }
+                if (h->wide[j]) {   // arcs 0-1 | 2-3, or 2 + overflow
+                    if (deg >= 2) { r.z = a[1].x; r.w = a[1].y; }
+                    uint4 r2 = make_uint4(INF, INF, INF, INF);
+                    if (deg >= 3) { r2.x = a[2].x; r2.y = a[2].y; }
+                    if (deg == 4) { r2.z = a[3].x; r2.w = a[3].y; }
+                    if (deg > 4) {
+                        r2.z = (uint32_t)ovf.size();
+                        ovf.push_back(Arc{deg - 3, 0});
+                        for (uint32_t e = 3; e < deg; e++) ovf.push_back(a[e]);
+                    }
+                    rec2[v] = r2;
+                } else {            // arcs 0-1, or 0 + overflow
+                    if (deg == 2) { r.z = a[1].x; r.w = a[1].y; }
+                    if (deg > 2) {
+                        r.z = (uint32_t)ovf.size();
+                        ovf.push_back(Arc{deg - 1, 0});
+                        for (uint32_t e = 1; e < deg; e++) ovf.push_back(a[e]);
+                    }
+                }
+                rec[v] = r;
+            }
+        uint4 *dr = nullptr, *dr2 = nullptr;
         uint2* dov = nullptr;
-        if (ovf.size() >= INF || (rc = dmalloc(&dr, rec.size())) || (rc = dmalloc(&dov, ovf.size()))) {
+        if (ovf.size() >= INF || (rc = dmalloc(&dr, rec.size())) || (rc = dmalloc(&dov, ovf.size())) ||
+            (any_wide && (rc = dmalloc(&dr2, rec2.size())))) {
             cudaFree(dr);
+            cudaFree(dov);
             free_device(h);
             return rc ? rc : PHAST_ERANGE;
         }
         g.dn_rec = dr;
+        g.dn_rec2 = dr2;
         g.dn_ovf = dov;
         if (cudaMemcpy(dr, rec.data(), rec.size() * sizeof(uint4), cudaMemcpyHostToDevice) != cudaSuccess ||
+            (any_wide && cudaMemcpy(dr2, rec2.data(), rec2.size() * sizeof(uint4), cudaMemcpyHostToDevice) != cudaSuccess) ||
             (!ovf.empty() && cudaMemcpy(dov, ovf.data(), ovf.size() * 8, cudaMemcpyHostToDevice) != cudaSuccess)) {
             cudaGetLastError();
             free_device(h);
@@ -577,7 +610,7 @@ int run_query(phast_ctx* h, const Sources& S, uint32_t kp, const QueryOut& o, cu
         const bool last = (j + 1 == levels);
         const bool store = !(o.diam && last);   // level-0 rows are never read again (diameter mode)
         if (launch_sweep_level(h->g, sl.flags, kp, h->L.lvl_off[j], h->L.lvl_off[j + 1], o.dist, o.diam, store, last,
-                               o.nogather, st) != cudaSuccess)
+                               o.nogather, h->wide[j] != 0, st) != cudaSuccess)
             return PHAST_ECUDA;
     }
     if (launch_clear_flags(sl, kp, h->g.seed_cap, st) != cudaSuccess) return PHAST_ECUDA;

@@ -25,6 +25,11 @@ struct DevImage {
     // len1 = INF with tail1 != INF: more than two in-arcs, tail1 indexes dn_ovf = {count,
     // 0} followed by the remaining count arcs {tail, len}
     const uint4* dn_rec = nullptr;       // [n]
+    // "wide" levels (capi.cu: many vertices with 3-4 in-arcs) use two records loaded
+    // side by side: rec[v] = {tail0, len0, tail1, len1} and rec2[v] = {tail2, len2,
+    // tail3, len3} (INF-padded); more than four in-arcs: len3 = INF with tail3 != INF
+    // indexing dn_ovf = {count, 0} followed by the arcs from the fourth on
+    const uint4* dn_rec2 = nullptr;      // [n] (entries of wide levels only)
     const uint2* dn_ovf = nullptr;       // [overflow entries]
     const uint32_t* up_first = nullptr;  // [n+1]   G-up out-arcs by tail
     const uint2* up_arc = nullptr;       // [m_up]   {head, len}
@@ -58,8 +63,9 @@ cudaError_t launch_seed(const DevImage& g, const Slot& sl, uint32_t k, uint32_t*
 // store == false skips the row stores (diameter mode: level-0 rows are never read);
 // last_level: rows are stored evict-first (nobody reads them again).
 // nogather (probe A34): every tail-row gather is replaced by the arc length itself.
+// wide: the level's records are in the two-record format (DevImage::dn_rec2).
 cudaError_t launch_sweep_level(const DevImage& g, const uint32_t* flags, uint32_t k, uint32_t vbeg, uint32_t vend,
-                               uint32_t* dist, uint32_t* diam, bool store, bool last_level, bool nogather,
+                               uint32_t* dist, uint32_t* diam, bool store, bool last_level, bool nogather, bool wide,
                                cudaStream_t st);
 // after the sweep: clear the visited bits of every search-space vertex ("After
 // scanning v we unmark the vertex", §IV-C).

@@ -240,10 +240,13 @@ constexpr int SWEEP_THREADS = 256;
 // NOGATHER (probe A34, §VIII-B "it takes 153 ms to traverse the graph
 // exactly as PHAST does, but storing at d(v) the sum of the lengths of all arcs into
 // v"): identical traversal, with every tail row replaced by the arc's length.
-template <int K, bool DIAM, bool STORE, bool STREAM, bool NOGATHER>
-__global__ void __launch_bounds__(SWEEP_THREADS, 8)
-    sweep_kernel(const uint4* __restrict__ rec, const uint2* __restrict__ ovf, uint32_t* __restrict__ d,
-                 const uint32_t* __restrict__ flags, uint32_t vbeg, uint32_t vend, uint32_t* __restrict__ diam) {
+// WIDE (levels where many vertices have 3-4 in-arcs): a second record with arcs 2-3 is
+// loaded beside the first, so up to four gathers depend on one round trip.
+template <int K, bool DIAM, bool STORE, bool STREAM, bool NOGATHER, bool WIDE>
+__global__ void __launch_bounds__(SWEEP_THREADS, WIDE ? 6 : 8)   // WIDE: registers for four rows in flight
+    sweep_kernel(const uint4* __restrict__ rec, const uint4* __restrict__ rec2, const uint2* __restrict__ ovf,
+                 uint32_t* __restrict__ d, const uint32_t* __restrict__ flags, uint32_t vbeg, uint32_t vend,
+                 uint32_t* __restrict__ diam) {
     using T = typename RowT<K>::T;
     constexpr uint32_t G = K / RowT<K>::W;   // lanes per vertex
     asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
@@ -258,17 +261,27 @@ __global__ void __launch_bounds__(SWEEP_THREADS, 8)
         T acc = inf_row<T>();
         if (visited(flags, v)) acc = __ldg(reinterpret_cast<const T*>(d + (size_t)v * K) + lane);
         const uint4 r = __ldg(&rec[v]);
-        T x0 = inf_row<T>(), x1 = inf_row<T>();
+        uint4 r2 = make_uint4(0u, INF, 0u, INF);
+        if constexpr (WIDE) r2 = __ldg(&rec2[v]);
+        const bool more = WIDE ? (r2.w == INF && r2.z != INF) : (r.w == INF && r.z != INF);   // overflow list
+        const uint32_t oi = WIDE ? r2.z : r.z;
         if constexpr (NOGATHER) {
-            acc = splat<T>(min(r.y, 0xFFFFFFFEu) + (r.w == INF ? 0u : r.w));
+            acc = splat<T>(sat_add(sat_add(min(r.y, 0xFFFFFFFEu), r.w == INF ? 0u : r.w),
+                                   sat_add(r2.y == INF ? 0u : r2.y, (r2.w == INF || !WIDE) ? 0u : r2.w)));
         } else {
             // a missing arc has len INF: relaxing an INF row by it changes nothing
+            T x0 = inf_row<T>(), x1 = inf_row<T>(), x2 = inf_row<T>(), x3 = inf_row<T>();
             if (r.y != INF) x0 = __ldg(reinterpret_cast<const T*>(d + (size_t)r.x * K) + lane);
             if (r.w != INF) x1 = __ldg(reinterpret_cast<const T*>(d + (size_t)r.z * K) + lane);
+            if constexpr (WIDE) {
+                if (r2.y != INF) x2 = __ldg(reinterpret_cast<const T*>(d + (size_t)r2.x * K) + lane);
+                if (r2.w != INF) x3 = __ldg(reinterpret_cast<const T*>(d + (size_t)r2.z * K) + lane);
+            }
             acc = relax(relax(acc, x0, r.y), x1, r.w);
+            if constexpr (WIDE) acc = relax(relax(acc, x2, r2.y), x3, r2.w);
         }
-        if (r.w == INF && r.z != INF) {   // more than two in-arcs: the rest in the overflow list
-            const uint2* o = ovf + r.z;
+        if (more) {   // the rest in the overflow list
+            const uint2* o = ovf + oi;
             const uint32_t cnt = __ldg(&o->x);
             for (uint32_t j = 1; j <= cnt; j++) {
                 const uint2 a = __ldg(&o[j]);
@@ -285,20 +298,20 @@ __global__ void __launch_bounds__(SWEEP_THREADS, 8)
     if constexpr (DIAM) cta_max_to<SWEEP_THREADS>(mx, diam);
 }
 
-template <int K, bool DIAM, bool STORE, bool STREAM, bool NOGATHER>
+template <int K, bool DIAM, bool STORE, bool STREAM, bool NOGATHER, bool WIDE>
 cudaError_t sweep_launch(const DevImage& g, const uint32_t* flags, uint32_t vbeg, uint32_t vend, uint32_t* dist,
                          uint32_t* diam, cudaStream_t st) {
     constexpr uint32_t G = K / RowT<K>::W;
     constexpr uint32_t VMAX = (1u << 31) / G;   // 32-bit item indices in the kernel
     if (vend - vbeg > VMAX) {                    // a level has no internal arcs: split it freely
-        cudaError_t e = sweep_launch<K, DIAM, STORE, STREAM, NOGATHER>(g, flags, vbeg, vbeg + VMAX, dist, diam, st);
+        cudaError_t e = sweep_launch<K, DIAM, STORE, STREAM, NOGATHER, WIDE>(g, flags, vbeg, vbeg + VMAX, dist, diam, st);
         return e != cudaSuccess ? e
-                                : sweep_launch<K, DIAM, STORE, STREAM, NOGATHER>(g, flags, vbeg + VMAX, vend, dist,
-                                                                                 diam, st);
+                                : sweep_launch<K, DIAM, STORE, STREAM, NOGATHER, WIDE>(g, flags, vbeg + VMAX, vend, dist,
+                                                                                       diam, st);
     }
     const uint64_t total = (uint64_t)(vend - vbeg) * G;
     uint64_t blocks = (total + SWEEP_THREADS - 1) / SWEEP_THREADS;
-    const uint64_t cap = (uint64_t)num_sms() * 8;   // one full wave of resident CTAs (launch bounds: 8)
+    const uint64_t cap = (uint64_t)num_sms() * (WIDE ? 6 : 8);   // one full wave of resident CTAs (launch bounds)
     if (blocks > cap) blocks = cap;
     if (blocks == 0) return cudaSuccess;
     cudaLaunchConfig_t cfg = {};
@@ -311,23 +324,30 @@ cudaError_t sweep_launch(const DevImage& g, const uint32_t* flags, uint32_t vbeg
     attr[0].val.programmaticStreamSerializationAllowed = 1;
     cfg.attrs = attr;
     cfg.numAttrs = 1;
-    cudaError_t e = cudaLaunchKernelEx(&cfg, sweep_kernel<K, DIAM, STORE, STREAM, NOGATHER>, g.dn_rec, g.dn_ovf,
-                                       dist, flags, vbeg, vend, diam);
+    cudaError_t e = cudaLaunchKernelEx(&cfg, sweep_kernel<K, DIAM, STORE, STREAM, NOGATHER, WIDE>, g.dn_rec, g.dn_rec2,
+                                       g.dn_ovf, dist, flags, vbeg, vend, diam);
     count_launch();
     return e;
 }
 
+template <int K, bool WIDE>
+cudaError_t sweep_kw(const DevImage& g, const uint32_t* flags, uint32_t vbeg, uint32_t vend, uint32_t* dist,
+                     uint32_t* diam, bool store, bool last, bool nogather, cudaStream_t st) {
+    if (nogather) return sweep_launch<K, false, true, false, true, WIDE>(g, flags, vbeg, vend, dist, diam, st);
+    if (diam) {
+        if (!store) return sweep_launch<K, true, false, false, false, WIDE>(g, flags, vbeg, vend, dist, diam, st);
+        return last ? sweep_launch<K, true, true, true, false, WIDE>(g, flags, vbeg, vend, dist, diam, st)
+                    : sweep_launch<K, true, true, false, false, WIDE>(g, flags, vbeg, vend, dist, diam, st);
+    }
+    return last ? sweep_launch<K, false, true, true, false, WIDE>(g, flags, vbeg, vend, dist, diam, st)
+                : sweep_launch<K, false, true, false, false, WIDE>(g, flags, vbeg, vend, dist, diam, st);
+}
+
 template <int K>
 cudaError_t sweep_k(const DevImage& g, const uint32_t* flags, uint32_t vbeg, uint32_t vend, uint32_t* dist,
-                    uint32_t* diam, bool store, bool last, bool nogather, cudaStream_t st) {
-    if (nogather) return sweep_launch<K, false, true, false, true>(g, flags, vbeg, vend, dist, diam, st);
-    if (diam) {
-        if (!store) return sweep_launch<K, true, false, false, false>(g, flags, vbeg, vend, dist, diam, st);
-        return last ? sweep_launch<K, true, true, true, false>(g, flags, vbeg, vend, dist, diam, st)
-                    : sweep_launch<K, true, true, false, false>(g, flags, vbeg, vend, dist, diam, st);
-    }
-    return last ? sweep_launch<K, false, true, true, false>(g, flags, vbeg, vend, dist, diam, st)
-                : sweep_launch<K, false, true, false, false>(g, flags, vbeg, vend, dist, diam, st);
+                    uint32_t* diam, bool store, bool last, bool nogather, bool wide, cudaStream_t st) {
+    return wide ? sweep_kw<K, true>(g, flags, vbeg, vend, dist, diam, store, last, nogather, st)
+                : sweep_kw<K, false>(g, flags, vbeg, vend, dist, diam, store, last, nogather, st);
 }
 
 // ------------------------------------------------------------------ probe A33
@@ -436,9 +456,9 @@ cudaError_t launch_seed(const DevImage& g, const Slot& sl, uint32_t k, uint32_t*
 }
 
 cudaError_t launch_sweep_level(const DevImage& g, const uint32_t* flags, uint32_t k, uint32_t vbeg, uint32_t vend,
-                               uint32_t* dist, uint32_t* diam, bool store, bool last_level, bool nogather,
+                               uint32_t* dist, uint32_t* diam, bool store, bool last_level, bool nogather, bool wide,
                                cudaStream_t st) {
-#define CALL_SW(K) sweep_k<K>(g, flags, vbeg, vend, dist, diam, store, last_level, nogather, st)
+#define CALL_SW(K) sweep_k<K>(g, flags, vbeg, vend, dist, diam, store, last_level, nogather, wide, st)
     PHAST_K_SWITCH(k, CALL_SW)
 #undef CALL_SW
 }
