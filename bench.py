@@ -220,6 +220,8 @@ def main():
     ap.add_argument("--cache", default="", help="hierarchy file to reuse/create (optional)")
     ap.add_argument("--layout", default="levels-bfs", choices=["levels", "levels-bfs"],
                     help="vertex order: the paper's level layout (DFS within a level) or BFS within a level")
+    ap.add_argument("--query-flags", type=int, default=0,
+                    help="phast_configure flags (schedule experiments: 1 no fused single-launch query, 2 no shared-memory top launch)")
     ap.add_argument("--parents", action="store_true",
                     help="also time the parent-pointer pass (phast_parents, NEXT-1) on the last batch")
     args = ap.parse_args()
@@ -277,6 +279,8 @@ def main():
         log(f"[bench] CH build {time.time() - t:.1f}s")
         if args.cache:
             h.save(args.cache)
+    if args.query_flags:
+        h.configure(flags=args.query_flags)
     n = h.n
     info = h.info()
     lsz = h.level_sizes()
