@@ -28,7 +28,7 @@ FLAG_LEVEL_LAYOUT = 2
 FLAG_BFS_IN_LEVEL = 4
 LAYOUT_FLAGS = {"levels-bfs": 0, "levels": FLAG_LEVEL_LAYOUT}
 LAYOUT_NAMES = {1: "levels", 2: "levels-bfs"}   # phast_info_t.layout
-Q_NO_FUSED, Q_NO_TOP, Q_HYBRID_ON, Q_HYBRID_OFF = 1, 2, 4, 8
+Q_NO_FUSED, Q_NO_TOP, Q_HYBRID_ON, Q_HYBRID_OFF, Q_NO_MULTI = 1, 2, 4, 8, 32
 
 STATUS = {0: "OK", -1: "EINVAL", -2: "ENOMEM", -3: "ECUDA", -4: "ERANGE", -5: "ESTATE", -6: "EIO",
           -7: "EINTERNAL"}

@@ -6,6 +6,7 @@
 // (§IV-A).  G-down: in-arcs by head, {tail, len} (§IV-A),
 // sentinel dn_first[n].  G-up: out-arcs by tail, {head, len}.
 #include <algorithm>
+#include <array>
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
@@ -67,6 +68,7 @@ struct phast_ctx {
     double* bc_sigma = nullptr;
     double* bc_delta = nullptr;
     uint32_t* bc_dist = nullptr;
+    uint32_t* bc_src = nullptr;         // [B*k] internal ids of a group's trees
     size_t bc_elems = 0;
     uint32_t* bc_changed = nullptr;
     uint32_t* bc_changed_host = nullptr;
@@ -78,6 +80,7 @@ struct phast_ctx {
     // top levels [0, J) swept in one single-CTA launch (launch_sweep_top), one plan per k
     struct Top {
         uint4* chunks = nullptr;   // device [nchunks] {vbeg, vend, first[vbeg], first[vend]}
+        uint4* rnd = nullptr;      // device [2 nchunks] rounds of multi-level chunks
         TopArgs a;                 // a.fused: the whole query in this one launch
         uint32_t J = 0;            // levels [0, J) in the shared-memory launch (0: none)
         uint32_t vtop = 0;         // upward searches stop expanding below this id (0: full searches)
@@ -152,6 +155,7 @@ int grow(T** p, size_t* have, size_t elems) {
 void free_tops(phast_ctx* h) {
     for (auto& kv : h->tops) {
         cudaFree(kv.second.chunks);
+        cudaFree(kv.second.rnd);
         cudaFree(kv.second.up_f);
         cudaFree(kv.second.up_a);
     }
@@ -220,7 +224,7 @@ void free_device(phast_ctx* h) {
     cudaFree(h->host_scratch); cudaFree(h->batch_max_scratch); cudaFree(h->wit);
     cudaFree(h->d_in_first); cudaFree(h->d_in_arc);
     cudaFree(h->d_out_first); cudaFree(h->d_out_arc);
-    cudaFree(h->bc_sigma); cudaFree(h->bc_delta); cudaFree(h->bc_dist);
+    cudaFree(h->bc_sigma); cudaFree(h->bc_delta); cudaFree(h->bc_dist); cudaFree(h->bc_src);
     cudaFree(h->bc_changed); cudaFreeHost(h->bc_changed_host); cudaFree(h->bc_q); cudaFree(h->bc_qs);
     if (h->bc_stream) cudaStreamDestroy(h->bc_stream);
     if (h->bc_ev) cudaEventDestroy(h->bc_ev);
@@ -229,7 +233,7 @@ void free_device(phast_ctx* h) {
     h->batch_max_scratch = nullptr; h->batch_max_elems = 0; h->wit = nullptr;
     h->d_in_first = nullptr; h->d_in_arc = nullptr;
     h->d_out_first = nullptr; h->d_out_arc = nullptr;
-    h->bc_sigma = h->bc_delta = nullptr; h->bc_dist = nullptr; h->bc_elems = 0;
+    h->bc_sigma = h->bc_delta = nullptr; h->bc_dist = nullptr; h->bc_src = nullptr; h->bc_elems = 0;
     h->bc_changed = nullptr; h->bc_changed_host = nullptr; h->bc_q = nullptr; h->bc_qs = nullptr;
     h->bc_stream = nullptr; h->bc_ev = nullptr;
     h->d_upin_first = nullptr; h->d_upin_arc = nullptr; h->upin_tried = false;
@@ -378,6 +382,58 @@ int map_sources(const phast_ctx* h, const uint32_t* src, uint32_t k, uint32_t kp
     return PHAST_OK;
 }
 
+// Multi-level chunks: runs of adjacent chunks [from, ch.size()) (one direction of the
+// top plan, in processing order) whose items together fit one warp -- (vertices) x G
+// <= 32, no heavy vertex, arcs within the stage -- become one chunk of consecutive ids
+// with a round per item (top.cu): round(v) = 1 + the largest round of v's tails inside
+// the chunk, 0 if none.  `up`: the chunks run in ascending levels (descending ids;
+// tails have larger ids), else descending levels (tails have smaller ids).
+void merge_tiny(std::vector<uint4>& ch, size_t from, const uint32_t* f, const std::vector<Arc>& arc, uint32_t G,
+                bool big, bool up, std::vector<std::array<uint8_t, 32>>& rnd, bool enabled) {
+    if (!enabled) return;
+    const uint32_t ECH = top_chunk_arcs(big), VM = top_chunk_vertices(big), HB = 0x80000000u;
+    std::vector<uint4> out(ch.begin(), ch.begin() + from);
+    std::vector<std::array<uint8_t, 32>> rout(rnd.begin(), rnd.begin() + from);
+    size_t i = from;
+    auto lanes = [&](const uint4& c) { return (uint64_t)((c.y & 0x3FFFFFFFu) - c.x) * G; };
+    while (i < ch.size()) {
+        size_t j = i + 1;
+        uint32_t vb = ch[i].x, ve = ch[i].y & 0x3FFFFFFFu;
+        if (!(ch[i].y & HB) && lanes(ch[i]) <= 32) {
+            while (j < ch.size() && !(ch[j].y & HB)) {
+                const uint32_t jb = ch[j].x, je = ch[j].y & 0x3FFFFFFFu;
+                const bool adj = up ? je == vb : jb == ve;
+                const uint32_t nb = up ? jb : vb, ne = up ? ve : je;
+                if (!adj || (uint64_t)(ne - nb) * G > 32 || ne - nb > VM || f[ne] - f[nb] > ECH) break;
+                vb = nb;
+                ve = ne;
+                j++;
+            }
+        }
+        if (j == i + 1) {   // nothing to merge
+            out.push_back(ch[i]);
+            rout.push_back({});
+            i++;
+            continue;
+        }
+        std::array<uint8_t, 32> r{};
+        std::vector<uint32_t> rv(ve - vb, 0);
+        for (uint32_t s = 0; s < ve - vb; s++) {
+            const uint32_t v = up ? ve - 1 - s : vb + s;   // tails first
+            uint32_t m = 0;
+            for (uint32_t e = f[v]; e < f[v + 1]; e++)
+                if (arc[e].x >= vb && arc[e].x < ve) m = std::max(m, rv[arc[e].x - vb] + 1);
+            rv[v - vb] = std::min(m, 255u);
+        }
+        for (uint32_t x = 0; x < (ve - vb) * G; x++) r[x] = (uint8_t)rv[x / G];
+        out.push_back(make_uint4(vb, ve | top_multi_bit(), f[vb], f[ve]));
+        rout.push_back(r);
+        i = j;
+    }
+    ch.swap(out);
+    rnd.swap(rout);
+}
+
 // Chunks of one level [a, b) over a CSR (offsets `f`): <= VCH vertices and <= ECH
 // arcs each; chunks without arcs change nothing and are skipped.
 void push_chunks(std::vector<uint4>& ch, const uint32_t* f, uint32_t a, uint32_t b, bool big) {
@@ -449,7 +505,7 @@ phast_ctx::Top* get_top(phast_ctx* h, uint32_t k) {
     if (it != h->tops.end()) return it->second.chunks ? &it->second : nullptr;
     phast_ctx::Top& T = h->tops[k];   // chunks stays nullptr: "no plan"
     const Layout& L = h->L;
-    if (L.lvl_off.size() < 2 || h->n >= 0x80000000u) return nullptr;   // chunk vend carries a flag bit
+    if (L.lvl_off.size() < 2 || h->n >= 0x40000000u) return nullptr;   // chunk vend carries two flag bits
     const uint32_t nseg = (uint32_t)L.lvl_off.size() - 1;
     const uint32_t G = k >= 4 ? k / 4 : 1;
     const uint64_t vmax_budget = top_label_budget() / (4ull * k);
@@ -474,10 +530,19 @@ phast_ctx::Top* get_top(phast_ctx* h, uint32_t k) {
     } else {
         fused = false;
     }
+    std::vector<std::array<uint8_t, 32>> rnd;
     if (fused) {
+        std::vector<uint32_t> hf;
+        std::vector<Arc> ha;
+        upin_csr(L, h->n, top_chunk_arcs(true), hf, ha);
         for (uint32_t j = nseg; j-- > 0;) push_chunks(ch, uf.data(), L.lvl_off[j], L.lvl_off[j + 1], fbig);   // ascending
+        rnd.resize(ch.size());
+        merge_tiny(ch, 0, hf.data(), ha, G, fbig, true, rnd, !(h->q.flags & PHAST_Q_NO_MULTI));
         T.a.split = (uint32_t)ch.size();
+        const size_t d0 = ch.size();
         for (uint32_t j = 0; j < nseg; j++) push_chunks(ch, L.dn_first.data(), L.lvl_off[j], L.lvl_off[j + 1], fbig);
+        rnd.resize(ch.size());
+        merge_tiny(ch, d0, L.dn_first.data(), L.dn_arc, G, fbig, false, rnd, !(h->q.flags & PHAST_Q_NO_MULTI));
         T.a.big = fbig;
         T.a.first[0] = h->d_upin_first;
         T.a.arcs[0] = h->d_upin_arc;
@@ -521,27 +586,38 @@ phast_ctx::Top* get_top(phast_ctx* h, uint32_t k) {
             std::vector<Arc> arc;
             if (upin_csr(L, V, top_chunk_arcs(big), f, arc) && upload_csr(f, arc, &T.up_f, &T.up_a)) {
                 for (uint32_t j = J; j-- > 0;) push_chunks(ch, f.data(), L.lvl_off[j], L.lvl_off[j + 1], big);
+                rnd.resize(ch.size());
+                merge_tiny(ch, 0, f.data(), arc, G, big, true, rnd, !(h->q.flags & PHAST_Q_NO_MULTI));
                 T.a.first[0] = T.up_f;
                 T.a.arcs[0] = T.up_a;
                 T.vtop = V;
             }
         }
         T.a.split = (uint32_t)ch.size();
+        const size_t d0 = ch.size();
         for (uint32_t j = 0; j < J; j++) push_chunks(ch, L.dn_first.data(), L.lvl_off[j], L.lvl_off[j + 1], big);
+        rnd.resize(ch.size());
+        merge_tiny(ch, d0, L.dn_first.data(), L.dn_arc, G, big, false, rnd, !(h->q.flags & PHAST_Q_NO_MULTI));
         T.J = J;
         T.a.V = V;
     }
     const bool none = ch.empty();
     if (none) ch.push_back(make_uint4(0, 0, 0, 0));   // keep a valid device array
+    rnd.resize(ch.size());
     uint4* dch = nullptr;
-    if (dmalloc(&dch, ch.size()) ||
-        cudaMemcpy(dch, ch.data(), ch.size() * sizeof(uint4), cudaMemcpyHostToDevice) != cudaSuccess) {
+    uint4* drn = nullptr;
+    if (dmalloc(&dch, ch.size()) || dmalloc(&drn, 2 * ch.size()) ||
+        cudaMemcpy(dch, ch.data(), ch.size() * sizeof(uint4), cudaMemcpyHostToDevice) != cudaSuccess ||
+        cudaMemcpy(drn, rnd.data(), rnd.size() * 32, cudaMemcpyHostToDevice) != cudaSuccess) {
         cudaGetLastError();
         cudaFree(dch);
+        cudaFree(drn);
         return nullptr;
     }
     T.chunks = dch;
+    T.rnd = drn;
     T.a.chunks = dch;
+    T.a.rnd = drn;
     T.a.nchunks = none ? 0u : (uint32_t)ch.size();
     T.a.first[1] = h->g.dn_first;
     T.a.arcs[1] = h->g.dn_arc;
@@ -806,7 +882,7 @@ int phast_configure(phast_ctx* h, const phast_query_opts* q) {
     int rc = check_handle(h);
     if (rc) return rc;
     phast_query_opts nq = q ? *q : phast_query_opts{0, 0, 0, 0};
-    const uint32_t known = PHAST_Q_NO_FUSED | PHAST_Q_NO_TOP | PHAST_Q_HYBRID_ON | PHAST_Q_HYBRID_OFF;
+    const uint32_t known = PHAST_Q_NO_FUSED | PHAST_Q_NO_TOP | PHAST_Q_HYBRID_ON | PHAST_Q_HYBRID_OFF | PHAST_Q_NO_MULTI;
     if ((nq.flags & ~known) || ((nq.flags & PHAST_Q_HYBRID_ON) && (nq.flags & PHAST_Q_HYBRID_OFF)))
         return PHAST_EINVAL;
     DeviceGuard dg(h->device);
@@ -969,9 +1045,17 @@ int centrality(phast_ctx* h, const uint32_t* sources, uint64_t count, uint32_t k
     if (!dg.ok) return PHAST_ECUDA;
     cudaStream_t st = (cudaStream_t)stream;
     const uint32_t n = h->n, k = kpad(k_batch);   // a batch is k sources (k_batch rounded up)
-    const size_t elems = (size_t)n * k;
-    if (elems >= 0xFFFFFFFFull) return PHAST_ERANGE;   // items are 32-bit
+    const uint64_t nk = (uint64_t)n * k;
+    if (nk >= 0xFFFFFFFFull) return PHAST_ERANGE;   // items are 32-bit
     if ((rc = ensure_in_csr(h)) || (rc = ensure_out_csr(h))) return rc;
+    // B batches share each chain of Kahn passes: as many as 32 n k bytes each fit a
+    // quarter of the free memory (at most 64, B n k < 2^32)
+    size_t free_b = 0, total_b = 0;
+    if (cudaMemGetInfo(&free_b, &total_b) != cudaSuccess) { cudaGetLastError(); free_b = 1ull << 32; }
+    const uint64_t nbatches = (count + k - 1) / k;
+    uint64_t B = std::max<uint64_t>(1, (free_b / 4 + (uint64_t)h->bc_elems * 32) / (32 * nk));
+    B = std::min<uint64_t>({B, 64, nbatches, 0xFFFFFFFEull / nk});
+    const size_t elems = (size_t)(B * nk);
     constexpr uint32_t R = 30;   // passes per graph launch / host convergence check (multiple of 6)
     if (!h->bc_changed) {
         if ((rc = dmalloc(&h->bc_changed, R)) || (rc = dmalloc(&h->bc_qs, 3))) return rc;
@@ -981,12 +1065,13 @@ int centrality(phast_ctx* h, const uint32_t* sources, uint64_t count, uint32_t k
         }
     }
     if (h->bc_elems < elems) {
-        cudaFree(h->bc_sigma); cudaFree(h->bc_delta); cudaFree(h->bc_q); cudaFree(h->bc_dist);
+        cudaFree(h->bc_sigma); cudaFree(h->bc_delta); cudaFree(h->bc_q); cudaFree(h->bc_dist); cudaFree(h->bc_src);
         h->bc_sigma = h->bc_delta = nullptr;
-        h->bc_q = h->bc_dist = nullptr;
+        h->bc_q = h->bc_dist = h->bc_src = nullptr;
         h->bc_elems = 0;
         if ((rc = dmalloc(&h->bc_sigma, elems)) || (rc = dmalloc(&h->bc_delta, elems)) ||
-            (rc = dmalloc(&h->bc_q, 3 * elems)) || (rc = dmalloc(&h->bc_dist, elems)))
+            (rc = dmalloc(&h->bc_q, 3 * elems)) || (rc = dmalloc(&h->bc_dist, elems)) ||
+            (rc = dmalloc(&h->bc_src, (size_t)B * k)))
             return rc;
         h->bc_elems = elems;
     }
@@ -999,9 +1084,9 @@ int centrality(phast_ctx* h, const uint32_t* sources, uint64_t count, uint32_t k
     uint32_t* qbuf[2] = {h->bc_q, h->bc_q + elems};
     uint32_t* cnt = h->bc_q + 2 * elems;
     // R passes (+ clearing the change words before, reading them back after) are one CUDA
-    // graph, captured once per call and direction on a private stream (the caller's stream
-    // may be the legacy default stream, which cannot be captured); R is a multiple of 6,
-    // so every chunk starts with the same queue/counter rotation.
+    // graph, captured once per group size and direction on a private stream (the caller's
+    // stream may be the legacy default stream, which cannot be captured); R is a multiple
+    // of 6, so every chunk starts with the same queue/counter rotation.
     if ((!h->bc_ev && cudaEventCreateWithFlags(&h->bc_ev, cudaEventDisableTiming) != cudaSuccess) ||
         (!h->bc_stream && cudaStreamCreateWithFlags(&h->bc_stream, cudaStreamNonBlocking) != cudaSuccess)) {
         cudaGetLastError();
@@ -1016,7 +1101,13 @@ int centrality(phast_ctx* h, const uint32_t* sources, uint64_t count, uint32_t k
                 if (e[j]) cudaGraphExecDestroy(e[j]);
         }
     } eg{execs};
+    uint32_t total = 0;   // items of the current group (B' batches)
+    uint32_t graph_total = 0;
     auto kahn = [&](int which, int backward, auto pass) -> int {
+        if (execs[which] && graph_total != total) {   // a smaller last group: re-capture
+            cudaGraphExecDestroy(execs[which]);
+            execs[which] = nullptr;
+        }
         if (!execs[which]) {
             cudaGraph_t graph = nullptr;
             if (cudaStreamBeginCapture(gs, cudaStreamCaptureModeThreadLocal) != cudaSuccess) return PHAST_ECUDA;
@@ -1045,7 +1136,7 @@ int centrality(phast_ctx* h, const uint32_t* sources, uint64_t count, uint32_t k
         // the count kernel and the chunks run on gs after everything queued on st so far
         if (cudaEventRecord(h->bc_ev, st) != cudaSuccess || cudaStreamWaitEvent(gs, h->bc_ev, 0) != cudaSuccess ||
             cudaMemsetAsync(h->bc_qs, 0, 12, gs) != cudaSuccess ||
-            launch_bc_count(G, d, n, k, backward, cnt, qbuf[0], h->bc_qs, gs) != cudaSuccess)
+            launch_bc_count(G, d, (uint32_t)nk, k, total, backward, cnt, qbuf[0], h->bc_qs, gs) != cudaSuccess)
             return PHAST_ECUDA;
         for (uint64_t it = 0; it <= (uint64_t)n + R; it += R) {
             if (cudaGraphLaunch(execs[which], gs) != cudaSuccess || cudaStreamSynchronize(gs) != cudaSuccess)
@@ -1057,33 +1148,46 @@ int centrality(phast_ctx* h, const uint32_t* sources, uint64_t count, uint32_t k
         return PHAST_EINTERNAL;   // cannot happen with lengths > 0
     };
     uint32_t* hgt = reinterpret_cast<uint32_t*>(h->bc_delta);
-    for (uint64_t base = 0; base < count; base += k) {
-        const uint32_t kv = (uint32_t)std::min<uint64_t>(k, count - base);
-        Sources S;
-        if ((rc = map_sources(h, sources + base, kv, k, S))) return rc;
-        QueryOut o{d};
-        if ((rc = run_query(h, S, k, o, st))) return rc;
+    std::vector<uint32_t> gsrc((size_t)B * k);
+    for (uint64_t base = 0; base < count; base += B * k) {
+        // a group: B' batches of k trees, labels into [b][n][k]
+        const uint64_t left = count - base;
+        const uint32_t Bg = (uint32_t)std::min<uint64_t>(B, (left + k - 1) / k);
+        const uint32_t valid = (uint32_t)std::min<uint64_t>(left, (uint64_t)Bg * k);
+        total = (uint32_t)(Bg * nk);
+        for (uint32_t b = 0; b < Bg; b++) {
+            const uint32_t kv = (uint32_t)std::min<uint64_t>(k, valid - (uint64_t)b * k);
+            Sources S;
+            if ((rc = map_sources(h, sources + base + (uint64_t)b * k, kv, k, S))) return rc;
+            for (uint32_t i = 0; i < k; i++) gsrc[(size_t)b * k + i] = S.s[i];
+            QueryOut o{d + (size_t)b * nk};
+            if ((rc = run_query(h, S, k, o, st))) return rc;
+        }
+        if (cudaMemcpyAsync(h->bc_src, gsrc.data(), (size_t)Bg * k * 4, cudaMemcpyHostToDevice, st) != cudaSuccess)
+            return PHAST_ECUDA;
         if (reach) {
-            if (cudaMemsetAsync(hgt, 0, elems * 4, st) != cudaSuccess) return PHAST_ECUDA;
+            if (cudaMemsetAsync(hgt, 0, (size_t)total * 4, st) != cudaSuccess) return PHAST_ECUDA;
             rc = kahn(2, 1, [&](const BcQueue& Q, uint32_t* ch, cudaStream_t s2) {
-                return launch_bc_back(G, d, nullptr, hgt, n, k, 1, Q, ch, s2);
+                return launch_bc_back(G, d, nullptr, hgt, (uint32_t)nk, k, total, 1, Q, ch, s2);
             });
             if (rc) return rc;
-            if (launch_reach_accum(d, hgt, (uint32_t*)out, n, k, kv, st) != cudaSuccess) return PHAST_ECUDA;
+            graph_total = total;
+            if (launch_reach_accum(d, hgt, (uint32_t*)out, n, k, valid, st) != cudaSuccess) return PHAST_ECUDA;
             continue;
         }
-        if (cudaMemsetAsync(h->bc_sigma, 0, elems * 8, st) != cudaSuccess ||
-            cudaMemsetAsync(h->bc_delta, 0, elems * 8, st) != cudaSuccess)
+        if (cudaMemsetAsync(h->bc_sigma, 0, (size_t)total * 8, st) != cudaSuccess ||
+            cudaMemsetAsync(h->bc_delta, 0, (size_t)total * 8, st) != cudaSuccess)
             return PHAST_ECUDA;
         rc = kahn(0, 0, [&](const BcQueue& Q, uint32_t* ch, cudaStream_t s2) {
-            return launch_bc_sigma(G, d, h->bc_sigma, n, k, Q, ch, s2);
+            return launch_bc_sigma(G, d, h->bc_sigma, (uint32_t)nk, k, total, Q, ch, s2);
         });
         if (rc) return rc;
         rc = kahn(1, 1, [&](const BcQueue& Q, uint32_t* ch, cudaStream_t s2) {
-            return launch_bc_back(G, d, h->bc_sigma, h->bc_delta, n, k, 0, Q, ch, s2);
+            return launch_bc_back(G, d, h->bc_sigma, h->bc_delta, (uint32_t)nk, k, total, 0, Q, ch, s2);
         });
         if (rc) return rc;
-        if (launch_bc_accum(h->bc_delta, (double*)out, n, k, kv, S, st) != cudaSuccess) return PHAST_ECUDA;
+        graph_total = total;
+        if (launch_bc_accum(h->bc_delta, (double*)out, n, k, valid, h->bc_src, st) != cudaSuccess) return PHAST_ECUDA;
     }
     return phast_sync(h, stream);
 }

@@ -86,6 +86,10 @@ struct TopArgs {
     const uint4* chunks = nullptr;
     uint32_t split = 0, nchunks = 0, V = 0, stages = 0, fused = 0;
     uint32_t big = 0;                    // chunk geometry: 0 = top_chunk_*(false), 1 = top_chunk_*(true)
+    // multi-level chunks (vend bit 30, top_multi_bit()): several tiny consecutive levels
+    // whose (vertex, lane) items fit one warp; rnd[2c..2c+1] = 32 bytes, byte i = the
+    // round (level inside the chunk, 0 first) of the chunk's i-th item's vertex
+    const uint4* rnd = nullptr;
 };
 cudaError_t launch_sweep_top(const TopArgs& A, uint32_t k, const Sources& src, uint32_t* dist,
                              const uint32_t* flags, uint32_t* diam, cudaStream_t st);
@@ -94,6 +98,7 @@ uint32_t top_chunk_vertices(bool big);
 uint32_t top_chunk_arcs(bool big);
 bool top_big_fits(uint32_t k, uint32_t V);   // the big geometry leaves room for the rows
 uint32_t top_heavy_arcs();   // chunk flag (bit 31 of vend): some vertex has more in-arcs than this
+uint32_t top_multi_bit();    // chunk flag (bit 30 of vend): a multi-level chunk (TopArgs::rnd)
 
 // a5: max of `count` per-batch maxima into *out
 cudaError_t launch_max_reduce(const uint32_t* in, uint32_t count, uint32_t* out, cudaStream_t st);
@@ -135,16 +140,18 @@ struct BcQueue {
     uint32_t* qs_clr;           // counter zeroed for the pass after next
     uint32_t* cnt;              // [n*k] unfinished inputs per item
 };
-cudaError_t launch_bc_count(const BcGraph& G, const uint32_t* d, uint32_t n, uint32_t k, int backward, uint32_t* cnt,
-                            uint32_t* q, uint32_t* qs, cudaStream_t st);
-cudaError_t launch_bc_sigma(const BcGraph& G, const uint32_t* d, double* sigma, uint32_t n, uint32_t k,
-                            const BcQueue& Q, uint32_t* changed, cudaStream_t st);
-cudaError_t launch_bc_back(const BcGraph& G, const uint32_t* d, const double* sigma, void* val, uint32_t n, uint32_t k,
-                           int mode, const BcQueue& Q, uint32_t* changed, cudaStream_t st);
-cudaError_t launch_reach_accum(const uint32_t* d, const uint32_t* hgt, uint32_t* r, uint32_t n, uint32_t k, uint32_t kv,
-                               cudaStream_t st);
-cudaError_t launch_bc_accum(const double* delta, double* cb, uint32_t n, uint32_t k, uint32_t kv, const Sources& src,
-                            cudaStream_t st);
+// B batches of k trees at once: arrays [B][n][k], nk = n*k, total = B*nk items (< 2^32)
+cudaError_t launch_bc_count(const BcGraph& G, const uint32_t* d, uint32_t nk, uint32_t k, uint32_t total, int backward,
+                            uint32_t* cnt, uint32_t* q, uint32_t* qs, cudaStream_t st);
+cudaError_t launch_bc_sigma(const BcGraph& G, const uint32_t* d, double* sigma, uint32_t nk, uint32_t k,
+                            uint32_t total, const BcQueue& Q, uint32_t* changed, cudaStream_t st);
+cudaError_t launch_bc_back(const BcGraph& G, const uint32_t* d, const double* sigma, void* val, uint32_t nk,
+                           uint32_t k, uint32_t total, int mode, const BcQueue& Q, uint32_t* changed, cudaStream_t st);
+// accumulation over trees j = b*k + i < valid; src: DEVICE internal ids of the trees
+cudaError_t launch_reach_accum(const uint32_t* d, const uint32_t* hgt, uint32_t* r, uint32_t n, uint32_t k,
+                               uint32_t valid, cudaStream_t st);
+cudaError_t launch_bc_accum(const double* delta, double* cb, uint32_t n, uint32_t k, uint32_t valid,
+                            const uint32_t* src, cudaStream_t st);
 
 uint64_t launches();
 // kernels replayed from a CUDA graph (counted at launch, not at capture)

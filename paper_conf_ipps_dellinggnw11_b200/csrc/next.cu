@@ -136,26 +136,35 @@ __device__ __forceinline__ bool tight(uint32_t du, uint32_t dv, uint32_t l) {
     return du <= dv && dv - du == l;   // du + l == dv without 32-bit overflow
 }
 // Schedule (not part of the method): Kahn's topological order of each tree's tight DAG.
-// An item t = v*k + i is computed ONCE, when all its inputs are final: cnt[t] counts the
-// item's unfinished inputs (forward: tight in-arcs; backward: tight out-arcs); a pass
-// computes the items of its queue and, for each dependent whose count drops to zero,
-// appends it to the next queue.  Passes = hop depth of the tight DAG + 1; each pass
-// touches only its frontier.  Queue sizes rotate over three counters: pass p reads
-// qs[p%3], appends with qs[(p+1)%3] and zeroes qs[(p+2)%3].
+// Items t = b*nk + v*k + i cover B batches of k trees at once (arrays [B][n][k]): an item
+// is computed ONCE, when all its inputs are final: cnt[t] counts the item's unfinished
+// inputs (forward: tight in-arcs; backward: tight out-arcs); a pass computes the items
+// of its queue and, for each dependent whose count drops to zero, appends it to the
+// next queue.  Passes = the largest hop depth of the trees' tight DAGs + 1, so B
+// batches share one chain of passes.  Queue sizes rotate over three counters: pass p
+// reads qs[p%3], appends with qs[(p+1)%3] and zeroes qs[(p+2)%3].
+// warp-aggregated append: the lanes pushing together take consecutive slots with ONE
+// atomic (a pass readies up to hundreds of thousands of items: one same-address atomic
+// each would serialise the pass)
 __device__ __forceinline__ void bc_push(uint32_t t, uint32_t* q, uint32_t* qs, bool& pushed) {
-    q[atomicAdd(qs, 1u)] = t;
+    const unsigned m = __activemask();
+    const uint32_t lane = threadIdx.x & 31, leader = __ffs(m) - 1;
+    uint32_t base = 0;
+    if (lane == leader) base = atomicAdd(qs, (uint32_t)__popc(m));
+    base = __shfl_sync(m, base, leader);
+    q[base + __popc(m & ((1u << lane) - 1u))] = t;
     pushed = true;
 }
+// the item of vertex u in item t's tree
+__device__ __forceinline__ uint32_t same_tree(uint32_t t, uint32_t v, uint32_t u, uint32_t k) { return t - v * k + u * k; }
 
 // cnt[t] = number of inputs of item t; items with none start the first queue
-__global__ void __launch_bounds__(256) bc_count_kernel(BcGraph G, const uint32_t* __restrict__ d, uint32_t n,
-                                                       uint32_t k, int backward, uint32_t* cnt, uint32_t* q,
-                                                       uint32_t* qs) {
-    const uint64_t total = (uint64_t)n * k;
+__global__ void __launch_bounds__(256) bc_count_kernel(BcGraph G, const uint32_t* __restrict__ d, uint32_t nk,
+                                                       uint32_t k, uint32_t total, int backward, uint32_t* cnt,
+                                                       uint32_t* q, uint32_t* qs) {
     bool pushed = false;
-    for (uint64_t t = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; t < total;
-         t += (uint64_t)gridDim.x * blockDim.x) {
-        const uint32_t v = (uint32_t)(t / k), i = (uint32_t)(t % k);
+    for (uint32_t t = blockIdx.x * blockDim.x + threadIdx.x; t < total; t += gridDim.x * blockDim.x) {
+        const uint32_t v = (t % nk) / k;
         const uint32_t dv = __ldg(&d[t]);
         if (dv == INF) continue;
         uint32_t c = 0;
@@ -163,18 +172,18 @@ __global__ void __launch_bounds__(256) bc_count_kernel(BcGraph G, const uint32_t
             const uint32_t e1 = __ldg(&G.in_first[v + 1]);
             for (uint32_t e = __ldg(&G.in_first[v]); e < e1; e++) {
                 const uint2 a = __ldg(&G.in_arc[e]);
-                c += tight(__ldg(&d[(size_t)a.x * k + i]), dv, a.y);
+                c += tight(__ldg(&d[same_tree(t, v, a.x, k)]), dv, a.y);
             }
         } else {
             const uint32_t e1 = __ldg(&G.out_first[v + 1]);
             for (uint32_t e = __ldg(&G.out_first[v]); e < e1; e++) {
                 const uint2 a = __ldg(&G.out_arc[e]);
-                const uint32_t dw = __ldg(&d[(size_t)a.x * k + i]);
+                const uint32_t dw = __ldg(&d[same_tree(t, v, a.x, k)]);
                 c += dw != INF && tight(dv, dw, a.y);
             }
         }
         cnt[t] = c;
-        if (c == 0) bc_push((uint32_t)t, q, qs, pushed);
+        if (c == 0) bc_push(t, q, qs, pushed);
     }
     (void)pushed;
 }
@@ -183,20 +192,20 @@ __global__ void __launch_bounds__(256) bc_count_kernel(BcGraph G, const uint32_t
 // the source is the only finite item without a tight in-arc, so [v = s] is "no tight
 // in-arc" (no source list in the parameters: the passes are graph-captured once per call)
 __global__ void __launch_bounds__(256) bc_sigma_kernel(BcGraph G, const uint32_t* __restrict__ d, double* sigma,
-                                                       uint32_t k, BcQueue Q, uint32_t* changed) {
+                                                       uint32_t nk, uint32_t k, BcQueue Q, uint32_t* changed) {
     const uint32_t size = *Q.qs_in;
     if (blockIdx.x == 0 && threadIdx.x == 0) *Q.qs_clr = 0;
     bool pushed = false;
     for (uint32_t x = blockIdx.x * blockDim.x + threadIdx.x; x < size; x += gridDim.x * blockDim.x) {
         const uint32_t t = Q.q_in[x];
-        const uint32_t v = t / k, i = t % k;
+        const uint32_t v = (t % nk) / k;
         const uint32_t dv = __ldg(&d[t]);
         double acc = 0.0;
         bool any = false;
         const uint32_t e1 = __ldg(&G.in_first[v + 1]);
         for (uint32_t e = __ldg(&G.in_first[v]); e < e1; e++) {
             const uint2 a = __ldg(&G.in_arc[e]);
-            const size_t u = (size_t)a.x * k + i;
+            const uint32_t u = same_tree(t, v, a.x, k);
             if (tight(__ldg(&d[u]), dv, a.y)) {
                 acc += sigma[u];
                 any = true;
@@ -207,7 +216,7 @@ __global__ void __launch_bounds__(256) bc_sigma_kernel(BcGraph G, const uint32_t
         const uint32_t f1 = __ldg(&G.out_first[v + 1]);
         for (uint32_t e = __ldg(&G.out_first[v]); e < f1; e++) {
             const uint2 a = __ldg(&G.out_arc[e]);
-            const uint32_t w = a.x * k + i;
+            const uint32_t w = same_tree(t, v, a.x, k);
             const uint32_t dw = __ldg(&d[w]);
             if (dw != INF && tight(dv, dw, a.y) && atomicSub(&Q.cnt[w], 1u) == 1u) bc_push(w, Q.q_out, Q.qs_out, pushed);
         }
@@ -219,8 +228,8 @@ __global__ void __launch_bounds__(256) bc_sigma_kernel(BcGraph G, const uint32_t
 // mode 1 (reach): height h(v) = max over tight (v, w) of l + h(w), stored as uint32 in
 // `val` (l + h(w) <= d(w) + h(w) - d(v) is at most the largest finite label: no wrap)
 __global__ void __launch_bounds__(256) bc_back_kernel(BcGraph G, const uint32_t* __restrict__ d,
-                                                      const double* __restrict__ sigma, void* val, uint32_t k,
-                                                      int mode, BcQueue Q, uint32_t* changed) {
+                                                      const double* __restrict__ sigma, void* val, uint32_t nk,
+                                                      uint32_t k, int mode, BcQueue Q, uint32_t* changed) {
     const uint32_t size = *Q.qs_in;
     if (blockIdx.x == 0 && threadIdx.x == 0) *Q.qs_clr = 0;
     bool pushed = false;
@@ -228,7 +237,7 @@ __global__ void __launch_bounds__(256) bc_back_kernel(BcGraph G, const uint32_t*
     uint32_t* hgt = static_cast<uint32_t*>(val);
     for (uint32_t x = blockIdx.x * blockDim.x + threadIdx.x; x < size; x += gridDim.x * blockDim.x) {
         const uint32_t t = Q.q_in[x];
-        const uint32_t v = t / k, i = t % k;
+        const uint32_t v = (t % nk) / k;
         const uint32_t dv = __ldg(&d[t]);
         const uint32_t e1 = __ldg(&G.out_first[v + 1]);
         if (mode == 0) {
@@ -236,7 +245,7 @@ __global__ void __launch_bounds__(256) bc_back_kernel(BcGraph G, const uint32_t*
             double acc = 0.0;
             for (uint32_t e = __ldg(&G.out_first[v]); e < e1; e++) {
                 const uint2 a = __ldg(&G.out_arc[e]);
-                const size_t w = (size_t)a.x * k + i;
+                const uint32_t w = same_tree(t, v, a.x, k);
                 const uint32_t dw = __ldg(&d[w]);
                 if (dw != INF && tight(dv, dw, a.y)) acc += sv / __ldg(&sigma[w]) * (1.0 + delta[w]);
             }
@@ -245,7 +254,7 @@ __global__ void __launch_bounds__(256) bc_back_kernel(BcGraph G, const uint32_t*
             uint32_t acc = 0;
             for (uint32_t e = __ldg(&G.out_first[v]); e < e1; e++) {
                 const uint2 a = __ldg(&G.out_arc[e]);
-                const size_t w = (size_t)a.x * k + i;
+                const uint32_t w = same_tree(t, v, a.x, k);
                 const uint32_t dw = __ldg(&d[w]);
                 if (dw != INF && tight(dv, dw, a.y)) acc = max(acc, a.y + hgt[w]);
             }
@@ -254,34 +263,38 @@ __global__ void __launch_bounds__(256) bc_back_kernel(BcGraph G, const uint32_t*
         const uint32_t f1 = __ldg(&G.in_first[v + 1]);
         for (uint32_t e = __ldg(&G.in_first[v]); e < f1; e++) {
             const uint2 a = __ldg(&G.in_arc[e]);
-            const uint32_t u = a.x * k + i;
+            const uint32_t u = same_tree(t, v, a.x, k);
             if (tight(__ldg(&d[u]), dv, a.y) && atomicSub(&Q.cnt[u], 1u) == 1u) bc_push(u, Q.q_out, Q.qs_out, pushed);
         }
     }
     if (__syncthreads_or(pushed) && threadIdx.x == 0) *changed = 1;
 }
 
-
-// c_B(v) += sum over the first kv trees i (in order) with sources[i] != v of delta_i(v)
+// c_B(v) += sum over trees j < valid (j = b*k + i: tree i of batch b) with src[j] != v of
+// delta_j(v), in tree order
 __global__ void __launch_bounds__(256) bc_accum_kernel(const double* __restrict__ delta, double* __restrict__ cb,
-                                                       uint32_t n, uint32_t k, uint32_t kv, Sources src) {
+                                                       uint32_t n, uint32_t k, uint32_t valid,
+                                                       const uint32_t* __restrict__ src) {
+    const uint32_t nk = n * k;
     for (uint32_t v = blockIdx.x * blockDim.x + threadIdx.x; v < n; v += gridDim.x * blockDim.x) {
         double s = 0.0;
-        for (uint32_t i = 0; i < kv; i++)
-            if (src.s[i] != v) s += __ldg(&delta[(size_t)v * k + i]);
+        for (uint32_t j = 0; j < valid; j++)
+            if (__ldg(&src[j]) != v) s += __ldg(&delta[(size_t)(j / k) * nk + (size_t)v * k + j % k]);
         cb[v] += s;
     }
 }
 
-// r(v) = max(r(v), max over the first kv trees of min(d_i(v), h_i(v)))
+// r(v) = max(r(v), max over trees j < valid of min(d_j(v), h_j(v)))
 __global__ void __launch_bounds__(256) reach_accum_kernel(const uint32_t* __restrict__ d,
                                                           const uint32_t* __restrict__ hgt, uint32_t* __restrict__ r,
-                                                          uint32_t n, uint32_t k, uint32_t kv) {
+                                                          uint32_t n, uint32_t k, uint32_t valid) {
+    const uint32_t nk = n * k;
     for (uint32_t v = blockIdx.x * blockDim.x + threadIdx.x; v < n; v += gridDim.x * blockDim.x) {
         uint32_t m = r[v];
-        for (uint32_t i = 0; i < kv; i++) {
-            const uint32_t dv = __ldg(&d[(size_t)v * k + i]);
-            if (dv != INF) m = max(m, min(dv, __ldg(&hgt[(size_t)v * k + i])));
+        for (uint32_t j = 0; j < valid; j++) {
+            const size_t t = (size_t)(j / k) * nk + (size_t)v * k + j % k;
+            const uint32_t dv = __ldg(&d[t]);
+            if (dv != INF) m = max(m, min(dv, __ldg(&hgt[t])));
         }
         r[v] = m;
     }
@@ -292,42 +305,42 @@ unsigned bc_blocks(uint64_t items) {
     return (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(b, (uint64_t)num_sms() * 8));
 }
 
-// the passes touch only their queue: a small fixed grid (queue sizes are read on the device)
-unsigned bc_pass_blocks(uint64_t items) { return std::min<unsigned>(bc_blocks(items), (unsigned)num_sms() * 2); }
+// the passes touch only their queue (its size is read on the device): a full wave
+unsigned bc_pass_blocks(uint64_t items) { return bc_blocks(items); }
 
 }  // namespace
 
-cudaError_t launch_bc_count(const BcGraph& G, const uint32_t* d, uint32_t n, uint32_t k, int backward, uint32_t* cnt,
-                            uint32_t* q, uint32_t* qs, cudaStream_t st) {
-    bc_count_kernel<<<bc_blocks((uint64_t)n * k), 256, 0, st>>>(G, d, n, k, backward, cnt, q, qs);
+cudaError_t launch_bc_count(const BcGraph& G, const uint32_t* d, uint32_t nk, uint32_t k, uint32_t total, int backward,
+                            uint32_t* cnt, uint32_t* q, uint32_t* qs, cudaStream_t st) {
+    bc_count_kernel<<<bc_blocks(total), 256, 0, st>>>(G, d, nk, k, total, backward, cnt, q, qs);
     count_launch();
     return cudaGetLastError();
 }
 
-cudaError_t launch_bc_sigma(const BcGraph& G, const uint32_t* d, double* sigma, uint32_t n, uint32_t k,
-                            const BcQueue& Q, uint32_t* changed, cudaStream_t st) {
-    bc_sigma_kernel<<<bc_pass_blocks((uint64_t)n * k), 256, 0, st>>>(G, d, sigma, k, Q, changed);
+cudaError_t launch_bc_sigma(const BcGraph& G, const uint32_t* d, double* sigma, uint32_t nk, uint32_t k,
+                            uint32_t total, const BcQueue& Q, uint32_t* changed, cudaStream_t st) {
+    bc_sigma_kernel<<<bc_pass_blocks(total), 256, 0, st>>>(G, d, sigma, nk, k, Q, changed);
     count_launch();
     return cudaGetLastError();
 }
 
-cudaError_t launch_bc_back(const BcGraph& G, const uint32_t* d, const double* sigma, void* val, uint32_t n, uint32_t k,
-                           int mode, const BcQueue& Q, uint32_t* changed, cudaStream_t st) {
-    bc_back_kernel<<<bc_pass_blocks((uint64_t)n * k), 256, 0, st>>>(G, d, sigma, val, k, mode, Q, changed);
+cudaError_t launch_bc_back(const BcGraph& G, const uint32_t* d, const double* sigma, void* val, uint32_t nk,
+                           uint32_t k, uint32_t total, int mode, const BcQueue& Q, uint32_t* changed, cudaStream_t st) {
+    bc_back_kernel<<<bc_pass_blocks(total), 256, 0, st>>>(G, d, sigma, val, nk, k, mode, Q, changed);
     count_launch();
     return cudaGetLastError();
 }
 
-cudaError_t launch_reach_accum(const uint32_t* d, const uint32_t* hgt, uint32_t* r, uint32_t n, uint32_t k, uint32_t kv,
-                               cudaStream_t st) {
-    reach_accum_kernel<<<bc_blocks(n), 256, 0, st>>>(d, hgt, r, n, k, kv);
+cudaError_t launch_reach_accum(const uint32_t* d, const uint32_t* hgt, uint32_t* r, uint32_t n, uint32_t k,
+                               uint32_t valid, cudaStream_t st) {
+    reach_accum_kernel<<<bc_blocks(n), 256, 0, st>>>(d, hgt, r, n, k, valid);
     count_launch();
     return cudaGetLastError();
 }
 
-cudaError_t launch_bc_accum(const double* delta, double* cb, uint32_t n, uint32_t k, uint32_t kv, const Sources& src,
-                            cudaStream_t st) {
-    bc_accum_kernel<<<bc_blocks(n), 256, 0, st>>>(delta, cb, n, k, kv, src);
+cudaError_t launch_bc_accum(const double* delta, double* cb, uint32_t n, uint32_t k, uint32_t valid,
+                            const uint32_t* src, cudaStream_t st) {
+    bc_accum_kernel<<<bc_blocks(n), 256, 0, st>>>(delta, cb, n, k, valid, src);
     count_launch();
     return cudaGetLastError();
 }

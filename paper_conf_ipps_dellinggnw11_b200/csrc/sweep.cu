@@ -84,7 +84,7 @@ struct UpTable {
 };
 
 struct UpShared {
-    uint32_t qn, nn, used, over, cnt;
+    uint32_t qn, nn, used, over, over_next, cnt;   // over_next: set during a wave, published between waves
 };
 
 // Returns the slot of w (inserting it), or EMPTY when the table is 3/4 full.
@@ -118,7 +118,7 @@ __device__ bool up_search(const uint32_t* __restrict__ up_first, const uint2* __
     if (tid == 0) {
         const uint32_t h = hash32(s) & (t.cap - 1);
         t.keys[h] = s; t.vals[h] = 0; t.inq[h] = 1; t.qa[0] = h;
-        c.qn = s >= vtop ? 1u : 0u; c.nn = 0; c.used = 1; c.over = 0; c.cnt = 0;
+        c.qn = s >= vtop ? 1u : 0u; c.nn = 0; c.used = 1; c.over = 0; c.over_next = 0; c.cnt = 0;
     }
     __syncthreads();
     uint32_t* qa = t.qa;
@@ -138,7 +138,7 @@ __device__ bool up_search(const uint32_t* __restrict__ up_first, const uint2* __
                 const uint32_t nd = sat_add(dv, a.y);
                 if (nd == INF) continue;
                 const uint32_t ws = up_insert(t, a.x, c);
-                if (ws == EMPTY) { c.over = 1; break; }
+                if (ws == EMPTY) { c.over_next = 1; break; }
                 const uint32_t old = atomicMin(&t.vals[ws], nd);
                 if (nd < old && a.x >= vtop) {
                     __threadfence_block();
@@ -147,7 +147,7 @@ __device__ bool up_search(const uint32_t* __restrict__ up_first, const uint2* __
             }
         }
         __syncthreads();
-        if (tid == 0) { c.qn = c.nn; c.nn = 0; }
+        if (tid == 0) { c.qn = c.nn; c.nn = 0; c.over = c.over_next; }   // every thread reads these after the barrier
         uint32_t* tmp = qa; qa = qb; qb = tmp;
         __syncthreads();
     }

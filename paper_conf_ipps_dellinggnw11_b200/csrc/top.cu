@@ -35,7 +35,8 @@
 namespace phast {
 namespace {
 
-constexpr int TOP_THREADS = 1024, TOP_CONS = TOP_THREADS - 32;
+constexpr int TOP_PROD = 4;   // producer warps: one warp's cp.async stream alone starved the consumers (ncu, C1)
+constexpr int TOP_THREADS = 1024, TOP_CONS = TOP_THREADS - 32 * TOP_PROD;
 // chunk geometry (per plan, TopArgs::big): small 256 vertices / 1 024 arcs (9 280-byte
 // stages), big 1 024 / 4 096 (36 928-byte stages) when the rows leave room for 4 big
 // stages: fewer, larger chunks = fewer barriers on the long levels of small-k queries
@@ -51,7 +52,8 @@ constexpr size_t TOP_STATIC = 2 * 2 * 1024 + 64;
 constexpr size_t TOP_SMEM_MAX = 227 * 1024 - TOP_STATIC;
 
 constexpr uint32_t TOP_HEAVY = 8;              // in-arcs above which a warp relaxes the vertex (k <= 4)
-constexpr uint32_t TOP_VMASK = 0x7FFFFFFFu;    // chunk vend; bit 31: the chunk has a vertex with > TOP_HEAVY in-arcs
+constexpr uint32_t TOP_VMASK = 0x3FFFFFFFu;    // chunk vend; bit 31: the chunk has a vertex with > TOP_HEAVY
+constexpr uint32_t TOP_MULTI = 0x40000000u;    // in-arcs; bit 30: a multi-level chunk (one warp, rounds)
 
 template <int K, bool DIAM>
 __global__ void __launch_bounds__(TOP_THREADS, 1) sweep_top_kernel(TopArgs A, Sources src, uint32_t* __restrict__ d,
@@ -71,7 +73,7 @@ __global__ void __launch_bounds__(TOP_THREADS, 1) sweep_top_kernel(TopArgs A, So
     const uint32_t tid = threadIdx.x;
     if (tid == 0) {
         for (uint32_t s = 0; s < S; s++) {
-            mbar_init(&full[s], 32);   // one cp.async arrival per producer lane
+            mbar_init(&full[s], 32 * TOP_PROD);   // one cp.async arrival per producer lane
             mbar_init(&empty[s], 1);
         }
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
@@ -86,10 +88,10 @@ __global__ void __launch_bounds__(TOP_THREADS, 1) sweep_top_kernel(TopArgs A, So
     }
     __syncthreads();
     uint32_t mx = 0;
-    if (tid < 32) {   // producer warp: all 32 lanes copy (cp.async, 16 B each), then arrive
+    if (tid < 32 * TOP_PROD) {   // producer warps: all their lanes copy (cp.async, 16 B each), then arrive
         // descriptors: each lane holds one of the current 32 and one of the next 32
         // (loaded a batch ahead), so the issue loop never waits on a global load
-        const uint32_t lane = tid;
+        const uint32_t lane = tid & 31, ptid = tid;
         uint4 cur = make_uint4(0, 0, 0, 0), nxt = make_uint4(0, 0, 0, 0);
         if (lane < A.nchunks) cur = __ldg(&A.chunks[lane]);
         if (32 + lane < A.nchunks) nxt = __ldg(&A.chunks[32 + lane]);
@@ -111,16 +113,18 @@ __global__ void __launch_bounds__(TOP_THREADS, 1) sweep_top_kernel(TopArgs A, So
             unsigned char* st = ring + (size_t)s * SB;
             const uint4* gf = reinterpret_cast<const uint4*>((up ? A.first[0] : A.first[1]) + f0);
             const uint4* ga = reinterpret_cast<const uint4*>((up ? A.arcs[0] : A.arcs[1]) + a0);
-            for (uint32_t u = lane; u < 1 + nf4 + na2; u += 32) {
+            const uint32_t nr = (ch.y & TOP_MULTI) ? 2u : 0u;   // + the rounds of a multi-level chunk
+            for (uint32_t u = ptid; u < 1 + nf4 + na2 + nr; u += 32 * TOP_PROD) {
                 if (u == 0) cp_async16(st, A.chunks + c);   // the consumers read the descriptor here
                 else if (u <= nf4) cp_async16(st + 16 * u, gf + (u - 1));
-                else cp_async16(st + 16 + OFFB * 4 + 16 * (u - 1 - nf4), ga + (u - 1 - nf4));
+                else if (u <= nf4 + na2) cp_async16(st + 16 + OFFB * 4 + 16 * (u - 1 - nf4), ga + (u - 1 - nf4));
+                else cp_async16(st + 16 + OFFB * 4 - 32 + 16 * (u - 1 - nf4 - na2), A.rnd + 2 * c + (u - 1 - nf4 - na2));
             }
             asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];" ::"r"(smem_u32(&full[s])) : "memory");
             if (++s == S) { s = 0; ph ^= 1u; }
         }
     } else {
-        const uint32_t ct = tid - 32;
+        const uint32_t ct = tid - 32 * TOP_PROD;
         __shared__ uint32_t hcnt[2];            // heavy vertices of the chunk (double-buffered)
         __shared__ uint16_t hlist[2][TOP_VCH_BIG];   // as offsets from the chunk's first vertex
         static_assert(sizeof(hcnt) + sizeof(hlist) <= TOP_STATIC, "static shared memory");
@@ -138,8 +142,30 @@ __global__ void __launch_bounds__(TOP_THREADS, 1) sweep_top_kernel(TopArgs A, So
             const uint32_t* sf = reinterpret_cast<const uint32_t*>(st + 16);
             const uint2* sa = reinterpret_cast<const uint2*>(st + 16 + OFFB * 4);
             const uint32_t vend = ch.y & TOP_VMASK;
-            const bool heavy = G == 1 && (ch.y & ~TOP_VMASK);   // host: some vertex has > TOP_HEAVY in-arcs
+            const bool heavy = G == 1 && (ch.y & 0x80000000u);   // host: some vertex has > TOP_HEAVY in-arcs
             const uint32_t total = (vend - ch.x) * G;
+            if (ch.y & TOP_MULTI) {
+                // several tiny levels, one warp: item i (vertex ch.x + i / G) runs in round
+                // rnd[i] (its level inside the chunk; every tail inside the chunk has a
+                // smaller round), with only a warp barrier between rounds
+                if (ct < 32) {
+                    const unsigned char* rb = st + 16 + OFFB * 4 - 32;
+                    const uint32_t r = ct < total ? rb[ct] : 0u;
+                    const uint32_t maxr = __reduce_max_sync(0xFFFFFFFFu, r);
+                    const uint32_t v = ch.x + ct / G, lane = ct % G;
+                    for (uint32_t q = 0; q <= maxr; q++) {
+                        if (ct < total && r == q) {
+                            T acc = srow[v * G + lane];
+                            for (uint32_t e = sf[v - f0], e1 = sf[v + 1 - f0]; e < e1; e++) {
+                                const uint2 a = sa[e - a0];
+                                acc = relax(acc, srow[a.x * G + lane], a.y);
+                            }
+                            srow[v * G + lane] = acc;
+                        }
+                        __syncwarp();
+                    }
+                }
+            } else
             for (uint32_t t = ct; t < total; t += TOP_CONS) {
                 const uint32_t v = ch.x + t / G, lane = t % G;
                 const uint32_t e0 = sf[v - f0], e1 = sf[v + 1 - f0];
@@ -157,7 +183,7 @@ __global__ void __launch_bounds__(TOP_THREADS, 1) sweep_top_kernel(TopArgs A, So
 #pragma unroll
                     for (int r = 0; r < 4; r++) a[r] = e + r < e1 ? sa[e + r - a0] : make_uint2(0u, INF);
 #pragma unroll
-                    for (int r = 0; r < 4; r++) x[r] = srow[a[r].x * G + lane];   // row 0 for padding (len INF)
+                    for (int r = 0; r < 4; r++) x[r] = e + r < e1 ? srow[a[r].x * G + lane] : inf_row<T>();   // no pad read
 #pragma unroll
                     for (int r = 0; r < 4; r++) acc = relax(acc, x[r], a[r].y);
                 }
@@ -180,7 +206,7 @@ __global__ void __launch_bounds__(TOP_THREADS, 1) sweep_top_kernel(TopArgs A, So
 #pragma unroll
                         for (int r = 0; r < 4; r++) a[r] = e + 32 * r < e1 ? sa[e + 32 * r - a0] : make_uint2(0u, INF);
 #pragma unroll
-                        for (int r = 0; r < 4; r++) x[r] = srow[a[r].x];
+                        for (int r = 0; r < 4; r++) x[r] = e + 32 * r < e1 ? srow[a[r].x] : inf_row<T>();
 #pragma unroll
                         for (int r = 0; r < 4; r++) acc = relax(acc, x[r], a[r].y);
                     }
@@ -233,6 +259,7 @@ bool top_big_fits(uint32_t k, uint32_t V) {   // rows + 4 big stages within shar
     return lab + 4 * (top_stage_bytes(true) + 16) <= TOP_SMEM_MAX;
 }
 uint32_t top_heavy_arcs() { return TOP_HEAVY; }
+uint32_t top_multi_bit() { return TOP_MULTI; }
 
 cudaError_t launch_sweep_top(const TopArgs& A, uint32_t k, const Sources& src, uint32_t* dist,
                              const uint32_t* flags, uint32_t* diam, cudaStream_t st) {
