@@ -5,7 +5,7 @@ path tree computations ... replacing Dijkstra's algorithm by PHAST makes exact
 betweenness tractable"), sources sharded over the ranks, one NCCL SUM all-reduce of
 the per-GPU partial sums.
 
-  python bench_betweenness.py [--config C2] [--count 1024] [--k 64]
+  python bench_betweenness.py [--config C2] [--count 2048] [--k 64]
   torchrun --nproc-per-node N --master-addr 127.0.0.1 bench_betweenness.py
 
 Prints one JSON line on rank 0: sources/s (device time, max over ranks) and a
@@ -32,7 +32,7 @@ def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--config", default="C2")
     ap.add_argument("--k", type=int, default=64)
-    ap.add_argument("--count", type=int, default=1024, help="sources (over all ranks)")
+    ap.add_argument("--count", type=int, default=2048, help="sources (over all ranks)")
     ap.add_argument("--reach", action="store_true", help="exact reach instead of betweenness")
     ap.add_argument("--check", type=int, default=2, help="sources cross-checked against the oracle (0 = none)")
     args = ap.parse_args()

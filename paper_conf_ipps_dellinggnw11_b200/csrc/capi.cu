@@ -1048,13 +1048,15 @@ int centrality(phast_ctx* h, const uint32_t* sources, uint64_t count, uint32_t k
     const uint64_t nk = (uint64_t)n * k;
     if (nk >= 0xFFFFFFFFull) return PHAST_ERANGE;   // items are 32-bit
     if ((rc = ensure_in_csr(h)) || (rc = ensure_out_csr(h))) return rc;
-    // B batches share each chain of Kahn passes: as many as 32 n k bytes each fit a
-    // quarter of the free memory (at most 64, B n k < 2^32)
+    // B batches share each chain of Kahn passes: as many as 40 n k bytes each fit half
+    // the free memory, at most 64 GiB and 32 batches (C2, k 64: 32 batches = 82 GB;
+    // larger groups were measured slower per source: the passes turn DRAM-bound), B n k < 2^32
     size_t free_b = 0, total_b = 0;
     if (cudaMemGetInfo(&free_b, &total_b) != cudaSuccess) { cudaGetLastError(); free_b = 1ull << 32; }
     const uint64_t nbatches = (count + k - 1) / k;
-    uint64_t B = std::max<uint64_t>(1, (free_b / 4 + (uint64_t)h->bc_elems * 32) / (32 * nk));
-    B = std::min<uint64_t>({B, 64, nbatches, 0xFFFFFFFEull / nk});
+    const uint64_t budget = std::min<uint64_t>(free_b / 2 + (uint64_t)h->bc_elems * 40, 64ull << 30);
+    uint64_t B = std::max<uint64_t>(1, budget / (40 * nk));
+    B = std::min<uint64_t>({B, 32, nbatches, 0xFFFFFFFEull / nk});
     const size_t elems = (size_t)(B * nk);
     constexpr uint32_t R = 30;   // passes per graph launch / host convergence check (multiple of 6)
     if (!h->bc_changed) {
@@ -1070,7 +1072,7 @@ int centrality(phast_ctx* h, const uint32_t* sources, uint64_t count, uint32_t k
         h->bc_q = h->bc_dist = h->bc_src = nullptr;
         h->bc_elems = 0;
         if ((rc = dmalloc(&h->bc_sigma, elems)) || (rc = dmalloc(&h->bc_delta, elems)) ||
-            (rc = dmalloc(&h->bc_q, 3 * elems)) || (rc = dmalloc(&h->bc_dist, elems)) ||
+            (rc = dmalloc(&h->bc_q, 5 * elems)) || (rc = dmalloc(&h->bc_dist, elems)) ||
             (rc = dmalloc(&h->bc_src, (size_t)B * k)))
             return rc;
         h->bc_elems = elems;
@@ -1083,6 +1085,8 @@ int centrality(phast_ctx* h, const uint32_t* sources, uint64_t count, uint32_t k
     const BcGraph G{h->d_in_first, h->d_in_arc, h->d_out_first, h->d_out_arc, h->g.err};
     uint32_t* qbuf[2] = {h->bc_q, h->bc_q + elems};
     uint32_t* cnt = h->bc_q + 2 * elems;
+    uint32_t* mask_in = h->bc_q + 3 * elems;    // tight-arc masks (the forward count computes both)
+    uint32_t* mask_out = h->bc_q + 4 * elems;
     // R passes (+ clearing the change words before, reading them back after) are one CUDA
     // graph, captured once per group size and direction on a private stream (the caller's
     // stream may be the legacy default stream, which cannot be captured); R is a multiple
@@ -1136,7 +1140,8 @@ int centrality(phast_ctx* h, const uint32_t* sources, uint64_t count, uint32_t k
         // the count kernel and the chunks run on gs after everything queued on st so far
         if (cudaEventRecord(h->bc_ev, st) != cudaSuccess || cudaStreamWaitEvent(gs, h->bc_ev, 0) != cudaSuccess ||
             cudaMemsetAsync(h->bc_qs, 0, 12, gs) != cudaSuccess ||
-            launch_bc_count(G, d, (uint32_t)nk, k, total, backward, cnt, qbuf[0], h->bc_qs, gs) != cudaSuccess)
+            launch_bc_count(G, d, (uint32_t)nk, k, total, backward, cnt, mask_in, mask_out, qbuf[0], h->bc_qs, gs) !=
+                cudaSuccess)
             return PHAST_ECUDA;
         for (uint64_t it = 0; it <= (uint64_t)n + R; it += R) {
             if (cudaGraphLaunch(execs[which], gs) != cudaSuccess || cudaStreamSynchronize(gs) != cudaSuccess)
@@ -1167,8 +1172,15 @@ int centrality(phast_ctx* h, const uint32_t* sources, uint64_t count, uint32_t k
             return PHAST_ECUDA;
         if (reach) {
             if (cudaMemsetAsync(hgt, 0, (size_t)total * 4, st) != cudaSuccess) return PHAST_ECUDA;
+            // the masks come from the forward count: run it (no passes) before the height
+            if (cudaEventRecord(h->bc_ev, st) != cudaSuccess || cudaStreamWaitEvent(gs, h->bc_ev, 0) != cudaSuccess ||
+                cudaMemsetAsync(h->bc_qs, 0, 12, gs) != cudaSuccess ||
+                launch_bc_count(G, d, (uint32_t)nk, k, total, 0, cnt, mask_in, mask_out, qbuf[0], h->bc_qs, gs) !=
+                    cudaSuccess ||
+                cudaEventRecord(h->bc_ev, gs) != cudaSuccess || cudaStreamWaitEvent(st, h->bc_ev, 0) != cudaSuccess)
+                return PHAST_ECUDA;
             rc = kahn(2, 1, [&](const BcQueue& Q, uint32_t* ch, cudaStream_t s2) {
-                return launch_bc_back(G, d, nullptr, hgt, (uint32_t)nk, k, total, 1, Q, ch, s2);
+                return launch_bc_back(G, d, nullptr, hgt, (uint32_t)nk, k, total, mask_in, mask_out, 1, Q, ch, s2);
             });
             if (rc) return rc;
             graph_total = total;
@@ -1179,11 +1191,12 @@ int centrality(phast_ctx* h, const uint32_t* sources, uint64_t count, uint32_t k
             cudaMemsetAsync(h->bc_delta, 0, (size_t)total * 8, st) != cudaSuccess)
             return PHAST_ECUDA;
         rc = kahn(0, 0, [&](const BcQueue& Q, uint32_t* ch, cudaStream_t s2) {
-            return launch_bc_sigma(G, d, h->bc_sigma, (uint32_t)nk, k, total, Q, ch, s2);
+            return launch_bc_sigma(G, d, h->bc_sigma, (uint32_t)nk, k, total, mask_in, mask_out, Q, ch, s2);
         });
         if (rc) return rc;
         rc = kahn(1, 1, [&](const BcQueue& Q, uint32_t* ch, cudaStream_t s2) {
-            return launch_bc_back(G, d, h->bc_sigma, h->bc_delta, (uint32_t)nk, k, total, 0, Q, ch, s2);
+            return launch_bc_back(G, d, h->bc_sigma, h->bc_delta, (uint32_t)nk, k, total, mask_in, mask_out, 0, Q, ch,
+                                  s2);
         });
         if (rc) return rc;
         graph_total = total;

@@ -140,13 +140,17 @@ struct BcQueue {
     uint32_t* qs_clr;           // counter zeroed for the pass after next
     uint32_t* cnt;              // [n*k] unfinished inputs per item
 };
-// B batches of k trees at once: arrays [B][n][k], nk = n*k, total = B*nk items (< 2^32)
+// B batches of k trees at once: arrays [B][n][k], nk = n*k, total = B*nk items (< 2^32).
+// Forward count (backward = 0) computes the tight-arc masks min_/mout of every item and
+// the forward counts; the backward count only popcounts mout (call it after).
 cudaError_t launch_bc_count(const BcGraph& G, const uint32_t* d, uint32_t nk, uint32_t k, uint32_t total, int backward,
-                            uint32_t* cnt, uint32_t* q, uint32_t* qs, cudaStream_t st);
+                            uint32_t* cnt, uint32_t* min_, uint32_t* mout, uint32_t* q, uint32_t* qs, cudaStream_t st);
 cudaError_t launch_bc_sigma(const BcGraph& G, const uint32_t* d, double* sigma, uint32_t nk, uint32_t k,
-                            uint32_t total, const BcQueue& Q, uint32_t* changed, cudaStream_t st);
+                            uint32_t total, const uint32_t* min_, const uint32_t* mout, const BcQueue& Q,
+                            uint32_t* changed, cudaStream_t st);
 cudaError_t launch_bc_back(const BcGraph& G, const uint32_t* d, const double* sigma, void* val, uint32_t nk,
-                           uint32_t k, uint32_t total, int mode, const BcQueue& Q, uint32_t* changed, cudaStream_t st);
+                           uint32_t k, uint32_t total, const uint32_t* min_, const uint32_t* mout, int mode,
+                           const BcQueue& Q, uint32_t* changed, cudaStream_t st);
 // accumulation over trees j = b*k + i < valid; src: DEVICE internal ids of the trees
 cudaError_t launch_reach_accum(const uint32_t* d, const uint32_t* hgt, uint32_t* r, uint32_t n, uint32_t k,
                                uint32_t valid, cudaStream_t st);

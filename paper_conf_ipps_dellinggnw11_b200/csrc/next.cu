@@ -158,29 +158,60 @@ __device__ __forceinline__ void bc_push(uint32_t t, uint32_t* q, uint32_t* qs, b
 // the item of vertex u in item t's tree
 __device__ __forceinline__ uint32_t same_tree(uint32_t t, uint32_t v, uint32_t u, uint32_t k) { return t - v * k + u * k; }
 
-// cnt[t] = number of inputs of item t; items with none start the first queue
+// tight-arc masks: bit j of min[t] / mout[t] = the j-th in- / out-arc of item t's vertex
+// is tight in t's tree (arcs past the 32nd are re-tested from the labels when used)
+__device__ __forceinline__ bool mbit(uint32_t mask, uint32_t j) { return j < 32 ? (mask >> j) & 1u : false; }
+
+// Once per group: the masks of every finite item, then the forward counts (tight in-arcs;
+// items with none start queue 0).  The backward counts are popcounts of mout
+// (bc_count_back_kernel).
 __global__ void __launch_bounds__(256) bc_count_kernel(BcGraph G, const uint32_t* __restrict__ d, uint32_t nk,
-                                                       uint32_t k, uint32_t total, int backward, uint32_t* cnt,
-                                                       uint32_t* q, uint32_t* qs) {
+                                                       uint32_t k, uint32_t total, uint32_t* cnt, uint32_t* min_,
+                                                       uint32_t* mout, uint32_t* q, uint32_t* qs) {
     bool pushed = false;
     for (uint32_t t = blockIdx.x * blockDim.x + threadIdx.x; t < total; t += gridDim.x * blockDim.x) {
         const uint32_t v = (t % nk) / k;
         const uint32_t dv = __ldg(&d[t]);
         if (dv == INF) continue;
-        uint32_t c = 0;
-        if (!backward) {
-            const uint32_t e1 = __ldg(&G.in_first[v + 1]);
-            for (uint32_t e = __ldg(&G.in_first[v]); e < e1; e++) {
-                const uint2 a = __ldg(&G.in_arc[e]);
-                c += tight(__ldg(&d[same_tree(t, v, a.x, k)]), dv, a.y);
+        uint32_t c = 0, mi = 0, mo = 0;
+        const uint32_t e0 = __ldg(&G.in_first[v]), e1 = __ldg(&G.in_first[v + 1]);
+        for (uint32_t e = e0; e < e1; e++) {
+            const uint2 a = __ldg(&G.in_arc[e]);
+            if (tight(__ldg(&d[same_tree(t, v, a.x, k)]), dv, a.y)) {
+                c++;
+                if (e - e0 < 32) mi |= 1u << (e - e0);
             }
-        } else {
-            const uint32_t e1 = __ldg(&G.out_first[v + 1]);
-            for (uint32_t e = __ldg(&G.out_first[v]); e < e1; e++) {
-                const uint2 a = __ldg(&G.out_arc[e]);
-                const uint32_t dw = __ldg(&d[same_tree(t, v, a.x, k)]);
-                c += dw != INF && tight(dv, dw, a.y);
-            }
+        }
+        const uint32_t f0 = __ldg(&G.out_first[v]), f1 = __ldg(&G.out_first[v + 1]);
+        for (uint32_t e = f0; e < f1 && e - f0 < 32; e++) {
+            const uint2 a = __ldg(&G.out_arc[e]);
+            const uint32_t dw = __ldg(&d[same_tree(t, v, a.x, k)]);
+            if (dw != INF && tight(dv, dw, a.y)) mo |= 1u << (e - f0);
+        }
+        cnt[t] = c;
+        min_[t] = mi;
+        mout[t] = mo;
+        if (c == 0) bc_push(t, q, qs, pushed);
+    }
+    (void)pushed;
+}
+
+// backward counts: tight out-arcs (from mout; past the 32nd from the labels)
+__global__ void __launch_bounds__(256) bc_count_back_kernel(BcGraph G, const uint32_t* __restrict__ d, uint32_t nk,
+                                                            uint32_t k, uint32_t total, uint32_t* cnt,
+                                                            const uint32_t* __restrict__ mout, uint32_t* q,
+                                                            uint32_t* qs) {
+    bool pushed = false;
+    for (uint32_t t = blockIdx.x * blockDim.x + threadIdx.x; t < total; t += gridDim.x * blockDim.x) {
+        const uint32_t dv = __ldg(&d[t]);
+        if (dv == INF) continue;
+        uint32_t c = __popc(__ldg(&mout[t]));
+        const uint32_t v = (t % nk) / k;
+        const uint32_t f0 = __ldg(&G.out_first[v]), f1 = __ldg(&G.out_first[v + 1]);
+        for (uint32_t e = f0 + 32; e < f1; e++) {   // rare: more than 32 out-arcs
+            const uint2 a = __ldg(&G.out_arc[e]);
+            const uint32_t dw = __ldg(&d[same_tree(t, v, a.x, k)]);
+            c += dw != INF && tight(dv, dw, a.y);
         }
         cnt[t] = c;
         if (c == 0) bc_push(t, q, qs, pushed);
@@ -188,38 +219,118 @@ __global__ void __launch_bounds__(256) bc_count_kernel(BcGraph G, const uint32_t
     (void)pushed;
 }
 
+// Readied dependents: a thread decrements the counts of up to NB dependents of its item
+// together (the atomics in flight at once), keeps the ones that reach zero in registers
+// and the warp appends all of them with ONE atomic after a warp scan; the loop over the
+// queue is warp-uniform so every lane joins the scan.
+constexpr uint32_t NB = 8;
+
+struct Ready {
+    uint32_t w[NB];
+    uint32_t n = 0;
+    __device__ __forceinline__ void add(uint32_t x, uint32_t* q, uint32_t* qs, bool& pushed) {
+        if (n < NB) {
+#pragma unroll
+            for (uint32_t j = 0; j < NB; j++)
+                if (j == n) w[j] = x;
+            n++;
+        } else {
+            q[atomicAdd(qs, 1u)] = x;   // rare: more than NB readied by one item
+            pushed = true;
+        }
+    }
+    // all 32 lanes of the warp call this together
+    __device__ __forceinline__ void flush(uint32_t* q, uint32_t* qs, bool& pushed) {
+        const uint32_t lane = threadIdx.x & 31;
+        uint32_t incl = n;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const uint32_t y = __shfl_up_sync(0xFFFFFFFFu, incl, o);
+            if (lane >= (uint32_t)o) incl += y;
+        }
+        const uint32_t tot = __shfl_sync(0xFFFFFFFFu, incl, 31);
+        if (tot == 0) return;
+        uint32_t base = 0;
+        if (lane == 31) base = atomicAdd(qs, tot);
+        base = __shfl_sync(0xFFFFFFFFu, base, 31) + incl - n;
+#pragma unroll
+        for (uint32_t j = 0; j < NB; j++)
+            if (j < n) q[base + j] = w[j];
+        pushed = true;
+        n = 0;
+    }
+};
+
+// decrement the counts of the items `dep` of the tight arcs (bits of `mask` over arcs
+// [a0, a1) of CSR `arcs`; past the 32nd arc tested from the labels) and collect the
+// ones that reach zero
+__device__ __forceinline__ void bc_release(const uint2* __restrict__ arcs, uint32_t a0, uint32_t a1, uint32_t mask,
+                                           const uint32_t* __restrict__ d, uint32_t t, uint32_t v, uint32_t k,
+                                           bool out, uint32_t* cnt, Ready& rd, uint32_t* q, uint32_t* qs,
+                                           bool& pushed) {
+    for (uint32_t e = a0; e < a1; e += NB) {
+        uint32_t w[NB], old[NB];
+        bool on[NB];
+#pragma unroll
+        for (uint32_t j = 0; j < NB; j++) {
+            on[j] = false;
+            w[j] = 0;
+            if (e + j < a1) {
+                const uint32_t jj = e + j - a0;
+                const uint2 a = __ldg(&arcs[e + j]);
+                w[j] = same_tree(t, v, a.x, k);
+                if (jj < 32) {
+                    on[j] = mbit(mask, jj);
+                } else {   // rare: tightness from the labels
+                    const uint32_t dt = __ldg(&d[t]), dw = __ldg(&d[w[j]]);
+                    on[j] = out ? (dw != INF && tight(dt, dw, a.y)) : tight(dw, dt, a.y);
+                }
+            }
+        }
+#pragma unroll
+        for (uint32_t j = 0; j < NB; j++) old[j] = on[j] ? atomicSub(&cnt[w[j]], 1u) : 0u;   // in flight together
+#pragma unroll
+        for (uint32_t j = 0; j < NB; j++)
+            if (on[j] && old[j] == 1u) rd.add(w[j], q, qs, pushed);
+    }
+}
+
 // forward pass: sigma(v) = [v = s] + sum over tight (u, v) of sigma(u).  With lengths > 0
 // the source is the only finite item without a tight in-arc, so [v = s] is "no tight
 // in-arc" (no source list in the parameters: the passes are graph-captured once per call)
 __global__ void __launch_bounds__(256) bc_sigma_kernel(BcGraph G, const uint32_t* __restrict__ d, double* sigma,
-                                                       uint32_t nk, uint32_t k, BcQueue Q, uint32_t* changed) {
+                                                       uint32_t nk, uint32_t k, const uint32_t* __restrict__ min_,
+                                                       const uint32_t* __restrict__ mout, BcQueue Q,
+                                                       uint32_t* changed) {
     const uint32_t size = *Q.qs_in;
     if (blockIdx.x == 0 && threadIdx.x == 0) *Q.qs_clr = 0;
     bool pushed = false;
-    for (uint32_t x = blockIdx.x * blockDim.x + threadIdx.x; x < size; x += gridDim.x * blockDim.x) {
-        const uint32_t t = Q.q_in[x];
-        const uint32_t v = (t % nk) / k;
-        const uint32_t dv = __ldg(&d[t]);
-        double acc = 0.0;
-        bool any = false;
-        const uint32_t e1 = __ldg(&G.in_first[v + 1]);
-        for (uint32_t e = __ldg(&G.in_first[v]); e < e1; e++) {
-            const uint2 a = __ldg(&G.in_arc[e]);
-            const uint32_t u = same_tree(t, v, a.x, k);
-            if (tight(__ldg(&d[u]), dv, a.y)) {
-                acc += sigma[u];
-                any = true;
+    Ready rd;
+    for (uint32_t x0 = blockIdx.x * blockDim.x; x0 < size; x0 += gridDim.x * blockDim.x) {   // block-uniform
+        const uint32_t x = x0 + threadIdx.x;
+        if (x < size) {
+            const uint32_t t = Q.q_in[x];
+            const uint32_t v = (t % nk) / k;
+            const uint32_t mi = __ldg(&min_[t]), mo = __ldg(&mout[t]);
+            double acc = 0.0;
+            bool any = false;
+            const uint32_t e0 = __ldg(&G.in_first[v]), e1 = __ldg(&G.in_first[v + 1]);
+            for (uint32_t e = e0; e < e1; e++) {
+                const bool fast = e - e0 < 32;
+                if (fast && !mbit(mi, e - e0)) continue;
+                const uint2 a = __ldg(&G.in_arc[e]);
+                const uint32_t u = same_tree(t, v, a.x, k);
+                if (fast || tight(__ldg(&d[u]), __ldg(&d[t]), a.y)) {
+                    acc += sigma[u];
+                    any = true;
+                }
             }
+            if (!(acc <= 9007199254740992.0)) atomicOr(G.err, 1u);   // > 2^53 or not finite: not exact
+            sigma[t] = any ? acc : 1.0;
+            bc_release(G.out_arc, __ldg(&G.out_first[v]), __ldg(&G.out_first[v + 1]), mo, d, t, v, k, true, Q.cnt, rd,
+                       Q.q_out, Q.qs_out, pushed);
         }
-        if (!(acc <= 9007199254740992.0)) atomicOr(G.err, 1u);   // > 2^53 or not finite: not exact
-        sigma[t] = any ? acc : 1.0;
-        const uint32_t f1 = __ldg(&G.out_first[v + 1]);
-        for (uint32_t e = __ldg(&G.out_first[v]); e < f1; e++) {
-            const uint2 a = __ldg(&G.out_arc[e]);
-            const uint32_t w = same_tree(t, v, a.x, k);
-            const uint32_t dw = __ldg(&d[w]);
-            if (dw != INF && tight(dv, dw, a.y) && atomicSub(&Q.cnt[w], 1u) == 1u) bc_push(w, Q.q_out, Q.qs_out, pushed);
-        }
+        rd.flush(Q.q_out, Q.qs_out, pushed);
     }
     if (__syncthreads_or(pushed) && threadIdx.x == 0) *changed = 1;
 }
@@ -229,43 +340,42 @@ __global__ void __launch_bounds__(256) bc_sigma_kernel(BcGraph G, const uint32_t
 // `val` (l + h(w) <= d(w) + h(w) - d(v) is at most the largest finite label: no wrap)
 __global__ void __launch_bounds__(256) bc_back_kernel(BcGraph G, const uint32_t* __restrict__ d,
                                                       const double* __restrict__ sigma, void* val, uint32_t nk,
-                                                      uint32_t k, int mode, BcQueue Q, uint32_t* changed) {
+                                                      uint32_t k, const uint32_t* __restrict__ min_,
+                                                      const uint32_t* __restrict__ mout, int mode, BcQueue Q,
+                                                      uint32_t* changed) {
     const uint32_t size = *Q.qs_in;
     if (blockIdx.x == 0 && threadIdx.x == 0) *Q.qs_clr = 0;
     bool pushed = false;
     double* delta = static_cast<double*>(val);
     uint32_t* hgt = static_cast<uint32_t*>(val);
-    for (uint32_t x = blockIdx.x * blockDim.x + threadIdx.x; x < size; x += gridDim.x * blockDim.x) {
-        const uint32_t t = Q.q_in[x];
-        const uint32_t v = (t % nk) / k;
-        const uint32_t dv = __ldg(&d[t]);
-        const uint32_t e1 = __ldg(&G.out_first[v + 1]);
-        if (mode == 0) {
-            const double sv = __ldg(&sigma[t]);
-            double acc = 0.0;
-            for (uint32_t e = __ldg(&G.out_first[v]); e < e1; e++) {
+    Ready rd;
+    for (uint32_t x0 = blockIdx.x * blockDim.x; x0 < size; x0 += gridDim.x * blockDim.x) {   // block-uniform
+        const uint32_t x = x0 + threadIdx.x;
+        if (x < size) {
+            const uint32_t t = Q.q_in[x];
+            const uint32_t v = (t % nk) / k;
+            const uint32_t mi = __ldg(&min_[t]), mo = __ldg(&mout[t]);
+            const uint32_t f0 = __ldg(&G.out_first[v]), f1 = __ldg(&G.out_first[v + 1]);
+            double dacc = 0.0;
+            uint32_t hacc = 0;
+            const double sv = mode == 0 ? __ldg(&sigma[t]) : 0.0;
+            for (uint32_t e = f0; e < f1; e++) {
+                const bool fast = e - f0 < 32;
+                if (fast && !mbit(mo, e - f0)) continue;
                 const uint2 a = __ldg(&G.out_arc[e]);
                 const uint32_t w = same_tree(t, v, a.x, k);
-                const uint32_t dw = __ldg(&d[w]);
-                if (dw != INF && tight(dv, dw, a.y)) acc += sv / __ldg(&sigma[w]) * (1.0 + delta[w]);
+                if (!fast) {
+                    const uint32_t dw = __ldg(&d[w]);
+                    if (dw == INF || !tight(__ldg(&d[t]), dw, a.y)) continue;
+                }
+                if (mode == 0) dacc += sv / __ldg(&sigma[w]) * (1.0 + delta[w]);
+                else hacc = max(hacc, a.y + hgt[w]);
             }
-            delta[t] = acc;
-        } else {
-            uint32_t acc = 0;
-            for (uint32_t e = __ldg(&G.out_first[v]); e < e1; e++) {
-                const uint2 a = __ldg(&G.out_arc[e]);
-                const uint32_t w = same_tree(t, v, a.x, k);
-                const uint32_t dw = __ldg(&d[w]);
-                if (dw != INF && tight(dv, dw, a.y)) acc = max(acc, a.y + hgt[w]);
-            }
-            hgt[t] = acc;
+            if (mode == 0) delta[t] = dacc; else hgt[t] = hacc;
+            bc_release(G.in_arc, __ldg(&G.in_first[v]), __ldg(&G.in_first[v + 1]), mi, d, t, v, k, false, Q.cnt, rd,
+                       Q.q_out, Q.qs_out, pushed);
         }
-        const uint32_t f1 = __ldg(&G.in_first[v + 1]);
-        for (uint32_t e = __ldg(&G.in_first[v]); e < f1; e++) {
-            const uint2 a = __ldg(&G.in_arc[e]);
-            const uint32_t u = same_tree(t, v, a.x, k);
-            if (tight(__ldg(&d[u]), dv, a.y) && atomicSub(&Q.cnt[u], 1u) == 1u) bc_push(u, Q.q_out, Q.qs_out, pushed);
-        }
+        rd.flush(Q.q_out, Q.qs_out, pushed);
     }
     if (__syncthreads_or(pushed) && threadIdx.x == 0) *changed = 1;
 }
@@ -311,22 +421,27 @@ unsigned bc_pass_blocks(uint64_t items) { return bc_blocks(items); }
 }  // namespace
 
 cudaError_t launch_bc_count(const BcGraph& G, const uint32_t* d, uint32_t nk, uint32_t k, uint32_t total, int backward,
-                            uint32_t* cnt, uint32_t* q, uint32_t* qs, cudaStream_t st) {
-    bc_count_kernel<<<bc_blocks(total), 256, 0, st>>>(G, d, nk, k, total, backward, cnt, q, qs);
+                            uint32_t* cnt, uint32_t* min_, uint32_t* mout, uint32_t* q, uint32_t* qs, cudaStream_t st) {
+    if (backward)
+        bc_count_back_kernel<<<bc_blocks(total), 256, 0, st>>>(G, d, nk, k, total, cnt, mout, q, qs);
+    else
+        bc_count_kernel<<<bc_blocks(total), 256, 0, st>>>(G, d, nk, k, total, cnt, min_, mout, q, qs);
     count_launch();
     return cudaGetLastError();
 }
 
 cudaError_t launch_bc_sigma(const BcGraph& G, const uint32_t* d, double* sigma, uint32_t nk, uint32_t k,
-                            uint32_t total, const BcQueue& Q, uint32_t* changed, cudaStream_t st) {
-    bc_sigma_kernel<<<bc_pass_blocks(total), 256, 0, st>>>(G, d, sigma, nk, k, Q, changed);
+                            uint32_t total, const uint32_t* min_, const uint32_t* mout, const BcQueue& Q,
+                            uint32_t* changed, cudaStream_t st) {
+    bc_sigma_kernel<<<bc_pass_blocks(total), 256, 0, st>>>(G, d, sigma, nk, k, min_, mout, Q, changed);
     count_launch();
     return cudaGetLastError();
 }
 
 cudaError_t launch_bc_back(const BcGraph& G, const uint32_t* d, const double* sigma, void* val, uint32_t nk,
-                           uint32_t k, uint32_t total, int mode, const BcQueue& Q, uint32_t* changed, cudaStream_t st) {
-    bc_back_kernel<<<bc_pass_blocks(total), 256, 0, st>>>(G, d, sigma, val, nk, k, mode, Q, changed);
+                           uint32_t k, uint32_t total, const uint32_t* min_, const uint32_t* mout, int mode,
+                           const BcQueue& Q, uint32_t* changed, cudaStream_t st) {
+    bc_back_kernel<<<bc_pass_blocks(total), 256, 0, st>>>(G, d, sigma, val, nk, k, min_, mout, mode, Q, changed);
     count_launch();
     return cudaGetLastError();
 }
