@@ -226,7 +226,7 @@ def main():
                     help="also time the parent-pointer pass (phast_parents, NEXT-1) on the last batch")
     args = ap.parse_args()
     args.warmup = max(3, args.warmup)
-    args.inflight = max(0, min(4, args.inflight))
+    args.inflight = max(0, min(8, args.inflight))
     if args.impl == "reference":
         return run_reference(args)
     if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
