@@ -427,10 +427,21 @@ def main():
         h.sync(stream)
         pms = p0.elapsed_time(p1) / reps
         B_par = 8 * info.m + 4 * (n + 1) + 12 * k * n
+        h.parents_ch(last, dist_t, out=par_buf, stream=stream)   # first use uploads the A-up in-arcs
+        h.sync(stream)
+        p0.record(stream)
+        for _ in range(reps):
+            h.parents_ch(last, dist_t, out=par_buf, stream=stream)
+        p1.record(stream)
+        h.sync(stream)
+        cms = p0.elapsed_time(p1) / reps
         parents = {"ms_per_pass": pms, "alg_bytes": B_par, "achieved_GBps": B_par / (pms / 1e3) / 1e9,
                    "frac": B_par / (pms / 1e3) / 1e9 / peak,
                    "note": "B = 8m + 4(n+1) + 12kn: in-arcs, offsets, own row read, in-neighbour rows read "
-                           "at least once, parent row written"}
+                           "at least once, parent row written",
+                   "hierarchy_ms_per_pass": cms,
+                   "hierarchy_note": "phast_parents_ch (G+ parents, reading R19): the same pass over the "
+                                     "A-down in-arcs, then the A-up in-arcs for trees still without a parent"}
         del par_buf
 
     # end to end through the public host entry point (sources in, all labels out)

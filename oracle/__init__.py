@@ -7,7 +7,8 @@ reference` legs may import this package.  The product path
 Plain binary-heap Dijkstra on the ORIGINAL graph (§II-A), exact by
 Theorem 3.1 (§III) for what PHAST computes; diameter (PAPER.md:20
 §VII-B); O(n+m) optimality certificate; canonical parent
-pointers by the tight-arc identity (§VII-A, reading R14); exact betweenness
+pointers by the tight-arc identity (§VII-A, reading R14) and in the hierarchy
+G+ (reading R19); exact betweenness
 and reach (§VII-B, readings R16/R17, plain Python below).  See oracle.c for the
 passage each function follows.  Pins: tests/test_oracle.py.  Parity status of
 every function: pinned.
@@ -131,6 +132,48 @@ def parents(g, s: int, d=None) -> np.ndarray:
     if rc:
         raise ValueError(f"oracle_parents: {rc}")
     return out
+
+
+def parents_ch(ex: dict, d_int, s_int: int) -> np.ndarray:
+    """uint32[n]: parent pointers in the contraction hierarchy G+ = A-down U A-up
+    (shortcuts included) -- "it suffices to remember the arc (u, v) responsible for
+    d(v)" (§VII-A) and "some of the parent pointers in this case will be
+    shortcuts" (§VII-A), reading R19.
+
+    Inputs are in INTERNAL ids: `ex` = the exported hierarchy (Phast.export(): dn_first /
+    dn_tail / dn_len = A-down in-arcs by head, up_first / up_head / up_len = A-up out-arcs
+    by tail), `d_int` = the TRUE distances from the source (oracle sssp, permuted to
+    internal ids), `s_int` = the source.  The definition written out: parent(s) = s;
+    parent(v) = INF where d(v) = INF; else the tail of v's first tight A-down in-arc
+    (d(u) + l = d(v), export order), and if there is none the tail of its first tight
+    A-up in-arc (tails in increasing id, each tail's arcs in export order).  A tight arc
+    always exists (a shortest up-down path reaches v either down an A-down arc or, at its
+    peak, up an A-up arc; §III) -- the pins check it.  Plain Python: small
+    graphs only."""
+    d = np.asarray(d_int, dtype=np.int64)
+    n = d.size
+    dn_first = ex["dn_first"].astype(np.int64)
+    dn_tail, dn_len = ex["dn_tail"].astype(np.int64), ex["dn_len"].astype(np.int64)
+    up_first = ex["up_first"].astype(np.int64)
+    up_head, up_len = ex["up_head"].astype(np.int64), ex["up_len"].astype(np.int64)
+    par = np.full(n, INF, dtype=np.int64)
+    for v in range(n):
+        if d[v] == INF or v == s_int:
+            continue
+        for e in range(dn_first[v], dn_first[v + 1]):
+            u = dn_tail[e]
+            if d[u] != INF and d[u] + dn_len[e] == d[v]:
+                par[v] = u
+                break
+    for u in range(n):                 # A-up in-arcs: tails in increasing id
+        if d[u] == INF:
+            continue
+        for e in range(up_first[u], up_first[u + 1]):
+            v = up_head[e]
+            if par[v] == INF and v != s_int and d[v] != INF and d[u] + up_len[e] == d[v]:
+                par[v] = u
+    par[s_int] = s_int
+    return par.astype(np.uint32)
 
 
 def betweenness(g, sources) -> np.ndarray:

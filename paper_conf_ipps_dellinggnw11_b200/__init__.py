@@ -73,6 +73,7 @@ def _load_lib():
         "phast_trees": ([vp, vp, u32, vp, vp], ci),
         "phast_trees_host": ([vp, vp, u32, vp, vp], ci),
         "phast_parents": ([vp, vp, u32, vp, vp, vp], ci),
+        "phast_parents_ch": ([vp, vp, u32, vp, vp, vp], ci),
         "phast_sync": ([vp, vp], ci),
         "phast_diameter": ([vp, vp, u64, u32, vp, vp, vp], ci),
         "phast_diameter_witness": ([vp, vp, u64, u32, vp, vp], ci),
@@ -282,6 +283,18 @@ class Phast:
         out = self._out(out, self.n * k, _u32_dtypes(), "parents(out)")
         _check("phast_parents", _lib.phast_parents(self._h, src.ctypes.data, k, dist.data_ptr(), out.data_ptr(),
                                                    _stream_ptr(stream)))
+        return out.view(self.n, k)
+
+    def parents_ch(self, sources, dist, out=None, stream=None):
+        """Parent pointers in the hierarchy G+ (phast_parents_ch, reading R19): device
+        tensor [n, k] of INTERNAL ids (parents may be shortcut tails)."""
+        src = _sources(sources)
+        k = int(src.size)
+        _check_k(k)
+        _device_out(dist, self.n * k, _u32_dtypes(), self.device, "parents_ch(dist)")
+        out = self._out(out, self.n * k, _u32_dtypes(), "parents_ch(out)")
+        _check("phast_parents_ch", _lib.phast_parents_ch(self._h, src.ctypes.data, k, dist.data_ptr(),
+                                                         out.data_ptr(), _stream_ptr(stream)))
         return out.view(self.n, k)
 
     def parents_to_original(self, rows: np.ndarray) -> np.ndarray:

@@ -88,6 +88,9 @@ struct phast_ctx {
         uint2* up_a = nullptr;
     };
     std::map<uint32_t, Top> tops;
+    // A-up in-arcs by head {tail, len}, all of them (hierarchy parents; uploaded on first use)
+    uint32_t* d_upall_first = nullptr;
+    uint2* d_upall_arc = nullptr;
     // A-up in-arcs by head {tail, len} (fused single-launch queries on small graphs)
     uint32_t* d_upin_first = nullptr;
     uint2* d_upin_arc = nullptr;
@@ -229,6 +232,8 @@ void free_device(phast_ctx* h) {
     if (h->bc_stream) cudaStreamDestroy(h->bc_stream);
     if (h->bc_ev) cudaEventDestroy(h->bc_ev);
     cudaFree(h->d_upin_first); cudaFree(h->d_upin_arc);
+    cudaFree(h->d_upall_first); cudaFree(h->d_upall_arc);
+    h->d_upall_first = nullptr; h->d_upall_arc = nullptr;
     h->host_scratch = nullptr; h->host_elems = 0;
     h->batch_max_scratch = nullptr; h->batch_max_elems = 0; h->wit = nullptr;
     h->d_in_first = nullptr; h->d_in_arc = nullptr;
@@ -950,6 +955,28 @@ int phast_parents(phast_ctx* h, const uint32_t* sources, uint32_t k, const uint3
     if (!dg.ok) return PHAST_ECUDA;
     if ((rc = ensure_in_csr(h))) return rc;
     if (launch_parents(h->d_in_first, h->d_in_arc, h->n, S, k, dist, parent, (cudaStream_t)stream) != cudaSuccess)
+        return PHAST_ECUDA;
+    return PHAST_OK;
+}
+
+int phast_parents_ch(phast_ctx* h, const uint32_t* sources, uint32_t k, const uint32_t* dist, uint32_t* parent,
+                     void* stream) {
+    int rc = check_handle(h);
+    if (rc) return rc;
+    if (!sources || !dist || !parent || !k_valid(k)) return PHAST_EINVAL;
+    if (k % 4 == 0 && kpad(k) == k && (((uintptr_t)dist & 15) || ((uintptr_t)parent & 15))) return PHAST_EINVAL;
+    Sources S;
+    if ((rc = map_sources(h, sources, k, k, S))) return rc;
+    DeviceGuard dg(h->device);
+    if (!dg.ok) return PHAST_ECUDA;
+    if (!h->d_upall_first) {
+        std::vector<uint32_t> f;
+        std::vector<Arc> arc;
+        if (!upin_csr(h->L, h->n, 0xFFFFFFFFu, f, arc) || !upload_csr(f, arc, &h->d_upall_first, &h->d_upall_arc))
+            return PHAST_ENOMEM;
+    }
+    if (launch_parents_ch(h->g.dn_first, h->g.dn_arc, h->d_upall_first, h->d_upall_arc, h->n, S, k, dist, parent,
+                          (cudaStream_t)stream) != cudaSuccess)
         return PHAST_ECUDA;
     return PHAST_OK;
 }

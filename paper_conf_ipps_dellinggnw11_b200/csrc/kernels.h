@@ -123,6 +123,14 @@ cudaError_t launch_probe_stream(const DevImage& g, uint32_t k, uint32_t* dist, c
 cudaError_t launch_parents(const uint32_t* in_first, const uint2* in_arc, uint32_t n, const Sources& src,
                            uint32_t k, const uint32_t* dist, uint32_t* parent, cudaStream_t st);
 
+// NEXT-1 parent pointers in the hierarchy G+ = A-down U A-up (reading R19): parent[r*k +
+// i] = the tail of v's first tight A-down in-arc (dn_first/dn_arc order), else of its
+// first tight A-up in-arc (upin: A-up in-arcs by head, tails increasing); the source's
+// own entry is itself; INF where d_i(v) = INF.  Any 1 <= k <= 64.
+cudaError_t launch_parents_ch(const uint32_t* dn_first, const uint2* dn_arc, const uint32_t* upin_first,
+                              const uint2* upin_arc, uint32_t n, const Sources& src, uint32_t k, const uint32_t* dist,
+                              uint32_t* parent, cudaStream_t st);
+
 // NEXT-3 betweenness / reach (next.cu): passes in Kahn order of each tree's tight DAG;
 // items t = v*k + i (n*k < 2^32).
 struct BcGraph {

@@ -18,9 +18,13 @@ constexpr int SWEEP_THREADS = 256;
 // the first tight arc (§VII-A).  The identity is tested as d(u) <= d(v)
 // and d(v) - d(u) = l, which equals d(u) + l = d(v) exactly (no 32-bit overflow).
 // The scan stops once every finite tree of the lane has its parent.
-template <int K>
+// PLUS (hierarchy parents, reading R19): a second in-arc CSR (A-up in-arcs) is scanned
+// after the first (A-down in-arcs) for the trees still without a parent.
+template <int K, bool PLUS>
 __global__ void __launch_bounds__(SWEEP_THREADS) parents_kernel(const uint32_t* __restrict__ in_first,
                                                                 const uint2* __restrict__ in_arc,
+                                                                const uint32_t* __restrict__ in_first2,
+                                                                const uint2* __restrict__ in_arc2,
                                                                 const uint32_t* __restrict__ d,
                                                                 uint32_t* __restrict__ parent, uint32_t n,
                                                                 Sources src) {
@@ -40,17 +44,21 @@ __global__ void __launch_bounds__(SWEEP_THREADS) parents_kernel(const uint32_t* 
             p[q] = INF;
             if (dv[q] != INF) need |= 1u << q;
         }
-        const uint32_t e1 = __ldg(&in_first[v + 1]);
-        for (uint32_t e = __ldg(&in_first[v]); need && e < e1; e++) {
-            const uint2 a = __ldg(&in_arc[e]);
-            const T ru = __ldg(reinterpret_cast<const T*>(d + (size_t)a.x * K) + lane);
-            const uint32_t* du = reinterpret_cast<const uint32_t*>(&ru);
+        for (int pass = 0; pass < (PLUS ? 2 : 1); pass++) {
+            const uint32_t* f = pass ? in_first2 : in_first;
+            const uint2* arcs = pass ? in_arc2 : in_arc;
+            const uint32_t e1 = __ldg(&f[v + 1]);
+            for (uint32_t e = __ldg(&f[v]); need && e < e1; e++) {
+                const uint2 a = __ldg(&arcs[e]);
+                const T ru = __ldg(reinterpret_cast<const T*>(d + (size_t)a.x * K) + lane);
+                const uint32_t* du = reinterpret_cast<const uint32_t*>(&ru);
 #pragma unroll
-            for (uint32_t q = 0; q < W; q++)
-                if (((need >> q) & 1u) && du[q] <= dv[q] && dv[q] - du[q] == a.y) {
-                    p[q] = a.x;
-                    need &= ~(1u << q);
-                }
+                for (uint32_t q = 0; q < W; q++)
+                    if (((need >> q) & 1u) && du[q] <= dv[q] && dv[q] - du[q] == a.y) {
+                        p[q] = a.x;
+                        need &= ~(1u << q);
+                    }
+            }
         }
 #pragma unroll
         for (uint32_t q = 0; q < W; q++)
@@ -96,12 +104,77 @@ cudaError_t parents_k(const uint32_t* in_first, const uint2* in_arc, uint32_t n,
     uint64_t blocks = ((uint64_t)n * G + SWEEP_THREADS - 1) / SWEEP_THREADS;
     blocks = std::min<uint64_t>(blocks, (uint64_t)num_sms() * 8);
     if (blocks == 0) return cudaSuccess;
-    parents_kernel<K><<<(unsigned)blocks, SWEEP_THREADS, 0, st>>>(in_first, in_arc, dist, parent, n, src);
+    parents_kernel<K, false><<<(unsigned)blocks, SWEEP_THREADS, 0, st>>>(in_first, in_arc, nullptr, nullptr, dist, parent,
+                                                                      n, src);
     count_launch();
     return cudaGetLastError();
 }
 
+// G+ parents (reading R19): one thread per (vertex, tree) item; A-down in-arcs first,
+// then A-up in-arcs, the first tight one wins
+__global__ void __launch_bounds__(SWEEP_THREADS) parents_ch_kernel(const uint32_t* __restrict__ dn_first,
+                                                                   const uint2* __restrict__ dn_arc,
+                                                                   const uint32_t* __restrict__ up_first,
+                                                                   const uint2* __restrict__ up_arc,
+                                                                   const uint32_t* __restrict__ d,
+                                                                   uint32_t* __restrict__ parent, uint32_t n,
+                                                                   uint32_t k, Sources src) {
+    const uint64_t total = (uint64_t)n * k;
+    for (uint64_t t = (uint64_t)blockIdx.x * SWEEP_THREADS + threadIdx.x; t < total;
+         t += (uint64_t)gridDim.x * SWEEP_THREADS) {
+        const uint32_t v = (uint32_t)(t / k), i = (uint32_t)(t % k);
+        const uint32_t dv = __ldg(&d[t]);
+        uint32_t p = INF;
+        if (dv != INF) {
+            const uint32_t e1 = __ldg(&dn_first[v + 1]);
+            for (uint32_t e = __ldg(&dn_first[v]); e < e1 && p == INF; e++) {
+                const uint2 a = __ldg(&dn_arc[e]);
+                const uint32_t du = __ldg(&d[(size_t)a.x * k + i]);
+                if (du <= dv && dv - du == a.y) p = a.x;
+            }
+            const uint32_t f1 = __ldg(&up_first[v + 1]);
+            for (uint32_t e = __ldg(&up_first[v]); e < f1 && p == INF; e++) {
+                const uint2 a = __ldg(&up_arc[e]);
+                const uint32_t du = __ldg(&d[(size_t)a.x * k + i]);
+                if (du <= dv && dv - du == a.y) p = a.x;
+            }
+        }
+        if (src.s[i] == v) p = v;
+        parent[t] = p;
+    }
+}
+
 }  // namespace
+
+template <int K>
+cudaError_t parents_ch_k(const uint32_t* dn_first, const uint2* dn_arc, const uint32_t* upin_first, const uint2* upin_arc,
+                         uint32_t n, const Sources& src, const uint32_t* dist, uint32_t* parent, cudaStream_t st) {
+    constexpr uint32_t G = K / RowT<K>::W;
+    uint64_t blocks = ((uint64_t)n * G + SWEEP_THREADS - 1) / SWEEP_THREADS;
+    blocks = std::min<uint64_t>(blocks, (uint64_t)num_sms() * 8);
+    if (blocks == 0) return cudaSuccess;
+    parents_kernel<K, true><<<(unsigned)blocks, SWEEP_THREADS, 0, st>>>(dn_first, dn_arc, upin_first, upin_arc, dist,
+                                                                        parent, n, src);
+    count_launch();
+    return cudaGetLastError();
+}
+
+cudaError_t launch_parents_ch(const uint32_t* dn_first, const uint2* dn_arc, const uint32_t* upin_first,
+                              const uint2* upin_arc, uint32_t n, const Sources& src, uint32_t k, const uint32_t* dist,
+                              uint32_t* parent, cudaStream_t st) {
+    if (k == 1 || k == 2 || k == 4 || k == 8 || k == 16 || k == 32 || k == 64) {
+#define CALL_PC(K) parents_ch_k<K>(dn_first, dn_arc, upin_first, upin_arc, n, src, dist, parent, st)
+        PHAST_K_SWITCH(k, CALL_PC)
+#undef CALL_PC
+    }
+    uint64_t blocks = ((uint64_t)n * k + SWEEP_THREADS - 1) / SWEEP_THREADS;
+    blocks = std::min<uint64_t>(blocks, (uint64_t)num_sms() * 8);
+    if (blocks == 0) return cudaSuccess;
+    parents_ch_kernel<<<(unsigned)blocks, SWEEP_THREADS, 0, st>>>(dn_first, dn_arc, upin_first, upin_arc, dist, parent,
+                                                                  n, k, src);
+    count_launch();
+    return cudaGetLastError();
+}
 
 cudaError_t launch_parents(const uint32_t* in_first, const uint2* in_arc, uint32_t n, const Sources& src,
                            uint32_t k, const uint32_t* dist, uint32_t* parent, cudaStream_t st) {

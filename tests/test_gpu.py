@@ -588,3 +588,30 @@ def test_centrality_padded_batches():
         r = h.vertex_to_original(h.reach(src, k_batch=11).cpu().numpy().view(np.uint32))
     bc_close(cb, oracle.betweenness(g, src))
     assert np.array_equal(r, oracle.reach(g, src))
+
+
+@pytest.mark.parametrize("name", ["c1", "road", "unit_grid", "unreachable", "zero_lengths"])
+def test_parents_ch_bit_exact(c1, road, name):
+    """NEXT-1 in the hierarchy (phast_parents_ch, reading R19): bit-exact with
+    oracle.parents_ch on the exported hierarchy and the oracle's distances, for k in
+    {1, 5, 16, 64}; parents are internal ids, shortcut tails included."""
+    if name == "c1":
+        g, h = c1
+    elif name == "road":
+        g, h = road
+    else:
+        g = EDGE_GRAPHS[name]()
+        h = P.Phast.from_graph(g)
+    ex = h.export()
+    perm = h.order()
+    for k in (1, 5, 16, 64):
+        src = phastgen.sources(g.n, k, seed=700 + k, distinct=False)
+        d = h.trees(src)
+        p = h.parents_ch(src, d)
+        h.sync()
+        rows = p.cpu().numpy().view(np.uint32).reshape(h.n, k)
+        for i in (0, k // 2, k - 1):
+            dint = np.empty(h.n, np.int64)
+            dint[perm] = oracle.sssp(g, int(src[i])).astype(np.int64)
+            want = oracle.parents_ch(ex, dint, int(perm[src[i]]))
+            assert np.array_equal(rows[:, i], want), (name, k, i)

@@ -10,6 +10,7 @@ import numpy as np
 import pytest
 
 import oracle
+from oracle import INF
 import phastgen
 import chref
 
@@ -232,3 +233,57 @@ def test_info_upward_search_space_stats():
     assert 10 < inf.mean_up_space < 2000
     small = P.Phast.from_graph(phastgen.grid(5, 4), host_only=True).info()
     assert small.up_space_samples == 20 and small.max_up_space <= 20
+
+
+CH_PARENT_GRAPHS = {
+    "grid": lambda: phastgen.grid(30, 20, 1, 1000, seed=11),
+    "unit_grid": lambda: phastgen.grid(20, 15, 1, 2, seed=12),        # many ties
+    "road": lambda: phastgen.road(5_000, seed=13),
+    "unreachable": lambda: phastgen.random_digraph(600, 500, 1, 50, seed=14),
+    "zero_lengths": lambda: phastgen.random_digraph(300, 1200, 0, 3, seed=15),
+}
+
+
+@pytest.mark.parametrize("name", sorted(CH_PARENT_GRAPHS))
+def test_oracle_parents_ch_pins(name):
+    """Pins of oracle.parents_ch (hierarchy parent pointers, reading R19) independent of
+    its own code: with the true distances (pinned Dijkstra), every finite v != s gets a
+    parent (an up-down shortest path always enters v by an A-down arc or, at its peak,
+    an A-up arc: §III); the parent arc exists in A-down U A-up (checked
+    against an arc map built here) and is tight; with lengths > 0 the pointers form a
+    tree rooted at s (following them from any v reaches s); unreachable stays INF."""
+    g = CH_PARENT_GRAPHS[name]()
+    h = P.Phast.from_graph(g, host_only=True)
+    ex = h.export()
+    perm = h.order()
+    n = h.n
+    arcs = {}
+    heads = np.repeat(np.arange(n), np.diff(ex["dn_first"].astype(np.int64)))
+    for t, v, l in zip(ex["dn_tail"].tolist(), heads.tolist(), ex["dn_len"].tolist()):
+        arcs[(t, v)] = min(arcs.get((t, v), 1 << 40), l)
+    tails = np.repeat(np.arange(n), np.diff(ex["up_first"].astype(np.int64)))
+    for u, v, l in zip(tails.tolist(), ex["up_head"].tolist(), ex["up_len"].tolist()):
+        arcs[(u, v)] = min(arcs.get((u, v), 1 << 40), l)
+    positive = int(np.asarray(g.len).min()) > 0
+    for s in phastgen.sources(g.n, 4, seed=3):
+        d = np.empty(n, np.int64)
+        d[perm] = oracle.sssp(g, int(s)).astype(np.int64)
+        si = int(perm[s])
+        par = oracle.parents_ch(ex, d, si).astype(np.int64)
+        assert par[si] == si
+        for v in range(n):
+            if d[v] == INF:
+                assert par[v] == INF
+                continue
+            if v == si:
+                continue
+            u = int(par[v])
+            assert u != INF, (name, s, v)
+            assert (u, v) in arcs and d[u] + arcs[(u, v)] == d[v], (name, s, v, u)
+        if positive:
+            for v in range(n):
+                x, steps = v, 0
+                while d[v] != INF and x != si:
+                    x = int(par[x])
+                    steps += 1
+                    assert steps <= n, (name, s, v)
