@@ -218,8 +218,13 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-probes", action="store_true")
     ap.add_argument("--cache", default="", help="hierarchy file to reuse/create (optional)")
-    ap.add_argument("--layout", default="levels-bfs", choices=["levels", "levels-bfs"],
-                    help="vertex order: the paper's level layout (DFS within a level) or BFS within a level")
+    ap.add_argument("--layout", default="levels-bands", choices=["levels", "levels-bfs", "levels-bands"],
+                    help="vertex order: the paper's level layout (DFS within a level), BFS within a level, or "
+                         "BFS with the bottom levels in bands of closed groups (default)")
+    ap.add_argument("--band-unit", type=int, default=0,
+                    help="vertices per work unit of a band launch (phast_query_opts band_unit; 0 = 8192/k)")
+    ap.add_argument("--band-threads", type=int, default=0, help="CTA size of a band launch (128/256; 0 = 128)")
+    ap.add_argument("--band-variant", type=int, default=0, help="band kernel variant (phast_query_opts band_variant)")
     ap.add_argument("--query-flags", type=int, default=0,
                     help="phast_configure flags (schedule experiments: 1 no fused single-launch query, 2 no shared-memory top launch)")
     ap.add_argument("--parents", action="store_true",
@@ -279,8 +284,9 @@ def main():
         log(f"[bench] CH build {time.time() - t:.1f}s")
         if args.cache:
             h.save(args.cache)
-    if args.query_flags:
-        h.configure(flags=args.query_flags)
+    if args.query_flags or args.band_unit or args.band_threads or args.band_variant:
+        h.configure(flags=args.query_flags, band_unit=args.band_unit, band_threads=args.band_threads,
+                    band_variant=args.band_variant)
     n = h.n
     info = h.info()
     lsz = h.level_sizes()

@@ -26,9 +26,10 @@ SLOTS = 4
 FLAG_HOST_ONLY = 1
 FLAG_LEVEL_LAYOUT = 2
 FLAG_BFS_IN_LEVEL = 4
-LAYOUT_FLAGS = {"levels-bfs": 0, "levels": FLAG_LEVEL_LAYOUT}
-LAYOUT_NAMES = {1: "levels", 2: "levels-bfs"}   # phast_info_t.layout
-Q_NO_FUSED, Q_NO_TOP, Q_HYBRID_ON, Q_HYBRID_OFF, Q_NO_MULTI = 1, 2, 4, 8, 32
+FLAG_NO_BANDS = 32
+LAYOUT_FLAGS = {"levels-bands": 0, "levels-bfs": FLAG_NO_BANDS, "levels": FLAG_LEVEL_LAYOUT}
+LAYOUT_NAMES = {1: "levels", 2: "levels-bfs", 3: "levels-bands"}   # phast_info_t.layout
+Q_NO_FUSED, Q_NO_TOP, Q_HYBRID_ON, Q_HYBRID_OFF, Q_NO_MULTI, Q_NO_BANDS = 1, 2, 4, 8, 32, 64
 
 STATUS = {0: "OK", -1: "EINVAL", -2: "ENOMEM", -3: "ECUDA", -4: "ERANGE", -5: "ESTATE", -6: "EIO",
           -7: "EINTERNAL"}
@@ -48,7 +49,9 @@ class _Opts(ctypes.Structure):
 
 class _QOpts(ctypes.Structure):
     _fields_ = [("flags", ctypes.c_uint32), ("top_max_vertices", ctypes.c_uint32),
-                ("seed_cap", ctypes.c_uint32), ("up_smem_cap", ctypes.c_uint32)]
+                ("seed_cap", ctypes.c_uint32), ("up_smem_cap", ctypes.c_uint32),
+                ("band_unit", ctypes.c_uint32), ("band_threads", ctypes.c_uint32),
+                ("band_variant", ctypes.c_uint32)]
 
 
 class _Info(ctypes.Structure):
@@ -83,6 +86,8 @@ def _load_lib():
         "phast_level_sizes": ([vp, vp], ci),
         "phast_order": ([vp, vp], ci),
         "phast_export": ([vp, vp, vp, vp, vp, vp, vp, vp], ci),
+        "phast_bands": ([vp, vp, vp], ci),
+        "phast_band_groups": ([vp, u32, vp], ci),
         "phast_schedule": ([vp, u32, vp], ci),
         "phast_save": ([vp, ctypes.c_char_p], ci),
         "phast_load": ([ctypes.c_char_p, u32, pp], ci),
@@ -179,7 +184,7 @@ class Phast:
     """A built hierarchy bound to one CUDA device (phast_ctx)."""
 
     def __init__(self, n=None, first=None, head=None, length=None, *, host_only=False, threads=0,
-                 hop_limit_lo=0, hop_limit_hi=0, settled_cap=0, layout="levels-bfs", _handle=None):
+                 hop_limit_lo=0, hop_limit_hi=0, settled_cap=0, layout="levels-bands", _handle=None):
         self._h = None
         if _handle is not None:
             self._h = _handle
@@ -217,9 +222,10 @@ class Phast:
     def save(self, path):
         _check("phast_save", _lib.phast_save(self._h, path.encode()))
 
-    def configure(self, flags=0, top_max_vertices=0, seed_cap=0, up_smem_cap=0):
+    def configure(self, flags=0, top_max_vertices=0, seed_cap=0, up_smem_cap=0, band_unit=0, band_threads=0,
+                  band_variant=0):
         """Query-path options (phast_configure): schedule choices only, same labels."""
-        q = _QOpts(flags, top_max_vertices, seed_cap, up_smem_cap)
+        q = _QOpts(flags, top_max_vertices, seed_cap, up_smem_cap, band_unit, band_threads, band_variant)
         _check("phast_configure", _lib.phast_configure(self._h, ctypes.byref(q)))
         return self
 
@@ -374,10 +380,10 @@ class Phast:
 
     def schedule(self, k: int) -> dict:
         """Launch schedule of a k-tree query (phast_schedule)."""
-        out = np.zeros(4, np.uint32)
+        out = np.zeros(6, np.uint32)
         _check("phast_schedule", _lib.phast_schedule(self._h, k, out.ctypes.data))
         return dict(fused=bool(out[0]), top_levels=int(out[1]), top_vertices=int(out[2]),
-                    level_launches=int(out[3]))
+                    level_launches=int(out[3]), band_launches=int(out[4]), band_levels=int(out[5]))
 
     def timing(self, enable: bool):
         _check("phast_timing", _lib.phast_timing(self._h, 1 if enable else 0))
@@ -423,6 +429,21 @@ class Phast:
         a["up_head"] = a["up_head"][:inf.m_up]
         a["up_len"] = a["up_len"][:inf.m_up]
         return a
+
+    def bands(self) -> list:
+        """The layout's bands (phast_bands / phast_band_groups): per band, top-most first,
+        dict(seg_lo, seg_hi, ngroups, goff [seg_hi - seg_lo, ngroups + 1] internal ids)."""
+        cnt = ctypes.c_uint32()
+        _check("phast_bands", _lib.phast_bands(self._h, ctypes.byref(cnt), None))
+        desc = np.zeros(3 * max(cnt.value, 1), np.uint32)
+        _check("phast_bands", _lib.phast_bands(self._h, ctypes.byref(cnt), desc.ctypes.data))
+        out = []
+        for b in range(cnt.value):
+            lo, hi, ng = (int(x) for x in desc[3 * b:3 * b + 3])
+            goff = np.zeros((hi - lo) * (ng + 1), np.uint32)
+            _check("phast_band_groups", _lib.phast_band_groups(self._h, b, goff.ctypes.data))
+            out.append(dict(seg_lo=lo, seg_hi=hi, ngroups=ng, goff=goff.reshape(hi - lo, ng + 1)))
+        return out
 
     def to_original(self, rows: np.ndarray) -> np.ndarray:
         """[n, k] internal-order labels (any 32-bit dtype) -> [k, n] uint32 in original ids."""

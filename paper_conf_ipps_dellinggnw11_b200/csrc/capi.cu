@@ -31,7 +31,7 @@ struct phast_ctx {
     double build_seconds = 0;
     Layout L;
     std::vector<uint8_t> wide;          // per level (top-down): the two-record ELL format (DevImage::dn_rec2)
-    phast_query_opts q = {0, 0, 0, 0};
+    phast_query_opts q = {0, 0, 0, 0, 0, 0, 0};
     // upward-search-space statistics of phast_info (host sample, computed once)
     mutable bool up_stats = false;
     mutable double up_mean = 0;
@@ -88,6 +88,13 @@ struct phast_ctx {
         uint2* up_a = nullptr;
     };
     std::map<uint32_t, Top> tops;
+    // band launches (layout.h Band) per k: work units of consecutive closed groups
+    struct BandRun {
+        uint32_t* off = nullptr;   // device [F][U+1]
+        BandArgs a;
+        uint32_t seg_lo = 0, seg_hi = 0;
+    };
+    std::map<uint32_t, std::vector<BandRun>> bandruns;
     // A-up in-arcs by head {tail, len}, all of them (hierarchy parents; uploaded on first use)
     uint32_t* d_upall_first = nullptr;
     uint2* d_upall_arc = nullptr;
@@ -163,6 +170,9 @@ void free_tops(phast_ctx* h) {
         cudaFree(kv.second.up_a);
     }
     h->tops.clear();
+    for (auto& kv : h->bandruns)
+        for (auto& b : kv.second) cudaFree(b.off);
+    h->bandruns.clear();
 }
 
 void free_seeds(phast_ctx* h) {
@@ -275,7 +285,7 @@ int upload(phast_ctx* h) {
     }
     g.dn_first = dnf; g.dn_arc = dna; g.up_first = upf; g.up_arc = upa;
     for (uint32_t s = 0; s < SLOTS; s++)
-        if ((rc = dmalloc(&h->slot[s].flags, nw)) || (rc = dmalloc(&h->slot[s].seed_cnt, KMAX))) {
+        if ((rc = dmalloc(&h->slot[s].flags, nw + 4)) || (rc = dmalloc(&h->slot[s].seed_cnt, KMAX))) {
             free_device(h);
             return rc;
         }
@@ -354,7 +364,7 @@ int upload(phast_ctx* h) {
               cudaStreamCreateWithFlags(&h->side, cudaStreamNonBlocking) == cudaSuccess &&
               cudaEventCreateWithFlags(&h->fork_ev, cudaEventDisableTiming) == cudaSuccess;
     for (uint32_t s = 0; ok && s < SLOTS; s++)
-        ok = cudaMemset(h->slot[s].flags, 0, nw * 4) == cudaSuccess &&
+        ok = cudaMemset(h->slot[s].flags, 0, (nw + 4) * 4) == cudaSuccess &&
              cudaMemset(h->slot[s].seed_cnt, 0, KMAX * 4) == cudaSuccess &&
              cudaEventCreateWithFlags(&h->up_done[s], cudaEventDisableTiming) == cudaSuccess &&
              cudaEventCreateWithFlags(&h->slot_free[s], cudaEventDisableTiming) == cudaSuccess &&
@@ -629,6 +639,62 @@ phast_ctx::Top* get_top(phast_ctx* h, uint32_t k) {
     return &T;
 }
 
+// Band launches for k (layout.h Band, sweep.cu band_kernel): each band's closed groups
+// merged into work units of at least `target` vertices (phast_query_opts band_unit,
+// default 8192 / k: 32 KB of rows per unit), fewer when the band has too few vertices
+// to give every resident CTA two units.
+int get_bands(phast_ctx* h, uint32_t k, std::vector<phast_ctx::BandRun>** out) {
+    *out = nullptr;
+    auto it = h->bandruns.find(k);
+    if (it != h->bandruns.end()) { *out = &it->second; return PHAST_OK; }
+    std::vector<phast_ctx::BandRun> runs;
+    const uint32_t threads = h->q.band_threads ? h->q.band_threads : 128u;
+    const uint32_t variant = k >= 16 ? h->q.band_variant : 0u;   // variants are built for k >= 16
+    const uint64_t resident = (uint64_t)num_sms() * band_sm_threads(variant, threads) / threads;
+    int rc = PHAST_OK;
+    for (const Band& B : h->L.bands) {
+        const uint32_t F = B.seg_hi - B.seg_lo, NG = B.ngroups;
+        const uint64_t total = h->L.lvl_off[B.seg_hi] - h->L.lvl_off[B.seg_lo];
+        uint64_t target = h->q.band_unit ? h->q.band_unit : std::max<uint32_t>(BAND_GROUP_MIN, 8192 / k);
+        target = std::min<uint64_t>(target, std::max<uint64_t>(BAND_GROUP_MIN, total / (2 * resident)));
+        std::vector<uint32_t> ub{0};
+        uint64_t acc = 0;
+        for (uint32_t g = 0; g < NG; g++) {
+            for (uint32_t j = 0; j < F; j++) acc += B.goff[(size_t)j * (NG + 1) + g + 1] - B.goff[(size_t)j * (NG + 1) + g];
+            if (acc >= target || g + 1 == NG) { ub.push_back(g + 1); acc = 0; }
+        }
+        const uint32_t U = (uint32_t)ub.size() - 1;
+        std::vector<uint32_t> off((size_t)F * (U + 1));
+        for (uint32_t j = 0; j < F; j++)
+            for (uint32_t u = 0; u <= U; u++) off[(size_t)j * (U + 1) + u] = B.goff[(size_t)j * (NG + 1) + ub[u]];
+        phast_ctx::BandRun r;
+        if ((rc = dmalloc(&r.off, off.size()))) break;
+        runs.push_back(r);
+        if (cudaMemcpy(runs.back().off, off.data(), off.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess) {
+            cudaGetLastError();
+            rc = PHAST_ECUDA;
+            break;
+        }
+        phast_ctx::BandRun& b = runs.back();
+        b.seg_lo = B.seg_lo;
+        b.seg_hi = B.seg_hi;
+        b.a.off = b.off;
+        b.a.F = F;
+        b.a.U = U;
+        b.a.threads = threads;
+        b.a.variant = variant;
+        for (uint32_t j = 0; j < F && j < 32; j++) b.a.wide |= (h->wide[B.seg_lo + j] ? 1u : 0u) << j;
+    }
+    if (rc) {
+        for (auto& b : runs) cudaFree(b.off);
+        return rc;
+    }
+    auto& slot = h->bandruns[k];
+    slot = std::move(runs);
+    *out = &slot;
+    return PHAST_OK;
+}
+
 constexpr size_t MAX_TIMED_BATCHES = 16384;
 
 cudaEvent_t timing_event(phast_ctx* h) {
@@ -687,12 +753,31 @@ int run_query(phast_ctx* h, const Sources& S, uint32_t kp, const QueryOut& o, cu
         if (launch_sweep_top(top->a, kp, S, o.dist, sl.flags, o.diam, st) != cudaSuccess) return PHAST_ECUDA;
         j0 = top->J;
     }
-    for (uint32_t j = j0; j < levels; j++) {
+    // then every band below the top launch in one launch each (a band that reaches into
+    // the top launch's levels is swept per level), every other level in its own launch
+    std::vector<phast_ctx::BandRun>* bands = nullptr;
+    if (!o.nogather && !(h->q.flags & PHAST_Q_NO_BANDS) && !h->L.bands.empty()) {
+        const int rc = get_bands(h, kp, &bands);
+        if (rc) return rc;
+    }
+    size_t bi = 0;
+    for (uint32_t j = j0; j < levels;) {
+        while (bands && bi < bands->size() && (*bands)[bi].seg_lo < j) bi++;
+        if (bands && bi < bands->size() && (*bands)[bi].seg_lo == j) {
+            const phast_ctx::BandRun& b = (*bands)[bi++];
+            BandArgs a = b.a;
+            a.store_last = !(o.diam && b.seg_hi == levels);   // level-0 rows are never read again
+            a.stream_last = b.seg_hi == levels;
+            if (launch_sweep_band(h->g, a, sl.flags, kp, o.dist, o.diam, st) != cudaSuccess) return PHAST_ECUDA;
+            j = b.seg_hi;
+            continue;
+        }
         const bool last = (j + 1 == levels);
         const bool store = !(o.diam && last);   // level-0 rows are never read again (diameter mode)
         if (launch_sweep_level(h->g, sl.flags, kp, h->L.lvl_off[j], h->L.lvl_off[j + 1], o.dist, o.diam, store, last,
                                o.nogather, h->wide[j] != 0, st) != cudaSuccess)
             return PHAST_ECUDA;
+        j++;
     }
     if (launch_clear_flags(sl, kp, h->g.seed_cap, st) != cudaSuccess) return PHAST_ECUDA;
     if (o.compact_to && launch_compact(o.dist, kp, o.compact_to, o.kc, h->n, st) != cudaSuccess) return PHAST_ECUDA;
@@ -852,7 +937,8 @@ int phast_build(uint32_t n, const uint64_t* first, const uint32_t* head, const u
     int rc = validate_csr(n, first, head, len);
     if (rc) return rc;
     const uint32_t flags = opts ? opts->flags : 0u;
-    if (flags & ~(PHAST_FLAG_HOST_ONLY | PHAST_FLAG_LEVEL_LAYOUT | PHAST_FLAG_BFS_IN_LEVEL)) return PHAST_EINVAL;
+    if (flags & ~(PHAST_FLAG_HOST_ONLY | PHAST_FLAG_LEVEL_LAYOUT | PHAST_FLAG_BFS_IN_LEVEL | PHAST_FLAG_NO_BANDS))
+        return PHAST_EINVAL;
     std::unique_ptr<phast_ctx> h(new (std::nothrow) phast_ctx());
     if (!h) return PHAST_ENOMEM;
     try {
@@ -865,7 +951,8 @@ int phast_build(uint32_t n, const uint64_t* first, const uint32_t* head, const u
         h->rounds = R.rounds;
         const uint32_t mode = ((flags & PHAST_FLAG_LEVEL_LAYOUT) && !(flags & PHAST_FLAG_BFS_IN_LEVEL))
                                   ? LAYOUT_LEVELS
-                                  : LAYOUT_LEVELS_BFS;
+                              : (flags & PHAST_FLAG_NO_BANDS) ? LAYOUT_LEVELS_BFS
+                                                              : LAYOUT_LEVELS_BANDS;
         rc = layout_build(R, first, head, mode, h->L);
         h->build_seconds = R.seconds;
         if (rc) return rc;
@@ -886,8 +973,11 @@ int phast_build(uint32_t n, const uint64_t* first, const uint32_t* head, const u
 int phast_configure(phast_ctx* h, const phast_query_opts* q) {
     int rc = check_handle(h);
     if (rc) return rc;
-    phast_query_opts nq = q ? *q : phast_query_opts{0, 0, 0, 0};
-    const uint32_t known = PHAST_Q_NO_FUSED | PHAST_Q_NO_TOP | PHAST_Q_HYBRID_ON | PHAST_Q_HYBRID_OFF | PHAST_Q_NO_MULTI;
+    phast_query_opts nq = q ? *q : phast_query_opts{0, 0, 0, 0, 0, 0, 0};
+    if (nq.band_threads && nq.band_threads != 128 && nq.band_threads != 256) return PHAST_EINVAL;
+    if (!(nq.band_variant <= 5 || nq.band_variant == 16)) return PHAST_EINVAL;
+    const uint32_t known = PHAST_Q_NO_FUSED | PHAST_Q_NO_TOP | PHAST_Q_HYBRID_ON | PHAST_Q_HYBRID_OFF | PHAST_Q_NO_MULTI |
+                           PHAST_Q_NO_BANDS;
     if ((nq.flags & ~known) || ((nq.flags & PHAST_Q_HYBRID_ON) && (nq.flags & PHAST_Q_HYBRID_OFF)))
         return PHAST_EINVAL;
     DeviceGuard dg(h->device);
@@ -1332,23 +1422,58 @@ int phast_export(const phast_ctx* h, uint32_t* level, uint32_t* dn_first, uint32
     return PHAST_OK;
 }
 
+int phast_bands(const phast_ctx* h, uint32_t* count, uint32_t* desc) {
+    if (!h || !count) return PHAST_EINVAL;
+    *count = (uint32_t)h->L.bands.size();
+    if (desc)
+        for (size_t b = 0; b < h->L.bands.size(); b++) {
+            desc[3 * b] = h->L.bands[b].seg_lo;
+            desc[3 * b + 1] = h->L.bands[b].seg_hi;
+            desc[3 * b + 2] = h->L.bands[b].ngroups;
+        }
+    return PHAST_OK;
+}
+
+int phast_band_groups(const phast_ctx* h, uint32_t b, uint32_t* goff) {
+    if (!h || !goff || b >= h->L.bands.size()) return PHAST_EINVAL;
+    const auto& g = h->L.bands[b].goff;
+    std::memcpy(goff, g.data(), g.size() * 4);
+    return PHAST_OK;
+}
+
 int phast_schedule(phast_ctx* h, uint32_t k, uint32_t* out) {
     int rc = check_handle(h);
     if (rc) return rc;
     if (!out || !k_valid(k)) return PHAST_EINVAL;
     DeviceGuard dg(h->device);
     if (!dg.ok) return PHAST_ECUDA;
-    const phast_ctx::Top* t = get_top(h, kpad(k));
+    const uint32_t kp = kpad(k);
+    const phast_ctx::Top* t = get_top(h, kp);
     const uint32_t levels = (uint32_t)h->L.lvl_off.size() - 1;
+    for (int i = 0; i < 6; i++) out[i] = 0;
     out[0] = t && t->a.fused ? 1u : 0u;
     out[1] = t ? t->J : 0u;
     out[2] = t ? t->a.V : 0u;
-    out[3] = t && t->a.fused ? 0u : levels - (t ? t->J : 0u);
+    if (out[0]) return PHAST_OK;
+    std::vector<phast_ctx::BandRun>* bands = nullptr;   // the walk of run_query
+    if (!(h->q.flags & PHAST_Q_NO_BANDS) && !h->L.bands.empty() && (rc = get_bands(h, kp, &bands))) return rc;
+    size_t bi = 0;
+    for (uint32_t j = t ? t->J : 0u; j < levels;) {
+        while (bands && bi < bands->size() && (*bands)[bi].seg_lo < j) bi++;
+        if (bands && bi < bands->size() && (*bands)[bi].seg_lo == j) {
+            out[4]++;
+            out[5] += (*bands)[bi].seg_hi - j;
+            j = (*bands)[bi++].seg_hi;
+        } else {
+            out[3]++;
+            j++;
+        }
+    }
     return PHAST_OK;
 }
 
 // ---------------------------------------------------------------- save / load
-static const char MAGIC[8] = {'P', 'H', 'A', 'S', 'T', 'B', '2', '4'};
+static const char MAGIC[8] = {'P', 'H', 'A', 'S', 'T', 'B', '2', '5'};
 
 int phast_save(const phast_ctx* h, const char* path) {
     if (!h || !path) return PHAST_EINVAL;
@@ -1364,6 +1489,12 @@ int phast_save(const phast_ctx* h, const char* path) {
               wr(L.dn_arc.data(), 8, L.dn_arc.size()) && wr(L.up_arc.data(), 8, L.up_arc.size());
     const uint64_t n_in = L.in_arc.size();
     ok = ok && wr(&n_in, 8, 1) && wr(L.in_first.data(), 4, L.in_first.size()) && wr(L.in_arc.data(), 8, n_in);
+    const uint64_t nb = L.bands.size();
+    ok = ok && wr(&nb, 8, 1);
+    for (const Band& B : L.bands) {
+        const uint32_t bh[3] = {B.seg_lo, B.seg_hi, B.ngroups};
+        ok = ok && wr(bh, 4, 3) && wr(B.goff.data(), 4, B.goff.size());
+    }
     ok = (std::fclose(f) == 0) && ok;
     return ok ? PHAST_OK : PHAST_EIO;
 }
@@ -1380,7 +1511,8 @@ int phast_load(const char* path, uint32_t flags, phast_ctx** out) {
     auto rd = [&](void* p, size_t sz, size_t cnt) { return std::fread(p, sz, cnt, f) == cnt; };
     bool ok = h && rd(magic, 1, 8) && std::memcmp(magic, MAGIC, 8) == 0 && rd(hdr, 8, 10) &&
               rd(&h->build_seconds, 8, 1) && hdr[0] > 0 && hdr[0] < 0xFFFFFFFFull &&
-              (hdr[7] == LAYOUT_LEVELS || hdr[7] == LAYOUT_LEVELS_BFS) && hdr[9] == hdr[1] + 1;
+              (hdr[7] == LAYOUT_LEVELS || hdr[7] == LAYOUT_LEVELS_BFS || hdr[7] == LAYOUT_LEVELS_BANDS) &&
+              hdr[9] == hdr[1] + 1;
     if (ok) {
         Layout& L = h->L;
         try {
@@ -1411,9 +1543,26 @@ int phast_load(const char* path, uint32_t flags, phast_ctx** out) {
             ok = rd(L.in_first.data(), 4, L.in_first.size()) && rd(L.in_arc.data(), 8, n_in) &&
                  L.in_first[h->n] == n_in;
         }
+        uint64_t nb = 0;
+        ok = ok && rd(&nb, 8, 1) && nb <= L.levels;
+        for (uint64_t b = 0; ok && b < nb; b++) {
+            uint32_t bh[3];
+            ok = rd(bh, 4, 3) && bh[0] < bh[1] && bh[1] <= L.levels && bh[2] <= h->n;
+            if (!ok) break;
+            Band B;
+            B.seg_lo = bh[0]; B.seg_hi = bh[1]; B.ngroups = bh[2];
+            try {
+                B.goff.resize((size_t)(B.seg_hi - B.seg_lo) * (B.ngroups + 1));
+            } catch (const std::bad_alloc&) {
+                std::fclose(f);
+                return PHAST_ENOMEM;
+            }
+            ok = rd(B.goff.data(), 4, B.goff.size());
+            L.bands.push_back(std::move(B));
+        }
     }
     std::fclose(f);
-    if (!ok) return PHAST_EIO;
+    if (!ok || check_bands(h->L) != 0) return PHAST_EIO;
     for (uint32_t v = 0; v < h->n; v++) {
         if (h->L.perm[v] >= h->n) return PHAST_EIO;
         h->L.iperm[h->L.perm[v]] = v;

@@ -67,6 +67,24 @@ cudaError_t launch_seed(const DevImage& g, const Slot& sl, uint32_t k, uint32_t*
 cudaError_t launch_sweep_level(const DevImage& g, const uint32_t* flags, uint32_t k, uint32_t vbeg, uint32_t vend,
                                uint32_t* dist, uint32_t* diam, bool store, bool last_level, bool nogather, bool wide,
                                cudaStream_t st);
+// a3 for a band of levels (layout.h Band) in ONE launch: work unit u (consecutive
+// closed groups) of level j (j = 0 the band's top level) is the id range [off[j*(U+1)
+// + u], off[j*(U+1) + u + 1]); one CTA sweeps a unit level by level (a CTA barrier
+// between levels, none between units: groups share no in-band arcs).  Rows of the
+// unit's upper levels are read back by its lower levels from L2.
+struct BandArgs {
+    const uint32_t* off = nullptr;   // device [F][U+1]
+    uint32_t F = 0, U = 0;
+    uint32_t wide = 0;               // bit j: level j uses the two-record format (DevImage::dn_rec2)
+    uint32_t store_last = 1;         // 0: the band's last level is not stored (diameter mode, CH level 0)
+    uint32_t stream_last = 0;        // 1: the last level's rows are stored evict-first (never read again)
+    uint32_t threads = 128;          // CTA size: 128 or 256
+    uint32_t variant = 0;            // sweep.cu band kernel variants (bits: PF_REG, PF_L2, FULL)
+};
+cudaError_t launch_sweep_band(const DevImage& g, const BandArgs& a, const uint32_t* flags, uint32_t k, uint32_t* dist,
+                              uint32_t* diam, cudaStream_t st);
+// resident threads of the band kernel per SM (its grid is at most num_sms() * this / threads)
+uint32_t band_sm_threads(uint32_t variant, uint32_t threads);
 // after the sweep: clear the visited bits of every search-space vertex ("After
 // scanning v we unmark the vertex", §IV-C).
 cudaError_t launch_clear_flags(const Slot& sl, uint32_t k, uint32_t seed_cap, cudaStream_t st);

@@ -10,8 +10,28 @@ namespace phast {
 
 enum LayoutMode : uint32_t {
     LAYOUT_LEVELS = 1,      // the paper's: level descending, input (DFS) order within a level
-    LAYOUT_LEVELS_BFS = 2,  // level descending, BFS (spatial sweep) order within a level (default)
+    LAYOUT_LEVELS_BFS = 2,  // level descending, BFS (spatial sweep) order within a level
+    LAYOUT_LEVELS_BANDS = 3,  // LEVELS_BFS, with the bottom levels cut into bands of closed groups (default)
 };
+
+// A band: consecutive levels (segments [seg_lo, seg_hi) in processing order) whose
+// vertices are partitioned into GROUPS closed under the band's own G-down arcs: an
+// arc (u, v) with both ends in the band has both ends in one group.  A group only
+// needs rows from above the band and from itself, so groups are independent work
+// (band_kernel, sweep.cu).  Within each level of the band, vertices are sorted by
+// group (then BFS rank), so group g of segment j is the contiguous id range
+// [goff[(j - seg_lo) * (ngroups + 1) + g], goff[... + g + 1]).  Groups are formed from
+// the connected components of the band's arcs in BFS-rank order, each group at least
+// BAND_GROUP_MIN vertices (the last may be smaller).
+struct Band {
+    uint32_t seg_lo = 0, seg_hi = 0, ngroups = 0;
+    std::vector<uint32_t> goff;   // [(seg_hi - seg_lo) * (ngroups + 1)]
+};
+constexpr uint32_t BAND_GROUP_MIN = 32;
+// a band grows upward while its largest component has at most this many vertices
+constexpr uint32_t BAND_COMP_CAP = 1024;
+// ... and has at most this many levels (BandArgs::wide is a 32-bit mask)
+constexpr uint32_t BAND_MAX_LEVELS = 32;
 
 struct Arc {
     uint32_t x, y;          // {tail, len} in G-down; {head, len} in G-up (same bytes as CUDA uint2)
@@ -33,7 +53,13 @@ struct Layout {
     // index per head; self-loops and length-0xFFFFFFFF arcs (never tight) dropped.
     std::vector<uint32_t> in_first;
     std::vector<Arc> in_arc;
+    // LAYOUT_LEVELS_BANDS: the bands, top-most first (their segments are the last ones)
+    std::vector<Band> bands;
 };
+
+// Checks the band invariants of L (group ranges tile each band level in order; every
+// G-down arc inside a band stays inside one group).  Returns 0 or PHAST_EINTERNAL.
+int check_bands(const Layout& L);
 
 // Fills L.in_first / L.in_arc from the input CSR (after layout_build).  Returns 0 or
 // PHAST_ERANGE (more than 2^32-2 kept arcs).

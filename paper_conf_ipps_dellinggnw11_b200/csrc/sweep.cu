@@ -350,6 +350,351 @@ cudaError_t sweep_k(const DevImage& g, const uint32_t* flags, uint32_t vbeg, uin
                 : sweep_kw<K, false>(g, flags, vbeg, vend, dist, diam, store, last, nogather, st);
 }
 
+// ------------------------------------------------------------------ a3 band sweep
+// Band kernel variants (BandArgs::variant; schedule choices, same labels):
+//   bit 0 PF_REG : each thread loads the next item's record while it gathers the
+//                  current item's tail rows (more registers: 1280 threads per SM)
+//   bit 1 PF_L2  : the next unit's records and visited-bit words are bulk-prefetched
+//                  into L2 (cp.async.bulk.prefetch) while this unit is swept
+//   bit 2 L1     : tail rows read through the L1 (band_ld)
+//   16 CHAIN     : sweep_band_chain_kernel (below)
+template <int VAR>
+constexpr int band_sm_threads_of() { return (VAR & 1) ? 1280 : 1536; }
+
+// The static inputs of one (vertex, lane) item of a band level: its ELL record(s) and
+// its visited-bit word.
+struct BandRec {
+    uint4 r, r2;
+    uint32_t fl;
+};
+template <bool WIDE>
+__device__ __forceinline__ BandRec band_rec(const uint4* __restrict__ rec, const uint4* __restrict__ rec2,
+                                            const uint32_t* __restrict__ flags, uint32_t v) {
+    BandRec b;
+    b.r = __ldg(&rec[v]);
+    b.r2 = make_uint4(0u, INF, 0u, INF);
+    if constexpr (WIDE) b.r2 = __ldg(&rec2[v]);
+    b.fl = __ldg(&flags[v >> 5]);
+    return b;
+}
+
+// One (vertex, lane) item of a band level.  Tail rows are read with ld.global.cg: rows
+// of the same work unit were written by this CTA earlier in this launch (visible after
+// the level barrier; the L1 is bypassed), rows from above the band by earlier launches.
+// Row loads of the band kernel: L1 = true reads through the L1 (plain ld.global: the
+// PTX memory model makes rows written by this CTA before the level barrier visible;
+// every row is written once per query and never read before its write in a launch, and
+// the L1 is invalidated at launch boundaries), false bypasses it (ld.global.cg).
+template <bool L1, class T>
+__device__ __forceinline__ T band_ld(const T* p) {
+    if constexpr (L1) return *p;
+    else return __ldcg(p);
+}
+
+template <int K, bool WIDE, bool DIAM, bool L1 = false>
+__device__ __forceinline__ void band_item(const BandRec& b, const uint2* __restrict__ ovf, uint32_t* __restrict__ d,
+                                          uint32_t v, uint32_t lane, bool store, bool stream, uint32_t& mx) {
+    using T = typename RowT<K>::T;
+    const uint4 r = b.r, r2 = b.r2;
+    T acc = inf_row<T>();
+    // the seeded own row: never through the L1 (this item overwrites it)
+    if ((b.fl >> (v & 31)) & 1u) acc = __ldcg(reinterpret_cast<const T*>(d + (size_t)v * K) + lane);
+    const bool more = WIDE ? (r2.w == INF && r2.z != INF) : (r.w == INF && r.z != INF);
+    const uint32_t oi = WIDE ? r2.z : r.z;
+    T x0 = inf_row<T>(), x1 = inf_row<T>(), x2 = inf_row<T>(), x3 = inf_row<T>();
+    if (r.y != INF) x0 = band_ld<L1>(reinterpret_cast<const T*>(d + (size_t)r.x * K) + lane);
+    if (r.w != INF) x1 = band_ld<L1>(reinterpret_cast<const T*>(d + (size_t)r.z * K) + lane);
+    if constexpr (WIDE) {
+        if (r2.y != INF) x2 = band_ld<L1>(reinterpret_cast<const T*>(d + (size_t)r2.x * K) + lane);
+        if (r2.w != INF) x3 = band_ld<L1>(reinterpret_cast<const T*>(d + (size_t)r2.z * K) + lane);
+    }
+    acc = relax(relax(acc, x0, r.y), x1, r.w);
+    if constexpr (WIDE) acc = relax(relax(acc, x2, r2.y), x3, r2.w);
+    if (more) {
+        const uint2* o = ovf + oi;
+        const uint32_t cnt = __ldg(&o->x);
+        for (uint32_t j = 1; j <= cnt; j++) {
+            const uint2 a = __ldg(&o[j]);
+            acc = relax(acc, band_ld<L1>(reinterpret_cast<const T*>(d + (size_t)a.x * K) + lane), a.y);
+        }
+    }
+    if (store) {
+        T* p = reinterpret_cast<T*>(d + (size_t)v * K) + lane;
+        if (stream) __stcs(p, acc); else *p = acc;
+    }
+    if constexpr (DIAM) mx = max(mx, fmax_of(acc));
+}
+
+template <int K, bool WIDE, bool DIAM, int THREADS, bool PF_REG, bool L1>
+__device__ __forceinline__ void band_level(const uint4* __restrict__ rec, const uint4* __restrict__ rec2,
+                                           const uint2* __restrict__ ovf, uint32_t* __restrict__ d,
+                                           const uint32_t* __restrict__ flags, uint32_t vb, uint32_t ve, bool store,
+                                           bool stream, uint32_t& mx) {
+    constexpr uint32_t G = K / RowT<K>::W;
+    const uint32_t total = (ve - vb) * G;
+    uint32_t t = threadIdx.x;
+    if constexpr (PF_REG) {
+        if (t >= total) return;
+        BandRec nx = band_rec<WIDE>(rec, rec2, flags, vb + t / G);
+        for (;;) {
+            const BandRec cur = nx;
+            const uint32_t tn = t + THREADS;
+            if (tn < total) nx = band_rec<WIDE>(rec, rec2, flags, vb + tn / G);
+            band_item<K, WIDE, DIAM, L1>(cur, ovf, d, vb + t / G, t % G, store, stream, mx);
+            if (tn >= total) break;
+            t = tn;
+        }
+    } else {
+        for (; t < total; t += THREADS)
+            band_item<K, WIDE, DIAM, L1>(band_rec<WIDE>(rec, rec2, flags, vb + t / G), ovf, d, vb + t / G, t % G,
+                                         store, stream, mx);
+    }
+}
+
+__device__ __forceinline__ void bulk_prefetch_l2(const void* p, uint32_t bytes) {
+    if (bytes) asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(p), "r"(bytes) : "memory");
+}
+
+// A band of levels in one launch (kernels.h BandArgs; layout.h Band).  Work units are
+// dealt round-robin to a grid of one resident wave, so the units in flight at any time
+// are neighbours in BFS order and share the rows they read from above the band.  The
+// unit's level ranges go to shared memory once per unit (the next unit's are loaded
+// into registers while this one is swept).
+template <int K, bool DIAM, int THREADS, int VAR>
+__global__ void __launch_bounds__(THREADS, band_sm_threads_of<VAR>() / THREADS)
+    sweep_band_kernel(BandArgs a, const uint4* __restrict__ rec, const uint4* __restrict__ rec2,
+                const uint2* __restrict__ ovf, uint32_t* __restrict__ d, const uint32_t* __restrict__ flags,
+                uint32_t* __restrict__ diam) {
+    static_assert(THREADS >= 32, "one warp at least");
+    constexpr bool PF_REG = VAR & 1, PF_L2 = VAR & 2, L1 = VAR & 4;
+    __shared__ uint32_t rng[2][32][2];   // [buffer][level][begin, end]
+    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+    asm volatile("griddepcontrol.wait;" ::: "memory");   // the levels above the band are complete and visible
+    uint32_t mx = 0;
+    const uint32_t U1 = a.U + 1, F = a.F, tid = threadIdx.x;
+    uint32_t nb = 0, ne = 0;   // thread j < F: level j's range of the next unit
+    uint32_t u = blockIdx.x;
+    if (u < a.U && tid < F) { nb = __ldg(&a.off[tid * U1 + u]); ne = __ldg(&a.off[tid * U1 + u + 1]); }
+    for (uint32_t buf = 0; u < a.U; u += gridDim.x, buf ^= 1u) {
+        if (tid < F) { rng[buf][tid][0] = nb; rng[buf][tid][1] = ne; }
+        __syncthreads();   // ranges visible; also orders this unit after the previous one
+        const uint32_t un = u + gridDim.x;
+        if (un < a.U && tid < F) {
+            nb = __ldg(&a.off[tid * U1 + un]);
+            ne = __ldg(&a.off[tid * U1 + un + 1]);
+            if constexpr (PF_L2) {   // the next unit's static inputs into L2
+                bulk_prefetch_l2(rec + nb, (ne - nb) * 16u);
+                if ((a.wide >> tid) & 1u) bulk_prefetch_l2(rec2 + nb, (ne - nb) * 16u);
+                if (ne > nb) {
+                    const uint32_t w0 = (nb >> 5) & ~3u, w1 = (((ne - 1) >> 5) | 3u) + 1u;   // 16-byte aligned
+                    bulk_prefetch_l2(flags + w0, (w1 - w0) * 4u);
+                }
+            }
+        }
+        for (uint32_t j = 0; j < F; j++) {
+            const uint32_t vb = rng[buf][j][0], ve = rng[buf][j][1];
+            const bool last = j + 1 == F;
+            const bool store = !last || a.store_last, stream = last && a.stream_last;
+            if ((a.wide >> j) & 1u)
+                band_level<K, true, DIAM, THREADS, PF_REG, L1>(rec, rec2, ovf, d, flags, vb, ve, store, stream, mx);
+            else
+                band_level<K, false, DIAM, THREADS, PF_REG, L1>(rec, rec2, ovf, d, flags, vb, ve, store, stream, mx);
+            if (!last) __syncthreads();   // level j's rows are written before level j+1 reads them
+        }
+    }
+    if constexpr (DIAM) cta_max_to<THREADS>(mx, diam);
+}
+
+// Chained variant (BandArgs::variant 16): every thread walks its items of a unit level
+// by level and loads the record and visited-bit word of its NEXT item -- the next one
+// in this level, else its first one in a later level of the unit, else its first one
+// in the next unit -- before it gathers the current item's tail rows, so a record
+// round trip is never on the critical path (ncu of the plain band kernel: 42 % of the
+// stall samples waited on a level's first record).  The level ranges of three units
+// are kept in shared memory (this unit, the next one, the one being written).
+constexpr int BAND_CHAIN_SM_THREADS = 1280;
+
+template <int K, bool DIAM, int THREADS>
+__global__ void __launch_bounds__(THREADS, BAND_CHAIN_SM_THREADS / THREADS)
+    sweep_band_chain_kernel(BandArgs a, const uint4* __restrict__ rec, const uint4* __restrict__ rec2,
+                            const uint2* __restrict__ ovf, uint32_t* __restrict__ d,
+                            const uint32_t* __restrict__ flags, uint32_t* __restrict__ diam) {
+    constexpr uint32_t G = K / RowT<K>::W;
+    __shared__ uint32_t rng[3][32][2];   // [unit mod 3][level][begin, end]
+    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+    asm volatile("griddepcontrol.wait;" ::: "memory");   // the levels above the band are complete and visible
+    uint32_t mx = 0;
+    const uint32_t U1 = a.U + 1, F = a.F, tid = threadIdx.x, gs = gridDim.x;
+    uint32_t u = blockIdx.x;
+    auto load_rng = [&](uint32_t uu, uint32_t& b, uint32_t& e) {
+        b = e = 0;
+        if (uu < a.U) { b = __ldg(&a.off[tid * U1 + uu]); e = __ldg(&a.off[tid * U1 + uu + 1]); }
+    };
+    uint32_t nb = 0, ne = 0;
+    if (tid < F) {
+        uint32_t b, e;
+        load_rng(u, b, e);      rng[0][tid][0] = b; rng[0][tid][1] = e;
+        load_rng(u + gs, b, e); rng[1][tid][0] = b; rng[1][tid][1] = e;
+        load_rng(u + 2 * gs, nb, ne);
+    }
+    __syncthreads();
+    // the thread's first item at or after (level j, item t) of the unit in rng[i]; j = F: none
+    auto seek = [&](uint32_t i, uint32_t& j, uint32_t& t) {
+        while (j < F && t >= (rng[i][j][1] - rng[i][j][0]) * G) { j++; t = tid; }
+    };
+    auto fetch = [&](uint32_t i, uint32_t j, uint32_t t) {
+        const uint32_t v = rng[i][j][0] + t / G;
+        return ((a.wide >> j) & 1u) ? band_rec<true>(rec, rec2, flags, v) : band_rec<false>(rec, rec2, flags, v);
+    };
+    uint32_t i = 0, j = 0, t = tid;
+    BandRec nx;
+    bool have = false;
+    if (u < a.U) {
+        seek(0, j, t);
+        if (j < F) { nx = fetch(0, j, t); have = true; }
+    }
+    for (; u < a.U; u += gs) {
+        const uint32_t inext = i == 2 ? 0u : i + 1;
+        for (uint32_t lj = 0; lj < F; lj++) {
+            const bool last = lj + 1 == F;
+            const bool store = !last || a.store_last, stream = last && a.stream_last;
+            const bool wide = (a.wide >> lj) & 1u;
+            const uint32_t vb = rng[i][lj][0];
+            while (have && j == lj) {
+                const BandRec cur = nx;
+                const uint32_t cv = vb + t / G, cl = t % G;
+                t += THREADS;
+                seek(i, j, t);
+                have = false;
+                if (j < F) {
+                    nx = fetch(i, j, t);
+                    have = true;
+                } else if (lj >= 1 && u + gs < a.U) {   // the next unit's ranges are visible after level 0's barrier
+                    uint32_t jn = 0, tn = tid;
+                    seek(inext, jn, tn);
+                    if (jn < F) { nx = fetch(inext, jn, tn); have = true; j = F + 1 + jn; t = tn; }
+                }
+                if (wide) band_item<K, true, DIAM>(cur, ovf, d, cv, cl, store, stream, mx);
+                else band_item<K, false, DIAM>(cur, ovf, d, cv, cl, store, stream, mx);
+            }
+            if (!last) __syncthreads();   // level lj's rows are written before level lj+1 reads them
+        }
+        // unit u + 2 gs goes to the buffer the previous unit used (free since its last barrier);
+        // it is read (cross-unit prefetch) only after the next unit's level-0 barrier
+        __syncthreads();
+        const uint32_t iw = i == 0 ? 2u : i - 1u;
+        if (tid < F) {
+            rng[iw][tid][0] = nb; rng[iw][tid][1] = ne;   // unit u + 2 gs
+            load_rng(u + 3 * gs, nb, ne);
+        }
+        i = inext;
+        if (j > F) {   // the first item of this (new) unit was prefetched
+            j -= F + 1;
+        } else {       // no item was left after level 0, or none prefetched yet
+            j = 0; t = tid;
+            have = false;
+            if (u + gs < a.U) {
+                seek(i, j, t);
+                if (j < F) { nx = fetch(i, j, t); have = true; }
+            }
+        }
+    }
+    if constexpr (DIAM) cta_max_to<THREADS>(mx, diam);
+}
+
+template <int K, int THREADS>
+cudaError_t band_chain_kt(const DevImage& g, const BandArgs& a, const uint32_t* flags, uint32_t* dist, uint32_t* diam,
+                          cudaStream_t st) {
+    uint64_t blocks = std::min<uint64_t>(a.U, (uint64_t)num_sms() * (BAND_CHAIN_SM_THREADS / THREADS));
+    if (blocks == 0 || a.F == 0) return cudaSuccess;
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3((unsigned)blocks);
+    cfg.blockDim = dim3(THREADS);
+    cfg.stream = st;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    cudaError_t e = diam ? cudaLaunchKernelEx(&cfg, sweep_band_chain_kernel<K, true, THREADS>, a, g.dn_rec, g.dn_rec2,
+                                              g.dn_ovf, dist, flags, diam)
+                         : cudaLaunchKernelEx(&cfg, sweep_band_chain_kernel<K, false, THREADS>, a, g.dn_rec, g.dn_rec2,
+                                              g.dn_ovf, dist, flags, diam);
+    count_launch();
+    return e;
+}
+
+// the band kernels use < 1 KB of shared memory: give the rest of the SM's 256 KB to the L1
+cudaError_t prefer_l1(const void* kern) {
+    static std::mutex mu;
+    static std::set<std::pair<const void*, int>> done;
+    int dev = 0;
+    cudaError_t e = cudaGetDevice(&dev);
+    if (e != cudaSuccess) return e;
+    std::lock_guard<std::mutex> lk(mu);
+    if (done.count({kern, dev})) return cudaSuccess;
+    e = cudaFuncSetAttribute(kern, cudaFuncAttributePreferredSharedMemoryCarveout, 0);
+    if (e == cudaSuccess) done.insert({kern, dev});
+    return e;
+}
+
+template <int K, int THREADS, int VAR>
+cudaError_t band_kt(const DevImage& g, const BandArgs& a, const uint32_t* flags, uint32_t* dist, uint32_t* diam,
+                    cudaStream_t st) {
+    if (VAR & 4) {
+        cudaError_t e = prefer_l1(diam ? (const void*)sweep_band_kernel<K, true, THREADS, VAR>
+                                       : (const void*)sweep_band_kernel<K, false, THREADS, VAR>);
+        if (e != cudaSuccess) return e;
+    }
+    uint64_t blocks = std::min<uint64_t>(a.U, (uint64_t)num_sms() * (band_sm_threads_of<VAR>() / THREADS));
+    if (blocks == 0 || a.F == 0) return cudaSuccess;
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3((unsigned)blocks);
+    cfg.blockDim = dim3(THREADS);
+    cfg.stream = st;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    cudaError_t e = diam ? cudaLaunchKernelEx(&cfg, sweep_band_kernel<K, true, THREADS, VAR>, a, g.dn_rec, g.dn_rec2,
+                                              g.dn_ovf, dist, flags, diam)
+                         : cudaLaunchKernelEx(&cfg, sweep_band_kernel<K, false, THREADS, VAR>, a, g.dn_rec, g.dn_rec2,
+                                              g.dn_ovf, dist, flags, diam);
+    count_launch();
+    return e;
+}
+
+template <int K, int VAR>
+cudaError_t band_kv(const DevImage& g, const BandArgs& a, const uint32_t* flags, uint32_t* dist, uint32_t* diam,
+                    cudaStream_t st) {
+    switch (a.threads) {
+        case 128: return band_kt<K, 128, VAR>(g, a, flags, dist, diam, st);
+        case 256: return band_kt<K, 256, VAR>(g, a, flags, dist, diam, st);
+        default: return cudaErrorInvalidValue;
+    }
+}
+
+template <int K>
+cudaError_t band_k(const DevImage& g, const BandArgs& a, const uint32_t* flags, uint32_t* dist, uint32_t* diam,
+                   cudaStream_t st) {
+    if constexpr (K < 16) {
+        return a.variant == 0 ? band_kv<K, 0>(g, a, flags, dist, diam, st) : cudaErrorInvalidValue;
+    } else {
+        switch (a.variant) {
+            case 0: return band_kv<K, 0>(g, a, flags, dist, diam, st);
+            case 1: return band_kv<K, 1>(g, a, flags, dist, diam, st);
+            case 2: return band_kv<K, 2>(g, a, flags, dist, diam, st);
+            case 3: return band_kv<K, 3>(g, a, flags, dist, diam, st);
+            case 4: return band_kv<K, 4>(g, a, flags, dist, diam, st);
+            case 5: return band_kv<K, 5>(g, a, flags, dist, diam, st);
+            case 16: return a.threads == 256 ? band_chain_kt<K, 256>(g, a, flags, dist, diam, st)
+                                             : band_chain_kt<K, 128>(g, a, flags, dist, diam, st);
+            default: return cudaErrorInvalidValue;
+        }
+    }
+}
+
 // ------------------------------------------------------------------ probe A33
 // Sequential stream over the sweep's arrays: every ELL record read, every label row
 // read and written once (no gathers, no level dependencies, ONE launch).
@@ -461,6 +806,17 @@ cudaError_t launch_sweep_level(const DevImage& g, const uint32_t* flags, uint32_
 #define CALL_SW(K) sweep_k<K>(g, flags, vbeg, vend, dist, diam, store, last_level, nogather, wide, st)
     PHAST_K_SWITCH(k, CALL_SW)
 #undef CALL_SW
+}
+
+cudaError_t launch_sweep_band(const DevImage& g, const BandArgs& a, const uint32_t* flags, uint32_t k, uint32_t* dist,
+                              uint32_t* diam, cudaStream_t st) {
+#define CALL_BD(K) band_k<K>(g, a, flags, dist, diam, st)
+    PHAST_K_SWITCH(k, CALL_BD)
+#undef CALL_BD
+}
+
+uint32_t band_sm_threads(uint32_t variant, uint32_t) {
+    return variant == 16 ? (uint32_t)BAND_CHAIN_SM_THREADS : variant & 1 ? 1280u : 1536u;
 }
 
 cudaError_t launch_clear_flags(const Slot& sl, uint32_t k, uint32_t seed_cap, cudaStream_t st) {

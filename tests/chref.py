@@ -48,10 +48,28 @@ def sweep(ex, d_init, n):
     return np.where(d >= INF, INF, d).astype(np.uint32)
 
 
-def phast_cpu(h, ex, sources):
+def sweep_in_order(ex, d_init, order):
+    """The same relaxation, one vertex at a time in the given processing order (which
+    must see every tail before its head)."""
+    d = [int(x) for x in d_init]
+    df = ex["dn_first"].tolist()
+    dt, dl = ex["dn_tail"].tolist(), ex["dn_len"].tolist()
+    for v in order.tolist():
+        best = d[v]
+        for e in range(df[v], df[v + 1]):
+            c = d[dt[e]] + dl[e]
+            if c < best:
+                best = c
+        d[v] = best
+    d = np.array(d, dtype=np.int64)
+    return np.where(d >= INF, INF, d).astype(np.uint32)
+
+
+def phast_cpu(h, ex, sources, order=None):
     perm = h.order()
     out = []
     for s in sources:
-        d = sweep(ex, upward_labels(ex, int(perm[s]), h.n), h.n)
+        up = upward_labels(ex, int(perm[s]), h.n)
+        d = sweep(ex, up, h.n) if order is None else sweep_in_order(ex, up, order)
         out.append(d[perm])
     return np.array(out, dtype=np.uint32)

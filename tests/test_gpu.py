@@ -166,10 +166,18 @@ SCHEDULES = {
     "top_40": dict(flags=P.Q_NO_FUSED, top_max_vertices=40),    # the prefix ends inside the hierarchy
     "top_700": dict(flags=P.Q_NO_FUSED, top_max_vertices=700),
     "top_3000_hybrid": dict(flags=P.Q_NO_FUSED | P.Q_HYBRID_ON, top_max_vertices=3000),
+    "no_bands": dict(flags=P.Q_NO_FUSED | P.Q_NO_BANDS),        # band levels one launch per level
+    "bands_unit_32": dict(flags=P.Q_NO_FUSED, band_unit=32),   # one closed group per work unit
+    "bands_unit_big": dict(flags=P.Q_NO_FUSED | P.Q_NO_TOP, band_unit=1 << 20),   # few units, no top launch
+    "bands_v3_256": dict(flags=P.Q_NO_FUSED, band_variant=3, band_threads=256),   # register + L2 prefetch
+    "bands_chain": dict(flags=P.Q_NO_FUSED, band_variant=16),                    # records prefetched across levels
+    "bands_l1": dict(flags=P.Q_NO_FUSED, band_variant=4),                        # tail rows through the L1
+    "bands_l1_pf": dict(flags=P.Q_NO_FUSED | P.Q_NO_TOP, band_variant=5, band_threads=256),
+    "bands_chain_256": dict(flags=P.Q_NO_FUSED | P.Q_NO_TOP, band_variant=16, band_threads=256, band_unit=64),
 }
 
 
-@pytest.mark.parametrize("layout", ["levels-bfs", "levels"])
+@pytest.mark.parametrize("layout", ["levels-bands", "levels-bfs", "levels"])
 @pytest.mark.parametrize("sched", sorted(SCHEDULES))
 def test_schedules(layout, sched):
     """Every launch schedule (phast_configure) on both vertex orders is bit-exact:
@@ -188,8 +196,9 @@ def test_schedules(layout, sched):
 
 
 def test_schedule_reports_launch_shape():
-    """phast_schedule: C1 at k <= 4 is one fused launch; a road graph gets a top launch
-    plus per-level launches; NO_TOP gives one launch per level."""
+    """phast_schedule: C1 at k <= 4 is one fused launch; a road graph gets a top launch,
+    band launches for the bottom levels and per-level launches between; NO_TOP|NO_BANDS
+    gives one launch per level."""
     g = phastgen.CONFIGS["C1"]["graph"]()
     with P.Phast.from_graph(g) as h:
         s = h.schedule(1)
@@ -197,9 +206,15 @@ def test_schedule_reports_launch_shape():
     g = phastgen.road(120_000, seed=33)
     with P.Phast.from_graph(g) as h:
         s = h.schedule(64)
-        assert not s["fused"] and s["top_levels"] >= 2 and s["top_levels"] + s["level_launches"] == h.levels
+        assert not s["fused"] and s["top_levels"] >= 2 and s["band_launches"] >= 1
+        assert s["top_levels"] + s["level_launches"] + s["band_levels"] == h.levels
+        h.configure(flags=P.Q_NO_TOP | P.Q_NO_FUSED | P.Q_NO_BANDS)
+        assert h.schedule(64) == dict(fused=False, top_levels=0, top_vertices=0, level_launches=h.levels,
+                                      band_launches=0, band_levels=0)
         h.configure(flags=P.Q_NO_TOP | P.Q_NO_FUSED)
-        assert h.schedule(64) == dict(fused=False, top_levels=0, top_vertices=0, level_launches=h.levels)
+        s = h.schedule(64)
+        assert s["band_levels"] == sum(b["seg_hi"] - b["seg_lo"] for b in h.bands())
+        assert s["band_launches"] == len(h.bands()) and s["level_launches"] + s["band_levels"] == h.levels
 
 
 def test_fused_query_edge_cases():

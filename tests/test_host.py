@@ -65,7 +65,7 @@ def test_host_hierarchy_sweep_equals_oracle(name):
     assert np.array_equal(got, want)
 
 
-LAYOUTS = {name: dict(layout=name) for name in ("levels", "levels-bfs")}
+LAYOUTS = {name: dict(layout=name) for name in ("levels", "levels-bfs", "levels-bands")}
 
 
 @pytest.mark.parametrize("layout", sorted(LAYOUTS))
@@ -92,7 +92,7 @@ def test_layout_invariants(name, layout):
     assert np.array_equal(np.sort(perm), np.arange(n, dtype=np.uint32))
     # level-0 vertices are never tails (their rows need not be stored in diameter mode)
     assert np.all(lev[tails] > 0)
-    assert h.info().layout == {"levels": 1, "levels-bfs": 2}[layout]
+    assert h.info().layout == {"levels": 1, "levels-bfs": 2, "levels-bands": 3}[layout]
     assert np.all(np.diff(lev) <= 0)                     # levels contiguous, highest first
     if layout == "levels":
         inv = np.empty_like(perm)
@@ -110,6 +110,87 @@ def test_every_layout_sweep_equals_oracle(layout):
     h = P.Phast.from_graph(g, host_only=True, **LAYOUTS[layout])
     src = phastgen.sources(g.n, 5, seed=3)
     assert np.array_equal(chref.phast_cpu(h, h.export(), src), oracle.sssp_many(g, src))
+
+
+def check_bands(h, ex):
+    """The band invariants (layout.h Band), recomputed here from the exported arrays:
+    the bands tile the bottom segments; each band level is tiled by its groups in
+    order; every G-down arc with both ends in a band stays inside one group, so a group
+    needs only rows from above the band and from itself."""
+    n = h.n
+    lev = ex["level"].astype(np.int64)
+    off = np.concatenate([[0], np.cumsum(h.level_sizes()[::-1].astype(np.int64))])   # segment offsets
+    heads = np.repeat(np.arange(n), np.diff(ex["dn_first"].astype(np.int64)))
+    tails = ex["dn_tail"].astype(np.int64)
+    bands = h.bands()
+    nxt = h.levels
+    for b in reversed(bands):
+        assert b["seg_hi"] == nxt and b["seg_hi"] - b["seg_lo"] >= 2
+        nxt = b["seg_lo"]
+        base, end = off[b["seg_lo"]], off[b["seg_hi"]]
+        g_of = np.full(end - base, -1, np.int64)
+        for j in range(b["seg_lo"], b["seg_hi"]):
+            go = b["goff"][j - b["seg_lo"]].astype(np.int64)
+            assert go[0] == off[j] and go[-1] == off[j + 1] and np.all(np.diff(go) >= 0)
+            g_of[go[0] - base:go[-1] - base] = np.repeat(np.arange(b["ngroups"]), np.diff(go))
+        assert np.all(g_of >= 0)
+        inb = (heads >= base) & (heads < end) & (tails >= base)
+        assert np.all(g_of[heads[inb] - base] == g_of[tails[inb] - base])
+        # every band level is one CH level, in processing order
+        assert np.all(lev[base:end] == h.levels - 1 - np.repeat(np.arange(b["seg_lo"], b["seg_hi"]),
+                                                                  np.diff(off[b["seg_lo"]:b["seg_hi"] + 1])))
+    return bands
+
+
+def test_band_layout_groups_are_closed():
+    """Default layout (levels-bands): on road graphs the bottom levels form bands whose
+    groups are closed under the band's own arcs (checked independently of the
+    library's own check), a group sweep order (group by group, levels top-down inside
+    a band) is a reverse topological order, and sweeping in that order gives the
+    oracle's labels."""
+    for g in (phastgen.road(60_000, seed=41), phastgen.road(30_000, seed=42, metric="distance"),
+              phastgen.CONFIGS["C1"]["graph"]()):
+        h = P.Phast.from_graph(g, host_only=True)
+        ex = h.export()
+        bands = check_bands(h, ex)
+        assert bands, "a road graph has at least one band"
+        assert bands[-1]["seg_hi"] == h.levels          # the bottom band holds level 0
+        # the group schedule of band_kernel: above the bands in id order, then each band
+        # group by group, levels top-down inside a group
+        order = [np.arange(0, int(bands[0]["goff"][0, 0]))]
+        for b in bands:
+            go = b["goff"].astype(np.int64)
+            for gi in range(b["ngroups"]):
+                for j in range(go.shape[0]):
+                    order.append(np.arange(go[j, gi], go[j, gi + 1]))
+        order = np.concatenate(order)
+        assert np.array_equal(np.sort(order), np.arange(h.n))
+        pos = np.empty(h.n, np.int64)
+        pos[order] = np.arange(h.n)
+        heads = np.repeat(np.arange(h.n), np.diff(ex["dn_first"].astype(np.int64)))
+        assert np.all(pos[ex["dn_tail"].astype(np.int64)] < pos[heads])
+        src = phastgen.sources(g.n, 3, seed=5)
+        assert np.array_equal(chref.phast_cpu(h, ex, src, order=order), oracle.sssp_many(g, src))
+
+
+def test_band_layout_save_load_roundtrip(tmp_path):
+    g = phastgen.road(20_000, seed=43)
+    h = P.Phast.from_graph(g, host_only=True)
+    p = str(tmp_path / "b.phast")
+    h.save(p)
+    h2 = P.Phast.load(p, host_only=True)
+    b1, b2 = h.bands(), h2.bands()
+    assert len(b1) == len(b2) > 0
+    for x, y in zip(b1, b2):
+        assert (x["seg_lo"], x["seg_hi"], x["ngroups"]) == (y["seg_lo"], y["seg_hi"], y["ngroups"])
+        assert np.array_equal(x["goff"], y["goff"])
+    assert np.array_equal(h.order(), h2.order())
+
+
+def test_no_bands_layouts():
+    g = phastgen.road(20_000, seed=44)
+    for layout in ("levels", "levels-bfs"):
+        assert P.Phast.from_graph(g, host_only=True, layout=layout).bands() == []
 
 
 def test_distance_metric_is_deeper():
