@@ -648,14 +648,16 @@ int get_bands(phast_ctx* h, uint32_t k, std::vector<phast_ctx::BandRun>** out) {
     auto it = h->bandruns.find(k);
     if (it != h->bandruns.end()) { *out = &it->second; return PHAST_OK; }
     std::vector<phast_ctx::BandRun> runs;
-    const uint32_t threads = h->q.band_threads ? h->q.band_threads : 128u;
-    const uint32_t variant = k >= 16 ? h->q.band_variant : 0u;   // variants are built for k >= 16
+    // defaults measured on C3: 256-thread CTAs, variant 5 (records one item
+    // ahead, tail rows through the L1), units of 32768 / k vertices (128 KB of rows)
+    const uint32_t threads = h->q.band_threads ? h->q.band_threads : 256u;
+    const uint32_t variant = k < 16 ? 0u : h->q.band_variant ? h->q.band_variant : 5u;   // variants: k >= 16
     const uint64_t resident = (uint64_t)num_sms() * band_sm_threads(variant, threads) / threads;
     int rc = PHAST_OK;
     for (const Band& B : h->L.bands) {
         const uint32_t F = B.seg_hi - B.seg_lo, NG = B.ngroups;
         const uint64_t total = h->L.lvl_off[B.seg_hi] - h->L.lvl_off[B.seg_lo];
-        uint64_t target = h->q.band_unit ? h->q.band_unit : std::max<uint32_t>(BAND_GROUP_MIN, 8192 / k);
+        uint64_t target = h->q.band_unit ? h->q.band_unit : std::max<uint32_t>(BAND_GROUP_MIN, 32768 / k);
         target = std::min<uint64_t>(target, std::max<uint64_t>(BAND_GROUP_MIN, total / (2 * resident)));
         std::vector<uint32_t> ub{0};
         uint64_t acc = 0;
@@ -974,8 +976,9 @@ int phast_configure(phast_ctx* h, const phast_query_opts* q) {
     int rc = check_handle(h);
     if (rc) return rc;
     phast_query_opts nq = q ? *q : phast_query_opts{0, 0, 0, 0, 0, 0, 0};
-    if (nq.band_threads && nq.band_threads != 128 && nq.band_threads != 256) return PHAST_EINVAL;
-    if (!(nq.band_variant <= 5 || nq.band_variant == 16)) return PHAST_EINVAL;
+    if (nq.band_threads && nq.band_threads != 128 && nq.band_threads != 256 && nq.band_threads != 640)
+        return PHAST_EINVAL;
+    if (!(nq.band_variant <= 5 || nq.band_variant == 7 || nq.band_variant == 16)) return PHAST_EINVAL;
     const uint32_t known = PHAST_Q_NO_FUSED | PHAST_Q_NO_TOP | PHAST_Q_HYBRID_ON | PHAST_Q_HYBRID_OFF | PHAST_Q_NO_MULTI |
                            PHAST_Q_NO_BANDS;
     if ((nq.flags & ~known) || ((nq.flags & PHAST_Q_HYBRID_ON) && (nq.flags & PHAST_Q_HYBRID_OFF)))

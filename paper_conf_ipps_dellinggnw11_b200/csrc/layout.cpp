@@ -99,8 +99,8 @@ struct UnionFind {
 
 // Bands of LAYOUT_LEVELS_BANDS over CH levels (original ids).  Greedy from level 0
 // up: a band [lo, hi) grows while the largest component of its internal G-down arcs
-// has at most BAND_COMP_CAP vertices and it has at most BAND_MAX_LEVELS levels; banding
-// stops at the first band of one level.
+// has at most min(BAND_COMP_CAP, vertices / BAND_COMP_DIV) vertices and it has at most
+// BAND_MAX_LEVELS levels; banding stops at the first band of one level.
 // grp[v] = group of v inside its band (INF outside bands); returns the level ranges.
 std::vector<std::pair<uint32_t, uint32_t>> make_bands(const ChResult& R, uint32_t levels,
                                                       const std::vector<uint32_t>& rank,
@@ -142,9 +142,11 @@ std::vector<std::pair<uint32_t, uint32_t>> make_bands(const ChResult& R, uint32_
     uint32_t lo = 0;
     while (lo + 1 < levels) {
         uint32_t mx = add_level(lo, lo), hi = lo + 1;
+        uint64_t nv = lf[lo + 1] - lf[lo];
         while (hi < levels && hi - lo < BAND_MAX_LEVELS) {
             mx = std::max(mx, add_level(hi, lo));
-            if (mx > BAND_COMP_CAP) break;
+            nv += lf[hi + 1] - lf[hi];
+            if (mx > BAND_COMP_CAP || (uint64_t)mx * BAND_COMP_DIV > nv) break;
             hi++;
         }
         if (hi - lo < 2) break;

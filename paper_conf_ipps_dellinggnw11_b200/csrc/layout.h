@@ -28,8 +28,12 @@ struct Band {
     std::vector<uint32_t> goff;   // [(seg_hi - seg_lo) * (ngroups + 1)]
 };
 constexpr uint32_t BAND_GROUP_MIN = 32;
-// a band grows upward while its largest component has at most this many vertices
+// a band grows upward while its largest component has at most this many vertices and
+// at most 1 / BAND_COMP_DIV of the band's vertices (one component is one CTA's serial
+// work: C3 k = 64, a 942-vertex component in a 2 764-vertex band took 55 us against 24
+// for its four per-level launches)
 constexpr uint32_t BAND_COMP_CAP = 1024;
+constexpr uint32_t BAND_COMP_DIV = 256;
 // ... and has at most this many levels (BandArgs::wide is a 32-bit mask)
 constexpr uint32_t BAND_MAX_LEVELS = 32;
 

@@ -671,6 +671,7 @@ cudaError_t band_kv(const DevImage& g, const BandArgs& a, const uint32_t* flags,
     switch (a.threads) {
         case 128: return band_kt<K, 128, VAR>(g, a, flags, dist, diam, st);
         case 256: return band_kt<K, 256, VAR>(g, a, flags, dist, diam, st);
+        case 640: return band_kt<K, 640, VAR>(g, a, flags, dist, diam, st);
         default: return cudaErrorInvalidValue;
     }
 }
@@ -688,6 +689,7 @@ cudaError_t band_k(const DevImage& g, const BandArgs& a, const uint32_t* flags, 
             case 3: return band_kv<K, 3>(g, a, flags, dist, diam, st);
             case 4: return band_kv<K, 4>(g, a, flags, dist, diam, st);
             case 5: return band_kv<K, 5>(g, a, flags, dist, diam, st);
+            case 7: return band_kv<K, 7>(g, a, flags, dist, diam, st);
             case 16: return a.threads == 256 ? band_chain_kt<K, 256>(g, a, flags, dist, diam, st)
                                              : band_chain_kt<K, 128>(g, a, flags, dist, diam, st);
             default: return cudaErrorInvalidValue;
