@@ -199,6 +199,15 @@ def run_reference(args):
     return 0
 
 
+def try_load(P, path):
+    """A cached hierarchy, or None if the file is stale (another format version) or unreadable."""
+    try:
+        return P.Phast.load(path)
+    except P.PhastError as e:
+        log(f"[bench] cache {path} not loaded ({e}); rebuilding")
+        return None
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -276,8 +285,8 @@ def main():
         t = time.time()
         h = share_hierarchy(lambda: P.Phast.from_graph(g, **bopts), P.Phast.load, path, rank, barrier)
         log(f"[bench] rank {rank}: hierarchy ready in {time.time() - t:.1f}s")
-    elif args.cache and os.path.exists(args.cache):
-        h = P.Phast.load(args.cache)
+    elif args.cache and os.path.exists(args.cache) and (h := try_load(P, args.cache)) is not None:
+        pass
     else:
         t = time.time()
         h = P.Phast.from_graph(g, **bopts)

@@ -976,9 +976,9 @@ int phast_configure(phast_ctx* h, const phast_query_opts* q) {
     int rc = check_handle(h);
     if (rc) return rc;
     phast_query_opts nq = q ? *q : phast_query_opts{0, 0, 0, 0, 0, 0, 0};
-    if (nq.band_threads && nq.band_threads != 128 && nq.band_threads != 256 && nq.band_threads != 640)
+    if (nq.band_threads && nq.band_threads != 128 && nq.band_threads != 256) return PHAST_EINVAL;
+    if (!(nq.band_variant == 0 || nq.band_variant == 1 || nq.band_variant == 4 || nq.band_variant == 5))
         return PHAST_EINVAL;
-    if (!(nq.band_variant <= 5 || nq.band_variant == 7 || nq.band_variant == 16)) return PHAST_EINVAL;
     const uint32_t known = PHAST_Q_NO_FUSED | PHAST_Q_NO_TOP | PHAST_Q_HYBRID_ON | PHAST_Q_HYBRID_OFF | PHAST_Q_NO_MULTI |
                            PHAST_Q_NO_BANDS;
     if ((nq.flags & ~known) || ((nq.flags & PHAST_Q_HYBRID_ON) && (nq.flags & PHAST_Q_HYBRID_OFF)))

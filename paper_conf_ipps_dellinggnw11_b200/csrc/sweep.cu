@@ -351,13 +351,14 @@ cudaError_t sweep_k(const DevImage& g, const uint32_t* flags, uint32_t vbeg, uin
 }
 
 // ------------------------------------------------------------------ a3 band sweep
-// Band kernel variants (BandArgs::variant; schedule choices, same labels):
+// Band kernel variants (BandArgs::variant; schedule choices, same labels).  Measured
+// on C3, the product keeps the ablation of the two that matter:
 //   bit 0 PF_REG : each thread loads the next item's record while it gathers the
-//                  current item's tail rows (more registers: 1280 threads per SM)
-//   bit 1 PF_L2  : the next unit's records and visited-bit words are bulk-prefetched
-//                  into L2 (cp.async.bulk.prefetch) while this unit is swept
-//   bit 2 L1     : tail rows read through the L1 (band_ld)
-//   16 CHAIN     : sweep_band_chain_kernel (below)
+//                  current item's tail rows (48 registers: 1280 threads per SM)
+//   bit 2 L1     : tail rows read through the L1 (band_ld); ~40 % L1 hits
+// 5 = both (the default for k >= 16), 0 = neither (k < 16), 1, 4.  Measured slower and
+// removed: L2 bulk prefetch of the next unit's records, two items per thread in flight,
+// records chained across levels and units, cp.async-staged gathers.
 template <int VAR>
 constexpr int band_sm_threads_of() { return (VAR & 1) ? 1280 : 1536; }
 
@@ -451,10 +452,6 @@ __device__ __forceinline__ void band_level(const uint4* __restrict__ rec, const 
     }
 }
 
-__device__ __forceinline__ void bulk_prefetch_l2(const void* p, uint32_t bytes) {
-    if (bytes) asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(p), "r"(bytes) : "memory");
-}
-
 // A band of levels in one launch (kernels.h BandArgs; layout.h Band).  Work units are
 // dealt round-robin to a grid of one resident wave, so the units in flight at any time
 // are neighbours in BFS order and share the rows they read from above the band.  The
@@ -466,7 +463,7 @@ __global__ void __launch_bounds__(THREADS, band_sm_threads_of<VAR>() / THREADS)
                 const uint2* __restrict__ ovf, uint32_t* __restrict__ d, const uint32_t* __restrict__ flags,
                 uint32_t* __restrict__ diam) {
     static_assert(THREADS >= 32, "one warp at least");
-    constexpr bool PF_REG = VAR & 1, PF_L2 = VAR & 2, L1 = VAR & 4;
+    constexpr bool PF_REG = VAR & 1, L1 = VAR & 4;
     __shared__ uint32_t rng[2][32][2];   // [buffer][level][begin, end]
     asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
     asm volatile("griddepcontrol.wait;" ::: "memory");   // the levels above the band are complete and visible
@@ -479,18 +476,7 @@ __global__ void __launch_bounds__(THREADS, band_sm_threads_of<VAR>() / THREADS)
         if (tid < F) { rng[buf][tid][0] = nb; rng[buf][tid][1] = ne; }
         __syncthreads();   // ranges visible; also orders this unit after the previous one
         const uint32_t un = u + gridDim.x;
-        if (un < a.U && tid < F) {
-            nb = __ldg(&a.off[tid * U1 + un]);
-            ne = __ldg(&a.off[tid * U1 + un + 1]);
-            if constexpr (PF_L2) {   // the next unit's static inputs into L2
-                bulk_prefetch_l2(rec + nb, (ne - nb) * 16u);
-                if ((a.wide >> tid) & 1u) bulk_prefetch_l2(rec2 + nb, (ne - nb) * 16u);
-                if (ne > nb) {
-                    const uint32_t w0 = (nb >> 5) & ~3u, w1 = (((ne - 1) >> 5) | 3u) + 1u;   // 16-byte aligned
-                    bulk_prefetch_l2(flags + w0, (w1 - w0) * 4u);
-                }
-            }
-        }
+        if (un < a.U && tid < F) { nb = __ldg(&a.off[tid * U1 + un]); ne = __ldg(&a.off[tid * U1 + un + 1]); }
         for (uint32_t j = 0; j < F; j++) {
             const uint32_t vb = rng[buf][j][0], ve = rng[buf][j][1];
             const bool last = j + 1 == F;
@@ -503,125 +489,6 @@ __global__ void __launch_bounds__(THREADS, band_sm_threads_of<VAR>() / THREADS)
         }
     }
     if constexpr (DIAM) cta_max_to<THREADS>(mx, diam);
-}
-
-// Chained variant (BandArgs::variant 16): every thread walks its items of a unit level
-// by level and loads the record and visited-bit word of its NEXT item -- the next one
-// in this level, else its first one in a later level of the unit, else its first one
-// in the next unit -- before it gathers the current item's tail rows, so a record
-// round trip is never on the critical path (ncu of the plain band kernel: 42 % of the
-// stall samples waited on a level's first record).  The level ranges of three units
-// are kept in shared memory (this unit, the next one, the one being written).
-constexpr int BAND_CHAIN_SM_THREADS = 1280;
-
-template <int K, bool DIAM, int THREADS>
-__global__ void __launch_bounds__(THREADS, BAND_CHAIN_SM_THREADS / THREADS)
-    sweep_band_chain_kernel(BandArgs a, const uint4* __restrict__ rec, const uint4* __restrict__ rec2,
-                            const uint2* __restrict__ ovf, uint32_t* __restrict__ d,
-                            const uint32_t* __restrict__ flags, uint32_t* __restrict__ diam) {
-    constexpr uint32_t G = K / RowT<K>::W;
-    __shared__ uint32_t rng[3][32][2];   // [unit mod 3][level][begin, end]
-    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
-    asm volatile("griddepcontrol.wait;" ::: "memory");   // the levels above the band are complete and visible
-    uint32_t mx = 0;
-    const uint32_t U1 = a.U + 1, F = a.F, tid = threadIdx.x, gs = gridDim.x;
-    uint32_t u = blockIdx.x;
-    auto load_rng = [&](uint32_t uu, uint32_t& b, uint32_t& e) {
-        b = e = 0;
-        if (uu < a.U) { b = __ldg(&a.off[tid * U1 + uu]); e = __ldg(&a.off[tid * U1 + uu + 1]); }
-    };
-    uint32_t nb = 0, ne = 0;
-    if (tid < F) {
-        uint32_t b, e;
-        load_rng(u, b, e);      rng[0][tid][0] = b; rng[0][tid][1] = e;
-        load_rng(u + gs, b, e); rng[1][tid][0] = b; rng[1][tid][1] = e;
-        load_rng(u + 2 * gs, nb, ne);
-    }
-    __syncthreads();
-    // the thread's first item at or after (level j, item t) of the unit in rng[i]; j = F: none
-    auto seek = [&](uint32_t i, uint32_t& j, uint32_t& t) {
-        while (j < F && t >= (rng[i][j][1] - rng[i][j][0]) * G) { j++; t = tid; }
-    };
-    auto fetch = [&](uint32_t i, uint32_t j, uint32_t t) {
-        const uint32_t v = rng[i][j][0] + t / G;
-        return ((a.wide >> j) & 1u) ? band_rec<true>(rec, rec2, flags, v) : band_rec<false>(rec, rec2, flags, v);
-    };
-    uint32_t i = 0, j = 0, t = tid;
-    BandRec nx;
-    bool have = false;
-    if (u < a.U) {
-        seek(0, j, t);
-        if (j < F) { nx = fetch(0, j, t); have = true; }
-    }
-    for (; u < a.U; u += gs) {
-        const uint32_t inext = i == 2 ? 0u : i + 1;
-        for (uint32_t lj = 0; lj < F; lj++) {
-            const bool last = lj + 1 == F;
-            const bool store = !last || a.store_last, stream = last && a.stream_last;
-            const bool wide = (a.wide >> lj) & 1u;
-            const uint32_t vb = rng[i][lj][0];
-            while (have && j == lj) {
-                const BandRec cur = nx;
-                const uint32_t cv = vb + t / G, cl = t % G;
-                t += THREADS;
-                seek(i, j, t);
-                have = false;
-                if (j < F) {
-                    nx = fetch(i, j, t);
-                    have = true;
-                } else if (lj >= 1 && u + gs < a.U) {   // the next unit's ranges are visible after level 0's barrier
-                    uint32_t jn = 0, tn = tid;
-                    seek(inext, jn, tn);
-                    if (jn < F) { nx = fetch(inext, jn, tn); have = true; j = F + 1 + jn; t = tn; }
-                }
-                if (wide) band_item<K, true, DIAM>(cur, ovf, d, cv, cl, store, stream, mx);
-                else band_item<K, false, DIAM>(cur, ovf, d, cv, cl, store, stream, mx);
-            }
-            if (!last) __syncthreads();   // level lj's rows are written before level lj+1 reads them
-        }
-        // unit u + 2 gs goes to the buffer the previous unit used (free since its last barrier);
-        // it is read (cross-unit prefetch) only after the next unit's level-0 barrier
-        __syncthreads();
-        const uint32_t iw = i == 0 ? 2u : i - 1u;
-        if (tid < F) {
-            rng[iw][tid][0] = nb; rng[iw][tid][1] = ne;   // unit u + 2 gs
-            load_rng(u + 3 * gs, nb, ne);
-        }
-        i = inext;
-        if (j > F) {   // the first item of this (new) unit was prefetched
-            j -= F + 1;
-        } else {       // no item was left after level 0, or none prefetched yet
-            j = 0; t = tid;
-            have = false;
-            if (u + gs < a.U) {
-                seek(i, j, t);
-                if (j < F) { nx = fetch(i, j, t); have = true; }
-            }
-        }
-    }
-    if constexpr (DIAM) cta_max_to<THREADS>(mx, diam);
-}
-
-template <int K, int THREADS>
-cudaError_t band_chain_kt(const DevImage& g, const BandArgs& a, const uint32_t* flags, uint32_t* dist, uint32_t* diam,
-                          cudaStream_t st) {
-    uint64_t blocks = std::min<uint64_t>(a.U, (uint64_t)num_sms() * (BAND_CHAIN_SM_THREADS / THREADS));
-    if (blocks == 0 || a.F == 0) return cudaSuccess;
-    cudaLaunchConfig_t cfg = {};
-    cfg.gridDim = dim3((unsigned)blocks);
-    cfg.blockDim = dim3(THREADS);
-    cfg.stream = st;
-    cudaLaunchAttribute attr[1];
-    attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
-    attr[0].val.programmaticStreamSerializationAllowed = 1;
-    cfg.attrs = attr;
-    cfg.numAttrs = 1;
-    cudaError_t e = diam ? cudaLaunchKernelEx(&cfg, sweep_band_chain_kernel<K, true, THREADS>, a, g.dn_rec, g.dn_rec2,
-                                              g.dn_ovf, dist, flags, diam)
-                         : cudaLaunchKernelEx(&cfg, sweep_band_chain_kernel<K, false, THREADS>, a, g.dn_rec, g.dn_rec2,
-                                              g.dn_ovf, dist, flags, diam);
-    count_launch();
-    return e;
 }
 
 // the band kernels use < 1 KB of shared memory: give the rest of the SM's 256 KB to the L1
@@ -671,7 +538,6 @@ cudaError_t band_kv(const DevImage& g, const BandArgs& a, const uint32_t* flags,
     switch (a.threads) {
         case 128: return band_kt<K, 128, VAR>(g, a, flags, dist, diam, st);
         case 256: return band_kt<K, 256, VAR>(g, a, flags, dist, diam, st);
-        case 640: return band_kt<K, 640, VAR>(g, a, flags, dist, diam, st);
         default: return cudaErrorInvalidValue;
     }
 }
@@ -685,13 +551,8 @@ cudaError_t band_k(const DevImage& g, const BandArgs& a, const uint32_t* flags, 
         switch (a.variant) {
             case 0: return band_kv<K, 0>(g, a, flags, dist, diam, st);
             case 1: return band_kv<K, 1>(g, a, flags, dist, diam, st);
-            case 2: return band_kv<K, 2>(g, a, flags, dist, diam, st);
-            case 3: return band_kv<K, 3>(g, a, flags, dist, diam, st);
             case 4: return band_kv<K, 4>(g, a, flags, dist, diam, st);
             case 5: return band_kv<K, 5>(g, a, flags, dist, diam, st);
-            case 7: return band_kv<K, 7>(g, a, flags, dist, diam, st);
-            case 16: return a.threads == 256 ? band_chain_kt<K, 256>(g, a, flags, dist, diam, st)
-                                             : band_chain_kt<K, 128>(g, a, flags, dist, diam, st);
             default: return cudaErrorInvalidValue;
         }
     }
@@ -818,7 +679,7 @@ cudaError_t launch_sweep_band(const DevImage& g, const BandArgs& a, const uint32
 }
 
 uint32_t band_sm_threads(uint32_t variant, uint32_t) {
-    return variant == 16 ? (uint32_t)BAND_CHAIN_SM_THREADS : variant & 1 ? 1280u : 1536u;
+    return variant & 1 ? 1280u : 1536u;
 }
 
 cudaError_t launch_clear_flags(const Slot& sl, uint32_t k, uint32_t seed_cap, cudaStream_t st) {

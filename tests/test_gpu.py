@@ -169,11 +169,8 @@ SCHEDULES = {
     "no_bands": dict(flags=P.Q_NO_FUSED | P.Q_NO_BANDS),        # band levels one launch per level
     "bands_unit_32": dict(flags=P.Q_NO_FUSED, band_unit=32),   # one closed group per work unit
     "bands_unit_big": dict(flags=P.Q_NO_FUSED | P.Q_NO_TOP, band_unit=1 << 20),   # few units, no top launch
-    "bands_v3_256": dict(flags=P.Q_NO_FUSED, band_variant=3, band_threads=256),   # register + L2 prefetch
-    "bands_chain": dict(flags=P.Q_NO_FUSED, band_variant=16),                    # records prefetched across levels
-    "bands_l1": dict(flags=P.Q_NO_FUSED, band_variant=4),                        # tail rows through the L1
-    "bands_l1_pf": dict(flags=P.Q_NO_FUSED | P.Q_NO_TOP, band_variant=5, band_threads=256),
-    "bands_chain_256": dict(flags=P.Q_NO_FUSED | P.Q_NO_TOP, band_variant=16, band_threads=256, band_unit=64),
+    "bands_v1_256": dict(flags=P.Q_NO_FUSED, band_variant=1, band_threads=256),   # records one item ahead
+    "bands_v4": dict(flags=P.Q_NO_FUSED | P.Q_NO_TOP, band_variant=4, band_threads=128),   # tails through the L1
 }
 
 

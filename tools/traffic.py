@@ -28,7 +28,7 @@ def main(path, key, layout, cache="all"):
     prof[key] = {"dram_bytes_per_sweep": (rd + wr) / n, "dram_read": rd / n, "dram_write": wr / n,
                  "ncu_sweep_s": t / n, "sweeps_averaged": n, "cache_control": cache,
                  "source": f"{os.path.relpath(path)} (ncu launch list, dram__bytes per sweep launch "
-                           f"(sweep_top_kernel + sweep_kernel), summed per sweep, averaged)",
+                           f"(sweep_top_kernel + sweep_band_kernel + sweep_kernel), summed per sweep, averaged)",
                  "layout": layout, "sweep": "levels", "arc_batch": "ell", "top": True}
     json.dump(prof, open(out, "w"), indent=1)
     print(key, prof[key])
