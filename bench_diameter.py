@@ -38,6 +38,8 @@ def main():
     ap.add_argument("--limit", type=int, default=0, help="use only the first N sources (0 = all n)")
     ap.add_argument("--check", type=int, default=1024, help="oracle trees sampled on rank 0 (<= D)")
     ap.add_argument("--no-witness", action="store_true")
+    ap.add_argument("--query-flags", type=int, default=0, help="phast_configure flags (64: no band launches)")
+    ap.add_argument("--band-unit", type=int, default=0, help="vertices per band work unit (0 = library default)")
     args = ap.parse_args()
     if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
         import subprocess
@@ -69,6 +71,8 @@ def main():
                             rank, barrier)
     else:
         h = P.Phast.from_graph(g)
+    if args.query_flags or args.band_unit:
+        h.configure(flags=args.query_flags, band_unit=args.band_unit)
     n = h.n
     count = args.limit or n
     sources = np.arange(count, dtype=np.uint32)

@@ -352,13 +352,16 @@ cudaError_t sweep_k(const DevImage& g, const uint32_t* flags, uint32_t vbeg, uin
 
 // ------------------------------------------------------------------ a3 band sweep
 // Band kernel variants (BandArgs::variant; schedule choices, same labels).  Measured
-// on C3, the product keeps the ablation of the two that matter:
+// on C3 (profiles/r2_band_variants.md), the product keeps the ablation of
+// the two that matter:
 //   bit 0 PF_REG : each thread loads the next item's record while it gathers the
 //                  current item's tail rows (48 registers: 1280 threads per SM)
-//   bit 2 L1     : tail rows read through the L1 (band_ld); ~40 % L1 hits
+//   bit 2 L1     : tail rows read through the L1 (band_ld); 28-42 % L1 hits
 // 5 = both (the default for k >= 16), 0 = neither (k < 16), 1, 4.  Measured slower and
 // removed: L2 bulk prefetch of the next unit's records, two items per thread in flight,
-// records chained across levels and units, cp.async-staged gathers.
+// records chained across levels and units or prefetched across the level barrier, no
+// barrier between units (three range buffers), 1536 / 2048 threads per SM with
+// spills, cp.async-staged gathers.
 template <int VAR>
 constexpr int band_sm_threads_of() { return (VAR & 1) ? 1280 : 1536; }
 
@@ -426,6 +429,8 @@ __device__ __forceinline__ void band_item(const BandRec& b, const uint2* __restr
     if constexpr (DIAM) mx = max(mx, fmax_of(acc));
 }
 
+// One unit level [vb, ve).  PF_REG: the next item's record is loaded before the
+// current item's gathers.
 template <int K, bool WIDE, bool DIAM, int THREADS, bool PF_REG, bool L1>
 __device__ __forceinline__ void band_level(const uint4* __restrict__ rec, const uint4* __restrict__ rec2,
                                            const uint2* __restrict__ ovf, uint32_t* __restrict__ d,
