@@ -216,7 +216,7 @@ def main():
     ap.add_argument("--config", default="C3")
     ap.add_argument("--k", type=int, default=64)
     ap.add_argument("--inflight", type=int, default=0,
-                    help="streams with a batch in flight (1..4; 0 = auto: 4 on small graphs whose labels fit L2, "
+                    help="streams with a batch in flight (1..8; 0 = auto: 8 on small graphs whose labels fit L2, "
                          "1 on large ones, where overlapping sweeps thrash L2: measured slower, DESIGN.md §6)")
     ap.add_argument("--total-sources", type=int, default=0,
                     help="strong scaling: this many sources split over the ranks (C4: 8192); steps is derived")
@@ -313,7 +313,7 @@ def main():
     args.steps = len(timed)
 
     small = 4 * k * n + 16 * info.m_down < 256e6
-    S = args.inflight or (4 if small else 1)
+    S = args.inflight or (8 if small else 1)
     stream = torch.cuda.current_stream()
     streams = [torch.cuda.Stream() for _ in range(S)]
     # L2 protocol: the C3/C4 label arrays (>= 1 GB) are far beyond the 126 MB L2; small

@@ -22,7 +22,7 @@ LIB_PATH = os.path.join(_HERE, "libphast.so")
 
 INF = 0xFFFFFFFF
 KMAX = 64
-SLOTS = 4
+SLOTS = 8
 FLAG_HOST_ONLY = 1
 FLAG_LEVEL_LAYOUT = 2
 FLAG_BFS_IN_LEVEL = 4

@@ -13,7 +13,7 @@ constexpr uint32_t INF = 0xFFFFFFFFu;
 constexpr uint32_t KMAX = 64;
 // per-call scratch slots: up to SLOTS queries of one handle may be in flight at once
 // (each on its own stream); a call waits on the device only for the call SLOTS back
-constexpr uint32_t SLOTS = 4;
+constexpr uint32_t SLOTS = 8;
 
 // Device image of the hierarchy (static after upload; all device pointers).
 struct DevImage {
