@@ -648,10 +648,12 @@ int get_bands(phast_ctx* h, uint32_t k, std::vector<phast_ctx::BandRun>** out) {
     auto it = h->bandruns.find(k);
     if (it != h->bandruns.end()) { *out = &it->second; return PHAST_OK; }
     std::vector<phast_ctx::BandRun> runs;
-    // defaults measured on C3: 256-thread CTAs, variant 5 (records one item
-    // ahead, tail rows through the L1), units of 32768 / k vertices (128 KB of rows)
+    // defaults measured on C3: 256-thread CTAs, variant 13 for k >= 32
+    // (records one item ahead, tail rows through the L1, two 16-byte lanes per thread),
+    // 5 for k = 16 (one lane per thread: equal at C3, 3 % faster at C2), units of 32768 / k
+    // vertices (128 KB of rows)
     const uint32_t threads = h->q.band_threads ? h->q.band_threads : 256u;
-    const uint32_t variant = k < 16 ? 0u : h->q.band_variant ? h->q.band_variant : 5u;   // variants: k >= 16
+    const uint32_t variant = k < 16 ? 0u : h->q.band_variant ? h->q.band_variant : k >= 32 ? 13u : 5u;
     const uint64_t resident = (uint64_t)num_sms() * band_sm_threads(variant, threads) / threads;
     int rc = PHAST_OK;
     for (const Band& B : h->L.bands) {
@@ -979,7 +981,8 @@ int phast_configure(phast_ctx* h, const phast_query_opts* q) {
     if (rc) return rc;
     phast_query_opts nq = q ? *q : phast_query_opts{0, 0, 0, 0, 0, 0, 0};
     if (nq.band_threads && nq.band_threads != 128 && nq.band_threads != 256) return PHAST_EINVAL;
-    if (!(nq.band_variant == 0 || nq.band_variant == 1 || nq.band_variant == 4 || nq.band_variant == 5))
+    if (!(nq.band_variant == 0 || nq.band_variant == 1 || nq.band_variant == 4 || nq.band_variant == 5 ||
+          nq.band_variant == 13))
         return PHAST_EINVAL;
     const uint32_t known = PHAST_Q_NO_FUSED | PHAST_Q_NO_TOP | PHAST_Q_HYBRID_ON | PHAST_Q_HYBRID_OFF | PHAST_Q_NO_MULTI |
                            PHAST_Q_NO_BANDS;

@@ -39,6 +39,13 @@ template <class T> __device__ __forceinline__ T inf_row();
 template <> __device__ __forceinline__ uint32_t inf_row<uint32_t>() { return INF; }
 template <> __device__ __forceinline__ uint2 inf_row<uint2>() { return make_uint2(INF, INF); }
 template <> __device__ __forceinline__ uint4 inf_row<uint4>() { return make_uint4(INF, INF, INF, INF); }
+// two adjacent 16-byte lanes (eight trees) handled by one thread (band kernel variant)
+struct alignas(16) U8 {
+    uint4 a, b;
+};
+template <> __device__ __forceinline__ U8 inf_row<U8>() { return U8{inf_row<uint4>(), inf_row<uint4>()}; }
+__device__ __forceinline__ U8 relax(U8 acc, U8 x, uint32_t l) { return U8{relax(acc.a, x.a, l), relax(acc.b, x.b, l)}; }
+__device__ __forceinline__ uint32_t fmax_of(U8 x) { return max(fmax_of(x.a), fmax_of(x.b)); }
 // a row whose every tree holds x (the no-gather probe A34)
 template <class T> __device__ __forceinline__ T splat(uint32_t x);
 template <> __device__ __forceinline__ uint32_t splat<uint32_t>(uint32_t x) { return x; }

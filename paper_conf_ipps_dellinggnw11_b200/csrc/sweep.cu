@@ -353,17 +353,20 @@ cudaError_t sweep_k(const DevImage& g, const uint32_t* flags, uint32_t vbeg, uin
 // ------------------------------------------------------------------ a3 band sweep
 // Band kernel variants (BandArgs::variant; schedule choices, same labels).  Measured
 // on C3 (profiles/r2_band_variants.md), the product keeps the ablation of
-// the two that matter:
+// the three that matter:
 //   bit 0 PF_REG : each thread loads the next item's record while it gathers the
 //                  current item's tail rows (48 registers: 1280 threads per SM)
 //   bit 2 L1     : tail rows read through the L1 (band_ld); 28-42 % L1 hits
-// 5 = both (the default for k >= 16), 0 = neither (k < 16), 1, 4.  Measured slower and
-// removed: L2 bulk prefetch of the next unit's records, two items per thread in flight,
-// records chained across levels and units or prefetched across the level barrier, no
-// barrier between units (three range buffers), 1536 / 2048 threads per SM with
-// spills, cp.async-staged gathers.
+//   bit 3 LPT2   : two 16-byte lanes per thread (U8; 64 registers, 1024 threads per SM):
+//                  two loads in flight per tail row, the record / flag / address work
+//                  amortised over 32 bytes of row
+// 13 = all three (the default for k >= 32), 5 = PF_REG + L1 (k = 16), 0 = none (k < 16),
+// 1, 4.  Measured slower and removed: four lanes per thread, L2 bulk prefetch of the
+// next unit's records, two items per thread in flight, records chained across levels
+// and units or prefetched across the level barrier, no barrier between units, 1536 /
+// 2048 threads per SM with spills, cp.async-staged gathers, in-unit rows in shared memory.
 template <int VAR>
-constexpr int band_sm_threads_of() { return (VAR & 1) ? 1280 : 1536; }
+constexpr int band_sm_threads_of() { return (VAR & 8) ? 1024 : (VAR & 1) ? 1280 : 1536; }
 
 // The static inputs of one (vertex, lane) item of a band level: its ELL record(s) and
 // its visited-bit word.
@@ -395,14 +398,37 @@ __device__ __forceinline__ T band_ld(const T* p) {
     else return __ldcg(p);
 }
 
-template <int K, bool WIDE, bool DIAM, bool L1 = false>
+// Two 16-byte lanes per thread (variant bit 3, k >= 8; U8 in device.cuh): half the
+// items, two loads in flight per tail row per thread, the per-item record / flag /
+// address work amortised over 32 bytes of row.
+template <bool L1>
+__device__ __forceinline__ U8 band_ld(const U8* p) {
+    const uint4* q = reinterpret_cast<const uint4*>(p);
+    return U8{band_ld<L1>(q), band_ld<L1>(q + 1)};
+}
+__device__ __forceinline__ U8 ldcg_row(const U8* p) {
+    const uint4* q = reinterpret_cast<const uint4*>(p);
+    return U8{__ldcg(q), __ldcg(q + 1)};
+}
+template <class T> __device__ __forceinline__ T ldcg_row(const T* p) { return __ldcg(p); }
+__device__ __forceinline__ void stcs_row(U8* p, U8 x) {
+    uint4* q = reinterpret_cast<uint4*>(p);
+    __stcs(q, x.a);
+    __stcs(q + 1, x.b);
+}
+template <class T> __device__ __forceinline__ void stcs_row(T* p, T x) { __stcs(p, x); }
+// lanes per thread: LPT = 1 (RowT) or 2 (U8, k >= 8)
+template <int K, int LPT> struct BandLane { using T = typename RowT<K>::T; static constexpr uint32_t G = K / RowT<K>::W; };
+template <int K> struct BandLane<K, 2> { using T = U8; static constexpr uint32_t G = K / 8; };
+
+template <int K, bool WIDE, bool DIAM, bool L1 = false, int LPT2 = 1>
 __device__ __forceinline__ void band_item(const BandRec& b, const uint2* __restrict__ ovf, uint32_t* __restrict__ d,
                                           uint32_t v, uint32_t lane, bool store, bool stream, uint32_t& mx) {
-    using T = typename RowT<K>::T;
+    using T = typename BandLane<K, LPT2>::T;
     const uint4 r = b.r, r2 = b.r2;
     T acc = inf_row<T>();
     // the seeded own row: never through the L1 (this item overwrites it)
-    if ((b.fl >> (v & 31)) & 1u) acc = __ldcg(reinterpret_cast<const T*>(d + (size_t)v * K) + lane);
+    if ((b.fl >> (v & 31)) & 1u) acc = ldcg_row(reinterpret_cast<const T*>(d + (size_t)v * K) + lane);
     const bool more = WIDE ? (r2.w == INF && r2.z != INF) : (r.w == INF && r.z != INF);
     const uint32_t oi = WIDE ? r2.z : r.z;
     T x0 = inf_row<T>(), x1 = inf_row<T>(), x2 = inf_row<T>(), x3 = inf_row<T>();
@@ -424,19 +450,19 @@ __device__ __forceinline__ void band_item(const BandRec& b, const uint2* __restr
     }
     if (store) {
         T* p = reinterpret_cast<T*>(d + (size_t)v * K) + lane;
-        if (stream) __stcs(p, acc); else *p = acc;
+        if (stream) stcs_row(p, acc); else *p = acc;
     }
     if constexpr (DIAM) mx = max(mx, fmax_of(acc));
 }
 
 // One unit level [vb, ve).  PF_REG: the next item's record is loaded before the
 // current item's gathers.
-template <int K, bool WIDE, bool DIAM, int THREADS, bool PF_REG, bool L1>
+template <int K, bool WIDE, bool DIAM, int THREADS, bool PF_REG, bool L1, int LPT2>
 __device__ __forceinline__ void band_level(const uint4* __restrict__ rec, const uint4* __restrict__ rec2,
                                            const uint2* __restrict__ ovf, uint32_t* __restrict__ d,
                                            const uint32_t* __restrict__ flags, uint32_t vb, uint32_t ve, bool store,
                                            bool stream, uint32_t& mx) {
-    constexpr uint32_t G = K / RowT<K>::W;
+    constexpr uint32_t G = BandLane<K, LPT2>::G;
     const uint32_t total = (ve - vb) * G;
     uint32_t t = threadIdx.x;
     if constexpr (PF_REG) {
@@ -446,14 +472,14 @@ __device__ __forceinline__ void band_level(const uint4* __restrict__ rec, const 
             const BandRec cur = nx;
             const uint32_t tn = t + THREADS;
             if (tn < total) nx = band_rec<WIDE>(rec, rec2, flags, vb + tn / G);
-            band_item<K, WIDE, DIAM, L1>(cur, ovf, d, vb + t / G, t % G, store, stream, mx);
+            band_item<K, WIDE, DIAM, L1, LPT2>(cur, ovf, d, vb + t / G, t % G, store, stream, mx);
             if (tn >= total) break;
             t = tn;
         }
     } else {
         for (; t < total; t += THREADS)
-            band_item<K, WIDE, DIAM, L1>(band_rec<WIDE>(rec, rec2, flags, vb + t / G), ovf, d, vb + t / G, t % G,
-                                         store, stream, mx);
+            band_item<K, WIDE, DIAM, L1, LPT2>(band_rec<WIDE>(rec, rec2, flags, vb + t / G), ovf, d, vb + t / G,
+                                               t % G, store, stream, mx);
     }
 }
 
@@ -469,6 +495,7 @@ __global__ void __launch_bounds__(THREADS, band_sm_threads_of<VAR>() / THREADS)
                 uint32_t* __restrict__ diam) {
     static_assert(THREADS >= 32, "one warp at least");
     constexpr bool PF_REG = VAR & 1, L1 = VAR & 4;
+    constexpr int LPT2 = ((VAR & 8) && K >= 8) ? 2 : 1;   // lanes per thread
     __shared__ uint32_t rng[2][32][2];   // [buffer][level][begin, end]
     asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
     asm volatile("griddepcontrol.wait;" ::: "memory");   // the levels above the band are complete and visible
@@ -487,9 +514,11 @@ __global__ void __launch_bounds__(THREADS, band_sm_threads_of<VAR>() / THREADS)
             const bool last = j + 1 == F;
             const bool store = !last || a.store_last, stream = last && a.stream_last;
             if ((a.wide >> j) & 1u)
-                band_level<K, true, DIAM, THREADS, PF_REG, L1>(rec, rec2, ovf, d, flags, vb, ve, store, stream, mx);
+                band_level<K, true, DIAM, THREADS, PF_REG, L1, LPT2>(rec, rec2, ovf, d, flags, vb, ve, store, stream,
+                                                                     mx);
             else
-                band_level<K, false, DIAM, THREADS, PF_REG, L1>(rec, rec2, ovf, d, flags, vb, ve, store, stream, mx);
+                band_level<K, false, DIAM, THREADS, PF_REG, L1, LPT2>(rec, rec2, ovf, d, flags, vb, ve, store, stream,
+                                                                      mx);
             if (!last) __syncthreads();   // level j's rows are written before level j+1 reads them
         }
     }
@@ -558,6 +587,7 @@ cudaError_t band_k(const DevImage& g, const BandArgs& a, const uint32_t* flags, 
             case 1: return band_kv<K, 1>(g, a, flags, dist, diam, st);
             case 4: return band_kv<K, 4>(g, a, flags, dist, diam, st);
             case 5: return band_kv<K, 5>(g, a, flags, dist, diam, st);
+            case 13: return band_kv<K, 13>(g, a, flags, dist, diam, st);
             default: return cudaErrorInvalidValue;
         }
     }
@@ -684,7 +714,7 @@ cudaError_t launch_sweep_band(const DevImage& g, const BandArgs& a, const uint32
 }
 
 uint32_t band_sm_threads(uint32_t variant, uint32_t) {
-    return variant & 1 ? 1280u : 1536u;
+    return variant & 8 ? 1024u : variant & 1 ? 1280u : 1536u;
 }
 
 cudaError_t launch_clear_flags(const Slot& sl, uint32_t k, uint32_t seed_cap, cudaStream_t st) {

@@ -27,7 +27,7 @@ def check(h, g, src):
 def main():
     import torch
     g1 = phastgen.grid(40, 30, 1, 1 << 20, seed=1)          # fused single-launch query (k <= 4)
-    g2 = phastgen.road(20_000, seed=35)                      # upward kernel, seeds, top launch, level launches
+    g2 = phastgen.road(20_000, seed=35)                      # upward kernel, seeds, top launch, level and band launches
     for g in (g1, g2):
         with P.Phast.from_graph(g) as h:
             for k in (1, 4, 16, 5):
@@ -36,6 +36,11 @@ def main():
             check(h, g, phastgen.sources(g.n, 16, seed=3))
             h.configure(flags=P.Q_NO_FUSED | P.Q_HYBRID_OFF, up_smem_cap=32)   # global-table fallback
             check(h, g, phastgen.sources(g.n, 8, seed=4))
+            for v in (1, 4, 5):                               # band kernel variants (k >= 16), k = 64
+                h.configure(flags=P.Q_NO_FUSED, band_variant=v)
+                check(h, g, phastgen.sources(g.n, 64, seed=6 + v))
+            h.configure(flags=P.Q_NO_FUSED | P.Q_NO_TOP, band_unit=32)   # one group per unit, no top launch
+            check(h, g, phastgen.sources(g.n, 16, seed=9))
             h.configure()
             src = phastgen.sources(g.n, 16, seed=5)
             d = check(h, g, src)
