@@ -29,7 +29,7 @@ FLAG_BFS_IN_LEVEL = 4
 FLAG_NO_BANDS = 32
 LAYOUT_FLAGS = {"levels-bands": 0, "levels-bfs": FLAG_NO_BANDS, "levels": FLAG_LEVEL_LAYOUT}
 LAYOUT_NAMES = {1: "levels", 2: "levels-bfs", 3: "levels-bands"}   # phast_info_t.layout
-Q_NO_FUSED, Q_NO_TOP, Q_HYBRID_ON, Q_HYBRID_OFF, Q_NO_MULTI, Q_NO_BANDS, Q_DIAM_BANDS = 1, 2, 4, 8, 32, 64, 128
+Q_NO_FUSED, Q_NO_TOP, Q_HYBRID_ON, Q_HYBRID_OFF, Q_NO_MULTI, Q_NO_BANDS = 1, 2, 4, 8, 32, 64
 
 STATUS = {0: "OK", -1: "EINVAL", -2: "ENOMEM", -3: "ECUDA", -4: "ERANGE", -5: "ESTATE", -6: "EIO",
           -7: "EINTERNAL"}

@@ -759,11 +759,8 @@ int run_query(phast_ctx* h, const Sources& S, uint32_t kp, const QueryOut& o, cu
     }
     // then every band below the top launch in one launch each (a band that reaches into
     // the top launch's levels is swept per level), every other level in its own launch
-    // diameter queries (no level-0 rows stored, up to SLOTS batches on library streams)
-    // run every level as its own launch: measured faster at C5 (461 k vs 422 k trees/s)
     std::vector<phast_ctx::BandRun>* bands = nullptr;
-    if (!o.nogather && (!o.diam || (h->q.flags & PHAST_Q_DIAM_BANDS)) && !(h->q.flags & PHAST_Q_NO_BANDS) &&
-        !h->L.bands.empty()) {
+    if (!o.nogather && !(h->q.flags & PHAST_Q_NO_BANDS) && !h->L.bands.empty()) {
         const int rc = get_bands(h, kp, &bands);
         if (rc) return rc;
     }
@@ -986,7 +983,7 @@ int phast_configure(phast_ctx* h, const phast_query_opts* q) {
           nq.band_variant == 13))
         return PHAST_EINVAL;
     const uint32_t known = PHAST_Q_NO_FUSED | PHAST_Q_NO_TOP | PHAST_Q_HYBRID_ON | PHAST_Q_HYBRID_OFF | PHAST_Q_NO_MULTI |
-                           PHAST_Q_NO_BANDS | PHAST_Q_DIAM_BANDS;
+                           PHAST_Q_NO_BANDS;
     if ((nq.flags & ~known) || ((nq.flags & PHAST_Q_HYBRID_ON) && (nq.flags & PHAST_Q_HYBRID_OFF)))
         return PHAST_EINVAL;
     DeviceGuard dg(h->device);

@@ -171,7 +171,7 @@ SCHEDULES = {
     "bands_unit_big": dict(flags=P.Q_NO_FUSED | P.Q_NO_TOP, band_unit=1 << 20),   # few units, no top launch
     "bands_v1_256": dict(flags=P.Q_NO_FUSED, band_variant=1, band_threads=256),   # records one item ahead
     "bands_v4": dict(flags=P.Q_NO_FUSED | P.Q_NO_TOP, band_variant=4, band_threads=128),   # tails through the L1
-    "bands_lpt2": dict(flags=P.Q_NO_FUSED | P.Q_DIAM_BANDS, band_variant=13),   # two lanes per thread; diameters too
+    "bands_lpt2": dict(flags=P.Q_NO_FUSED, band_variant=13),                   # two 16-byte lanes per thread
     "bands_v5_k32": dict(flags=P.Q_NO_FUSED | P.Q_NO_TOP, band_variant=5, band_threads=256),
 }
 
