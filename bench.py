@@ -234,6 +234,8 @@ def main():
                     help="vertices per work unit of a band launch (phast_query_opts band_unit; 0 = 8192/k)")
     ap.add_argument("--band-threads", type=int, default=0, help="CTA size of a band launch (128/256; 0 = 128)")
     ap.add_argument("--band-variant", type=int, default=0, help="band kernel variant (phast_query_opts band_variant)")
+    ap.add_argument("--top-max-vertices", type=int, default=0,
+                    help="cap on the vertices of the shared-memory top launch (phast_query_opts top_max_vertices)")
     ap.add_argument("--query-flags", type=int, default=0,
                     help="phast_configure flags (schedule experiments: 1 no fused single-launch query, 2 no shared-memory top launch)")
     ap.add_argument("--parents", action="store_true",
@@ -293,9 +295,9 @@ def main():
         log(f"[bench] CH build {time.time() - t:.1f}s")
         if args.cache:
             h.save(args.cache)
-    if args.query_flags or args.band_unit or args.band_threads or args.band_variant:
+    if args.query_flags or args.band_unit or args.band_threads or args.band_variant or args.top_max_vertices:
         h.configure(flags=args.query_flags, band_unit=args.band_unit, band_threads=args.band_threads,
-                    band_variant=args.band_variant)
+                    band_variant=args.band_variant, top_max_vertices=args.top_max_vertices)
     n = h.n
     info = h.info()
     lsz = h.level_sizes()
