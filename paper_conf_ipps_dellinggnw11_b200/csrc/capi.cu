@@ -45,7 +45,7 @@ struct phast_ctx {
     cudaEvent_t up_done[SLOTS] = {};
     cudaEvent_t slot_free[SLOTS] = {};
     uint32_t slot_next = 0;
-    cudaStream_t side = nullptr;
+    cudaStream_t side[SLOTS] = {};     // upward searches, one stream per slot (they overlap)
     uint32_t* pad[SLOTS] = {};          // padded-k label scratch per slot (phast_trees with k not a power of two)
     size_t pad_elems[SLOTS] = {};
     // library streams for batches in flight (phast_diameter) and their label buffers
@@ -181,8 +181,10 @@ void free_seeds(phast_ctx* h) {
         cudaFree(h->slot[s].seed_d);
         h->slot[s].seed_v = h->slot[s].seed_d = nullptr;
     }
-    cudaFree(h->g.gscratch);
-    h->g.gscratch = nullptr;
+    for (uint32_t s = 0; s < SLOTS; s++) {
+        cudaFree(h->slot[s].gscratch);
+        h->slot[s].gscratch = nullptr;
+    }
 }
 
 // search-space buffers for the current options (phast_query_opts seed_cap / up_smem_cap)
@@ -199,7 +201,9 @@ int alloc_seeds(phast_ctx* h) {
         if ((rc = dmalloc(&h->slot[s].seed_v, (size_t)KMAX * h->g.seed_cap)) ||
             (rc = dmalloc(&h->slot[s].seed_d, (size_t)KMAX * h->g.seed_cap)))
             return rc;
-    return dmalloc(&h->g.gscratch, (size_t)KMAX * h->g.seed_cap * 5);
+    for (uint32_t s = 0; s < SLOTS; s++)
+        if ((rc = dmalloc(&h->slot[s].gscratch, (size_t)KMAX * h->g.seed_cap * 5))) return rc;
+    return PHAST_OK;
 }
 
 void free_device(phast_ctx* h) {
@@ -228,8 +232,10 @@ void free_device(phast_ctx* h) {
     }
     if (h->fork_ev) cudaEventDestroy(h->fork_ev);
     h->fork_ev = nullptr;
-    if (h->side) cudaStreamDestroy(h->side);
-    h->side = nullptr;
+    for (uint32_t s = 0; s < SLOTS; s++) {
+        if (h->side[s]) cudaStreamDestroy(h->side[s]);
+        h->side[s] = nullptr;
+    }
     cudaFree((void*)h->g.dn_first); cudaFree((void*)h->g.dn_arc);
     cudaFree((void*)h->g.dn_rec); cudaFree((void*)h->g.dn_rec2); cudaFree((void*)h->g.dn_ovf);
     cudaFree((void*)h->g.up_first); cudaFree((void*)h->g.up_arc);
@@ -361,7 +367,7 @@ int upload(phast_ctx* h) {
               cudaMemcpy(upf, L.up_first.data(), L.up_first.size() * 4, cudaMemcpyHostToDevice) == cudaSuccess &&
               cudaMemcpy(upa, L.up_arc.data(), L.up_arc.size() * 8, cudaMemcpyHostToDevice) == cudaSuccess &&
               cudaMemset(g.err, 0, 4) == cudaSuccess &&
-              cudaStreamCreateWithFlags(&h->side, cudaStreamNonBlocking) == cudaSuccess &&
+
               cudaEventCreateWithFlags(&h->fork_ev, cudaEventDisableTiming) == cudaSuccess;
     for (uint32_t s = 0; ok && s < SLOTS; s++)
         ok = cudaMemset(h->slot[s].flags, 0, (nw + 4) * 4) == cudaSuccess &&
@@ -369,7 +375,8 @@ int upload(phast_ctx* h) {
              cudaEventCreateWithFlags(&h->up_done[s], cudaEventDisableTiming) == cudaSuccess &&
              cudaEventCreateWithFlags(&h->slot_free[s], cudaEventDisableTiming) == cudaSuccess &&
              cudaEventCreateWithFlags(&h->lane_ev[s], cudaEventDisableTiming) == cudaSuccess &&
-             cudaStreamCreateWithFlags(&h->lane[s], cudaStreamNonBlocking) == cudaSuccess;
+             cudaStreamCreateWithFlags(&h->lane[s], cudaStreamNonBlocking) == cudaSuccess &&
+             cudaStreamCreateWithFlags(&h->side[s], cudaStreamNonBlocking) == cudaSuccess;
     ok = ok && cudaDeviceSynchronize() == cudaSuccess;
     if (!ok) { cudaGetLastError(); free_device(h); return PHAST_ECUDA; }
     return PHAST_OK;
@@ -742,9 +749,9 @@ int run_query(phast_ctx* h, const Sources& S, uint32_t kp, const QueryOut& o, cu
     }
     if (top && top->a.fused) top = nullptr;   // the A34 probe runs every level as its own launch
     // a1 on the side stream (overlaps earlier sweeps), after this slot's previous query
-    if (cudaStreamWaitEvent(h->side, h->slot_free[s], 0) != cudaSuccess) return PHAST_ECUDA;
-    if (launch_upward(h->g, sl, S, kp, top ? top->vtop : 0u, h->side) != cudaSuccess) return PHAST_ECUDA;
-    if (cudaEventRecord(h->up_done[s], h->side) != cudaSuccess) return PHAST_ECUDA;
+    if (cudaStreamWaitEvent(h->side[s], h->slot_free[s], 0) != cudaSuccess) return PHAST_ECUDA;
+    if (launch_upward(h->g, sl, S, kp, top ? top->vtop : 0u, h->side[s]) != cudaSuccess) return PHAST_ECUDA;
+    if (cudaEventRecord(h->up_done[s], h->side[s]) != cudaSuccess) return PHAST_ECUDA;
     if (cudaStreamWaitEvent(st, h->up_done[s], 0) != cudaSuccess) return PHAST_ECUDA;
     // a2 on the caller's stream
     if (launch_seed(h->g, sl, kp, o.dist, st) != cudaSuccess) return PHAST_ECUDA;

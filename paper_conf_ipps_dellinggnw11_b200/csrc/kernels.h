@@ -33,7 +33,6 @@ struct DevImage {
     const uint2* dn_ovf = nullptr;       // [overflow entries]
     const uint32_t* up_first = nullptr;  // [n+1]   G-up out-arcs by tail
     const uint2* up_arc = nullptr;       // [m_up]   {head, len}
-    uint32_t* gscratch = nullptr;        // [KMAX * seed_cap * 5] global fallback tables of the upward search
     uint32_t* err = nullptr;             // [1] sticky device error word (bit 0: search-space overflow)
     uint32_t seed_cap = 0;               // search-space entries per source (power of two)
     uint32_t smem_cap = 4096;            // shared-memory table entries per search (power of two, <= 4096)
@@ -45,6 +44,7 @@ struct Slot {
     uint32_t* seed_v = nullptr;     // [KMAX][seed_cap] upward search space: vertex
     uint32_t* seed_d = nullptr;     // [KMAX][seed_cap] upward search space: label
     uint32_t* seed_cnt = nullptr;   // [KMAX]
+    uint32_t* gscratch = nullptr;   // [KMAX * seed_cap * 5] global fallback tables of this slot's upward searches
 };
 
 struct Sources {

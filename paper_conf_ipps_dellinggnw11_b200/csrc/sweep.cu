@@ -167,9 +167,9 @@ __global__ void __launch_bounds__(UP_THREADS) upward_kernel(DevImage g, Slot sl,
     const uint32_t sc = g.smem_cap;
     UpTable t{smem, smem + sc, smem + 2 * sc, smem + 3 * sc, smem + 4 * sc, sc};
     bool ok = up_search(g.up_first, g.up_arc, s, t, c, vtop);
-    if (!ok) {   // global-memory fallback with the per-source capacity (searches of one
-                 // handle run on one side stream, one launch at a time: one table set)
-        uint32_t* base = g.gscratch + (size_t)i * g.seed_cap * 5;
+    if (!ok) {   // global-memory fallback with the per-source capacity (the slot's own
+                 // table set: searches of different slots may run at once)
+        uint32_t* base = sl.gscratch + (size_t)i * g.seed_cap * 5;
         UpTable gt{base, base + g.seed_cap, base + 2 * (size_t)g.seed_cap, base + 3 * (size_t)g.seed_cap,
                    base + 4 * (size_t)g.seed_cap, g.seed_cap};
         t = gt;
