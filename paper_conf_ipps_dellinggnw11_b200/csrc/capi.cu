@@ -40,7 +40,7 @@ struct phast_ctx {
     int device = -1;
     DevImage g;
     // per-query slots (PHAST_SLOTS in flight): visited bits + search spaces; upward
-    // searches run on one side stream, each waiting for its slot's previous query
+    // searches run on their slot's side stream, each waiting for its slot's previous query
     Slot slot[SLOTS];
     cudaEvent_t up_done[SLOTS] = {};
     cudaEvent_t slot_free[SLOTS] = {};
@@ -748,7 +748,7 @@ int run_query(phast_ctx* h, const Sources& S, uint32_t kp, const QueryOut& o, cu
         return PHAST_OK;
     }
     if (top && top->a.fused) top = nullptr;   // the A34 probe runs every level as its own launch
-    // a1 on the side stream (overlaps earlier sweeps), after this slot's previous query
+    // a1 on the slot's side stream (overlaps earlier sweeps and the other slots' searches), after this slot's previous query
     if (cudaStreamWaitEvent(h->side[s], h->slot_free[s], 0) != cudaSuccess) return PHAST_ECUDA;
     if (launch_upward(h->g, sl, S, kp, top ? top->vtop : 0u, h->side[s]) != cudaSuccess) return PHAST_ECUDA;
     if (cudaEventRecord(h->up_done[s], h->side[s]) != cudaSuccess) return PHAST_ECUDA;
