@@ -432,7 +432,8 @@ def main():
     if args.parents:
         par_buf = torch.empty(n * k, dtype=torch.int32, device="cuda")
         last = timed[-1]
-        dist_t = bufs[(len(timed) - 1) % nbuf]
+        dist_t = bufs[0]
+        h.trees_into(last, dist_t.data_ptr(), stream.cuda_stream)   # the probes above overwrote the buffers
         h.parents(last, dist_t, out=par_buf, stream=stream)
         h.sync(stream)
         p0, p1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
