@@ -629,3 +629,28 @@ def test_parents_ch_bit_exact(c1, road, name):
             dint[perm] = oracle.sssp(g, int(src[i])).astype(np.int64)
             want = oracle.parents_ch(ex, dint, int(perm[src[i]]))
             assert np.array_equal(rows[:, i], want), (name, k, i)
+
+
+@pytest.mark.gpu
+def test_band_layout_save_load_device(tmp_path):
+    """The band layout (R20) survives phast_save / phast_load onto the device: same
+    bands, same schedule, bit-exact trees and diameter against the oracle, with the
+    band launches on (default) and off."""
+    g = phastgen.road(60_000, seed=45)
+    p = str(tmp_path / "bands.phast")
+    with P.Phast.from_graph(g) as h:
+        h.save(p)
+        b1, s1 = h.bands(), h.schedule(64)
+    with P.Phast.load(p) as h:
+        b2 = h.bands()
+        assert len(b1) == len(b2) > 0 and h.schedule(64) == s1
+        for x, y in zip(b1, b2):
+            assert np.array_equal(x["goff"], y["goff"])
+        assert s1["band_launches"] > 0
+        for flags in (P.Q_NO_FUSED, P.Q_NO_FUSED | P.Q_NO_BANDS):
+            h.configure(flags=flags)
+            for k in (16, 64):
+                src = phastgen.sources(g.n, k, seed=460 + k)
+                assert np.array_equal(gpu_trees(h, src), oracle.sssp_many(g, src)), (flags, k)
+            src = phastgen.sources(g.n, 200, seed=461)
+            assert h.diameter(src, k_batch=64) == oracle.diameter(g, src)
