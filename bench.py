@@ -516,7 +516,7 @@ def main():
                        else ms * 1e3 / trees_here,
                        "ch_build_s": round(info.build_seconds, 1)},
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
-                         "traffic": traffic, "kernel": "sweep_top_kernel + sweep_kernel (all levels of one sweep)",
+                         "traffic": traffic, "kernel": "sweep_top_kernel + sweep_band_kernel + sweep_kernel (all levels of one sweep)",
                          "alg_bytes_per_sweep": B_alg, "sweep_ms": sweep_ms, "sweep_ms_events": sweep_ms_events,
                          "upward_ms": ms_up / max(nb, 1), "how": how, "peak_source": peak_src},
             "ceiling": ceiling, "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": launches,
